@@ -1,0 +1,202 @@
+/*
+ * qoserve.h — C ABI of libqoserve.so, the B200 (sm_100a) hybrid-batch forward step under the
+ * QoServe scheduler (Goel et al., "QoServe: Breaking the Silos of LLM Inference Serving",
+ * ASPLOS'26; text in PAPER.md).
+ *
+ * What one call computes.  QoServe builds each iteration from ALL requests in the decode queue
+ * plus prefill chunk(s) taken from deadline-selected prefill requests (§3.1
+ * step 1; Algorithm 1 lines 2, 17-20 = PAPER.md:755, 770-773) and dispatches them as ONE fused
+ * prefill+decode token batch (PAPER.md:542-545 step 5; §3.3 "fused
+ * prefill-decode MLP") to a vLLM engine with tensor parallelism and PagedAttention
+ * (§3.6).  Chunk sizes change every iteration at no extra cost
+ * (§3.6.1), so the step must reach exactly the result of the plain causal
+ * forward for any chunk split (§2.1), and its latency must be predictable
+ * from (chunk_len, n_decode, ctx) for the dynamic-chunking predictor (§3.6.1).
+ *
+ * Model: decoder-only pre-norm transformer, Llama/Qwen2 convention (reading s1-s3 in
+ * DESIGN.md §2): RMSNorm, rotate-half RoPE, GQA (kv head = h / (H/Hkv)), SwiGLU, untied LM
+ * head, optional QKV bias.  Precision (reading s4): bf16 weights / activations / KV cache,
+ * fp32 accumulation, fp32 softmax and norm statistics, fp32 residual stream.
+ *
+ * Conventions (all calls):
+ *   - Return value: QOS_OK (0) or a negative QOS_ERR_*; no exception or abort crosses the ABI.
+ *     qos_last_error() returns a thread-local message for the last failing call.
+ *   - Pointers are plain host pointers unless documented "device".  Caller-owned inputs are
+ *     only read during the call.  The engine owns weights, KV pool, block tables, workspaces
+ *     (or borrows caller-provided device arenas, see qos_engine_create).
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *   - An engine is single-threaded: calls on one engine must not overlap.
+ *   - Under tensor parallelism every rank is called with the same arguments (rank 0's
+ *     scheduler broadcasts the descriptor); KV tables are identical on every rank.
+ *   - There is no CPU fallback: every compute step runs in this library's sm_100a kernels.
+ */
+#ifndef QOSERVE_H_
+#define QOSERVE_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ---------------------------------------------------------------- return codes, dtypes */
+enum {
+  QOS_OK = 0,
+  QOS_ERR_INVALID_ARG = -1,   /* bad pointer / shape / descriptor field                    */
+  QOS_ERR_OOM = -2,           /* KV pool or device memory exhausted (state unchanged)       */
+  QOS_ERR_UNKNOWN_REQ = -3,   /* request id has no KV table                                */
+  QOS_ERR_BAD_KV_START = -4,  /* kv_start / ctx_len != the request's cached length         */
+  QOS_ERR_NOT_ALLOCATED = -5, /* the step would write past the request's allocated blocks  */
+  QOS_ERR_CUDA = -6,          /* CUDA runtime / driver error (message in qos_last_error)   */
+  QOS_ERR_COMM = -7,          /* NCCL error; the communicator is aborted                   */
+  QOS_ERR_UNSUPPORTED = -8    /* shape the kernels do not support (e.g. head_dim != 64/128) */
+};
+
+enum { QOS_F32 = 0, QOS_BF16 = 1 };
+
+typedef struct qos_engine qos_engine_t;  /* opaque; one per (process, GPU, TP rank) */
+
+/* ---------------------------------------------------------------- model / engine config */
+typedef struct {
+  int32_t n_layers, d_model, n_heads, n_kv_heads, head_dim, ffn_dim, vocab;
+  float rope_theta, rms_eps;
+  int32_t qkv_bias;         /* 1: q/k/v projections carry a bias (Qwen2)                    */
+  int32_t block_size;       /* KV block size in tokens; must be 16 (reading s12)             */
+  int64_t num_blocks;       /* KV pool size in blocks (per rank)                             */
+  int32_t max_seq_len;      /* max tokens per request; block-table width = ceil(/16)         */
+  int32_t max_requests;     /* max live requests (block-table rows)                          */
+  int32_t max_batch_tokens; /* max T = sum(chunk_len) + n_decode per step                    */
+  int32_t max_batch_rows;   /* max R = n_prefill + n_decode per step                         */
+} qos_model_cfg;
+
+typedef struct {
+  uint64_t weight_bytes;    /* this rank's weight shard                                     */
+  uint64_t kv_bytes;        /* KV pool: L x {K,V} x num_blocks x Hkv/tp x 16 x hd x 2 B      */
+  uint64_t workspace_bytes; /* activations, metadata, split-K partials for max_batch_tokens  */
+} qos_mem_sizes;
+
+typedef struct {            /* optional caller-provided DEVICE arenas (256-byte aligned);    */
+  void* weights;            /* any NULL member is cudaMalloc'ed by the engine. Ownership of  */
+  void* kv;                 /* provided arenas stays with the caller, who must keep them      */
+  void* workspace;          /* alive until qos_engine_destroy.                                */
+} qos_mem;
+
+/* Sizes of the three arenas for `cfg` at TP degree `tp_size`. */
+int qos_engine_mem_sizes(const qos_model_cfg* cfg, int tp_size, qos_mem_sizes* out);
+
+/* Create an engine on CUDA device `device` for TP rank `tp_rank` of `tp_size`.
+ * nccl_uid: the 128-byte ncclUniqueId shared by all ranks (rank 0 creates it with
+ * qos_nccl_unique_id and broadcasts it, e.g. over torch.distributed); NULL iff tp_size == 1.
+ * Sharding: rank r owns q heads [r*H/tp, (r+1)*H/tp), kv heads
+ * [r*Hkv/tp, ...), FFN columns [r*F/tp, ...), the matching rows of o_proj / down_proj, and
+ * vocab rows [r*V/tp, ...) of lm_head; embeddings and norms are replicated.
+ * Requires tp_size | n_kv_heads, tp_size | n_heads, tp_size | ffn_dim, tp_size | vocab. */
+int qos_engine_create(const qos_model_cfg* cfg, int device, int tp_rank, int tp_size,
+                      const uint8_t* nccl_uid, const qos_mem* mem, qos_engine_t** out);
+int qos_engine_destroy(qos_engine_t* eng);
+
+/* 128-byte ncclUniqueId for tp_size > 1 (call on rank 0 only). */
+int qos_nccl_unique_id(uint8_t out[128]);
+
+/* Fill this rank's weight shard with the synthetic generator of DESIGN.md §3:
+ * w = bf16_rne(f(a)), a = ((splitmix64((seed ^ fnv1a64(name)) + i) >> 40) - 2^23) / 2^23,
+ * i the flat row-major index in the Hugging Face tensor `name`; f per kind (linear:
+ * a * fp32(1/sqrt(fan_in)); embed: a; norm: 1 + 0.1 a; bias: 0.02 a).  Synchronous. */
+int qos_engine_load_synthetic(qos_engine_t* eng, uint64_t seed);
+
+/* Copy rows [row0, row0+nrows) of this rank's shard of HF tensor `name` (e.g.
+ * "model.layers.3.mlp.up_proj.weight", shard-local row numbering) to host bf16 bits. */
+int qos_engine_read_weight(qos_engine_t* eng, const char* name, int64_t row0, int64_t nrows,
+                           uint16_t* out_bf16);
+
+/* ---------------------------------------------------------------- paged KV (a6 storage, D7) */
+/* Grow req's block table to ceil(n_tokens_total / 16) blocks, taking the lowest free block
+ * indices in ascending order (reading s12).  All-or-nothing: QOS_ERR_OOM leaves every table
+ * unchanged.  Never shrinks.  The device copy of the table row is updated stream-ordered on
+ * the engine's internal stream before the next step.  KV is held only while needed
+ * (§3.4). */
+int qos_kv_alloc(qos_engine_t* eng, int64_t req, int32_t n_tokens_total);
+/* Release all of req's blocks (QOS_ERR_UNKNOWN_REQ if it has none). */
+int qos_kv_free(qos_engine_t* eng, int64_t req);
+/* Inspect req's table: writes min(cap, n) block ids to out, n to *n_out. */
+int qos_kv_table(qos_engine_t* eng, int64_t req, int32_t* out, int32_t cap, int32_t* n_out);
+/* Same, read back from the DEVICE copy of the table (flushes pending updates; synchronous). */
+int qos_kv_table_device(qos_engine_t* eng, int64_t req, int32_t* out, int32_t cap, int32_t* n_out);
+/* Tokens of req already in the cache (what the next kv_start / ctx_len must equal). */
+int qos_kv_cached_len(qos_engine_t* eng, int64_t req, int32_t* out);
+/* Number of free blocks. */
+int qos_kv_free_blocks(qos_engine_t* eng, int64_t* out);
+/* Fill positions [0, n_tokens) of req, every layer, with synthetic K/V (DESIGN.md §3:
+ * name "kvfill.{layer}.{k|v}.{req}", i = (pos*Hkv + h)*hd + j over GLOBAL kv heads, value
+ * bf16_rne(a)) and set its cached length to n_tokens.  Used by benches / profiling where
+ * a decode's prefix need not come from a prefill.  Synchronous. */
+int qos_kv_fill_synthetic(qos_engine_t* eng, int64_t req, int32_t n_tokens, uint64_t seed);
+
+/* ---------------------------------------------------------------- the hybrid step (a1..a14) */
+typedef struct {
+  int64_t req;
+  int32_t kv_start;        /* == cached length of req (strict append, no recompute)          */
+  int32_t chunk_len;       /* >= 1 prefill tokens at positions kv_start .. kv_start+len-1    */
+  const int32_t* tokens;   /* host, [chunk_len] token ids in [0, vocab)                      */
+} qos_prefill_chunk;
+
+typedef struct {
+  int64_t req;
+  int32_t ctx_len;         /* cached tokens; the new token sits at position ctx_len and     */
+  int32_t token;           /* attends ctx_len + 1 keys (reading s7)                          */
+} qos_decode;
+
+typedef struct {
+  int32_t n_prefill;
+  const qos_prefill_chunk* prefill;  /* host array [n_prefill]; distinct requests            */
+  int32_t n_decode;
+  const qos_decode* decode;          /* host array [n_decode]; distinct from the chunks'     */
+} qos_batch;
+
+/* One hybrid-batch forward iteration.
+ * Rows of the outputs: one per chunk (its LAST token, reading s8) in descriptor order, then one
+ * per decode in descriptor order; R = n_prefill + n_decode.
+ *   logits      : [R][vocab] of logits_dtype (QOS_F32 | QOS_BF16), or NULL;
+ *   next_tokens : [R] int32 greedy argmax (lowest index on ties), or NULL;
+ *   outputs_on_host = 0: both are DEVICE pointers and the call is stream-ordered/asynchronous;
+ *   outputs_on_host = 1: both are HOST pointers; the call copies them back and synchronises.
+ * Effects: appends the K/V of every processed token to the paged cache and advances the
+ * requests' cached lengths by chunk_len / 1.  Errors are detected before any device work
+ * (INVALID_ARG, UNKNOWN_REQ, BAD_KV_START, NOT_ALLOCATED); state is then unchanged. */
+int qos_hybrid_step(qos_engine_t* eng, const qos_batch* batch, void* logits, int logits_dtype,
+                    int32_t* next_tokens, int outputs_on_host, void* stream);
+
+/* Device-timed latency of one synthetic step for the scheduler's iteration-time model
+ * (replaces the paper's Vidur-profiled random forest, §3.6.1): a chunk of
+ * chunk_len tokens at kv_start 0 plus n_decode decodes with contexts ctx_lens[j] (host), on
+ * scratch requests with synthetic KV.  Runs 3 warm-up steps, then `reps` steps each timed with
+ * CUDA events on the engine stream; *ms_out = median.  Synchronous; scratch KV is freed. */
+int qos_profile_step(qos_engine_t* eng, int32_t chunk_len, int32_t n_decode,
+                     const int32_t* ctx_lens, int32_t reps, float* ms_out);
+/* Same with an explicit chunk kv_start (prefix already cached) and p95 output. */
+int qos_profile_step_ex(qos_engine_t* eng, int32_t chunk_len, int32_t kv_start,
+                        int32_t n_decode, const int32_t* ctx_lens, int32_t reps,
+                        float* ms_median, float* ms_p95);
+
+/* ---------------------------------------------------------------- per-kernel timing (a15) */
+enum {
+  QOS_T_META = 0, QOS_T_EMBED, QOS_T_NORM, QOS_T_GEMM_QKV, QOS_T_ROPE_APPEND, QOS_T_PREFILL_ATTN,
+  QOS_T_DECODE_ATTN, QOS_T_GEMM_O, QOS_T_GEMM_GATEUP, QOS_T_GEMM_DOWN, QOS_T_ALLREDUCE,
+  QOS_T_HEAD, QOS_T_ARGMAX, QOS_T_COUNT
+};
+/* When enabled, every kernel class of each step is bracketed by CUDA events on the step's
+ * stream; qos_last_step_timing then returns per-class summed device ms and launch counts of
+ * the last step (it synchronises on the step's final event). */
+int qos_engine_set_timing(qos_engine_t* eng, int enable);
+int qos_last_step_timing(qos_engine_t* eng, float ms[QOS_T_COUNT], int32_t launches[QOS_T_COUNT]);
+/* Total kernel launches issued by this engine since creation (the bench's gpu_launches). */
+int qos_engine_launch_count(qos_engine_t* eng, int64_t* out);
+
+const char* qos_strerror(int code);
+const char* qos_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* QOSERVE_H_ */

@@ -1,0 +1,65 @@
+/*
+ * qoserve_ops.h — kernel-level entry points of libqoserve.so, one per step of the hybrid
+ * iteration (SURVEY.md §8(a) rows a3, a4/a9/a11/a12/a13, a5+a6, a7+a8).  They exist so each
+ * row can be checked against the fp64 oracle on inputs the TEST builds on the host (no oracle
+ * input ever comes from the CUDA path) and timed on its own.  Same conventions as qoserve.h.
+ */
+#ifndef QOSERVE_OPS_H_
+#define QOSERVE_OPS_H_
+
+#include "qoserve.h"
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* GEMM epilogues (a4, a9, a11, a12, a13). */
+enum {
+  QOS_EPI_STORE_BF16 = 0, /* C bf16 [M][N] = acc                                              */
+  QOS_EPI_STORE_F32 = 1,  /* C f32  [M][N] = acc                                              */
+  QOS_EPI_BIAS_BF16 = 2,  /* C bf16 [M][N] = acc + bias[n]  (bias: device f32 [N]; Qwen QKV)   */
+  QOS_EPI_SILU_GATE = 3,  /* C bf16 [M][N/2]: B rows are gate/up interleaved in groups of 64:  */
+                          /*   B rows [128j, 128j+64) = gate rows [64j, 64j+64),               */
+                          /*   B rows [128j+64, 128j+128) = up rows [64j, 64j+64);             */
+                          /*   C[m][64j+c] = silu(acc[m][128j+c]) * acc[m][128j+64+c]          */
+  QOS_EPI_ADD_F32 = 4     /* C f32  [M][N] += acc  (residual-stream accumulate, a9/a12 + a3)  */
+};
+
+/* C = epi(A · B^T) with A device bf16 [M][K] row-major (K contiguous), B device bf16 [N][K]
+ * row-major (nn.Linear weight layout), fp32 accumulation on tcgen05 tensor cores.
+ * Requires K % 64 == 0, N % 32 == 0 (N % 128 == 0 for SILU_GATE), 16-byte aligned rows.
+ * M may be any value >= 1.  Stream-ordered. */
+int qos_op_gemm(const void* A, const void* B, void* C, int64_t M, int64_t N, int64_t K, int epi,
+                const float* bias, void* stream);
+
+/* a3: out[t][:] = bf16( x[t][:] / sqrt(mean(x[t]^2) + eps) * g[:] ), x device f32 [T][d],
+ * g device bf16 [d], out device bf16 [T][d].  Stream-ordered. */
+int qos_op_rmsnorm(const float* x, const void* g, void* out, int32_t T, int32_t d, float eps,
+                   void* stream);
+
+/* Write / read cached K and V of `req` at `layer`, positions [pos0, pos0+n), as host bf16 bits
+ * [n][Hkv_local][hd] (Hkv_local = this rank's kv heads).  The blocks must be allocated.
+ * qos_kv_write does not change the cached length.  Synchronous. */
+int qos_kv_write(qos_engine_t* eng, int32_t layer, int64_t req, int32_t pos0, int32_t n,
+                 const uint16_t* k_bf16, const uint16_t* v_bf16);
+int qos_kv_read(qos_engine_t* eng, int32_t layer, int64_t req, int32_t pos0, int32_t n,
+                uint16_t* k_bf16, uint16_t* v_bf16);
+
+/* a5 + a6: RoPE on q and k at each token's position, then append k and v to the paged cache
+ * at `layer`, for the token rows of `batch` (chunks then decodes, T rows).
+ * qkv: host bf16 [T][(H_local + 2 Hkv_local) * hd] (q | k | v per row, pre-RoPE);
+ * q_out: host bf16 [T][H_local * hd] post-RoPE q.  Does not change cached lengths.  Synchronous. */
+int qos_op_rope_kv_append(qos_engine_t* eng, int32_t layer, const qos_batch* batch,
+                          const uint16_t* qkv_bf16, uint16_t* q_out_bf16);
+
+/* a7 + a8: attention of the batch's token rows at `layer` over the paged cache (which must
+ * already hold every key the rows attend to: chunk keys 0..kv_start+len-1, decode keys
+ * 0..ctx_len).  q: host bf16 [T][H_local][hd] (post-RoPE); out: host f32 [T][H_local][hd]
+ * (the fp32 accumulator before the bf16 store, reading s10).  Synchronous. */
+int qos_op_attention(qos_engine_t* eng, int32_t layer, const qos_batch* batch,
+                     const uint16_t* q_bf16, float* out_f32);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* QOSERVE_OPS_H_ */

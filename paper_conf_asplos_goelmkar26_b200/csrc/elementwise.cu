@@ -1,0 +1,333 @@
+// elementwise.cu — HBM-bound per-token kernels of the hybrid step (SURVEY.md §8(a) rows a2, a3,
+// a5+a6, a13 gather, a14):
+//   embed_rmsnorm   x = E[tok] (fp32 residual init) and h = RMSNorm(x)·g1 of layer 0   (a2+a3)
+//   rmsnorm         h = RMSNorm(r)·g from the fp32 residual stream                       (a3)
+//   gather_rmsnorm  the R logit rows (last token of each chunk, every decode) + final norm (a13)
+//   rope_append     rotate-half RoPE of q and k at each row's position, K/V written to the
+//                   paged cache with 16-byte stores                                       (a5+a6)
+//   argmax          greedy token, lowest index on ties                                    (a14)
+// One CTA per token row; 16-byte vector loads/stores; fp32 statistics.
+#include <cfloat>
+
+#include "common.cuh"
+#include "internal.h"
+
+namespace qos {
+
+constexpr int kRowThreads = 256;
+
+QOS_DEV float block_sum(float v, float* red) {
+  v = warp_sum(v);
+  const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
+  __syncthreads();
+  if (l == 0) red[w] = v;
+  __syncthreads();
+  float s = 0.f;
+  for (int i = 0; i < (int)(blockDim.x >> 5); ++i) s += red[i];
+  return s;
+}
+
+// d is a multiple of 8; each thread handles 8 contiguous elements per iteration.  Two passes
+// over the row: sum of squares, then scale (the second read hits L1).
+QOS_DEV void norm_row(const float* x, const __nv_bfloat16* g, __nv_bfloat16* out, int d, float eps, float* red) {
+  float ss = 0.f;
+  for (int c = threadIdx.x * 8; c < d; c += blockDim.x * 8) {
+    const float4 a = *reinterpret_cast<const float4*>(x + c);
+    const float4 b = *reinterpret_cast<const float4*>(x + c + 4);
+    ss += a.x * a.x + a.y * a.y + a.z * a.z + a.w * a.w + b.x * b.x + b.y * b.y + b.z * b.z + b.w * b.w;
+  }
+  const float tot = block_sum(ss, red);
+  const float inv = rsqrtf(tot / float(d) + eps);
+  for (int c = threadIdx.x * 8; c < d; c += blockDim.x * 8) {
+    const float4 a = *reinterpret_cast<const float4*>(x + c);
+    const float4 b = *reinterpret_cast<const float4*>(x + c + 4);
+    const float v[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
+    const uint4 gw = *reinterpret_cast<const uint4*>(g + c);
+    const uint32_t gg[4] = {gw.x, gw.y, gw.z, gw.w};
+    uint32_t pk[4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+      pk[i] = pack_bf16(v[2 * i] * inv * bf16_lo(gg[i]), v[2 * i + 1] * inv * bf16_hi(gg[i]));
+    *reinterpret_cast<uint4*>(out + c) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+  }
+}
+
+__global__ void __launch_bounds__(kRowThreads) embed_rmsnorm_kernel(const int32_t* __restrict__ tokens,
+                                                                    const __nv_bfloat16* __restrict__ emb,
+                                                                    const __nv_bfloat16* __restrict__ g,
+                                                                    float* __restrict__ resid,
+                                                                    __nv_bfloat16* __restrict__ out, int d, float eps) {
+  __shared__ float red[32];
+  const int t = blockIdx.x;
+  const __nv_bfloat16* e = emb + size_t(tokens[t]) * d;
+  float* r = resid + size_t(t) * d;
+  for (int c = threadIdx.x * 8; c < d; c += blockDim.x * 8) {
+    const uint4 w = *reinterpret_cast<const uint4*>(e + c);
+    *reinterpret_cast<float4*>(r + c) = make_float4(bf16_lo(w.x), bf16_hi(w.x), bf16_lo(w.y), bf16_hi(w.y));
+    *reinterpret_cast<float4*>(r + c + 4) = make_float4(bf16_lo(w.z), bf16_hi(w.z), bf16_lo(w.w), bf16_hi(w.w));
+  }
+  // each thread re-reads only the elements it wrote: no barrier needed before norm_row
+  norm_row(r, g, out + size_t(t) * d, d, eps, red);
+}
+
+__global__ void __launch_bounds__(kRowThreads) rmsnorm_kernel(const float* __restrict__ x,
+                                                              const __nv_bfloat16* __restrict__ g,
+                                                              __nv_bfloat16* __restrict__ out, int d, float eps) {
+  __shared__ float red[32];
+  const int t = blockIdx.x;
+  norm_row(x + size_t(t) * d, g, out + size_t(t) * d, d, eps, red);
+}
+
+__global__ void __launch_bounds__(kRowThreads) gather_rmsnorm_kernel(const float* __restrict__ x,
+                                                                     const int32_t* __restrict__ rows,
+                                                                     const __nv_bfloat16* __restrict__ g,
+                                                                     __nv_bfloat16* __restrict__ out, int d,
+                                                                     float eps) {
+  __shared__ float red[32];
+  const int r = blockIdx.x;
+  norm_row(x + size_t(rows[r]) * d, g, out + size_t(r) * d, d, eps, red);
+}
+
+// resid[t] += add[t] (bf16); out[t] = RMSNorm(resid[t]) * g.  `out` may alias `add`: every
+// thread reads add[c] in pass 1 before it writes out[c] in pass 2 (same indices, same thread).
+__global__ void __launch_bounds__(kRowThreads) add_rmsnorm_kernel(float* __restrict__ resid, const __nv_bfloat16* add,
+                                                                  const __nv_bfloat16* __restrict__ g,
+                                                                  __nv_bfloat16* out, int d, float eps) {
+  __shared__ float red[32];
+  const int t = blockIdx.x;
+  float* r = resid + size_t(t) * d;
+  const __nv_bfloat16* a = add + size_t(t) * d;
+  for (int c = threadIdx.x * 8; c < d; c += blockDim.x * 8) {
+    const uint4 w = *reinterpret_cast<const uint4*>(a + c);
+    float4 x0 = *reinterpret_cast<float4*>(r + c), x1 = *reinterpret_cast<float4*>(r + c + 4);
+    x0.x += bf16_lo(w.x); x0.y += bf16_hi(w.x); x0.z += bf16_lo(w.y); x0.w += bf16_hi(w.y);
+    x1.x += bf16_lo(w.z); x1.y += bf16_hi(w.z); x1.z += bf16_lo(w.w); x1.w += bf16_hi(w.w);
+    *reinterpret_cast<float4*>(r + c) = x0;
+    *reinterpret_cast<float4*>(r + c + 4) = x1;
+  }
+  norm_row(r, g, out + size_t(t) * d, d, eps, red);
+}
+
+__global__ void add_f32_kernel(float* __restrict__ resid, const __nv_bfloat16* __restrict__ add, int64_t n) {
+  for (int64_t i = blockIdx.x * int64_t(blockDim.x) + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x)
+    resid[i] += __bfloat162float(add[i]);
+}
+
+__global__ void unshard_logits_kernel(const float* __restrict__ in, float* __restrict__ out, int R, int Vl, int tp) {
+  const int64_t n = int64_t(R) * Vl * tp;
+  for (int64_t i = blockIdx.x * int64_t(blockDim.x) + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x) {
+    const int j = int(i % Vl);
+    const int r = int((i / Vl) % R);
+    const int k = int(i / (int64_t(Vl) * R));
+    out[int64_t(r) * Vl * tp + int64_t(k) * Vl + j] = in[i];
+  }
+}
+
+// One CTA per token row.  qkv row = [q heads | k heads | v heads], each head hd bf16.
+// rope_tab[pos][i] = (cos, sin)(pos * theta^(-2i/hd)), i < hd/2, built in fp64 on the host.
+// slot = physical block * 16 + offset; cache plane layout [block][Hkv][16][hd].
+__global__ void rope_append_kernel(__nv_bfloat16* qkv, int qkv_ld, __nv_bfloat16* q_out,  // may alias (in place)
+                                   int q_ld, const int32_t* __restrict__ pos, const int32_t* __restrict__ slot,
+                                   const float2* __restrict__ rope_tab, __nv_bfloat16* __restrict__ kplane,
+                                   __nv_bfloat16* __restrict__ vplane, int H, int Hkv, int hd) {
+  const int t = blockIdx.x;
+  const int p = pos[t];
+  const int sl = slot[t];
+  const int blk = sl >> 4, off = sl & 15;
+  const int half = hd / 2;
+  const float2* tab = rope_tab + size_t(p) * half;
+  __nv_bfloat16* row = qkv + size_t(t) * qkv_ld;
+  // q and k: each thread rotates 8 pairs (i .. i+7 with i + half)
+  const int npair_vec = half / 8;
+  for (int w = threadIdx.x; w < (H + Hkv) * npair_vec; w += blockDim.x) {
+    const int h = w / npair_vec, i0 = (w % npair_vec) * 8;
+    const __nv_bfloat16* src = row + size_t(h) * hd;
+    const uint4 a = *reinterpret_cast<const uint4*>(src + i0);
+    const uint4 b = *reinterpret_cast<const uint4*>(src + half + i0);
+    const uint32_t aw[4] = {a.x, a.y, a.z, a.w}, bw[4] = {b.x, b.y, b.z, b.w};
+    uint32_t ra[4], rb[4];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      const float2 cs0 = tab[i0 + 2 * k], cs1 = tab[i0 + 2 * k + 1];
+      const float x0 = bf16_lo(aw[k]), x1 = bf16_hi(aw[k]);
+      const float y0 = bf16_lo(bw[k]), y1 = bf16_hi(bw[k]);
+      ra[k] = pack_bf16(x0 * cs0.x - y0 * cs0.y, x1 * cs1.x - y1 * cs1.y);
+      rb[k] = pack_bf16(y0 * cs0.x + x0 * cs0.y, y1 * cs1.x + x1 * cs1.y);
+    }
+    __nv_bfloat16* dst;
+    if (h < H) {
+      dst = q_out + size_t(t) * q_ld + size_t(h) * hd;
+    } else {
+      dst = kplane + ((size_t(blk) * Hkv + (h - H)) * 16 + off) * hd;
+    }
+    *reinterpret_cast<uint4*>(dst + i0) = make_uint4(ra[0], ra[1], ra[2], ra[3]);
+    *reinterpret_cast<uint4*>(dst + half + i0) = make_uint4(rb[0], rb[1], rb[2], rb[3]);
+  }
+  // v: straight copy, 16 B per thread
+  const int nv = Hkv * hd / 8;
+  for (int w = threadIdx.x; w < nv; w += blockDim.x) {
+    const int h = (w * 8) / hd, c = (w * 8) % hd;
+    const uint4 v = *reinterpret_cast<const uint4*>(row + size_t(H + Hkv + h) * hd + c);
+    *reinterpret_cast<uint4*>(vplane + ((size_t(blk) * Hkv + h) * 16 + off) * hd + c) = v;
+  }
+}
+
+// argmax per row; ties -> lowest index.  logits f32 or bf16 [R][V].
+__global__ void argmax_kernel(const void* __restrict__ logits, int is_f32, int V, int32_t* __restrict__ out) {
+  const int r = blockIdx.x;
+  float best = -INFINITY;
+  int bi = 0x7fffffff;
+  for (int i = threadIdx.x; i < V; i += blockDim.x) {
+    const float v = is_f32 ? reinterpret_cast<const float*>(logits)[size_t(r) * V + i]
+                           : __bfloat162float(reinterpret_cast<const __nv_bfloat16*>(logits)[size_t(r) * V + i]);
+    if (v > best || (v == best && i < bi)) {
+      best = v;
+      bi = i;
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const float ov = __shfl_xor_sync(0xffffffffu, best, o);
+    const int oi = __shfl_xor_sync(0xffffffffu, bi, o);
+    if (ov > best || (ov == best && oi < bi)) {
+      best = ov;
+      bi = oi;
+    }
+  }
+  __shared__ float sv[32];
+  __shared__ int si[32];
+  const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
+  if (l == 0) {
+    sv[w] = best;
+    si[w] = bi;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    for (int k = 1; k < (int)(blockDim.x >> 5); ++k)
+      if (sv[k] > best || (sv[k] == best && si[k] < bi)) {
+        best = sv[k];
+        bi = si[k];
+      }
+    out[r] = bi;
+  }
+}
+
+__global__ void f32_to_bf16_kernel(const float* __restrict__ x, __nv_bfloat16* __restrict__ y, int64_t n) {
+  for (int64_t i = blockIdx.x * int64_t(blockDim.x) + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x)
+    y[i] = __float2bfloat16_rn(x[i]);
+}
+
+__global__ void kv_scatter_kernel(__nv_bfloat16* __restrict__ plane, const int32_t* __restrict__ trow, int pos0, int n,
+                                  int Hkv, int hd, const __nv_bfloat16* __restrict__ src) {
+  const int64_t total = int64_t(n) * Hkv * hd;
+  for (int64_t e = blockIdx.x * int64_t(blockDim.x) + threadIdx.x; e < total; e += int64_t(gridDim.x) * blockDim.x) {
+    const int j = int(e % hd), h = int((e / hd) % Hkv), i = int(e / (int64_t(hd) * Hkv));
+    const int p = pos0 + i;
+    plane[((int64_t(trow[p >> 4]) * Hkv + h) * 16 + (p & 15)) * hd + j] = src[e];
+  }
+}
+__global__ void kv_gather_kernel(const __nv_bfloat16* __restrict__ plane, const int32_t* __restrict__ trow, int pos0,
+                                 int n, int Hkv, int hd, __nv_bfloat16* __restrict__ dst) {
+  const int64_t total = int64_t(n) * Hkv * hd;
+  for (int64_t e = blockIdx.x * int64_t(blockDim.x) + threadIdx.x; e < total; e += int64_t(gridDim.x) * blockDim.x) {
+    const int j = int(e % hd), h = int((e / hd) % Hkv), i = int(e / (int64_t(hd) * Hkv));
+    const int p = pos0 + i;
+    dst[e] = plane[((int64_t(trow[p >> 4]) * Hkv + h) * 16 + (p & 15)) * hd + j];
+  }
+}
+__global__ void table_update_kernel(int32_t* __restrict__ tables, int table_w, const int32_t* __restrict__ tr, int n) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) tables[size_t(tr[3 * i]) * table_w + tr[3 * i + 1]] = tr[3 * i + 2];
+}
+
+// ------------------------------------------------------------------------------ host
+static int grid_of(int64_t n) {
+  const int64_t b = (n + 255) / 256;
+  return int(b < 1 ? 1 : (b > 4096 ? 4096 : b));
+}
+cudaError_t launch_kv_scatter(void* plane, const int32_t* d_table_row, int pos0, int n, int Hkv, int hd,
+                              const void* src, cudaStream_t st) {
+  if (n == 0) return cudaSuccess;
+  count_launch();
+  kv_scatter_kernel<<<grid_of(int64_t(n) * Hkv * hd), 256, 0, st>>>((__nv_bfloat16*)plane, d_table_row, pos0, n, Hkv,
+                                                                     hd, (const __nv_bfloat16*)src);
+  return cudaGetLastError();
+}
+cudaError_t launch_kv_gather(const void* plane, const int32_t* d_table_row, int pos0, int n, int Hkv, int hd, void* dst,
+                             cudaStream_t st) {
+  if (n == 0) return cudaSuccess;
+  count_launch();
+  kv_gather_kernel<<<grid_of(int64_t(n) * Hkv * hd), 256, 0, st>>>((const __nv_bfloat16*)plane, d_table_row, pos0, n,
+                                                                    Hkv, hd, (__nv_bfloat16*)dst);
+  return cudaGetLastError();
+}
+cudaError_t launch_table_update(int32_t* tables, int table_w, const int32_t* triples, int n, cudaStream_t st) {
+  if (n == 0) return cudaSuccess;
+  count_launch();
+  table_update_kernel<<<(n + 255) / 256, 256, 0, st>>>(tables, table_w, triples, n);
+  return cudaGetLastError();
+}
+cudaError_t launch_embed_rmsnorm(const int32_t* tokens, const void* emb, const void* g, float* resid, void* out,
+                                 int T, int d, float eps, cudaStream_t st) {
+  if (T == 0) return cudaSuccess;
+  count_launch();
+  embed_rmsnorm_kernel<<<T, kRowThreads, 0, st>>>(tokens, (const __nv_bfloat16*)emb, (const __nv_bfloat16*)g, resid,
+                                                  (__nv_bfloat16*)out, d, eps);
+  return cudaGetLastError();
+}
+cudaError_t launch_rmsnorm(const float* x, const void* g, void* out, int T, int d, float eps, cudaStream_t st) {
+  if (T == 0) return cudaSuccess;
+  count_launch();
+  rmsnorm_kernel<<<T, kRowThreads, 0, st>>>(x, (const __nv_bfloat16*)g, (__nv_bfloat16*)out, d, eps);
+  return cudaGetLastError();
+}
+cudaError_t launch_gather_rmsnorm(const float* x, const int32_t* rows, const void* g, void* out, int R, int d,
+                                  float eps, cudaStream_t st) {
+  if (R == 0) return cudaSuccess;
+  count_launch();
+  gather_rmsnorm_kernel<<<R, kRowThreads, 0, st>>>(x, rows, (const __nv_bfloat16*)g, (__nv_bfloat16*)out, d, eps);
+  return cudaGetLastError();
+}
+cudaError_t launch_rope_append(void* qkv, int qkv_ld, void* q_out, int q_ld, const int32_t* pos, const int32_t* slot,
+                               const float2* rope_tab, void* kplane, void* vplane, int T, int H, int Hkv, int hd,
+                               cudaStream_t st) {
+  if (T == 0) return cudaSuccess;
+  count_launch();
+  rope_append_kernel<<<T, 128, 0, st>>>((__nv_bfloat16*)qkv, qkv_ld, (__nv_bfloat16*)q_out, q_ld, pos, slot, rope_tab,
+                                        (__nv_bfloat16*)kplane, (__nv_bfloat16*)vplane, H, Hkv, hd);
+  return cudaGetLastError();
+}
+cudaError_t launch_add_rmsnorm(float* resid, const void* add, const void* g, void* out, int T, int d, float eps,
+                               cudaStream_t st) {
+  if (T == 0) return cudaSuccess;
+  count_launch();
+  add_rmsnorm_kernel<<<T, kRowThreads, 0, st>>>(resid, (const __nv_bfloat16*)add, (const __nv_bfloat16*)g,
+                                                (__nv_bfloat16*)out, d, eps);
+  return cudaGetLastError();
+}
+cudaError_t launch_add_f32(float* resid, const void* add_bf16, size_t n, cudaStream_t st) {
+  if (n == 0) return cudaSuccess;
+  count_launch();
+  add_f32_kernel<<<grid_of(int64_t(n)), 256, 0, st>>>(resid, (const __nv_bfloat16*)add_bf16, int64_t(n));
+  return cudaGetLastError();
+}
+cudaError_t launch_unshard_logits(const float* in, float* out, int R, int Vl, int tp, cudaStream_t st) {
+  count_launch();
+  unshard_logits_kernel<<<grid_of(int64_t(R) * Vl * tp), 256, 0, st>>>(in, out, R, Vl, tp);
+  return cudaGetLastError();
+}
+cudaError_t launch_argmax(const void* logits, int logits_f32, int R, int V, int32_t* out, cudaStream_t st) {
+  if (R == 0) return cudaSuccess;
+  count_launch();
+  argmax_kernel<<<R, 1024, 0, st>>>(logits, logits_f32, V, out);
+  return cudaGetLastError();
+}
+cudaError_t launch_f32_to_bf16(const float* x, void* y, int64_t n, cudaStream_t st) {
+  if (n == 0) return cudaSuccess;
+  count_launch();
+  const int blocks = int((n + 1023) / 1024 < 4096 ? (n + 1023) / 1024 : 4096);
+  f32_to_bf16_kernel<<<blocks, 1024, 0, st>>>(x, (__nv_bfloat16*)y, n);
+  return cudaGetLastError();
+}
+
+}  // namespace qos

@@ -1,0 +1,1285 @@
+// engine.cu — host runtime of libqoserve.so: the C ABI of include/qoserve.h and
+// include/qoserve_ops.h.  Owns the weight shard, the paged KV pool with its deterministic block
+// allocator and device-resident block tables, the step workspaces, and the per-step metadata
+// builder that turns a QoServe batch descriptor (all decodes + the
+// deadline-selected prefill chunks, Alg. 1) into the kernels' work lists.
+#include <dlfcn.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <queue>
+#include <string>
+#include <unordered_map>
+#include <unordered_set>
+#include <vector>
+
+#include "internal.h"
+#include <cuda_bf16.h>
+#include <nccl.h>
+
+namespace qos {
+
+static thread_local std::string g_last_error;
+static std::atomic<int64_t> g_launches{0};
+
+int set_error(int code, const char* msg) {
+  g_last_error = msg ? msg : "";
+  return code;
+}
+int set_cuda_error(cudaError_t e, const char* where) {
+  g_last_error = std::string(where) + ": " + cudaGetErrorString(e);
+  return QOS_ERR_CUDA;
+}
+int count_launch(int n) {
+  g_launches.fetch_add(n, std::memory_order_relaxed);
+  return 0;
+}
+
+#define QOS_CU(call)                                                   \
+  do {                                                                 \
+    cudaError_t _e = (call);                                           \
+    if (_e != cudaSuccess) return set_cuda_error(_e, #call);           \
+  } while (0)
+#define QOS_TRY(call)             \
+  do {                            \
+    int _r = (call);              \
+    if (_r != QOS_OK) return _r;  \
+  } while (0)
+
+static inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+// ------------------------------------------------------------------ NCCL (dlopen'ed)
+struct Nccl {
+  void* so = nullptr;
+  decltype(&ncclGetUniqueId) getUniqueId = nullptr;
+  decltype(&ncclCommInitRank) commInitRank = nullptr;
+  decltype(&ncclCommDestroy) commDestroy = nullptr;
+  decltype(&ncclCommAbort) commAbort = nullptr;
+  decltype(&ncclAllReduce) allReduce = nullptr;
+  decltype(&ncclAllGather) allGather = nullptr;
+  decltype(&ncclGetErrorString) errStr = nullptr;
+  bool load() {
+    if (so) return true;
+    const char* names[] = {"libnccl.so.2", "libnccl.so"};
+    for (const char* n : names) {
+      so = dlopen(n, RTLD_NOW | RTLD_GLOBAL);
+      if (so) break;
+    }
+    if (!so) return false;
+    getUniqueId = (decltype(getUniqueId))dlsym(so, "ncclGetUniqueId");
+    commInitRank = (decltype(commInitRank))dlsym(so, "ncclCommInitRank");
+    commDestroy = (decltype(commDestroy))dlsym(so, "ncclCommDestroy");
+    commAbort = (decltype(commAbort))dlsym(so, "ncclCommAbort");
+    allReduce = (decltype(allReduce))dlsym(so, "ncclAllReduce");
+    allGather = (decltype(allGather))dlsym(so, "ncclAllGather");
+    errStr = (decltype(errStr))dlsym(so, "ncclGetErrorString");
+    return getUniqueId && commInitRank && commDestroy && allReduce && allGather;
+  }
+};
+static Nccl g_nccl;
+static std::mutex g_nccl_mu;
+
+// ------------------------------------------------------------------ shapes / sharding
+struct Shard {
+  int H, Hkv, F, V;       // local counts
+  int h0, kv0, f0, v0;    // first global index owned
+};
+static Shard make_shard(const qos_model_cfg& c, int rank, int tp) {
+  Shard s;
+  s.H = c.n_heads / tp;
+  s.Hkv = c.n_kv_heads / tp;
+  s.F = c.ffn_dim / tp;
+  s.V = c.vocab / tp;
+  s.h0 = rank * s.H;
+  s.kv0 = rank * s.Hkv;
+  s.f0 = rank * s.F;
+  s.v0 = rank * s.V;
+  return s;
+}
+
+struct WeightLayout {   // byte offsets inside the weight arena
+  struct L {
+    size_t ln1, ln2, wqkv, bqkv, wo, wgu, wd;
+  };
+  std::vector<L> layers;
+  size_t emb, lnf, head, total;
+};
+static WeightLayout weight_layout(const qos_model_cfg& c, const Shard& s) {
+  WeightLayout w;
+  size_t off = 0;
+  auto take = [&](size_t bytes) {
+    size_t o = off;
+    off = align_up(off + bytes, 256);
+    return o;
+  };
+  const size_t d = c.d_model, hd = c.head_dim;
+  const size_t nqkv = (size_t(s.H) + 2 * s.Hkv) * hd;
+  for (int l = 0; l < c.n_layers; ++l) {
+    WeightLayout::L L;
+    L.ln1 = take(d * 2);
+    L.ln2 = take(d * 2);
+    L.wqkv = take(nqkv * d * 2);
+    L.bqkv = c.qkv_bias ? take(nqkv * 4) : 0;
+    L.wo = take(d * size_t(s.H) * hd * 2);
+    L.wgu = take(2 * size_t(s.F) * d * 2);
+    L.wd = take(d * size_t(s.F) * 2);
+    w.layers.push_back(L);
+  }
+  w.emb = take(size_t(c.vocab) * d * 2);
+  w.lnf = take(d * 2);
+  w.head = take(size_t(s.V) * d * 2);
+  w.total = off;
+  return w;
+}
+
+struct WsLayout {
+  size_t resid, h, qkv, attn, act, hR, logits, logits_loc, argmax, partials, meta[2], dbg, total;
+  size_t meta_bytes;
+  int max_items;
+};
+static constexpr int kMaxDecodeItems = 1 << 16;
+static WsLayout ws_layout(const qos_model_cfg& c, const Shard& s, int tp) {
+  WsLayout w;
+  size_t off = 0;
+  auto take = [&](size_t bytes) {
+    size_t o = off;
+    off = align_up(off + bytes, 1024);
+    return o;
+  };
+  const size_t Tm = c.max_batch_tokens, Rm = c.max_batch_rows, d = c.d_model, hd = c.head_dim;
+  const size_t nqkv = (size_t(s.H) + 2 * s.Hkv) * hd;
+  const size_t group = c.n_heads / c.n_kv_heads;
+  w.resid = take(Tm * d * 4);
+  w.h = take(Tm * d * 2);
+  w.qkv = take(Tm * nqkv * 2);
+  w.attn = take(Tm * size_t(s.H) * hd * 2);
+  w.act = take(Tm * size_t(s.F) * 2);
+  w.hR = take(Rm * d * 2);
+  w.logits = take(Rm * size_t(c.vocab) * 4);
+  w.logits_loc = tp > 1 ? take(Rm * size_t(c.vocab) * 4) : 0;
+  w.argmax = take(Rm * 4);
+  w.max_items = kMaxDecodeItems;
+  w.partials = take(size_t(w.max_items) * group * (hd + 2) * 4);
+  // metadata: tokens, pos, slot [Tm]; logit rows [Rm]; prefill items; decode items/rows; table updates
+  const int ppt = prefill_positions_per_tile(int(group));
+  const size_t max_pitems = (Tm / ppt + Rm + 1) * size_t(s.Hkv);
+  w.meta_bytes = align_up(3 * Tm * 4 + Rm * 4 + 64, 256) + align_up(max_pitems * sizeof(PrefillItem), 256) +
+                 align_up(size_t(w.max_items) * sizeof(DecodeItem), 256) + align_up(Rm * sizeof(DecodeRow), 256) +
+                 align_up(size_t(3) * 65536 * 4, 256);
+  w.meta[0] = take(w.meta_bytes);
+  w.meta[1] = take(w.meta_bytes);
+  w.dbg = 0;
+  w.total = off;
+  return w;
+}
+
+// ------------------------------------------------------------------ batch metadata (a1)
+struct StepMeta {
+  int T = 0, R = 0, n_prefill = 0, n_decode = 0;
+  int n_pitems = 0, n_ditems = 0, n_drows = 0, n_upd = 0;
+  // offsets (bytes) inside the metadata block
+  size_t o_tok, o_pos, o_slot, o_rows, o_pitems, o_ditems, o_drows, o_upd, used;
+};
+
+struct ReqState {
+  int row = -1;                 // block-table row
+  std::vector<int32_t> blocks;  // physical block ids
+  int cached = 0;               // tokens in cache
+};
+
+}  // namespace qos
+
+using namespace qos;
+
+struct qos_engine {
+  qos_model_cfg cfg{};
+  int device = 0, tp_rank = 0, tp_size = 1, num_sms = 148;
+  Shard sh{};
+  int nqkv = 0, table_w = 0;
+  WeightLayout wl;
+  WsLayout wsl{};
+  uint8_t *w = nullptr, *kv = nullptr, *ws = nullptr;
+  bool own_w = false, own_kv = false, own_ws = false;
+  size_t kv_bytes = 0, plane_elems = 0;
+  // tensor maps
+  struct LMaps {
+    CUtensorMap qkv[2], o[2], gu[2], d[2];  // [0]: box 128 rows, [1]: box 256 rows
+  };
+  std::vector<LMaps> lmaps;
+  CUtensorMap head_map[2];
+  CUtensorMap a_h, a_attn, a_act, a_hR, kv_map;
+  float2* rope_tab = nullptr;
+  int32_t* d_tables = nullptr;
+  // host state
+  std::vector<int32_t> free_heap;  // min-heap of free block ids
+  std::vector<int> free_rows;      // min-heap of free table rows
+  std::unordered_map<int64_t, ReqState> reqs;
+  std::vector<int32_t> pending_upd;  // (row, col, block) triples not yet on the device
+  // staging
+  uint8_t* h_meta[2] = {nullptr, nullptr};
+  cudaEvent_t meta_free[2] = {nullptr, nullptr};
+  int meta_cur = 0;
+  cudaStream_t stream = nullptr;  // internal stream for synchronous calls
+  // timing
+  bool timing = false;
+  std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> tev;
+  std::vector<cudaEvent_t> ev_pool;
+  size_t ev_used = 0;
+  // comm
+  ncclComm_t comm = nullptr;
+  // debug buffers for ops
+  void* dbg = nullptr;
+  size_t dbg_bytes = 0;
+};
+
+namespace {
+
+cudaEvent_t next_event(qos_engine* e) {
+  if (e->ev_used == e->ev_pool.size()) {
+    cudaEvent_t ev;
+    cudaEventCreate(&ev);
+    e->ev_pool.push_back(ev);
+  }
+  return e->ev_pool[e->ev_used++];
+}
+
+struct TimerScope {  // brackets one kernel class with events when timing is enabled
+  qos_engine* e;
+  int cls;
+  cudaStream_t st;
+  cudaEvent_t a = nullptr;
+  TimerScope(qos_engine* e_, int c, cudaStream_t s) : e(e_), cls(c), st(s) {
+    if (e->timing) {
+      a = next_event(e);
+      cudaEventRecord(a, st);
+    }
+  }
+  ~TimerScope() {
+    if (e->timing) {
+      cudaEvent_t b = next_event(e);
+      cudaEventRecord(b, st);
+      e->tev.push_back({cls, {a, b}});
+    }
+  }
+};
+
+int alloc_table_row(qos_engine* e) {
+  if (e->free_rows.empty()) return -1;
+  std::pop_heap(e->free_rows.begin(), e->free_rows.end(), std::greater<int>());
+  int r = e->free_rows.back();
+  e->free_rows.pop_back();
+  return r;
+}
+
+inline __nv_bfloat16* W(qos_engine* e, size_t off) { return reinterpret_cast<__nv_bfloat16*>(e->w + off); }
+
+int build_maps(qos_engine* e) {
+  const auto& c = e->cfg;
+  const int d = c.d_model, hd = c.head_dim;
+  e->lmaps.resize(c.n_layers);
+  for (int l = 0; l < c.n_layers; ++l) {
+    const auto& L = e->wl.layers[l];
+    for (int b = 0; b < 2; ++b) {
+      const uint32_t br = b ? 256 : 128;
+      QOS_TRY(make_tmap_2d_bf16(&e->lmaps[l].qkv[b], W(e, L.wqkv), e->nqkv, d, d, br, 64, true));
+      QOS_TRY(make_tmap_2d_bf16(&e->lmaps[l].o[b], W(e, L.wo), d, e->sh.H * hd, e->sh.H * hd, br, 64, true));
+      QOS_TRY(make_tmap_2d_bf16(&e->lmaps[l].gu[b], W(e, L.wgu), 2 * e->sh.F, d, d, br, 64, true));
+      QOS_TRY(make_tmap_2d_bf16(&e->lmaps[l].d[b], W(e, L.wd), d, e->sh.F, e->sh.F, br, 64, true));
+    }
+  }
+  for (int b = 0; b < 2; ++b)
+    QOS_TRY(make_tmap_2d_bf16(&e->head_map[b], W(e, e->wl.head), e->sh.V, d, d, b ? 256 : 128, 64, true));
+  const auto& s = e->wsl;
+  QOS_TRY(make_tmap_2d_bf16(&e->a_h, e->ws + s.h, c.max_batch_tokens, d, d, 128, 64, true));
+  QOS_TRY(make_tmap_2d_bf16(&e->a_attn, e->ws + s.attn, c.max_batch_tokens, e->sh.H * hd, e->sh.H * hd, 128, 64, true));
+  QOS_TRY(make_tmap_2d_bf16(&e->a_act, e->ws + s.act, c.max_batch_tokens, e->sh.F, e->sh.F, 128, 64, true));
+  QOS_TRY(make_tmap_2d_bf16(&e->a_hR, e->ws + s.hR, c.max_batch_rows, d, d, 128, 64, true));
+  QOS_TRY(make_tmap_3d_bf16(&e->kv_map, e->kv, hd, uint64_t(c.num_blocks) * e->sh.Hkv * 16, uint64_t(c.n_layers) * 2,
+                            64, 16, 1));
+  return QOS_OK;
+}
+
+int check_cfg(const qos_model_cfg* c, int tp) {
+  if (!c) return set_error(QOS_ERR_INVALID_ARG, "cfg is NULL");
+  if (c->n_layers < 1 || c->d_model < 64 || c->n_heads < 1 || c->n_kv_heads < 1 || c->ffn_dim < 64 || c->vocab < 32)
+    return set_error(QOS_ERR_INVALID_ARG, "bad model dims");
+  if (c->n_heads % c->n_kv_heads) return set_error(QOS_ERR_INVALID_ARG, "n_heads % n_kv_heads != 0");
+  if (c->head_dim != 64 && c->head_dim != 128) return set_error(QOS_ERR_UNSUPPORTED, "head_dim must be 64 or 128");
+  if (c->n_heads / c->n_kv_heads > 16) return set_error(QOS_ERR_UNSUPPORTED, "GQA group > 16");
+  if (c->block_size != 16) return set_error(QOS_ERR_UNSUPPORTED, "block_size must be 16");
+  if (tp < 1 || c->n_kv_heads % tp || c->n_heads % tp || c->ffn_dim % tp || c->vocab % tp)
+    return set_error(QOS_ERR_INVALID_ARG, "tp_size must divide n_kv_heads, n_heads, ffn_dim, vocab");
+  if (c->d_model % 64 || (c->ffn_dim / tp) % 128 || ((c->n_heads / tp) * c->head_dim) % 64 || (c->vocab / tp) % 32)
+    return set_error(QOS_ERR_UNSUPPORTED, "d_model % 64, (F/tp) % 128, (V/tp) % 32 required");
+  if (c->num_blocks < 1 || c->max_seq_len < 1 || c->max_requests < 1 || c->max_batch_tokens < 1 ||
+      c->max_batch_rows < 1)
+    return set_error(QOS_ERR_INVALID_ARG, "capacities must be >= 1");
+  if (c->max_batch_rows > c->max_batch_tokens) return set_error(QOS_ERR_INVALID_ARG, "max_batch_rows > max_batch_tokens");
+  return QOS_OK;
+}
+
+// Validate a batch and build its metadata into host staging `buf`.
+int build_step(qos_engine* e, const qos_batch* b, bool check_lengths, uint8_t* buf, StepMeta& m,
+               std::vector<int>* out_rows_tables = nullptr) {
+  const auto& c = e->cfg;
+  if (!b) return set_error(QOS_ERR_INVALID_ARG, "batch is NULL");
+  if (b->n_prefill < 0 || b->n_decode < 0 || (b->n_prefill && !b->prefill) || (b->n_decode && !b->decode))
+    return set_error(QOS_ERR_INVALID_ARG, "bad batch arrays");
+  m.n_prefill = b->n_prefill;
+  m.n_decode = b->n_decode;
+  m.R = b->n_prefill + b->n_decode;
+  int64_t T = b->n_decode;
+  for (int i = 0; i < b->n_prefill; ++i) {
+    if (b->prefill[i].chunk_len < 1 || !b->prefill[i].tokens) return set_error(QOS_ERR_INVALID_ARG, "chunk_len < 1");
+    T += b->prefill[i].chunk_len;
+  }
+  if (m.R == 0) return set_error(QOS_ERR_INVALID_ARG, "empty batch");
+  if (T > c.max_batch_tokens || m.R > c.max_batch_rows) return set_error(QOS_ERR_INVALID_ARG, "batch exceeds capacity");
+  m.T = int(T);
+  std::unordered_set<int64_t> seen;
+  auto lookup = [&](int64_t req, int start, int n, const ReqState** out) -> int {
+    auto it = e->reqs.find(req);
+    if (it == e->reqs.end()) return set_error(QOS_ERR_UNKNOWN_REQ, "request has no KV table");
+    if (!seen.insert(req).second) return set_error(QOS_ERR_INVALID_ARG, "request appears twice in one step");
+    if (start < 0 || n < 1) return set_error(QOS_ERR_INVALID_ARG, "bad position");
+    if (check_lengths && it->second.cached != start) return set_error(QOS_ERR_BAD_KV_START, "kv_start != cached length");
+    if (int64_t(start) + n > int64_t(it->second.blocks.size()) * 16)
+      return set_error(QOS_ERR_NOT_ALLOCATED, "step writes past the allocated blocks");
+    if (int64_t(start) + n > c.max_seq_len) return set_error(QOS_ERR_INVALID_ARG, "position >= max_seq_len");
+    *out = &it->second;
+    return QOS_OK;
+  };
+  // layout of the metadata block
+  size_t off = 0;
+  auto take = [&](size_t bytes) {
+    size_t o = off;
+    off = align_up(off + bytes, 256);
+    return o;
+  };
+  m.o_tok = take(size_t(T) * 4);
+  m.o_pos = take(size_t(T) * 4);
+  m.o_slot = take(size_t(T) * 4);
+  m.o_rows = take(size_t(m.R) * 4);
+  int32_t* tok = reinterpret_cast<int32_t*>(buf + m.o_tok);
+  int32_t* pos = reinterpret_cast<int32_t*>(buf + m.o_pos);
+  int32_t* slot = reinterpret_cast<int32_t*>(buf + m.o_slot);
+  int32_t* rows = reinterpret_cast<int32_t*>(buf + m.o_rows);
+
+  const int group = c.n_heads / c.n_kv_heads;
+  const int ppt = prefill_positions_per_tile(group);
+  std::vector<PrefillItem> pitems;
+  int t = 0;
+  for (int i = 0; i < b->n_prefill; ++i) {
+    const auto& ch = b->prefill[i];
+    const ReqState* rs;
+    QOS_TRY(lookup(ch.req, ch.kv_start, ch.chunk_len, &rs));
+    for (int j = 0; j < ch.chunk_len; ++j) {
+      const int tk = ch.tokens[j];
+      if (tk < 0 || tk >= c.vocab) return set_error(QOS_ERR_INVALID_ARG, "token id out of range");
+      const int p = ch.kv_start + j;
+      tok[t + j] = tk;
+      pos[t + j] = p;
+      slot[t + j] = rs->blocks[p >> 4] * 16 + (p & 15);
+    }
+    for (int p0 = 0; p0 < ch.chunk_len; p0 += ppt) {
+      for (int h = 0; h < e->sh.Hkv; ++h) {
+        PrefillItem it;
+        it.row0 = t + p0;
+        it.npos = std::min(ppt, ch.chunk_len - p0);
+        it.pos0 = ch.kv_start + p0;
+        it.table = rs->row;
+        it.kv_head = h;
+        it.pad = 0;
+        pitems.push_back(it);
+      }
+    }
+    t += ch.chunk_len;
+    rows[i] = t - 1;
+  }
+  // LPT: longest key ranges first
+  std::stable_sort(pitems.begin(), pitems.end(),
+                   [](const PrefillItem& a, const PrefillItem& b2) { return a.pos0 + a.npos > b2.pos0 + b2.npos; });
+  // decode split-K work list (balanced on sum of keys)
+  int64_t total_keys = 0;
+  for (int i = 0; i < b->n_decode; ++i) total_keys += int64_t(b->decode[i].ctx_len) + 1;
+  int split = 512;
+  {
+    const int64_t target = int64_t(e->num_sms) * 4;  // items per kv head per ... heuristic
+    auto count_items = [&](int s) {
+      int64_t n = 0;
+      for (int i = 0; i < b->n_decode; ++i) n += (int64_t(b->decode[i].ctx_len) + s) / s;
+      return n * e->sh.Hkv;
+    };
+    while (split > 64 && count_items(split) < target) split /= 2;
+    while (count_items(split) > e->wsl.max_items) split *= 2;
+  }
+  std::vector<DecodeItem> ditems;
+  std::vector<DecodeRow> drows;
+  int part = 0;
+  for (int i = 0; i < b->n_decode; ++i) {
+    const auto& dc = b->decode[i];
+    const ReqState* rs;
+    QOS_TRY(lookup(dc.req, dc.ctx_len, 1, &rs));
+    if (dc.token < 0 || dc.token >= c.vocab) return set_error(QOS_ERR_INVALID_ARG, "token id out of range");
+    const int p = dc.ctx_len;
+    tok[t] = dc.token;
+    pos[t] = p;
+    slot[t] = rs->blocks[p >> 4] * 16 + (p & 15);
+    rows[b->n_prefill + i] = t;
+    const int keys = p + 1;
+    const int nsplit = (keys + split - 1) / split;
+    DecodeRow dr;
+    dr.row = t;
+    dr.part0 = part;
+    dr.nsplit = nsplit;
+    drows.push_back(dr);
+    for (int h = 0; h < e->sh.Hkv; ++h)
+      for (int s = 0; s < nsplit; ++s) {
+        DecodeItem it;
+        it.row = t;
+        it.table = rs->row;
+        it.kv_head = h;
+        it.key0 = s * split;
+        it.key1 = std::min(keys, (s + 1) * split);
+        it.part = part + h * nsplit + s;
+        ditems.push_back(it);
+      }
+    part += e->sh.Hkv * nsplit;
+    ++t;
+  }
+  // longest items first
+  std::stable_sort(ditems.begin(), ditems.end(),
+                   [](const DecodeItem& a, const DecodeItem& b2) { return a.key1 - a.key0 > b2.key1 - b2.key0; });
+  m.n_pitems = int(pitems.size());
+  m.n_ditems = int(ditems.size());
+  m.n_drows = int(drows.size());
+  m.o_pitems = take(pitems.size() * sizeof(PrefillItem));
+  m.o_ditems = take(ditems.size() * sizeof(DecodeItem));
+  m.o_drows = take(drows.size() * sizeof(DecodeRow));
+  const size_t max_upd = 65536;
+  m.n_upd = int(std::min(e->pending_upd.size() / 3, max_upd));
+  m.o_upd = take(size_t(m.n_upd) * 12);
+  m.used = off;
+  if (m.used > e->wsl.meta_bytes) return set_error(QOS_ERR_INVALID_ARG, "metadata exceeds workspace");
+  if (!pitems.empty()) memcpy(buf + m.o_pitems, pitems.data(), pitems.size() * sizeof(PrefillItem));
+  if (!ditems.empty()) memcpy(buf + m.o_ditems, ditems.data(), ditems.size() * sizeof(DecodeItem));
+  if (!drows.empty()) memcpy(buf + m.o_drows, drows.data(), drows.size() * sizeof(DecodeRow));
+  if (m.n_upd) memcpy(buf + m.o_upd, e->pending_upd.data(), size_t(m.n_upd) * 12);
+  (void)out_rows_tables;
+  return QOS_OK;
+}
+
+// Upload staging -> device metadata block of the current buffer; returns device base.
+int upload_meta(qos_engine* e, const StepMeta& m, cudaStream_t st, uint8_t** d_meta) {
+  const int cur = e->meta_cur;
+  uint8_t* dm = e->ws + e->wsl.meta[cur];
+  QOS_CU(cudaStreamWaitEvent(st, e->meta_free[cur], 0));
+  QOS_CU(cudaMemcpyAsync(dm, e->h_meta[cur], m.used, cudaMemcpyHostToDevice, st));
+  if (m.n_upd) {
+    QOS_CU(launch_table_update(e->d_tables, e->table_w, reinterpret_cast<int32_t*>(dm + m.o_upd), m.n_upd, st));
+    e->pending_upd.erase(e->pending_upd.begin(), e->pending_upd.begin() + size_t(m.n_upd) * 3);
+  }
+  *d_meta = dm;
+  return QOS_OK;
+}
+
+// Wait until the staging buffer `cur` is no longer read by an in-flight copy/step.
+int acquire_staging(qos_engine* e) {
+  e->meta_cur ^= 1;
+  QOS_CU(cudaEventSynchronize(e->meta_free[e->meta_cur]));
+  return QOS_OK;
+}
+
+int release_staging(qos_engine* e, cudaStream_t st) {
+  QOS_CU(cudaEventRecord(e->meta_free[e->meta_cur], st));
+  return QOS_OK;
+}
+
+int flush_table_updates(qos_engine* e, cudaStream_t st) {
+  while (!e->pending_upd.empty()) {
+    QOS_TRY(acquire_staging(e));
+    const size_t n = std::min<size_t>(e->pending_upd.size() / 3, 65536);
+    memcpy(e->h_meta[e->meta_cur], e->pending_upd.data(), n * 12);
+    uint8_t* dm = e->ws + e->wsl.meta[e->meta_cur];
+    QOS_CU(cudaStreamWaitEvent(st, e->meta_free[e->meta_cur], 0));
+    QOS_CU(cudaMemcpyAsync(dm, e->h_meta[e->meta_cur], n * 12, cudaMemcpyHostToDevice, st));
+    QOS_CU(launch_table_update(e->d_tables, e->table_w, reinterpret_cast<int32_t*>(dm), int(n), st));
+    QOS_TRY(release_staging(e, st));
+    e->pending_upd.erase(e->pending_upd.begin(), e->pending_upd.begin() + n * 3);
+  }
+  return QOS_OK;
+}
+
+int gemm(qos_engine* e, const CUtensorMap& ta, const CUtensorMap (&tb)[2], int64_t M, int64_t N, int64_t K, int epi,
+         void* C, int64_t ldc, const float* bias, cudaStream_t st) {
+  const int bn = gemm_pick_bn(M, N, epi, e->num_sms);
+  count_launch();
+  return gemm_run(ta, tb[bn == 256 ? 1 : 0], bn, M, N, K, epi, C, ldc, bias, e->num_sms, st);
+}
+
+int allreduce_bf16(qos_engine* e, void* buf, size_t count, cudaStream_t st) {
+  ncclResult_t r = g_nccl.allReduce(buf, buf, count, ncclBfloat16, ncclSum, e->comm, st);
+  if (r != ncclSuccess) {
+    if (g_nccl.commAbort) g_nccl.commAbort(e->comm);
+    e->comm = nullptr;
+    return set_error(QOS_ERR_COMM, g_nccl.errStr ? g_nccl.errStr(r) : "ncclAllReduce failed");
+  }
+  return QOS_OK;
+}
+
+// The layer loop.  `dm` = device metadata block of this step.
+int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int logits_dtype, int32_t* next_tokens,
+               bool out_device, cudaStream_t st) {
+  const auto& c = e->cfg;
+  const int d = c.d_model, hd = c.head_dim, T = m.T, R = m.R;
+  const auto& s = e->wsl;
+  float* resid = reinterpret_cast<float*>(e->ws + s.resid);
+  void* h = e->ws + s.h;
+  __nv_bfloat16* qkv = reinterpret_cast<__nv_bfloat16*>(e->ws + s.qkv);
+  void* attn = e->ws + s.attn;
+  void* act = e->ws + s.act;
+  void* hR = e->ws + s.hR;
+  const int32_t* tok = reinterpret_cast<const int32_t*>(dm + m.o_tok);
+  const int32_t* pos = reinterpret_cast<const int32_t*>(dm + m.o_pos);
+  const int32_t* slot = reinterpret_cast<const int32_t*>(dm + m.o_slot);
+  const int32_t* rows = reinterpret_cast<const int32_t*>(dm + m.o_rows);
+  const size_t plane = e->plane_elems;
+  const bool tp = e->tp_size > 1;
+  {
+    TimerScope ts(e, QOS_T_EMBED, st);
+    QOS_CU(launch_embed_rmsnorm(tok, W(e, e->wl.emb), W(e, e->wl.layers[0].ln1), resid, h, T, d, c.rms_eps, st));
+  }
+  AttnLaunch al;
+  al.q = qkv;
+  al.q_ld = e->nqkv;
+  al.out = attn;
+  al.out_ld = e->sh.H * hd;
+  al.out_f32 = 0;
+  al.kv_tmap = &e->kv_map;
+  al.H = e->sh.H;
+  al.Hkv = e->sh.Hkv;
+  al.hd = hd;
+  al.num_blocks = int(c.num_blocks);
+  al.tables = e->d_tables;
+  al.table_w = e->table_w;
+  al.scale_log2 = float(1.4426950408889634 / std::sqrt(double(hd)));
+  for (int l = 0; l < c.n_layers; ++l) {
+    const auto& L = e->wl.layers[l];
+    const auto& M = e->lmaps[l];
+    if (l > 0 && !tp) {  // (tp: ln1 was applied by the add+norm after the previous all-reduce)
+      TimerScope ts(e, QOS_T_NORM, st);
+      QOS_CU(launch_rmsnorm(resid, W(e, L.ln1), h, T, d, c.rms_eps, st));
+    }
+    {
+      TimerScope ts(e, QOS_T_GEMM_QKV, st);
+      QOS_TRY(gemm(e, e->a_h, M.qkv, T, e->nqkv, d, c.qkv_bias ? EPI_BIAS_BF16 : EPI_STORE_BF16, qkv, e->nqkv,
+                   c.qkv_bias ? reinterpret_cast<const float*>(e->w + L.bqkv) : nullptr, st));
+    }
+    __nv_bfloat16* kpl = reinterpret_cast<__nv_bfloat16*>(e->kv) + (size_t(l) * 2 + 0) * plane;
+    __nv_bfloat16* vpl = reinterpret_cast<__nv_bfloat16*>(e->kv) + (size_t(l) * 2 + 1) * plane;
+    {
+      TimerScope ts(e, QOS_T_ROPE_APPEND, st);
+      QOS_CU(launch_rope_append(qkv, e->nqkv, qkv, e->nqkv, pos, slot, e->rope_tab, kpl, vpl, T, e->sh.H, e->sh.Hkv,
+                                hd, st));
+    }
+    al.layer = l;
+    if (m.n_pitems) {
+      TimerScope ts(e, QOS_T_PREFILL_ATTN, st);
+      QOS_CU(launch_prefill_attention(al, reinterpret_cast<const PrefillItem*>(dm + m.o_pitems), m.n_pitems, st));
+    }
+    if (m.n_ditems) {
+      TimerScope ts(e, QOS_T_DECODE_ATTN, st);
+      QOS_CU(launch_decode_attention(al, reinterpret_cast<const DecodeItem*>(dm + m.o_ditems), m.n_ditems,
+                                     reinterpret_cast<const DecodeRow*>(dm + m.o_drows), m.n_drows,
+                                     reinterpret_cast<float*>(e->ws + s.partials), 0, st));
+    }
+    if (!tp) {
+      TimerScope ts(e, QOS_T_GEMM_O, st);
+      QOS_TRY(gemm(e, e->a_attn, M.o, T, d, e->sh.H * hd, EPI_ADD_F32, resid, d, nullptr, st));
+    } else {
+      {
+        TimerScope ts(e, QOS_T_GEMM_O, st);
+        QOS_TRY(gemm(e, e->a_attn, M.o, T, d, e->sh.H * hd, EPI_STORE_BF16, h, d, nullptr, st));
+      }
+      TimerScope ts(e, QOS_T_ALLREDUCE, st);
+      QOS_TRY(allreduce_bf16(e, h, size_t(T) * d, st));
+    }
+    {
+      TimerScope ts(e, QOS_T_NORM, st);
+      if (tp) QOS_CU(launch_add_rmsnorm(resid, h, W(e, L.ln2), h, T, d, c.rms_eps, st));
+      else QOS_CU(launch_rmsnorm(resid, W(e, L.ln2), h, T, d, c.rms_eps, st));
+    }
+    {
+      TimerScope ts(e, QOS_T_GEMM_GATEUP, st);
+      QOS_TRY(gemm(e, e->a_h, M.gu, T, 2 * e->sh.F, d, EPI_SILU_GATE, act, e->sh.F, nullptr, st));
+    }
+    if (!tp) {
+      TimerScope ts(e, QOS_T_GEMM_DOWN, st);
+      QOS_TRY(gemm(e, e->a_act, M.d, T, d, e->sh.F, EPI_ADD_F32, resid, d, nullptr, st));
+    } else {
+      {
+        TimerScope ts(e, QOS_T_GEMM_DOWN, st);
+        QOS_TRY(gemm(e, e->a_act, M.d, T, d, e->sh.F, EPI_STORE_BF16, h, d, nullptr, st));
+      }
+      {
+        TimerScope ts(e, QOS_T_ALLREDUCE, st);
+        QOS_TRY(allreduce_bf16(e, h, size_t(T) * d, st));
+      }
+      if (l + 1 < c.n_layers) {
+        TimerScope ts(e, QOS_T_NORM, st);
+        QOS_CU(launch_add_rmsnorm(resid, h, W(e, e->wl.layers[l + 1].ln1), h, T, d, c.rms_eps, st));
+      } else {
+        TimerScope ts(e, QOS_T_NORM, st);
+        QOS_CU(launch_add_f32(resid, h, size_t(T) * d, st));
+      }
+    }
+  }
+  // final norm on the R logit rows + LM head
+  {
+    TimerScope ts(e, QOS_T_HEAD, st);
+    QOS_CU(launch_gather_rmsnorm(resid, rows, W(e, e->wl.lnf), hR, R, d, c.rms_eps, st));
+  }
+  // logits destination: f32 logits land in the caller's device buffer when possible
+  float* lg = reinterpret_cast<float*>(e->ws + s.logits);
+  const bool direct = out_device && logits && logits_dtype == QOS_F32 && !tp;
+  float* lout = direct ? reinterpret_cast<float*>(logits) : lg;
+  {
+    TimerScope ts(e, QOS_T_HEAD, st);
+    if (!tp) {
+      QOS_TRY(gemm(e, e->a_hR, e->head_map, R, c.vocab, d, EPI_STORE_F32, lout, c.vocab, nullptr, st));
+    } else {
+      float* loc = reinterpret_cast<float*>(e->ws + s.logits_loc);
+      QOS_TRY(gemm(e, e->a_hR, e->head_map, R, e->sh.V, d, EPI_STORE_F32, loc, e->sh.V, nullptr, st));
+      // all-gather of [R][V/tp] shards -> [tp][R][V/tp], then transpose into [R][V]
+      ncclResult_t r = g_nccl.allGather(loc, lg, size_t(R) * e->sh.V, ncclFloat32, e->comm, st);
+      if (r != ncclSuccess) return set_error(QOS_ERR_COMM, "ncclAllGather failed");
+      // gathered layout [tp][R][V/tp] -> [R][V] (logits_loc holds Rm*V floats when tp > 1)
+      QOS_CU(launch_unshard_logits(lg, loc, R, e->sh.V, e->tp_size, st));
+      lout = loc;
+    }
+  }
+  {
+    TimerScope ts(e, QOS_T_ARGMAX, st);
+    int32_t* am = reinterpret_cast<int32_t*>(e->ws + s.argmax);
+    QOS_CU(launch_argmax(lout, 1, R, c.vocab, am, st));
+    if (next_tokens) {
+      QOS_CU(cudaMemcpyAsync(next_tokens, am, size_t(R) * 4, out_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost,
+                             st));
+    }
+  }
+  if (logits && !direct) {
+    if (logits_dtype == QOS_F32) {
+      QOS_CU(cudaMemcpyAsync(logits, lout, size_t(R) * c.vocab * 4,
+                             out_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, st));
+    } else {
+      void* dst = out_device ? logits : e->ws + s.act;  // act is free at this point
+      QOS_CU(launch_f32_to_bf16(lout, dst, size_t(R) * c.vocab, st));
+      if (!out_device) QOS_CU(cudaMemcpyAsync(logits, dst, size_t(R) * c.vocab * 2, cudaMemcpyDeviceToHost, st));
+    }
+  }
+  return QOS_OK;
+}
+
+int do_step(qos_engine* e, const qos_batch* b, void* logits, int logits_dtype, int32_t* next_tokens, int on_host,
+            cudaStream_t st, bool check_and_advance) {
+  if (logits && logits_dtype != QOS_F32 && logits_dtype != QOS_BF16)
+    return set_error(QOS_ERR_INVALID_ARG, "logits_dtype");
+  if (cudaSetDevice(e->device) != cudaSuccess) return set_error(QOS_ERR_CUDA, "cudaSetDevice");
+  QOS_TRY(acquire_staging(e));
+  StepMeta m;
+  int r = build_step(e, b, check_and_advance, e->h_meta[e->meta_cur], m);
+  if (r != QOS_OK) {
+    e->meta_cur ^= 1;  // staging not used
+    return r;
+  }
+  e->tev.clear();
+  e->ev_used = 0;
+  uint8_t* dm = nullptr;
+  {
+    TimerScope ts(e, QOS_T_META, st);
+    QOS_TRY(upload_meta(e, m, st, &dm));
+  }
+  QOS_TRY(run_layers(e, m, dm, logits, logits_dtype, next_tokens, !on_host, st));
+  QOS_TRY(release_staging(e, st));
+  if (check_and_advance) {
+    for (int i = 0; i < b->n_prefill; ++i) e->reqs[b->prefill[i].req].cached += b->prefill[i].chunk_len;
+    for (int i = 0; i < b->n_decode; ++i) e->reqs[b->decode[i].req].cached += 1;
+  }
+  if (on_host) QOS_CU(cudaStreamSynchronize(st));
+  return QOS_OK;
+}
+
+}  // namespace
+
+// =================================================================== C ABI
+extern "C" {
+
+const char* qos_strerror(int code) {
+  switch (code) {
+    case QOS_OK: return "ok";
+    case QOS_ERR_INVALID_ARG: return "invalid argument";
+    case QOS_ERR_OOM: return "out of memory";
+    case QOS_ERR_UNKNOWN_REQ: return "unknown request";
+    case QOS_ERR_BAD_KV_START: return "kv_start/ctx_len does not match cached length";
+    case QOS_ERR_NOT_ALLOCATED: return "KV blocks not allocated";
+    case QOS_ERR_CUDA: return "CUDA error";
+    case QOS_ERR_COMM: return "NCCL error";
+    case QOS_ERR_UNSUPPORTED: return "unsupported shape";
+    default: return "unknown error";
+  }
+}
+const char* qos_last_error(void) { return g_last_error.c_str(); }
+
+int qos_engine_mem_sizes(const qos_model_cfg* cfg, int tp_size, qos_mem_sizes* out) {
+  QOS_TRY(check_cfg(cfg, tp_size));
+  if (!out) return set_error(QOS_ERR_INVALID_ARG, "out is NULL");
+  Shard s = make_shard(*cfg, 0, tp_size);
+  out->weight_bytes = weight_layout(*cfg, s).total;
+  out->kv_bytes = uint64_t(cfg->n_layers) * 2 * cfg->num_blocks * s.Hkv * 16 * cfg->head_dim * 2;
+  out->workspace_bytes = ws_layout(*cfg, s, tp_size).total;
+  return QOS_OK;
+}
+
+int qos_nccl_unique_id(uint8_t out[128]) {
+  std::lock_guard<std::mutex> g(g_nccl_mu);
+  if (!g_nccl.load()) return set_error(QOS_ERR_COMM, "libnccl.so.2 not loadable");
+  ncclUniqueId id;
+  if (g_nccl.getUniqueId(&id) != ncclSuccess) return set_error(QOS_ERR_COMM, "ncclGetUniqueId failed");
+  memcpy(out, &id, 128);
+  return QOS_OK;
+}
+
+int qos_engine_create(const qos_model_cfg* cfg, int device, int tp_rank, int tp_size, const uint8_t* nccl_uid,
+                      const qos_mem* mem, qos_engine_t** out) {
+  QOS_TRY(check_cfg(cfg, tp_size));
+  if (!out) return set_error(QOS_ERR_INVALID_ARG, "out is NULL");
+  if (tp_rank < 0 || tp_rank >= tp_size) return set_error(QOS_ERR_INVALID_ARG, "tp_rank");
+  if (tp_size > 1 && !nccl_uid) return set_error(QOS_ERR_INVALID_ARG, "nccl_uid required for tp_size > 1");
+  QOS_CU(cudaSetDevice(device));
+  auto* e = new qos_engine();
+  e->cfg = *cfg;
+  e->device = device;
+  e->tp_rank = tp_rank;
+  e->tp_size = tp_size;
+  cudaDeviceGetAttribute(&e->num_sms, cudaDevAttrMultiProcessorCount, device);
+  e->sh = make_shard(*cfg, tp_rank, tp_size);
+  e->nqkv = (e->sh.H + 2 * e->sh.Hkv) * cfg->head_dim;
+  e->table_w = (cfg->max_seq_len + 15) / 16;
+  e->wl = weight_layout(*cfg, e->sh);
+  e->wsl = ws_layout(*cfg, e->sh, tp_size);
+  e->plane_elems = size_t(cfg->num_blocks) * e->sh.Hkv * 16 * cfg->head_dim;
+  e->kv_bytes = uint64_t(cfg->n_layers) * 2 * e->plane_elems * 2;
+  auto fail = [&](int code) {
+    qos_engine_destroy(e);
+    return code;
+  };
+  auto get = [&](void* given, size_t bytes, uint8_t** dst, bool* own) -> int {
+    if (given) {
+      *dst = reinterpret_cast<uint8_t*>(given);
+      *own = false;
+      return QOS_OK;
+    }
+    void* p = nullptr;
+    cudaError_t er = cudaMalloc(&p, bytes);
+    if (er != cudaSuccess) return set_error(QOS_ERR_OOM, "cudaMalloc of an engine arena failed");
+    *dst = reinterpret_cast<uint8_t*>(p);
+    *own = true;
+    return QOS_OK;
+  };
+  int r;
+  if ((r = get(mem ? mem->weights : nullptr, e->wl.total, &e->w, &e->own_w)) != QOS_OK) return fail(r);
+  if ((r = get(mem ? mem->kv : nullptr, e->kv_bytes, &e->kv, &e->own_kv)) != QOS_OK) return fail(r);
+  if ((r = get(mem ? mem->workspace : nullptr, e->wsl.total, &e->ws, &e->own_ws)) != QOS_OK) return fail(r);
+  if (cudaMalloc(&e->d_tables, size_t(cfg->max_requests) * e->table_w * 4) != cudaSuccess)
+    return fail(set_error(QOS_ERR_OOM, "block tables"));
+  cudaMemset(e->d_tables, 0, size_t(cfg->max_requests) * e->table_w * 4);
+  // RoPE table in fp64 -> fp32 (reading s2)
+  {
+    const int half = cfg->head_dim / 2;
+    std::vector<float2> tab(size_t(cfg->max_seq_len) * half);
+    for (int p = 0; p < cfg->max_seq_len; ++p)
+      for (int i = 0; i < half; ++i) {
+        const double inv = std::pow(double(cfg->rope_theta), -2.0 * i / cfg->head_dim);
+        const double a = double(p) * inv;
+        tab[size_t(p) * half + i] = make_float2(float(std::cos(a)), float(std::sin(a)));
+      }
+    if (cudaMalloc(&e->rope_tab, tab.size() * sizeof(float2)) != cudaSuccess)
+      return fail(set_error(QOS_ERR_OOM, "rope table"));
+    cudaMemcpy(e->rope_tab, tab.data(), tab.size() * sizeof(float2), cudaMemcpyHostToDevice);
+  }
+  for (int i = 0; i < 2; ++i) {
+    if (cudaMallocHost(&e->h_meta[i], e->wsl.meta_bytes) != cudaSuccess) return fail(set_error(QOS_ERR_OOM, "pinned"));
+    cudaEventCreateWithFlags(&e->meta_free[i], cudaEventDisableTiming);
+  }
+  cudaStreamCreateWithFlags(&e->stream, cudaStreamNonBlocking);
+  e->free_heap.resize(size_t(cfg->num_blocks));
+  for (int64_t i = 0; i < cfg->num_blocks; ++i) e->free_heap[size_t(i)] = int32_t(i);  // sorted = valid min-heap
+  e->free_rows.resize(size_t(cfg->max_requests));
+  for (int i = 0; i < cfg->max_requests; ++i) e->free_rows[size_t(i)] = i;
+  if ((r = build_maps(e)) != QOS_OK) return fail(r);
+  if (tp_size > 1) {
+    std::lock_guard<std::mutex> g(g_nccl_mu);
+    if (!g_nccl.load()) return fail(set_error(QOS_ERR_COMM, "libnccl.so.2 not loadable"));
+    ncclUniqueId id;
+    memcpy(&id, nccl_uid, 128);
+    if (g_nccl.commInitRank(&e->comm, tp_size, id, tp_rank) != ncclSuccess)
+      return fail(set_error(QOS_ERR_COMM, "ncclCommInitRank failed"));
+  }
+  if (cudaDeviceSynchronize() != cudaSuccess) return fail(set_error(QOS_ERR_CUDA, "engine init"));
+  *out = e;
+  return QOS_OK;
+}
+
+int qos_engine_destroy(qos_engine_t* e) {
+  if (!e) return QOS_OK;
+  cudaSetDevice(e->device);
+  cudaDeviceSynchronize();
+  if (e->comm && g_nccl.commDestroy) g_nccl.commDestroy(e->comm);
+  if (e->own_w) cudaFree(e->w);
+  if (e->own_kv) cudaFree(e->kv);
+  if (e->own_ws) cudaFree(e->ws);
+  if (e->d_tables) cudaFree(e->d_tables);
+  if (e->rope_tab) cudaFree(e->rope_tab);
+  if (e->dbg) cudaFree(e->dbg);
+  for (int i = 0; i < 2; ++i) {
+    if (e->h_meta[i]) cudaFreeHost(e->h_meta[i]);
+    if (e->meta_free[i]) cudaEventDestroy(e->meta_free[i]);
+  }
+  for (auto ev : e->ev_pool) cudaEventDestroy(ev);
+  if (e->stream) cudaStreamDestroy(e->stream);
+  delete e;
+  return QOS_OK;
+}
+
+int qos_engine_load_synthetic(qos_engine_t* e, uint64_t seed) {
+  if (!e) return set_error(QOS_ERR_INVALID_ARG, "engine is NULL");
+  QOS_CU(cudaSetDevice(e->device));
+  const auto& c = e->cfg;
+  const auto& sh = e->sh;
+  const int d = c.d_model, hd = c.head_dim;
+  cudaStream_t st = e->stream;
+  char name[256];
+  auto H = [&](const char* s) { return fnv1a64(s); };
+  for (int l = 0; l < c.n_layers; ++l) {
+    const auto& L = e->wl.layers[l];
+    snprintf(name, sizeof name, "model.layers.%d.input_layernorm.weight", l);
+    QOS_CU(gen_fill_bf16(W(e, L.ln1), d, 1, d, seed, H(name), 0, 0, d, GEN_NORM, 1, st));
+    snprintf(name, sizeof name, "model.layers.%d.post_attention_layernorm.weight", l);
+    QOS_CU(gen_fill_bf16(W(e, L.ln2), d, 1, d, seed, H(name), 0, 0, d, GEN_NORM, 1, st));
+    // fused QKV [q rows | k rows | v rows] of this rank's heads
+    __nv_bfloat16* wqkv = W(e, L.wqkv);
+    snprintf(name, sizeof name, "model.layers.%d.self_attn.q_proj.weight", l);
+    QOS_CU(gen_fill_bf16(wqkv, d, int64_t(sh.H) * hd, d, seed, H(name), int64_t(sh.h0) * hd, 0, d, GEN_LINEAR, d, st));
+    snprintf(name, sizeof name, "model.layers.%d.self_attn.k_proj.weight", l);
+    QOS_CU(gen_fill_bf16(wqkv + size_t(sh.H) * hd * d, d, int64_t(sh.Hkv) * hd, d, seed, H(name),
+                         int64_t(sh.kv0) * hd, 0, d, GEN_LINEAR, d, st));
+    snprintf(name, sizeof name, "model.layers.%d.self_attn.v_proj.weight", l);
+    QOS_CU(gen_fill_bf16(wqkv + size_t(sh.H + sh.Hkv) * hd * d, d, int64_t(sh.Hkv) * hd, d, seed, H(name),
+                         int64_t(sh.kv0) * hd, 0, d, GEN_LINEAR, d, st));
+    if (c.qkv_bias) {
+      float* b = reinterpret_cast<float*>(e->w + L.bqkv);
+      snprintf(name, sizeof name, "model.layers.%d.self_attn.q_proj.bias", l);
+      QOS_CU(gen_fill_f32_bias(b, int64_t(sh.H) * hd, seed, H(name), int64_t(sh.h0) * hd, st));
+      snprintf(name, sizeof name, "model.layers.%d.self_attn.k_proj.bias", l);
+      QOS_CU(gen_fill_f32_bias(b + sh.H * hd, int64_t(sh.Hkv) * hd, seed, H(name), int64_t(sh.kv0) * hd, st));
+      snprintf(name, sizeof name, "model.layers.%d.self_attn.v_proj.bias", l);
+      QOS_CU(gen_fill_f32_bias(b + (sh.H + sh.Hkv) * hd, int64_t(sh.Hkv) * hd, seed, H(name), int64_t(sh.kv0) * hd, st));
+    }
+    // o_proj [d][H*hd]: this rank's columns
+    snprintf(name, sizeof name, "model.layers.%d.self_attn.o_proj.weight", l);
+    QOS_CU(gen_fill_bf16(W(e, L.wo), int64_t(sh.H) * hd, d, int64_t(sh.H) * hd, seed, H(name), 0, int64_t(sh.h0) * hd,
+                         int64_t(c.n_heads) * hd, GEN_LINEAR, c.n_heads * hd, st));
+    // gate/up interleaved in groups of 64 rows (QOS_EPI_SILU_GATE layout)
+    snprintf(name, sizeof name, "model.layers.%d.mlp.gate_proj.weight", l);
+    QOS_CU(gen_fill_bf16_ex(W(e, L.wgu), d, sh.F, d, seed, H(name), sh.f0, 0, d, GEN_LINEAR, d, 0, st));
+    snprintf(name, sizeof name, "model.layers.%d.mlp.up_proj.weight", l);
+    QOS_CU(gen_fill_bf16_ex(W(e, L.wgu), d, sh.F, d, seed, H(name), sh.f0, 0, d, GEN_LINEAR, d, 1, st));
+    // down_proj [d][F]: this rank's columns
+    snprintf(name, sizeof name, "model.layers.%d.mlp.down_proj.weight", l);
+    QOS_CU(gen_fill_bf16(W(e, L.wd), sh.F, d, sh.F, seed, H(name), 0, sh.f0, c.ffn_dim, GEN_LINEAR, c.ffn_dim, st));
+  }
+  QOS_CU(gen_fill_bf16(W(e, e->wl.emb), d, c.vocab, d, seed, H("model.embed_tokens.weight"), 0, 0, d, GEN_EMBED, 1, st));
+  QOS_CU(gen_fill_bf16(W(e, e->wl.lnf), d, 1, d, seed, H("model.norm.weight"), 0, 0, d, GEN_NORM, 1, st));
+  QOS_CU(gen_fill_bf16(W(e, e->wl.head), d, sh.V, d, seed, H("lm_head.weight"), sh.v0, 0, d, GEN_LINEAR, d, st));
+  QOS_CU(cudaStreamSynchronize(st));
+  return QOS_OK;
+}
+
+int qos_engine_read_weight(qos_engine_t* e, const char* name, int64_t row0, int64_t nrows, uint16_t* out) {
+  if (!e || !name || !out || row0 < 0 || nrows < 0) return set_error(QOS_ERR_INVALID_ARG, "read_weight args");
+  QOS_CU(cudaSetDevice(e->device));
+  const auto& c = e->cfg;
+  const auto& sh = e->sh;
+  const int d = c.d_model, hd = c.head_dim;
+  std::string n(name);
+  // generic: (device base, rows, cols, row stride, row remap)
+  const __nv_bfloat16* base = nullptr;
+  int64_t rows = 0, cols = 0, ld = 0;
+  int interleave = -1;
+  int layer = -1;
+  char suffix[128] = {0};
+  if (sscanf(name, "model.layers.%d.%127s", &layer, suffix) == 2) {
+    if (layer < 0 || layer >= c.n_layers) return set_error(QOS_ERR_INVALID_ARG, "layer");
+    const auto& L = e->wl.layers[layer];
+    std::string s(suffix);
+    if (s == "input_layernorm.weight") { base = W(e, L.ln1); rows = 1; cols = d; ld = d; }
+    else if (s == "post_attention_layernorm.weight") { base = W(e, L.ln2); rows = 1; cols = d; ld = d; }
+    else if (s == "self_attn.q_proj.weight") { base = W(e, L.wqkv); rows = int64_t(sh.H) * hd; cols = d; ld = d; }
+    else if (s == "self_attn.k_proj.weight") { base = W(e, L.wqkv) + size_t(sh.H) * hd * d; rows = int64_t(sh.Hkv) * hd; cols = d; ld = d; }
+    else if (s == "self_attn.v_proj.weight") { base = W(e, L.wqkv) + size_t(sh.H + sh.Hkv) * hd * d; rows = int64_t(sh.Hkv) * hd; cols = d; ld = d; }
+    else if (s == "self_attn.o_proj.weight") { base = W(e, L.wo); rows = d; cols = int64_t(sh.H) * hd; ld = cols; }
+    else if (s == "mlp.gate_proj.weight") { base = W(e, L.wgu); rows = sh.F; cols = d; ld = d; interleave = 0; }
+    else if (s == "mlp.up_proj.weight") { base = W(e, L.wgu); rows = sh.F; cols = d; ld = d; interleave = 1; }
+    else if (s == "mlp.down_proj.weight") { base = W(e, L.wd); rows = d; cols = sh.F; ld = cols; }
+    else return set_error(QOS_ERR_INVALID_ARG, "unknown tensor name");
+  } else if (n == "model.embed_tokens.weight") { base = W(e, e->wl.emb); rows = c.vocab; cols = d; ld = d; }
+  else if (n == "model.norm.weight") { base = W(e, e->wl.lnf); rows = 1; cols = d; ld = d; }
+  else if (n == "lm_head.weight") { base = W(e, e->wl.head); rows = sh.V; cols = d; ld = d; }
+  else return set_error(QOS_ERR_INVALID_ARG, "unknown tensor name");
+  if (row0 + nrows > rows) return set_error(QOS_ERR_INVALID_ARG, "row range");
+  for (int64_t r = 0; r < nrows; ++r) {
+    int64_t sr = row0 + r;
+    int64_t dr = interleave >= 0 ? (sr / 64) * 128 + interleave * 64 + sr % 64 : sr;
+    QOS_CU(cudaMemcpy(out + r * cols, base + dr * ld, size_t(cols) * 2, cudaMemcpyDeviceToHost));
+  }
+  return QOS_OK;
+}
+
+// ------------------------------------------------------------------ KV allocator
+int qos_kv_alloc(qos_engine_t* e, int64_t req, int32_t n_tokens_total) {
+  if (!e || n_tokens_total < 0) return set_error(QOS_ERR_INVALID_ARG, "kv_alloc args");
+  if (n_tokens_total > e->cfg.max_seq_len) return set_error(QOS_ERR_INVALID_ARG, "n_tokens_total > max_seq_len");
+  const int need_total = (n_tokens_total + 15) / 16;
+  auto it = e->reqs.find(req);
+  const int have = it == e->reqs.end() ? 0 : int(it->second.blocks.size());
+  const int need = need_total - have;
+  if (need > int64_t(e->free_heap.size())) return set_error(QOS_ERR_OOM, "KV pool exhausted");
+  if (it == e->reqs.end()) {
+    if (e->free_rows.empty()) return set_error(QOS_ERR_OOM, "max_requests reached");
+    ReqState rs;
+    rs.row = alloc_table_row(e);
+    it = e->reqs.emplace(req, std::move(rs)).first;
+  }
+  ReqState& rs = it->second;
+  for (int k = 0; k < need; ++k) {
+    std::pop_heap(e->free_heap.begin(), e->free_heap.end(), std::greater<int32_t>());
+    const int32_t blk = e->free_heap.back();
+    e->free_heap.pop_back();
+    const int col = int(rs.blocks.size());
+    rs.blocks.push_back(blk);
+    e->pending_upd.push_back(rs.row);
+    e->pending_upd.push_back(col);
+    e->pending_upd.push_back(blk);
+  }
+  return QOS_OK;
+}
+
+int qos_kv_free(qos_engine_t* e, int64_t req) {
+  if (!e) return set_error(QOS_ERR_INVALID_ARG, "engine is NULL");
+  auto it = e->reqs.find(req);
+  if (it == e->reqs.end()) return set_error(QOS_ERR_UNKNOWN_REQ, "unknown request");
+  for (int32_t b : it->second.blocks) {
+    e->free_heap.push_back(b);
+    std::push_heap(e->free_heap.begin(), e->free_heap.end(), std::greater<int32_t>());
+  }
+  e->free_rows.push_back(it->second.row);
+  std::push_heap(e->free_rows.begin(), e->free_rows.end(), std::greater<int>());
+  e->reqs.erase(it);
+  return QOS_OK;
+}
+
+int qos_kv_table(qos_engine_t* e, int64_t req, int32_t* out, int32_t cap, int32_t* n_out) {
+  if (!e || !n_out || (cap > 0 && !out)) return set_error(QOS_ERR_INVALID_ARG, "kv_table args");
+  auto it = e->reqs.find(req);
+  if (it == e->reqs.end()) return set_error(QOS_ERR_UNKNOWN_REQ, "unknown request");
+  const auto& b = it->second.blocks;
+  *n_out = int32_t(b.size());
+  for (int32_t i = 0; i < cap && i < int32_t(b.size()); ++i) out[i] = b[size_t(i)];
+  return QOS_OK;
+}
+
+int qos_kv_table_device(qos_engine_t* e, int64_t req, int32_t* out, int32_t cap, int32_t* n_out) {
+  if (!e || !n_out || (cap > 0 && !out)) return set_error(QOS_ERR_INVALID_ARG, "kv_table_device args");
+  auto it = e->reqs.find(req);
+  if (it == e->reqs.end()) return set_error(QOS_ERR_UNKNOWN_REQ, "unknown request");
+  QOS_CU(cudaSetDevice(e->device));
+  QOS_TRY(flush_table_updates(e, e->stream));
+  QOS_CU(cudaStreamSynchronize(e->stream));
+  const int n = int(it->second.blocks.size());
+  *n_out = n;
+  const int k = std::min(n, int(cap));
+  if (k > 0) QOS_CU(cudaMemcpy(out, e->d_tables + size_t(it->second.row) * e->table_w, size_t(k) * 4, cudaMemcpyDeviceToHost));
+  return QOS_OK;
+}
+
+int qos_kv_cached_len(qos_engine_t* e, int64_t req, int32_t* out) {
+  if (!e || !out) return set_error(QOS_ERR_INVALID_ARG, "args");
+  auto it = e->reqs.find(req);
+  if (it == e->reqs.end()) return set_error(QOS_ERR_UNKNOWN_REQ, "unknown request");
+  *out = it->second.cached;
+  return QOS_OK;
+}
+
+int qos_kv_free_blocks(qos_engine_t* e, int64_t* out) {
+  if (!e || !out) return set_error(QOS_ERR_INVALID_ARG, "args");
+  *out = int64_t(e->free_heap.size());
+  return QOS_OK;
+}
+
+int qos_kv_fill_synthetic(qos_engine_t* e, int64_t req, int32_t n_tokens, uint64_t seed) {
+  if (!e || n_tokens < 0) return set_error(QOS_ERR_INVALID_ARG, "args");
+  auto it = e->reqs.find(req);
+  if (it == e->reqs.end()) return set_error(QOS_ERR_UNKNOWN_REQ, "unknown request");
+  if (int64_t(it->second.blocks.size()) * 16 < n_tokens) return set_error(QOS_ERR_NOT_ALLOCATED, "not allocated");
+  QOS_CU(cudaSetDevice(e->device));
+  cudaStream_t st = e->stream;
+  QOS_TRY(flush_table_updates(e, st));
+  const int32_t* trow = e->d_tables + size_t(it->second.row) * e->table_w;
+  char name[128];
+  for (int l = 0; l < e->cfg.n_layers; ++l)
+    for (int kv = 0; kv < 2; ++kv) {
+      snprintf(name, sizeof name, "kvfill.%d.%c.%lld", l, kv ? 'v' : 'k', (long long)req);
+      void* plane = reinterpret_cast<__nv_bfloat16*>(e->kv) + (size_t(l) * 2 + kv) * e->plane_elems;
+      QOS_CU(kvfill_launch(plane, trow, n_tokens, e->sh.Hkv, e->cfg.n_kv_heads, e->sh.kv0, e->cfg.head_dim, seed,
+                           fnv1a64(name), st));
+    }
+  QOS_CU(cudaStreamSynchronize(st));
+  it->second.cached = n_tokens;
+  return QOS_OK;
+}
+
+// ------------------------------------------------------------------ step / profile / timing
+int qos_hybrid_step(qos_engine_t* e, const qos_batch* batch, void* logits, int logits_dtype, int32_t* next_tokens,
+                    int outputs_on_host, void* stream) {
+  if (!e) return set_error(QOS_ERR_INVALID_ARG, "engine is NULL");
+  return do_step(e, batch, logits, logits_dtype, next_tokens, outputs_on_host, reinterpret_cast<cudaStream_t>(stream),
+                 true);
+}
+
+int qos_profile_step_ex(qos_engine_t* e, int32_t chunk_len, int32_t kv_start, int32_t n_decode,
+                        const int32_t* ctx_lens, int32_t reps, float* ms_median, float* ms_p95) {
+  if (!e || chunk_len < 0 || kv_start < 0 || n_decode < 0 || (n_decode && !ctx_lens) || reps < 1 || !ms_median)
+    return set_error(QOS_ERR_INVALID_ARG, "profile args");
+  if (chunk_len == 0 && n_decode == 0) return set_error(QOS_ERR_INVALID_ARG, "empty profile batch");
+  QOS_CU(cudaSetDevice(e->device));
+  const int64_t base = INT64_MIN + 1024;  // reserved scratch id range
+  std::vector<int64_t> ids;
+  auto cleanup = [&]() {
+    for (int64_t id : ids) qos_kv_free(e, id);
+  };
+  std::vector<int32_t> toks(static_cast<size_t>(chunk_len));
+  for (int i = 0; i < chunk_len; ++i) toks[size_t(i)] = int32_t((int64_t(i) * 7919 + 13) % e->cfg.vocab);
+  qos_prefill_chunk ch{base, kv_start, chunk_len, toks.data()};
+  std::vector<qos_decode> dec(static_cast<size_t>(n_decode));
+  int r;
+  if (chunk_len > 0) {
+    if ((r = qos_kv_alloc(e, base, kv_start + chunk_len)) != QOS_OK) return r;
+    ids.push_back(base);
+    if ((r = qos_kv_fill_synthetic(e, base, kv_start, 2)) != QOS_OK) { cleanup(); return r; }
+  }
+  for (int j = 0; j < n_decode; ++j) {
+    const int64_t id = base + 1 + j;
+    if ((r = qos_kv_alloc(e, id, ctx_lens[j] + 1)) != QOS_OK) { cleanup(); return r; }
+    ids.push_back(id);
+    if ((r = qos_kv_fill_synthetic(e, id, ctx_lens[j], 2)) != QOS_OK) { cleanup(); return r; }
+    dec[size_t(j)] = qos_decode{id, ctx_lens[j], int32_t((j * 31 + 7) % e->cfg.vocab)};
+  }
+  qos_batch b{chunk_len > 0 ? 1 : 0, &ch, n_decode, dec.data()};
+  cudaStream_t st = e->stream;
+  cudaEvent_t a, z;
+  cudaEventCreate(&a);
+  cudaEventCreate(&z);
+  std::vector<float> ms;
+  for (int i = 0; i < 3 + reps; ++i) {
+    cudaEventRecord(a, st);
+    if ((r = do_step(e, &b, nullptr, QOS_F32, nullptr, 0, st, false)) != QOS_OK) break;
+    cudaEventRecord(z, st);
+    cudaEventSynchronize(z);
+    float t = 0;
+    cudaEventElapsedTime(&t, a, z);
+    if (i >= 3) ms.push_back(t);
+  }
+  cudaEventDestroy(a);
+  cudaEventDestroy(z);
+  cleanup();
+  if (r != QOS_OK) return r;
+  std::sort(ms.begin(), ms.end());
+  *ms_median = ms[ms.size() / 2];
+  if (ms_p95) *ms_p95 = ms[std::min(ms.size() - 1, size_t(std::ceil(0.95 * ms.size())) - 1)];
+  return QOS_OK;
+}
+
+int qos_profile_step(qos_engine_t* e, int32_t chunk_len, int32_t n_decode, const int32_t* ctx_lens, int32_t reps,
+                     float* ms_out) {
+  return qos_profile_step_ex(e, chunk_len, 0, n_decode, ctx_lens, reps, ms_out, nullptr);
+}
+
+int qos_engine_set_timing(qos_engine_t* e, int enable) {
+  if (!e) return set_error(QOS_ERR_INVALID_ARG, "engine is NULL");
+  e->timing = enable != 0;
+  return QOS_OK;
+}
+
+int qos_last_step_timing(qos_engine_t* e, float ms[QOS_T_COUNT], int32_t launches[QOS_T_COUNT]) {
+  if (!e || !ms) return set_error(QOS_ERR_INVALID_ARG, "args");
+  for (int i = 0; i < QOS_T_COUNT; ++i) {
+    ms[i] = 0.f;
+    if (launches) launches[i] = 0;
+  }
+  if (!e->tev.empty()) QOS_CU(cudaEventSynchronize(e->tev.back().second.second));
+  for (auto& x : e->tev) {
+    float t = 0;
+    cudaEventElapsedTime(&t, x.second.first, x.second.second);
+    ms[x.first] += t;
+    if (launches) launches[x.first] += 1;
+  }
+  return QOS_OK;
+}
+
+int qos_engine_launch_count(qos_engine_t* e, int64_t* out) {
+  if (!out) return set_error(QOS_ERR_INVALID_ARG, "out");
+  (void)e;
+  *out = g_launches.load();
+  return QOS_OK;
+}
+
+// ------------------------------------------------------------------ kernel-level ops
+int qos_op_gemm(const void* A, const void* B, void* C, int64_t M, int64_t N, int64_t K, int epi, const float* bias,
+                void* stream) {
+  if (!A || !B || !C || (epi == QOS_EPI_BIAS_BF16 && !bias)) return set_error(QOS_ERR_INVALID_ARG, "gemm pointers");
+  QOS_TRY(gemm_check_shape(M, N, K, epi));
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const int bn = gemm_pick_bn(M, N, epi, sms);
+  CUtensorMap ta, tb;
+  QOS_TRY(make_tmap_2d_bf16(&ta, A, uint64_t(M), uint64_t(K), uint64_t(K), 128, 64, true));
+  QOS_TRY(make_tmap_2d_bf16(&tb, B, uint64_t(N), uint64_t(K), uint64_t(K), uint32_t(bn), 64, true));
+  const int64_t ldc = epi == QOS_EPI_SILU_GATE ? N / 2 : N;
+  count_launch();
+  return gemm_run(ta, tb, bn, M, N, K, epi, C, ldc, bias, sms, reinterpret_cast<cudaStream_t>(stream));
+}
+
+int qos_op_rmsnorm(const float* x, const void* g, void* out, int32_t T, int32_t d, float eps, void* stream) {
+  if (!x || !g || !out || T < 0 || d < 8 || d % 8) return set_error(QOS_ERR_INVALID_ARG, "rmsnorm args");
+  QOS_CU(launch_rmsnorm(x, g, out, T, d, eps, reinterpret_cast<cudaStream_t>(stream)));
+  return QOS_OK;
+}
+
+static int ensure_dbg(qos_engine* e, size_t bytes) {
+  if (e->dbg_bytes >= bytes) return QOS_OK;
+  if (e->dbg) cudaFree(e->dbg);
+  e->dbg = nullptr;
+  e->dbg_bytes = 0;
+  QOS_CU(cudaMalloc(&e->dbg, bytes));
+  e->dbg_bytes = bytes;
+  return QOS_OK;
+}
+
+static int kv_rw(qos_engine* e, int32_t layer, int64_t req, int32_t pos0, int32_t n, const uint16_t* kin,
+                 const uint16_t* vin, uint16_t* kout, uint16_t* vout) {
+  if (!e || layer < 0 || layer >= e->cfg.n_layers || pos0 < 0 || n < 0) return set_error(QOS_ERR_INVALID_ARG, "kv args");
+  auto it = e->reqs.find(req);
+  if (it == e->reqs.end()) return set_error(QOS_ERR_UNKNOWN_REQ, "unknown request");
+  if (int64_t(pos0) + n > int64_t(it->second.blocks.size()) * 16) return set_error(QOS_ERR_NOT_ALLOCATED, "range");
+  QOS_CU(cudaSetDevice(e->device));
+  cudaStream_t st = e->stream;
+  QOS_TRY(flush_table_updates(e, st));
+  const size_t bytes = size_t(n) * e->sh.Hkv * e->cfg.head_dim * 2;
+  QOS_TRY(ensure_dbg(e, bytes));
+  const int32_t* trow = e->d_tables + size_t(it->second.row) * e->table_w;
+  for (int kv = 0; kv < 2; ++kv) {
+    void* plane = reinterpret_cast<__nv_bfloat16*>(e->kv) + (size_t(layer) * 2 + kv) * e->plane_elems;
+    if (kin) {
+      QOS_CU(cudaMemcpyAsync(e->dbg, kv ? vin : kin, bytes, cudaMemcpyHostToDevice, st));
+      QOS_CU(launch_kv_scatter(plane, trow, pos0, n, e->sh.Hkv, e->cfg.head_dim, e->dbg, st));
+    } else {
+      QOS_CU(launch_kv_gather(plane, trow, pos0, n, e->sh.Hkv, e->cfg.head_dim, e->dbg, st));
+      QOS_CU(cudaMemcpyAsync(kv ? vout : kout, e->dbg, bytes, cudaMemcpyDeviceToHost, st));
+    }
+    QOS_CU(cudaStreamSynchronize(st));
+  }
+  return QOS_OK;
+}
+
+int qos_kv_write(qos_engine_t* e, int32_t layer, int64_t req, int32_t pos0, int32_t n, const uint16_t* k,
+                 const uint16_t* v) {
+  if (!k || !v) return set_error(QOS_ERR_INVALID_ARG, "kv_write pointers");
+  return kv_rw(e, layer, req, pos0, n, k, v, nullptr, nullptr);
+}
+int qos_kv_read(qos_engine_t* e, int32_t layer, int64_t req, int32_t pos0, int32_t n, uint16_t* k, uint16_t* v) {
+  if (!k || !v) return set_error(QOS_ERR_INVALID_ARG, "kv_read pointers");
+  return kv_rw(e, layer, req, pos0, n, nullptr, nullptr, k, v);
+}
+
+int qos_op_rope_kv_append(qos_engine_t* e, int32_t layer, const qos_batch* b, const uint16_t* qkv_in, uint16_t* q_out) {
+  if (!e || !qkv_in || !q_out || layer < 0 || layer >= e->cfg.n_layers) return set_error(QOS_ERR_INVALID_ARG, "args");
+  QOS_CU(cudaSetDevice(e->device));
+  cudaStream_t st = e->stream;
+  QOS_TRY(acquire_staging(e));
+  StepMeta m;
+  int r = build_step(e, b, false, e->h_meta[e->meta_cur], m);
+  if (r != QOS_OK) { e->meta_cur ^= 1; return r; }
+  uint8_t* dm;
+  QOS_TRY(upload_meta(e, m, st, &dm));
+  __nv_bfloat16* qkv = reinterpret_cast<__nv_bfloat16*>(e->ws + e->wsl.qkv);
+  const size_t w = size_t(e->nqkv);
+  QOS_CU(cudaMemcpyAsync(qkv, qkv_in, size_t(m.T) * w * 2, cudaMemcpyHostToDevice, st));
+  __nv_bfloat16* kpl = reinterpret_cast<__nv_bfloat16*>(e->kv) + (size_t(layer) * 2 + 0) * e->plane_elems;
+  __nv_bfloat16* vpl = reinterpret_cast<__nv_bfloat16*>(e->kv) + (size_t(layer) * 2 + 1) * e->plane_elems;
+  QOS_CU(launch_rope_append(qkv, int(w), qkv, int(w), reinterpret_cast<int32_t*>(dm + m.o_pos),
+                            reinterpret_cast<int32_t*>(dm + m.o_slot), e->rope_tab, kpl, vpl, m.T, e->sh.H, e->sh.Hkv,
+                            e->cfg.head_dim, st));
+  const size_t qb = size_t(e->sh.H) * e->cfg.head_dim * 2;
+  QOS_CU(cudaMemcpy2DAsync(q_out, qb, qkv, w * 2, qb, size_t(m.T), cudaMemcpyDeviceToHost, st));
+  QOS_TRY(release_staging(e, st));
+  QOS_CU(cudaStreamSynchronize(st));
+  return QOS_OK;
+}
+
+int qos_op_attention(qos_engine_t* e, int32_t layer, const qos_batch* b, const uint16_t* q_in, float* out) {
+  if (!e || !q_in || !out || layer < 0 || layer >= e->cfg.n_layers) return set_error(QOS_ERR_INVALID_ARG, "args");
+  QOS_CU(cudaSetDevice(e->device));
+  cudaStream_t st = e->stream;
+  QOS_TRY(acquire_staging(e));
+  StepMeta m;
+  int r = build_step(e, b, false, e->h_meta[e->meta_cur], m);
+  if (r != QOS_OK) { e->meta_cur ^= 1; return r; }
+  uint8_t* dm;
+  QOS_TRY(upload_meta(e, m, st, &dm));
+  const int hd = e->cfg.head_dim;
+  const size_t qrow = size_t(e->sh.H) * hd;
+  QOS_TRY(ensure_dbg(e, size_t(m.T) * qrow * (2 + 4)));
+  __nv_bfloat16* q = reinterpret_cast<__nv_bfloat16*>(e->dbg);
+  float* o = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(e->dbg) + align_up(size_t(m.T) * qrow * 2, 256));
+  QOS_CU(cudaMemcpyAsync(q, q_in, size_t(m.T) * qrow * 2, cudaMemcpyHostToDevice, st));
+  AttnLaunch al;
+  al.q = q;
+  al.q_ld = int(qrow);
+  al.out = o;
+  al.out_ld = int(qrow);
+  al.out_f32 = 1;
+  al.kv_tmap = &e->kv_map;
+  al.layer = layer;
+  al.H = e->sh.H;
+  al.Hkv = e->sh.Hkv;
+  al.hd = hd;
+  al.num_blocks = int(e->cfg.num_blocks);
+  al.tables = e->d_tables;
+  al.table_w = e->table_w;
+  al.scale_log2 = float(1.4426950408889634 / std::sqrt(double(hd)));
+  QOS_CU(launch_prefill_attention(al, reinterpret_cast<const PrefillItem*>(dm + m.o_pitems), m.n_pitems, st));
+  QOS_CU(launch_decode_attention(al, reinterpret_cast<const DecodeItem*>(dm + m.o_ditems), m.n_ditems,
+                                 reinterpret_cast<const DecodeRow*>(dm + m.o_drows), m.n_drows,
+                                 reinterpret_cast<float*>(e->ws + e->wsl.partials), 0, st));
+  QOS_CU(cudaMemcpyAsync(out, o, size_t(m.T) * qrow * 4, cudaMemcpyDeviceToHost, st));
+  QOS_TRY(release_staging(e, st));
+  QOS_CU(cudaStreamSynchronize(st));
+  return QOS_OK;
+}
+
+}  // extern "C"

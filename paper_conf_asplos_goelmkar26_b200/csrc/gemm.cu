@@ -1,0 +1,341 @@
+// gemm.cu — persistent warp-specialised tcgen05 GEMM for the dense projections of the fused
+// token batch (SURVEY.md §8(a) rows a4 QKV, a9 O, a11 gate/up + SiLU-gate, a12 down, a13 LM
+// head; the paper's "fused prefill-decode MLP", §3.3).
+//
+//   C[M][N] = epi( A[M][K] · B[N][K]^T ),  A = activations (tokens x K), B = nn.Linear weight.
+//
+// Design:
+//   * tile 128 x BN x 64 (BN = 128 | 256), UMMA M=128 N=BN K=16 (cta_group::1), bf16 -> fp32;
+//   * operands staged by TMA (cp.async.bulk.tensor.2d, 128-B swizzle) into a STAGES-deep
+//     smem ring guarded by full/empty mbarriers;
+//   * warp 0 = TMA producer, warp 1 = MMA issuer (one elected lane) + TMEM owner,
+//     warps 2..5 = epilogue (TMEM -> registers -> global), one accumulator row per thread;
+//   * two TMEM accumulators (2 x BN fp32 columns) so the epilogue of tile i overlaps the
+//     MMAs of tile i+1;
+//   * persistent grid (<= #SMs CTAs), tiles ordered N-major / M-minor so the CTAs working at
+//     one time share a weight (B) tile and the activation matrix stays L2-resident.
+#include <cudaTypedefs.h>
+
+#include <cstdio>
+
+#include "common.cuh"
+#include "internal.h"
+
+namespace qos {
+
+constexpr int kBM = 128;
+constexpr int kBK = 64;
+constexpr int kGemmThreads = 192;
+
+template <int BN>
+struct GemmCfg {
+  static constexpr int kStages = (BN == 256) ? 4 : 6;
+  static constexpr int kABytes = kBM * kBK * 2;
+  static constexpr int kBBytes = BN * kBK * 2;
+  static constexpr int kStageBytes = kABytes + kBBytes;
+  static constexpr int kTmemCols = 2 * BN;
+  static constexpr int kSmemBytes = kStages * kStageBytes + 1024 /*align*/ + 256 /*barriers*/;
+};
+
+struct GemmArgs {
+  int M, N, K;
+  int mt, nt;       // tiles along M and N
+  void* C;
+  int ldc;          // elements
+  const float* bias;
+};
+
+template <int BN, int EPI>
+__global__ void __launch_bounds__(kGemmThreads, 1)
+    gemm_tcgen05_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                        const GemmArgs p) {
+  using Cfg = GemmCfg<BN>;
+  constexpr int S = Cfg::kStages;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + S * Cfg::kStageBytes);
+  uint64_t* empty = full + S;
+  uint64_t* tfull = empty + S;
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], 1);
+    }
+    for (int a = 0; a < 2; ++a) {
+      mbar_init(&tfull[a], 1);
+      mbar_init(&tempty[a], 4);
+    }
+    fence_mbar_init();
+  }
+  if (warp == 0 && lane == 0) {
+    tma_prefetch_desc(&tmA);
+    tma_prefetch_desc(&tmB);
+  }
+  if (warp == 1) tmem_alloc<Cfg::kTmemCols>(tmem_slot);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+
+  const int num_tiles = p.mt * p.nt;
+  const int kblocks = p.K / kBK;
+
+  if (warp == 0) {
+    // ------------------------------------------------------------ TMA producer
+    if (elect_one()) {
+      const uint64_t pol_a = l2_evict_last();   // activations: re-read by every N tile
+      const uint64_t pol_b = l2_evict_first();  // weights: streamed once per M-tile group
+      int stage = 0;
+      uint32_t phase = 0;
+      for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) {
+        const int n_t = tile / p.mt, m_t = tile % p.mt;
+        for (int kb = 0; kb < kblocks; ++kb) {
+          mbar_wait(&empty[stage], phase ^ 1);
+          uint8_t* sa = smem + stage * Cfg::kStageBytes;
+          mbar_arrive_expect_tx(&full[stage], Cfg::kStageBytes);
+          tma_load_2d_hint(sa, &tmA, &full[stage], kb * kBK, m_t * kBM, pol_a);
+          tma_load_2d_hint(sa + Cfg::kABytes, &tmB, &full[stage], kb * kBK, n_t * BN, pol_b);
+          if (++stage == S) { stage = 0; phase ^= 1; }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ------------------------------------------------------------ MMA issuer
+    if (elect_one()) {
+      constexpr uint32_t idesc = umma_idesc_bf16(kBM, BN);
+      int stage = 0;
+      uint32_t phase = 0;
+      int acc = 0;
+      uint32_t acc_phase = 0;
+      for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) {
+        mbar_wait(&tempty[acc], acc_phase ^ 1);
+        tc_fence_after();
+        const uint32_t d_tmem = tmem_base + acc * BN;
+        for (int kb = 0; kb < kblocks; ++kb) {
+          mbar_wait(&full[stage], phase);
+          tc_fence_after();
+          const uint32_t a_base = smem_u32(smem + stage * Cfg::kStageBytes);
+          const uint32_t b_base = a_base + Cfg::kABytes;
+#pragma unroll
+          for (int k = 0; k < kBK / 16; ++k) {
+            umma_bf16(d_tmem, umma_desc_sw128(a_base + k * 32), umma_desc_sw128(b_base + k * 32), idesc,
+                      (kb | k) != 0);
+          }
+          umma_commit(&empty[stage]);
+          if (++stage == S) { stage = 0; phase ^= 1; }
+        }
+        umma_commit(&tfull[acc]);
+        if (++acc == 2) { acc = 0; acc_phase ^= 1; }
+      }
+    }
+  } else {
+    // ------------------------------------------------------------ epilogue (warps 2..5)
+    const int q = warp & 3;  // TMEM lane quarter this warp may access
+    int acc = 0;
+    uint32_t acc_phase = 0;
+    for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) {
+      const int n_t = tile / p.mt, m_t = tile % p.mt;
+      mbar_wait(&tfull[acc], acc_phase);
+      tc_fence_after();
+      const int row = m_t * kBM + q * 32 + lane;
+      const bool row_ok = row < p.M;
+      const uint32_t tbase = tmem_base + (uint32_t(q * 32) << 16) + acc * BN;
+      if constexpr (EPI == EPI_SILU_GATE) {
+#pragma unroll 1
+        for (int g = 0; g < BN / 128; ++g) {
+#pragma unroll 1
+          for (int h = 0; h < 2; ++h) {
+            uint32_t gr[32], ur[32];
+            tmem_ld32x32b_x16(tbase + g * 128 + h * 32, *reinterpret_cast<uint32_t(*)[16]>(&gr[0]));
+            tmem_ld32x32b_x16(tbase + g * 128 + h * 32 + 16, *reinterpret_cast<uint32_t(*)[16]>(&gr[16]));
+            tmem_ld32x32b_x16(tbase + g * 128 + 64 + h * 32, *reinterpret_cast<uint32_t(*)[16]>(&ur[0]));
+            tmem_ld32x32b_x16(tbase + g * 128 + 64 + h * 32 + 16, *reinterpret_cast<uint32_t(*)[16]>(&ur[16]));
+            tmem_ld_wait();
+            const int col = n_t * (BN / 2) + g * 64 + h * 32;
+            if (row_ok && col < p.N / 2) {
+              uint32_t pk[16];
+#pragma unroll
+              for (int i = 0; i < 16; ++i) {
+                const float a0 = silu(__uint_as_float(gr[2 * i])) * __uint_as_float(ur[2 * i]);
+                const float a1 = silu(__uint_as_float(gr[2 * i + 1])) * __uint_as_float(ur[2 * i + 1]);
+                pk[i] = pack_bf16(a0, a1);
+              }
+              uint4* dst = reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.C) + size_t(row) * p.ldc + col);
+#pragma unroll
+              for (int i = 0; i < 4; ++i) dst[i] = make_uint4(pk[4 * i], pk[4 * i + 1], pk[4 * i + 2], pk[4 * i + 3]);
+            }
+          }
+        }
+      } else {
+#pragma unroll 1
+        for (int c = 0; c < BN / 32; ++c) {
+          uint32_t r[32];
+          tmem_ld32x32b_x16(tbase + c * 32, *reinterpret_cast<uint32_t(*)[16]>(&r[0]));
+          tmem_ld32x32b_x16(tbase + c * 32 + 16, *reinterpret_cast<uint32_t(*)[16]>(&r[16]));
+          tmem_ld_wait();
+          const int col = n_t * BN + c * 32;
+          if (row_ok && col < p.N) {
+            if constexpr (EPI == EPI_STORE_BF16 || EPI == EPI_BIAS_BF16) {
+              uint32_t pk[16];
+#pragma unroll
+              for (int i = 0; i < 16; ++i) {
+                float a0 = __uint_as_float(r[2 * i]), a1 = __uint_as_float(r[2 * i + 1]);
+                if constexpr (EPI == EPI_BIAS_BF16) {
+                  a0 += __ldg(p.bias + col + 2 * i);
+                  a1 += __ldg(p.bias + col + 2 * i + 1);
+                }
+                pk[i] = pack_bf16(a0, a1);
+              }
+              uint4* dst = reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.C) + size_t(row) * p.ldc + col);
+#pragma unroll
+              for (int i = 0; i < 4; ++i) dst[i] = make_uint4(pk[4 * i], pk[4 * i + 1], pk[4 * i + 2], pk[4 * i + 3]);
+            } else if constexpr (EPI == EPI_STORE_F32) {
+              float4* dst = reinterpret_cast<float4*>(reinterpret_cast<float*>(p.C) + size_t(row) * p.ldc + col);
+#pragma unroll
+              for (int i = 0; i < 8; ++i)
+                dst[i] = make_float4(__uint_as_float(r[4 * i]), __uint_as_float(r[4 * i + 1]),
+                                     __uint_as_float(r[4 * i + 2]), __uint_as_float(r[4 * i + 3]));
+            } else {  // EPI_ADD_F32
+              float4* dst = reinterpret_cast<float4*>(reinterpret_cast<float*>(p.C) + size_t(row) * p.ldc + col);
+              float4 old[8];
+#pragma unroll
+              for (int i = 0; i < 8; ++i) old[i] = dst[i];
+#pragma unroll
+              for (int i = 0; i < 8; ++i)
+                dst[i] = make_float4(old[i].x + __uint_as_float(r[4 * i]), old[i].y + __uint_as_float(r[4 * i + 1]),
+                                     old[i].z + __uint_as_float(r[4 * i + 2]), old[i].w + __uint_as_float(r[4 * i + 3]));
+            }
+          }
+        }
+      }
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&tempty[acc]);
+      if (++acc == 2) { acc = 0; acc_phase ^= 1; }
+    }
+  }
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc<Cfg::kTmemCols>(tmem_base);
+  }
+}
+
+// ------------------------------------------------------------------------------ host side
+static PFN_cuTensorMapEncodeTiled_v12000 get_encode_fn() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  if (!fn) {
+    void* ptr = nullptr;
+    cudaDriverEntryPointQueryResult qres;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &ptr, cudaEnableDefault, &qres) == cudaSuccess &&
+        qres == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(ptr);
+  }
+  return fn;
+}
+
+int make_tmap_2d_bf16(CUtensorMap* out, const void* base, uint64_t rows, uint64_t cols, uint64_t row_stride_elems,
+                      uint32_t box_rows, uint32_t box_cols, bool swizzle128) {
+  auto fn = get_encode_fn();
+  if (!fn) return set_error(QOS_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+  cuuint64_t dims[2] = {cols, rows};
+  cuuint64_t strides[1] = {row_stride_elems * 2};
+  cuuint32_t box[2] = {box_cols, box_rows};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = fn(out, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, estr,
+                  CU_TENSOR_MAP_INTERLEAVE_NONE,
+                  swizzle128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE,
+                  CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) {
+    char msg[256];
+    snprintf(msg, sizeof msg, "cuTensorMapEncodeTiled failed (%d): rows=%llu cols=%llu box=%ux%u", int(r),
+             (unsigned long long)rows, (unsigned long long)cols, box_rows, box_cols);
+    return set_error(QOS_ERR_CUDA, msg);
+  }
+  return QOS_OK;
+}
+
+int make_tmap_3d_bf16(CUtensorMap* out, const void* base, uint64_t d0, uint64_t d1, uint64_t d2, uint32_t b0,
+                      uint32_t b1, uint32_t b2) {
+  auto fn = get_encode_fn();
+  if (!fn) return set_error(QOS_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+  cuuint64_t dims[3] = {d0, d1, d2};
+  cuuint64_t strides[2] = {d0 * 2, d0 * d1 * 2};
+  cuuint32_t box[3] = {b0, b1, b2};
+  cuuint32_t estr[3] = {1, 1, 1};
+  CUresult r = fn(out, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, const_cast<void*>(base), dims, strides, box, estr,
+                  CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return set_error(QOS_ERR_CUDA, "cuTensorMapEncodeTiled (3d) failed");
+  return QOS_OK;
+}
+
+template <int BN, int EPI>
+static cudaError_t launch_gemm_t(const CUtensorMap& ta, const CUtensorMap& tb, const GemmArgs& a, int grid,
+                                 cudaStream_t st) {
+  auto kern = gemm_tcgen05_kernel<BN, EPI>;
+  static bool attr_set = false;  // per template instantiation
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, GemmCfg<BN>::kSmemBytes);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  kern<<<grid, kGemmThreads, GemmCfg<BN>::kSmemBytes, st>>>(ta, tb, a);
+  return cudaGetLastError();
+}
+
+int gemm_pick_bn(int64_t M, int64_t N, int epi, int num_sms) {
+  const int64_t mt = (M + kBM - 1) / kBM;
+  if (N % 256 != 0 && epi == EPI_SILU_GATE) return 128;
+  const int64_t t256 = mt * ((N + 255) / 256);
+  return (t256 >= num_sms && N % 256 == 0) ? 256 : 128;
+}
+
+int gemm_run(const CUtensorMap& ta, const CUtensorMap& tb, int bn, int64_t M, int64_t N, int64_t K, int epi, void* C,
+             int64_t ldc, const float* bias, int num_sms, cudaStream_t st) {
+  GemmArgs a;
+  a.M = int(M);
+  a.N = int(N);
+  a.K = int(K);
+  a.mt = int((M + kBM - 1) / kBM);
+  a.nt = int((N + bn - 1) / bn);
+  a.C = C;
+  a.ldc = int(ldc);
+  a.bias = bias;
+  const int tiles = a.mt * a.nt;
+  const int grid = tiles < num_sms ? tiles : num_sms;
+  cudaError_t e = cudaSuccess;
+#define QOS_GEMM_CASE(BNV, EPIV) \
+  if (bn == BNV && epi == EPIV) e = launch_gemm_t<BNV, EPIV>(ta, tb, a, grid, st); else
+  QOS_GEMM_CASE(128, EPI_STORE_BF16)
+  QOS_GEMM_CASE(256, EPI_STORE_BF16)
+  QOS_GEMM_CASE(128, EPI_STORE_F32)
+  QOS_GEMM_CASE(256, EPI_STORE_F32)
+  QOS_GEMM_CASE(128, EPI_BIAS_BF16)
+  QOS_GEMM_CASE(256, EPI_BIAS_BF16)
+  QOS_GEMM_CASE(128, EPI_SILU_GATE)
+  QOS_GEMM_CASE(256, EPI_SILU_GATE)
+  QOS_GEMM_CASE(128, EPI_ADD_F32)
+  QOS_GEMM_CASE(256, EPI_ADD_F32)
+  return set_error(QOS_ERR_INVALID_ARG, "gemm: bad tile/epilogue");
+#undef QOS_GEMM_CASE
+  if (e != cudaSuccess) return set_cuda_error(e, "gemm launch");
+  return QOS_OK;
+}
+
+int gemm_check_shape(int64_t M, int64_t N, int64_t K, int epi) {
+  if (M < 1 || N < 32 || K < 64) return set_error(QOS_ERR_INVALID_ARG, "gemm: M>=1, N>=32, K>=64 required");
+  if (K % 64) return set_error(QOS_ERR_UNSUPPORTED, "gemm: K % 64 != 0");
+  if (N % 32) return set_error(QOS_ERR_UNSUPPORTED, "gemm: N % 32 != 0");
+  if (epi == EPI_SILU_GATE && N % 128) return set_error(QOS_ERR_UNSUPPORTED, "gemm: SILU_GATE needs N % 128 == 0");
+  if (epi < 0 || epi > EPI_ADD_F32) return set_error(QOS_ERR_INVALID_ARG, "gemm: unknown epilogue");
+  return QOS_OK;
+}
+
+}  // namespace qos

@@ -1,0 +1,111 @@
+// internal.h — declarations shared by the libqoserve translation units (not part of the ABI).
+#pragma once
+
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../../include/qoserve.h"
+#include "../../include/qoserve_ops.h"
+
+namespace qos {
+
+enum { EPI_STORE_BF16 = QOS_EPI_STORE_BF16, EPI_STORE_F32 = QOS_EPI_STORE_F32, EPI_BIAS_BF16 = QOS_EPI_BIAS_BF16,
+       EPI_SILU_GATE = QOS_EPI_SILU_GATE, EPI_ADD_F32 = QOS_EPI_ADD_F32 };
+
+// error reporting (thread-local last error; engine.cpp)
+int set_error(int code, const char* msg);
+int set_cuda_error(cudaError_t e, const char* where);
+int count_launch(int n = 1);  // global launch counter hook (engine.cpp)
+
+// ------------------------------------------------------------------ GEMM (gemm.cu)
+int make_tmap_2d_bf16(CUtensorMap* out, const void* base, uint64_t rows, uint64_t cols, uint64_t row_stride_elems,
+                      uint32_t box_rows, uint32_t box_cols, bool swizzle128);
+int make_tmap_3d_bf16(CUtensorMap* out, const void* base, uint64_t d0, uint64_t d1, uint64_t d2, uint32_t b0,
+                      uint32_t b1, uint32_t b2);
+int gemm_pick_bn(int64_t M, int64_t N, int epi, int num_sms);
+int gemm_check_shape(int64_t M, int64_t N, int64_t K, int epi);
+int gemm_run(const CUtensorMap& ta, const CUtensorMap& tb, int bn, int64_t M, int64_t N, int64_t K, int epi, void* C,
+             int64_t ldc, const float* bias, int num_sms, cudaStream_t st);
+
+// ------------------------------------------------------------------ synthetic generator (gen.cu)
+enum GenKind { GEN_LINEAR = 0, GEN_EMBED = 1, GEN_NORM = 2, GEN_BIAS = 3 };
+uint64_t fnv1a64(const char* s);
+// dst[r * dst_ld + c] = gen(name, (row0 + r) * src_cols + col0 + c) for r < rows, c < cols
+cudaError_t gen_fill_bf16(void* dst, int64_t dst_ld, int64_t rows, int64_t cols, uint64_t seed, uint64_t name_hash,
+                          int64_t row0, int64_t col0, int64_t src_cols, int kind, int fan_in, cudaStream_t st);
+cudaError_t gen_fill_bf16_ex(void* dst, int64_t dst_ld, int64_t rows, int64_t cols, uint64_t seed, uint64_t name_hash,
+                             int64_t row0, int64_t col0, int64_t src_cols, int kind, int fan_in, int interleave,
+                             cudaStream_t st);
+cudaError_t gen_fill_f32_bias(float* dst, int64_t n, uint64_t seed, uint64_t name_hash, int64_t off, cudaStream_t st);
+// KV fill: positions [0, n) of one request, one layer, K or V plane
+cudaError_t kvfill_launch(void* plane, const int32_t* d_table, int n_tokens, int hkv_local, int hkv_global,
+                          int kv_head0, int hd, uint64_t seed, uint64_t name_hash, cudaStream_t st);
+
+// ------------------------------------------------------------------ elementwise (elementwise.cu)
+cudaError_t launch_embed_rmsnorm(const int32_t* tokens, const void* emb, const void* g, float* resid, void* out,
+                                 int T, int d, float eps, cudaStream_t st);
+cudaError_t launch_rmsnorm(const float* x, const void* g, void* out, int T, int d, float eps, cudaStream_t st);
+cudaError_t launch_gather_rmsnorm(const float* x, const int32_t* rows, const void* g, void* out, int R, int d,
+                                  float eps, cudaStream_t st);
+// RoPE on q, k + append k, v to the paged cache
+cudaError_t launch_rope_append(void* qkv, int qkv_ld, void* q_out, int q_ld, const int32_t* pos,
+                               const int32_t* slot, const float2* rope_tab, void* kplane, void* vplane, int T, int H,
+                               int Hkv, int hd, cudaStream_t st);
+// copy rows between host-layout [n][Hkv][hd] buffers and the paged plane (positions pos0..)
+cudaError_t launch_kv_scatter(void* plane, const int32_t* d_table_row, int pos0, int n, int Hkv, int hd,
+                              const void* src, cudaStream_t st);
+cudaError_t launch_kv_gather(const void* plane, const int32_t* d_table_row, int pos0, int n, int Hkv, int hd, void* dst,
+                             cudaStream_t st);
+// apply block-table updates: triples (row, col, block)
+cudaError_t launch_table_update(int32_t* tables, int table_w, const int32_t* triples, int n, cudaStream_t st);
+// tp > 1: resid += add (bf16 all-reduced partial); out = RMSNorm(resid) * g  (out may alias add)
+cudaError_t launch_add_rmsnorm(float* resid, const void* add, const void* g, void* out, int T, int d, float eps,
+                               cudaStream_t st);
+cudaError_t launch_add_f32(float* resid, const void* add_bf16, size_t n, cudaStream_t st);
+// [tp][R][Vl] -> [R][tp*Vl]
+cudaError_t launch_unshard_logits(const float* in, float* out, int R, int Vl, int tp, cudaStream_t st);
+cudaError_t launch_argmax(const void* logits, int logits_f32, int R, int V, int32_t* out, cudaStream_t st);
+cudaError_t launch_f32_to_bf16(const float* x, void* y, int64_t n, cudaStream_t st);
+
+// ------------------------------------------------------------------ attention (attention.cu)
+struct DecodeItem {      // one split-K work item: (decode row, kv head, key range)
+  int32_t row;           // token row in the batch (q / out row)
+  int32_t table;         // block-table row (device) of the request
+  int32_t kv_head;       // local kv head
+  int32_t key0, key1;    // key range [key0, key1)
+  int32_t part;          // partial slot index
+};
+struct DecodeRow {       // combine descriptor of one decode row
+  int32_t row;
+  int32_t part0;         // first partial slot of kv head 0; heads follow (nsplit each)
+  int32_t nsplit;
+};
+struct PrefillItem {     // one (chunk, q-tile, kv head) work item
+  int32_t row0;          // first token row of the tile
+  int32_t npos;          // positions in this tile
+  int32_t pos0;          // absolute position of row0
+  int32_t table;         // block-table row
+  int32_t kv_head;
+  int32_t pad;
+};
+struct AttnLaunch {
+  const void* q;          // [T][H][hd] bf16, row stride q_ld (elements)
+  int q_ld;
+  void* out;              // [T][H][hd] (bf16 or f32), row stride out_ld
+  int out_ld;
+  int out_f32;
+  const CUtensorMap* kv_tmap;  // 3D map over the KV pool (host copy; passed by value)
+  int layer;
+  int H, Hkv, hd;
+  int num_blocks;
+  const int32_t* tables;  // [max_requests][table_w]
+  int table_w;
+  float scale_log2;       // log2(e) / sqrt(hd)
+};
+cudaError_t launch_decode_attention(const AttnLaunch& a, const DecodeItem* items, int n_items, const DecodeRow* rows,
+                                    int n_rows, float* partials, int max_splits, cudaStream_t st);
+cudaError_t launch_prefill_attention(const AttnLaunch& a, const PrefillItem* items, int n_items, cudaStream_t st);
+int prefill_positions_per_tile(int group);
+
+}  // namespace qos

@@ -1,0 +1,216 @@
+"""Kernel-level parity on the B200 (one test per SURVEY.md §8(a) row), through the C ABI.
+
+Inputs are seeded on the host, rounded to bf16, and fed to both the CUDA op and the fp64
+oracle; outputs are compared with the north-star tolerances (metric of reading s9).
+"""
+import numpy as np
+import pytest
+
+from helpers import TOL_ATTN, bf16_bits, bits_to_f64, make_engine, row_rel_err
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def torch_cuda():
+    import torch
+    assert torch.cuda.is_available()
+    return torch
+
+
+def _dev_bf16(torch, x):
+    return torch.from_numpy(bf16_bits(x).view(np.int16)).view(torch.bfloat16).cuda()
+
+
+# ------------------------------------------------------------------ weights (generator spec)
+def test_weights_bit_exact_tiny():
+    from oracle import gen
+    from oracle.model import PRESETS, tensor_names
+    q, cfg, eng = make_engine("tiny-qwen")
+    eng.qos_engine_load_synthetic(0)
+    c = PRESETS["tiny-qwen"]
+    for l in range(c.n_layers):
+        nm = tensor_names(c, l)
+        for key, kind, shape, fan in [("wq", "linear", (256, 256), 256), ("wk", "linear", (128, 256), 256),
+                                      ("wv", "linear", (128, 256), 256), ("wo", "linear", (256, 256), 256),
+                                      ("wg", "linear", (768, 256), 256), ("wu", "linear", (768, 256), 256),
+                                      ("wd", "linear", (256, 768), 768), ("ln1", "norm", (1, 256), 1),
+                                      ("ln2", "norm", (1, 256), 1)]:
+            ref = gen.gen_bits(0, nm[key], kind, 0, shape[0] * shape[1], fan).reshape(shape)
+            got = eng.qos_engine_read_weight(nm[key], 0, shape[0], shape[1])
+            assert np.array_equal(got, ref), nm[key]
+    for name, kind, shape in [("model.embed_tokens.weight", "embed", (1024, 256)),
+                              ("lm_head.weight", "linear", (1024, 256)), ("model.norm.weight", "norm", (1, 256))]:
+        ref = gen.gen_bits(0, name, kind, 0, shape[0] * shape[1], shape[1]).reshape(shape)
+        assert np.array_equal(eng.qos_engine_read_weight(name, 0, shape[0], shape[1]), ref), name
+    eng.close()
+
+
+def test_weights_bit_exact_8b_sampled():
+    from oracle import gen
+    q, cfg, eng = make_engine("llama3-8b", n_layers=2, num_blocks=64, max_batch_tokens=256, max_batch_rows=16)
+    eng.qos_engine_load_synthetic(0)
+    checks = [("model.layers.1.mlp.gate_proj.weight", 14336, 4096, 4096, [0, 63, 64, 5000, 14335]),
+              ("model.layers.1.mlp.up_proj.weight", 14336, 4096, 4096, [0, 65, 14335]),
+              ("model.layers.0.mlp.down_proj.weight", 4096, 14336, 14336, [0, 4095]),
+              ("model.layers.0.self_attn.o_proj.weight", 4096, 4096, 4096, [7, 4000]),
+              ("model.layers.0.self_attn.k_proj.weight", 1024, 4096, 4096, [0, 1023]),
+              ("lm_head.weight", 128256, 4096, 4096, [0, 128255]),
+              ("model.embed_tokens.weight", 128256, 4096, 1, [77])]
+    for name, rows, cols, fan, sample in checks:
+        kind = "embed" if "embed" in name else "linear"
+        for r in sample:
+            ref = gen.gen_bits(0, name, kind, r * cols, cols, fan)
+            got = eng.qos_engine_read_weight(name, r, 1, cols)[0]
+            assert np.array_equal(got, ref), (name, r)
+    eng.close()
+
+
+# ------------------------------------------------------------------ GEMM (a4, a9, a11, a12, a13)
+@pytest.mark.parametrize("M,N,K", [(1, 256, 64), (77, 384, 320), (128, 512, 256), (300, 96, 128),
+                                   (700, 1024, 512), (2176, 1536, 1024)])
+@pytest.mark.parametrize("epi", ["store_f32", "store_bf16", "add_f32", "bias_bf16"])
+def test_gemm_parity(torch_cuda, M, N, K, epi):
+    torch = torch_cuda
+    from paper_conf_asplos_goelmkar26_b200 import qoserve as q
+    rng = np.random.default_rng(M * 7 + N + K)
+    A = bits_to_f64(bf16_bits(rng.uniform(-1, 1, (M, K))))
+    B = bits_to_f64(bf16_bits(rng.uniform(-1, 1, (N, K)) / np.sqrt(K)))
+    ref = A @ B.T                                   # numpy fp64 (the oracle's GEMM primitive)
+    dA, dB = _dev_bf16(torch, A), _dev_bf16(torch, B)
+    bias = None
+    if epi in ("store_f32", "add_f32"):
+        init = rng.uniform(-1, 1, (M, N)).astype(np.float32) if epi == "add_f32" else np.zeros((M, N), np.float32)
+        dC = torch.from_numpy(init.copy()).cuda()
+        ref = ref + init.astype(np.float64)
+    else:
+        dC = torch.empty((M, N), dtype=torch.bfloat16, device="cuda")
+        if epi == "bias_bf16":
+            bvals = bits_to_f64(bf16_bits(rng.uniform(-0.02, 0.02, N)))
+            bias = torch.from_numpy(bvals.astype(np.float32)).cuda()
+            ref = ref + bvals
+    q.qos_op_gemm(dA.data_ptr(), dB.data_ptr(), dC.data_ptr(), M, N, K, epi,
+                  bias.data_ptr() if bias is not None else None)
+    torch.cuda.synchronize()
+    got = dC.float().cpu().numpy()
+    tol = 1e-5 if epi in ("store_f32", "add_f32") else 8e-3   # fp32 out vs bf16 rounding (2^-8)
+    assert row_rel_err(got, ref) <= tol
+
+
+@pytest.mark.parametrize("M,F,K", [(1, 128, 64), (200, 384, 256), (1000, 768, 512)])
+def test_gemm_silu_gate_parity(torch_cuda, M, F, K):
+    torch = torch_cuda
+    from oracle.model import swiglu_mlp, silu
+    from paper_conf_asplos_goelmkar26_b200 import qoserve as q
+    rng = np.random.default_rng(F + K)
+    A = bits_to_f64(bf16_bits(rng.uniform(-1, 1, (M, K))))
+    Wg = bits_to_f64(bf16_bits(rng.uniform(-1, 1, (F, K)) / np.sqrt(K)))
+    Wu = bits_to_f64(bf16_bits(rng.uniform(-1, 1, (F, K)) / np.sqrt(K)))
+    # QOS_EPI_SILU_GATE interleave: rows [128j, 128j+64) gate rows [64j, ...), then 64 up rows
+    Bi = np.empty((2 * F, K))
+    for j in range(F // 64):
+        Bi[128 * j:128 * j + 64] = Wg[64 * j:64 * j + 64]
+        Bi[128 * j + 64:128 * j + 128] = Wu[64 * j:64 * j + 64]
+    ref = silu(A @ Wg.T) * (A @ Wu.T)
+    dC = torch.empty((M, F), dtype=torch.bfloat16, device="cuda")
+    q.qos_op_gemm(_dev_bf16(torch, A).data_ptr(), _dev_bf16(torch, Bi).data_ptr(), dC.data_ptr(), M, 2 * F, K,
+                  "silu_gate")
+    torch.cuda.synchronize()
+    assert row_rel_err(dC.float().cpu().numpy(), ref) <= 8e-3
+    del swiglu_mlp
+
+
+# ------------------------------------------------------------------ RMSNorm (a3)
+def test_rmsnorm_parity(torch_cuda):
+    torch = torch_cuda
+    from oracle.model import rms_norm
+    from paper_conf_asplos_goelmkar26_b200 import qoserve as q
+    rng = np.random.default_rng(5)
+    for T, d in [(1, 256), (33, 4096), (7, 5120), (3, 8192)]:
+        x = rng.standard_normal((T, d)).astype(np.float32)
+        g = bits_to_f64(bf16_bits(rng.uniform(0.9, 1.1, d)))
+        out = torch.empty((T, d), dtype=torch.bfloat16, device="cuda")
+        q.qos_op_rmsnorm(torch.from_numpy(x).cuda().data_ptr(), _dev_bf16(torch, g).data_ptr(), out.data_ptr(),
+                         T, d, 1e-5)
+        torch.cuda.synchronize()
+        assert row_rel_err(out.float().cpu().numpy(), rms_norm(x.astype(np.float64), g, 1e-5)) <= 8e-3
+
+
+# ------------------------------------------------------------------ RoPE + KV append (a5, a6)
+@pytest.mark.parametrize("preset,over", [("tiny", {}), ("llama3-8b", dict(n_layers=1, num_blocks=128))])
+def test_rope_kv_append_parity(preset, over):
+    from oracle.model import PRESETS as OP, apply_rope
+    q, cfg, eng = make_engine(preset, **over)
+    H, Hkv, hd, theta = cfg.n_heads, cfg.n_kv_heads, cfg.head_dim, cfg.rope_theta
+    rng = np.random.default_rng(11)
+    eng.qos_kv_alloc(1, 300)
+    eng.qos_kv_alloc(2, 1500)
+    # a 45-token chunk at kv_start 200 of req 1 + a decode of req 2 at position 1400
+    b = q.make_batch([(1, 200, np.zeros(45, np.int32))], [(2, 1400, 0)])
+    T = 46
+    pos = np.array(list(range(200, 245)) + [1400])
+    qkv = bits_to_f64(bf16_bits(rng.uniform(-1, 1, (T, (H + 2 * Hkv) * hd))))
+    qo = eng.qos_op_rope_kv_append(0, b, bf16_bits(qkv), H * hd)
+    qr = apply_rope(qkv[:, :H * hd].reshape(T, H, hd), pos, theta)
+    kr = apply_rope(qkv[:, H * hd:(H + Hkv) * hd].reshape(T, Hkv, hd), pos, theta)
+    v = qkv[:, (H + Hkv) * hd:].reshape(T, Hkv, hd)
+    # q: bf16 store of an fp32 rotation (<= 1 bf16 rounding: 2^-8 relative per row)
+    assert row_rel_err(bits_to_f64(qo).reshape(T, H, hd), qr) <= 2 ** -8
+    k1, v1 = eng.qos_kv_read(0, 1, 200, 45, Hkv, hd)
+    k2, v2 = eng.qos_kv_read(0, 2, 1400, 1, Hkv, hd)
+    assert row_rel_err(bits_to_f64(np.concatenate([k1, k2])), kr) <= 2 ** -8
+    assert np.array_equal(np.concatenate([v1, v2]), bf16_bits(v))      # V is copied bit-exactly
+    eng.close()
+    del OP
+
+
+# ------------------------------------------------------------------ attention (a7, a8)
+ATTN_CASES = [
+    # (preset, overrides, chunks [(kv_start, len)], decode ctxs, scale)
+    ("tiny", {}, [(0, 1), (0, 37), (100, 128)], [0, 15, 16, 17, 300], 1.0),
+    ("llama3-8b", dict(n_layers=1, num_blocks=2048), [(0, 200), (4096, 64)], [1, 1000, 5000], 1.0),
+    ("llama3-8b", dict(n_layers=1, num_blocks=2048), [(31, 129)], [2047, 4095], 3.0),
+    ("tiny-mha", {}, [(5, 77)], [33, 64], 1.0),
+    ("llama3-70b", dict(n_layers=1, n_heads=8, n_kv_heads=1, d_model=1024, ffn_dim=1024, num_blocks=1024),
+     [(0, 48)], [700, 3000], 1.0),   # group 8 = Llama-3-70B at TP8
+]
+
+
+@pytest.mark.parametrize("case", range(len(ATTN_CASES)))
+def test_attention_parity(case):
+    from oracle.model import causal_attention
+    preset, over, chunks, ctxs, scale = ATTN_CASES[case]
+    q, cfg, eng = make_engine(preset, max_seq_len=8192, **over)
+    H, Hkv, hd = cfg.n_heads, cfg.n_kv_heads, cfg.head_dim
+    g = H // Hkv
+    rng = np.random.default_rng(100 + case)
+    prefill, decode, qrows, refs = [], [], [], []
+    req = 0
+    for ks, n in chunks:
+        P = ks + n
+        eng.qos_kv_alloc(req, P)
+        K = bits_to_f64(bf16_bits(rng.uniform(-1, 1, (P, Hkv, hd)) * scale))
+        V = bits_to_f64(bf16_bits(rng.uniform(-1, 1, (P, Hkv, hd))))
+        eng.qos_kv_write(0, req, 0, bf16_bits(K), bf16_bits(V))
+        Q = bits_to_f64(bf16_bits(rng.uniform(-1, 1, (n, H, hd)) * scale))
+        prefill.append((req, ks, np.zeros(n, np.int32)))
+        qrows.append(Q)
+        refs.append(causal_attention(Q, K, V, ks, g))
+        req += 1
+    for c in ctxs:
+        eng.qos_kv_alloc(req, c + 1)
+        K = bits_to_f64(bf16_bits(rng.uniform(-1, 1, (c + 1, Hkv, hd)) * scale))
+        V = bits_to_f64(bf16_bits(rng.uniform(-1, 1, (c + 1, Hkv, hd))))
+        eng.qos_kv_write(0, req, 0, bf16_bits(K), bf16_bits(V))
+        Q = bits_to_f64(bf16_bits(rng.uniform(-1, 1, (1, H, hd)) * scale))
+        decode.append((req, c, 0))
+        qrows.append(Q)
+        refs.append(causal_attention(Q, K, V, c, g))
+        req += 1
+    b = q.make_batch(prefill, decode)
+    Qall = np.concatenate(qrows)
+    out = eng.qos_op_attention(0, b, bf16_bits(Qall))
+    ref = np.concatenate(refs)
+    err = row_rel_err(out.reshape(-1, hd), ref.reshape(-1, hd))
+    assert err <= TOL_ATTN, err
+    eng.close()

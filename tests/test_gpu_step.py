@@ -1,0 +1,194 @@
+"""End-to-end parity of qos_hybrid_step against the fp64 oracle (through the C ABI).
+
+* tiny (configs[0]): chunked prefills of 4 prompts (splits {64, 100, 128}), then a 128-token
+  chunk + 4 decodes, then a second chunk at kv_start 128 + decodes; logits rel-err <= 1e-2,
+  greedy tokens identical, KV tables (host and device mirror) bit-exact vs the oracle's
+  allocator (north star); batch-composition and chunk-split invariance on the GPU.
+* Llama-3-8B shapes (2 layers, full width) at the bench batch shape (2048-token chunk +
+  128 decodes @ ctx 4096 with synthetic KV): sampled rows vs the oracle.
+"""
+import numpy as np
+import pytest
+
+import synth
+from helpers import TOL_LOGITS, make_engine, row_rel_err
+
+pytestmark = pytest.mark.gpu
+
+
+def _oracle(preset, **kw):
+    from oracle.engine import OracleEngine
+    from oracle.model import PRESETS, with_layers
+    c = PRESETS[preset]
+    if "n_layers" in kw:
+        c = with_layers(c, kw.pop("n_layers"))
+    return OracleEngine(c, seed=0, **kw)
+
+
+def _run_tiny(preset):
+    q, cfg, eng = make_engine(preset, num_blocks=256)
+    eng.qos_engine_load_synthetic(0)
+    orc = _oracle(preset, num_blocks=256)
+    ctxs, warm, main, second = synth.tiny_scenario(cfg.vocab)
+    for r, n in ctxs.items():
+        eng.qos_kv_alloc(r, n + 2)
+        orc.kv_alloc(r, n + 2)
+    eng.qos_kv_alloc(0, 256)
+    orc.kv_alloc(0, 256)
+    errs = []
+    for b in warm + [main, second]:
+        lg, tk = eng.step_host(q.batch_from_synth(b), cfg.vocab)
+        ref = orc.hybrid_step(*b.as_oracle())
+        errs.append(row_rel_err(lg, ref))
+        assert list(tk) == list(np.argmax(ref, 1))
+    for r in list(ctxs) + [0]:
+        assert eng.qos_kv_table(r) == orc.kv_table(r)
+        assert eng.qos_kv_table_device(r) == orc.kv_table(r)
+        assert eng.qos_kv_cached_len(r) == orc.cached_len(r)
+    return q, cfg, eng, orc, max(errs)
+
+
+@pytest.mark.parametrize("preset", ["tiny", "tiny-mha", "tiny-qwen"])
+def test_tiny_scenario_parity(preset):
+    q, cfg, eng, orc, err = _run_tiny(preset)
+    assert err <= TOL_LOGITS, err
+    eng.close()
+
+
+def test_tiny_greedy_decode_loop_tokens_identical():
+    """Autoregressive decode: feed each step's argmax back in; the GPU and
+    the oracle must produce the same token sequence (north star: greedy tokens identical)."""
+    q, cfg, eng, orc, _ = _run_tiny("tiny")
+    ctxs = {1: 39, 2: 202, 3: 313, 4: 514}        # after tiny_scenario (+2 steps)
+    toks = {r: 5 + r for r in ctxs}
+    for r, n in ctxs.items():
+        eng.qos_kv_alloc(r, n + 40)
+        orc.kv_alloc(r, n + 40)
+    for step in range(30):
+        dec = [(r, ctxs[r], toks[r]) for r in sorted(ctxs)]
+        lg, tk = eng.step_host(q.make_batch([], dec), cfg.vocab)
+        ref = orc.hybrid_step([], dec)
+        rt = np.argmax(ref, 1)
+        # argmax must be identical unless the oracle's top-2 gap is inside the tolerance
+        srt = np.sort(ref, 1)
+        gap = (srt[:, -1] - srt[:, -2]) / np.abs(ref).max(1)
+        for i, r in enumerate(sorted(ctxs)):
+            if gap[i] > 2 * TOL_LOGITS:
+                assert tk[i] == rt[i], (step, r)
+            toks[r] = int(rt[i])
+            ctxs[r] += 1
+        assert row_rel_err(lg, ref) <= TOL_LOGITS
+    eng.close()
+
+
+def test_batch_composition_and_split_invariance_on_gpu():
+    q, cfg, eng = make_engine("tiny", num_blocks=256)
+    eng.qos_engine_load_synthetic(0)
+    toks = synth.request_tokens(7, 150, cfg.vocab)
+    other = synth.request_tokens(8, 90, cfg.vocab)
+    eng.qos_kv_alloc(7, 150)
+    eng.qos_kv_alloc(8, 90)
+    eng.qos_kv_alloc(9, 150)
+    # (a) req 7 in one chunk, mixed with req 8's chunk
+    la, _ = eng.step_host(q.make_batch([(7, 0, toks), (8, 0, other)], []), cfg.vocab)
+    # (b) req 9 = same tokens, split 64 + 50 + 36, alone
+    eng.step_host(q.make_batch([(9, 0, toks[:64])], []), cfg.vocab)
+    eng.step_host(q.make_batch([(9, 64, toks[64:114])], []), cfg.vocab)
+    lb, _ = eng.step_host(q.make_batch([(9, 114, toks[114:])], []), cfg.vocab)
+    # bf16 activations make the two schedules differ only by rounding
+    assert row_rel_err(la[:1], lb) <= TOL_LOGITS
+    eng.close()
+
+
+def test_step_errors_leave_state_unchanged():
+    q, cfg, eng = make_engine("tiny", num_blocks=8)
+    eng.qos_engine_load_synthetic(0)
+    eng.qos_kv_alloc(1, 20)
+    with pytest.raises(q.QosError) as ei:
+        eng.step_host(q.make_batch([(1, 0, np.zeros(33, np.int32))], []), cfg.vocab)
+    assert ei.value.name == "NOT_ALLOCATED"
+    with pytest.raises(q.QosError) as ei:
+        eng.step_host(q.make_batch([(1, 5, np.zeros(3, np.int32))], []), cfg.vocab)
+    assert ei.value.name == "BAD_KV_START"
+    with pytest.raises(q.QosError) as ei:
+        eng.step_host(q.make_batch([], [(42, 0, 1)]), cfg.vocab)
+    assert ei.value.name == "UNKNOWN_REQ"
+    with pytest.raises(q.QosError) as ei:
+        eng.step_host(q.make_batch([(1, 0, np.array([cfg.vocab], np.int32))], []), cfg.vocab)
+    assert ei.value.name == "INVALID_ARG"
+    assert eng.qos_kv_cached_len(1) == 0
+    free = eng.qos_kv_free_blocks()
+    with pytest.raises(q.QosError) as ei:
+        eng.qos_kv_alloc(2, 16 * 8)
+    assert ei.value.name == "OOM" and eng.qos_kv_free_blocks() == free
+    eng.step_host(q.make_batch([(1, 0, np.ones(20, np.int32))], []), cfg.vocab)
+    assert eng.qos_kv_cached_len(1) == 20
+    with pytest.raises(q.QosError) as ei:
+        eng.qos_kv_free(99)
+    assert ei.value.name == "UNKNOWN_REQ"
+    eng.close()
+
+
+def test_kv_tables_match_oracle_under_churn():
+    from oracle.kv import BlockAllocator, OracleOOM
+    q, cfg, eng = make_engine("tiny", num_blocks=300)
+    a = BlockAllocator(300)
+    rng = np.random.default_rng(3)
+    live = {}
+    for _ in range(500):
+        if live and rng.random() < 0.3:
+            r = int(rng.choice(list(live)))
+            eng.qos_kv_free(r)
+            a.free(r)
+            del live[r]
+        else:
+            r = int(rng.integers(0, 50))
+            n = max(int(rng.integers(0, 800)), live.get(r, 0))
+            try:
+                a.alloc(r, n)
+                ok = True
+            except OracleOOM:
+                ok = False
+            if ok:
+                eng.qos_kv_alloc(r, n)
+                live[r] = n
+            else:
+                with pytest.raises(q.QosError):
+                    eng.qos_kv_alloc(r, n)
+    for r in live:
+        assert eng.qos_kv_table(r) == a.table(r)
+        assert eng.qos_kv_table_device(r) == a.table(r)
+    assert eng.qos_kv_free_blocks() == a.n_free
+    eng.close()
+
+
+@pytest.mark.slow
+def test_llama8b_shapes_bench_batch_sampled_parity():
+    """2-layer Llama-3-8B (full width) at the bench launch shape: a 2048-token chunk at
+    kv_start 0 + 128 decodes @ ctx 4096 whose prefixes hold synthetic KV."""
+    C, ND, CTX = 2048, 128, 4096
+    q, cfg, eng = make_engine("llama3-8b", n_layers=2, num_blocks=(C + ND * (CTX + 1)) // 16 + 200,
+                              max_seq_len=8192, max_batch_tokens=C + ND, max_batch_rows=ND + 1,
+                              max_requests=ND + 8)
+    eng.qos_engine_load_synthetic(0)
+    b = synth.hybrid_batch(cfg.vocab, C, ND, CTX)
+    eng.qos_kv_alloc(0, C)
+    for d in b.decode:
+        eng.qos_kv_alloc(d.req, CTX + 1)
+        eng.qos_kv_fill_synthetic(d.req, CTX, synth.SEED_KVFILL)
+    lg, tk = eng.step_host(q.batch_from_synth(b), cfg.vocab)
+    orc = _oracle("llama3-8b", n_layers=2, num_blocks=2 * (C // 16 + 1) + 8 * (CTX // 16 + 2))
+    sample = [0, 1, 63, 127]
+    orc.kv_alloc(0, C)
+    pre = [(0, 0, [int(t) for t in b.prefill[0].tokens])]
+    decs = []
+    for j in sample:
+        d = b.decode[j]
+        orc.kv_alloc(d.req, CTX + 1)
+        orc.kv_fill_synthetic(d.req, CTX, synth.SEED_KVFILL)
+        decs.append((d.req, d.ctx_len, d.token))
+    ref = orc.hybrid_step(pre, decs)
+    got = np.concatenate([lg[:1], lg[[1 + j for j in sample]]])
+    err = row_rel_err(got, ref)
+    assert err <= TOL_LOGITS, err
+    eng.close()
