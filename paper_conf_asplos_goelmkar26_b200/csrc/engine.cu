@@ -689,6 +689,7 @@ int do_step(qos_engine* e, const qos_batch* b, void* logits, int logits_dtype, i
   if (logits && logits_dtype != QOS_F32 && logits_dtype != QOS_BF16)
     return set_error(QOS_ERR_INVALID_ARG, "logits_dtype");
   if (cudaSetDevice(e->device) != cudaSuccess) return set_error(QOS_ERR_CUDA, "cudaSetDevice");
+  if (e->pending_upd.size() / 3 > 65536) QOS_TRY(flush_table_updates(e, st));  // step carries <= 64Ki
   QOS_TRY(acquire_staging(e));
   StepMeta m;
   int r = build_step(e, b, check_and_advance, e->h_meta[e->meta_cur], m);
@@ -982,6 +983,20 @@ int qos_kv_free(qos_engine_t* e, int64_t req) {
   if (!e) return set_error(QOS_ERR_INVALID_ARG, "engine is NULL");
   auto it = e->reqs.find(req);
   if (it == e->reqs.end()) return set_error(QOS_ERR_UNKNOWN_REQ, "unknown request");
+  // table updates of this row not yet on the device are obsolete: drop them so a later owner
+  // of the row can never be overwritten by them (the update kernel applies triples unordered)
+  {
+    const int row = it->second.row;
+    size_t w = 0;
+    for (size_t i = 0; i < e->pending_upd.size(); i += 3)
+      if (e->pending_upd[i] != row) {
+        e->pending_upd[w] = e->pending_upd[i];
+        e->pending_upd[w + 1] = e->pending_upd[i + 1];
+        e->pending_upd[w + 2] = e->pending_upd[i + 2];
+        w += 3;
+      }
+    e->pending_upd.resize(w);
+  }
   for (int32_t b : it->second.blocks) {
     e->free_heap.push_back(b);
     std::push_heap(e->free_heap.begin(), e->free_heap.end(), std::greater<int32_t>());

@@ -113,8 +113,8 @@ def test_gemm_silu_gate_parity(torch_cuda, M, F, K):
         Bi[128 * j + 64:128 * j + 128] = Wu[64 * j:64 * j + 64]
     ref = silu(A @ Wg.T) * (A @ Wu.T)
     dC = torch.empty((M, F), dtype=torch.bfloat16, device="cuda")
-    q.qos_op_gemm(_dev_bf16(torch, A).data_ptr(), _dev_bf16(torch, Bi).data_ptr(), dC.data_ptr(), M, 2 * F, K,
-                  "silu_gate")
+    dA, dB = _dev_bf16(torch, A), _dev_bf16(torch, Bi)     # keep the device inputs alive
+    q.qos_op_gemm(dA.data_ptr(), dB.data_ptr(), dC.data_ptr(), M, 2 * F, K, "silu_gate")
     torch.cuda.synchronize()
     assert row_rel_err(dC.float().cpu().numpy(), ref) <= 8e-3
     del swiglu_mlp
@@ -130,8 +130,8 @@ def test_rmsnorm_parity(torch_cuda):
         x = rng.standard_normal((T, d)).astype(np.float32)
         g = bits_to_f64(bf16_bits(rng.uniform(0.9, 1.1, d)))
         out = torch.empty((T, d), dtype=torch.bfloat16, device="cuda")
-        q.qos_op_rmsnorm(torch.from_numpy(x).cuda().data_ptr(), _dev_bf16(torch, g).data_ptr(), out.data_ptr(),
-                         T, d, 1e-5)
+        dx, dg = torch.from_numpy(x).cuda(), _dev_bf16(torch, g)   # keep the device inputs alive
+        q.qos_op_rmsnorm(dx.data_ptr(), dg.data_ptr(), out.data_ptr(), T, d, 1e-5)
         torch.cuda.synchronize()
         assert row_rel_err(out.float().cpu().numpy(), rms_norm(x.astype(np.float64), g, 1e-5)) <= 8e-3
 
