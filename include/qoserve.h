@@ -186,8 +186,9 @@ enum {
   QOS_T_HEAD, QOS_T_ARGMAX, QOS_T_COUNT
 };
 /* When enabled, every kernel class of each step is bracketed by CUDA events on the step's
- * stream; qos_last_step_timing then returns per-class summed device ms and launch counts of
- * the last step (it synchronises on the step's final event). */
+ * stream (no host synchronisation).  qos_last_step_timing returns the per-class summed device
+ * ms and bracket counts of all steps since timing was enabled or since its previous call, and
+ * resets the accumulation (it synchronises on the last recorded event). */
 int qos_engine_set_timing(qos_engine_t* eng, int enable);
 int qos_last_step_timing(qos_engine_t* eng, float ms[QOS_T_COUNT], int32_t launches[QOS_T_COUNT]);
 /* Total kernel launches issued by this engine since creation (the bench's gpu_launches). */

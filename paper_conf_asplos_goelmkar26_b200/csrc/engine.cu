@@ -697,8 +697,6 @@ int do_step(qos_engine* e, const qos_batch* b, void* logits, int logits_dtype, i
     e->meta_cur ^= 1;  // staging not used
     return r;
   }
-  e->tev.clear();
-  e->ev_used = 0;
   uint8_t* dm = nullptr;
   {
     TimerScope ts(e, QOS_T_META, st);
@@ -1135,7 +1133,10 @@ int qos_profile_step(qos_engine_t* e, int32_t chunk_len, int32_t n_decode, const
 
 int qos_engine_set_timing(qos_engine_t* e, int enable) {
   if (!e) return set_error(QOS_ERR_INVALID_ARG, "engine is NULL");
+  if (cudaDeviceSynchronize() != cudaSuccess) return set_error(QOS_ERR_CUDA, "set_timing sync");
   e->timing = enable != 0;
+  e->tev.clear();
+  e->ev_used = 0;
   return QOS_OK;
 }
 
@@ -1152,6 +1153,8 @@ int qos_last_step_timing(qos_engine_t* e, float ms[QOS_T_COUNT], int32_t launche
     ms[x.first] += t;
     if (launches) launches[x.first] += 1;
   }
+  e->tev.clear();
+  e->ev_used = 0;
   return QOS_OK;
 }
 
