@@ -96,123 +96,127 @@ def _dist():
 
 
 # ------------------------------------------------------------------------------ our arm
+class Workload:
+    """The bench workload on one GPU: engine with Llama-3-8B shapes, 128 decode requests with
+    synthetic ctx-4096 prefixes, and a fresh 2048-token chunk request per step.  Decodes advance
+    one token per step (steady-state serving); each step's chunk request is freed after it."""
+
+    def __init__(self, device: int, n_steps: int, chunk=CHUNK, n_dec=N_DEC, ctx=CTX, n_layers=None):
+        import synth
+        from paper_conf_asplos_goelmkar26_b200 import qoserve as q
+        from paper_conf_asplos_goelmkar26_b200.presets import preset
+        self.q = q
+        self.chunk, self.n_dec = chunk, n_dec
+        ctx_cap = ctx + n_steps + 2
+        over = {} if n_layers is None else {"n_layers": n_layers}
+        num_blocks = n_dec * ((ctx_cap + 15) // 16) + (n_steps + 4) * ((chunk + 15) // 16) + 64
+        self.cfg = q.model_cfg(**preset("llama3-8b", **over), num_blocks=num_blocks, max_seq_len=8192,
+                               max_requests=n_dec + 64, max_batch_tokens=chunk + n_dec, max_batch_rows=n_dec + 1)
+        self.eng = q.Engine(self.cfg, device=device)
+        self.eng.qos_engine_load_synthetic(synth.SEED_WEIGHTS)
+        self.dec_reqs = list(range(1, n_dec + 1))
+        for r in self.dec_reqs:
+            self.eng.qos_kv_alloc(r, ctx_cap)
+            self.eng.qos_kv_fill_synthetic(r, ctx, synth.SEED_KVFILL)
+        self.ctx = {r: ctx for r in self.dec_reqs}
+        self.tokens = synth.request_tokens(0, chunk, self.cfg.vocab)
+        self._next_req = 10_000
+        self.live = []
+        self.tokens_per_step = chunk + n_dec
+
+    def next_batch(self):
+        cr = self._next_req
+        self._next_req += 1
+        self.eng.qos_kv_alloc(cr, self.chunk)
+        self.live.append(cr)
+        dec = [(r, self.ctx[r], (r * 7 + self.ctx[r]) % self.cfg.vocab) for r in self.dec_reqs]
+        for r in self.dec_reqs:
+            self.ctx[r] += 1
+        return self.q.make_batch([(cr, 0, self.tokens)], dec)
+
+    def retire(self):
+        # the oldest enqueued step's chunk request leaves the engine; freeing right after the
+        # (asynchronous) step is safe: later steps reusing its blocks are stream-ordered
+        self.eng.qos_kv_free(self.live.pop(0))
+
+    def step(self, batch, out_ptr, on_host, stream_ptr):
+        self.eng.qos_hybrid_step(batch, None, self.q.QOS_F32, out_ptr, on_host, stream_ptr)
+        self.retire()
+
+
 def run_ours(args):
     import torch
     import torch.distributed as dist
-    import synth
-    from paper_conf_asplos_goelmkar26_b200 import qoserve as q
-    from paper_conf_asplos_goelmkar26_b200.presets import preset
 
     ws, rank, local = _dist()
     torch.cuda.set_device(local)
     if ws > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     K, W = args.steps, args.warmup
-    n_steps = W + 3 * K + 2          # warm-up + three timed passes
-    ctx_cap = CTX + n_steps + 2
-    chunk_reqs = list(range(10_000, 10_000 + 2 * n_steps + 4))
-    num_blocks = N_DEC * ((ctx_cap + 15) // 16) + 2 * ((CHUNK + 15) // 16) + 64
-    cfg = q.model_cfg(**preset("llama3-8b"), num_blocks=num_blocks, max_seq_len=8192, max_requests=N_DEC + 64,
-                      max_batch_tokens=CHUNK + N_DEC, max_batch_rows=N_DEC + 1)
-    eng = q.Engine(cfg, device=local)
-    eng.qos_engine_load_synthetic(synth.SEED_WEIGHTS)
-    dec_reqs = list(range(1, N_DEC + 1))
-    for r in dec_reqs:
-        eng.qos_kv_alloc(r, ctx_cap)
-        eng.qos_kv_fill_synthetic(r, CTX, synth.SEED_KVFILL)
-    ctx = {r: CTX for r in dec_reqs}
-    tokens = synth.request_tokens(0, CHUNK, cfg.vocab)
+    wl = Workload(local, W + 3 * K + 2)
+    q, eng, T = wl.q, wl.eng, wl.tokens_per_step
     stream = torch.cuda.current_stream()
     sptr = stream.cuda_stream
     out_tok = torch.empty(N_DEC + 1, dtype=torch.int32, device="cuda")
-    it = iter(chunk_reqs)
-    live_chunk = []
-
-    def next_batch():
-        cr = next(it)
-        eng.qos_kv_alloc(cr, CHUNK)
-        live_chunk.append(cr)
-        dec = [(r, ctx[r], (r * 7 + ctx[r]) % cfg.vocab) for r in dec_reqs]
-        for r in dec_reqs:
-            ctx[r] += 1
-        return q.make_batch([(cr, 0, tokens)], dec)
-
-    def retire():
-        while len(live_chunk) > 2:          # the chunk request leaves the step; free its KV
-            eng.qos_kv_free(live_chunk.pop(0))
-
-    T = CHUNK + N_DEC
     # -------- warm-up
     for _ in range(W):
-        eng.qos_hybrid_step(next_batch(), None, q.QOS_F32, out_tok.data_ptr(), False, sptr)
-        retire()
+        wl.step(wl.next_batch(), out_tok.data_ptr(), False, sptr)
     torch.cuda.synchronize()
-    batches = [next_batch() for _ in range(K)]
-    # -------- timed region (device-resident outputs), per-kernel events on the step stream
-    eng.qos_engine_set_timing(True)
-    per_class = {}
+
+    def timed_pass(instrument: bool):
+        batches = [wl.next_batch() for _ in range(K)]
+        eng.qos_engine_set_timing(instrument)
+        if ws > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in batches]
+        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ev0.record(stream)
+        for b, (e0, e1) in zip(batches, evs):
+            e0.record(stream)
+            wl.step(b, out_tok.data_ptr(), False, sptr)
+            e1.record(stream)
+        ev1.record(stream)
+        torch.cuda.synchronize()
+        if ws > 1:
+            dist.barrier()
+        per = eng.qos_last_step_timing() if instrument else None
+        eng.qos_engine_set_timing(False)
+        return ev0.elapsed_time(ev1) / K, [a.elapsed_time(b) for a, b in evs], per
+
+    # -------- headline timed pass: device-resident outputs, no instrumentation
     clocks = ClockSampler(local)
     clocks.start()
     l0 = q.launch_count()
-    if ws > 1:
-        dist.barrier()
-    torch.cuda.synchronize()
-    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    step_ms = []
-    ev0.record(stream)
-    for b in batches:
-        e0 = torch.cuda.Event(enable_timing=True)
-        e1 = torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        eng.qos_hybrid_step(b, None, q.QOS_F32, out_tok.data_ptr(), False, sptr)
-        e1.record(stream)
-        step_ms.append((e0, e1))
-        retire()
-    ev1.record(stream)
-    torch.cuda.synchronize()
-    for k, (ms, n) in eng.qos_last_step_timing().items():   # summed over the K timed steps
-        per_class[k] = [ms, n]
-    if ws > 1:
-        dist.barrier()
+    ms_step, steps_ms, _ = timed_pass(False)
     launches = q.launch_count() - l0
     clk = clocks.stop()
-    eng.qos_engine_set_timing(False)
-    total_ms = ev0.elapsed_time(ev1)
-    steps_ms = [a.elapsed_time(b) for a, b in step_ms]
-    # -------- second timed pass without per-kernel events (overhead check; reported)
-    batches = [next_batch() for _ in range(K)]
-    torch.cuda.synchronize()
-    ev0.record(stream)
-    for b in batches:
-        eng.qos_hybrid_step(b, None, q.QOS_F32, out_tok.data_ptr(), False, sptr)
-        retire()
-    ev1.record(stream)
-    torch.cuda.synchronize()
-    plain_ms = ev0.elapsed_time(ev1) / K
+    # -------- instrumented timed pass: CUDA events around every kernel class on the step stream
+    ms_instr, _, per_class = timed_pass(True)
     # -------- e2e: through the public API with host buffers (descriptor in, tokens out)
-    batches = [next_batch() for _ in range(K)]
+    batches = [wl.next_batch() for _ in range(K)]
     host_tok = np.empty(N_DEC + 1, dtype=np.int32)
     torch.cuda.synchronize()
     t0 = time.perf_counter()
     for b in batches:
-        eng.qos_hybrid_step(b, None, q.QOS_F32, host_tok.ctypes.data, True, sptr)
-        retire()
+        wl.step(b, host_tok.ctypes.data, True, sptr)
     e2e_ms = (time.perf_counter() - t0) * 1e3 / K
+    h2d, d2h = eng.qos_last_step_io()
     # -------- max over ranks
-    ms_step = total_ms / K
     if ws > 1:
-        t = torch.tensor([ms_step, e2e_ms], device="cuda")
+        t = torch.tensor([ms_step, e2e_ms, ms_instr], device="cuda")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms_step, e2e_ms = float(t[0]), float(t[1])
+        ms_step, e2e_ms, ms_instr = float(t[0]), float(t[1]), float(t[2])
     peaks = _peaks()
-    d, F, hd, Hkv, L = 4096, 14336, 128, 8, 32
+    d, F, hd, Hkv = 4096, 14336, 128, 8
     gu_ms, gu_n = per_class["gemm_gateup"]
-    gu_flops = 2.0 * T * d * (2 * F)                    # per launch (one layer)
+    gu_flops = 2.0 * T * d * (2 * F)                    # algorithmic FLOPs per launch (one layer)
     gu_tfs = gu_flops / (gu_ms / gu_n * 1e-3) / 1e12
     peak_tc = peaks.get("bf16_tflops_sustained") or 1400.0
     da_ms, da_n = per_class["decode_attn"]
-    # decode attention: K+V bytes of every decode's (ctx+1) keys per layer
-    mean_ctx = CTX + W + K + 0.5 * K                   # contexts grew one token per step
+    # decode attention: K+V bytes of every decode's (ctx+1) keys per layer (SURVEY.md §8(d));
+    # the instrumented pass ran after warm-up + one timed pass, contexts grew 1 token per step
+    mean_ctx = CTX + W + K + (K - 1) / 2.0
     da_bytes = 4.0 * hd * Hkv * N_DEC * (mean_ctx + 1)
     da_gbs = da_bytes / (da_ms / da_n * 1e-3) / 1e9
     peak_hbm = peaks.get("hbm_gbs") or 6650.0
@@ -237,7 +241,7 @@ def run_ours(args):
                    "n_decode": N_DEC, "ctx": CTX, "tokens_per_step": T, "parallelism": f"replicas{ws}",
                    "l2": "inputs larger than L2 (16 GB weights + 69 GB KV streamed per step)"},
         "latency_ms": {"median": round(statistics.median(steps_ms), 4), "min": round(min(steps_ms), 4),
-                       "max": round(max(steps_ms), 4), "without_kernel_events": round(plain_ms, 4)},
+                       "max": round(max(steps_ms), 4), "instrumented_pass": round(ms_instr, 4)},
         "breakdown_ms_per_step": {k: round(v[0] / K, 4) for k, v in per_class.items() if v[1]},
         "roofline": {"kernel": "gemm_gateup (tcgen05, a11)", "bound": "tensor", "achieved": round(gu_tfs, 1),
                      "peak": peak_tc, "unit": "TFLOP/s", "frac": round(gu_tfs / peak_tc, 4),
@@ -250,7 +254,7 @@ def run_ours(args):
         "clocks": clk,
         "e2e": {"value": round(ws * T / (e2e_ms * 1e-3), 1), "unit": "tokens/s",
                 "ms_per_step": round(e2e_ms, 4),
-                "h2d_bytes_per_step": int(T * 4 + N_DEC * 12 + 64), "d2h_bytes_per_step": int((N_DEC + 1) * 4),
+                "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
                 "how": "qos_hybrid_step with host descriptor and host next_tokens (outputs_on_host=1), wall clock"},
     }
     if rank == 0 and not args.no_cpu_baseline:

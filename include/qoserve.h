@@ -191,7 +191,10 @@ enum {
  * resets the accumulation (it synchronises on the last recorded event). */
 int qos_engine_set_timing(qos_engine_t* eng, int enable);
 int qos_last_step_timing(qos_engine_t* eng, float ms[QOS_T_COUNT], int32_t launches[QOS_T_COUNT]);
-/* Total kernel launches issued by this engine since creation (the bench's gpu_launches). */
+/* Host->device bytes (descriptor metadata + table updates) and device->host bytes (outputs
+ * when outputs_on_host) moved by the last qos_hybrid_step. */
+int qos_last_step_io(qos_engine_t* eng, int64_t* h2d_bytes, int64_t* d2h_bytes);
+/* Total kernel launches issued by this library in this process (the bench's gpu_launches). */
 int qos_engine_launch_count(qos_engine_t* eng, int64_t* out);
 
 const char* qos_strerror(int code);

@@ -231,6 +231,7 @@ struct qos_engine {
   size_t ev_used = 0;
   // comm
   ncclComm_t comm = nullptr;
+  int64_t last_h2d = 0, last_d2h = 0;  // bytes moved host<->device by the last step
   // debug buffers for ops
   void* dbg = nullptr;
   size_t dbg_bytes = 0;
@@ -704,6 +705,10 @@ int do_step(qos_engine* e, const qos_batch* b, void* logits, int logits_dtype, i
   }
   QOS_TRY(run_layers(e, m, dm, logits, logits_dtype, next_tokens, !on_host, st));
   QOS_TRY(release_staging(e, st));
+  e->last_h2d = int64_t(m.used);
+  e->last_d2h = on_host ? int64_t(m.R) * ((next_tokens ? 4 : 0) +
+                                          (logits ? int64_t(e->cfg.vocab) * (logits_dtype == QOS_F32 ? 4 : 2) : 0))
+                        : 0;
   if (check_and_advance) {
     for (int i = 0; i < b->n_prefill; ++i) e->reqs[b->prefill[i].req].cached += b->prefill[i].chunk_len;
     for (int i = 0; i < b->n_decode; ++i) e->reqs[b->decode[i].req].cached += 1;
@@ -1155,6 +1160,13 @@ int qos_last_step_timing(qos_engine_t* e, float ms[QOS_T_COUNT], int32_t launche
   }
   e->tev.clear();
   e->ev_used = 0;
+  return QOS_OK;
+}
+
+int qos_last_step_io(qos_engine_t* e, int64_t* h2d_bytes, int64_t* d2h_bytes) {
+  if (!e || !h2d_bytes || !d2h_bytes) return set_error(QOS_ERR_INVALID_ARG, "args");
+  *h2d_bytes = e->last_h2d;
+  *d2h_bytes = e->last_d2h;
   return QOS_OK;
 }
 

@@ -91,6 +91,7 @@ _SIGS = {
                             C.POINTER(C.c_float), C.POINTER(C.c_float)],
     "qos_engine_set_timing": [_P, C.c_int],
     "qos_last_step_timing": [_P, C.POINTER(C.c_float), C.POINTER(C.c_int32)],
+    "qos_last_step_io": [_P, C.POINTER(C.c_int64), C.POINTER(C.c_int64)],
     "qos_engine_launch_count": [_P, C.POINTER(C.c_int64)],
     "qos_op_gemm": [_P, _P, _P, C.c_int64, C.c_int64, C.c_int64, C.c_int, _P, _P],
     "qos_op_rmsnorm": [_P, _P, _P, C.c_int32, C.c_int32, C.c_float, _P],
@@ -303,6 +304,11 @@ class Engine:
         n = (C.c_int32 * len(TIMING_CLASSES))()
         _call("qos_last_step_timing", self.h, ms, n)
         return {k: (ms[i], n[i]) for i, k in enumerate(TIMING_CLASSES)}
+
+    def qos_last_step_io(self):
+        a, b = C.c_int64(), C.c_int64()
+        _call("qos_last_step_io", self.h, C.byref(a), C.byref(b))
+        return a.value, b.value
 
     # ops
     def qos_op_rope_kv_append(self, layer: int, batch: _BatchKeep, qkv_bits: np.ndarray, q_cols: int):
