@@ -167,7 +167,7 @@ QOS_DEV void softmax_step(float (&s)[2][4], float (&m)[2], float (&l)[2], float 
 
 // ------------------------------------------------------------------------------ decode
 template <int HD>
-__global__ void __launch_bounds__(kAttnThreads)
+__global__ void __launch_bounds__(kAttnThreads, 3)
     decode_attn_kernel(const __grid_constant__ CUtensorMap kvmap, const AttnParams p, const DecodeItem* __restrict__ items,
                        float* __restrict__ partials) {
   using C = AttnCfg<HD>;

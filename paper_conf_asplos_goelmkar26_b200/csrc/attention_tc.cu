@@ -1,0 +1,369 @@
+// attention_tc.cu — varlen causal prefill attention over the paged KV cache on tcgen05 tensor
+// cores with TMEM accumulators ("prefill chunk attends to its own
+// earlier KV blocks plus itself", BASELINE.json:north_star; chunked prefill).
+//
+// Work item = (chunk, 128-row Q tile, kv head).  The 128 rows pack (position, head-in-group)
+// pairs, so one K/V tile serves the whole GQA group: 128/g positions x g heads.
+//   warp 0      TMA producer: K and V tiles of 128 keys (8 paged blocks x 2 halves of 64 dims,
+//               128-B swizzle) into 2-stage K and V rings
+//   warp 1      MMA issuer (one lane): S_j = Q K_j^T  (UMMA 128x128x16, A,B from smem) into
+//               TMEM S[j%2];  O += P_j V_j  (UMMA 128xHDx16, A = P from TMEM, B = V MN-major)
+//   warps 2..5  softmax, one TMEM lane (= one row) per thread: masked fp32 online softmax with
+//               exp2, P (bf16) written back over S[j%2] in TMEM; O is rescaled in TMEM only
+//               when the running max grows by more than 2^8 (P <= 2^8 otherwise); epilogue
+//               O / l -> global.
+// The QK of tile j+1 overlaps the softmax of tile j (two S buffers); the PV of tile j runs
+// while the softmax of tile j+1 computes.
+#include <cfloat>
+
+#include "common.cuh"
+#include "internal.h"
+
+namespace qos {
+
+template <int HD>
+struct FaCfg {
+  static constexpr int kRows = 128;                  // Q-tile rows (UMMA M)
+  static constexpr int kKeys = 128;                  // keys per K/V tile
+  static constexpr int kHalves = HD / 64;
+  static constexpr int kQBytes = kRows * HD * 2;     // 32 KB at HD 128
+  static constexpr int kTileBytes = kKeys * HD * 2;  // one K or V tile
+  static constexpr int kStages = 2;
+  static constexpr int kSmem = kQBytes + 2 * kStages * kTileBytes + 1024 + 256;
+  static constexpr uint32_t kColS0 = 0, kColS1 = 128, kColO = 256;
+  static constexpr uint32_t kTmemCols = 512;
+};
+
+constexpr int kFaThreads = 192;
+
+QOS_DEV void tmem_st32x32b_x16(uint32_t taddr, const uint32_t (&r)[16]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(
+          taddr),
+      "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]), "r"(r[6]), "r"(r[7]), "r"(r[8]), "r"(r[9]),
+      "r"(r[10]), "r"(r[11]), "r"(r[12]), "r"(r[13]), "r"(r[14]), "r"(r[15])
+      : "memory");
+}
+QOS_DEV void tmem_st_wait() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
+
+// D[tmem] (+)= A[tmem] · B[smem desc]   (kind::f16, A = bf16 pairs packed in 32-bit columns)
+QOS_DEV void umma_bf16_ts(uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc, uint32_t idesc, uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n\t}" ::"r"(d_tmem),
+      "r"(a_tmem), "l"(b_desc), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+
+// MN-major 128-B swizzled operand (V: key rows of 64 contiguous dims): atoms of 8 K-rows x
+// 64 MN elements (1 KB); K atoms stacked at SBO = 1024 B, MN atoms (the second 64 dims) at
+// LBO = one 64-dim half of the tile.
+QOS_DEV uint64_t umma_desc_sw128_mn(uint32_t smem_addr, uint32_t lbo_bytes) {
+  uint64_t d = 0;
+  d |= (uint64_t)((smem_addr & 0x3FFFF) >> 4);
+  d |= (uint64_t)((lbo_bytes >> 4) & 0x3FFF) << 16;
+  d |= (uint64_t)(1024 >> 4) << 32;
+  d |= (uint64_t)1 << 46;
+  d |= (uint64_t)2 << 61;
+  return d;
+}
+
+struct FaParams {
+  const __nv_bfloat16* q;
+  int q_ld;
+  void* out;
+  int out_ld;
+  int out_f32;
+  int layer, H, Hkv;
+  const int32_t* tables;
+  int table_w;
+  float scale_log2;
+};
+
+template <int HD>
+__global__ void __launch_bounds__(kFaThreads, 1)
+    prefill_attn_tc_kernel(const __grid_constant__ CUtensorMap kvmap, const FaParams p,
+                           const PrefillItem* __restrict__ items) {
+  using C = FaCfg<HD>;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sQ = smem;
+  uint8_t* sK = smem + C::kQBytes;
+  uint8_t* sV = sK + C::kStages * C::kTileBytes;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(sV + C::kStages * C::kTileBytes);
+  uint64_t* k_full = bar;
+  uint64_t* k_empty = bar + 2;
+  uint64_t* v_full = bar + 4;
+  uint64_t* v_empty = bar + 6;
+  uint64_t* s_full = bar + 8;
+  uint64_t* p_full = bar + 10;
+  uint64_t* o_full = bar + 12;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 14);
+
+  const PrefillItem it = items[blockIdx.x];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int group = p.H / p.Hkv;
+  const int ppt = C::kRows / group;  // positions per tile
+  const int last_pos = it.pos0 + it.npos - 1;
+  const int ntiles = last_pos / C::kKeys + 1;
+  const int last_blk = last_pos >> 4;
+
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&k_full[i], 1);
+      mbar_init(&k_empty[i], 1);
+      mbar_init(&v_full[i], 1);
+      mbar_init(&v_empty[i], 1);
+      mbar_init(&s_full[i], 1);
+      mbar_init(&p_full[i], 128);
+    }
+    mbar_init(o_full, 1);
+    fence_mbar_init();
+  }
+  if (warp == 1) tmem_alloc<C::kTmemCols>(tmem_slot);
+
+  // ---- Q tile -> smem (softmax warps; one row per thread), K-major 128-B swizzle
+  int row = 0, pos_r = -1;
+  size_t tok_off = 0;
+  if (warp >= 2) {
+    row = (warp & 3) * 32 + lane;  // TMEM lane quarter of this warp
+    const int pi = row / group, hh = row % group;
+    const bool ok = row < ppt * group && pi < it.npos;
+    pos_r = ok ? it.pos0 + pi : -1;
+    tok_off = size_t(it.row0 + pi) * p.out_ld + size_t(it.kv_head * group + hh) * HD;
+    const __nv_bfloat16* src = p.q + size_t(it.row0 + pi) * p.q_ld + size_t(it.kv_head * group + hh) * HD;
+#pragma unroll
+    for (int ch = 0; ch < HD / 8; ++ch) {
+      const uint4 v = ok ? *reinterpret_cast<const uint4*>(src + ch * 8) : make_uint4(0, 0, 0, 0);
+      const int hf = ch >> 3, c = ch & 7;
+      *reinterpret_cast<uint4*>(sQ + hf * (C::kRows * 128) + row * 128 + ((c ^ (row & 7)) << 4)) = v;
+    }
+    fence_proxy_async_smem();
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == 0) {
+    // ------------------------------------------------------------------ TMA producer
+    if (elect_one()) {
+      tma_prefetch_desc(&kvmap);
+      const int32_t* trow = p.tables + size_t(it.table) * p.table_w;
+      for (int j = 0; j < ntiles; ++j) {
+        const int s = j & 1;
+        const uint32_t ph = (j >> 1) & 1;
+        mbar_wait(&k_empty[s], ph ^ 1);
+        mbar_arrive_expect_tx(&k_full[s], C::kTileBytes);
+        uint8_t* kt = sK + s * C::kTileBytes;
+        for (int b = 0; b < 8; ++b) {
+          const int blk = min(j * 8 + b, last_blk);  // past the causal end: any valid block (P = 0)
+          const int r = (__ldg(trow + blk) * p.Hkv + it.kv_head) * 16;
+#pragma unroll
+          for (int hf = 0; hf < C::kHalves; ++hf)
+            tma_load_3d(kt + hf * (C::kKeys * 128) + b * 2048, &kvmap, &k_full[s], hf * 64, r, p.layer * 2 + 0);
+        }
+        mbar_wait(&v_empty[s], ph ^ 1);
+        mbar_arrive_expect_tx(&v_full[s], C::kTileBytes);
+        uint8_t* vt = sV + s * C::kTileBytes;
+        for (int b = 0; b < 8; ++b) {
+          const int blk = min(j * 8 + b, last_blk);
+          const int r = (__ldg(trow + blk) * p.Hkv + it.kv_head) * 16;
+#pragma unroll
+          for (int hf = 0; hf < C::kHalves; ++hf)
+            tma_load_3d(vt + hf * (C::kKeys * 128) + b * 2048, &kvmap, &v_full[s], hf * 64, r, p.layer * 2 + 1);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ------------------------------------------------------------------ MMA issuer
+    if (elect_one()) {
+      constexpr uint32_t idesc_qk = umma_idesc_bf16(128, C::kKeys);
+      constexpr uint32_t idesc_pv = umma_idesc_bf16(128, HD) | (1u << 16);  // B (V) MN-major
+      const uint32_t q_base = smem_u32(sQ);
+      auto issue_pv = [&](int t) {
+        const int s = t & 1;
+        const uint32_t ph = (t >> 1) & 1;
+        mbar_wait(&p_full[s], ph);
+        mbar_wait(&v_full[s], ph);
+        tc_fence_after();
+        const uint32_t v_base = smem_u32(sV + s * C::kTileBytes);
+        const uint32_t p_tmem = tmem + (s ? C::kColS1 : C::kColS0);
+#pragma unroll
+        for (int kk = 0; kk < C::kKeys / 16; ++kk) {
+          const uint64_t vd = umma_desc_sw128_mn(v_base + kk * 2048, C::kKeys * 128);
+          const uint32_t pc = p_tmem + (kk >> 1) * 32 + (kk & 1) * 8;
+          umma_bf16_ts(tmem + C::kColO, pc, vd, idesc_pv, (t | kk) != 0);   // P_hi
+          umma_bf16_ts(tmem + C::kColO, pc + 16, vd, idesc_pv, 1);          // P_lo
+        }
+        umma_commit(o_full);
+        umma_commit(&v_empty[s]);
+      };
+      for (int j = 0; j < ntiles; ++j) {
+        const int s = j & 1;
+        const uint32_t ph = (j >> 1) & 1;
+        mbar_wait(&k_full[s], ph);
+        tc_fence_after();
+        const uint32_t k_base = smem_u32(sK + s * C::kTileBytes);
+        const uint32_t s_tmem = tmem + (s ? C::kColS1 : C::kColS0);
+#pragma unroll
+        for (int ks = 0; ks < HD / 16; ++ks) {
+          const uint32_t off = (ks >> 2) * (C::kRows * 128) + (ks & 3) * 32;
+          const uint32_t koff = (ks >> 2) * (C::kKeys * 128) + (ks & 3) * 32;
+          umma_bf16(s_tmem, umma_desc_sw128(q_base + off), umma_desc_sw128(k_base + koff), idesc_qk, ks != 0);
+        }
+        umma_commit(&s_full[s]);
+        umma_commit(&k_empty[s]);
+        if (j >= 1) issue_pv(j - 1);
+      }
+      issue_pv(ntiles - 1);
+    }
+  } else {
+    // ------------------------------------------------------------------ softmax (warps 2..5)
+    const uint32_t lane_base = tmem + (uint32_t((warp & 3) * 32) << 16);
+    float m_used = -INFINITY, l = 0.f;
+    for (int j = 0; j < ntiles; ++j) {
+      const int s = j & 1;
+      const uint32_t ph = (j >> 1) & 1;
+      mbar_wait(&s_full[s], ph);
+      tc_fence_after();
+      const uint32_t s_addr = lane_base + (s ? C::kColS1 : C::kColS0);
+      const int key0 = j * C::kKeys;
+      // pass 1: row max of the masked, log2-scaled scores
+      float mx = -INFINITY;
+#pragma unroll
+      for (int c = 0; c < C::kKeys / 32; ++c) {
+        uint32_t r[32];
+        tmem_ld32x32b_x16(s_addr + c * 32, *reinterpret_cast<uint32_t(*)[16]>(&r[0]));
+        tmem_ld32x32b_x16(s_addr + c * 32 + 16, *reinterpret_cast<uint32_t(*)[16]>(&r[16]));
+        tmem_ld_wait();
+#pragma unroll
+        for (int i = 0; i < 32; ++i)
+          if (key0 + c * 32 + i <= pos_r) mx = fmaxf(mx, __uint_as_float(r[i]) * p.scale_log2);
+      }
+      // lazy rescale: keep the previous max unless the new one exceeds it by > 8 (P <= 2^8)
+      const bool rescale = mx > m_used + 8.f;
+      const float m_new = rescale ? mx : m_used;
+      const float alpha = (rescale && m_used != -INFINITY) ? exp2f(m_used - m_new) : 1.f;
+      const float mb = (m_new == -INFINITY) ? 0.f : m_new;
+      // pass 2: P = 2^(s - m) and the row sum; P is written as two bf16 terms (P = P_hi + P_lo,
+      // exact to ~2^-16 so the fp32 P.V meets the 2e-3 attention bar) over the 32 S columns each
+      // chunk has just read: columns [32c, 32c+16) = P_hi, [32c+16, 32c+32) = P_lo of keys
+      // 32c .. 32c+31, bf16 pairs packed in 32-bit columns.
+      float sum = 0.f;
+#pragma unroll
+      for (int c = 0; c < C::kKeys / 32; ++c) {
+        uint32_t r[32];
+        tmem_ld32x32b_x16(s_addr + c * 32, *reinterpret_cast<uint32_t(*)[16]>(&r[0]));
+        tmem_ld32x32b_x16(s_addr + c * 32 + 16, *reinterpret_cast<uint32_t(*)[16]>(&r[16]));
+        tmem_ld_wait();
+        uint32_t hi[16], lo[16];
+#pragma unroll
+        for (int i = 0; i < 16; ++i) {
+          const int k = key0 + c * 32 + 2 * i;
+          const float p0 = (k <= pos_r) ? exp2f(__uint_as_float(r[2 * i]) * p.scale_log2 - mb) : 0.f;
+          const float p1 = (k + 1 <= pos_r) ? exp2f(__uint_as_float(r[2 * i + 1]) * p.scale_log2 - mb) : 0.f;
+          hi[i] = pack_bf16(p0, p1);
+          lo[i] = pack_bf16(p0 - bf16_lo(hi[i]), p1 - bf16_hi(hi[i]));
+          sum += p0 + p1;
+        }
+        tmem_st32x32b_x16(s_addr + c * 32, hi);
+        tmem_st32x32b_x16(s_addr + c * 32 + 16, lo);
+      }
+      tmem_st_wait();
+      l = l * alpha + sum;
+      if (j >= 1) {
+        // O holds tiles < j once PV_{j-1} is done; rescale it before PV_j accumulates
+        mbar_wait(o_full, (j - 1) & 1);
+        tc_fence_after();
+        if (__any_sync(0xffffffffu, alpha != 1.f)) {
+#pragma unroll 1
+          for (int c = 0; c < HD / 16; ++c) {
+            uint32_t r[16];
+            tmem_ld32x32b_x16(lane_base + C::kColO + c * 16, r);
+            tmem_ld_wait();
+#pragma unroll
+            for (int i = 0; i < 16; ++i) r[i] = __float_as_uint(__uint_as_float(r[i]) * alpha);
+            tmem_st32x32b_x16(lane_base + C::kColO + c * 16, r);
+          }
+          tmem_st_wait();
+        }
+      }
+      m_used = m_new;
+      tc_fence_before();
+      mbar_arrive(&p_full[s]);
+    }
+    // epilogue: O / l
+    mbar_wait(o_full, (ntiles - 1) & 1);
+    tc_fence_after();
+    const float inv = (l > 0.f) ? 1.f / l : 0.f;
+#pragma unroll 1
+    for (int c = 0; c < HD / 32; ++c) {
+      uint32_t r[32];
+      tmem_ld32x32b_x16(lane_base + C::kColO + c * 32, *reinterpret_cast<uint32_t(*)[16]>(&r[0]));
+      tmem_ld32x32b_x16(lane_base + C::kColO + c * 32 + 16, *reinterpret_cast<uint32_t(*)[16]>(&r[16]));
+      tmem_ld_wait();
+      if (pos_r >= 0) {
+        if (p.out_f32) {
+          float4* dst = reinterpret_cast<float4*>(reinterpret_cast<float*>(p.out) + tok_off + c * 32);
+#pragma unroll
+          for (int i = 0; i < 8; ++i)
+            dst[i] = make_float4(__uint_as_float(r[4 * i]) * inv, __uint_as_float(r[4 * i + 1]) * inv,
+                                 __uint_as_float(r[4 * i + 2]) * inv, __uint_as_float(r[4 * i + 3]) * inv);
+        } else {
+          uint4* dst = reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.out) + tok_off + c * 32);
+#pragma unroll
+          for (int i = 0; i < 4; ++i)
+            dst[i] = make_uint4(pack_bf16(__uint_as_float(r[8 * i]) * inv, __uint_as_float(r[8 * i + 1]) * inv),
+                                pack_bf16(__uint_as_float(r[8 * i + 2]) * inv, __uint_as_float(r[8 * i + 3]) * inv),
+                                pack_bf16(__uint_as_float(r[8 * i + 4]) * inv, __uint_as_float(r[8 * i + 5]) * inv),
+                                pack_bf16(__uint_as_float(r[8 * i + 6]) * inv, __uint_as_float(r[8 * i + 7]) * inv));
+        }
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc<C::kTmemCols>(tmem);
+  }
+}
+
+template <int HD>
+static cudaError_t prefill_tc_t(const AttnLaunch& a, const PrefillItem* items, int n_items, cudaStream_t st) {
+  static bool set = false;
+  if (!set) {
+    cudaError_t e = cudaFuncSetAttribute(prefill_attn_tc_kernel<HD>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         FaCfg<HD>::kSmem);
+    if (e != cudaSuccess) return e;
+    set = true;
+  }
+  FaParams p;
+  p.q = reinterpret_cast<const __nv_bfloat16*>(a.q);
+  p.q_ld = a.q_ld;
+  p.out = a.out;
+  p.out_ld = a.out_ld;
+  p.out_f32 = a.out_f32;
+  p.layer = a.layer;
+  p.H = a.H;
+  p.Hkv = a.Hkv;
+  p.tables = a.tables;
+  p.table_w = a.table_w;
+  p.scale_log2 = a.scale_log2;
+  prefill_attn_tc_kernel<HD><<<n_items, kFaThreads, FaCfg<HD>::kSmem, st>>>(*a.kv_tmap, p, items);
+  return cudaGetLastError();
+}
+
+int prefill_tc_positions_per_tile(int group) { return 128 / group; }
+
+cudaError_t launch_prefill_attention_tc(const AttnLaunch& a, const PrefillItem* items, int n_items, cudaStream_t st) {
+  if (n_items == 0) return cudaSuccess;
+  count_launch(1);
+  if (a.hd == 128) return prefill_tc_t<128>(a, items, n_items, st);
+  if (a.hd == 64) return prefill_tc_t<64>(a, items, n_items, st);
+  return cudaErrorInvalidValue;
+}
+
+}  // namespace qos

@@ -165,7 +165,7 @@ static WsLayout ws_layout(const qos_model_cfg& c, const Shard& s, int tp) {
   w.max_items = kMaxDecodeItems;
   w.partials = take(size_t(w.max_items) * group * (hd + 2) * 4);
   // metadata: tokens, pos, slot [Tm]; logit rows [Rm]; prefill items; decode items/rows; table updates
-  const int ppt = prefill_positions_per_tile(int(group));
+  const int ppt = prefill_tc_positions_per_tile(int(group));
   const size_t max_pitems = (Tm / ppt + Rm + 1) * size_t(s.Hkv);
   w.meta_bytes = align_up(3 * Tm * 4 + Rm * 4 + 64, 256) + align_up(max_pitems * sizeof(PrefillItem), 256) +
                  align_up(size_t(w.max_items) * sizeof(DecodeItem), 256) + align_up(Rm * sizeof(DecodeRow), 256) +
@@ -224,6 +224,8 @@ struct qos_engine {
   cudaEvent_t meta_free[2] = {nullptr, nullptr};
   int meta_cur = 0;
   cudaStream_t stream = nullptr;  // internal stream for synchronous calls
+  cudaStream_t side = nullptr;    // high-priority stream: prefill attention overlapped with decode
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
   // timing
   bool timing = false;
   std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> tev;
@@ -371,7 +373,7 @@ int build_step(qos_engine* e, const qos_batch* b, bool check_lengths, uint8_t* b
   int32_t* rows = reinterpret_cast<int32_t*>(buf + m.o_rows);
 
   const int group = c.n_heads / c.n_kv_heads;
-  const int ppt = prefill_positions_per_tile(group);
+  const int ppt = prefill_tc_positions_per_tile(group);
   std::vector<PrefillItem> pitems;
   int t = 0;
   for (int i = 0; i < b->n_prefill; ++i) {
@@ -588,15 +590,28 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
                                 hd, st));
     }
     al.layer = l;
+    // a7 || a8: prefill attention (tensor-bound) and decode attention (HBM-bound) read the same
+    // freshly appended cache and write disjoint rows of `attn`, so they run concurrently: the
+    // prefill tiles on a high-priority side stream, the decode split-K items on the step stream.
+    const bool overlap = m.n_pitems && m.n_ditems;
+    cudaStream_t pst = overlap ? e->side : st;
+    if (overlap) {
+      QOS_CU(cudaEventRecord(e->ev_fork, st));
+      QOS_CU(cudaStreamWaitEvent(e->side, e->ev_fork, 0));
+    }
     if (m.n_pitems) {
-      TimerScope ts(e, QOS_T_PREFILL_ATTN, st);
-      QOS_CU(launch_prefill_attention(al, reinterpret_cast<const PrefillItem*>(dm + m.o_pitems), m.n_pitems, st));
+      TimerScope ts(e, QOS_T_PREFILL_ATTN, pst);
+      QOS_CU(launch_prefill_attention_tc(al, reinterpret_cast<const PrefillItem*>(dm + m.o_pitems), m.n_pitems, pst));
     }
     if (m.n_ditems) {
       TimerScope ts(e, QOS_T_DECODE_ATTN, st);
       QOS_CU(launch_decode_attention(al, reinterpret_cast<const DecodeItem*>(dm + m.o_ditems), m.n_ditems,
                                      reinterpret_cast<const DecodeRow*>(dm + m.o_drows), m.n_drows,
                                      reinterpret_cast<float*>(e->ws + s.partials), 0, st));
+    }
+    if (overlap) {
+      QOS_CU(cudaEventRecord(e->ev_join, e->side));
+      QOS_CU(cudaStreamWaitEvent(st, e->ev_join, 0));
     }
     if (!tp) {
       TimerScope ts(e, QOS_T_GEMM_O, st);
@@ -798,6 +813,9 @@ int qos_engine_create(const qos_model_cfg* cfg, int device, int tp_rank, int tp_
   if ((r = get(mem ? mem->weights : nullptr, e->wl.total, &e->w, &e->own_w)) != QOS_OK) return fail(r);
   if ((r = get(mem ? mem->kv : nullptr, e->kv_bytes, &e->kv, &e->own_kv)) != QOS_OK) return fail(r);
   if ((r = get(mem ? mem->workspace : nullptr, e->wsl.total, &e->ws, &e->own_ws)) != QOS_OK) return fail(r);
+  // zero the KV pool once: slots past a request's length are read (with P = 0) by the attention
+  // tiles, and 0 * NaN from uninitialised memory would poison the accumulators
+  if (cudaMemset(e->kv, 0, e->kv_bytes) != cudaSuccess) return fail(set_error(QOS_ERR_CUDA, "kv memset"));
   if (cudaMalloc(&e->d_tables, size_t(cfg->max_requests) * e->table_w * 4) != cudaSuccess)
     return fail(set_error(QOS_ERR_OOM, "block tables"));
   cudaMemset(e->d_tables, 0, size_t(cfg->max_requests) * e->table_w * 4);
@@ -820,6 +838,13 @@ int qos_engine_create(const qos_model_cfg* cfg, int device, int tp_rank, int tp_
     cudaEventCreateWithFlags(&e->meta_free[i], cudaEventDisableTiming);
   }
   cudaStreamCreateWithFlags(&e->stream, cudaStreamNonBlocking);
+  {
+    int lo = 0, hi = 0;
+    cudaDeviceGetStreamPriorityRange(&lo, &hi);
+    cudaStreamCreateWithPriority(&e->side, cudaStreamNonBlocking, hi);
+    cudaEventCreateWithFlags(&e->ev_fork, cudaEventDisableTiming);
+    cudaEventCreateWithFlags(&e->ev_join, cudaEventDisableTiming);
+  }
   e->free_heap.resize(size_t(cfg->num_blocks));
   for (int64_t i = 0; i < cfg->num_blocks; ++i) e->free_heap[size_t(i)] = int32_t(i);  // sorted = valid min-heap
   e->free_rows.resize(size_t(cfg->max_requests));
@@ -855,6 +880,9 @@ int qos_engine_destroy(qos_engine_t* e) {
   }
   for (auto ev : e->ev_pool) cudaEventDestroy(ev);
   if (e->stream) cudaStreamDestroy(e->stream);
+  if (e->side) cudaStreamDestroy(e->side);
+  if (e->ev_fork) cudaEventDestroy(e->ev_fork);
+  if (e->ev_join) cudaEventDestroy(e->ev_join);
   delete e;
   return QOS_OK;
 }
@@ -1302,7 +1330,7 @@ int qos_op_attention(qos_engine_t* e, int32_t layer, const qos_batch* b, const u
   al.tables = e->d_tables;
   al.table_w = e->table_w;
   al.scale_log2 = float(1.4426950408889634 / std::sqrt(double(hd)));
-  QOS_CU(launch_prefill_attention(al, reinterpret_cast<const PrefillItem*>(dm + m.o_pitems), m.n_pitems, st));
+  QOS_CU(launch_prefill_attention_tc(al, reinterpret_cast<const PrefillItem*>(dm + m.o_pitems), m.n_pitems, st));
   QOS_CU(launch_decode_attention(al, reinterpret_cast<const DecodeItem*>(dm + m.o_ditems), m.n_ditems,
                                  reinterpret_cast<const DecodeRow*>(dm + m.o_drows), m.n_drows,
                                  reinterpret_cast<float*>(e->ws + e->wsl.partials), 0, st));

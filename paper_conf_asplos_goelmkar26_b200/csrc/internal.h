@@ -107,5 +107,7 @@ cudaError_t launch_decode_attention(const AttnLaunch& a, const DecodeItem* items
                                     int n_rows, float* partials, int max_splits, cudaStream_t st);
 cudaError_t launch_prefill_attention(const AttnLaunch& a, const PrefillItem* items, int n_items, cudaStream_t st);
 int prefill_positions_per_tile(int group);
+cudaError_t launch_prefill_attention_tc(const AttnLaunch& a, const PrefillItem* items, int n_items, cudaStream_t st);
+int prefill_tc_positions_per_tile(int group);
 
 }  // namespace qos
