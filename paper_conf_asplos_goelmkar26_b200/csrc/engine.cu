@@ -9,6 +9,7 @@
 #include <atomic>
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <queue>
@@ -226,6 +227,7 @@ struct qos_engine {
   cudaStream_t stream = nullptr;  // internal stream for synchronous calls
   cudaStream_t side = nullptr;    // high-priority stream: prefill attention overlapped with decode
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+  bool overlap_attn = true;       // QOS_OVERLAP_ATTN=0 serialises a7 and a8 (for measurement)
   // timing
   bool timing = false;
   std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> tev;
@@ -593,7 +595,7 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
     // a7 || a8: prefill attention (tensor-bound) and decode attention (HBM-bound) read the same
     // freshly appended cache and write disjoint rows of `attn`, so they run concurrently: the
     // prefill tiles on a high-priority side stream, the decode split-K items on the step stream.
-    const bool overlap = m.n_pitems && m.n_ditems;
+    const bool overlap = e->overlap_attn && m.n_pitems && m.n_ditems;
     cudaStream_t pst = overlap ? e->side : st;
     if (overlap) {
       QOS_CU(cudaEventRecord(e->ev_fork, st));
@@ -838,6 +840,7 @@ int qos_engine_create(const qos_model_cfg* cfg, int device, int tp_rank, int tp_
     cudaEventCreateWithFlags(&e->meta_free[i], cudaEventDisableTiming);
   }
   cudaStreamCreateWithFlags(&e->stream, cudaStreamNonBlocking);
+  if (const char* ov = getenv("QOS_OVERLAP_ATTN")) e->overlap_attn = atoi(ov) != 0;
   {
     int lo = 0, hi = 0;
     cudaDeviceGetStreamPriorityRange(&lo, &hi);
