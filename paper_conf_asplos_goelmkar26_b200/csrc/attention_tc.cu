@@ -5,16 +5,17 @@
 // Work item = (chunk, 128-row Q tile, kv head).  The 128 rows pack (position, head-in-group)
 // pairs, so one K/V tile serves the whole GQA group: 128/g positions x g heads.
 //   warp 0      TMA producer: K and V tiles of 128 keys (8 paged blocks x 2 halves of 64 dims,
-//               128-B swizzle) into 2-stage K and V rings
+//               128-B swizzle)
 //   warp 1      MMA issuer (one lane): S_j = Q K_j^T  (UMMA 128x128x16, A,B from smem) into
-//               TMEM S[j%2];  O += P_j V_j  (UMMA 128xHDx16, A = P from TMEM, B = V MN-major)
+//               TMEM;  O += P_j V_j  (UMMA 128xHDx16, A = P from TMEM, B = V MN-major)
 //   warps 2..5  softmax, one TMEM lane (= one row) per thread: masked fp32 online softmax with
-//               exp2, P (bf16) written back over S[j%2] in TMEM; O is rescaled in TMEM only
-//               when the running max grows by more than 2^8 (P <= 2^8 otherwise); epilogue
-//               O / l -> global.
-// The QK of tile j+1 overlaps the softmax of tile j (two S buffers); the PV of tile j runs
-// while the softmax of tile j+1 computes.
+//               exp2, P written back over S in TMEM as two bf16 terms; O is rescaled in TMEM
+//               only when the running max grows by more than 2^8 (P <= 2^8 otherwise);
+//               epilogue O / l -> global.
+// Two CTAs share an SM (96 KB smem, 256 TMEM columns each) so one CTA's softmax overlaps the
+// other's MMAs.
 #include <cfloat>
+#include <climits>
 
 #include "common.cuh"
 #include "internal.h"
@@ -28,10 +29,11 @@ struct FaCfg {
   static constexpr int kHalves = HD / 64;
   static constexpr int kQBytes = kRows * HD * 2;     // 32 KB at HD 128
   static constexpr int kTileBytes = kKeys * HD * 2;  // one K or V tile
-  static constexpr int kStages = 2;
-  static constexpr int kSmem = kQBytes + 2 * kStages * kTileBytes + 1024 + 256;
-  static constexpr uint32_t kColS0 = 0, kColS1 = 128, kColO = 256;
-  static constexpr uint32_t kTmemCols = 512;
+  // 2 CTAs per SM: Q + one K + one V tile (96 KB at HD 128) and 256 TMEM columns each; the two
+  // co-resident CTAs interleave their serial QK -> softmax -> PV chains on the tensor core.
+  static constexpr int kSmem = kQBytes + 2 * kTileBytes + 1024 + 256;
+  static constexpr uint32_t kColS = 0, kColO = 128;
+  static constexpr uint32_t kTmemCols = 256;
 };
 
 constexpr int kFaThreads = 192;
@@ -45,6 +47,11 @@ QOS_DEV void tmem_st32x32b_x16(uint32_t taddr, const uint32_t (&r)[16]) {
       : "memory");
 }
 QOS_DEV void tmem_st_wait() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
+QOS_DEV float ex2(float x) {  // MUFU.EX2 (flush-to-zero; arguments are <= 8 here)
+  float y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
 
 // D[tmem] (+)= A[tmem] · B[smem desc]   (kind::f16, A = bf16 pairs packed in 32-bit columns)
 QOS_DEV void umma_bf16_ts(uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc, uint32_t idesc, uint32_t accumulate) {
@@ -82,7 +89,7 @@ struct FaParams {
 };
 
 template <int HD>
-__global__ void __launch_bounds__(kFaThreads, 1)
+__global__ void __launch_bounds__(kFaThreads, 2)
     prefill_attn_tc_kernel(const __grid_constant__ CUtensorMap kvmap, const FaParams p,
                            const PrefillItem* __restrict__ items) {
   using C = FaCfg<HD>;
@@ -90,16 +97,16 @@ __global__ void __launch_bounds__(kFaThreads, 1)
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sQ = smem;
   uint8_t* sK = smem + C::kQBytes;
-  uint8_t* sV = sK + C::kStages * C::kTileBytes;
-  uint64_t* bar = reinterpret_cast<uint64_t*>(sV + C::kStages * C::kTileBytes);
-  uint64_t* k_full = bar;
-  uint64_t* k_empty = bar + 2;
-  uint64_t* v_full = bar + 4;
-  uint64_t* v_empty = bar + 6;
-  uint64_t* s_full = bar + 8;
-  uint64_t* p_full = bar + 10;
-  uint64_t* o_full = bar + 12;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 14);
+  uint8_t* sV = sK + C::kTileBytes;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(sV + C::kTileBytes);
+  uint64_t* k_full = bar + 0;
+  uint64_t* k_empty = bar + 1;
+  uint64_t* v_full = bar + 2;
+  uint64_t* v_empty = bar + 3;
+  uint64_t* s_full = bar + 4;
+  uint64_t* p_full = bar + 5;
+  uint64_t* o_full = bar + 6;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 8);
 
   const PrefillItem it = items[blockIdx.x];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -110,14 +117,12 @@ __global__ void __launch_bounds__(kFaThreads, 1)
   const int last_blk = last_pos >> 4;
 
   if (threadIdx.x == 0) {
-    for (int i = 0; i < 2; ++i) {
-      mbar_init(&k_full[i], 1);
-      mbar_init(&k_empty[i], 1);
-      mbar_init(&v_full[i], 1);
-      mbar_init(&v_empty[i], 1);
-      mbar_init(&s_full[i], 1);
-      mbar_init(&p_full[i], 128);
-    }
+    mbar_init(k_full, 1);
+    mbar_init(k_empty, 1);
+    mbar_init(v_full, 1);
+    mbar_init(v_empty, 1);
+    mbar_init(s_full, 1);
+    mbar_init(p_full, 128);
     mbar_init(o_full, 1);
     fence_mbar_init();
   }
@@ -127,17 +132,19 @@ __global__ void __launch_bounds__(kFaThreads, 1)
   int row = 0, pos_r = -1;
   size_t tok_off = 0;
   if (warp >= 2) {
-    row = (warp & 3) * 32 + lane;  // TMEM lane quarter of this warp
+    row = (warp & 3) * 32 + lane;  // the TMEM lane quarter this warp may access
     const int pi = row / group, hh = row % group;
     const bool ok = row < ppt * group && pi < it.npos;
     pos_r = ok ? it.pos0 + pi : -1;
     tok_off = size_t(it.row0 + pi) * p.out_ld + size_t(it.kv_head * group + hh) * HD;
     const __nv_bfloat16* src = p.q + size_t(it.row0 + pi) * p.q_ld + size_t(it.kv_head * group + hh) * HD;
+    uint4 v[HD / 8];
+#pragma unroll
+    for (int ch = 0; ch < HD / 8; ++ch) v[ch] = ok ? *reinterpret_cast<const uint4*>(src + ch * 8) : make_uint4(0, 0, 0, 0);
 #pragma unroll
     for (int ch = 0; ch < HD / 8; ++ch) {
-      const uint4 v = ok ? *reinterpret_cast<const uint4*>(src + ch * 8) : make_uint4(0, 0, 0, 0);
       const int hf = ch >> 3, c = ch & 7;
-      *reinterpret_cast<uint4*>(sQ + hf * (C::kRows * 128) + row * 128 + ((c ^ (row & 7)) << 4)) = v;
+      *reinterpret_cast<uint4*>(sQ + hf * (C::kRows * 128) + row * 128 + ((c ^ (row & 7)) << 4)) = v[ch];
     }
     fence_proxy_async_smem();
   }
@@ -151,29 +158,23 @@ __global__ void __launch_bounds__(kFaThreads, 1)
     if (elect_one()) {
       tma_prefetch_desc(&kvmap);
       const int32_t* trow = p.tables + size_t(it.table) * p.table_w;
-      for (int j = 0; j < ntiles; ++j) {
-        const int s = j & 1;
-        const uint32_t ph = (j >> 1) & 1;
-        mbar_wait(&k_empty[s], ph ^ 1);
-        mbar_arrive_expect_tx(&k_full[s], C::kTileBytes);
-        uint8_t* kt = sK + s * C::kTileBytes;
+      auto load_tile = [&](uint8_t* dst, uint64_t* full, int j, int plane) {
         for (int b = 0; b < 8; ++b) {
           const int blk = min(j * 8 + b, last_blk);  // past the causal end: any valid block (P = 0)
           const int r = (__ldg(trow + blk) * p.Hkv + it.kv_head) * 16;
 #pragma unroll
           for (int hf = 0; hf < C::kHalves; ++hf)
-            tma_load_3d(kt + hf * (C::kKeys * 128) + b * 2048, &kvmap, &k_full[s], hf * 64, r, p.layer * 2 + 0);
+            tma_load_3d(dst + hf * (C::kKeys * 128) + b * 2048, &kvmap, full, hf * 64, r, p.layer * 2 + plane);
         }
-        mbar_wait(&v_empty[s], ph ^ 1);
-        mbar_arrive_expect_tx(&v_full[s], C::kTileBytes);
-        uint8_t* vt = sV + s * C::kTileBytes;
-        for (int b = 0; b < 8; ++b) {
-          const int blk = min(j * 8 + b, last_blk);
-          const int r = (__ldg(trow + blk) * p.Hkv + it.kv_head) * 16;
-#pragma unroll
-          for (int hf = 0; hf < C::kHalves; ++hf)
-            tma_load_3d(vt + hf * (C::kKeys * 128) + b * 2048, &kvmap, &v_full[s], hf * 64, r, p.layer * 2 + 1);
-        }
+      };
+      for (int j = 0; j < ntiles; ++j) {
+        const uint32_t ph = j & 1;
+        mbar_wait(k_empty, ph ^ 1);
+        mbar_arrive_expect_tx(k_full, C::kTileBytes);
+        load_tile(sK, k_full, j, 0);
+        mbar_wait(v_empty, ph ^ 1);
+        mbar_arrive_expect_tx(v_full, C::kTileBytes);
+        load_tile(sV, v_full, j, 1);
       }
     }
   } else if (warp == 1) {
@@ -181,56 +182,50 @@ __global__ void __launch_bounds__(kFaThreads, 1)
     if (elect_one()) {
       constexpr uint32_t idesc_qk = umma_idesc_bf16(128, C::kKeys);
       constexpr uint32_t idesc_pv = umma_idesc_bf16(128, HD) | (1u << 16);  // B (V) MN-major
-      const uint32_t q_base = smem_u32(sQ);
-      auto issue_pv = [&](int t) {
-        const int s = t & 1;
-        const uint32_t ph = (t >> 1) & 1;
-        mbar_wait(&p_full[s], ph);
-        mbar_wait(&v_full[s], ph);
+      const uint32_t q_base = smem_u32(sQ), k_base = smem_u32(sK), v_base = smem_u32(sV);
+      for (int j = 0; j < ntiles; ++j) {
+        const uint32_t ph = j & 1;
+        // S_j = Q K_j^T (S is free: PV_{j-1}, its last reader, was issued before, in order)
+        mbar_wait(k_full, ph);
         tc_fence_after();
-        const uint32_t v_base = smem_u32(sV + s * C::kTileBytes);
-        const uint32_t p_tmem = tmem + (s ? C::kColS1 : C::kColS0);
+#pragma unroll
+        for (int ks = 0; ks < HD / 16; ++ks) {
+          const uint32_t qoff = (ks >> 2) * (C::kRows * 128) + (ks & 3) * 32;
+          const uint32_t koff = (ks >> 2) * (C::kKeys * 128) + (ks & 3) * 32;
+          umma_bf16(tmem + C::kColS, umma_desc_sw128(q_base + qoff), umma_desc_sw128(k_base + koff), idesc_qk,
+                    ks != 0);
+        }
+        umma_commit(s_full);
+        umma_commit(k_empty);
+        // O += P_j V_j with P = P_hi + P_lo from TMEM
+        mbar_wait(p_full, ph);
+        mbar_wait(v_full, ph);
+        tc_fence_after();
 #pragma unroll
         for (int kk = 0; kk < C::kKeys / 16; ++kk) {
           const uint64_t vd = umma_desc_sw128_mn(v_base + kk * 2048, C::kKeys * 128);
-          const uint32_t pc = p_tmem + (kk >> 1) * 32 + (kk & 1) * 8;
-          umma_bf16_ts(tmem + C::kColO, pc, vd, idesc_pv, (t | kk) != 0);   // P_hi
-          umma_bf16_ts(tmem + C::kColO, pc + 16, vd, idesc_pv, 1);          // P_lo
+          const uint32_t pc = tmem + C::kColS + (kk >> 1) * 32 + (kk & 1) * 8;
+          umma_bf16_ts(tmem + C::kColO, pc, vd, idesc_pv, (j | kk) != 0);  // P_hi
+          umma_bf16_ts(tmem + C::kColO, pc + 16, vd, idesc_pv, 1);         // P_lo
         }
         umma_commit(o_full);
-        umma_commit(&v_empty[s]);
-      };
-      for (int j = 0; j < ntiles; ++j) {
-        const int s = j & 1;
-        const uint32_t ph = (j >> 1) & 1;
-        mbar_wait(&k_full[s], ph);
-        tc_fence_after();
-        const uint32_t k_base = smem_u32(sK + s * C::kTileBytes);
-        const uint32_t s_tmem = tmem + (s ? C::kColS1 : C::kColS0);
-#pragma unroll
-        for (int ks = 0; ks < HD / 16; ++ks) {
-          const uint32_t off = (ks >> 2) * (C::kRows * 128) + (ks & 3) * 32;
-          const uint32_t koff = (ks >> 2) * (C::kKeys * 128) + (ks & 3) * 32;
-          umma_bf16(s_tmem, umma_desc_sw128(q_base + off), umma_desc_sw128(k_base + koff), idesc_qk, ks != 0);
-        }
-        umma_commit(&s_full[s]);
-        umma_commit(&k_empty[s]);
-        if (j >= 1) issue_pv(j - 1);
+        umma_commit(v_empty);
       }
-      issue_pv(ntiles - 1);
     }
   } else {
     // ------------------------------------------------------------------ softmax (warps 2..5)
-    const uint32_t lane_base = tmem + (uint32_t((warp & 3) * 32) << 16);
+    const uint32_t s_addr = tmem + (uint32_t((warp & 3) * 32) << 16) + C::kColS;
+    const uint32_t o_addr = tmem + (uint32_t((warp & 3) * 32) << 16) + C::kColO;
+    const int warp_min_pos = __shfl_sync(0xffffffffu, pos_r < 0 ? INT_MAX : pos_r, 0);  // row 0 of the warp
     float m_used = -INFINITY, l = 0.f;
     for (int j = 0; j < ntiles; ++j) {
-      const int s = j & 1;
-      const uint32_t ph = (j >> 1) & 1;
-      mbar_wait(&s_full[s], ph);
+      mbar_wait(s_full, j & 1);
       tc_fence_after();
-      const uint32_t s_addr = lane_base + (s ? C::kColS1 : C::kColS0);
       const int key0 = j * C::kKeys;
-      // pass 1: row max of the masked, log2-scaled scores
+      // masking only where a key of this tile can exceed a row's position
+      const bool masked = __any_sync(0xffffffffu, key0 + C::kKeys - 1 > (pos_r < 0 ? -1 : pos_r)) ||
+                          warp_min_pos == INT_MAX;
+      // pass 1: row max of the raw scores (scaled afterwards; the scale is positive)
       float mx = -INFINITY;
 #pragma unroll
       for (int c = 0; c < C::kKeys / 32; ++c) {
@@ -238,19 +233,24 @@ __global__ void __launch_bounds__(kFaThreads, 1)
         tmem_ld32x32b_x16(s_addr + c * 32, *reinterpret_cast<uint32_t(*)[16]>(&r[0]));
         tmem_ld32x32b_x16(s_addr + c * 32 + 16, *reinterpret_cast<uint32_t(*)[16]>(&r[16]));
         tmem_ld_wait();
+        if (masked) {
 #pragma unroll
-        for (int i = 0; i < 32; ++i)
-          if (key0 + c * 32 + i <= pos_r) mx = fmaxf(mx, __uint_as_float(r[i]) * p.scale_log2);
+          for (int i = 0; i < 32; ++i)
+            if (key0 + c * 32 + i <= pos_r) mx = fmaxf(mx, __uint_as_float(r[i]));
+        } else {
+#pragma unroll
+          for (int i = 0; i < 32; ++i) mx = fmaxf(mx, __uint_as_float(r[i]));
+        }
       }
+      mx *= p.scale_log2;
       // lazy rescale: keep the previous max unless the new one exceeds it by > 8 (P <= 2^8)
       const bool rescale = mx > m_used + 8.f;
       const float m_new = rescale ? mx : m_used;
-      const float alpha = (rescale && m_used != -INFINITY) ? exp2f(m_used - m_new) : 1.f;
+      const float alpha = (rescale && m_used != -INFINITY) ? ex2(m_used - m_new) : 1.f;
       const float mb = (m_new == -INFINITY) ? 0.f : m_new;
-      // pass 2: P = 2^(s - m) and the row sum; P is written as two bf16 terms (P = P_hi + P_lo,
+      // pass 2: P = 2^(s*scale - m) and the row sum; P written as two bf16 terms (P_hi + P_lo,
       // exact to ~2^-16 so the fp32 P.V meets the 2e-3 attention bar) over the 32 S columns each
-      // chunk has just read: columns [32c, 32c+16) = P_hi, [32c+16, 32c+32) = P_lo of keys
-      // 32c .. 32c+31, bf16 pairs packed in 32-bit columns.
+      // chunk has just read: [32c, 32c+16) = P_hi, [32c+16, 32c+32) = P_lo of keys 32c..32c+31.
       float sum = 0.f;
 #pragma unroll
       for (int c = 0; c < C::kKeys / 32; ++c) {
@@ -261,9 +261,13 @@ __global__ void __launch_bounds__(kFaThreads, 1)
         uint32_t hi[16], lo[16];
 #pragma unroll
         for (int i = 0; i < 16; ++i) {
-          const int k = key0 + c * 32 + 2 * i;
-          const float p0 = (k <= pos_r) ? exp2f(__uint_as_float(r[2 * i]) * p.scale_log2 - mb) : 0.f;
-          const float p1 = (k + 1 <= pos_r) ? exp2f(__uint_as_float(r[2 * i + 1]) * p.scale_log2 - mb) : 0.f;
+          float p0 = ex2(fmaf(__uint_as_float(r[2 * i]), p.scale_log2, -mb));
+          float p1 = ex2(fmaf(__uint_as_float(r[2 * i + 1]), p.scale_log2, -mb));
+          if (masked) {
+            const int k = key0 + c * 32 + 2 * i;
+            p0 = (k <= pos_r) ? p0 : 0.f;
+            p1 = (k + 1 <= pos_r) ? p1 : 0.f;
+          }
           hi[i] = pack_bf16(p0, p1);
           lo[i] = pack_bf16(p0 - bf16_lo(hi[i]), p1 - bf16_hi(hi[i]));
           sum += p0 + p1;
@@ -274,25 +278,25 @@ __global__ void __launch_bounds__(kFaThreads, 1)
       tmem_st_wait();
       l = l * alpha + sum;
       if (j >= 1) {
-        // O holds tiles < j once PV_{j-1} is done; rescale it before PV_j accumulates
+        // PV_{j-1} (issued before QK_j) is complete; rescale O before PV_j accumulates into it
         mbar_wait(o_full, (j - 1) & 1);
         tc_fence_after();
         if (__any_sync(0xffffffffu, alpha != 1.f)) {
 #pragma unroll 1
           for (int c = 0; c < HD / 16; ++c) {
             uint32_t r[16];
-            tmem_ld32x32b_x16(lane_base + C::kColO + c * 16, r);
+            tmem_ld32x32b_x16(o_addr + c * 16, r);
             tmem_ld_wait();
 #pragma unroll
             for (int i = 0; i < 16; ++i) r[i] = __float_as_uint(__uint_as_float(r[i]) * alpha);
-            tmem_st32x32b_x16(lane_base + C::kColO + c * 16, r);
+            tmem_st32x32b_x16(o_addr + c * 16, r);
           }
           tmem_st_wait();
         }
       }
       m_used = m_new;
       tc_fence_before();
-      mbar_arrive(&p_full[s]);
+      mbar_arrive(p_full);
     }
     // epilogue: O / l
     mbar_wait(o_full, (ntiles - 1) & 1);
@@ -301,8 +305,8 @@ __global__ void __launch_bounds__(kFaThreads, 1)
 #pragma unroll 1
     for (int c = 0; c < HD / 32; ++c) {
       uint32_t r[32];
-      tmem_ld32x32b_x16(lane_base + C::kColO + c * 32, *reinterpret_cast<uint32_t(*)[16]>(&r[0]));
-      tmem_ld32x32b_x16(lane_base + C::kColO + c * 32 + 16, *reinterpret_cast<uint32_t(*)[16]>(&r[16]));
+      tmem_ld32x32b_x16(o_addr + c * 32, *reinterpret_cast<uint32_t(*)[16]>(&r[0]));
+      tmem_ld32x32b_x16(o_addr + c * 32 + 16, *reinterpret_cast<uint32_t(*)[16]>(&r[16]));
       tmem_ld_wait();
       if (pos_r >= 0) {
         if (p.out_f32) {
