@@ -169,7 +169,7 @@ QOS_DEV void softmax_step(float (&s)[2][4], float (&m)[2], float (&l)[2], float 
 template <int HD>
 __global__ void __launch_bounds__(kAttnThreads, 3)
     decode_attn_kernel(const __grid_constant__ CUtensorMap kvmap, const AttnParams p, const DecodeItem* __restrict__ items,
-                       float* __restrict__ partials) {
+                       float* __restrict__ partials, int* __restrict__ counters) {
   using C = AttnCfg<HD>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -267,13 +267,13 @@ __global__ void __launch_bounds__(kAttnThreads, 3)
     }
   }
   __syncthreads();
-  float* part = partials + size_t(it.part) * group * (HD + 2);
-  for (int idx = threadIdx.x; idx < group * HD; idx += blockDim.x) {
-    const int r = idx / HD, d = idx % HD;
-    float M = -INFINITY;
+  // merge the 4 warps: (M, L, acc) per (row r < group, dim d)
+  auto merged = [&](int r, int d, float& M, float& L) {
+    M = -INFINITY;
 #pragma unroll
     for (int w = 0; w < kConsumerWarps; ++w) M = fmaxf(M, sm[w * 16 + r]);
-    float acc = 0.f, L = 0.f;
+    float acc = 0.f;
+    L = 0.f;
 #pragma unroll
     for (int w = 0; w < kConsumerWarps; ++w) {
       const float mw = sm[w * 16 + r];
@@ -281,39 +281,59 @@ __global__ void __launch_bounds__(kAttnThreads, 3)
       acc += f * so[(w * 16 + r) * HD + d];
       L += f * sl[w * 16 + r];
     }
+    return acc;
+  };
+  auto store_out = [&](int r, int d, float v) {
+    const size_t off = size_t(it.row) * p.out_ld + size_t(it.kv_head * group + r) * HD + d;
+    if (p.out_f32)
+      reinterpret_cast<float*>(p.out)[off] = v;
+    else
+      reinterpret_cast<__nv_bfloat16*>(p.out)[off] = __float2bfloat16_rn(v);
+  };
+  if (it.nsplit == 1) {  // the whole key range in one item: normalise and store
+    for (int idx = threadIdx.x; idx < group * HD; idx += blockDim.x) {
+      float M, L;
+      const float acc = merged(idx / HD, idx % HD, M, L);
+      store_out(idx / HD, idx % HD, acc / L);
+    }
+    return;
+  }
+  float* part = partials + size_t(it.part) * group * (HD + 2);
+  for (int idx = threadIdx.x; idx < group * HD; idx += blockDim.x) {
+    const int r = idx / HD, d = idx % HD;
+    float M, L;
+    const float acc = merged(r, d, M, L);
     part[r * (HD + 2) + d] = acc;
     if (d == 0) {
       part[r * (HD + 2) + HD] = M;
       part[r * (HD + 2) + HD + 1] = L;
     }
   }
-}
-
-// merge the splits of one (decode row, q head): out = sum_s 2^(m_s - M) o_s / sum_s 2^(m_s - M) l_s
-template <int HD>
-__global__ void decode_combine_kernel(const AttnParams p, const DecodeRow* __restrict__ rows,
-                                      const float* __restrict__ partials) {
-  const DecodeRow dr = rows[blockIdx.x];
-  const int group = p.H / p.Hkv;
-  const int hq = blockIdx.y;  // q head
-  const int kvh = hq / group, r = hq % group;
-  const float* base = partials + size_t(dr.part0 + kvh * dr.nsplit) * group * (HD + 2) + r * (HD + 2);
+  // split-K combine fused into the last finishing item of this (decode row, kv head):
+  // out = sum_s 2^(m_s - M) o_s / sum_s 2^(m_s - M) l_s   (LSE merge)
+  __threadfence();
+  __syncthreads();
+  __shared__ int s_last;
+  if (threadIdx.x == 0) s_last = (atomicAdd(counters + it.counter, 1) == it.nsplit - 1);
+  __syncthreads();
+  if (!s_last) return;
+  __threadfence();
   const size_t stride = size_t(group) * (HD + 2);
-  float M = -INFINITY;
-  for (int s = 0; s < dr.nsplit; ++s) M = fmaxf(M, base[s * stride + HD]);
-  float L = 0.f;
-  for (int s = 0; s < dr.nsplit; ++s) L += exp2f(base[s * stride + HD] - M) * base[s * stride + HD + 1];
-  const float inv = 1.f / L;
-  for (int d = threadIdx.x; d < HD; d += blockDim.x) {
-    float acc = 0.f;
-    for (int s = 0; s < dr.nsplit; ++s) acc += exp2f(base[s * stride + HD] - M) * base[s * stride + d];
-    acc *= inv;
-    const size_t off = size_t(dr.row) * p.out_ld + size_t(hq) * HD + d;
-    if (p.out_f32)
-      reinterpret_cast<float*>(p.out)[off] = acc;
-    else
-      reinterpret_cast<__nv_bfloat16*>(p.out)[off] = __float2bfloat16_rn(acc);
+  const float* pb = partials + size_t(it.part_base) * stride;
+  for (int idx = threadIdx.x; idx < group * HD; idx += blockDim.x) {
+    const int r = idx / HD, d = idx % HD;
+    float M = -INFINITY;
+    for (int s2 = 0; s2 < it.nsplit; ++s2) M = fmaxf(M, __ldcg(pb + s2 * stride + r * (HD + 2) + HD));
+    float L = 0.f, acc = 0.f;
+    for (int s2 = 0; s2 < it.nsplit; ++s2) {
+      const float* ps = pb + s2 * stride + r * (HD + 2);
+      const float f = exp2f(__ldcg(ps + HD) - M);
+      L += f * __ldcg(ps + HD + 1);
+      acc += f * __ldcg(ps + d);
+    }
+    store_out(r, d, acc / L);
   }
+  if (threadIdx.x == 0) counters[it.counter] = 0;  // ready for the next layer
 }
 
 // ------------------------------------------------------------------------------ prefill
@@ -444,8 +464,8 @@ static AttnParams to_params(const AttnLaunch& a) {
 int prefill_positions_per_tile(int group) { return kConsumerWarps * (16 / group); }
 
 template <int HD>
-static cudaError_t decode_t(const AttnLaunch& a, const DecodeItem* items, int n_items, const DecodeRow* rows,
-                            int n_rows, float* partials, cudaStream_t st) {
+static cudaError_t decode_t(const AttnLaunch& a, const DecodeItem* items, int n_items, float* partials, int* counters,
+                            cudaStream_t st) {
   static bool set = false;
   if (!set) {
     cudaError_t e = cudaFuncSetAttribute(decode_attn_kernel<HD>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -454,19 +474,17 @@ static cudaError_t decode_t(const AttnLaunch& a, const DecodeItem* items, int n_
     set = true;
   }
   AttnParams p = to_params(a);
-  decode_attn_kernel<HD><<<n_items, kAttnThreads, AttnCfg<HD>::kSmemBytes, st>>>(*a.kv_tmap, p, items, partials);
-  cudaError_t e = cudaGetLastError();
-  if (e != cudaSuccess) return e;
-  decode_combine_kernel<HD><<<dim3(n_rows, a.H), 64, 0, st>>>(p, rows, partials);
+  decode_attn_kernel<HD><<<n_items, kAttnThreads, AttnCfg<HD>::kSmemBytes, st>>>(*a.kv_tmap, p, items, partials,
+                                                                                  counters);
   return cudaGetLastError();
 }
 
-cudaError_t launch_decode_attention(const AttnLaunch& a, const DecodeItem* items, int n_items, const DecodeRow* rows,
-                                    int n_rows, float* partials, int /*max_splits*/, cudaStream_t st) {
+cudaError_t launch_decode_attention(const AttnLaunch& a, const DecodeItem* items, int n_items, float* partials,
+                                    int* counters, cudaStream_t st) {
   if (n_items == 0) return cudaSuccess;
-  count_launch(2);
-  if (a.hd == 128) return decode_t<128>(a, items, n_items, rows, n_rows, partials, st);
-  if (a.hd == 64) return decode_t<64>(a, items, n_items, rows, n_rows, partials, st);
+  count_launch(1);
+  if (a.hd == 128) return decode_t<128>(a, items, n_items, partials, counters, st);
+  if (a.hd == 64) return decode_t<64>(a, items, n_items, partials, counters, st);
   return cudaErrorInvalidValue;
 }
 

@@ -138,7 +138,7 @@ static WeightLayout weight_layout(const qos_model_cfg& c, const Shard& s) {
 }
 
 struct WsLayout {
-  size_t resid, h, qkv, attn, act, hR, logits, logits_loc, argmax, partials, meta[2], dbg, total;
+  size_t resid, h, qkv, attn, act, hR, logits, logits_loc, argmax, partials, counters, meta[2], dbg, total;
   size_t meta_bytes;
   int max_items;
 };
@@ -165,11 +165,12 @@ static WsLayout ws_layout(const qos_model_cfg& c, const Shard& s, int tp) {
   w.argmax = take(Rm * 4);
   w.max_items = kMaxDecodeItems;
   w.partials = take(size_t(w.max_items) * group * (hd + 2) * 4);
+  w.counters = take(Rm * size_t(s.Hkv) * 4);
   // metadata: tokens, pos, slot [Tm]; logit rows [Rm]; prefill items; decode items/rows; table updates
   const int ppt = prefill_tc_positions_per_tile(int(group));
   const size_t max_pitems = (Tm / ppt + Rm + 1) * size_t(s.Hkv);
   w.meta_bytes = align_up(3 * Tm * 4 + Rm * 4 + 64, 256) + align_up(max_pitems * sizeof(PrefillItem), 256) +
-                 align_up(size_t(w.max_items) * sizeof(DecodeItem), 256) + align_up(Rm * sizeof(DecodeRow), 256) +
+                 align_up(size_t(w.max_items) * sizeof(DecodeItem), 256) +
                  align_up(size_t(3) * 65536 * 4, 256);
   w.meta[0] = take(w.meta_bytes);
   w.meta[1] = take(w.meta_bytes);
@@ -181,9 +182,9 @@ static WsLayout ws_layout(const qos_model_cfg& c, const Shard& s, int tp) {
 // ------------------------------------------------------------------ batch metadata (a1)
 struct StepMeta {
   int T = 0, R = 0, n_prefill = 0, n_decode = 0;
-  int n_pitems = 0, n_ditems = 0, n_drows = 0, n_upd = 0;
+  int n_pitems = 0, n_ditems = 0, n_upd = 0;
   // offsets (bytes) inside the metadata block
-  size_t o_tok, o_pos, o_slot, o_rows, o_pitems, o_ditems, o_drows, o_upd, used;
+  size_t o_tok, o_pos, o_slot, o_rows, o_pitems, o_ditems, o_upd, used;
 };
 
 struct ReqState {
@@ -423,7 +424,6 @@ int build_step(qos_engine* e, const qos_batch* b, bool check_lengths, uint8_t* b
     while (count_items(split) > e->wsl.max_items) split *= 2;
   }
   std::vector<DecodeItem> ditems;
-  std::vector<DecodeRow> drows;
   int part = 0;
   for (int i = 0; i < b->n_decode; ++i) {
     const auto& dc = b->decode[i];
@@ -437,11 +437,6 @@ int build_step(qos_engine* e, const qos_batch* b, bool check_lengths, uint8_t* b
     rows[b->n_prefill + i] = t;
     const int keys = p + 1;
     const int nsplit = (keys + split - 1) / split;
-    DecodeRow dr;
-    dr.row = t;
-    dr.part0 = part;
-    dr.nsplit = nsplit;
-    drows.push_back(dr);
     for (int h = 0; h < e->sh.Hkv; ++h)
       for (int s = 0; s < nsplit; ++s) {
         DecodeItem it;
@@ -450,7 +445,10 @@ int build_step(qos_engine* e, const qos_batch* b, bool check_lengths, uint8_t* b
         it.kv_head = h;
         it.key0 = s * split;
         it.key1 = std::min(keys, (s + 1) * split);
-        it.part = part + h * nsplit + s;
+        it.part_base = part + h * nsplit;
+        it.part = it.part_base + s;
+        it.nsplit = nsplit;
+        it.counter = i * e->sh.Hkv + h;
         ditems.push_back(it);
       }
     part += e->sh.Hkv * nsplit;
@@ -461,10 +459,8 @@ int build_step(qos_engine* e, const qos_batch* b, bool check_lengths, uint8_t* b
                    [](const DecodeItem& a, const DecodeItem& b2) { return a.key1 - a.key0 > b2.key1 - b2.key0; });
   m.n_pitems = int(pitems.size());
   m.n_ditems = int(ditems.size());
-  m.n_drows = int(drows.size());
   m.o_pitems = take(pitems.size() * sizeof(PrefillItem));
   m.o_ditems = take(ditems.size() * sizeof(DecodeItem));
-  m.o_drows = take(drows.size() * sizeof(DecodeRow));
   const size_t max_upd = 65536;
   m.n_upd = int(std::min(e->pending_upd.size() / 3, max_upd));
   m.o_upd = take(size_t(m.n_upd) * 12);
@@ -472,7 +468,6 @@ int build_step(qos_engine* e, const qos_batch* b, bool check_lengths, uint8_t* b
   if (m.used > e->wsl.meta_bytes) return set_error(QOS_ERR_INVALID_ARG, "metadata exceeds workspace");
   if (!pitems.empty()) memcpy(buf + m.o_pitems, pitems.data(), pitems.size() * sizeof(PrefillItem));
   if (!ditems.empty()) memcpy(buf + m.o_ditems, ditems.data(), ditems.size() * sizeof(DecodeItem));
-  if (!drows.empty()) memcpy(buf + m.o_drows, drows.data(), drows.size() * sizeof(DecodeRow));
   if (m.n_upd) memcpy(buf + m.o_upd, e->pending_upd.data(), size_t(m.n_upd) * 12);
   (void)out_rows_tables;
   return QOS_OK;
@@ -608,8 +603,8 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
     if (m.n_ditems) {
       TimerScope ts(e, QOS_T_DECODE_ATTN, st);
       QOS_CU(launch_decode_attention(al, reinterpret_cast<const DecodeItem*>(dm + m.o_ditems), m.n_ditems,
-                                     reinterpret_cast<const DecodeRow*>(dm + m.o_drows), m.n_drows,
-                                     reinterpret_cast<float*>(e->ws + s.partials), 0, st));
+                                     reinterpret_cast<float*>(e->ws + s.partials),
+                                     reinterpret_cast<int*>(e->ws + s.counters), st));
     }
     if (overlap) {
       QOS_CU(cudaEventRecord(e->ev_join, e->side));
@@ -818,6 +813,9 @@ int qos_engine_create(const qos_model_cfg* cfg, int device, int tp_rank, int tp_
   // zero the KV pool once: slots past a request's length are read (with P = 0) by the attention
   // tiles, and 0 * NaN from uninitialised memory would poison the accumulators
   if (cudaMemset(e->kv, 0, e->kv_bytes) != cudaSuccess) return fail(set_error(QOS_ERR_CUDA, "kv memset"));
+  // split-K arrival counters start at zero; the combining item resets its counter
+  if (cudaMemset(e->ws + e->wsl.counters, 0, size_t(cfg->max_batch_rows) * e->sh.Hkv * 4) != cudaSuccess)
+    return fail(set_error(QOS_ERR_CUDA, "counter memset"));
   if (cudaMalloc(&e->d_tables, size_t(cfg->max_requests) * e->table_w * 4) != cudaSuccess)
     return fail(set_error(QOS_ERR_OOM, "block tables"));
   cudaMemset(e->d_tables, 0, size_t(cfg->max_requests) * e->table_w * 4);
@@ -1335,8 +1333,8 @@ int qos_op_attention(qos_engine_t* e, int32_t layer, const qos_batch* b, const u
   al.scale_log2 = float(1.4426950408889634 / std::sqrt(double(hd)));
   QOS_CU(launch_prefill_attention_tc(al, reinterpret_cast<const PrefillItem*>(dm + m.o_pitems), m.n_pitems, st));
   QOS_CU(launch_decode_attention(al, reinterpret_cast<const DecodeItem*>(dm + m.o_ditems), m.n_ditems,
-                                 reinterpret_cast<const DecodeRow*>(dm + m.o_drows), m.n_drows,
-                                 reinterpret_cast<float*>(e->ws + e->wsl.partials), 0, st));
+                                 reinterpret_cast<float*>(e->ws + e->wsl.partials),
+                                 reinterpret_cast<int*>(e->ws + e->wsl.counters), st));
   QOS_CU(cudaMemcpyAsync(out, o, size_t(m.T) * qrow * 4, cudaMemcpyDeviceToHost, st));
   QOS_TRY(release_staging(e, st));
   QOS_CU(cudaStreamSynchronize(st));

@@ -74,12 +74,10 @@ struct DecodeItem {      // one split-K work item: (decode row, kv head, key ran
   int32_t table;         // block-table row (device) of the request
   int32_t kv_head;       // local kv head
   int32_t key0, key1;    // key range [key0, key1)
-  int32_t part;          // partial slot index
-};
-struct DecodeRow {       // combine descriptor of one decode row
-  int32_t row;
-  int32_t part0;         // first partial slot of kv head 0; heads follow (nsplit each)
-  int32_t nsplit;
+  int32_t part;          // partial slot of this item
+  int32_t part_base;     // first partial slot of this (row, kv head); its splits follow
+  int32_t nsplit;        // splits of this (row, kv head); 1 = no partial, store directly
+  int32_t counter;       // arrival counter of this (row, kv head) for the fused combine
 };
 struct PrefillItem {     // one (chunk, q-tile, kv head) work item
   int32_t row0;          // first token row of the tile
@@ -103,8 +101,8 @@ struct AttnLaunch {
   int table_w;
   float scale_log2;       // log2(e) / sqrt(hd)
 };
-cudaError_t launch_decode_attention(const AttnLaunch& a, const DecodeItem* items, int n_items, const DecodeRow* rows,
-                                    int n_rows, float* partials, int max_splits, cudaStream_t st);
+cudaError_t launch_decode_attention(const AttnLaunch& a, const DecodeItem* items, int n_items, float* partials,
+                                    int* counters, cudaStream_t st);
 cudaError_t launch_prefill_attention(const AttnLaunch& a, const PrefillItem* items, int n_items, cudaStream_t st);
 int prefill_positions_per_tile(int group);
 cudaError_t launch_prefill_attention_tc(const AttnLaunch& a, const PrefillItem* items, int n_items, cudaStream_t st);
