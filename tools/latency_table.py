@@ -1,0 +1,106 @@
+"""configs[1] latency table + predictability test (north star: "iteration
+latency must be predictable to within 5% of the profiled model across chunk sizes 256-8192").
+
+  python tools/latency_table.py --out gpurun_out/latency_table.json [--test 200] [--layers 32]
+
+1. profiles a grid of (chunk, n_decode, ctx, kv_start) points with qos_profile_step (device-timed
+   median of `reps` steps after 3 warm-ups);
+2. fits paper_conf_asplos_goelmkar26_b200.latency_model on them;
+3. measures `--test` random heterogeneous batches (chunk ~ U[256, 8192], n_dec ~ U[0, 256],
+   ctx_j ~ U[1k, 8k], kv_start ~ U[0, 4096], subject to the KV capacity mask) and reports
+   |measured - predicted| / measured (max, p95), plus the Fig. 4-style throughput curve.
+"""
+import argparse
+import json
+import os
+import sys
+import time
+
+import numpy as np
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+from paper_conf_asplos_goelmkar26_b200 import qoserve as q  # noqa: E402
+from paper_conf_asplos_goelmkar26_b200.latency_model import LatencyModel, StepShape  # noqa: E402
+from paper_conf_asplos_goelmkar26_b200.presets import preset  # noqa: E402
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--out", default="gpurun_out/latency_table.json")
+    ap.add_argument("--test", type=int, default=200)
+    ap.add_argument("--reps", type=int, default=5)
+    ap.add_argument("--layers", type=int, default=None)
+    ap.add_argument("--kv-gb", type=float, default=140.0)
+    a = ap.parse_args()
+    import torch
+    torch.cuda.set_device(0)
+    over = {} if a.layers is None else {"n_layers": a.layers}
+    p = preset("llama3-8b", **over)
+    per_tok = p["n_layers"] * 2 * p["n_kv_heads"] * p["head_dim"] * 2
+    num_blocks = int(a.kv_gb * 1e9 / (per_tok * 16))
+    cap_tokens = num_blocks * 16 - 16 * 600
+    cfg = q.model_cfg(**p, num_blocks=num_blocks, max_seq_len=16384, max_requests=300,
+                      max_batch_tokens=8192 + 256, max_batch_rows=257)
+    eng = q.Engine(cfg)
+    eng.qos_engine_load_synthetic(0)
+    rng = np.random.default_rng(3)
+    t0 = time.time()
+
+    def prof(chunk, ctx, kv_start=0):
+        ms, p95 = eng.qos_profile_step(chunk, ctx, reps=a.reps, kv_start=kv_start)
+        return ms, p95
+
+    fit_shapes, fit_ms, table = [], [], []
+    for ctx in (1024, 4096):
+        for nd in (0, 32, 128, 256):
+            if nd * (ctx + 1) > cap_tokens:
+                continue
+            for chunk in (0, 256, 512, 1024, 1536, 2048, 3072, 4096, 6144, 8192):
+                if chunk == 0 and nd == 0:
+                    continue
+                ms, p95 = prof(chunk, [ctx] * nd)
+                s = StepShape([(0, chunk)] if chunk else [], [ctx] * nd)
+                fit_shapes.append(s)
+                fit_ms.append(ms)
+                table.append({"chunk": chunk, "n_decode": nd, "ctx": ctx, "kv_start": 0, "ms": ms, "p95_ms": p95,
+                              "tokens_per_s": s.T / (ms * 1e-3)})
+    for chunk in (256, 1024, 2048, 4096):
+        for nd in (0, 128):
+            ms, p95 = prof(chunk, [2048] * nd, kv_start=4096)
+            s = StepShape([(4096, chunk)], [2048] * nd)
+            fit_shapes.append(s)
+            fit_ms.append(ms)
+            table.append({"chunk": chunk, "n_decode": nd, "ctx": 2048, "kv_start": 4096, "ms": ms, "p95_ms": p95,
+                          "tokens_per_s": s.T / (ms * 1e-3)})
+    model = LatencyModel().fit(fit_shapes, fit_ms)
+    fit_err = [abs(model.predict(s) - m) / m for s, m in zip(fit_shapes, fit_ms)]
+    tests = []
+    for _ in range(a.test):
+        chunk = int(rng.integers(256, 8193))
+        nd = int(rng.integers(0, 257))
+        ks = int(rng.integers(0, 4097))
+        ctx = rng.integers(1024, 8193, size=nd)
+        while ctx.sum() + nd > cap_tokens:
+            ctx = ctx[: max(0, len(ctx) - 8)]
+        ctx = [int(c) for c in ctx]
+        ms, p95 = prof(chunk, ctx, kv_start=ks)
+        s = StepShape([(ks, chunk)], ctx)
+        pred = model.predict(s)
+        tests.append({"chunk": chunk, "kv_start": ks, "n_decode": len(ctx), "sum_ctx": int(sum(ctx)), "ms": ms,
+                      "pred_ms": pred, "rel_err": abs(pred - ms) / ms})
+    errs = np.array([t["rel_err"] for t in tests]) if tests else np.zeros(1)
+    out = {"model": "llama3-8b" + (f" (L={a.layers})" if a.layers else ""), "reps": a.reps,
+           "kv_capacity_tokens": cap_tokens, "fit_points": len(fit_ms),
+           "fit_rel_err_max": float(max(fit_err)), "test_points": len(tests),
+           "test_rel_err_max": float(errs.max()), "test_rel_err_p95": float(np.percentile(errs, 95)),
+           "test_rel_err_mean": float(errs.mean()), "within_5pct": float((errs <= 0.05).mean()),
+           "seconds": time.time() - t0, "model_json": json.loads(model.to_json()), "table": table, "tests": tests}
+    os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
+    json.dump(out, open(a.out, "w"), indent=1)
+    print(json.dumps({k: v for k, v in out.items() if k not in ("table", "tests", "model_json")}))
+    eng.close()
+
+
+if __name__ == "__main__":
+    main()
