@@ -31,6 +31,12 @@ enum {
  * M may be any value >= 1.  Stream-ordered. */
 int qos_op_gemm(const void* A, const void* B, void* C, int64_t M, int64_t N, int64_t K, int epi,
                 const float* bias, void* stream);
+/* Same with an explicit split-K factor (0 = the engine's automatic choice, 1 = no split).
+ * Split-K (weight-bound small-M GEMMs): each of `ksplit` CTAs accumulates a K slice of a tile,
+ * parks an fp32 partial, and the last one to arrive sums the slices in slice order and applies
+ * the epilogue (deterministic). */
+int qos_op_gemm_ex(const void* A, const void* B, void* C, int64_t M, int64_t N, int64_t K, int epi,
+                   const float* bias, int ksplit, void* stream);
 
 /* a3: out[t][:] = bf16( x[t][:] / sqrt(mean(x[t]^2) + eps) * g[:] ), x device f32 [T][d],
  * g device bf16 [d], out device bf16 [T][d].  Stream-ordered. */

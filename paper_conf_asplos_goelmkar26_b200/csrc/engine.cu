@@ -138,11 +138,14 @@ static WeightLayout weight_layout(const qos_model_cfg& c, const Shard& s) {
 }
 
 struct WsLayout {
-  size_t resid, h, qkv, attn, act, hR, logits, logits_loc, argmax, partials, counters, meta[2], dbg, total;
+  size_t resid, h, qkv, attn, act, hR, logits, logits_loc, argmax, partials, counters, gemm_part, gemm_cnt, meta[2], dbg,
+      total;
   size_t meta_bytes;
   int max_items;
 };
 static constexpr int kMaxDecodeItems = 1 << 16;
+static constexpr int kGemmMaxUnits = 512;   // split-K partial slots (128 x 256 fp32 each)
+static constexpr int kGemmMaxTiles = 4096;  // split-K arrival counters
 static WsLayout ws_layout(const qos_model_cfg& c, const Shard& s, int tp) {
   WsLayout w;
   size_t off = 0;
@@ -166,6 +169,8 @@ static WsLayout ws_layout(const qos_model_cfg& c, const Shard& s, int tp) {
   w.max_items = kMaxDecodeItems;
   w.partials = take(size_t(w.max_items) * group * (hd + 2) * 4);
   w.counters = take(Rm * size_t(s.Hkv) * 4);
+  w.gemm_part = take(size_t(kGemmMaxUnits) * 128 * 256 * 4);
+  w.gemm_cnt = take(size_t(kGemmMaxTiles) * 4);
   // metadata: tokens, pos, slot [Tm]; logit rows [Rm]; prefill items; decode items/rows; table updates
   const int ppt = prefill_tc_positions_per_tile(int(group));
   const size_t max_pitems = (Tm / ppt + Rm + 1) * size_t(s.Hkv);
@@ -229,6 +234,7 @@ struct qos_engine {
   cudaStream_t side = nullptr;    // high-priority stream: prefill attention overlapped with decode
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
   bool overlap_attn = true;       // QOS_OVERLAP_ATTN=0 serialises a7 and a8 (for measurement)
+  bool gemm_splitk = true;        // QOS_GEMM_SPLITK=0 disables split-K for small-M GEMMs
   // timing
   bool timing = false;
   std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> tev;
@@ -517,8 +523,10 @@ int flush_table_updates(qos_engine* e, cudaStream_t st) {
 int gemm(qos_engine* e, const CUtensorMap& ta, const CUtensorMap (&tb)[2], int64_t M, int64_t N, int64_t K, int epi,
          void* C, int64_t ldc, const float* bias, cudaStream_t st) {
   const int bn = gemm_pick_bn(M, N, epi, e->num_sms);
+  const int ks = e->gemm_splitk ? gemm_pick_ksplit(M, N, K, bn, e->num_sms, kGemmMaxUnits) : 1;
   count_launch();
-  return gemm_run(ta, tb[bn == 256 ? 1 : 0], bn, M, N, K, epi, C, ldc, bias, e->num_sms, st);
+  return gemm_run(ta, tb[bn == 256 ? 1 : 0], bn, M, N, K, epi, C, ldc, bias, e->num_sms, st, ks,
+                  reinterpret_cast<float*>(e->ws + e->wsl.gemm_part), reinterpret_cast<int*>(e->ws + e->wsl.gemm_cnt));
 }
 
 int allreduce_bf16(qos_engine* e, void* buf, size_t count, cudaStream_t st) {
@@ -813,8 +821,9 @@ int qos_engine_create(const qos_model_cfg* cfg, int device, int tp_rank, int tp_
   // zero the KV pool once: slots past a request's length are read (with P = 0) by the attention
   // tiles, and 0 * NaN from uninitialised memory would poison the accumulators
   if (cudaMemset(e->kv, 0, e->kv_bytes) != cudaSuccess) return fail(set_error(QOS_ERR_CUDA, "kv memset"));
-  // split-K arrival counters start at zero; the combining item resets its counter
-  if (cudaMemset(e->ws + e->wsl.counters, 0, size_t(cfg->max_batch_rows) * e->sh.Hkv * 4) != cudaSuccess)
+  // split-K arrival counters start at zero; the combining item / reducing CTA resets its counter
+  if (cudaMemset(e->ws + e->wsl.counters, 0, size_t(cfg->max_batch_rows) * e->sh.Hkv * 4) != cudaSuccess ||
+      cudaMemset(e->ws + e->wsl.gemm_cnt, 0, size_t(kGemmMaxTiles) * 4) != cudaSuccess)
     return fail(set_error(QOS_ERR_CUDA, "counter memset"));
   if (cudaMalloc(&e->d_tables, size_t(cfg->max_requests) * e->table_w * 4) != cudaSuccess)
     return fail(set_error(QOS_ERR_OOM, "block tables"));
@@ -839,6 +848,7 @@ int qos_engine_create(const qos_model_cfg* cfg, int device, int tp_rank, int tp_
   }
   cudaStreamCreateWithFlags(&e->stream, cudaStreamNonBlocking);
   if (const char* ov = getenv("QOS_OVERLAP_ATTN")) e->overlap_attn = atoi(ov) != 0;
+  if (const char* sk = getenv("QOS_GEMM_SPLITK")) e->gemm_splitk = atoi(sk) != 0;
   {
     int lo = 0, hi = 0;
     cudaDeviceGetStreamPriorityRange(&lo, &hi);
@@ -1207,20 +1217,41 @@ int qos_engine_launch_count(qos_engine_t* e, int64_t* out) {
 }
 
 // ------------------------------------------------------------------ kernel-level ops
-int qos_op_gemm(const void* A, const void* B, void* C, int64_t M, int64_t N, int64_t K, int epi, const float* bias,
-                void* stream) {
+static int op_gemm(const void* A, const void* B, void* C, int64_t M, int64_t N, int64_t K, int epi, const float* bias,
+                   int ksplit, void* stream) {
   if (!A || !B || !C || (epi == QOS_EPI_BIAS_BF16 && !bias)) return set_error(QOS_ERR_INVALID_ARG, "gemm pointers");
   QOS_TRY(gemm_check_shape(M, N, K, epi));
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   const int bn = gemm_pick_bn(M, N, epi, sms);
+  static float* part = nullptr;  // process-wide split-K workspace of the op entry point
+  static int* cnt = nullptr;
+  if (!part) {
+    if (cudaMalloc(&part, size_t(kGemmMaxUnits) * 128 * 256 * 4) != cudaSuccess ||
+        cudaMalloc(&cnt, size_t(kGemmMaxTiles) * 4) != cudaSuccess || cudaMemset(cnt, 0, size_t(kGemmMaxTiles) * 4))
+      return set_error(QOS_ERR_OOM, "gemm split-K workspace");
+  }
+  const int64_t tiles = ((M + 127) / 128) * ((N + bn - 1) / bn);
+  int ks = ksplit <= 0 ? gemm_pick_ksplit(M, N, K, bn, sms, kGemmMaxUnits) : ksplit;
+  if (ks > 1 && (tiles > kGemmMaxTiles || tiles * ks > kGemmMaxUnits || (K / 64) < ks))
+    return set_error(QOS_ERR_INVALID_ARG, "gemm: ksplit too large for the shape / workspace");
   CUtensorMap ta, tb;
   QOS_TRY(make_tmap_2d_bf16(&ta, A, uint64_t(M), uint64_t(K), uint64_t(K), 128, 64, true));
   QOS_TRY(make_tmap_2d_bf16(&tb, B, uint64_t(N), uint64_t(K), uint64_t(K), uint32_t(bn), 64, true));
   const int64_t ldc = epi == QOS_EPI_SILU_GATE ? N / 2 : N;
   count_launch();
-  return gemm_run(ta, tb, bn, M, N, K, epi, C, ldc, bias, sms, reinterpret_cast<cudaStream_t>(stream));
+  return gemm_run(ta, tb, bn, M, N, K, epi, C, ldc, bias, sms, reinterpret_cast<cudaStream_t>(stream), ks, part, cnt);
+}
+
+int qos_op_gemm(const void* A, const void* B, void* C, int64_t M, int64_t N, int64_t K, int epi, const float* bias,
+                void* stream) {
+  return op_gemm(A, B, C, M, N, K, epi, bias, 0, stream);
+}
+
+int qos_op_gemm_ex(const void* A, const void* B, void* C, int64_t M, int64_t N, int64_t K, int epi, const float* bias,
+                   int ksplit, void* stream) {
+  return op_gemm(A, B, C, M, N, K, epi, bias, ksplit, stream);
 }
 
 int qos_op_rmsnorm(const float* x, const void* g, void* out, int32_t T, int32_t d, float eps, void* stream) {

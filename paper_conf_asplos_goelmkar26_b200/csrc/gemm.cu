@@ -40,10 +40,65 @@ struct GemmCfg {
 struct GemmArgs {
   int M, N, K;
   int mt, nt;       // tiles along M and N
+  int ksplit;       // K slices per tile (split-K for weight-bound small-M GEMMs); 1 = off
   void* C;
   int ldc;          // elements
   const float* bias;
+  float* part;      // split-K partials [unit][128][BN] fp32 (ksplit > 1)
+  int* counters;    // split-K arrival counter per tile (ksplit > 1), zero between launches
 };
+
+// ---- epilogue stores of one thread's 32 consecutive accumulator columns of one row
+template <int EPI>
+QOS_DEV void epi_store32(const GemmArgs& p, int row, int col, const float (&v)[32]) {
+  if constexpr (EPI == EPI_STORE_BF16 || EPI == EPI_BIAS_BF16) {
+    uint32_t pk[16];
+#pragma unroll
+    for (int i = 0; i < 16; ++i) {
+      float a0 = v[2 * i], a1 = v[2 * i + 1];
+      if constexpr (EPI == EPI_BIAS_BF16) {
+        a0 += __ldg(p.bias + col + 2 * i);
+        a1 += __ldg(p.bias + col + 2 * i + 1);
+      }
+      pk[i] = pack_bf16(a0, a1);
+    }
+    uint4* dst = reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.C) + size_t(row) * p.ldc + col);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) dst[i] = make_uint4(pk[4 * i], pk[4 * i + 1], pk[4 * i + 2], pk[4 * i + 3]);
+  } else if constexpr (EPI == EPI_STORE_F32) {
+    float4* dst = reinterpret_cast<float4*>(reinterpret_cast<float*>(p.C) + size_t(row) * p.ldc + col);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) dst[i] = make_float4(v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
+  } else if constexpr (EPI == EPI_ADD_F32) {
+    float4* dst = reinterpret_cast<float4*>(reinterpret_cast<float*>(p.C) + size_t(row) * p.ldc + col);
+    float4 old[8];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) old[i] = dst[i];
+#pragma unroll
+    for (int i = 0; i < 8; ++i)
+      dst[i] = make_float4(old[i].x + v[4 * i], old[i].y + v[4 * i + 1], old[i].z + v[4 * i + 2], old[i].w + v[4 * i + 3]);
+  }
+}
+// SiLU-gate: 32 gate columns + the 32 matching up columns -> 32 output columns
+QOS_DEV void epi_silu32(const GemmArgs& p, int row, int outcol, const float (&g)[32], const float (&u)[32]) {
+  uint32_t pk[16];
+#pragma unroll
+  for (int i = 0; i < 16; ++i) pk[i] = pack_bf16(silu(g[2 * i]) * u[2 * i], silu(g[2 * i + 1]) * u[2 * i + 1]);
+  uint4* dst = reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.C) + size_t(row) * p.ldc + outcol);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) dst[i] = make_uint4(pk[4 * i], pk[4 * i + 1], pk[4 * i + 2], pk[4 * i + 3]);
+}
+
+QOS_DEV void tmem_ld32(uint32_t taddr, float (&v)[32]) {
+  uint32_t r[32];
+  tmem_ld32x32b_x16(taddr, *reinterpret_cast<uint32_t(*)[16]>(&r[0]));
+  tmem_ld32x32b_x16(taddr + 16, *reinterpret_cast<uint32_t(*)[16]>(&r[16]));
+  tmem_ld_wait();
+#pragma unroll
+  for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
+}
+
+QOS_DEV void epi_bar_sync() { asm volatile("bar.sync 1, 128;" ::: "memory"); }  // the 4 epilogue warps
 
 template <int BN, int EPI>
 __global__ void __launch_bounds__(kGemmThreads, 1)
@@ -58,6 +113,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
   uint64_t* tfull = empty + S;
   uint64_t* tempty = tfull + 2;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+  int* s_last = reinterpret_cast<int*>(tmem_slot + 1);
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -83,8 +139,18 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
 
-  const int num_tiles = p.mt * p.nt;
+  // work unit u = ((n_t * ksplit) + split) * mt + m_t: consecutive units share a weight slice
+  const int ks = p.ksplit;
+  const int num_units = p.mt * p.nt * ks;
   const int kblocks = p.K / kBK;
+  auto decode_unit = [&](int u, int& m_t, int& n_t, int& sp, int& kb0, int& kb1) {
+    m_t = u % p.mt;
+    const int r = u / p.mt;
+    sp = r % ks;
+    n_t = r / ks;
+    kb0 = sp * kblocks / ks;
+    kb1 = (sp + 1) * kblocks / ks;
+  };
 
   if (warp == 0) {
     // ------------------------------------------------------------ TMA producer
@@ -93,9 +159,10 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
       const uint64_t pol_b = l2_evict_first();  // weights: streamed once per M-tile group
       int stage = 0;
       uint32_t phase = 0;
-      for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) {
-        const int n_t = tile / p.mt, m_t = tile % p.mt;
-        for (int kb = 0; kb < kblocks; ++kb) {
+      for (int u = blockIdx.x; u < num_units; u += gridDim.x) {
+        int m_t, n_t, sp, kb0, kb1;
+        decode_unit(u, m_t, n_t, sp, kb0, kb1);
+        for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
           uint8_t* sa = smem + stage * Cfg::kStageBytes;
           mbar_arrive_expect_tx(&full[stage], Cfg::kStageBytes);
@@ -113,11 +180,13 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
       uint32_t phase = 0;
       int acc = 0;
       uint32_t acc_phase = 0;
-      for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) {
+      for (int u = blockIdx.x; u < num_units; u += gridDim.x) {
+        int m_t, n_t, sp, kb0, kb1;
+        decode_unit(u, m_t, n_t, sp, kb0, kb1);
         mbar_wait(&tempty[acc], acc_phase ^ 1);
         tc_fence_after();
         const uint32_t d_tmem = tmem_base + acc * BN;
-        for (int kb = 0; kb < kblocks; ++kb) {
+        for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(&full[stage], phase);
           tc_fence_after();
           const uint32_t a_base = smem_u32(smem + stage * Cfg::kStageBytes);
@@ -125,7 +194,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
 #pragma unroll
           for (int k = 0; k < kBK / 16; ++k) {
             umma_bf16(d_tmem, umma_desc_sw128(a_base + k * 32), umma_desc_sw128(b_base + k * 32), idesc,
-                      (kb | k) != 0);
+                      (kb > kb0 || k > 0) ? 1u : 0u);
           }
           umma_commit(&empty[stage]);
           if (++stage == S) { stage = 0; phase ^= 1; }
@@ -137,86 +206,109 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
   } else {
     // ------------------------------------------------------------ epilogue (warps 2..5)
     const int q = warp & 3;  // TMEM lane quarter this warp may access
+    const int rit = q * 32 + lane;  // row inside the tile
     int acc = 0;
     uint32_t acc_phase = 0;
-    for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) {
-      const int n_t = tile / p.mt, m_t = tile % p.mt;
+    for (int u = blockIdx.x; u < num_units; u += gridDim.x) {
+      int m_t, n_t, sp, kb0, kb1;
+      decode_unit(u, m_t, n_t, sp, kb0, kb1);
       mbar_wait(&tfull[acc], acc_phase);
       tc_fence_after();
-      const int row = m_t * kBM + q * 32 + lane;
+      const int row = m_t * kBM + rit;
       const bool row_ok = row < p.M;
       const uint32_t tbase = tmem_base + (uint32_t(q * 32) << 16) + acc * BN;
-      if constexpr (EPI == EPI_SILU_GATE) {
+      if (ks == 1) {
+        if constexpr (EPI == EPI_SILU_GATE) {
 #pragma unroll 1
-        for (int g = 0; g < BN / 128; ++g) {
+          for (int g = 0; g < BN / 128; ++g) {
 #pragma unroll 1
-          for (int h = 0; h < 2; ++h) {
-            uint32_t gr[32], ur[32];
-            tmem_ld32x32b_x16(tbase + g * 128 + h * 32, *reinterpret_cast<uint32_t(*)[16]>(&gr[0]));
-            tmem_ld32x32b_x16(tbase + g * 128 + h * 32 + 16, *reinterpret_cast<uint32_t(*)[16]>(&gr[16]));
-            tmem_ld32x32b_x16(tbase + g * 128 + 64 + h * 32, *reinterpret_cast<uint32_t(*)[16]>(&ur[0]));
-            tmem_ld32x32b_x16(tbase + g * 128 + 64 + h * 32 + 16, *reinterpret_cast<uint32_t(*)[16]>(&ur[16]));
-            tmem_ld_wait();
-            const int col = n_t * (BN / 2) + g * 64 + h * 32;
-            if (row_ok && col < p.N / 2) {
-              uint32_t pk[16];
-#pragma unroll
-              for (int i = 0; i < 16; ++i) {
-                const float a0 = silu(__uint_as_float(gr[2 * i])) * __uint_as_float(ur[2 * i]);
-                const float a1 = silu(__uint_as_float(gr[2 * i + 1])) * __uint_as_float(ur[2 * i + 1]);
-                pk[i] = pack_bf16(a0, a1);
-              }
-              uint4* dst = reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.C) + size_t(row) * p.ldc + col);
-#pragma unroll
-              for (int i = 0; i < 4; ++i) dst[i] = make_uint4(pk[4 * i], pk[4 * i + 1], pk[4 * i + 2], pk[4 * i + 3]);
+            for (int h = 0; h < 2; ++h) {
+              float gv[32], uv[32];
+              tmem_ld32(tbase + g * 128 + h * 32, gv);
+              tmem_ld32(tbase + g * 128 + 64 + h * 32, uv);
+              const int col = n_t * (BN / 2) + g * 64 + h * 32;
+              if (row_ok && col < p.N / 2) epi_silu32(p, row, col, gv, uv);
             }
           }
+        } else {
+#pragma unroll 1
+          for (int c = 0; c < BN / 32; ++c) {
+            float v[32];
+            tmem_ld32(tbase + c * 32, v);
+            const int col = n_t * BN + c * 32;
+            if (row_ok && col < p.N) epi_store32<EPI>(p, row, col, v);
+          }
         }
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&tempty[acc]);
       } else {
+        // split-K: park the fp32 partial, release TMEM, the last slice of the tile reduces
+        float* mine = p.part + (size_t(u) * kBM + rit) * BN;
 #pragma unroll 1
         for (int c = 0; c < BN / 32; ++c) {
-          uint32_t r[32];
-          tmem_ld32x32b_x16(tbase + c * 32, *reinterpret_cast<uint32_t(*)[16]>(&r[0]));
-          tmem_ld32x32b_x16(tbase + c * 32 + 16, *reinterpret_cast<uint32_t(*)[16]>(&r[16]));
-          tmem_ld_wait();
-          const int col = n_t * BN + c * 32;
-          if (row_ok && col < p.N) {
-            if constexpr (EPI == EPI_STORE_BF16 || EPI == EPI_BIAS_BF16) {
-              uint32_t pk[16];
+          float v[32];
+          tmem_ld32(tbase + c * 32, v);
 #pragma unroll
-              for (int i = 0; i < 16; ++i) {
-                float a0 = __uint_as_float(r[2 * i]), a1 = __uint_as_float(r[2 * i + 1]);
-                if constexpr (EPI == EPI_BIAS_BF16) {
-                  a0 += __ldg(p.bias + col + 2 * i);
-                  a1 += __ldg(p.bias + col + 2 * i + 1);
+          for (int i = 0; i < 8; ++i)
+            reinterpret_cast<float4*>(mine + c * 32)[i] = make_float4(v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
+        }
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&tempty[acc]);
+        __threadfence();
+        epi_bar_sync();
+        const int tile = n_t * p.mt + m_t;
+        if (threadIdx.x == 64) *s_last = (atomicAdd(p.counters + tile, 1) == ks - 1);
+        epi_bar_sync();
+        if (*s_last) {
+          __threadfence();
+          auto part_row = [&](int s2) {
+            return p.part + (size_t((n_t * ks + s2) * p.mt + m_t) * kBM + rit) * BN;
+          };
+          if constexpr (EPI == EPI_SILU_GATE) {
+#pragma unroll 1
+            for (int g = 0; g < BN / 128; ++g)
+#pragma unroll 1
+              for (int h = 0; h < 2; ++h) {
+                float gv[32], uv[32];
+#pragma unroll
+                for (int i = 0; i < 32; ++i) gv[i] = uv[i] = 0.f;
+                for (int s2 = 0; s2 < ks; ++s2) {
+                  const float* pr = part_row(s2);
+#pragma unroll
+                  for (int i = 0; i < 32; ++i) {
+                    gv[i] += __ldcg(pr + g * 128 + h * 32 + i);
+                    uv[i] += __ldcg(pr + g * 128 + 64 + h * 32 + i);
+                  }
                 }
-                pk[i] = pack_bf16(a0, a1);
+                const int col = n_t * (BN / 2) + g * 64 + h * 32;
+                if (row_ok && col < p.N / 2) epi_silu32(p, row, col, gv, uv);
               }
-              uint4* dst = reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.C) + size_t(row) * p.ldc + col);
+          } else {
+#pragma unroll 1
+            for (int c = 0; c < BN / 32; ++c) {
+              float v[32];
 #pragma unroll
-              for (int i = 0; i < 4; ++i) dst[i] = make_uint4(pk[4 * i], pk[4 * i + 1], pk[4 * i + 2], pk[4 * i + 3]);
-            } else if constexpr (EPI == EPI_STORE_F32) {
-              float4* dst = reinterpret_cast<float4*>(reinterpret_cast<float*>(p.C) + size_t(row) * p.ldc + col);
+              for (int i = 0; i < 32; ++i) v[i] = 0.f;
+              for (int s2 = 0; s2 < ks; ++s2) {
+                const float4* pr = reinterpret_cast<const float4*>(part_row(s2) + c * 32);
 #pragma unroll
-              for (int i = 0; i < 8; ++i)
-                dst[i] = make_float4(__uint_as_float(r[4 * i]), __uint_as_float(r[4 * i + 1]),
-                                     __uint_as_float(r[4 * i + 2]), __uint_as_float(r[4 * i + 3]));
-            } else {  // EPI_ADD_F32
-              float4* dst = reinterpret_cast<float4*>(reinterpret_cast<float*>(p.C) + size_t(row) * p.ldc + col);
-              float4 old[8];
-#pragma unroll
-              for (int i = 0; i < 8; ++i) old[i] = dst[i];
-#pragma unroll
-              for (int i = 0; i < 8; ++i)
-                dst[i] = make_float4(old[i].x + __uint_as_float(r[4 * i]), old[i].y + __uint_as_float(r[4 * i + 1]),
-                                     old[i].z + __uint_as_float(r[4 * i + 2]), old[i].w + __uint_as_float(r[4 * i + 3]));
+                for (int i = 0; i < 8; ++i) {
+                  const float4 x = __ldcg(pr + i);
+                  v[4 * i] += x.x;
+                  v[4 * i + 1] += x.y;
+                  v[4 * i + 2] += x.z;
+                  v[4 * i + 3] += x.w;
+                }
+              }
+              const int col = n_t * BN + c * 32;
+              if (row_ok && col < p.N) epi_store32<EPI>(p, row, col, v);
             }
           }
+          if (threadIdx.x == 64) p.counters[tile] = 0;  // ready for the next launch
         }
       }
-      tc_fence_before();
-      __syncwarp();
-      if (lane == 0) mbar_arrive(&tempty[acc]);
       if (++acc == 2) { acc = 0; acc_phase ^= 1; }
     }
   }
@@ -297,18 +389,30 @@ int gemm_pick_bn(int64_t M, int64_t N, int epi, int num_sms) {
   return (t256 >= num_sms && N % 256 == 0) ? 256 : 128;
 }
 
+int gemm_pick_ksplit(int64_t M, int64_t N, int64_t K, int bn, int num_sms, int64_t max_units) {
+  // weight-bound small-M GEMMs: split K until the units cover the SMs (>= 4 k-blocks each)
+  const int64_t tiles = ((M + kBM - 1) / kBM) * ((N + bn - 1) / bn);
+  int ks = 1;
+  while (tiles * ks * 2 <= num_sms + num_sms / 4 && (K / kBK) / (ks * 2) >= 4 && tiles * ks * 2 <= max_units) ks *= 2;
+  return ks;
+}
+
 int gemm_run(const CUtensorMap& ta, const CUtensorMap& tb, int bn, int64_t M, int64_t N, int64_t K, int epi, void* C,
-             int64_t ldc, const float* bias, int num_sms, cudaStream_t st) {
+             int64_t ldc, const float* bias, int num_sms, cudaStream_t st, int ksplit, float* part, int* counters) {
   GemmArgs a;
   a.M = int(M);
   a.N = int(N);
   a.K = int(K);
   a.mt = int((M + kBM - 1) / kBM);
   a.nt = int((N + bn - 1) / bn);
+  a.ksplit = ksplit < 1 ? 1 : ksplit;
   a.C = C;
   a.ldc = int(ldc);
   a.bias = bias;
-  const int tiles = a.mt * a.nt;
+  a.part = part;
+  a.counters = counters;
+  if (a.ksplit > 1 && (!part || !counters)) return set_error(QOS_ERR_INVALID_ARG, "gemm: split-K needs workspace");
+  const int tiles = a.mt * a.nt * a.ksplit;
   const int grid = tiles < num_sms ? tiles : num_sms;
   cudaError_t e = cudaSuccess;
 #define QOS_GEMM_CASE(BNV, EPIV) \

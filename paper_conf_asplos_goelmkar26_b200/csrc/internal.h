@@ -25,8 +25,12 @@ int make_tmap_3d_bf16(CUtensorMap* out, const void* base, uint64_t d0, uint64_t 
                       uint32_t b1, uint32_t b2);
 int gemm_pick_bn(int64_t M, int64_t N, int epi, int num_sms);
 int gemm_check_shape(int64_t M, int64_t N, int64_t K, int epi);
+int gemm_pick_ksplit(int64_t M, int64_t N, int64_t K, int bn, int num_sms, int64_t max_units);
+// ksplit > 1: split-K with fp32 partials in `part` ([units][128][bn]) and per-tile arrival
+// counters (zero-initialised; each reducing CTA resets its own) — deterministic reduction order
 int gemm_run(const CUtensorMap& ta, const CUtensorMap& tb, int bn, int64_t M, int64_t N, int64_t K, int epi, void* C,
-             int64_t ldc, const float* bias, int num_sms, cudaStream_t st);
+             int64_t ldc, const float* bias, int num_sms, cudaStream_t st, int ksplit = 1, float* part = nullptr,
+             int* counters = nullptr);
 
 // ------------------------------------------------------------------ synthetic generator (gen.cu)
 enum GenKind { GEN_LINEAR = 0, GEN_EMBED = 1, GEN_NORM = 2, GEN_BIAS = 3 };

@@ -94,6 +94,7 @@ _SIGS = {
     "qos_last_step_io": [_P, C.POINTER(C.c_int64), C.POINTER(C.c_int64)],
     "qos_engine_launch_count": [_P, C.POINTER(C.c_int64)],
     "qos_op_gemm": [_P, _P, _P, C.c_int64, C.c_int64, C.c_int64, C.c_int, _P, _P],
+    "qos_op_gemm_ex": [_P, _P, _P, C.c_int64, C.c_int64, C.c_int64, C.c_int, _P, C.c_int, _P],
     "qos_op_rmsnorm": [_P, _P, _P, C.c_int32, C.c_int32, C.c_float, _P],
     "qos_kv_write": [_P, C.c_int32, C.c_int64, C.c_int32, C.c_int32, _P, _P],
     "qos_kv_read": [_P, C.c_int32, C.c_int64, C.c_int32, C.c_int32, _P, _P],
@@ -135,6 +136,11 @@ def qos_nccl_unique_id() -> bytes:
 
 def qos_op_gemm(A, B, Cout, M: int, N: int, K: int, epi: str = "store_bf16", bias=None, stream=None):
     _call("qos_op_gemm", A, B, Cout, M, N, K, EPI[epi], bias, stream)
+
+
+def qos_op_gemm_ex(A, B, Cout, M: int, N: int, K: int, epi: str = "store_bf16", bias=None, ksplit: int = 0,
+                   stream=None):
+    _call("qos_op_gemm_ex", A, B, Cout, M, N, K, EPI[epi], bias, ksplit, stream)
 
 
 def qos_op_rmsnorm(x, g, out, T: int, d: int, eps: float, stream=None):

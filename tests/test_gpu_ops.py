@@ -214,3 +214,42 @@ def test_attention_parity(case):
     err = row_rel_err(out.reshape(-1, hd), ref.reshape(-1, hd))
     assert err <= TOL_ATTN, err
     eng.close()
+
+
+@pytest.mark.parametrize("M,N,K,ks", [(1, 512, 1024, 4), (130, 1024, 4096, 8), (256, 768, 512, 2), (77, 384, 640, 3)])
+@pytest.mark.parametrize("epi", ["store_f32", "store_bf16", "add_f32", "bias_bf16", "silu_gate"])
+def test_gemm_splitk_parity(torch_cuda, M, N, K, ks, epi):
+    """Split-K (weight-bound small-M GEMMs): slices reduced in order by the last CTA."""
+    torch = torch_cuda
+    from oracle.model import silu
+    from paper_conf_asplos_goelmkar26_b200 import qoserve as q
+    rng = np.random.default_rng(M + N + K + ks)
+    A = bits_to_f64(bf16_bits(rng.uniform(-1, 1, (M, K))))
+    B = bits_to_f64(bf16_bits(rng.uniform(-1, 1, (N, K)) / np.sqrt(K)))
+    dA, dB = _dev_bf16(torch, A), _dev_bf16(torch, B)
+    ref = A @ B.T
+    bias = None
+    if epi == "silu_gate":
+        g = np.concatenate([ref[:, 128 * j:128 * j + 64] for j in range(N // 128)], axis=1)
+        u = np.concatenate([ref[:, 128 * j + 64:128 * j + 128] for j in range(N // 128)], axis=1)
+        ref = silu(g) * u
+        dC = torch.empty((M, N // 2), dtype=torch.bfloat16, device="cuda")
+    elif epi in ("store_f32", "add_f32"):
+        init = rng.uniform(-1, 1, (M, N)).astype(np.float32) if epi == "add_f32" else np.zeros((M, N), np.float32)
+        dC = torch.from_numpy(init.copy()).cuda()
+        ref = ref + init.astype(np.float64)
+    else:
+        dC = torch.empty((M, N), dtype=torch.bfloat16, device="cuda")
+        if epi == "bias_bf16":
+            bvals = bits_to_f64(bf16_bits(rng.uniform(-0.02, 0.02, N)))
+            bias = torch.from_numpy(bvals.astype(np.float32)).cuda()
+            ref = ref + bvals
+    for _ in range(2):   # twice: the arrival counters must be reset by the reducing CTA
+        if epi == "add_f32":
+            dC.copy_(torch.from_numpy(init.copy()).cuda())
+        q.qos_op_gemm_ex(dA.data_ptr(), dB.data_ptr(), dC.data_ptr(), M, N, K, epi,
+                         bias.data_ptr() if bias is not None else None, ks)
+        torch.cuda.synchronize()
+        got = dC.float().cpu().numpy()
+        tol = 1e-5 if epi in ("store_f32", "add_f32") else 8e-3
+        assert row_rel_err(got, ref) <= tol
