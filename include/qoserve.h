@@ -96,6 +96,16 @@ int qos_engine_create(const qos_model_cfg* cfg, int device, int tp_rank, int tp_
                       const uint8_t* nccl_uid, const qos_mem* mem, qos_engine_t** out);
 int qos_engine_destroy(qos_engine_t* eng);
 
+/* This rank's slice under tensor parallelism (pure host function):
+ * q heads [head0, head0+n_heads), kv heads [kv_head0, +n_kv_heads), FFN columns
+ * [ffn0, +ffn), vocab rows [vocab0, +vocab) of lm_head.  o_proj / down_proj take the matching
+ * input columns; their partial outputs are summed by the all-reduce. */
+typedef struct {
+  int32_t n_heads, n_kv_heads, ffn, vocab;
+  int32_t head0, kv_head0, ffn0, vocab0;
+} qos_shard;
+int qos_shard_plan(const qos_model_cfg* cfg, int tp_rank, int tp_size, qos_shard* out);
+
 /* 128-byte ncclUniqueId for tp_size > 1 (call on rank 0 only). */
 int qos_nccl_unique_id(uint8_t out[128]);
 

@@ -768,6 +768,14 @@ int qos_engine_mem_sizes(const qos_model_cfg* cfg, int tp_size, qos_mem_sizes* o
   return QOS_OK;
 }
 
+int qos_shard_plan(const qos_model_cfg* cfg, int tp_rank, int tp_size, qos_shard* out) {
+  QOS_TRY(check_cfg(cfg, tp_size));
+  if (!out || tp_rank < 0 || tp_rank >= tp_size) return set_error(QOS_ERR_INVALID_ARG, "shard plan args");
+  const Shard s = make_shard(*cfg, tp_rank, tp_size);
+  *out = qos_shard{s.H, s.Hkv, s.F, s.V, s.h0, s.kv0, s.f0, s.v0};
+  return QOS_OK;
+}
+
 int qos_nccl_unique_id(uint8_t out[128]) {
   std::lock_guard<std::mutex> g(g_nccl_mu);
   if (!g_nccl.load()) return set_error(QOS_ERR_COMM, "libnccl.so.2 not loadable");

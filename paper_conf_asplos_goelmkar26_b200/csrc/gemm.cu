@@ -230,6 +230,32 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
               if (row_ok && col < p.N / 2) epi_silu32(p, row, col, gv, uv);
             }
           }
+        } else if constexpr (EPI == EPI_ADD_F32) {
+          // residual read-modify-write, software-pipelined: the residual loads of chunk c+1 are
+          // in flight while chunk c is added and stored (one exposed load latency per tile)
+          float* rrow = reinterpret_cast<float*>(p.C) + size_t(row) * p.ldc + n_t * BN;
+          const bool ok0 = row_ok;
+          float4 cur[8], nxt[8];
+#pragma unroll
+          for (int i = 0; i < 8; ++i) cur[i] = (ok0 && n_t * BN < p.N) ? reinterpret_cast<const float4*>(rrow)[i] : make_float4(0, 0, 0, 0);
+#pragma unroll 1
+          for (int c = 0; c < BN / 32; ++c) {
+            const bool ok_next = ok0 && c + 1 < BN / 32 && n_t * BN + (c + 1) * 32 < p.N;
+#pragma unroll
+            for (int i = 0; i < 8; ++i)
+              nxt[i] = ok_next ? reinterpret_cast<const float4*>(rrow + (c + 1) * 32)[i] : make_float4(0, 0, 0, 0);
+            float v[32];
+            tmem_ld32(tbase + c * 32, v);
+            if (row_ok && n_t * BN + c * 32 < p.N) {
+              float4* dst = reinterpret_cast<float4*>(rrow + c * 32);
+#pragma unroll
+              for (int i = 0; i < 8; ++i)
+                dst[i] = make_float4(cur[i].x + v[4 * i], cur[i].y + v[4 * i + 1], cur[i].z + v[4 * i + 2],
+                                     cur[i].w + v[4 * i + 3]);
+            }
+#pragma unroll
+            for (int i = 0; i < 8; ++i) cur[i] = nxt[i];
+          }
         } else {
 #pragma unroll 1
           for (int c = 0; c < BN / 32; ++c) {

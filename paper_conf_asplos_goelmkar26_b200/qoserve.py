@@ -55,6 +55,11 @@ class qos_mem(C.Structure):
     _fields_ = [("weights", C.c_void_p), ("kv", C.c_void_p), ("workspace", C.c_void_p)]
 
 
+class qos_shard(C.Structure):
+    _fields_ = [("n_heads", C.c_int32), ("n_kv_heads", C.c_int32), ("ffn", C.c_int32), ("vocab", C.c_int32),
+                ("head0", C.c_int32), ("kv_head0", C.c_int32), ("ffn0", C.c_int32), ("vocab0", C.c_int32)]
+
+
 class qos_prefill_chunk(C.Structure):
     _fields_ = [("req", C.c_int64), ("kv_start", C.c_int32), ("chunk_len", C.c_int32),
                 ("tokens", C.POINTER(C.c_int32))]
@@ -76,6 +81,7 @@ _SIGS = {
                           C.POINTER(qos_mem), C.POINTER(_P)],
     "qos_engine_destroy": [_P],
     "qos_nccl_unique_id": [C.c_char_p],
+    "qos_shard_plan": [C.POINTER(qos_model_cfg), C.c_int, C.c_int, C.POINTER(qos_shard)],
     "qos_engine_load_synthetic": [_P, C.c_uint64],
     "qos_engine_read_weight": [_P, C.c_char_p, C.c_int64, C.c_int64, _P],
     "qos_kv_alloc": [_P, C.c_int64, C.c_int32],
@@ -125,6 +131,12 @@ def _call(name: str, *args) -> None:
 def qos_engine_mem_sizes(cfg: qos_model_cfg, tp_size: int = 1) -> qos_mem_sizes:
     out = qos_mem_sizes()
     _call("qos_engine_mem_sizes", C.byref(cfg), tp_size, C.byref(out))
+    return out
+
+
+def qos_shard_plan(cfg: qos_model_cfg, tp_rank: int, tp_size: int) -> qos_shard:
+    out = qos_shard()
+    _call("qos_shard_plan", C.byref(cfg), tp_rank, tp_size, C.byref(out))
     return out
 
 

@@ -14,6 +14,7 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--points", default="256:0:0,512:0:0,256:128:1024,512:128:1024,2048:128:4096,8192:0:0")
 ap.add_argument("--layers", type=int, default=None)
 ap.add_argument("--reps", type=int, default=5)
+ap.add_argument("--breakdown", action="store_true", help="per-kernel-class ms per step (events)")
 a = ap.parse_args()
 import torch  # noqa: E402
 torch.cuda.set_device(0)
@@ -25,7 +26,14 @@ cfg = q.model_cfg(**preset("llama3-8b", **over), num_blocks=need // 16 + 600, ma
 eng = q.Engine(cfg)
 eng.qos_engine_load_synthetic(0)
 for c, nd, ctx in pts:
+    if a.breakdown:
+        eng.qos_engine_set_timing(True)
     ms, p95 = eng.qos_profile_step(c, [ctx] * nd, reps=a.reps)
-    print(json.dumps({"chunk": c, "n_decode": nd, "ctx": ctx, "ms": round(ms, 3), "p95": round(p95, 3),
-                      "tok_s": round((c + nd) / ms * 1e3)}), flush=True)
+    rec = {"chunk": c, "n_decode": nd, "ctx": ctx, "ms": round(ms, 3), "p95": round(p95, 3),
+           "tok_s": round((c + nd) / ms * 1e3)}
+    if a.breakdown:
+        tm = eng.qos_last_step_timing()
+        rec["breakdown"] = {k: round(v[0] / (3 + a.reps), 3) for k, v in tm.items() if v[1]}
+        eng.qos_engine_set_timing(False)
+    print(json.dumps(rec), flush=True)
 eng.close()
