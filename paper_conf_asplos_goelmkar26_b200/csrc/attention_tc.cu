@@ -25,14 +25,16 @@ namespace qos {
 template <int HD>
 struct FaCfg {
   static constexpr int kRows = 128;                  // Q-tile rows (UMMA M)
-  static constexpr int kKeys = 128;                  // keys per K/V tile
+  static constexpr int kKeys = 64;                   // keys per K/V tile (4 paged blocks)
   static constexpr int kHalves = HD / 64;
   static constexpr int kQBytes = kRows * HD * 2;     // 32 KB at HD 128
   static constexpr int kTileBytes = kKeys * HD * 2;  // one K or V tile
-  // 2 CTAs per SM: Q + one K + one V tile (96 KB at HD 128) and 256 TMEM columns each; the two
-  // co-resident CTAs interleave their serial QK -> softmax -> PV chains on the tensor core.
-  static constexpr int kSmem = kQBytes + 2 * kTileBytes + 1024 + 256;
-  static constexpr uint32_t kColS = 0, kColO = 128;
+  // 2 CTAs per SM: Q + 2-stage K and V rings (96 KB at HD 128) and 256 TMEM columns each
+  // (two 64-column S/P buffers + the O accumulator).  With two S buffers the MMA warp issues
+  // QK of tile j+1 before PV of tile j, so the softmax never waits on its own PV.
+  static constexpr int kStages = 2;
+  static constexpr int kSmem = kQBytes + 2 * kStages * kTileBytes + 1024 + 256;
+  static constexpr uint32_t kColS0 = 0, kColS1 = 64, kColO = 128;
   static constexpr uint32_t kTmemCols = 256;
 };
 
@@ -97,16 +99,16 @@ __global__ void __launch_bounds__(kFaThreads, 2)
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sQ = smem;
   uint8_t* sK = smem + C::kQBytes;
-  uint8_t* sV = sK + C::kTileBytes;
-  uint64_t* bar = reinterpret_cast<uint64_t*>(sV + C::kTileBytes);
+  uint8_t* sV = sK + C::kStages * C::kTileBytes;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(sV + C::kStages * C::kTileBytes);
   uint64_t* k_full = bar + 0;
-  uint64_t* k_empty = bar + 1;
-  uint64_t* v_full = bar + 2;
-  uint64_t* v_empty = bar + 3;
-  uint64_t* s_full = bar + 4;
-  uint64_t* p_full = bar + 5;
-  uint64_t* o_full = bar + 6;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 8);
+  uint64_t* k_empty = bar + 2;
+  uint64_t* v_full = bar + 4;
+  uint64_t* v_empty = bar + 6;
+  uint64_t* s_full = bar + 8;
+  uint64_t* p_full = bar + 10;
+  uint64_t* o_full = bar + 12;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 14);
 
   const PrefillItem it = items[blockIdx.x];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -117,12 +119,14 @@ __global__ void __launch_bounds__(kFaThreads, 2)
   const int last_blk = last_pos >> 4;
 
   if (threadIdx.x == 0) {
-    mbar_init(k_full, 1);
-    mbar_init(k_empty, 1);
-    mbar_init(v_full, 1);
-    mbar_init(v_empty, 1);
-    mbar_init(s_full, 1);
-    mbar_init(p_full, 128);
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&k_full[i], 1);
+      mbar_init(&k_empty[i], 1);
+      mbar_init(&v_full[i], 1);
+      mbar_init(&v_empty[i], 1);
+      mbar_init(&s_full[i], 1);
+      mbar_init(&p_full[i], 128);
+    }
     mbar_init(o_full, 1);
     fence_mbar_init();
   }
@@ -159,8 +163,8 @@ __global__ void __launch_bounds__(kFaThreads, 2)
       tma_prefetch_desc(&kvmap);
       const int32_t* trow = p.tables + size_t(it.table) * p.table_w;
       auto load_tile = [&](uint8_t* dst, uint64_t* full, int j, int plane) {
-        for (int b = 0; b < 8; ++b) {
-          const int blk = min(j * 8 + b, last_blk);  // past the causal end: any valid block (P = 0)
+        for (int b = 0; b < C::kKeys / 16; ++b) {
+          const int blk = min(j * (C::kKeys / 16) + b, last_blk);  // past the causal end: a valid block (P = 0)
           const int r = (__ldg(trow + blk) * p.Hkv + it.kv_head) * 16;
 #pragma unroll
           for (int hf = 0; hf < C::kHalves; ++hf)
@@ -168,13 +172,14 @@ __global__ void __launch_bounds__(kFaThreads, 2)
         }
       };
       for (int j = 0; j < ntiles; ++j) {
-        const uint32_t ph = j & 1;
-        mbar_wait(k_empty, ph ^ 1);
-        mbar_arrive_expect_tx(k_full, C::kTileBytes);
-        load_tile(sK, k_full, j, 0);
-        mbar_wait(v_empty, ph ^ 1);
-        mbar_arrive_expect_tx(v_full, C::kTileBytes);
-        load_tile(sV, v_full, j, 1);
+        const int s = j & 1;
+        const uint32_t ph = (j >> 1) & 1;
+        mbar_wait(&k_empty[s], ph ^ 1);
+        mbar_arrive_expect_tx(&k_full[s], C::kTileBytes);
+        load_tile(sK + s * C::kTileBytes, &k_full[s], j, 0);
+        mbar_wait(&v_empty[s], ph ^ 1);
+        mbar_arrive_expect_tx(&v_full[s], C::kTileBytes);
+        load_tile(sV + s * C::kTileBytes, &v_full[s], j, 1);
       }
     }
   } else if (warp == 1) {
@@ -182,45 +187,57 @@ __global__ void __launch_bounds__(kFaThreads, 2)
     if (elect_one()) {
       constexpr uint32_t idesc_qk = umma_idesc_bf16(128, C::kKeys);
       constexpr uint32_t idesc_pv = umma_idesc_bf16(128, HD) | (1u << 16);  // B (V) MN-major
-      const uint32_t q_base = smem_u32(sQ), k_base = smem_u32(sK), v_base = smem_u32(sV);
-      for (int j = 0; j < ntiles; ++j) {
-        const uint32_t ph = j & 1;
-        // S_j = Q K_j^T (S is free: PV_{j-1}, its last reader, was issued before, in order)
-        mbar_wait(k_full, ph);
+      const uint32_t q_base = smem_u32(sQ);
+      auto issue_pv = [&](int t) {
+        const int s = t & 1;
+        const uint32_t ph = (t >> 1) & 1;
+        mbar_wait(&p_full[s], ph);
+        mbar_wait(&v_full[s], ph);
         tc_fence_after();
+        const uint32_t v_base = smem_u32(sV + s * C::kTileBytes);
+        const uint32_t p_tmem = tmem + (s ? C::kColS1 : C::kColS0);
+#pragma unroll
+        for (int kk = 0; kk < C::kKeys / 16; ++kk) {
+          const uint64_t vd = umma_desc_sw128_mn(v_base + kk * 2048, C::kKeys * 128);
+          const uint32_t pc = p_tmem + (kk >> 1) * 32 + (kk & 1) * 8;
+          umma_bf16_ts(tmem + C::kColO, pc, vd, idesc_pv, (t | kk) != 0);  // P_hi
+          umma_bf16_ts(tmem + C::kColO, pc + 16, vd, idesc_pv, 1);         // P_lo
+        }
+        umma_commit(o_full);
+        umma_commit(&v_empty[s]);
+      };
+      for (int j = 0; j < ntiles; ++j) {
+        // S_j = Q K_j^T into S[j%2]; its previous tenant P_{j-2} was consumed by PV_{j-2},
+        // which is issued before this point (tcgen05 ops execute in issue order)
+        const int s = j & 1;
+        const uint32_t ph = (j >> 1) & 1;
+        mbar_wait(&k_full[s], ph);
+        tc_fence_after();
+        const uint32_t k_base = smem_u32(sK + s * C::kTileBytes);
+        const uint32_t s_tmem = tmem + (s ? C::kColS1 : C::kColS0);
 #pragma unroll
         for (int ks = 0; ks < HD / 16; ++ks) {
           const uint32_t qoff = (ks >> 2) * (C::kRows * 128) + (ks & 3) * 32;
           const uint32_t koff = (ks >> 2) * (C::kKeys * 128) + (ks & 3) * 32;
-          umma_bf16(tmem + C::kColS, umma_desc_sw128(q_base + qoff), umma_desc_sw128(k_base + koff), idesc_qk,
-                    ks != 0);
+          umma_bf16(s_tmem, umma_desc_sw128(q_base + qoff), umma_desc_sw128(k_base + koff), idesc_qk, ks != 0);
         }
-        umma_commit(s_full);
-        umma_commit(k_empty);
-        // O += P_j V_j with P = P_hi + P_lo from TMEM
-        mbar_wait(p_full, ph);
-        mbar_wait(v_full, ph);
-        tc_fence_after();
-#pragma unroll
-        for (int kk = 0; kk < C::kKeys / 16; ++kk) {
-          const uint64_t vd = umma_desc_sw128_mn(v_base + kk * 2048, C::kKeys * 128);
-          const uint32_t pc = tmem + C::kColS + (kk >> 1) * 32 + (kk & 1) * 8;
-          umma_bf16_ts(tmem + C::kColO, pc, vd, idesc_pv, (j | kk) != 0);  // P_hi
-          umma_bf16_ts(tmem + C::kColO, pc + 16, vd, idesc_pv, 1);         // P_lo
-        }
-        umma_commit(o_full);
-        umma_commit(v_empty);
+        umma_commit(&s_full[s]);
+        umma_commit(&k_empty[s]);
+        if (j >= 1) issue_pv(j - 1);   // O += P_{j-1} V_{j-1} while the softmax works on S_j
       }
+      issue_pv(ntiles - 1);
     }
   } else {
     // ------------------------------------------------------------------ softmax (warps 2..5)
-    const uint32_t s_addr = tmem + (uint32_t((warp & 3) * 32) << 16) + C::kColS;
+    const uint32_t lane_base = tmem + (uint32_t((warp & 3) * 32) << 16);
     const uint32_t o_addr = tmem + (uint32_t((warp & 3) * 32) << 16) + C::kColO;
     const int warp_min_pos = __shfl_sync(0xffffffffu, pos_r < 0 ? INT_MAX : pos_r, 0);  // row 0 of the warp
     float m_used = -INFINITY, l = 0.f;
     for (int j = 0; j < ntiles; ++j) {
-      mbar_wait(s_full, j & 1);
+      const int sb = j & 1;
+      mbar_wait(&s_full[sb], (j >> 1) & 1);
       tc_fence_after();
+      const uint32_t s_addr = lane_base + (sb ? C::kColS1 : C::kColS0);
       const int key0 = j * C::kKeys;
       // masking only where a key of this tile can exceed a row's position
       const bool masked = __any_sync(0xffffffffu, key0 + C::kKeys - 1 > (pos_r < 0 ? -1 : pos_r)) ||
@@ -278,7 +295,7 @@ __global__ void __launch_bounds__(kFaThreads, 2)
       tmem_st_wait();
       l = l * alpha + sum;
       if (j >= 1) {
-        // PV_{j-1} (issued before QK_j) is complete; rescale O before PV_j accumulates into it
+        // wait for PV_{j-1}; rescale O (if needed) before PV_j accumulates into it
         mbar_wait(o_full, (j - 1) & 1);
         tc_fence_after();
         if (__any_sync(0xffffffffu, alpha != 1.f)) {
@@ -296,7 +313,7 @@ __global__ void __launch_bounds__(kFaThreads, 2)
       }
       m_used = m_new;
       tc_fence_before();
-      mbar_arrive(p_full);
+      mbar_arrive(&p_full[sb]);
     }
     // epilogue: O / l
     mbar_wait(o_full, (ntiles - 1) & 1);
