@@ -321,7 +321,7 @@ int check_cfg(const qos_model_cfg* c, int tp) {
     return set_error(QOS_ERR_INVALID_ARG, "bad model dims");
   if (c->n_heads % c->n_kv_heads) return set_error(QOS_ERR_INVALID_ARG, "n_heads % n_kv_heads != 0");
   if (c->head_dim != 64 && c->head_dim != 128) return set_error(QOS_ERR_UNSUPPORTED, "head_dim must be 64 or 128");
-  if (c->n_heads / c->n_kv_heads > 16) return set_error(QOS_ERR_UNSUPPORTED, "GQA group > 16");
+  if (c->n_heads / c->n_kv_heads > 8) return set_error(QOS_ERR_UNSUPPORTED, "GQA group > 8");
   if (c->block_size != 16) return set_error(QOS_ERR_UNSUPPORTED, "block_size must be 16");
   if (tp < 1 || c->n_kv_heads % tp || c->n_heads % tp || c->ffn_dim % tp || c->vocab % tp)
     return set_error(QOS_ERR_INVALID_ARG, "tp_size must divide n_kv_heads, n_heads, ffn_dim, vocab");

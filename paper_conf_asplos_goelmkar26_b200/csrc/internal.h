@@ -107,8 +107,6 @@ struct AttnLaunch {
 };
 cudaError_t launch_decode_attention(const AttnLaunch& a, const DecodeItem* items, int n_items, float* partials,
                                     int* counters, cudaStream_t st);
-cudaError_t launch_prefill_attention(const AttnLaunch& a, const PrefillItem* items, int n_items, cudaStream_t st);
-int prefill_positions_per_tile(int group);
 cudaError_t launch_prefill_attention_tc(const AttnLaunch& a, const PrefillItem* items, int n_items, cudaStream_t st);
 int prefill_tc_positions_per_tile(int group);
 
