@@ -24,6 +24,10 @@ namespace qos {
 constexpr int kAttnStages = 8;
 constexpr int kConsumerWarps = 4;
 constexpr int kAttnThreads = (kConsumerWarps + 1) * 32;
+// Block i goes to consumer warp i % kConsumerWarps and ring stage i % kAttnStages.  With a
+// multiple, stage s is always consumed by the same warp, in order, so no waiter can run a full
+// phase ahead of an mbarrier (parity waits would then alias).
+static_assert(kAttnStages % kConsumerWarps == 0, "ring depth must be a multiple of the consumer warps");
 
 template <int HD>
 struct AttnCfg {
