@@ -184,9 +184,10 @@ int qos_hybrid_step(qos_engine_t* eng, const qos_batch* batch, void* logits, int
  * CUDA events on the engine stream; *ms_out = median.  Synchronous; scratch KV is freed. */
 int qos_profile_step(qos_engine_t* eng, int32_t chunk_len, int32_t n_decode,
                      const int32_t* ctx_lens, int32_t reps, float* ms_out);
-/* Same with an explicit chunk kv_start (prefix already cached) and p95 output. */
+/* Same with an explicit chunk kv_start (prefix already cached), warm-up step count and p95
+ * output (`warmup` < 0 selects the default of 3). */
 int qos_profile_step_ex(qos_engine_t* eng, int32_t chunk_len, int32_t kv_start,
-                        int32_t n_decode, const int32_t* ctx_lens, int32_t reps,
+                        int32_t n_decode, const int32_t* ctx_lens, int32_t warmup, int32_t reps,
                         float* ms_median, float* ms_p95);
 
 /* ---------------------------------------------------------------- per-kernel timing (a15) */

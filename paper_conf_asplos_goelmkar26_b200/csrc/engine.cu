@@ -1126,7 +1126,8 @@ int qos_hybrid_step(qos_engine_t* e, const qos_batch* batch, void* logits, int l
 }
 
 int qos_profile_step_ex(qos_engine_t* e, int32_t chunk_len, int32_t kv_start, int32_t n_decode,
-                        const int32_t* ctx_lens, int32_t reps, float* ms_median, float* ms_p95) {
+                        const int32_t* ctx_lens, int32_t warmup, int32_t reps, float* ms_median, float* ms_p95) {
+  if (warmup < 0) warmup = 3;
   if (!e || chunk_len < 0 || kv_start < 0 || n_decode < 0 || (n_decode && !ctx_lens) || reps < 1 || !ms_median)
     return set_error(QOS_ERR_INVALID_ARG, "profile args");
   if (chunk_len == 0 && n_decode == 0) return set_error(QOS_ERR_INVALID_ARG, "empty profile batch");
@@ -1159,14 +1160,14 @@ int qos_profile_step_ex(qos_engine_t* e, int32_t chunk_len, int32_t kv_start, in
   cudaEventCreate(&a);
   cudaEventCreate(&z);
   std::vector<float> ms;
-  for (int i = 0; i < 3 + reps; ++i) {
+  for (int i = 0; i < warmup + reps; ++i) {
     cudaEventRecord(a, st);
     if ((r = do_step(e, &b, nullptr, QOS_F32, nullptr, 0, st, false)) != QOS_OK) break;
     cudaEventRecord(z, st);
     cudaEventSynchronize(z);
     float t = 0;
     cudaEventElapsedTime(&t, a, z);
-    if (i >= 3) ms.push_back(t);
+    if (i >= warmup) ms.push_back(t);
   }
   cudaEventDestroy(a);
   cudaEventDestroy(z);
@@ -1180,7 +1181,7 @@ int qos_profile_step_ex(qos_engine_t* e, int32_t chunk_len, int32_t kv_start, in
 
 int qos_profile_step(qos_engine_t* e, int32_t chunk_len, int32_t n_decode, const int32_t* ctx_lens, int32_t reps,
                      float* ms_out) {
-  return qos_profile_step_ex(e, chunk_len, 0, n_decode, ctx_lens, reps, ms_out, nullptr);
+  return qos_profile_step_ex(e, chunk_len, 0, n_decode, ctx_lens, -1, reps, ms_out, nullptr);
 }
 
 int qos_engine_set_timing(qos_engine_t* e, int enable) {

@@ -93,7 +93,7 @@ _SIGS = {
     "qos_kv_fill_synthetic": [_P, C.c_int64, C.c_int32, C.c_uint64],
     "qos_hybrid_step": [_P, C.POINTER(qos_batch), _P, C.c_int, _P, C.c_int, _P],
     "qos_profile_step": [_P, C.c_int32, C.c_int32, C.POINTER(C.c_int32), C.c_int32, C.POINTER(C.c_float)],
-    "qos_profile_step_ex": [_P, C.c_int32, C.c_int32, C.c_int32, C.POINTER(C.c_int32), C.c_int32,
+    "qos_profile_step_ex": [_P, C.c_int32, C.c_int32, C.c_int32, C.POINTER(C.c_int32), C.c_int32, C.c_int32,
                             C.POINTER(C.c_float), C.POINTER(C.c_float)],
     "qos_engine_set_timing": [_P, C.c_int],
     "qos_last_step_timing": [_P, C.POINTER(C.c_float), C.POINTER(C.c_int32)],
@@ -307,11 +307,11 @@ class Engine:
         self.qos_hybrid_step(batch, lg.ctypes.data, QOS_F32, tk.ctypes.data, True, None)
         return lg, tk
 
-    def qos_profile_step(self, chunk_len: int, ctx_lens, reps: int = 10, kv_start: int = 0):
+    def qos_profile_step(self, chunk_len: int, ctx_lens, reps: int = 10, kv_start: int = 0, warmup: int = -1):
         ctx = np.ascontiguousarray(np.asarray(ctx_lens, dtype=np.int32))
         med, p95 = C.c_float(), C.c_float()
         _call("qos_profile_step_ex", self.h, chunk_len, kv_start, len(ctx),
-              ctx.ctypes.data_as(C.POINTER(C.c_int32)), reps, C.byref(med), C.byref(p95))
+              ctx.ctypes.data_as(C.POINTER(C.c_int32)), warmup, reps, C.byref(med), C.byref(p95))
         return med.value, p95.value
 
     def qos_engine_set_timing(self, enable: bool):

@@ -29,7 +29,8 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--out", default="gpurun_out/latency_table.json")
     ap.add_argument("--test", type=int, default=200)
-    ap.add_argument("--reps", type=int, default=5)
+    ap.add_argument("--reps", type=int, default=7)
+    ap.add_argument("--warmup", type=int, default=8)
     ap.add_argument("--layers", type=int, default=None)
     ap.add_argument("--kv-gb", type=float, default=140.0)
     a = ap.parse_args()
@@ -48,10 +49,13 @@ def main():
     t0 = time.time()
 
     def prof(chunk, ctx, kv_start=0):
-        ms, p95 = eng.qos_profile_step(chunk, ctx, reps=a.reps, kv_start=kv_start)
+        # warm-up steps of the same shape settle the power-capped clock before timing
+        ms, p95 = eng.qos_profile_step(chunk, ctx, reps=a.reps, kv_start=kv_start, warmup=a.warmup)
         return ms, p95
 
-    fit_shapes, fit_ms, table = [], [], []
+    # the GPU is brought to its loaded (power-capped) clock first
+    eng.qos_profile_step(4096, [4096] * 64, reps=20, warmup=10)
+    grid = []
     for ctx in (1024, 4096):
         for nd in (0, 32, 128, 256):
             if nd * (ctx + 1) > cap_tokens:
@@ -59,20 +63,20 @@ def main():
             for chunk in (0, 256, 512, 1024, 1536, 2048, 3072, 4096, 6144, 8192):
                 if chunk == 0 and nd == 0:
                     continue
-                ms, p95 = prof(chunk, [ctx] * nd)
-                s = StepShape([(0, chunk)] if chunk else [], [ctx] * nd)
-                fit_shapes.append(s)
-                fit_ms.append(ms)
-                table.append({"chunk": chunk, "n_decode": nd, "ctx": ctx, "kv_start": 0, "ms": ms, "p95_ms": p95,
-                              "tokens_per_s": s.T / (ms * 1e-3)})
+                grid.append((chunk, nd, ctx, 0))
     for chunk in (256, 1024, 2048, 4096):
         for nd in (0, 128):
-            ms, p95 = prof(chunk, [2048] * nd, kv_start=4096)
-            s = StepShape([(4096, chunk)], [2048] * nd)
-            fit_shapes.append(s)
-            fit_ms.append(ms)
-            table.append({"chunk": chunk, "n_decode": nd, "ctx": 2048, "kv_start": 4096, "ms": ms, "p95_ms": p95,
-                          "tokens_per_s": s.T / (ms * 1e-3)})
+            grid.append((chunk, nd, 2048, 4096))
+    order = rng.permutation(len(grid))   # random order: no systematic clock drift along the grid
+    fit_shapes, fit_ms, table = [], [], []
+    for gi in order:
+        chunk, nd, ctx, ks = grid[gi]
+        ms, p95 = prof(chunk, [ctx] * nd, kv_start=ks)
+        s = StepShape([(ks, chunk)] if chunk else [], [ctx] * nd)
+        fit_shapes.append(s)
+        fit_ms.append(ms)
+        table.append({"chunk": chunk, "n_decode": nd, "ctx": ctx, "kv_start": ks, "ms": ms, "p95_ms": p95,
+                      "tokens_per_s": s.T / (ms * 1e-3)})
     model = LatencyModel().fit(fit_shapes, fit_ms)
     fit_err = [abs(model.predict(s) - m) / m for s, m in zip(fit_shapes, fit_ms)]
     tests = []
