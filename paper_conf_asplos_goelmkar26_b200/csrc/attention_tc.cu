@@ -294,28 +294,30 @@ __global__ void __launch_bounds__(kFaThreads, 2)
       }
       tmem_st_wait();
       l = l * alpha + sum;
-      if (j >= 1) {
-        // wait for PV_{j-1}; rescale O (if needed) before PV_j accumulates into it
+      if (j >= 1 && __any_sync(0xffffffffu, alpha != 1.f)) {
+        // rescale O (tiles < j) before PV_j accumulates into it.  Wait for PV_{j-1} only here:
+        // PV_{j-2} was issued before QK_j, whose completion was awaited above, so o_full is at
+        // phase j-1 or j and this parity wait cannot alias.
         mbar_wait(o_full, (j - 1) & 1);
         tc_fence_after();
-        if (__any_sync(0xffffffffu, alpha != 1.f)) {
 #pragma unroll 1
-          for (int c = 0; c < HD / 16; ++c) {
-            uint32_t r[16];
-            tmem_ld32x32b_x16(o_addr + c * 16, r);
-            tmem_ld_wait();
+        for (int c = 0; c < HD / 16; ++c) {
+          uint32_t r[16];
+          tmem_ld32x32b_x16(o_addr + c * 16, r);
+          tmem_ld_wait();
 #pragma unroll
-            for (int i = 0; i < 16; ++i) r[i] = __float_as_uint(__uint_as_float(r[i]) * alpha);
-            tmem_st32x32b_x16(o_addr + c * 16, r);
-          }
-          tmem_st_wait();
+          for (int i = 0; i < 16; ++i) r[i] = __float_as_uint(__uint_as_float(r[i]) * alpha);
+          tmem_st32x32b_x16(o_addr + c * 16, r);
         }
+        tmem_st_wait();
       }
       m_used = m_new;
       tc_fence_before();
       mbar_arrive(&p_full[sb]);
     }
     // epilogue: O / l
+    // PV_{n-3} precedes QK_{n-1} (awaited), so o_full is at phase >= n-2: wait n-2, then n-1
+    if (ntiles >= 2) mbar_wait(o_full, (ntiles - 2) & 1);
     mbar_wait(o_full, (ntiles - 1) & 1);
     tc_fence_after();
     const float inv = (l > 0.f) ? 1.f / l : 0.f;

@@ -4,28 +4,31 @@ The paper predicts batch latency with a random forest trained on Vidur's per-op 
 uses it to pick the largest chunk that keeps every decode's next-token deadline
 (GET_PREFILL_BUDGET, Alg. 1 line 7 = PAPER.md:760; §3.6.1; "<10% error",
 "err on the side of under-predicting" PAPER.md:941-944).  Here the model is fitted to the
-engine's OWN device-timed steps (`qos_profile_step`), with features taken from the step's
-roofline work:
+engine's OWN device-timed steps (`qos_profile_step`) with features that follow the step's
+work and the engine's tiling:
 
-    t(batch) = G(T) + a * Bdec + b * Fpre + c
+    t(batch) = c0 * Wgemm(T) + c1 * T + c2 * Bdec + c3 * n_dec + c4 * [n_dec > 0] + c5 + c6 * Fpre
 
-* G(T): piecewise-linear in T = sum(chunk_len) + n_decode (hat basis on knots) — the dense
-  projections, norms, RoPE/append, LM head (their cost depends on T only, with the GEMM tile
-  steps of 128 rows);
-* Bdec = sum_j (ctx_j + 1): decode-attention KV bytes are proportional (HBM-bound);
+* Wgemm(T): sum over the four projections of (waves of 128 x BN tiles over the SMs) x (k-blocks
+  per tile) x BN/256 — the tensor-core GEMM time with the engine's tile-quantisation (the
+  same BN / split-K choice as csrc/gemm.cu), T = sum(chunk_len) + n_decode;
+* T: per-token elementwise work (norms, RoPE/append, embedding);
+* Bdec = sum_j (ctx_j + 1): decode-attention KV bytes (HBM-bound);
+* n_dec and [n_dec > 0]: per-decode and per-launch latency of the split-K decode attention;
 * Fpre = sum_c [len_c * kv_start_c + len_c (len_c + 1) / 2]: prefill-attention work.
 
-Least squares (numpy) over profiled points; `predict` is pure host arithmetic.  The north
-star asks iteration latency to be predictable within 5% across chunk sizes 256-8192.
+Least squares (numpy, relative weights) over profiled points; `predict` is host arithmetic.
+The north star asks iteration latency to be predictable within 5% across chunks 256-8192.
 """
 from __future__ import annotations
 
 import json
+import math
 from dataclasses import dataclass, field
 
 import numpy as np
 
-KNOTS = (1, 64, 128, 256, 512, 768, 1024, 1536, 2048, 3072, 4096, 5120, 6144, 7168, 8192, 8448)
+N_FEAT = 7
 
 
 @dataclass
@@ -38,66 +41,66 @@ class StepShape:
         return sum(n for _, n in self.chunks) + len(self.ctx)
 
 
-def features(s: StepShape, knots=KNOTS) -> np.ndarray:
-    T = s.T
-    k = np.asarray(knots, dtype=np.float64)
-    hat = np.zeros(len(k))
-    if T <= k[0]:
-        hat[0] = 1.0
-    elif T >= k[-1]:
-        hat[-1] = 1.0
-    else:
-        i = int(np.searchsorted(k, T) - 1)
-        w = (T - k[i]) / (k[i + 1] - k[i])
-        hat[i], hat[i + 1] = 1 - w, w
-    bdec = float(sum(c + 1 for c in s.ctx)) / 1e6
-    fpre = float(sum(n * ks + n * (n + 1) / 2 for ks, n in s.chunks)) / 1e7
-    return np.concatenate([hat, [bdec, fpre]])
+@dataclass(frozen=True)
+class GemmShapes:
+    """(N, K) of the QKV, O, gate/up and down projections of one TP rank + the SM count."""
+    gemms: tuple = ((6144, 4096), (4096, 4096), (28672, 4096), (4096, 14336))
+    num_sms: int = 148
+
+    @staticmethod
+    def for_model(d_model, n_heads, n_kv_heads, head_dim, ffn_dim, tp=1, num_sms=148):
+        nqkv = (n_heads + 2 * n_kv_heads) // tp * head_dim
+        return GemmShapes(((nqkv, d_model), (d_model, n_heads // tp * head_dim), (2 * ffn_dim // tp, d_model),
+                           (d_model, ffn_dim // tp)), num_sms)
+
+
+def _bn(M: int, N: int, sms: int) -> int:      # mirrors gemm_pick_bn (csrc/gemm.cu)
+    mt = (M + 127) // 128
+    return 256 if (mt * ((N + 255) // 256) >= sms and N % 256 == 0) else 128
+
+
+def gemm_work(T: int, g: GemmShapes) -> float:
+    if T <= 0:
+        return 0.0
+    tot = 0.0
+    for N, K in g.gemms:
+        bn = _bn(T, N, g.num_sms)
+        tiles = ((T + 127) // 128) * ((N + bn - 1) // bn)
+        ks = 1                                 # mirrors gemm_pick_ksplit
+        while tiles * ks * 2 <= g.num_sms + g.num_sms // 4 and (K // 64) // (ks * 2) >= 4:
+            ks *= 2
+        tot += math.ceil(tiles * ks / g.num_sms) * (K // 64 // ks) * (bn / 256)
+    return tot
+
+
+def features(s: StepShape, g: GemmShapes = GemmShapes()) -> np.ndarray:
+    nd = len(s.ctx)
+    return np.array([gemm_work(s.T, g) / 100.0, s.T / 1000.0, sum(c + 1 for c in s.ctx) / 1e6, nd / 100.0,
+                     1.0 if nd else 0.0, 1.0, sum(n * ks + n * (n + 1) / 2 for ks, n in s.chunks) / 1e7])
 
 
 class LatencyModel:
-    def __init__(self, knots=KNOTS):
-        self.knots = tuple(knots)
+    def __init__(self, shapes: GemmShapes = GemmShapes()):
+        self.shapes = shapes
         self.coef = None
 
     def fit(self, shapes, ms):
-        X = np.stack([features(s, self.knots) for s in shapes])
+        X = np.stack([features(s, self.shapes) for s in shapes])
         y = np.asarray(ms, dtype=np.float64)
-        # relative least squares (weights 1/y) so every chunk size counts the same
-        w = 1.0 / y
-        # only knots that carry weight enter the fit; the rest interpolate to neighbours
-        used = X[:, :len(self.knots)].sum(0) > 0
-        cols = np.concatenate([used, [True, True]])
-        coef, *_ = np.linalg.lstsq(X[:, cols] * w[:, None], y * w, rcond=None)
-        full = np.zeros(X.shape[1])
-        full[cols] = coef
-        # fill unused knots by linear interpolation between used ones
-        kx = np.asarray(self.knots, dtype=np.float64)
-        ui = np.where(used)[0]
-        if len(ui) >= 2:
-            full[:len(kx)] = np.interp(kx, kx[ui], full[ui])
-        self.coef = full
+        w = 1.0 / y                         # relative least squares: every point counts alike
+        self.coef, *_ = np.linalg.lstsq(X * w[:, None], y * w, rcond=None)
         return self
 
     def predict(self, s: StepShape) -> float:
-        return float(features(s, self.knots) @ self.coef)
-
-    def max_chunk(self, budget_ms: float, ctx, kv_start: int = 0, lo: int = 256, hi: int = 8192,
-                  step: int = 256, margin: float = 0.05) -> int:
-        """Largest chunk on the grid whose predicted step time fits budget*(1-margin); 0 if
-        none (a decode-only step).  The margin under-predicts chunk size."""
-        best = 0
-        for c in range(lo, hi + 1, step):
-            if self.predict(StepShape([(kv_start, c)], list(ctx))) <= budget_ms * (1 - margin):
-                best = c
-        return best
+        return float(features(s, self.shapes) @ self.coef)
 
     def to_json(self) -> str:
-        return json.dumps({"knots": list(self.knots), "coef": [float(x) for x in self.coef]})
+        return json.dumps({"gemms": [list(x) for x in self.shapes.gemms], "num_sms": self.shapes.num_sms,
+                           "coef": [float(x) for x in self.coef]})
 
     @classmethod
     def from_json(cls, s: str) -> "LatencyModel":
         d = json.loads(s)
-        m = cls(d["knots"])
+        m = cls(GemmShapes(tuple(tuple(x) for x in d["gemms"]), d["num_sms"]))
         m.coef = np.asarray(d["coef"])
         return m

@@ -1,0 +1,44 @@
+"""Latency model (dynamic chunking predictor) on CPU: recovers a known linear cost, mirrors the
+engine's GEMM tiling, and (when the committed profile exists) predicts the measured B200
+latency table within the north star's 5% on most points."""
+import json
+import os
+
+import numpy as np
+
+from paper_conf_asplos_goelmkar26_b200.latency_model import GemmShapes, LatencyModel, StepShape, features, gemm_work
+
+PROF = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles", "latency_table_r1.json")
+
+
+def test_recovers_known_coefficients():
+    rng = np.random.default_rng(0)
+    true = np.array([2.0, 3.0, 20.0, 0.5, 1.0, 4.0, 9.0])
+    shapes = []
+    for _ in range(120):
+        c = int(rng.integers(0, 8193))
+        nd = int(rng.integers(0, 257))
+        shapes.append(StepShape([(int(rng.integers(0, 4097)), c)] if c else [], list(rng.integers(1024, 8193, nd))))
+    y = [features(s) @ true for s in shapes if s.T > 0]
+    m = LatencyModel().fit([s for s in shapes if s.T > 0], y)
+    pred = [m.predict(s) for s in shapes if s.T > 0]
+    assert np.allclose(pred, y, rtol=1e-8)
+    m2 = LatencyModel.from_json(m.to_json())
+    assert abs(m2.predict(shapes[0]) - m.predict(shapes[0])) < 1e-9
+
+
+def test_gemm_work_is_tile_quantised():
+    g = GemmShapes()
+    assert gemm_work(2048, g) == gemm_work(2048 - 100, g)        # same 16 M-tiles
+    w = [gemm_work(t, g) for t in range(128, 8449, 128)]
+    assert all(a <= b for a, b in zip(w, w[1:]))                   # steps, never decreasing
+    assert len(set(w)) > 20
+    assert gemm_work(8448, g) > 3 * gemm_work(2176, g)
+
+
+def test_committed_profile_predictability():
+    if not os.path.exists(PROF):
+        return
+    d = json.load(open(PROF))
+    assert d["test_points"] >= 100
+    assert d["within_5pct"] >= 0.9 and d["test_rel_err_max"] < 0.1
