@@ -108,6 +108,7 @@ __global__ void __launch_bounds__(kFaThreads, 2)
   uint64_t* s_full = bar + 8;
   uint64_t* p_full = bar + 10;
   uint64_t* o_full = bar + 12;
+  uint64_t* o_final = bar + 13;   // completes once, when the last PV has landed
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 14);
 
   const PrefillItem it = items[blockIdx.x];
@@ -128,6 +129,7 @@ __global__ void __launch_bounds__(kFaThreads, 2)
       mbar_init(&p_full[i], 128);
     }
     mbar_init(o_full, 1);
+    mbar_init(o_final, 1);
     fence_mbar_init();
   }
   if (warp == 1) tmem_alloc<C::kTmemCols>(tmem_slot);
@@ -226,6 +228,7 @@ __global__ void __launch_bounds__(kFaThreads, 2)
         if (j >= 1) issue_pv(j - 1);   // O += P_{j-1} V_{j-1} while the softmax works on S_j
       }
       issue_pv(ntiles - 1);
+      umma_commit(o_final);
     }
   } else {
     // ------------------------------------------------------------------ softmax (warps 2..5)
@@ -316,9 +319,9 @@ __global__ void __launch_bounds__(kFaThreads, 2)
       mbar_arrive(&p_full[sb]);
     }
     // epilogue: O / l
-    // PV_{n-3} precedes QK_{n-1} (awaited), so o_full is at phase >= n-2: wait n-2, then n-1
-    if (ntiles >= 2) mbar_wait(o_full, (ntiles - 2) & 1);
-    mbar_wait(o_full, (ntiles - 1) & 1);
+    // o_full may be anywhere in phases n-2..n here (its waits are skipped when no rescale is
+    // needed), so a parity wait on it could alias; the dedicated o_final barrier completes once
+    mbar_wait(o_final, 0);
     tc_fence_after();
     const float inv = (l > 0.f) ? 1.f / l : 0.f;
 #pragma unroll 1
