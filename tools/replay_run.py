@@ -1,0 +1,91 @@
+"""configs[4]: trace replay on Llama-3-8B shapes driving the QoServe scheduler.
+
+  python tools/replay_run.py --mode engine --dataset azure_conv --qps 10,20,30 --duration 60
+  python tools/replay_run.py --mode model  --dataset azure_code --qps 5,10,20,30,40 --duration 1800
+
+engine: every step is a real device-timed qos_hybrid_step (virtual clock += measured ms); the
+        scheduler's latency model is fitted to a quick qos_profile_step sweep of this engine.
+model:  steps are priced by the latency model committed in profiles/latency_table_r1.json
+        (fitted to the B200 profile) — fast what-if replays over long horizons.
+Prints one JSON line per QPS and a summary with goodput = max QPS with <= 1% violations
+(PAPER.md:1152-1155).
+"""
+import argparse
+import json
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import synth  # noqa: E402
+from paper_conf_asplos_goelmkar26_b200.latency_model import LatencyModel, StepShape  # noqa: E402
+from paper_conf_asplos_goelmkar26_b200.replay import EngineExecutor, ModelExecutor, replay  # noqa: E402
+from paper_conf_asplos_goelmkar26_b200.scheduler import QoServeScheduler, SchedulerConfig  # noqa: E402
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--mode", default="engine", choices=["engine", "model"])
+    ap.add_argument("--dataset", default="azure_conv")
+    ap.add_argument("--qps", default="10,20,30")
+    ap.add_argument("--duration", type=float, default=60.0)
+    ap.add_argument("--alpha", type=float, default=8.0)
+    ap.add_argument("--max-chunk", type=int, default=4096)
+    ap.add_argument("--out", default=None)
+    a = ap.parse_args()
+    results = []
+    eng = None
+    if a.mode == "engine":
+        import torch
+        from paper_conf_asplos_goelmkar26_b200 import qoserve as q
+        from paper_conf_asplos_goelmkar26_b200.presets import preset
+        torch.cuda.set_device(0)
+        cfg = q.model_cfg(**preset("llama3-8b"), num_blocks=int(140e9 / (32 * 2 * 8 * 128 * 2 * 16)),
+                          max_seq_len=8192, max_requests=4096, max_batch_tokens=a.max_chunk + 512,
+                          max_batch_rows=257)
+        eng = q.Engine(cfg)
+        eng.qos_engine_load_synthetic(0)
+        shapes, ms = [], []
+        eng.qos_profile_step(2048, [2048] * 64, reps=5, warmup=5)
+        for c in (0, 256, 512, 1024, 2048, 3072, 4096):
+            for nd in (0, 16, 64, 128, 256):
+                if (c == 0 and nd == 0) or c > a.max_chunk:
+                    continue
+                t, _ = eng.qos_profile_step(c, [1536] * nd, reps=3, warmup=3)
+                shapes.append(StepShape([(0, c)] if c else [], [1536] * nd))
+                ms.append(t)
+        model = LatencyModel().fit(shapes, ms)
+    else:
+        model = LatencyModel.from_json(json.dumps(
+            json.load(open(os.path.join(ROOT, "profiles", "latency_table_r1.json")))["refit"]["model_json"]))
+
+    def pred(chunks, ctx):
+        return model.predict(StepShape(list(chunks), list(ctx)))
+
+    for qps in [float(x) for x in a.qps.split(",")]:
+        tr = synth.trace(qps, a.duration, a.dataset)
+        sched = QoServeScheduler(SchedulerConfig(alpha_ms_per_token=a.alpha, max_chunk=a.max_chunk), pred)
+        if a.mode == "engine":
+            ex = EngineExecutor(eng, 128256, lambda r, s, n: synth.request_tokens(r, n, 128256, start=s))
+        else:
+            ex = ModelExecutor(pred)
+        out = replay(tr, sched, ex)
+        out.update({"qps": qps, "dataset": a.dataset, "mode": a.mode, "duration_s": a.duration, "alpha": a.alpha})
+        series = out.pop("chunk_series", None)
+        print(json.dumps(out), flush=True)
+        out["chunk_series"] = series
+        results.append(out)
+    ok = [r["qps"] for r in results if r["violations_pct"] <= 1.0]
+    summary = {"goodput_qps": max(ok) if ok else 0.0, "dataset": a.dataset, "mode": a.mode,
+               "qps_tested": [r["qps"] for r in results]}
+    print(json.dumps(summary), flush=True)
+    if a.out:
+        json.dump({"summary": summary, "runs": results}, open(a.out, "w"), indent=1)
+    if eng is not None:
+        eng.close()
+
+
+if __name__ == "__main__":
+    main()
