@@ -138,8 +138,8 @@ static WeightLayout weight_layout(const qos_model_cfg& c, const Shard& s) {
 }
 
 struct WsLayout {
-  size_t resid, h, qkv, attn, act, hR, logits, logits_loc, argmax, partials, counters, gemm_part, gemm_cnt, meta[2], dbg,
-      total;
+  size_t resid, h, qkv, attn, act, hR, logits, logits_loc, argmax, partials, counters, gemm_part, gemm_cnt, gemm_part2,
+      gemm_cnt2, meta[2], dbg, total;
   size_t meta_bytes;
   int max_items;
 };
@@ -171,6 +171,8 @@ static WsLayout ws_layout(const qos_model_cfg& c, const Shard& s, int tp) {
   w.counters = take(Rm * size_t(s.Hkv) * 4);
   w.gemm_part = take(size_t(kGemmMaxUnits) * 128 * 256 * 4);
   w.gemm_cnt = take(size_t(kGemmMaxTiles) * 4);
+  w.gemm_part2 = take(size_t(kGemmMaxUnits) * 128 * 256 * 4);   // second stream's split-K workspace
+  w.gemm_cnt2 = take(size_t(kGemmMaxTiles) * 4);
   // metadata: tokens, pos, slot [Tm]; logit rows [Rm]; prefill items; decode items/rows; table updates
   const int ppt = prefill_tc_positions_per_tile(int(group));
   const size_t max_pitems = (Tm / ppt + Rm + 1) * size_t(s.Hkv);
@@ -232,7 +234,10 @@ struct qos_engine {
   int meta_cur = 0;
   cudaStream_t stream = nullptr;  // internal stream for synchronous calls
   cudaStream_t side = nullptr;    // high-priority stream: prefill attention overlapped with decode
-  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr, ev_fork2 = nullptr, ev_join2 = nullptr;
+  bool dual_stream = false;       // QOS_DUAL=1: prefill rows and decode rows on two streams
+  int dual_min_prefill = 512, dual_min_decode = 16;
+  int dual_sms_pre = 0, dual_sms_dec = 0;  // SM budgets of the two streams' GEMMs (0 = all)
   bool overlap_attn = true;       // QOS_OVERLAP_ATTN=0 serialises a7 and a8 (for measurement)
   bool gemm_splitk = true;        // QOS_GEMM_SPLITK=0 disables split-K for small-M GEMMs
   // timing
@@ -540,16 +545,39 @@ int allreduce_bf16(qos_engine* e, void* buf, size_t count, cudaStream_t st) {
 }
 
 // The layer loop.  `dm` = device metadata block of this step.
+// One row range of the batch pushed through all layers on one stream.  `pre` / `dec` select
+// which attention work lists the range owns.
+struct Seg {
+  int row0, n;
+  cudaStream_t st;
+  bool pre, dec;
+  float* gpart;  // split-K workspace of this stream
+  int* gcnt;
+  int sms;       // SM budget of this stream's GEMMs (0 = all)
+};
+
+int gemm_seg(qos_engine* e, const Seg& g, const CUtensorMap& ta, const CUtensorMap (&tb)[2], int64_t N, int64_t K,
+             int epi, void* C, int64_t ldc, const float* bias) {
+  const int sms = g.sms > 0 ? g.sms : e->num_sms;
+  const int bn = gemm_pick_bn(g.n, N, epi, sms);
+  const int ks = e->gemm_splitk ? gemm_pick_ksplit(g.n, N, K, bn, sms, kGemmMaxUnits) : 1;
+  count_launch();
+  const size_t esz = (epi == EPI_STORE_F32 || epi == EPI_ADD_F32) ? 4 : 2;
+  return gemm_run(ta, tb[bn == 256 ? 1 : 0], bn, g.n, N, K, epi, reinterpret_cast<uint8_t*>(C) + size_t(g.row0) * ldc * esz,
+                  ldc, bias, sms, g.st, ks, g.gpart, g.gcnt, g.row0, sms);
+}
+
+// The layer loop.  `dm` = device metadata block of this step.
 int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int logits_dtype, int32_t* next_tokens,
                bool out_device, cudaStream_t st) {
   const auto& c = e->cfg;
   const int d = c.d_model, hd = c.head_dim, T = m.T, R = m.R;
   const auto& s = e->wsl;
   float* resid = reinterpret_cast<float*>(e->ws + s.resid);
-  void* h = e->ws + s.h;
+  __nv_bfloat16* h = reinterpret_cast<__nv_bfloat16*>(e->ws + s.h);
   __nv_bfloat16* qkv = reinterpret_cast<__nv_bfloat16*>(e->ws + s.qkv);
   void* attn = e->ws + s.attn;
-  void* act = e->ws + s.act;
+  __nv_bfloat16* act = reinterpret_cast<__nv_bfloat16*>(e->ws + s.act);
   void* hR = e->ws + s.hR;
   const int32_t* tok = reinterpret_cast<const int32_t*>(dm + m.o_tok);
   const int32_t* pos = reinterpret_cast<const int32_t*>(dm + m.o_pos);
@@ -557,10 +585,6 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
   const int32_t* rows = reinterpret_cast<const int32_t*>(dm + m.o_rows);
   const size_t plane = e->plane_elems;
   const bool tp = e->tp_size > 1;
-  {
-    TimerScope ts(e, QOS_T_EMBED, st);
-    QOS_CU(launch_embed_rmsnorm(tok, W(e, e->wl.emb), W(e, e->wl.layers[0].ln1), resid, h, T, d, c.rms_eps, st));
-  }
   AttnLaunch al;
   al.q = qkv;
   al.q_ld = e->nqkv;
@@ -575,89 +599,120 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
   al.tables = e->d_tables;
   al.table_w = e->table_w;
   al.scale_log2 = float(1.4426950408889634 / std::sqrt(double(hd)));
+  const int n_pre_rows = T - m.n_decode;
+  float* gpart0 = reinterpret_cast<float*>(e->ws + s.gemm_part);
+  int* gcnt0 = reinterpret_cast<int*>(e->ws + s.gemm_cnt);
+  // dual mode: the prefill rows and the decode rows are independent requests that share only the
+  // weights, so they run as two sub-batches on two streams — the tensor-bound projections of the
+  // chunk overlap the HBM-bound decode attention (and the weight-bound decode-row GEMMs)
+  const bool dual = !tp && e->dual_stream && n_pre_rows >= e->dual_min_prefill && m.n_decode >= e->dual_min_decode;
+  Seg segs[2];
+  int nseg = 0;
+  if (dual) {
+    segs[nseg++] = Seg{0, n_pre_rows, st, true, false, gpart0, gcnt0, e->dual_sms_pre};
+    segs[nseg++] = Seg{n_pre_rows, m.n_decode, e->side, false, true,
+                       reinterpret_cast<float*>(e->ws + s.gemm_part2), reinterpret_cast<int*>(e->ws + s.gemm_cnt2),
+                       e->dual_sms_dec};
+    QOS_CU(cudaEventRecord(e->ev_fork, st));
+    QOS_CU(cudaStreamWaitEvent(e->side, e->ev_fork, 0));
+  } else {
+    segs[nseg++] = Seg{0, T, st, m.n_pitems > 0, m.n_ditems > 0, gpart0, gcnt0, 0};
+  }
   for (int l = 0; l < c.n_layers; ++l) {
     const auto& L = e->wl.layers[l];
     const auto& M = e->lmaps[l];
-    if (l > 0 && !tp) {  // (tp: ln1 was applied by the add+norm after the previous all-reduce)
-      TimerScope ts(e, QOS_T_NORM, st);
-      QOS_CU(launch_rmsnorm(resid, W(e, L.ln1), h, T, d, c.rms_eps, st));
-    }
-    {
-      TimerScope ts(e, QOS_T_GEMM_QKV, st);
-      QOS_TRY(gemm(e, e->a_h, M.qkv, T, e->nqkv, d, c.qkv_bias ? EPI_BIAS_BF16 : EPI_STORE_BF16, qkv, e->nqkv,
-                   c.qkv_bias ? reinterpret_cast<const float*>(e->w + L.bqkv) : nullptr, st));
-    }
     __nv_bfloat16* kpl = reinterpret_cast<__nv_bfloat16*>(e->kv) + (size_t(l) * 2 + 0) * plane;
     __nv_bfloat16* vpl = reinterpret_cast<__nv_bfloat16*>(e->kv) + (size_t(l) * 2 + 1) * plane;
-    {
-      TimerScope ts(e, QOS_T_ROPE_APPEND, st);
-      QOS_CU(launch_rope_append(qkv, e->nqkv, qkv, e->nqkv, pos, slot, e->rope_tab, kpl, vpl, T, e->sh.H, e->sh.Hkv,
-                                hd, st));
-    }
     al.layer = l;
-    // a7 || a8: prefill attention (tensor-bound) and decode attention (HBM-bound) read the same
-    // freshly appended cache and write disjoint rows of `attn`, so they run concurrently: the
-    // prefill tiles on a high-priority side stream, the decode split-K items on the step stream.
-    const bool overlap = e->overlap_attn && m.n_pitems && m.n_ditems;
-    cudaStream_t pst = overlap ? e->side : st;
-    if (overlap) {
-      QOS_CU(cudaEventRecord(e->ev_fork, st));
-      QOS_CU(cudaStreamWaitEvent(e->side, e->ev_fork, 0));
-    }
-    if (m.n_pitems) {
-      TimerScope ts(e, QOS_T_PREFILL_ATTN, pst);
-      QOS_CU(launch_prefill_attention_tc(al, reinterpret_cast<const PrefillItem*>(dm + m.o_pitems), m.n_pitems, pst));
-    }
-    if (m.n_ditems) {
-      TimerScope ts(e, QOS_T_DECODE_ATTN, st);
-      QOS_CU(launch_decode_attention(al, reinterpret_cast<const DecodeItem*>(dm + m.o_ditems), m.n_ditems,
-                                     reinterpret_cast<float*>(e->ws + s.partials),
-                                     reinterpret_cast<int*>(e->ws + s.counters), st));
-    }
-    if (overlap) {
-      QOS_CU(cudaEventRecord(e->ev_join, e->side));
-      QOS_CU(cudaStreamWaitEvent(st, e->ev_join, 0));
-    }
-    if (!tp) {
-      TimerScope ts(e, QOS_T_GEMM_O, st);
-      QOS_TRY(gemm(e, e->a_attn, M.o, T, d, e->sh.H * hd, EPI_ADD_F32, resid, d, nullptr, st));
-    } else {
-      {
-        TimerScope ts(e, QOS_T_GEMM_O, st);
-        QOS_TRY(gemm(e, e->a_attn, M.o, T, d, e->sh.H * hd, EPI_STORE_BF16, h, d, nullptr, st));
-      }
-      TimerScope ts(e, QOS_T_ALLREDUCE, st);
-      QOS_TRY(allreduce_bf16(e, h, size_t(T) * d, st));
-    }
-    {
-      TimerScope ts(e, QOS_T_NORM, st);
-      if (tp) QOS_CU(launch_add_rmsnorm(resid, h, W(e, L.ln2), h, T, d, c.rms_eps, st));
-      else QOS_CU(launch_rmsnorm(resid, W(e, L.ln2), h, T, d, c.rms_eps, st));
-    }
-    {
-      TimerScope ts(e, QOS_T_GEMM_GATEUP, st);
-      QOS_TRY(gemm(e, e->a_h, M.gu, T, 2 * e->sh.F, d, EPI_SILU_GATE, act, e->sh.F, nullptr, st));
-    }
-    if (!tp) {
-      TimerScope ts(e, QOS_T_GEMM_DOWN, st);
-      QOS_TRY(gemm(e, e->a_act, M.d, T, d, e->sh.F, EPI_ADD_F32, resid, d, nullptr, st));
-    } else {
-      {
-        TimerScope ts(e, QOS_T_GEMM_DOWN, st);
-        QOS_TRY(gemm(e, e->a_act, M.d, T, d, e->sh.F, EPI_STORE_BF16, h, d, nullptr, st));
+    for (int si = 0; si < nseg; ++si) {
+      const Seg& g = segs[si];
+      const cudaStream_t gs = g.st;
+      const size_t r0 = size_t(g.row0);
+      if (l == 0) {
+        TimerScope ts(e, QOS_T_EMBED, gs);
+        QOS_CU(launch_embed_rmsnorm(tok + r0, W(e, e->wl.emb), W(e, L.ln1), resid + r0 * d, h + r0 * d, g.n, d,
+                                    c.rms_eps, gs));
+      } else if (!tp) {  // (tp: ln1 was applied by the add+norm after the previous all-reduce)
+        TimerScope ts(e, QOS_T_NORM, gs);
+        QOS_CU(launch_rmsnorm(resid + r0 * d, W(e, L.ln1), h + r0 * d, g.n, d, c.rms_eps, gs));
       }
       {
-        TimerScope ts(e, QOS_T_ALLREDUCE, st);
-        QOS_TRY(allreduce_bf16(e, h, size_t(T) * d, st));
+        TimerScope ts(e, QOS_T_GEMM_QKV, gs);
+        QOS_TRY(gemm_seg(e, g, e->a_h, M.qkv, e->nqkv, d, c.qkv_bias ? EPI_BIAS_BF16 : EPI_STORE_BF16, qkv, e->nqkv,
+                         c.qkv_bias ? reinterpret_cast<const float*>(e->w + L.bqkv) : nullptr));
       }
-      if (l + 1 < c.n_layers) {
-        TimerScope ts(e, QOS_T_NORM, st);
-        QOS_CU(launch_add_rmsnorm(resid, h, W(e, e->wl.layers[l + 1].ln1), h, T, d, c.rms_eps, st));
+      {
+        TimerScope ts(e, QOS_T_ROPE_APPEND, gs);
+        QOS_CU(launch_rope_append(qkv + r0 * e->nqkv, e->nqkv, qkv + r0 * e->nqkv, e->nqkv, pos + r0, slot + r0,
+                                  e->rope_tab, kpl, vpl, g.n, e->sh.H, e->sh.Hkv, hd, gs));
+      }
+      // a7 || a8: within one segment, the prefill tiles go to the high-priority side stream and
+      // the decode split-K items stay on the segment's stream (disjoint rows of `attn`)
+      const bool overlap = !dual && e->overlap_attn && g.pre && g.dec;
+      cudaStream_t pst = overlap ? e->side : gs;
+      if (overlap) {
+        QOS_CU(cudaEventRecord(e->ev_fork2, gs));
+        QOS_CU(cudaStreamWaitEvent(e->side, e->ev_fork2, 0));
+      }
+      if (g.pre && m.n_pitems) {
+        TimerScope ts(e, QOS_T_PREFILL_ATTN, pst);
+        QOS_CU(launch_prefill_attention_tc(al, reinterpret_cast<const PrefillItem*>(dm + m.o_pitems), m.n_pitems, pst));
+      }
+      if (g.dec && m.n_ditems) {
+        TimerScope ts(e, QOS_T_DECODE_ATTN, gs);
+        QOS_CU(launch_decode_attention(al, reinterpret_cast<const DecodeItem*>(dm + m.o_ditems), m.n_ditems,
+                                       reinterpret_cast<float*>(e->ws + s.partials),
+                                       reinterpret_cast<int*>(e->ws + s.counters), gs));
+      }
+      if (overlap) {
+        QOS_CU(cudaEventRecord(e->ev_join2, e->side));
+        QOS_CU(cudaStreamWaitEvent(gs, e->ev_join2, 0));
+      }
+      if (!tp) {
+        TimerScope ts(e, QOS_T_GEMM_O, gs);
+        QOS_TRY(gemm_seg(e, g, e->a_attn, M.o, d, e->sh.H * hd, EPI_ADD_F32, resid, d, nullptr));
       } else {
-        TimerScope ts(e, QOS_T_NORM, st);
-        QOS_CU(launch_add_f32(resid, h, size_t(T) * d, st));
+        {
+          TimerScope ts(e, QOS_T_GEMM_O, gs);
+          QOS_TRY(gemm_seg(e, g, e->a_attn, M.o, d, e->sh.H * hd, EPI_STORE_BF16, h, d, nullptr));
+        }
+        TimerScope ts(e, QOS_T_ALLREDUCE, gs);
+        QOS_TRY(allreduce_bf16(e, h, size_t(T) * d, gs));
+      }
+      {
+        TimerScope ts(e, QOS_T_NORM, gs);
+        if (tp) QOS_CU(launch_add_rmsnorm(resid, h, W(e, L.ln2), h, T, d, c.rms_eps, gs));
+        else QOS_CU(launch_rmsnorm(resid + r0 * d, W(e, L.ln2), h + r0 * d, g.n, d, c.rms_eps, gs));
+      }
+      {
+        TimerScope ts(e, QOS_T_GEMM_GATEUP, gs);
+        QOS_TRY(gemm_seg(e, g, e->a_h, M.gu, 2 * e->sh.F, d, EPI_SILU_GATE, act, e->sh.F, nullptr));
+      }
+      if (!tp) {
+        TimerScope ts(e, QOS_T_GEMM_DOWN, gs);
+        QOS_TRY(gemm_seg(e, g, e->a_act, M.d, d, e->sh.F, EPI_ADD_F32, resid, d, nullptr));
+      } else {
+        {
+          TimerScope ts(e, QOS_T_GEMM_DOWN, gs);
+          QOS_TRY(gemm_seg(e, g, e->a_act, M.d, d, e->sh.F, EPI_STORE_BF16, h, d, nullptr));
+        }
+        {
+          TimerScope ts(e, QOS_T_ALLREDUCE, gs);
+          QOS_TRY(allreduce_bf16(e, h, size_t(T) * d, gs));
+        }
+        if (l + 1 < c.n_layers) {
+          TimerScope ts(e, QOS_T_NORM, gs);
+          QOS_CU(launch_add_rmsnorm(resid, h, W(e, e->wl.layers[l + 1].ln1), h, T, d, c.rms_eps, gs));
+        } else {
+          TimerScope ts(e, QOS_T_NORM, gs);
+          QOS_CU(launch_add_f32(resid, h, size_t(T) * d, gs));
+        }
       }
     }
+  }
+  if (dual) {
+    QOS_CU(cudaEventRecord(e->ev_join, e->side));
+    QOS_CU(cudaStreamWaitEvent(st, e->ev_join, 0));
   }
   // final norm on the R logit rows + LM head
   {
@@ -831,7 +886,8 @@ int qos_engine_create(const qos_model_cfg* cfg, int device, int tp_rank, int tp_
   if (cudaMemset(e->kv, 0, e->kv_bytes) != cudaSuccess) return fail(set_error(QOS_ERR_CUDA, "kv memset"));
   // split-K arrival counters start at zero; the combining item / reducing CTA resets its counter
   if (cudaMemset(e->ws + e->wsl.counters, 0, size_t(cfg->max_batch_rows) * e->sh.Hkv * 4) != cudaSuccess ||
-      cudaMemset(e->ws + e->wsl.gemm_cnt, 0, size_t(kGemmMaxTiles) * 4) != cudaSuccess)
+      cudaMemset(e->ws + e->wsl.gemm_cnt, 0, size_t(kGemmMaxTiles) * 4) != cudaSuccess ||
+      cudaMemset(e->ws + e->wsl.gemm_cnt2, 0, size_t(kGemmMaxTiles) * 4) != cudaSuccess)
     return fail(set_error(QOS_ERR_CUDA, "counter memset"));
   if (cudaMalloc(&e->d_tables, size_t(cfg->max_requests) * e->table_w * 4) != cudaSuccess)
     return fail(set_error(QOS_ERR_OOM, "block tables"));
@@ -857,12 +913,19 @@ int qos_engine_create(const qos_model_cfg* cfg, int device, int tp_rank, int tp_
   cudaStreamCreateWithFlags(&e->stream, cudaStreamNonBlocking);
   if (const char* ov = getenv("QOS_OVERLAP_ATTN")) e->overlap_attn = atoi(ov) != 0;
   if (const char* sk = getenv("QOS_GEMM_SPLITK")) e->gemm_splitk = atoi(sk) != 0;
+  if (const char* du = getenv("QOS_DUAL")) e->dual_stream = atoi(du) != 0;
+  if (const char* a = getenv("QOS_DUAL_MIN_PREFILL")) e->dual_min_prefill = atoi(a);
+  if (const char* a = getenv("QOS_DUAL_MIN_DECODE")) e->dual_min_decode = atoi(a);
+  if (const char* a = getenv("QOS_DUAL_SMS_PRE")) e->dual_sms_pre = atoi(a);
+  if (const char* a = getenv("QOS_DUAL_SMS_DEC")) e->dual_sms_dec = atoi(a);
   {
     int lo = 0, hi = 0;
     cudaDeviceGetStreamPriorityRange(&lo, &hi);
     cudaStreamCreateWithPriority(&e->side, cudaStreamNonBlocking, hi);
     cudaEventCreateWithFlags(&e->ev_fork, cudaEventDisableTiming);
     cudaEventCreateWithFlags(&e->ev_join, cudaEventDisableTiming);
+    cudaEventCreateWithFlags(&e->ev_fork2, cudaEventDisableTiming);
+    cudaEventCreateWithFlags(&e->ev_join2, cudaEventDisableTiming);
   }
   e->free_heap.resize(size_t(cfg->num_blocks));
   for (int64_t i = 0; i < cfg->num_blocks; ++i) e->free_heap[size_t(i)] = int32_t(i);  // sorted = valid min-heap
@@ -902,6 +965,8 @@ int qos_engine_destroy(qos_engine_t* e) {
   if (e->side) cudaStreamDestroy(e->side);
   if (e->ev_fork) cudaEventDestroy(e->ev_fork);
   if (e->ev_join) cudaEventDestroy(e->ev_join);
+  if (e->ev_fork2) cudaEventDestroy(e->ev_fork2);
+  if (e->ev_join2) cudaEventDestroy(e->ev_join2);
   delete e;
   return QOS_OK;
 }

@@ -46,6 +46,7 @@ struct GemmArgs {
   const float* bias;
   float* part;      // split-K partials [unit][128][BN] fp32 (ksplit > 1)
   int* counters;    // split-K arrival counter per tile (ksplit > 1), zero between launches
+  int a_row0;       // first row of A (TMA coordinate offset): GEMM over a row range of a buffer
 };
 
 // ---- epilogue stores of one thread's 32 consecutive accumulator columns of one row
@@ -166,7 +167,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
           mbar_wait(&empty[stage], phase ^ 1);
           uint8_t* sa = smem + stage * Cfg::kStageBytes;
           mbar_arrive_expect_tx(&full[stage], Cfg::kStageBytes);
-          tma_load_2d_hint(sa, &tmA, &full[stage], kb * kBK, m_t * kBM, pol_a);
+          tma_load_2d_hint(sa, &tmA, &full[stage], kb * kBK, p.a_row0 + m_t * kBM, pol_a);
           tma_load_2d_hint(sa + Cfg::kABytes, &tmB, &full[stage], kb * kBK, n_t * BN, pol_b);
           if (++stage == S) { stage = 0; phase ^= 1; }
         }
@@ -424,7 +425,8 @@ int gemm_pick_ksplit(int64_t M, int64_t N, int64_t K, int bn, int num_sms, int64
 }
 
 int gemm_run(const CUtensorMap& ta, const CUtensorMap& tb, int bn, int64_t M, int64_t N, int64_t K, int epi, void* C,
-             int64_t ldc, const float* bias, int num_sms, cudaStream_t st, int ksplit, float* part, int* counters) {
+             int64_t ldc, const float* bias, int num_sms, cudaStream_t st, int ksplit, float* part, int* counters,
+             int a_row0, int max_ctas) {
   GemmArgs a;
   a.M = int(M);
   a.N = int(N);
@@ -437,9 +439,11 @@ int gemm_run(const CUtensorMap& ta, const CUtensorMap& tb, int bn, int64_t M, in
   a.bias = bias;
   a.part = part;
   a.counters = counters;
+  a.a_row0 = a_row0;
   if (a.ksplit > 1 && (!part || !counters)) return set_error(QOS_ERR_INVALID_ARG, "gemm: split-K needs workspace");
   const int tiles = a.mt * a.nt * a.ksplit;
-  const int grid = tiles < num_sms ? tiles : num_sms;
+  int grid = tiles < num_sms ? tiles : num_sms;
+  if (max_ctas > 0 && grid > max_ctas) grid = max_ctas;   // SM budget (co-scheduled streams)
   cudaError_t e = cudaSuccess;
 #define QOS_GEMM_CASE(BNV, EPIV) \
   if (bn == BNV && epi == EPIV) e = launch_gemm_t<BNV, EPIV>(ta, tb, a, grid, st); else

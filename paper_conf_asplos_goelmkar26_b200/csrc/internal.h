@@ -30,7 +30,7 @@ int gemm_pick_ksplit(int64_t M, int64_t N, int64_t K, int bn, int num_sms, int64
 // counters (zero-initialised; each reducing CTA resets its own) — deterministic reduction order
 int gemm_run(const CUtensorMap& ta, const CUtensorMap& tb, int bn, int64_t M, int64_t N, int64_t K, int epi, void* C,
              int64_t ldc, const float* bias, int num_sms, cudaStream_t st, int ksplit = 1, float* part = nullptr,
-             int* counters = nullptr);
+             int* counters = nullptr, int a_row0 = 0, int max_ctas = 0);
 
 // ------------------------------------------------------------------ synthetic generator (gen.cu)
 enum GenKind { GEN_LINEAR = 0, GEN_EMBED = 1, GEN_NORM = 2, GEN_BIAS = 3 };
