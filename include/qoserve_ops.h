@@ -51,12 +51,12 @@ int qos_kv_write(qos_engine_t* eng, int32_t layer, int64_t req, int32_t pos0, in
 int qos_kv_read(qos_engine_t* eng, int32_t layer, int64_t req, int32_t pos0, int32_t n,
                 uint16_t* k_bf16, uint16_t* v_bf16);
 
-/* a5 + a6: RoPE on q and k at each token's position, then append k and v to the paged cache
- * at `layer`, for the token rows of `batch` (chunks then decodes, T rows).
- * qkv: host bf16 [T][(H_local + 2 Hkv_local) * hd] (q | k | v per row, pre-RoPE);
+/* a4 + a5 + a6 (fused): the layer's QKV projection of normalised activations h (host bf16
+ * [T][d], T = token rows of `batch`, chunks then decodes) with RoPE on q and k at each row's
+ * position and k, v appended to the paged cache at `layer` — the epilogue the step uses.
  * q_out: host bf16 [T][H_local * hd] post-RoPE q.  Does not change cached lengths.  Synchronous. */
-int qos_op_rope_kv_append(qos_engine_t* eng, int32_t layer, const qos_batch* batch,
-                          const uint16_t* qkv_bf16, uint16_t* q_out_bf16);
+int qos_op_qkv_rope_append(qos_engine_t* eng, int32_t layer, const qos_batch* batch,
+                           const uint16_t* h_bf16, uint16_t* q_out_bf16);
 
 /* a7 + a8: attention of the batch's token rows at `layer` over the paged cache (which must
  * already hold every key the rows attend to: chunk keys 0..kv_start+len-1, decode keys

@@ -55,6 +55,26 @@ QOS_DEV float ex2(float x) {  // MUFU.EX2 (flush-to-zero; arguments are <= 8 her
   return y;
 }
 
+// packed fp32 pair arithmetic (sm_100: FFMA2 / FADD2)
+QOS_DEV float2 fma2(float2 a, float2 b, float2 c) {
+  float2 d;
+  asm("{\n\t.reg .b64 ra, rb, rc, rd;\n\t"
+      "mov.b64 ra, {%2, %3};\n\tmov.b64 rb, {%4, %5};\n\tmov.b64 rc, {%6, %7};\n\t"
+      "fma.rn.f32x2 rd, ra, rb, rc;\n\tmov.b64 {%0, %1}, rd;\n\t}"
+      : "=f"(d.x), "=f"(d.y)
+      : "f"(a.x), "f"(a.y), "f"(b.x), "f"(b.y), "f"(c.x), "f"(c.y));
+  return d;
+}
+QOS_DEV float2 add2(float2 a, float2 b) {
+  float2 d;
+  asm("{\n\t.reg .b64 ra, rb, rd;\n\t"
+      "mov.b64 ra, {%2, %3};\n\tmov.b64 rb, {%4, %5};\n\t"
+      "add.rn.f32x2 rd, ra, rb;\n\tmov.b64 {%0, %1}, rd;\n\t}"
+      : "=f"(d.x), "=f"(d.y)
+      : "f"(a.x), "f"(a.y), "f"(b.x), "f"(b.y));
+  return d;
+}
+
 // D[tmem] (+)= A[tmem] · B[smem desc]   (kind::f16, A = bf16 pairs packed in 32-bit columns)
 QOS_DEV void umma_bf16_ts(uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc, uint32_t idesc, uint32_t accumulate) {
   asm volatile(
@@ -245,22 +265,21 @@ __global__ void __launch_bounds__(kFaThreads, 2)
       // masking only where a key of this tile can exceed a row's position
       const bool masked = __any_sync(0xffffffffu, key0 + C::kKeys - 1 > (pos_r < 0 ? -1 : pos_r)) ||
                           warp_min_pos == INT_MAX;
-      // pass 1: row max of the raw scores (scaled afterwards; the scale is positive)
+      // the whole S row (64 fp32) in one batch of TMEM loads and a single wait
+      uint32_t r[C::kKeys];
+#pragma unroll
+      for (int c = 0; c < C::kKeys / 16; ++c)
+        tmem_ld32x32b_x16(s_addr + c * 16, *reinterpret_cast<uint32_t(*)[16]>(&r[c * 16]));
+      tmem_ld_wait();
+      // row max of the raw scores (scaled afterwards; the scale is positive)
       float mx = -INFINITY;
+      if (masked) {
 #pragma unroll
-      for (int c = 0; c < C::kKeys / 32; ++c) {
-        uint32_t r[32];
-        tmem_ld32x32b_x16(s_addr + c * 32, *reinterpret_cast<uint32_t(*)[16]>(&r[0]));
-        tmem_ld32x32b_x16(s_addr + c * 32 + 16, *reinterpret_cast<uint32_t(*)[16]>(&r[16]));
-        tmem_ld_wait();
-        if (masked) {
+        for (int i = 0; i < C::kKeys; ++i)
+          if (key0 + i <= pos_r) mx = fmaxf(mx, __uint_as_float(r[i]));
+      } else {
 #pragma unroll
-          for (int i = 0; i < 32; ++i)
-            if (key0 + c * 32 + i <= pos_r) mx = fmaxf(mx, __uint_as_float(r[i]));
-        } else {
-#pragma unroll
-          for (int i = 0; i < 32; ++i) mx = fmaxf(mx, __uint_as_float(r[i]));
-        }
+        for (int i = 0; i < C::kKeys; ++i) mx = fmaxf(mx, __uint_as_float(r[i]));
       }
       mx *= p.scale_log2;
       // lazy rescale: keep the previous max unless the new one exceeds it by > 8 (P <= 2^8)
@@ -271,30 +290,31 @@ __global__ void __launch_bounds__(kFaThreads, 2)
       // pass 2: P = 2^(s*scale - m) and the row sum; P written as two bf16 terms (P_hi + P_lo,
       // exact to ~2^-16 so the fp32 P.V meets the 2e-3 attention bar) over the 32 S columns each
       // chunk has just read: [32c, 32c+16) = P_hi, [32c+16, 32c+32) = P_lo of keys 32c..32c+31.
-      float sum = 0.f;
+      float2 sum2 = make_float2(0.f, 0.f);
+      const float2 scale2 = make_float2(p.scale_log2, p.scale_log2), nmb2 = make_float2(-mb, -mb);
 #pragma unroll
       for (int c = 0; c < C::kKeys / 32; ++c) {
-        uint32_t r[32];
-        tmem_ld32x32b_x16(s_addr + c * 32, *reinterpret_cast<uint32_t(*)[16]>(&r[0]));
-        tmem_ld32x32b_x16(s_addr + c * 32 + 16, *reinterpret_cast<uint32_t(*)[16]>(&r[16]));
-        tmem_ld_wait();
         uint32_t hi[16], lo[16];
 #pragma unroll
         for (int i = 0; i < 16; ++i) {
-          float p0 = ex2(fmaf(__uint_as_float(r[2 * i]), p.scale_log2, -mb));
-          float p1 = ex2(fmaf(__uint_as_float(r[2 * i + 1]), p.scale_log2, -mb));
+          // paired fp32 ops (FFMA2 / FADD2) halve the softmax's FMA-pipe instructions
+          const float2 x = fma2(make_float2(__uint_as_float(r[c * 32 + 2 * i]), __uint_as_float(r[c * 32 + 2 * i + 1])),
+                                scale2, nmb2);
+          float2 pp = make_float2(ex2(x.x), ex2(x.y));
           if (masked) {
             const int k = key0 + c * 32 + 2 * i;
-            p0 = (k <= pos_r) ? p0 : 0.f;
-            p1 = (k + 1 <= pos_r) ? p1 : 0.f;
+            pp.x = (k <= pos_r) ? pp.x : 0.f;
+            pp.y = (k + 1 <= pos_r) ? pp.y : 0.f;
           }
-          hi[i] = pack_bf16(p0, p1);
-          lo[i] = pack_bf16(p0 - bf16_lo(hi[i]), p1 - bf16_hi(hi[i]));
-          sum += p0 + p1;
+          hi[i] = pack_bf16(pp.x, pp.y);
+          const float2 rs = add2(pp, make_float2(-bf16_lo(hi[i]), -bf16_hi(hi[i])));
+          lo[i] = pack_bf16(rs.x, rs.y);
+          sum2 = add2(sum2, pp);
         }
         tmem_st32x32b_x16(s_addr + c * 32, hi);
         tmem_st32x32b_x16(s_addr + c * 32 + 16, lo);
       }
+      const float sum = sum2.x + sum2.y;
       tmem_st_wait();
       l = l * alpha + sum;
       if (j >= 1 && __any_sync(0xffffffffu, alpha != 1.f)) {

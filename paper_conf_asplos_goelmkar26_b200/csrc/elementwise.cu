@@ -3,8 +3,7 @@
 //   embed_rmsnorm   x = E[tok] (fp32 residual init) and h = RMSNorm(x)·g1 of layer 0   (a2+a3)
 //   rmsnorm         h = RMSNorm(r)·g from the fp32 residual stream                       (a3)
 //   gather_rmsnorm  the R logit rows (last token of each chunk, every decode) + final norm (a13)
-//   rope_append     rotate-half RoPE of q and k at each row's position, K/V written to the
-//                   paged cache with 16-byte stores                                       (a5+a6)
+//   (RoPE + the paged KV append (a5+a6) run in the QKV GEMM epilogue, gemm.cu)
 //   argmax          greedy token, lowest index on ties                                    (a14)
 // One CTA per token row; 16-byte vector loads/stores; fp32 statistics.
 #include <cfloat>
@@ -123,55 +122,6 @@ __global__ void unshard_logits_kernel(const float* __restrict__ in, float* __res
   }
 }
 
-// One CTA per token row.  qkv row = [q heads | k heads | v heads], each head hd bf16.
-// rope_tab[pos][i] = (cos, sin)(pos * theta^(-2i/hd)), i < hd/2, built in fp64 on the host.
-// slot = physical block * 16 + offset; cache plane layout [block][Hkv][16][hd].
-__global__ void rope_append_kernel(__nv_bfloat16* qkv, int qkv_ld, __nv_bfloat16* q_out,  // may alias (in place)
-                                   int q_ld, const int32_t* __restrict__ pos, const int32_t* __restrict__ slot,
-                                   const float2* __restrict__ rope_tab, __nv_bfloat16* __restrict__ kplane,
-                                   __nv_bfloat16* __restrict__ vplane, int H, int Hkv, int hd) {
-  const int t = blockIdx.x;
-  const int p = pos[t];
-  const int sl = slot[t];
-  const int blk = sl >> 4, off = sl & 15;
-  const int half = hd / 2;
-  const float2* tab = rope_tab + size_t(p) * half;
-  __nv_bfloat16* row = qkv + size_t(t) * qkv_ld;
-  // q and k: each thread rotates 8 pairs (i .. i+7 with i + half)
-  const int npair_vec = half / 8;
-  for (int w = threadIdx.x; w < (H + Hkv) * npair_vec; w += blockDim.x) {
-    const int h = w / npair_vec, i0 = (w % npair_vec) * 8;
-    const __nv_bfloat16* src = row + size_t(h) * hd;
-    const uint4 a = *reinterpret_cast<const uint4*>(src + i0);
-    const uint4 b = *reinterpret_cast<const uint4*>(src + half + i0);
-    const uint32_t aw[4] = {a.x, a.y, a.z, a.w}, bw[4] = {b.x, b.y, b.z, b.w};
-    uint32_t ra[4], rb[4];
-#pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      const float2 cs0 = tab[i0 + 2 * k], cs1 = tab[i0 + 2 * k + 1];
-      const float x0 = bf16_lo(aw[k]), x1 = bf16_hi(aw[k]);
-      const float y0 = bf16_lo(bw[k]), y1 = bf16_hi(bw[k]);
-      ra[k] = pack_bf16(x0 * cs0.x - y0 * cs0.y, x1 * cs1.x - y1 * cs1.y);
-      rb[k] = pack_bf16(y0 * cs0.x + x0 * cs0.y, y1 * cs1.x + x1 * cs1.y);
-    }
-    __nv_bfloat16* dst;
-    if (h < H) {
-      dst = q_out + size_t(t) * q_ld + size_t(h) * hd;
-    } else {
-      dst = kplane + ((size_t(blk) * Hkv + (h - H)) * 16 + off) * hd;
-    }
-    *reinterpret_cast<uint4*>(dst + i0) = make_uint4(ra[0], ra[1], ra[2], ra[3]);
-    *reinterpret_cast<uint4*>(dst + half + i0) = make_uint4(rb[0], rb[1], rb[2], rb[3]);
-  }
-  // v: straight copy, 16 B per thread
-  const int nv = Hkv * hd / 8;
-  for (int w = threadIdx.x; w < nv; w += blockDim.x) {
-    const int h = (w * 8) / hd, c = (w * 8) % hd;
-    const uint4 v = *reinterpret_cast<const uint4*>(row + size_t(H + Hkv + h) * hd + c);
-    *reinterpret_cast<uint4*>(vplane + ((size_t(blk) * Hkv + h) * 16 + off) * hd + c) = v;
-  }
-}
-
 // argmax per row; ties -> lowest index.  logits f32 or bf16 [R][V].
 __global__ void argmax_kernel(const void* __restrict__ logits, int is_f32, int V, int32_t* __restrict__ out) {
   const int r = blockIdx.x;
@@ -286,15 +236,6 @@ cudaError_t launch_gather_rmsnorm(const float* x, const int32_t* rows, const voi
   if (R == 0) return cudaSuccess;
   count_launch();
   gather_rmsnorm_kernel<<<R, kRowThreads, 0, st>>>(x, rows, (const __nv_bfloat16*)g, (__nv_bfloat16*)out, d, eps);
-  return cudaGetLastError();
-}
-cudaError_t launch_rope_append(void* qkv, int qkv_ld, void* q_out, int q_ld, const int32_t* pos, const int32_t* slot,
-                               const float2* rope_tab, void* kplane, void* vplane, int T, int H, int Hkv, int hd,
-                               cudaStream_t st) {
-  if (T == 0) return cudaSuccess;
-  count_launch();
-  rope_append_kernel<<<T, 128, 0, st>>>((__nv_bfloat16*)qkv, qkv_ld, (__nv_bfloat16*)q_out, q_ld, pos, slot, rope_tab,
-                                        (__nv_bfloat16*)kplane, (__nv_bfloat16*)vplane, H, Hkv, hd);
   return cudaGetLastError();
 }
 cudaError_t launch_add_rmsnorm(float* resid, const void* add, const void* g, void* out, int T, int d, float eps,

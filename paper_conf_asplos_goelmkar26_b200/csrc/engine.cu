@@ -557,14 +557,14 @@ struct Seg {
 };
 
 int gemm_seg(qos_engine* e, const Seg& g, const CUtensorMap& ta, const CUtensorMap (&tb)[2], int64_t N, int64_t K,
-             int epi, void* C, int64_t ldc, const float* bias) {
+             int epi, void* C, int64_t ldc, const float* bias, const QkvRopeArgs* rope = nullptr) {
   const int sms = g.sms > 0 ? g.sms : e->num_sms;
   const int bn = gemm_pick_bn(g.n, N, epi, sms);
   const int ks = e->gemm_splitk ? gemm_pick_ksplit(g.n, N, K, bn, sms, kGemmMaxUnits) : 1;
   count_launch();
   const size_t esz = (epi == EPI_STORE_F32 || epi == EPI_ADD_F32) ? 4 : 2;
   return gemm_run(ta, tb[bn == 256 ? 1 : 0], bn, g.n, N, K, epi, reinterpret_cast<uint8_t*>(C) + size_t(g.row0) * ldc * esz,
-                  ldc, bias, sms, g.st, ks, g.gpart, g.gcnt, g.row0, sms);
+                  ldc, bias, sms, g.st, ks, g.gpart, g.gcnt, g.row0, sms, rope);
 }
 
 // The layer loop.  `dm` = device metadata block of this step.
@@ -637,14 +637,11 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
         QOS_CU(launch_rmsnorm(resid + r0 * d, W(e, L.ln1), h + r0 * d, g.n, d, c.rms_eps, gs));
       }
       {
+        // a4 + a5 + a6: QKV projection (+bias) with RoPE and the paged KV append in its epilogue
         TimerScope ts(e, QOS_T_GEMM_QKV, gs);
-        QOS_TRY(gemm_seg(e, g, e->a_h, M.qkv, e->nqkv, d, c.qkv_bias ? EPI_BIAS_BF16 : EPI_STORE_BF16, qkv, e->nqkv,
-                         c.qkv_bias ? reinterpret_cast<const float*>(e->w + L.bqkv) : nullptr));
-      }
-      {
-        TimerScope ts(e, QOS_T_ROPE_APPEND, gs);
-        QOS_CU(launch_rope_append(qkv + r0 * e->nqkv, e->nqkv, qkv + r0 * e->nqkv, e->nqkv, pos + r0, slot + r0,
-                                  e->rope_tab, kpl, vpl, g.n, e->sh.H, e->sh.Hkv, hd, gs));
+        const QkvRopeArgs ra{pos + r0, slot + r0, e->rope_tab, kpl, vpl, e->sh.H, e->sh.Hkv, hd};
+        QOS_TRY(gemm_seg(e, g, e->a_h, M.qkv, e->nqkv, d, EPI_QKV_ROPE, qkv, e->nqkv,
+                         c.qkv_bias ? reinterpret_cast<const float*>(e->w + L.bqkv) : nullptr, &ra));
       }
       // a7 || a8: within one segment, the prefill tiles go to the high-priority side stream and
       // the decode split-K items stay on the segment's stream (disjoint rows of `attn`)
@@ -1380,8 +1377,8 @@ int qos_kv_read(qos_engine_t* e, int32_t layer, int64_t req, int32_t pos0, int32
   return kv_rw(e, layer, req, pos0, n, nullptr, nullptr, k, v);
 }
 
-int qos_op_rope_kv_append(qos_engine_t* e, int32_t layer, const qos_batch* b, const uint16_t* qkv_in, uint16_t* q_out) {
-  if (!e || !qkv_in || !q_out || layer < 0 || layer >= e->cfg.n_layers) return set_error(QOS_ERR_INVALID_ARG, "args");
+int qos_op_qkv_rope_append(qos_engine_t* e, int32_t layer, const qos_batch* b, const uint16_t* h_in, uint16_t* q_out) {
+  if (!e || !h_in || !q_out || layer < 0 || layer >= e->cfg.n_layers) return set_error(QOS_ERR_INVALID_ARG, "args");
   QOS_CU(cudaSetDevice(e->device));
   cudaStream_t st = e->stream;
   QOS_TRY(acquire_staging(e));
@@ -1390,16 +1387,20 @@ int qos_op_rope_kv_append(qos_engine_t* e, int32_t layer, const qos_batch* b, co
   if (r != QOS_OK) { e->meta_cur ^= 1; return r; }
   uint8_t* dm;
   QOS_TRY(upload_meta(e, m, st, &dm));
-  __nv_bfloat16* qkv = reinterpret_cast<__nv_bfloat16*>(e->ws + e->wsl.qkv);
-  const size_t w = size_t(e->nqkv);
-  QOS_CU(cudaMemcpyAsync(qkv, qkv_in, size_t(m.T) * w * 2, cudaMemcpyHostToDevice, st));
+  const int d = e->cfg.d_model, hd = e->cfg.head_dim;
+  QOS_CU(cudaMemcpyAsync(e->ws + e->wsl.h, h_in, size_t(m.T) * d * 2, cudaMemcpyHostToDevice, st));
   __nv_bfloat16* kpl = reinterpret_cast<__nv_bfloat16*>(e->kv) + (size_t(layer) * 2 + 0) * e->plane_elems;
   __nv_bfloat16* vpl = reinterpret_cast<__nv_bfloat16*>(e->kv) + (size_t(layer) * 2 + 1) * e->plane_elems;
-  QOS_CU(launch_rope_append(qkv, int(w), qkv, int(w), reinterpret_cast<int32_t*>(dm + m.o_pos),
-                            reinterpret_cast<int32_t*>(dm + m.o_slot), e->rope_tab, kpl, vpl, m.T, e->sh.H, e->sh.Hkv,
-                            e->cfg.head_dim, st));
-  const size_t qb = size_t(e->sh.H) * e->cfg.head_dim * 2;
-  QOS_CU(cudaMemcpy2DAsync(q_out, qb, qkv, w * 2, qb, size_t(m.T), cudaMemcpyDeviceToHost, st));
+  const QkvRopeArgs ra{reinterpret_cast<int32_t*>(dm + m.o_pos), reinterpret_cast<int32_t*>(dm + m.o_slot), e->rope_tab,
+                       kpl, vpl, e->sh.H, e->sh.Hkv, hd};
+  const Seg g{0, m.T, st, false, false, reinterpret_cast<float*>(e->ws + e->wsl.gemm_part),
+              reinterpret_cast<int*>(e->ws + e->wsl.gemm_cnt), 0};
+  const auto& L = e->wl.layers[layer];
+  __nv_bfloat16* qkv = reinterpret_cast<__nv_bfloat16*>(e->ws + e->wsl.qkv);
+  QOS_TRY(gemm_seg(e, g, e->a_h, e->lmaps[layer].qkv, e->nqkv, d, EPI_QKV_ROPE, qkv, e->nqkv,
+                   e->cfg.qkv_bias ? reinterpret_cast<const float*>(e->w + L.bqkv) : nullptr, &ra));
+  const size_t qb = size_t(e->sh.H) * hd * 2;
+  QOS_CU(cudaMemcpy2DAsync(q_out, qb, qkv, size_t(e->nqkv) * 2, qb, size_t(m.T), cudaMemcpyDeviceToHost, st));
   QOS_TRY(release_staging(e, st));
   QOS_CU(cudaStreamSynchronize(st));
   return QOS_OK;

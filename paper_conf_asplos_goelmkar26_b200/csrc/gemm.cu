@@ -47,6 +47,13 @@ struct GemmArgs {
   float* part;      // split-K partials [unit][128][BN] fp32 (ksplit > 1)
   int* counters;    // split-K arrival counter per tile (ksplit > 1), zero between launches
   int a_row0;       // first row of A (TMA coordinate offset): GEMM over a row range of a buffer
+  // EPI_QKV_ROPE: RoPE on q and k at each row's position; q -> C, k / v -> the paged cache
+  const int32_t* pos;     // [M] positions of the rows
+  const int32_t* slot;    // [M] cache slots (block * 16 + offset)
+  const float2* rope;     // [max_pos][hd/2] (cos, sin)
+  __nv_bfloat16* kplane;  // [blocks][Hkv][16][hd] of this layer
+  __nv_bfloat16* vplane;
+  int H, Hkv, hd;
 };
 
 // ---- epilogue stores of one thread's 32 consecutive accumulator columns of one row
@@ -88,6 +95,65 @@ QOS_DEV void epi_silu32(const GemmArgs& p, int row, int outcol, const float (&g)
   uint4* dst = reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.C) + size_t(row) * p.ldc + outcol);
 #pragma unroll
   for (int i = 0; i < 4; ++i) dst[i] = make_uint4(pk[4 * i], pk[4 * i + 1], pk[4 * i + 2], pk[4 * i + 3]);
+}
+
+// Fused a4+a5+a6 epilogue: for every head of the tile, RoPE (rotate-half, pairs i / i+hd/2)
+// on q and k, q written to C (the qkv buffer, read by the attention kernels), k and v written
+// straight into the paged cache at the row's slot with 32-byte stores.  `fetch(col, v16)`
+// returns 16 accumulator columns of this thread's row (TMEM or summed split-K partials).
+template <int BN, typename Fetch>
+QOS_DEV void epi_qkv_rope(const GemmArgs& p, int row, bool row_ok, int n_t, Fetch fetch) {
+  const int hd = p.hd, half = hd / 2;
+  const int ps = row_ok ? __ldg(p.pos + row) : 0;
+  const int sl = row_ok ? __ldg(p.slot + row) : 0;
+  const float2* cs = p.rope + size_t(ps) * half;
+  for (int hh = 0; hh < BN / hd; ++hh) {
+    const int col0 = n_t * BN + hh * hd;
+    if (col0 >= p.N) break;  // warp-uniform
+    const int head = col0 / hd;
+    __nv_bfloat16* dst;
+    if (head < p.H)
+      dst = reinterpret_cast<__nv_bfloat16*>(p.C) + size_t(row) * p.ldc + col0;
+    else if (head < p.H + p.Hkv)
+      dst = p.kplane + ((size_t(sl >> 4) * p.Hkv + (head - p.H)) * 16 + (sl & 15)) * hd;
+    else
+      dst = p.vplane + ((size_t(sl >> 4) * p.Hkv + (head - p.H - p.Hkv)) * 16 + (sl & 15)) * hd;
+    if (head < p.H + p.Hkv) {
+      for (int i0 = 0; i0 < half; i0 += 16) {
+        float x[16], y[16];
+        fetch(hh * hd + i0, x);
+        fetch(hh * hd + half + i0, y);
+        if (row_ok) {
+          uint32_t a[8], b[8];
+#pragma unroll
+          for (int k = 0; k < 8; ++k) {
+            const float2 c0 = __ldg(cs + i0 + 2 * k), c1 = __ldg(cs + i0 + 2 * k + 1);
+            a[k] = pack_bf16(x[2 * k] * c0.x - y[2 * k] * c0.y, x[2 * k + 1] * c1.x - y[2 * k + 1] * c1.y);
+            b[k] = pack_bf16(y[2 * k] * c0.x + x[2 * k] * c0.y, y[2 * k + 1] * c1.x + x[2 * k + 1] * c1.y);
+          }
+          uint4* da = reinterpret_cast<uint4*>(dst + i0);
+          uint4* db = reinterpret_cast<uint4*>(dst + half + i0);
+          da[0] = make_uint4(a[0], a[1], a[2], a[3]);
+          da[1] = make_uint4(a[4], a[5], a[6], a[7]);
+          db[0] = make_uint4(b[0], b[1], b[2], b[3]);
+          db[1] = make_uint4(b[4], b[5], b[6], b[7]);
+        }
+      }
+    } else {
+      for (int i0 = 0; i0 < hd; i0 += 16) {
+        float x[16];
+        fetch(hh * hd + i0, x);
+        if (row_ok) {
+          uint32_t a[8];
+#pragma unroll
+          for (int k = 0; k < 8; ++k) a[k] = pack_bf16(x[2 * k], x[2 * k + 1]);
+          uint4* da = reinterpret_cast<uint4*>(dst + i0);
+          da[0] = make_uint4(a[0], a[1], a[2], a[3]);
+          da[1] = make_uint4(a[4], a[5], a[6], a[7]);
+        }
+      }
+    }
+  }
 }
 
 QOS_DEV void tmem_ld32(uint32_t taddr, float (&v)[32]) {
@@ -219,7 +285,15 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
       const bool row_ok = row < p.M;
       const uint32_t tbase = tmem_base + (uint32_t(q * 32) << 16) + acc * BN;
       if (ks == 1) {
-        if constexpr (EPI == EPI_SILU_GATE) {
+        if constexpr (EPI == EPI_QKV_ROPE) {
+          epi_qkv_rope<BN>(p, row, row_ok, n_t, [&](int col, float (&v)[16]) {
+            uint32_t r[16];
+            tmem_ld32x32b_x16(tbase + col, r);
+            tmem_ld_wait();
+#pragma unroll
+            for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]) + (p.bias ? __ldg(p.bias + n_t * BN + col + i) : 0.f);
+          });
+        } else if constexpr (EPI == EPI_SILU_GATE) {
 #pragma unroll 1
           for (int g = 0; g < BN / 128; ++g) {
 #pragma unroll 1
@@ -293,7 +367,17 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
           auto part_row = [&](int s2) {
             return p.part + (size_t((n_t * ks + s2) * p.mt + m_t) * kBM + rit) * BN;
           };
-          if constexpr (EPI == EPI_SILU_GATE) {
+          if constexpr (EPI == EPI_QKV_ROPE) {
+            epi_qkv_rope<BN>(p, row, row_ok, n_t, [&](int col, float (&v)[16]) {
+#pragma unroll
+              for (int i = 0; i < 16; ++i) v[i] = p.bias ? __ldg(p.bias + n_t * BN + col + i) : 0.f;
+              for (int s2 = 0; s2 < ks; ++s2) {
+                const float* pr = part_row(s2) + col;
+#pragma unroll
+                for (int i = 0; i < 16; ++i) v[i] += __ldcg(pr + i);
+              }
+            });
+          } else if constexpr (EPI == EPI_SILU_GATE) {
 #pragma unroll 1
             for (int g = 0; g < BN / 128; ++g)
 #pragma unroll 1
@@ -426,7 +510,7 @@ int gemm_pick_ksplit(int64_t M, int64_t N, int64_t K, int bn, int num_sms, int64
 
 int gemm_run(const CUtensorMap& ta, const CUtensorMap& tb, int bn, int64_t M, int64_t N, int64_t K, int epi, void* C,
              int64_t ldc, const float* bias, int num_sms, cudaStream_t st, int ksplit, float* part, int* counters,
-             int a_row0, int max_ctas) {
+             int a_row0, int max_ctas, const QkvRopeArgs* rope) {
   GemmArgs a;
   a.M = int(M);
   a.N = int(N);
@@ -440,6 +524,16 @@ int gemm_run(const CUtensorMap& ta, const CUtensorMap& tb, int bn, int64_t M, in
   a.part = part;
   a.counters = counters;
   a.a_row0 = a_row0;
+  a.pos = rope ? rope->pos : nullptr;
+  a.slot = rope ? rope->slot : nullptr;
+  a.rope = rope ? rope->tab : nullptr;
+  a.kplane = rope ? reinterpret_cast<__nv_bfloat16*>(rope->kplane) : nullptr;
+  a.vplane = rope ? reinterpret_cast<__nv_bfloat16*>(rope->vplane) : nullptr;
+  a.H = rope ? rope->H : 0;
+  a.Hkv = rope ? rope->Hkv : 0;
+  a.hd = rope ? rope->hd : 0;
+  if (epi == EPI_QKV_ROPE && (!rope || a.hd <= 0 || bn % a.hd))
+    return set_error(QOS_ERR_INVALID_ARG, "gemm: QKV_ROPE needs rope args and BN % hd == 0");
   if (a.ksplit > 1 && (!part || !counters)) return set_error(QOS_ERR_INVALID_ARG, "gemm: split-K needs workspace");
   const int tiles = a.mt * a.nt * a.ksplit;
   int grid = tiles < num_sms ? tiles : num_sms;
@@ -457,6 +551,8 @@ int gemm_run(const CUtensorMap& ta, const CUtensorMap& tb, int bn, int64_t M, in
   QOS_GEMM_CASE(256, EPI_SILU_GATE)
   QOS_GEMM_CASE(128, EPI_ADD_F32)
   QOS_GEMM_CASE(256, EPI_ADD_F32)
+  QOS_GEMM_CASE(128, EPI_QKV_ROPE)
+  QOS_GEMM_CASE(256, EPI_QKV_ROPE)
   return set_error(QOS_ERR_INVALID_ARG, "gemm: bad tile/epilogue");
 #undef QOS_GEMM_CASE
   if (e != cudaSuccess) return set_cuda_error(e, "gemm launch");
@@ -468,7 +564,7 @@ int gemm_check_shape(int64_t M, int64_t N, int64_t K, int epi) {
   if (K % 64) return set_error(QOS_ERR_UNSUPPORTED, "gemm: K % 64 != 0");
   if (N % 32) return set_error(QOS_ERR_UNSUPPORTED, "gemm: N % 32 != 0");
   if (epi == EPI_SILU_GATE && N % 128) return set_error(QOS_ERR_UNSUPPORTED, "gemm: SILU_GATE needs N % 128 == 0");
-  if (epi < 0 || epi > EPI_ADD_F32) return set_error(QOS_ERR_INVALID_ARG, "gemm: unknown epilogue");
+  if (epi < 0 || epi > EPI_ADD_F32) return set_error(QOS_ERR_INVALID_ARG, "gemm: unknown epilogue");  // public ones
   return QOS_OK;
 }
 

@@ -11,7 +11,17 @@
 namespace qos {
 
 enum { EPI_STORE_BF16 = QOS_EPI_STORE_BF16, EPI_STORE_F32 = QOS_EPI_STORE_F32, EPI_BIAS_BF16 = QOS_EPI_BIAS_BF16,
-       EPI_SILU_GATE = QOS_EPI_SILU_GATE, EPI_ADD_F32 = QOS_EPI_ADD_F32 };
+       EPI_SILU_GATE = QOS_EPI_SILU_GATE, EPI_ADD_F32 = QOS_EPI_ADD_F32,
+       EPI_QKV_ROPE = 5 /* internal: a4 + a5 + a6 fused (RoPE, q -> C, k/v -> paged cache; +bias) */ };
+
+struct QkvRopeArgs {
+  const int32_t* pos;
+  const int32_t* slot;
+  const float2* tab;
+  void* kplane;
+  void* vplane;
+  int H, Hkv, hd;
+};
 
 // error reporting (thread-local last error; engine.cpp)
 int set_error(int code, const char* msg);
@@ -30,7 +40,7 @@ int gemm_pick_ksplit(int64_t M, int64_t N, int64_t K, int bn, int num_sms, int64
 // counters (zero-initialised; each reducing CTA resets its own) — deterministic reduction order
 int gemm_run(const CUtensorMap& ta, const CUtensorMap& tb, int bn, int64_t M, int64_t N, int64_t K, int epi, void* C,
              int64_t ldc, const float* bias, int num_sms, cudaStream_t st, int ksplit = 1, float* part = nullptr,
-             int* counters = nullptr, int a_row0 = 0, int max_ctas = 0);
+             int* counters = nullptr, int a_row0 = 0, int max_ctas = 0, const QkvRopeArgs* rope = nullptr);
 
 // ------------------------------------------------------------------ synthetic generator (gen.cu)
 enum GenKind { GEN_LINEAR = 0, GEN_EMBED = 1, GEN_NORM = 2, GEN_BIAS = 3 };
@@ -52,10 +62,6 @@ cudaError_t launch_embed_rmsnorm(const int32_t* tokens, const void* emb, const v
 cudaError_t launch_rmsnorm(const float* x, const void* g, void* out, int T, int d, float eps, cudaStream_t st);
 cudaError_t launch_gather_rmsnorm(const float* x, const int32_t* rows, const void* g, void* out, int R, int d,
                                   float eps, cudaStream_t st);
-// RoPE on q, k + append k, v to the paged cache
-cudaError_t launch_rope_append(void* qkv, int qkv_ld, void* q_out, int q_ld, const int32_t* pos,
-                               const int32_t* slot, const float2* rope_tab, void* kplane, void* vplane, int T, int H,
-                               int Hkv, int hd, cudaStream_t st);
 // copy rows between host-layout [n][Hkv][hd] buffers and the paged plane (positions pos0..)
 cudaError_t launch_kv_scatter(void* plane, const int32_t* d_table_row, int pos0, int n, int Hkv, int hd,
                               const void* src, cudaStream_t st);

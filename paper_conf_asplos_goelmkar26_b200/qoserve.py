@@ -104,7 +104,7 @@ _SIGS = {
     "qos_op_rmsnorm": [_P, _P, _P, C.c_int32, C.c_int32, C.c_float, _P],
     "qos_kv_write": [_P, C.c_int32, C.c_int64, C.c_int32, C.c_int32, _P, _P],
     "qos_kv_read": [_P, C.c_int32, C.c_int64, C.c_int32, C.c_int32, _P, _P],
-    "qos_op_rope_kv_append": [_P, C.c_int32, C.POINTER(qos_batch), _P, _P],
+    "qos_op_qkv_rope_append": [_P, C.c_int32, C.POINTER(qos_batch), _P, _P],
     "qos_op_attention": [_P, C.c_int32, C.POINTER(qos_batch), _P, _P],
 }
 EXPORTED = sorted(list(_SIGS) + ["qos_strerror", "qos_last_error"])
@@ -329,10 +329,10 @@ class Engine:
         return a.value, b.value
 
     # ops
-    def qos_op_rope_kv_append(self, layer: int, batch: _BatchKeep, qkv_bits: np.ndarray, q_cols: int):
-        qkv = np.ascontiguousarray(qkv_bits, dtype=np.uint16)
-        q = np.empty((qkv.shape[0], q_cols), dtype=np.uint16)
-        _call("qos_op_rope_kv_append", self.h, layer, C.byref(batch.b), qkv.ctypes.data, q.ctypes.data)
+    def qos_op_qkv_rope_append(self, layer: int, batch: _BatchKeep, h_bits: np.ndarray, q_cols: int):
+        hh = np.ascontiguousarray(h_bits, dtype=np.uint16)
+        q = np.empty((hh.shape[0], q_cols), dtype=np.uint16)
+        _call("qos_op_qkv_rope_append", self.h, layer, C.byref(batch.b), hh.ctypes.data, q.ctypes.data)
         return q
 
     def qos_op_attention(self, layer: int, batch: _BatchKeep, q_bits: np.ndarray) -> np.ndarray:
