@@ -190,6 +190,18 @@ int qos_profile_step_ex(qos_engine_t* eng, int32_t chunk_len, int32_t kv_start,
                         int32_t n_decode, const int32_t* ctx_lens, int32_t warmup, int32_t reps,
                         float* ms_median, float* ms_p95);
 
+/* Execution options (defaults in parentheses; the QOS_* environment variables of the same
+ * meaning set the defaults at engine creation):
+ *   "overlap_attn" (1)     run prefill attention on a high-priority side stream concurrently
+ *                          with the decode attention of the same layer
+ *   "gemm_splitk" (1)      split-K for weight-bound small-M projections
+ *   "dual_stream" (0)      prefill rows and decode rows as two sub-batches on two streams
+ *                          (measured slower on B200; kept for experiments), with
+ *                          "dual_min_prefill" (512), "dual_min_decode" (16),
+ *                          "dual_sms_prefill" / "dual_sms_decode" (0 = all SMs)
+ * Results do not depend on the options (parity tests run with the defaults and variants). */
+int qos_engine_set_option(qos_engine_t* eng, const char* name, int64_t value);
+
 /* ---------------------------------------------------------------- per-kernel timing (a15) */
 enum {
   QOS_T_META = 0, QOS_T_EMBED, QOS_T_NORM, QOS_T_GEMM_QKV, QOS_T_ROPE_APPEND, QOS_T_PREFILL_ATTN,

@@ -1246,6 +1246,20 @@ int qos_profile_step(qos_engine_t* e, int32_t chunk_len, int32_t n_decode, const
   return qos_profile_step_ex(e, chunk_len, 0, n_decode, ctx_lens, -1, reps, ms_out, nullptr);
 }
 
+int qos_engine_set_option(qos_engine_t* e, const char* name, int64_t value) {
+  if (!e || !name) return set_error(QOS_ERR_INVALID_ARG, "args");
+  const std::string n(name);
+  if (n == "overlap_attn") e->overlap_attn = value != 0;
+  else if (n == "gemm_splitk") e->gemm_splitk = value != 0;
+  else if (n == "dual_stream") e->dual_stream = value != 0;
+  else if (n == "dual_min_prefill") e->dual_min_prefill = int(value);
+  else if (n == "dual_min_decode") e->dual_min_decode = int(value);
+  else if (n == "dual_sms_prefill") e->dual_sms_pre = int(value);
+  else if (n == "dual_sms_decode") e->dual_sms_dec = int(value);
+  else return set_error(QOS_ERR_INVALID_ARG, "unknown option");
+  return QOS_OK;
+}
+
 int qos_engine_set_timing(qos_engine_t* e, int enable) {
   if (!e) return set_error(QOS_ERR_INVALID_ARG, "engine is NULL");
   if (cudaDeviceSynchronize() != cudaSuccess) return set_error(QOS_ERR_CUDA, "set_timing sync");

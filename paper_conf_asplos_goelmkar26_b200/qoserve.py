@@ -95,6 +95,7 @@ _SIGS = {
     "qos_profile_step": [_P, C.c_int32, C.c_int32, C.POINTER(C.c_int32), C.c_int32, C.POINTER(C.c_float)],
     "qos_profile_step_ex": [_P, C.c_int32, C.c_int32, C.c_int32, C.POINTER(C.c_int32), C.c_int32, C.c_int32,
                             C.POINTER(C.c_float), C.POINTER(C.c_float)],
+    "qos_engine_set_option": [_P, C.c_char_p, C.c_int64],
     "qos_engine_set_timing": [_P, C.c_int],
     "qos_last_step_timing": [_P, C.POINTER(C.c_float), C.POINTER(C.c_int32)],
     "qos_last_step_io": [_P, C.POINTER(C.c_int64), C.POINTER(C.c_int64)],
@@ -313,6 +314,9 @@ class Engine:
         _call("qos_profile_step_ex", self.h, chunk_len, kv_start, len(ctx),
               ctx.ctypes.data_as(C.POINTER(C.c_int32)), warmup, reps, C.byref(med), C.byref(p95))
         return med.value, p95.value
+
+    def qos_engine_set_option(self, name: str, value: int):
+        _call("qos_engine_set_option", self.h, name.encode(), int(value))
 
     def qos_engine_set_timing(self, enable: bool):
         _call("qos_engine_set_timing", self.h, int(bool(enable)))
