@@ -198,3 +198,28 @@ def test_llama8b_shapes_bench_batch_sampled_parity():
     err = row_rel_err(got, ref)
     assert err <= TOL_LOGITS, err
     eng.close()
+
+
+@pytest.mark.parametrize("opts", [{"overlap_attn": 0}, {"gemm_splitk": 0},
+                                  {"dual_stream": 1, "dual_min_prefill": 1, "dual_min_decode": 1}])
+def test_execution_options_do_not_change_results(opts):
+    """qos_engine_set_option variants (serial attention, no split-K, two-stream sub-batches)
+    stay within tolerance of the oracle and give the same greedy tokens."""
+    q, cfg, eng = make_engine("tiny", num_blocks=256)
+    eng.qos_engine_load_synthetic(0)
+    for k, v in opts.items():
+        eng.qos_engine_set_option(k, v)
+    orc = _oracle("tiny", num_blocks=256)
+    ctxs, warm, main, second = synth.tiny_scenario(cfg.vocab)
+    for r, n in ctxs.items():
+        eng.qos_kv_alloc(r, n + 2)
+        orc.kv_alloc(r, n + 2)
+    eng.qos_kv_alloc(0, 256)
+    orc.kv_alloc(0, 256)
+    for b in warm + [main, second]:
+        lg, tk = eng.step_host(q.batch_from_synth(b), cfg.vocab)
+        ref = orc.hybrid_step(*b.as_oracle())
+        assert row_rel_err(lg, ref) <= TOL_LOGITS
+    with pytest.raises(q.QosError):
+        eng.qos_engine_set_option("no_such_option", 1)
+    eng.close()
