@@ -199,6 +199,12 @@ int qos_profile_step_ex(qos_engine_t* eng, int32_t chunk_len, int32_t kv_start,
  *                          (measured slower on B200; kept for experiments), with
  *                          "dual_min_prefill" (512), "dual_min_decode" (16),
  *                          "dual_sms_prefill" / "dual_sms_decode" (0 = all SMs)
+ *   "gemm_swab" (1)        weight-streaming swap-AB GEMM for small token counts: 0 never,
+ *                          1 automatic (small T, or T <= 256 with few output tiles), 2 always
+ *                          (where N % 128 == 0); env QOS_GEMM_SWAB
+ *   "pdl" (1)              programmatic dependent launch of the step's kernel chain (each
+ *                          kernel's prologue and weight prefetch overlap the previous kernel's
+ *                          tail); process-wide, env QOS_PDL
  * Results do not depend on the options (parity tests run with the defaults and variants). */
 int qos_engine_set_option(qos_engine_t* eng, const char* name, int64_t value);
 

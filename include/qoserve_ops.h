@@ -31,10 +31,19 @@ enum {
  * M may be any value >= 1.  Stream-ordered. */
 int qos_op_gemm(const void* A, const void* B, void* C, int64_t M, int64_t N, int64_t K, int epi,
                 const float* bias, void* stream);
-/* Same with an explicit split-K factor (0 = the engine's automatic choice, 1 = no split).
- * Split-K (weight-bound small-M GEMMs): each of `ksplit` CTAs accumulates a K slice of a tile,
- * parks an fp32 partial, and the last one to arrive sums the slices in slice order and applies
- * the epilogue (deterministic). */
+/* Same with an explicit kernel choice:
+ *   ksplit = 0   automatic: the weight-streaming kernel when N % 128 == 0 and M <= 16, or
+ *                M <= 32 with fewer output tiles of 128 than SMs, or M <= 256 with fewer than
+ *                SMs/4 tiles (env QOS_GEMM_SWAB=0 disables it), else the tile kernel with
+ *                automatic split-K;
+ *   ksplit >= 1  the tile kernel (128-token x 128/256-feature tiles) with that split-K factor:
+ *                each of `ksplit` CTAs accumulates a K slice of a tile, parks an fp32 partial,
+ *                and the last one to arrive sums the slices in slice order (deterministic);
+ *   ksplit < 0   the weight-streaming kernel (requires N % 128 == 0): computes C^T tile by
+ *                tile as W_tile(128 rows) · A^T on tcgen05 (token count = UMMA N), the
+ *                (tile, k-block) space split in equal contiguous ranges over the SMs
+ *                ("stream-K"); tiles cut by a range boundary are summed by their last
+ *                arriving CTA in CTA order (deterministic). */
 int qos_op_gemm_ex(const void* A, const void* B, void* C, int64_t M, int64_t N, int64_t K, int epi,
                    const float* bias, int ksplit, void* stream);
 

@@ -113,6 +113,8 @@ __global__ void __launch_bounds__(kAttnThreads, 3)
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + kAttnStages * C::kStageBytes);
   uint64_t* empty = full + kAttnStages;
 
+  griddep_wait();  // q and the appended K/V come from the previous kernel
+  griddep_launch_dependents();
   const DecodeItem it = items[blockIdx.x];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int group = p.H / p.Hkv;
@@ -326,9 +328,8 @@ static cudaError_t decode_t(const AttnLaunch& a, const DecodeItem* items, int n_
     if (e != cudaSuccess) return e;
     set = true;
   }
-  decode_attn_kernel<HD><<<n_items, kAttnThreads, AttnCfg<HD>::kSmemBytes, st>>>(*a.kv_tmap, to_params(a), items,
-                                                                                  partials, counters);
-  return cudaGetLastError();
+  return launch_pdl(decode_attn_kernel<HD>, dim3(n_items), dim3(kAttnThreads), AttnCfg<HD>::kSmemBytes, st,
+                    *a.kv_tmap, to_params(a), items, partials, counters);
 }
 
 cudaError_t launch_decode_attention(const AttnLaunch& a, const DecodeItem* items, int n_items, float* partials,

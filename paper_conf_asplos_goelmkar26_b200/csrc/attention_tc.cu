@@ -153,6 +153,8 @@ __global__ void __launch_bounds__(kFaThreads, 2)
     fence_mbar_init();
   }
   if (warp == 1) tmem_alloc<C::kTmemCols>(tmem_slot);
+  griddep_wait();  // q and the appended K/V come from the previous kernel
+  griddep_launch_dependents();
 
   // ---- Q tile -> smem (softmax warps; one row per thread), K-major 128-B swizzle
   int row = 0, pos_r = -1;
@@ -398,8 +400,8 @@ static cudaError_t prefill_tc_t(const AttnLaunch& a, const PrefillItem* items, i
   p.tables = a.tables;
   p.table_w = a.table_w;
   p.scale_log2 = a.scale_log2;
-  prefill_attn_tc_kernel<HD><<<n_items, kFaThreads, FaCfg<HD>::kSmem, st>>>(*a.kv_tmap, p, items);
-  return cudaGetLastError();
+  return launch_pdl(prefill_attn_tc_kernel<HD>, dim3(n_items), dim3(kFaThreads), FaCfg<HD>::kSmem, st, *a.kv_tmap, p,
+                    items);
 }
 
 int prefill_tc_positions_per_tile(int group) { return 128 / group; }

@@ -8,6 +8,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <utility>
+
 #define QOS_DEV __device__ __forceinline__
 
 namespace qos {
@@ -171,6 +173,33 @@ QOS_DEV void tmem_ld32x32b_x16(uint32_t taddr, uint32_t (&r)[16]) {
       : "r"(taddr));
 }
 QOS_DEV void tmem_ld_wait() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
+
+// ------------------------------------------------------------------------------ PDL
+// Programmatic dependent launch: kernels of the step chain are launched with
+// cudaLaunchAttributeProgrammaticStreamSerialization, so kernel i+1's prologue (barrier init,
+// TMEM alloc, descriptor prefetch, weight prefetch) overlaps kernel i's tail.  Every kernel
+// calls griddep_wait() before touching data written (or still read) by earlier kernels, and
+// griddep_launch_dependents() once all its CTAs are resident-safe to be followed.
+QOS_DEV void griddep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+QOS_DEV void griddep_launch_dependents() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
+bool pdl_enabled();  // engine-wide switch (QOS_PDL=0 disables)
+
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                              Args&&... args) {
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
+}
 
 // ------------------------------------------------------------------------------ mma.sync
 // m16n8k16 bf16 -> f32 (legacy warp MMA; used by the HBM-bound decode attention where the

@@ -56,6 +56,8 @@ __global__ void __launch_bounds__(kRowThreads) embed_rmsnorm_kernel(const int32_
                                                                     const __nv_bfloat16* __restrict__ g,
                                                                     float* __restrict__ resid,
                                                                     __nv_bfloat16* __restrict__ out, int d, float eps) {
+  griddep_wait();
+  griddep_launch_dependents();
   __shared__ float red[32];
   const int t = blockIdx.x;
   const __nv_bfloat16* e = emb + size_t(tokens[t]) * d;
@@ -72,6 +74,8 @@ __global__ void __launch_bounds__(kRowThreads) embed_rmsnorm_kernel(const int32_
 __global__ void __launch_bounds__(kRowThreads) rmsnorm_kernel(const float* __restrict__ x,
                                                               const __nv_bfloat16* __restrict__ g,
                                                               __nv_bfloat16* __restrict__ out, int d, float eps) {
+  griddep_wait();
+  griddep_launch_dependents();
   __shared__ float red[32];
   const int t = blockIdx.x;
   norm_row(x + size_t(t) * d, g, out + size_t(t) * d, d, eps, red);
@@ -82,6 +86,8 @@ __global__ void __launch_bounds__(kRowThreads) gather_rmsnorm_kernel(const float
                                                                      const __nv_bfloat16* __restrict__ g,
                                                                      __nv_bfloat16* __restrict__ out, int d,
                                                                      float eps) {
+  griddep_wait();
+  griddep_launch_dependents();
   __shared__ float red[32];
   const int r = blockIdx.x;
   norm_row(x + size_t(rows[r]) * d, g, out + size_t(r) * d, d, eps, red);
@@ -92,6 +98,8 @@ __global__ void __launch_bounds__(kRowThreads) gather_rmsnorm_kernel(const float
 __global__ void __launch_bounds__(kRowThreads) add_rmsnorm_kernel(float* __restrict__ resid, const __nv_bfloat16* add,
                                                                   const __nv_bfloat16* __restrict__ g,
                                                                   __nv_bfloat16* out, int d, float eps) {
+  griddep_wait();
+  griddep_launch_dependents();
   __shared__ float red[32];
   const int t = blockIdx.x;
   float* r = resid + size_t(t) * d;
@@ -108,11 +116,15 @@ __global__ void __launch_bounds__(kRowThreads) add_rmsnorm_kernel(float* __restr
 }
 
 __global__ void add_f32_kernel(float* __restrict__ resid, const __nv_bfloat16* __restrict__ add, int64_t n) {
+  griddep_wait();
+  griddep_launch_dependents();
   for (int64_t i = blockIdx.x * int64_t(blockDim.x) + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x)
     resid[i] += __bfloat162float(add[i]);
 }
 
 __global__ void unshard_logits_kernel(const float* __restrict__ in, float* __restrict__ out, int R, int Vl, int tp) {
+  griddep_wait();
+  griddep_launch_dependents();
   const int64_t n = int64_t(R) * Vl * tp;
   for (int64_t i = blockIdx.x * int64_t(blockDim.x) + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x) {
     const int j = int(i % Vl);
@@ -124,6 +136,8 @@ __global__ void unshard_logits_kernel(const float* __restrict__ in, float* __res
 
 // argmax per row; ties -> lowest index.  logits f32 or bf16 [R][V].
 __global__ void argmax_kernel(const void* __restrict__ logits, int is_f32, int V, int32_t* __restrict__ out) {
+  griddep_wait();
+  griddep_launch_dependents();
   const int r = blockIdx.x;
   float best = -INFINITY;
   int bi = 0x7fffffff;
@@ -163,6 +177,8 @@ __global__ void argmax_kernel(const void* __restrict__ logits, int is_f32, int V
 }
 
 __global__ void f32_to_bf16_kernel(const float* __restrict__ x, __nv_bfloat16* __restrict__ y, int64_t n) {
+  griddep_wait();
+  griddep_launch_dependents();
   for (int64_t i = blockIdx.x * int64_t(blockDim.x) + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x)
     y[i] = __float2bfloat16_rn(x[i]);
 }
@@ -186,6 +202,8 @@ __global__ void kv_gather_kernel(const __nv_bfloat16* __restrict__ plane, const 
   }
 }
 __global__ void table_update_kernel(int32_t* __restrict__ tables, int table_w, const int32_t* __restrict__ tr, int n) {
+  griddep_wait();
+  griddep_launch_dependents();
   const int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i < n) tables[size_t(tr[3 * i]) * table_w + tr[3 * i + 1]] = tr[3 * i + 2];
 }
@@ -214,61 +232,52 @@ cudaError_t launch_kv_gather(const void* plane, const int32_t* d_table_row, int 
 cudaError_t launch_table_update(int32_t* tables, int table_w, const int32_t* triples, int n, cudaStream_t st) {
   if (n == 0) return cudaSuccess;
   count_launch();
-  table_update_kernel<<<(n + 255) / 256, 256, 0, st>>>(tables, table_w, triples, n);
-  return cudaGetLastError();
+  return launch_pdl(table_update_kernel, dim3((n + 255) / 256), dim3(256), 0, st, tables, table_w, triples, n);
 }
 cudaError_t launch_embed_rmsnorm(const int32_t* tokens, const void* emb, const void* g, float* resid, void* out,
                                  int T, int d, float eps, cudaStream_t st) {
   if (T == 0) return cudaSuccess;
   count_launch();
-  embed_rmsnorm_kernel<<<T, kRowThreads, 0, st>>>(tokens, (const __nv_bfloat16*)emb, (const __nv_bfloat16*)g, resid,
+  return launch_pdl(embed_rmsnorm_kernel, dim3(T), dim3(kRowThreads), 0, st, tokens, (const __nv_bfloat16*)emb, (const __nv_bfloat16*)g, resid,
                                                   (__nv_bfloat16*)out, d, eps);
-  return cudaGetLastError();
 }
 cudaError_t launch_rmsnorm(const float* x, const void* g, void* out, int T, int d, float eps, cudaStream_t st) {
   if (T == 0) return cudaSuccess;
   count_launch();
-  rmsnorm_kernel<<<T, kRowThreads, 0, st>>>(x, (const __nv_bfloat16*)g, (__nv_bfloat16*)out, d, eps);
-  return cudaGetLastError();
+  return launch_pdl(rmsnorm_kernel, dim3(T), dim3(kRowThreads), 0, st, x, (const __nv_bfloat16*)g, (__nv_bfloat16*)out, d, eps);
 }
 cudaError_t launch_gather_rmsnorm(const float* x, const int32_t* rows, const void* g, void* out, int R, int d,
                                   float eps, cudaStream_t st) {
   if (R == 0) return cudaSuccess;
   count_launch();
-  gather_rmsnorm_kernel<<<R, kRowThreads, 0, st>>>(x, rows, (const __nv_bfloat16*)g, (__nv_bfloat16*)out, d, eps);
-  return cudaGetLastError();
+  return launch_pdl(gather_rmsnorm_kernel, dim3(R), dim3(kRowThreads), 0, st, x, rows, (const __nv_bfloat16*)g, (__nv_bfloat16*)out, d, eps);
 }
 cudaError_t launch_add_rmsnorm(float* resid, const void* add, const void* g, void* out, int T, int d, float eps,
                                cudaStream_t st) {
   if (T == 0) return cudaSuccess;
   count_launch();
-  add_rmsnorm_kernel<<<T, kRowThreads, 0, st>>>(resid, (const __nv_bfloat16*)add, (const __nv_bfloat16*)g,
+  return launch_pdl(add_rmsnorm_kernel, dim3(T), dim3(kRowThreads), 0, st, resid, (const __nv_bfloat16*)add, (const __nv_bfloat16*)g,
                                                 (__nv_bfloat16*)out, d, eps);
-  return cudaGetLastError();
 }
 cudaError_t launch_add_f32(float* resid, const void* add_bf16, size_t n, cudaStream_t st) {
   if (n == 0) return cudaSuccess;
   count_launch();
-  add_f32_kernel<<<grid_of(int64_t(n)), 256, 0, st>>>(resid, (const __nv_bfloat16*)add_bf16, int64_t(n));
-  return cudaGetLastError();
+  return launch_pdl(add_f32_kernel, dim3(grid_of(int64_t(n))), dim3(256), 0, st, resid, (const __nv_bfloat16*)add_bf16, int64_t(n));
 }
 cudaError_t launch_unshard_logits(const float* in, float* out, int R, int Vl, int tp, cudaStream_t st) {
   count_launch();
-  unshard_logits_kernel<<<grid_of(int64_t(R) * Vl * tp), 256, 0, st>>>(in, out, R, Vl, tp);
-  return cudaGetLastError();
+  return launch_pdl(unshard_logits_kernel, dim3(grid_of(int64_t(R) * Vl * tp)), dim3(256), 0, st, in, out, R, Vl, tp);
 }
 cudaError_t launch_argmax(const void* logits, int logits_f32, int R, int V, int32_t* out, cudaStream_t st) {
   if (R == 0) return cudaSuccess;
   count_launch();
-  argmax_kernel<<<R, 1024, 0, st>>>(logits, logits_f32, V, out);
-  return cudaGetLastError();
+  return launch_pdl(argmax_kernel, dim3(R), dim3(1024), 0, st, logits, logits_f32, V, out);
 }
 cudaError_t launch_f32_to_bf16(const float* x, void* y, int64_t n, cudaStream_t st) {
   if (n == 0) return cudaSuccess;
   count_launch();
   const int blocks = int((n + 1023) / 1024 < 4096 ? (n + 1023) / 1024 : 4096);
-  f32_to_bf16_kernel<<<blocks, 1024, 0, st>>>(x, (__nv_bfloat16*)y, n);
-  return cudaGetLastError();
+  return launch_pdl(f32_to_bf16_kernel, dim3(blocks), dim3(1024), 0, st, x, (__nv_bfloat16*)y, n);
 }
 
 }  // namespace qos

@@ -220,7 +220,12 @@ struct qos_engine {
   };
   std::vector<LMaps> lmaps;
   CUtensorMap head_map[2];
-  CUtensorMap a_h, a_attn, a_act, a_hR, kv_map;
+  struct ActMap {
+    CUtensorMap m128;    // box 128 rows: A operand of gemm.cu
+    CUtensorMap sw[5];   // box 16/32/64/128/256 rows: token operand of gemm_swab.cu
+  };
+  ActMap a_h, a_attn, a_act, a_hR;
+  CUtensorMap kv_map;
   float2* rope_tab = nullptr;
   int32_t* d_tables = nullptr;
   // host state
@@ -240,6 +245,7 @@ struct qos_engine {
   int dual_sms_pre = 0, dual_sms_dec = 0;  // SM budgets of the two streams' GEMMs (0 = all)
   bool overlap_attn = true;       // QOS_OVERLAP_ATTN=0 serialises a7 and a8 (for measurement)
   bool gemm_splitk = true;        // QOS_GEMM_SPLITK=0 disables split-K for small-M GEMMs
+  int gemm_swab = 1;              // weight-streaming GEMM (gemm_swab.cu): 0 never, 1 auto, 2 always
   // timing
   bool timing = false;
   std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> tev;
@@ -311,10 +317,15 @@ int build_maps(qos_engine* e) {
   for (int b = 0; b < 2; ++b)
     QOS_TRY(make_tmap_2d_bf16(&e->head_map[b], W(e, e->wl.head), e->sh.V, d, d, b ? 256 : 128, 64, true));
   const auto& s = e->wsl;
-  QOS_TRY(make_tmap_2d_bf16(&e->a_h, e->ws + s.h, c.max_batch_tokens, d, d, 128, 64, true));
-  QOS_TRY(make_tmap_2d_bf16(&e->a_attn, e->ws + s.attn, c.max_batch_tokens, e->sh.H * hd, e->sh.H * hd, 128, 64, true));
-  QOS_TRY(make_tmap_2d_bf16(&e->a_act, e->ws + s.act, c.max_batch_tokens, e->sh.F, e->sh.F, 128, 64, true));
-  QOS_TRY(make_tmap_2d_bf16(&e->a_hR, e->ws + s.hR, c.max_batch_rows, d, d, 128, 64, true));
+  auto act = [&](qos_engine::ActMap& m, const void* base, int64_t rows, int64_t cols) -> int {
+    QOS_TRY(make_tmap_2d_bf16(&m.m128, base, rows, cols, cols, 128, 64, true));
+    for (int i = 0; i < 5; ++i) QOS_TRY(make_tmap_2d_bf16(&m.sw[i], base, rows, cols, cols, 16u << i, 64, true));
+    return QOS_OK;
+  };
+  QOS_TRY(act(e->a_h, e->ws + s.h, c.max_batch_tokens, d));
+  QOS_TRY(act(e->a_attn, e->ws + s.attn, c.max_batch_tokens, e->sh.H * hd));
+  QOS_TRY(act(e->a_act, e->ws + s.act, c.max_batch_tokens, e->sh.F));
+  QOS_TRY(act(e->a_hR, e->ws + s.hR, c.max_batch_rows, d));
   QOS_TRY(make_tmap_3d_bf16(&e->kv_map, e->kv, hd, uint64_t(c.num_blocks) * e->sh.Hkv * 16, uint64_t(c.n_layers) * 2,
                             64, 16, 1));
   return QOS_OK;
@@ -525,13 +536,30 @@ int flush_table_updates(qos_engine* e, cudaStream_t st) {
   return QOS_OK;
 }
 
-int gemm(qos_engine* e, const CUtensorMap& ta, const CUtensorMap (&tb)[2], int64_t M, int64_t N, int64_t K, int epi,
-         void* C, int64_t ldc, const float* bias, cudaStream_t st) {
-  const int bn = gemm_pick_bn(M, N, epi, e->num_sms);
-  const int ks = e->gemm_splitk ? gemm_pick_ksplit(M, N, K, bn, e->num_sms, kGemmMaxUnits) : 1;
+static int swab_index(int bnt) { return bnt == 16 ? 0 : bnt == 32 ? 1 : bnt == 64 ? 2 : bnt == 128 ? 3 : 4; }
+
+// One projection GEMM of M rows: gemm_swab.cu (weight-streaming, swap-AB, stream-K) at small M,
+// else gemm.cu (activation-stationary tiles, optional split-K).
+int gemm_any(qos_engine* e, const qos_engine::ActMap& am, const CUtensorMap (&tb)[2], int64_t M, int64_t N, int64_t K,
+             int epi, void* C, int64_t ldc, const float* bias, cudaStream_t st, int sms, float* part, int* cnt,
+             int a_row0, const QkvRopeArgs* rope) {
   count_launch();
-  return gemm_run(ta, tb[bn == 256 ? 1 : 0], bn, M, N, K, epi, C, ldc, bias, e->num_sms, st, ks,
-                  reinterpret_cast<float*>(e->ws + e->wsl.gemm_part), reinterpret_cast<int*>(e->ws + e->wsl.gemm_cnt));
+  if (N % 128 == 0 && (e->gemm_swab == 2 || (e->gemm_swab == 1 && swab_prefer(M, N, sms)))) {
+    const int bnt = swab_pick_bnt(M);
+    return gemm_swab_run(tb[0], am.sw[swab_index(bnt)], bnt, M, N, K, epi, C, ldc, bias, sms, st, part, cnt,
+                         int64_t(kGemmMaxUnits) * 128 * 256, kGemmMaxTiles, a_row0, rope, !e->dual_stream);
+  }
+  const int bn = gemm_pick_bn(M, N, epi, sms);
+  const int ks = e->gemm_splitk ? gemm_pick_ksplit(M, N, K, bn, sms, kGemmMaxUnits) : 1;
+  return gemm_run(am.m128, tb[bn == 256 ? 1 : 0], bn, M, N, K, epi, C, ldc, bias, sms, st, ks, part, cnt, a_row0, sms,
+                  rope);
+}
+
+int gemm(qos_engine* e, const qos_engine::ActMap& am, const CUtensorMap (&tb)[2], int64_t M, int64_t N, int64_t K,
+         int epi, void* C, int64_t ldc, const float* bias, cudaStream_t st) {
+  return gemm_any(e, am, tb, M, N, K, epi, C, ldc, bias, st, e->num_sms,
+                  reinterpret_cast<float*>(e->ws + e->wsl.gemm_part), reinterpret_cast<int*>(e->ws + e->wsl.gemm_cnt), 0,
+                  nullptr);
 }
 
 int allreduce_bf16(qos_engine* e, void* buf, size_t count, cudaStream_t st) {
@@ -556,15 +584,12 @@ struct Seg {
   int sms;       // SM budget of this stream's GEMMs (0 = all)
 };
 
-int gemm_seg(qos_engine* e, const Seg& g, const CUtensorMap& ta, const CUtensorMap (&tb)[2], int64_t N, int64_t K,
-             int epi, void* C, int64_t ldc, const float* bias, const QkvRopeArgs* rope = nullptr) {
+int gemm_seg(qos_engine* e, const Seg& g, const qos_engine::ActMap& am, const CUtensorMap (&tb)[2], int64_t N,
+             int64_t K, int epi, void* C, int64_t ldc, const float* bias, const QkvRopeArgs* rope = nullptr) {
   const int sms = g.sms > 0 ? g.sms : e->num_sms;
-  const int bn = gemm_pick_bn(g.n, N, epi, sms);
-  const int ks = e->gemm_splitk ? gemm_pick_ksplit(g.n, N, K, bn, sms, kGemmMaxUnits) : 1;
-  count_launch();
   const size_t esz = (epi == EPI_STORE_F32 || epi == EPI_ADD_F32) ? 4 : 2;
-  return gemm_run(ta, tb[bn == 256 ? 1 : 0], bn, g.n, N, K, epi, reinterpret_cast<uint8_t*>(C) + size_t(g.row0) * ldc * esz,
-                  ldc, bias, sms, g.st, ks, g.gpart, g.gcnt, g.row0, sms, rope);
+  return gemm_any(e, am, tb, g.n, N, K, epi, reinterpret_cast<uint8_t*>(C) + size_t(g.row0) * ldc * esz, ldc, bias,
+                  g.st, sms, g.gpart, g.gcnt, g.row0, rope);
 }
 
 // The layer loop.  `dm` = device metadata block of this step.
@@ -910,6 +935,7 @@ int qos_engine_create(const qos_model_cfg* cfg, int device, int tp_rank, int tp_
   cudaStreamCreateWithFlags(&e->stream, cudaStreamNonBlocking);
   if (const char* ov = getenv("QOS_OVERLAP_ATTN")) e->overlap_attn = atoi(ov) != 0;
   if (const char* sk = getenv("QOS_GEMM_SPLITK")) e->gemm_splitk = atoi(sk) != 0;
+  if (const char* sw = getenv("QOS_GEMM_SWAB")) e->gemm_swab = atoi(sw);
   if (const char* du = getenv("QOS_DUAL")) e->dual_stream = atoi(du) != 0;
   if (const char* a = getenv("QOS_DUAL_MIN_PREFILL")) e->dual_min_prefill = atoi(a);
   if (const char* a = getenv("QOS_DUAL_MIN_DECODE")) e->dual_min_decode = atoi(a);
@@ -1251,6 +1277,8 @@ int qos_engine_set_option(qos_engine_t* e, const char* name, int64_t value) {
   const std::string n(name);
   if (n == "overlap_attn") e->overlap_attn = value != 0;
   else if (n == "gemm_splitk") e->gemm_splitk = value != 0;
+  else if (n == "pdl") set_pdl(value != 0);  // process-wide
+  else if (n == "gemm_swab") e->gemm_swab = int(value < 0 ? 0 : value > 2 ? 2 : value);
   else if (n == "dual_stream") e->dual_stream = value != 0;
   else if (n == "dual_min_prefill") e->dual_min_prefill = int(value);
   else if (n == "dual_min_decode") e->dual_min_decode = int(value);
@@ -1317,6 +1345,18 @@ static int op_gemm(const void* A, const void* B, void* C, int64_t M, int64_t N, 
         cudaMalloc(&cnt, size_t(kGemmMaxTiles) * 4) != cudaSuccess || cudaMemset(cnt, 0, size_t(kGemmMaxTiles) * 4))
       return set_error(QOS_ERR_OOM, "gemm split-K workspace");
   }
+  static const bool swab_env = !(getenv("QOS_GEMM_SWAB") && atoi(getenv("QOS_GEMM_SWAB")) == 0);
+  const int64_t ldc = epi == QOS_EPI_SILU_GATE ? N / 2 : N;
+  if (ksplit < 0 || (ksplit == 0 && swab_env && swab_prefer(M, N, sms))) {
+    // weight-streaming swap-AB kernel (gemm_swab.cu)
+    const int bnt = swab_pick_bnt(M);
+    CUtensorMap tw, tt;
+    QOS_TRY(make_tmap_2d_bf16(&tw, B, uint64_t(N), uint64_t(K), uint64_t(K), 128, 64, true));
+    QOS_TRY(make_tmap_2d_bf16(&tt, A, uint64_t(M), uint64_t(K), uint64_t(K), uint32_t(bnt), 64, true));
+    count_launch();
+    return gemm_swab_run(tw, tt, bnt, M, N, K, epi, C, ldc, bias, sms, reinterpret_cast<cudaStream_t>(stream), part,
+                         cnt, int64_t(kGemmMaxUnits) * 128 * 256, kGemmMaxTiles, 0, nullptr);
+  }
   const int64_t tiles = ((M + 127) / 128) * ((N + bn - 1) / bn);
   int ks = ksplit <= 0 ? gemm_pick_ksplit(M, N, K, bn, sms, kGemmMaxUnits) : ksplit;
   if (ks > 1 && (tiles > kGemmMaxTiles || tiles * ks > kGemmMaxUnits || (K / 64) < ks))
@@ -1324,7 +1364,6 @@ static int op_gemm(const void* A, const void* B, void* C, int64_t M, int64_t N, 
   CUtensorMap ta, tb;
   QOS_TRY(make_tmap_2d_bf16(&ta, A, uint64_t(M), uint64_t(K), uint64_t(K), 128, 64, true));
   QOS_TRY(make_tmap_2d_bf16(&tb, B, uint64_t(N), uint64_t(K), uint64_t(K), uint32_t(bn), 64, true));
-  const int64_t ldc = epi == QOS_EPI_SILU_GATE ? N / 2 : N;
   count_launch();
   return gemm_run(ta, tb, bn, M, N, K, epi, C, ldc, bias, sms, reinterpret_cast<cudaStream_t>(stream), ks, part, cnt);
 }

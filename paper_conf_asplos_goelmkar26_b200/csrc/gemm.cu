@@ -17,11 +17,23 @@
 #include <cudaTypedefs.h>
 
 #include <cstdio>
+#include <cstdlib>
 
 #include "common.cuh"
 #include "internal.h"
 
 namespace qos {
+
+// Programmatic dependent launch switch for the step-chain kernels (see common.cuh).
+static int g_pdl = -1;
+bool pdl_enabled() {
+  if (g_pdl < 0) {
+    const char* v = getenv("QOS_PDL");
+    g_pdl = (v && atoi(v) == 0) ? 0 : 1;
+  }
+  return g_pdl != 0;
+}
+void set_pdl(bool on) { g_pdl = on ? 1 : 0; }
 
 constexpr int kBM = 128;
 constexpr int kBK = 64;
@@ -205,6 +217,8 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  griddep_launch_dependents();  // the next kernel may start its prologue as SMs free up
+  if (warp != 0) griddep_wait();  // epilogue reads/writes C (residual, KV cache) of earlier kernels
 
   // work unit u = ((n_t * ksplit) + split) * mt + m_t: consecutive units share a weight slice
   const int ks = p.ksplit;
@@ -226,10 +240,34 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
       const uint64_t pol_b = l2_evict_first();  // weights: streamed once per M-tile group
       int stage = 0;
       uint32_t phase = 0;
+      // Programmatic dependent launch: the weight (B) tiles of the first stages do not depend on
+      // the previous kernel, so they are requested before griddepcontrol.wait; the activation (A)
+      // tiles, produced by the previous kernel, only after it.
+      int npre = 0;
+      if (blockIdx.x < num_units) {
+        int m_t, n_t, sp, kb0, kb1;
+        decode_unit(blockIdx.x, m_t, n_t, sp, kb0, kb1);
+        npre = min(S, kb1 - kb0);
+        for (int i = 0; i < npre; ++i) {
+          uint8_t* sa = smem + i * Cfg::kStageBytes;
+          mbar_arrive_expect_tx(&full[i], Cfg::kStageBytes);
+          tma_load_2d_hint(sa + Cfg::kABytes, &tmB, &full[i], (kb0 + i) * kBK, n_t * BN, pol_b);
+        }
+        griddep_wait();
+        for (int i = 0; i < npre; ++i)
+          tma_load_2d_hint(smem + i * Cfg::kStageBytes, &tmA, &full[i], (kb0 + i) * kBK, p.a_row0 + m_t * kBM, pol_a);
+      } else {
+        griddep_wait();
+      }
+      int it = 0;
       for (int u = blockIdx.x; u < num_units; u += gridDim.x) {
         int m_t, n_t, sp, kb0, kb1;
         decode_unit(u, m_t, n_t, sp, kb0, kb1);
-        for (int kb = kb0; kb < kb1; ++kb) {
+        for (int kb = kb0; kb < kb1; ++kb, ++it) {
+          if (it < npre) {  // issued above
+            if (++stage == S) { stage = 0; phase ^= 1; }
+            continue;
+          }
           mbar_wait(&empty[stage], phase ^ 1);
           uint8_t* sa = smem + stage * Cfg::kStageBytes;
           mbar_arrive_expect_tx(&full[stage], Cfg::kStageBytes);
@@ -489,8 +527,7 @@ static cudaError_t launch_gemm_t(const CUtensorMap& ta, const CUtensorMap& tb, c
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
-  kern<<<grid, kGemmThreads, GemmCfg<BN>::kSmemBytes, st>>>(ta, tb, a);
-  return cudaGetLastError();
+  return launch_pdl(kern, dim3(grid), dim3(kGemmThreads), GemmCfg<BN>::kSmemBytes, st, ta, tb, a);
 }
 
 int gemm_pick_bn(int64_t M, int64_t N, int epi, int num_sms) {

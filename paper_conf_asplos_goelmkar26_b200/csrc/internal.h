@@ -10,6 +10,9 @@
 
 namespace qos {
 
+bool pdl_enabled();
+void set_pdl(bool on);
+
 enum { EPI_STORE_BF16 = QOS_EPI_STORE_BF16, EPI_STORE_F32 = QOS_EPI_STORE_F32, EPI_BIAS_BF16 = QOS_EPI_BIAS_BF16,
        EPI_SILU_GATE = QOS_EPI_SILU_GATE, EPI_ADD_F32 = QOS_EPI_ADD_F32,
        EPI_QKV_ROPE = 5 /* internal: a4 + a5 + a6 fused (RoPE, q -> C, k/v -> paged cache; +bias) */ };
@@ -41,6 +44,19 @@ int gemm_pick_ksplit(int64_t M, int64_t N, int64_t K, int bn, int num_sms, int64
 int gemm_run(const CUtensorMap& ta, const CUtensorMap& tb, int bn, int64_t M, int64_t N, int64_t K, int epi, void* C,
              int64_t ldc, const float* bias, int num_sms, cudaStream_t st, int ksplit = 1, float* part = nullptr,
              int* counters = nullptr, int a_row0 = 0, int max_ctas = 0, const QkvRopeArgs* rope = nullptr);
+
+// ------------------------------------------------------------------ small-T GEMM (gemm_swab.cu)
+// Swap-AB weight-streaming GEMM: tw = weight map (box 128 x 64), tt = token map (box bnt x 64).
+// Requires N % 128 == 0.  part: >= 2 * grid * bnt * 128 floats; counters: >= (N/128) * ceil(M/bnt).
+// coop: split tiles are reduced by all their participants after their ranges (spin-waits on
+// the other CTAs of the grid: only when no concurrent kernel can hold SMs indefinitely —
+// false in the two-stream mode, where the last arriving CTA reduces alone).
+int swab_pick_bnt(int64_t M);
+bool swab_prefer(int64_t M, int64_t N, int num_sms);  // automatic kernel choice
+int swab_grid(int64_t M, int64_t N, int64_t K, int bnt, int num_sms);
+int gemm_swab_run(const CUtensorMap& tw, const CUtensorMap& tt, int bnt, int64_t M, int64_t N, int64_t K, int epi,
+                  void* C, int64_t ldc, const float* bias, int num_sms, cudaStream_t st, float* part, int* counters,
+                  int64_t part_floats, int max_tiles, int a_row0, const QkvRopeArgs* rope, bool coop = true);
 
 // ------------------------------------------------------------------ synthetic generator (gen.cu)
 enum GenKind { GEN_LINEAR = 0, GEN_EMBED = 1, GEN_NORM = 2, GEN_BIAS = 3 };

@@ -261,3 +261,49 @@ def test_gemm_splitk_parity(torch_cuda, M, N, K, ks, epi):
         got = dC.float().cpu().numpy()
         tol = 1e-5 if epi in ("store_f32", "add_f32") else 8e-3
         assert row_rel_err(got, ref) <= tol
+
+
+@pytest.mark.parametrize("M,N,K", [(1, 128, 64), (16, 4096, 4096), (17, 1024, 2048), (100, 640, 1536),
+                                   (256, 512, 8192), (300, 384, 1024)])
+@pytest.mark.parametrize("epi", ["store_f32", "store_bf16", "add_f32", "bias_bf16", "silu_gate"])
+def test_gemm_swab_parity(torch_cuda, M, N, K, epi):
+    """Weight-streaming swap-AB stream-K kernel (ksplit < 0): every epilogue, ragged token
+    counts, tiles cut across CTAs (K up to 8192), two token tiles (M = 300); run twice —
+    the per-tile arrival counters must be reset, and the fixed-order reduction makes the two
+    results bit-identical."""
+    torch = torch_cuda
+    from oracle.model import silu
+    from paper_conf_asplos_goelmkar26_b200 import qoserve as q
+    rng = np.random.default_rng(M * 3 + N + K)
+    A = bits_to_f64(bf16_bits(rng.uniform(-1, 1, (M, K))))
+    B = bits_to_f64(bf16_bits(rng.uniform(-1, 1, (N, K)) / np.sqrt(K)))
+    dA, dB = _dev_bf16(torch, A), _dev_bf16(torch, B)
+    ref = A @ B.T
+    bias = None
+    init = None
+    if epi == "silu_gate":
+        g = np.concatenate([ref[:, 128 * j:128 * j + 64] for j in range(N // 128)], axis=1)
+        u = np.concatenate([ref[:, 128 * j + 64:128 * j + 128] for j in range(N // 128)], axis=1)
+        ref = silu(g) * u
+        dC = torch.empty((M, N // 2), dtype=torch.bfloat16, device="cuda")
+    elif epi in ("store_f32", "add_f32"):
+        init = rng.uniform(-1, 1, (M, N)).astype(np.float32) if epi == "add_f32" else np.zeros((M, N), np.float32)
+        dC = torch.from_numpy(init.copy()).cuda()
+        ref = ref + init.astype(np.float64)
+    else:
+        dC = torch.empty((M, N), dtype=torch.bfloat16, device="cuda")
+        if epi == "bias_bf16":
+            bvals = bits_to_f64(bf16_bits(rng.uniform(-0.02, 0.02, N)))
+            bias = torch.from_numpy(bvals.astype(np.float32)).cuda()
+            ref = ref + bvals
+    outs = []
+    for _ in range(2):
+        if init is not None:
+            dC.copy_(torch.from_numpy(init.copy()).cuda())
+        q.qos_op_gemm_ex(dA.data_ptr(), dB.data_ptr(), dC.data_ptr(), M, N, K, epi,
+                         bias.data_ptr() if bias is not None else None, -1)
+        torch.cuda.synchronize()
+        outs.append(dC.float().cpu().numpy())
+        tol = 1e-5 if epi in ("store_f32", "add_f32") else 8e-3
+        assert row_rel_err(outs[-1], ref) <= tol
+    assert np.array_equal(outs[0], outs[1])

@@ -1,7 +1,13 @@
-"""Microbenchmark of the tcgen05 GEMM (qos_op_gemm_ex) on the Llama-3-8B projection shapes across
-M (= tokens in the step): achieved TFLOP/s and weight-streaming GB/s per launch.
+"""Microbenchmark of the tcgen05 GEMMs (qos_op_gemm_ex) on the Llama-3-8B projection shapes
+across M (= tokens in the step): per-launch time, achieved TFLOP/s and weight-streaming GB/s.
 
-  python tools/gemm_bench.py [--ms 16,64,128,256,512,2176] [--ksplit 0]
+Launches run back to back (as in a step, PDL on) over rotating copies of the weight matrix
+whose total size exceeds L2, so every launch streams its weights from HBM and no launch pays
+for write-backs of a dirty L2 (a zero-fill flush before each launch costs ~20 us of write-back
+to the next kernel and hides the small-M behaviour).
+
+  python tools/gemm_bench.py [--ms 1,16,64,128,256,512,2176] [--ksplit 0] [--shapes qkv,o]
+  ksplit: 0 auto, >= 1 tile kernel with that split-K, -1 weight-streaming (swap-AB) kernel
 """
 import argparse
 import json
@@ -18,32 +24,49 @@ SHAPES = {"qkv": (6144, 4096, "store_bf16"), "o": (4096, 4096, "add_f32"), "gate
           "down": (4096, 14336, "add_f32"), "head": (128256, 4096, "store_f32")}
 
 ap = argparse.ArgumentParser()
-ap.add_argument("--ms", default="16,64,128,256,384,512,1024,2176")
+ap.add_argument("--ms", default="1,16,64,128,256,384,512,1024,2176")
 ap.add_argument("--ksplit", type=int, default=0)
-ap.add_argument("--iters", type=int, default=20)
+ap.add_argument("--iters", type=int, default=24)
+ap.add_argument("--shapes", default=",".join(SHAPES))
 a = ap.parse_args()
 torch.cuda.set_device(0)
-flush = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device="cuda")   # > L2: weights come from HBM
-for name, (N, K, epi) in SHAPES.items():
-    B = (torch.randn(N, K, device="cuda") / K ** 0.5).to(torch.bfloat16)
+L2 = 126 * 1024 * 1024
+for name in a.shapes.split(","):
+    N, K, epi = SHAPES[name]
+    wbytes = N * K * 2
+    ncopy = max(2, -(-3 * L2 // wbytes))
+    Bs = [(torch.randn(N, K, device="cuda") / K ** 0.5).to(torch.bfloat16) for _ in range(ncopy)]
     for M in [int(x) for x in a.ms.split(",")]:
         if name == "head" and M > 512:
             continue
         A = torch.randn(M, K, device="cuda").to(torch.bfloat16)
         Cn = N // 2 if epi == "silu_gate" else N
         Cout = torch.zeros(M, Cn, device="cuda", dtype=torch.float32 if "f32" in epi else torch.bfloat16)
-        ts = []
-        for it in range(a.iters + 3):
-            flush.zero_()
-            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            e0.record()
-            q.qos_op_gemm_ex(A.data_ptr(), B.data_ptr(), Cout.data_ptr(), M, N, K, epi, None, a.ksplit)
-            e1.record()
-            torch.cuda.synchronize()
-            if it >= 3:
-                ts.append(e0.elapsed_time(e1))
-        ts.sort()
-        ms = ts[len(ts) // 2]
-        print(json.dumps({"gemm": name, "M": M, "N": N, "K": K, "us": round(ms * 1e3, 1),
-                          "tflops": round(2 * M * N * K / ms / 1e9, 1),
-                          "weight_gbs": round(N * K * 2 / ms / 1e6, 1)}), flush=True)
+
+        def launch(i, st=None):
+            q.qos_op_gemm_ex(A.data_ptr(), Bs[i % ncopy].data_ptr(), Cout.data_ptr(), M, N, K, epi, None, a.ksplit,
+                             st)
+
+        for i in range(ncopy + 2):
+            launch(i)
+        torch.cuda.synchronize()
+        # captured in a CUDA graph so host-side launch cost does not starve short kernels
+        s = torch.cuda.Stream()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=s):
+            for i in range(a.iters):
+                launch(i, s.cuda_stream)
+        g.replay()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        g.replay()
+        e1.record()
+        torch.cuda.synchronize()
+        us = e0.elapsed_time(e1) * 1e3 / a.iters
+        print(json.dumps({"gemm": name, "M": M, "N": N, "K": K, "ksplit": a.ksplit, "us": round(us, 2),
+                          "tflops": round(2 * M * N * K / us / 1e6, 1),
+                          "weight_gbs": round(wbytes / us / 1e3, 1)}), flush=True)
+        del A, Cout
+    del Bs
+    torch.cuda.empty_cache()
