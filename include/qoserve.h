@@ -202,6 +202,9 @@ int qos_profile_step_ex(qos_engine_t* eng, int32_t chunk_len, int32_t kv_start,
  *   "gemm_swab" (1)        weight-streaming swap-AB GEMM for small token counts: 0 never,
  *                          1 automatic (small T, or T <= 256 with few output tiles), 2 always
  *                          (where N % 128 == 0); env QOS_GEMM_SWAB
+ *   "gemm_streamk" (0)     stream-K mode of the tile GEMM: 0 never, 1 when whole-tile waves
+ *                          leave > 5% of the last wave idle, 2 always (experiments; slower on
+ *                          B200 at large T: ranges out of phase lose L2 reuse); env QOS_GEMM_STREAMK
  *   "pdl" (1)              programmatic dependent launch of the step's kernel chain (each
  *                          kernel's prologue and weight prefetch overlap the previous kernel's
  *                          tail); process-wide, env QOS_PDL

@@ -39,7 +39,12 @@ int qos_op_gemm(const void* A, const void* B, void* C, int64_t M, int64_t N, int
  *   ksplit >= 1  the tile kernel (128-token x 128/256-feature tiles) with that split-K factor:
  *                each of `ksplit` CTAs accumulates a K slice of a tile, parks an fp32 partial,
  *                and the last one to arrive sums the slices in slice order (deterministic);
- *   ksplit < 0   the weight-streaming kernel (requires N % 128 == 0): computes C^T tile by
+ *   ksplit <= -2 the tile kernel in stream-K mode: the (tile, k-block) space cut into equal
+ *                contiguous ranges, one per CTA; tiles cut by a range boundary are summed from
+ *                fp32 partials in CTA order (deterministic).  Never chosen automatically: on
+ *                B200 the unaligned ranges lose the L2 reuse of lock-step whole-tile waves
+ *                (1.5-1.8x slower at T = 2176, tools/gemm_bench.py).
+ *   ksplit = -1  the weight-streaming kernel (requires N % 128 == 0): computes C^T tile by
  *                tile as W_tile(128 rows) · A^T on tcgen05 (token count = UMMA N), the
  *                (tile, k-block) space split in equal contiguous ranges over the SMs
  *                ("stream-K"); tiles cut by a range boundary are summed by their last

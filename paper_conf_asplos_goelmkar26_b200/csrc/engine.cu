@@ -246,6 +246,8 @@ struct qos_engine {
   bool overlap_attn = true;       // QOS_OVERLAP_ATTN=0 serialises a7 and a8 (for measurement)
   bool gemm_splitk = true;        // QOS_GEMM_SPLITK=0 disables split-K for small-M GEMMs
   int gemm_swab = 1;              // weight-streaming GEMM (gemm_swab.cu): 0 never, 1 auto, 2 always
+  int gemm_streamk = 0;           // stream-K tile GEMM: 0 never (default: measured slower on B200,
+                                  // unaligned ranges lose the L2 reuse of lock-step waves), 1 auto, 2 always
   // timing
   bool timing = false;
   std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> tev;
@@ -552,7 +554,7 @@ int gemm_any(qos_engine* e, const qos_engine::ActMap& am, const CUtensorMap (&tb
   const int bn = gemm_pick_bn(M, N, epi, sms);
   const int ks = e->gemm_splitk ? gemm_pick_ksplit(M, N, K, bn, sms, kGemmMaxUnits) : 1;
   return gemm_run(am.m128, tb[bn == 256 ? 1 : 0], bn, M, N, K, epi, C, ldc, bias, sms, st, ks, part, cnt, a_row0, sms,
-                  rope);
+                  rope, e->gemm_streamk, !e->dual_stream);
 }
 
 int gemm(qos_engine* e, const qos_engine::ActMap& am, const CUtensorMap (&tb)[2], int64_t M, int64_t N, int64_t K,
@@ -936,6 +938,7 @@ int qos_engine_create(const qos_model_cfg* cfg, int device, int tp_rank, int tp_
   if (const char* ov = getenv("QOS_OVERLAP_ATTN")) e->overlap_attn = atoi(ov) != 0;
   if (const char* sk = getenv("QOS_GEMM_SPLITK")) e->gemm_splitk = atoi(sk) != 0;
   if (const char* sw = getenv("QOS_GEMM_SWAB")) e->gemm_swab = atoi(sw);
+  if (const char* sk = getenv("QOS_GEMM_STREAMK")) e->gemm_streamk = atoi(sk);
   if (const char* du = getenv("QOS_DUAL")) e->dual_stream = atoi(du) != 0;
   if (const char* a = getenv("QOS_DUAL_MIN_PREFILL")) e->dual_min_prefill = atoi(a);
   if (const char* a = getenv("QOS_DUAL_MIN_DECODE")) e->dual_min_decode = atoi(a);
@@ -1279,6 +1282,7 @@ int qos_engine_set_option(qos_engine_t* e, const char* name, int64_t value) {
   else if (n == "gemm_splitk") e->gemm_splitk = value != 0;
   else if (n == "pdl") set_pdl(value != 0);  // process-wide
   else if (n == "gemm_swab") e->gemm_swab = int(value < 0 ? 0 : value > 2 ? 2 : value);
+  else if (n == "gemm_streamk") e->gemm_streamk = int(value < 0 ? 0 : value > 2 ? 2 : value);
   else if (n == "dual_stream") e->dual_stream = value != 0;
   else if (n == "dual_min_prefill") e->dual_min_prefill = int(value);
   else if (n == "dual_min_decode") e->dual_min_decode = int(value);
@@ -1347,7 +1351,7 @@ static int op_gemm(const void* A, const void* B, void* C, int64_t M, int64_t N, 
   }
   static const bool swab_env = !(getenv("QOS_GEMM_SWAB") && atoi(getenv("QOS_GEMM_SWAB")) == 0);
   const int64_t ldc = epi == QOS_EPI_SILU_GATE ? N / 2 : N;
-  if (ksplit < 0 || (ksplit == 0 && swab_env && swab_prefer(M, N, sms))) {
+  if (ksplit == -1 || (ksplit == 0 && swab_env && swab_prefer(M, N, sms))) {
     // weight-streaming swap-AB kernel (gemm_swab.cu)
     const int bnt = swab_pick_bnt(M);
     CUtensorMap tw, tt;
@@ -1358,14 +1362,16 @@ static int op_gemm(const void* A, const void* B, void* C, int64_t M, int64_t N, 
                          cnt, int64_t(kGemmMaxUnits) * 128 * 256, kGemmMaxTiles, 0, nullptr);
   }
   const int64_t tiles = ((M + 127) / 128) * ((N + bn - 1) / bn);
-  int ks = ksplit <= 0 ? gemm_pick_ksplit(M, N, K, bn, sms, kGemmMaxUnits) : ksplit;
+  const int sk_mode = ksplit <= -2 ? 2 : 0;
+  int ks = ksplit <= -2 ? 1 : ksplit <= 0 ? gemm_pick_ksplit(M, N, K, bn, sms, kGemmMaxUnits) : ksplit;
   if (ks > 1 && (tiles > kGemmMaxTiles || tiles * ks > kGemmMaxUnits || (K / 64) < ks))
     return set_error(QOS_ERR_INVALID_ARG, "gemm: ksplit too large for the shape / workspace");
   CUtensorMap ta, tb;
   QOS_TRY(make_tmap_2d_bf16(&ta, A, uint64_t(M), uint64_t(K), uint64_t(K), 128, 64, true));
   QOS_TRY(make_tmap_2d_bf16(&tb, B, uint64_t(N), uint64_t(K), uint64_t(K), uint32_t(bn), 64, true));
   count_launch();
-  return gemm_run(ta, tb, bn, M, N, K, epi, C, ldc, bias, sms, reinterpret_cast<cudaStream_t>(stream), ks, part, cnt);
+  return gemm_run(ta, tb, bn, M, N, K, epi, C, ldc, bias, sms, reinterpret_cast<cudaStream_t>(stream), ks, part, cnt,
+                  0, 0, nullptr, sk_mode, true);
 }
 
 int qos_op_gemm(const void* A, const void* B, void* C, int64_t M, int64_t N, int64_t K, int epi, const float* bias,

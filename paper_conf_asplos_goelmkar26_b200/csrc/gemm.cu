@@ -53,6 +53,9 @@ struct GemmArgs {
   int M, N, K;
   int mt, nt;       // tiles along M and N
   int ksplit;       // K slices per tile (split-K for weight-bound small-M GEMMs); 1 = off
+  int sk;           // stream-K: the (tile, k-block) space in equal contiguous ranges per CTA
+  int coop;         // stream-K: cut tiles reduced by all their CTAs after their ranges
+  int64_t work;     // stream-K: mt * nt * kblocks
   void* C;
   int ldc;          // elements
   const float* bias;
@@ -114,12 +117,12 @@ QOS_DEV void epi_silu32(const GemmArgs& p, int row, int outcol, const float (&g)
 // straight into the paged cache at the row's slot with 32-byte stores.  `fetch(col, v16)`
 // returns 16 accumulator columns of this thread's row (TMEM or summed split-K partials).
 template <int BN, typename Fetch>
-QOS_DEV void epi_qkv_rope(const GemmArgs& p, int row, bool row_ok, int n_t, Fetch fetch) {
+QOS_DEV void epi_qkv_rope(const GemmArgs& p, int row, bool row_ok, int n_t, Fetch fetch, int h0 = 0, int hstep = 1) {
   const int hd = p.hd, half = hd / 2;
   const int ps = row_ok ? __ldg(p.pos + row) : 0;
   const int sl = row_ok ? __ldg(p.slot + row) : 0;
   const float2* cs = p.rope + size_t(ps) * half;
-  for (int hh = 0; hh < BN / hd; ++hh) {
+  for (int hh = h0; hh < BN / hd; hh += hstep) {
     const int col0 = n_t * BN + hh * hd;
     if (col0 >= p.N) break;  // warp-uniform
     const int head = col0 / hd;
@@ -166,6 +169,37 @@ QOS_DEV void epi_qkv_rope(const GemmArgs& p, int row, bool row_ok, int n_t, Fetc
       }
     }
   }
+}
+
+// Epilogue of one row of a tile from summed fp32 partials, in independent column units
+// u0, u0 + ustep, ... (32 columns; SiLU: 32 outputs = 32 gate + 32 up columns; QKV: one head),
+// so several CTAs can share the reduction of one tile.  fetch32(col, v) / fetch16(col, v)
+// return accumulator columns col.. of this thread's row.
+template <int BN, int EPI, typename F32, typename F16>
+QOS_DEV void epi_units(const GemmArgs& p, int row, bool row_ok, int n_t, int u0, int ustep, F32 fetch32, F16 fetch16) {
+  if constexpr (EPI == EPI_QKV_ROPE) {
+    epi_qkv_rope<BN>(p, row, row_ok, n_t, fetch16, u0, ustep);
+  } else if constexpr (EPI == EPI_SILU_GATE) {
+    for (int u = u0; u < BN / 64; u += ustep) {
+      const int g = u >> 1, h = u & 1;
+      float gv[32], uv[32];
+      fetch32(g * 128 + h * 32, gv);
+      fetch32(g * 128 + 64 + h * 32, uv);
+      const int col = n_t * (BN / 2) + g * 64 + h * 32;
+      if (row_ok && col < p.N / 2) epi_silu32(p, row, col, gv, uv);
+    }
+  } else {
+    for (int u = u0; u < BN / 32; u += ustep) {
+      float v[32];
+      fetch32(u * 32, v);
+      const int col = n_t * BN + u * 32;
+      if (row_ok && col < p.N) epi_store32<EPI>(p, row, col, v);
+    }
+  }
+}
+template <int BN, int EPI>
+QOS_DEV int epi_num_units(const GemmArgs& p) {
+  return EPI == EPI_QKV_ROPE ? BN / p.hd : EPI == EPI_SILU_GATE ? BN / 64 : BN / 32;
 }
 
 QOS_DEV void tmem_ld32(uint32_t taddr, float (&v)[32]) {
@@ -232,12 +266,45 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     kb0 = sp * kblocks / ks;
     kb1 = (sp + 1) * kblocks / ks;
   };
+  // stream-K ranges: CTA c owns linear iterations [rstart(c), rstart(c+1)) of t * kblocks + kb
+  const int64_t skW = p.work, skG = gridDim.x;
+  auto rstart = [&](int64_t c) { return c * skW / skG; };
+  auto cta_of = [&](int64_t idx) { return int(((idx + 1) * skG - 1) / skW); };
+  const int64_t s0 = p.sk ? rstart(blockIdx.x) : 0, e0 = p.sk ? rstart(blockIdx.x + 1) : 0;
 
   if (warp == 0) {
     // ------------------------------------------------------------ TMA producer
     if (elect_one()) {
       const uint64_t pol_a = l2_evict_last();   // activations: re-read by every N tile
       const uint64_t pol_b = l2_evict_first();  // weights: streamed once per M-tile group
+      if (p.sk) {
+        const int n = int(e0 - s0);
+        const int npre = min(S, n);
+        for (int i = 0; i < npre; ++i) {  // PDL: weights before the wait
+          const int64_t idx = s0 + i;
+          const int t = int(idx / kblocks), kb = int(idx - int64_t(t) * kblocks);
+          mbar_arrive_expect_tx(&full[i], Cfg::kStageBytes);
+          tma_load_2d_hint(smem + i * Cfg::kStageBytes + Cfg::kABytes, &tmB, &full[i], kb * kBK, (t / p.mt) * BN, pol_b);
+        }
+        griddep_wait();
+        for (int i = 0; i < npre; ++i) {
+          const int64_t idx = s0 + i;
+          const int t = int(idx / kblocks), kb = int(idx - int64_t(t) * kblocks);
+          tma_load_2d_hint(smem + i * Cfg::kStageBytes, &tmA, &full[i], kb * kBK, p.a_row0 + (t % p.mt) * kBM, pol_a);
+        }
+        int stage = npre % S;
+        uint32_t phase = (npre == S) ? 1u : 0u;
+        for (int i = npre; i < n; ++i) {
+          const int64_t idx = s0 + i;
+          const int t = int(idx / kblocks), kb = int(idx - int64_t(t) * kblocks);
+          mbar_wait(&empty[stage], phase ^ 1);
+          uint8_t* sa = smem + stage * Cfg::kStageBytes;
+          mbar_arrive_expect_tx(&full[stage], Cfg::kStageBytes);
+          tma_load_2d_hint(sa, &tmA, &full[stage], kb * kBK, p.a_row0 + (t % p.mt) * kBM, pol_a);
+          tma_load_2d_hint(sa + Cfg::kABytes, &tmB, &full[stage], kb * kBK, (t / p.mt) * BN, pol_b);
+          if (++stage == S) { stage = 0; phase ^= 1; }
+        }
+      } else {
       int stage = 0;
       uint32_t phase = 0;
       // Programmatic dependent launch: the weight (B) tiles of the first stages do not depend on
@@ -276,6 +343,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
           if (++stage == S) { stage = 0; phase ^= 1; }
         }
       }
+      }
     }
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer
@@ -285,9 +353,22 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
       uint32_t phase = 0;
       int acc = 0;
       uint32_t acc_phase = 0;
-      for (int u = blockIdx.x; u < num_units; u += gridDim.x) {
-        int m_t, n_t, sp, kb0, kb1;
-        decode_unit(u, m_t, n_t, sp, kb0, kb1);
+      int u = blockIdx.x;
+      int64_t idx = s0;
+      for (;;) {
+        int kb0, kb1;
+        if (p.sk) {  // next stream-K segment
+          if (idx >= e0) break;
+          const int t = int(idx / kblocks);
+          kb0 = int(idx - int64_t(t) * kblocks);
+          kb1 = int(min(int64_t(kblocks), int64_t(kb0) + (e0 - idx)));
+          idx += kb1 - kb0;
+        } else {
+          if (u >= num_units) break;
+          int m_t, n_t, sp;
+          decode_unit(u, m_t, n_t, sp, kb0, kb1);
+          u += gridDim.x;
+        }
         mbar_wait(&tempty[acc], acc_phase ^ 1);
         tc_fence_after();
         const uint32_t d_tmem = tmem_base + acc * BN;
@@ -314,15 +395,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     const int rit = q * 32 + lane;  // row inside the tile
     int acc = 0;
     uint32_t acc_phase = 0;
-    for (int u = blockIdx.x; u < num_units; u += gridDim.x) {
-      int m_t, n_t, sp, kb0, kb1;
-      decode_unit(u, m_t, n_t, sp, kb0, kb1);
-      mbar_wait(&tfull[acc], acc_phase);
-      tc_fence_after();
-      const int row = m_t * kBM + rit;
-      const bool row_ok = row < p.M;
-      const uint32_t tbase = tmem_base + (uint32_t(q * 32) << 16) + acc * BN;
-      if (ks == 1) {
+    auto epi_tmem = [&](int n_t, int row, bool row_ok, uint32_t tbase) {
         if constexpr (EPI == EPI_QKV_ROPE) {
           epi_qkv_rope<BN>(p, row, row_ok, n_t, [&](int col, float (&v)[16]) {
             uint32_t r[16];
@@ -378,6 +451,130 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
             if (row_ok && col < p.N) epi_store32<EPI>(p, row, col, v);
           }
         }
+    };
+    if (p.sk) {
+      // stream-K: whole tiles straight from TMEM; a tile cut by a range boundary parks one fp32
+      // partial per CTA (slot 2c for a CTA's first segment, 2c+1 for its last)
+      const int bid = blockIdx.x;
+      int pend[2], npend = 0;
+      auto slot_of = [&](int t, int cc) { return rstart(cc) >= int64_t(t) * kblocks ? 2 * cc : 2 * cc + 1; };
+      auto red32 = [&](int t, int cf, int cl) {
+        return [=](int col, float (&v)[32]) {
+#pragma unroll
+          for (int i = 0; i < 32; ++i) v[i] = 0.f;
+          for (int cc = cf; cc <= cl; ++cc) {  // CTA order: deterministic
+            const float4* pr = reinterpret_cast<const float4*>(p.part + (size_t(slot_of(t, cc)) * kBM + rit) * BN + col);
+            float4 x[8];
+#pragma unroll
+            for (int i = 0; i < 8; ++i) x[i] = __ldcg(pr + i);
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+              v[4 * i] += x[i].x;
+              v[4 * i + 1] += x[i].y;
+              v[4 * i + 2] += x[i].z;
+              v[4 * i + 3] += x[i].w;
+            }
+          }
+        };
+      };
+      auto red16 = [&](int t, int cf, int cl, int n_t) {
+        return [=](int col, float (&v)[16]) {
+#pragma unroll
+          for (int i = 0; i < 16; ++i) v[i] = p.bias ? __ldg(p.bias + n_t * BN + col + i) : 0.f;
+          for (int cc = cf; cc <= cl; ++cc) {
+            const float4* pr = reinterpret_cast<const float4*>(p.part + (size_t(slot_of(t, cc)) * kBM + rit) * BN + col);
+            float4 x[4];
+#pragma unroll
+            for (int i = 0; i < 4; ++i) x[i] = __ldcg(pr + i);
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+              v[4 * i] += x[i].x;
+              v[4 * i + 1] += x[i].y;
+              v[4 * i + 2] += x[i].z;
+              v[4 * i + 3] += x[i].w;
+            }
+          }
+        };
+      };
+      for (int64_t idx = s0; idx < e0;) {
+        const int t = int(idx / kblocks), kb0 = int(idx - int64_t(t) * kblocks);
+        const int kb1 = int(min(int64_t(kblocks), int64_t(kb0) + (e0 - idx)));
+        const int m_t = t % p.mt, n_t = t / p.mt;
+        mbar_wait(&tfull[acc], acc_phase);
+        tc_fence_after();
+        const int row = m_t * kBM + rit;
+        const bool row_ok = row < p.M;
+        const uint32_t tbase = tmem_base + (uint32_t(q * 32) << 16) + acc * BN;
+        if (kb0 == 0 && kb1 == kblocks) {
+          epi_tmem(n_t, row, row_ok, tbase);
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&tempty[acc]);
+        } else {
+          float* mine = p.part + (size_t(idx == s0 ? 2 * bid : 2 * bid + 1) * kBM + rit) * BN;
+#pragma unroll 1
+          for (int c = 0; c < BN / 32; ++c) {
+            float v[32];
+            tmem_ld32(tbase + c * 32, v);
+            if (row_ok) {
+#pragma unroll
+              for (int i = 0; i < 8; ++i)
+                __stcg(reinterpret_cast<float4*>(mine + c * 32) + i,
+                       make_float4(v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]));
+            }
+          }
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&tempty[acc]);
+          __threadfence();
+          epi_bar_sync();
+          const int cf = cta_of(int64_t(t) * kblocks), cl = cta_of(int64_t(t + 1) * kblocks - 1);
+          if (p.coop) {
+            if (threadIdx.x == 64) atomicAdd(p.counters + t, 1);
+            pend[npend++] = t;
+          } else {
+            if (threadIdx.x == 64) *s_last = (atomicAdd(p.counters + t, 1) == cl - cf);
+            epi_bar_sync();
+            if (*s_last) {
+              __threadfence();
+              epi_units<BN, EPI>(p, row, row_ok, n_t, 0, 1, red32(t, cf, cl), red16(t, cf, cl, n_t));
+              if (threadIdx.x == 64) p.counters[t] = 0;
+            }
+          }
+        }
+        if (++acc == 2) { acc = 0; acc_phase ^= 1; }
+        idx += kb1 - kb0;
+      }
+      // cooperative reduction of the cut tiles (all CTAs are co-resident: one per SM)
+      for (int i = 0; i < npend; ++i) {
+        const int t = pend[i];
+        const int m_t = t % p.mt, n_t = t / p.mt;
+        const int row = m_t * kBM + rit;
+        const bool row_ok = row < p.M;
+        const int cf = cta_of(int64_t(t) * kblocks), cl = cta_of(int64_t(t + 1) * kblocks - 1);
+        const int n = cl - cf + 1;
+        if (threadIdx.x == 64) {
+          int v;
+          do {
+            asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p.counters + t) : "memory");
+          } while (v < n);
+        }
+        epi_bar_sync();
+        epi_units<BN, EPI>(p, row, row_ok, n_t, bid - cf, n, red32(t, cf, cl), red16(t, cf, cl, n_t));
+        epi_bar_sync();
+        if (threadIdx.x == 64 && atomicAdd(p.counters + t, 1) == 2 * n - 1) p.counters[t] = 0;
+      }
+    } else
+    for (int u = blockIdx.x; u < num_units; u += gridDim.x) {
+      int m_t, n_t, sp, kb0, kb1;
+      decode_unit(u, m_t, n_t, sp, kb0, kb1);
+      mbar_wait(&tfull[acc], acc_phase);
+      tc_fence_after();
+      const int row = m_t * kBM + rit;
+      const bool row_ok = row < p.M;
+      const uint32_t tbase = tmem_base + (uint32_t(q * 32) << 16) + acc * BN;
+      if (ks == 1) {
+        epi_tmem(n_t, row, row_ok, tbase);
         tc_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(&tempty[acc]);
@@ -547,7 +744,7 @@ int gemm_pick_ksplit(int64_t M, int64_t N, int64_t K, int bn, int num_sms, int64
 
 int gemm_run(const CUtensorMap& ta, const CUtensorMap& tb, int bn, int64_t M, int64_t N, int64_t K, int epi, void* C,
              int64_t ldc, const float* bias, int num_sms, cudaStream_t st, int ksplit, float* part, int* counters,
-             int a_row0, int max_ctas, const QkvRopeArgs* rope) {
+             int a_row0, int max_ctas, const QkvRopeArgs* rope, int sk_mode, bool coop) {
   GemmArgs a;
   a.M = int(M);
   a.N = int(N);
@@ -575,6 +772,21 @@ int gemm_run(const CUtensorMap& ta, const CUtensorMap& tb, int bn, int64_t M, in
   const int tiles = a.mt * a.nt * a.ksplit;
   int grid = tiles < num_sms ? tiles : num_sms;
   if (max_ctas > 0 && grid > max_ctas) grid = max_ctas;   // SM budget (co-scheduled streams)
+  // Stream-K when whole-tile waves would leave SMs idle in the last wave (e.g. 272 tiles on
+  // 148 SMs: 92%): every CTA gets tiles * kblocks / grid k-blocks; cut tiles are reduced from
+  // fp32 partials (2 slots of 128 x BN per CTA in `part`, one counter per tile).
+  a.sk = 0;
+  a.coop = coop ? 1 : 0;
+  a.work = int64_t(a.mt) * a.nt * (K / kBK);
+  if (a.ksplit == 1 && sk_mode > 0 && part && counters && tiles <= 4096 && 2 * grid <= 512 && a.work >= grid) {
+    const int waves = (tiles + grid - 1) / grid;
+    if (sk_mode == 2 || (tiles > grid && double(tiles) < 0.95 * double(waves) * grid)) a.sk = 1;
+    if (sk_mode == 2) {  // forced (tests): as many CTAs as give >= 4 k-blocks each
+      int64_t g = a.work / 4;
+      const int cap = max_ctas > 0 ? min(max_ctas, num_sms) : num_sms;
+      grid = int(g < 1 ? 1 : g > cap ? cap : g);
+    }
+  }
   cudaError_t e = cudaSuccess;
 #define QOS_GEMM_CASE(BNV, EPIV) \
   if (bn == BNV && epi == EPIV) e = launch_gemm_t<BNV, EPIV>(ta, tb, a, grid, st); else

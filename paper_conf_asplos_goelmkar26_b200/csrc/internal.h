@@ -43,7 +43,10 @@ int gemm_pick_ksplit(int64_t M, int64_t N, int64_t K, int bn, int num_sms, int64
 // counters (zero-initialised; each reducing CTA resets its own) — deterministic reduction order
 int gemm_run(const CUtensorMap& ta, const CUtensorMap& tb, int bn, int64_t M, int64_t N, int64_t K, int epi, void* C,
              int64_t ldc, const float* bias, int num_sms, cudaStream_t st, int ksplit = 1, float* part = nullptr,
-             int* counters = nullptr, int a_row0 = 0, int max_ctas = 0, const QkvRopeArgs* rope = nullptr);
+             int* counters = nullptr, int a_row0 = 0, int max_ctas = 0, const QkvRopeArgs* rope = nullptr,
+             int sk_mode = 1, bool coop = true);
+// sk_mode: 0 no stream-K, 1 automatic (last-wave quantisation), 2 always (needs part/counters:
+// part >= 512 x 128 x 256 fp32, counters >= 4096); coop as in gemm_swab_run.
 
 // ------------------------------------------------------------------ small-T GEMM (gemm_swab.cu)
 // Swap-AB weight-streaming GEMM: tw = weight map (box 128 x 64), tt = token map (box bnt x 64).

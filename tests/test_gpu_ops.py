@@ -307,3 +307,46 @@ def test_gemm_swab_parity(torch_cuda, M, N, K, epi):
         tol = 1e-5 if epi in ("store_f32", "add_f32") else 8e-3
         assert row_rel_err(outs[-1], ref) <= tol
     assert np.array_equal(outs[0], outs[1])
+
+
+@pytest.mark.parametrize("M,N,K", [(1, 256, 1024), (300, 512, 640), (2176, 1536, 1024), (777, 1280, 2048)])
+@pytest.mark.parametrize("epi", ["store_f32", "store_bf16", "add_f32", "bias_bf16", "silu_gate"])
+def test_gemm_streamk_parity(torch_cuda, M, N, K, epi):
+    """Tile kernel in stream-K mode (ksplit = -2): tiles cut across CTAs, cooperative
+    fixed-order reduction; run twice (counter reset) and bit-identical."""
+    torch = torch_cuda
+    from oracle.model import silu
+    from paper_conf_asplos_goelmkar26_b200 import qoserve as q
+    rng = np.random.default_rng(M * 5 + N + K)
+    A = bits_to_f64(bf16_bits(rng.uniform(-1, 1, (M, K))))
+    B = bits_to_f64(bf16_bits(rng.uniform(-1, 1, (N, K)) / np.sqrt(K)))
+    dA, dB = _dev_bf16(torch, A), _dev_bf16(torch, B)
+    ref = A @ B.T
+    bias = None
+    init = None
+    if epi == "silu_gate":
+        g = np.concatenate([ref[:, 128 * j:128 * j + 64] for j in range(N // 128)], axis=1)
+        u = np.concatenate([ref[:, 128 * j + 64:128 * j + 128] for j in range(N // 128)], axis=1)
+        ref = silu(g) * u
+        dC = torch.empty((M, N // 2), dtype=torch.bfloat16, device="cuda")
+    elif epi in ("store_f32", "add_f32"):
+        init = rng.uniform(-1, 1, (M, N)).astype(np.float32) if epi == "add_f32" else np.zeros((M, N), np.float32)
+        dC = torch.from_numpy(init.copy()).cuda()
+        ref = ref + init.astype(np.float64)
+    else:
+        dC = torch.empty((M, N), dtype=torch.bfloat16, device="cuda")
+        if epi == "bias_bf16":
+            bvals = bits_to_f64(bf16_bits(rng.uniform(-0.02, 0.02, N)))
+            bias = torch.from_numpy(bvals.astype(np.float32)).cuda()
+            ref = ref + bvals
+    outs = []
+    for _ in range(2):
+        if init is not None:
+            dC.copy_(torch.from_numpy(init.copy()).cuda())
+        q.qos_op_gemm_ex(dA.data_ptr(), dB.data_ptr(), dC.data_ptr(), M, N, K, epi,
+                         bias.data_ptr() if bias is not None else None, -2)
+        torch.cuda.synchronize()
+        outs.append(dC.float().cpu().numpy())
+        tol = 1e-5 if epi in ("store_f32", "add_f32") else 8e-3
+        assert row_rel_err(outs[-1], ref) <= tol
+    assert np.array_equal(outs[0], outs[1])
