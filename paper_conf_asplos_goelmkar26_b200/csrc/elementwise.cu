@@ -26,9 +26,46 @@ QOS_DEV float block_sum(float v, float* red) {
   return s;
 }
 
-// d is a multiple of 8; each thread handles 8 contiguous elements per iteration.  Two passes
-// over the row: sum of squares, then scale (the second read hits L1).
+// d is a multiple of 8; each thread handles 8 contiguous elements per chunk.  Rows up to
+// kRowThreads * 8 * kMaxChunks elements (8192 at 256 threads: Llama-3-70B) are held in
+// registers: one HBM read of the row, all loads issued before the reduction.
+constexpr int kMaxChunks = 4;
 QOS_DEV void norm_row(const float* x, const __nv_bfloat16* g, __nv_bfloat16* out, int d, float eps, float* red) {
+  if (d <= int(blockDim.x) * 8 * kMaxChunks) {
+    float4 a[kMaxChunks], b[kMaxChunks];
+    float ss = 0.f;
+#pragma unroll
+    for (int k = 0; k < kMaxChunks; ++k) {
+      const int c = (threadIdx.x + k * blockDim.x) * 8;
+      if (c < d) {
+        a[k] = __ldcs(reinterpret_cast<const float4*>(x + c));
+        b[k] = __ldcs(reinterpret_cast<const float4*>(x + c + 4));
+      } else {
+        a[k] = b[k] = make_float4(0.f, 0.f, 0.f, 0.f);
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < kMaxChunks; ++k)
+      ss += a[k].x * a[k].x + a[k].y * a[k].y + a[k].z * a[k].z + a[k].w * a[k].w + b[k].x * b[k].x +
+            b[k].y * b[k].y + b[k].z * b[k].z + b[k].w * b[k].w;
+    const float inv = rsqrtf(block_sum(ss, red) / float(d) + eps);
+#pragma unroll
+    for (int k = 0; k < kMaxChunks; ++k) {
+      const int c = (threadIdx.x + k * blockDim.x) * 8;
+      if (c < d) {
+        const float v[8] = {a[k].x, a[k].y, a[k].z, a[k].w, b[k].x, b[k].y, b[k].z, b[k].w};
+        const uint4 gw = __ldg(reinterpret_cast<const uint4*>(g + c));
+        const uint32_t gg[4] = {gw.x, gw.y, gw.z, gw.w};
+        uint32_t pk[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+          pk[i] = pack_bf16(v[2 * i] * inv * bf16_lo(gg[i]), v[2 * i + 1] * inv * bf16_hi(gg[i]));
+        *reinterpret_cast<uint4*>(out + c) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+      }
+    }
+    return;
+  }
+  // longer rows: two passes (the second read hits L1/L2)
   float ss = 0.f;
   for (int c = threadIdx.x * 8; c < d; c += blockDim.x * 8) {
     const float4 a = *reinterpret_cast<const float4*>(x + c);
