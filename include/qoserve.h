@@ -139,7 +139,7 @@ int qos_kv_cached_len(qos_engine_t* eng, int64_t req, int32_t* out);
 int qos_kv_free_blocks(qos_engine_t* eng, int64_t* out);
 /* Fill positions [0, n_tokens) of req, every layer, with synthetic K/V (DESIGN.md §3:
  * name "kvfill.{layer}.{k|v}.{req}", i = (pos*Hkv + h)*hd + j over GLOBAL kv heads, value
- * bf16_rne(a)) and set its cached length to n_tokens.  Used by benches / profiling where
+ * bf16_rne(a) for K, fp16_rne(a) for V) and set its cached length to n_tokens.  Used by benches / profiling where
  * a decode's prefix need not come from a prefill.  Synchronous. */
 int qos_kv_fill_synthetic(qos_engine_t* eng, int64_t req, int32_t n_tokens, uint64_t seed);
 

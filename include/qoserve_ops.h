@@ -57,13 +57,14 @@ int qos_op_gemm_ex(const void* A, const void* B, void* C, int64_t M, int64_t N, 
 int qos_op_rmsnorm(const float* x, const void* g, void* out, int32_t T, int32_t d, float eps,
                    void* stream);
 
-/* Write / read cached K and V of `req` at `layer`, positions [pos0, pos0+n), as host bf16 bits
- * [n][Hkv_local][hd] (Hkv_local = this rank's kv heads).  The blocks must be allocated.
- * qos_kv_write does not change the cached length.  Synchronous. */
+/* Write / read cached K and V of `req` at `layer`, positions [pos0, pos0+n), as host 16-bit
+ * patterns [n][Hkv_local][hd] (Hkv_local = this rank's kv heads): K in bf16, V in IEEE fp16
+ * (the cache keeps V in fp16 so P.V runs as one fp16 MMA; reading r-v16).  The
+ * blocks must be allocated.  qos_kv_write does not change the cached length.  Synchronous. */
 int qos_kv_write(qos_engine_t* eng, int32_t layer, int64_t req, int32_t pos0, int32_t n,
-                 const uint16_t* k_bf16, const uint16_t* v_bf16);
+                 const uint16_t* k_bf16, const uint16_t* v_f16);
 int qos_kv_read(qos_engine_t* eng, int32_t layer, int64_t req, int32_t pos0, int32_t n,
-                uint16_t* k_bf16, uint16_t* v_bf16);
+                uint16_t* k_bf16, uint16_t* v_f16);
 
 /* a4 + a5 + a6 (fused): the layer's QKV projection of normalised activations h (host bf16
  * [T][d], T = token rows of `batch`, chunks then decodes) with RoPE on q and k at each row's

@@ -11,7 +11,8 @@ network here, so both sides draw the SAME bf16 bits from a counter-based generat
     embed   w = bf16_rne( a )
     norm    w = bf16_rne( fp32( 1 + fp32(0.1 * a) ) )
     bias    w = bf16_rne( fp32( 0.02 * a ) )
-    kvfill  w = bf16_rne( a )      name "kvfill.{layer}.{k|v}.{req}", i = (pos*Hkv + h)*hd + j
+    kvfill  K: w = bf16_rne( a ),  V: w = fp16_rne( a )   (reading r-v16: the cache
+            holds V in fp16)   name "kvfill.{layer}.{k|v}.{req}", i = (pos*Hkv + h)*hd + j
 
 This module is an independent numpy implementation of that spec.  The CUDA library has its
 own implementation (device kernel); the two are compared bit-for-bit on the generated bf16
@@ -59,6 +60,16 @@ def bf16_rne_bits(x32: np.ndarray) -> np.ndarray:
     return (u >> np.uint64(16)).astype(np.uint16)
 
 
+def f16_rne_bits(x32: np.ndarray) -> np.ndarray:
+    """Round fp32 values to IEEE fp16 (round-to-nearest-even, numpy's conversion); uint16 bits."""
+    return np.ascontiguousarray(x32, dtype=np.float32).astype(np.float16).view(np.uint16)
+
+
+def f16_bits_to_f64(bits: np.ndarray) -> np.ndarray:
+    """Exact widening of fp16 bit patterns to fp64."""
+    return np.ascontiguousarray(bits, dtype=np.uint16).view(np.float16).astype(np.float64)
+
+
 def bf16_bits_to_f64(bits: np.ndarray) -> np.ndarray:
     """Exact widening of bf16 bit patterns to fp64."""
     return (bits.astype(np.uint32) << np.uint32(16)).view(np.float32).astype(np.float64)
@@ -80,8 +91,11 @@ def _a_values(seed: int, name: str, start: int, count: int) -> np.ndarray:
 
 
 def gen_bits(seed: int, name: str, kind: str, start: int, count: int, fan_in: int = 1) -> np.ndarray:
-    """bf16 bit patterns of elements [start, start+count) of tensor ``name``."""
+    """bf16 bit patterns of elements [start, start+count) of tensor ``name`` (fp16 bit patterns
+    for kind "kvfill_v", the synthetic cached V)."""
     a = _a_values(seed, name, start, count)
+    if kind == "kvfill_v":
+        return f16_rne_bits(a)
     if kind == "linear":
         s = np.float32(1.0 / np.sqrt(np.float64(fan_in)))
         w = a * s                                   # fp32 multiply, RNE
@@ -112,8 +126,12 @@ def gen_tensor(seed: int, name: str, kind: str, shape, fan_in: int = 1,
 def kvfill_rows(seed: int, layer: int, which: str, req: int, pos0: int, pos1: int,
                 n_kv_heads: int, head_dim: int) -> np.ndarray:
     """Synthetic cached K or V of request ``req`` for positions [pos0, pos1) at ``layer``:
-    fp64 array [pos1-pos0, n_kv_heads, head_dim] of bf16-exact values."""
+    fp64 array [pos1-pos0, n_kv_heads, head_dim] of bf16-exact K / fp16-exact V values
+    (reading r-v16)."""
     name = f"kvfill.{layer}.{which}.{req}"
     per_pos = n_kv_heads * head_dim
+    if which == "v":
+        bits = gen_bits(seed, name, "kvfill_v", pos0 * per_pos, (pos1 - pos0) * per_pos)
+        return f16_bits_to_f64(bits).reshape(pos1 - pos0, n_kv_heads, head_dim)
     bits = gen_bits(seed, name, "kvfill", pos0 * per_pos, (pos1 - pos0) * per_pos)
     return bf16_bits_to_f64(bits).reshape(pos1 - pos0, n_kv_heads, head_dim)

@@ -5,7 +5,8 @@
 // the whole pool (dims {hd, blocks*Hkv*16, L*2}, box {64, 16, 1}, 128-B swizzle), so every
 // (block, head) tile lands bank-conflict-free for ldmatrix.  A producer warp keeps a ring of
 // 8 block-stages in flight (full/empty mbarriers); consumer warps run flash-attention style
-// online softmax (fp32, exp2) with m16n8k16 bf16 tensor-core MMAs.
+// online softmax (fp32, exp2) with m16n8k16 tensor-core MMAs (Q K^T in bf16; P V in fp16:
+// V is cached in fp16, P rounded to fp16).
 //
 //  * decode (a8): split-K.  Work item = (decode row, kv head, key range).  The MMAs are
 //    transposed so the 16 keys of a paged block are the M rows and the GQA group (<= 8 query
@@ -87,18 +88,17 @@ QOS_DEV void qk_block_t(const uint32_t (&qb)[HD / 16][2], uint32_t ktile, int la
   }
 }
 
-// O^T[HD][8] += V^T[HD][16 keys] · P^T[16 keys][8]   (A = V^T via ldmatrix.trans, B = P^T)
+// O^T[HD][8] += V^T[HD][16 keys] · P^T[16 keys][8]   (A = V^T via ldmatrix.trans, B = P^T;
+// fp16 operands: V is cached in fp16 and P is rounded to fp16, 2^-11 relative)
 template <int HD>
-QOS_DEV void pv_block_t(uint32_t b0, uint32_t b1, uint32_t l0, uint32_t l1, uint32_t vtile, int lane,
-                        float (&o)[HD / 16][4]) {
+QOS_DEV void pv_block_t(uint32_t b0, uint32_t b1, uint32_t vtile, int lane, float (&o)[HD / 16][4]) {
   const int kr = (lane & 7) + (lane >> 4) * 8;
   const int csel = (lane >> 3) & 1;
 #pragma unroll
   for (int md = 0; md < HD / 16; ++md) {
     uint32_t a[4];
     ldmatrix_x4_trans(vtile + tile_off(kr, 2 * md + csel), a[0], a[1], a[2], a[3]);
-    mma_bf16_16816(o[md], a, b0, b1);   // P_hi
-    mma_bf16_16816(o[md], a, l0, l1);   // P_lo
+    mma_f16_16816(o[md], a, b0, b1);
   }
 }
 
@@ -193,12 +193,8 @@ __global__ void __launch_bounds__(kAttnThreads, 3)
         o[md][2] *= a0;
         o[md][3] *= a1;
       }
-      // P^T as B fragments: transpose the two 8x8 (keys x heads) halves; P = P_hi + P_lo
-      const uint32_t h0 = pack_bf16(p0, p1), h1 = pack_bf16(p2, p3);
-      const uint32_t lo0 = pack_bf16(p0 - bf16_lo(h0), p1 - bf16_hi(h0));
-      const uint32_t lo1 = pack_bf16(p2 - bf16_lo(h1), p3 - bf16_hi(h1));
-      pv_block_t<HD>(movmatrix_trans(h0), movmatrix_trans(h1), movmatrix_trans(lo0), movmatrix_trans(lo1),
-                     kt + C::kBlockBytes, lane, o);
+      // P^T as B fragments: transpose the two 8x8 (keys x heads) halves of fp16 P
+      pv_block_t<HD>(movmatrix_trans(pack_f16(p0, p1)), movmatrix_trans(pack_f16(p2, p3)), kt + C::kBlockBytes, lane, o);
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[s]);
     }

@@ -9,7 +9,8 @@
 //   warp 1      MMA issuer (one lane): S_j = Q K_j^T  (UMMA 128x128x16, A,B from smem) into
 //               TMEM;  O += P_j V_j  (UMMA 128xHDx16, A = P from TMEM, B = V MN-major)
 //   warps 2..5  softmax, one TMEM lane (= one row) per thread: masked fp32 online softmax with
-//               exp2, P written back over S in TMEM as two bf16 terms; O is rescaled in TMEM
+//               exp2, P written back over S in TMEM in fp16 (V is cached in fp16, so P.V is
+//               one kind::f16 MMA with f16 operands); O is rescaled in TMEM
 //               only when the running max grows by more than 2^8 (P <= 2^8 otherwise);
 //               epilogue O / l -> global.
 // Two CTAs share an SM (96 KB smem, 256 TMEM columns each) so one CTA's softmax overlaps the
@@ -19,6 +20,10 @@
 
 #include "common.cuh"
 #include "internal.h"
+
+#ifndef QOS_FA_LAZY
+#define QOS_FA_LAZY 8.f   // rescale O only when the running max grows by more than this (log2)
+#endif
 
 namespace qos {
 
@@ -55,6 +60,12 @@ QOS_DEV float ex2(float x) {  // MUFU.EX2 (flush-to-zero; arguments are <= 8 her
   return y;
 }
 
+QOS_DEV float fmax3(float a, float b, float c) {  // FMNMX3
+  float d;
+  asm("max.f32 %0, %1, %2, %3;" : "=f"(d) : "f"(a), "f"(b), "f"(c));
+  return d;
+}
+
 // packed fp32 pair arithmetic (sm_100: FFMA2 / FADD2)
 QOS_DEV float2 fma2(float2 a, float2 b, float2 c) {
   float2 d;
@@ -75,7 +86,7 @@ QOS_DEV float2 add2(float2 a, float2 b) {
   return d;
 }
 
-// D[tmem] (+)= A[tmem] · B[smem desc]   (kind::f16, A = bf16 pairs packed in 32-bit columns)
+// D[tmem] (+)= A[tmem] · B[smem desc]   (kind::f16, A = 16-bit pairs packed in 32-bit columns)
 QOS_DEV void umma_bf16_ts(uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc, uint32_t idesc, uint32_t accumulate) {
   asm volatile(
       "{\n\t.reg .pred p;\n\t"
@@ -210,7 +221,8 @@ __global__ void __launch_bounds__(kFaThreads, 2)
     // ------------------------------------------------------------------ MMA issuer
     if (elect_one()) {
       constexpr uint32_t idesc_qk = umma_idesc_bf16(128, C::kKeys);
-      constexpr uint32_t idesc_pv = umma_idesc_bf16(128, HD) | (1u << 16);  // B (V) MN-major
+      // P.V in fp16 (A = P in TMEM, B = V cached in fp16, MN-major): formats a/b = f16 (0)
+      constexpr uint32_t idesc_pv = (1u << 4) | (1u << 16) | ((uint32_t(HD) >> 3) << 17) | ((128u >> 4) << 24);
       const uint32_t q_base = smem_u32(sQ);
       auto issue_pv = [&](int t) {
         const int s = t & 1;
@@ -224,8 +236,7 @@ __global__ void __launch_bounds__(kFaThreads, 2)
         for (int kk = 0; kk < C::kKeys / 16; ++kk) {
           const uint64_t vd = umma_desc_sw128_mn(v_base + kk * 2048, C::kKeys * 128);
           const uint32_t pc = p_tmem + (kk >> 1) * 32 + (kk & 1) * 8;
-          umma_bf16_ts(tmem + C::kColO, pc, vd, idesc_pv, (t | kk) != 0);  // P_hi
-          umma_bf16_ts(tmem + C::kColO, pc + 16, vd, idesc_pv, 1);         // P_lo
+          umma_bf16_ts(tmem + C::kColO, pc, vd, idesc_pv, (t | kk) != 0);
         }
         umma_commit(o_full);
         umma_commit(&v_empty[s]);
@@ -274,29 +285,35 @@ __global__ void __launch_bounds__(kFaThreads, 2)
         tmem_ld32x32b_x16(s_addr + c * 16, *reinterpret_cast<uint32_t(*)[16]>(&r[c * 16]));
       tmem_ld_wait();
       // row max of the raw scores (scaled afterwards; the scale is positive)
-      float mx = -INFINITY;
+      // (four independent 3-input max chains: a short dependency chain)
+      float mq[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
       if (masked) {
 #pragma unroll
-        for (int i = 0; i < C::kKeys; ++i)
-          if (key0 + i <= pos_r) mx = fmaxf(mx, __uint_as_float(r[i]));
+        for (int i = 0; i < C::kKeys; i += 2) {
+          const float a = key0 + i <= pos_r ? __uint_as_float(r[i]) : -INFINITY;
+          const float b = key0 + i + 1 <= pos_r ? __uint_as_float(r[i + 1]) : -INFINITY;
+          mq[(i >> 1) & 3] = fmax3(mq[(i >> 1) & 3], a, b);
+        }
       } else {
 #pragma unroll
-        for (int i = 0; i < C::kKeys; ++i) mx = fmaxf(mx, __uint_as_float(r[i]));
+        for (int i = 0; i < C::kKeys; i += 2)
+          mq[(i >> 1) & 3] = fmax3(mq[(i >> 1) & 3], __uint_as_float(r[i]), __uint_as_float(r[i + 1]));
       }
+      float mx = fmax3(mq[0], mq[1], fmaxf(mq[2], mq[3]));
       mx *= p.scale_log2;
       // lazy rescale: keep the previous max unless the new one exceeds it by > 8 (P <= 2^8)
-      const bool rescale = mx > m_used + 8.f;
+      const bool rescale = mx > m_used + QOS_FA_LAZY;
       const float m_new = rescale ? mx : m_used;
       const float alpha = (rescale && m_used != -INFINITY) ? ex2(m_used - m_new) : 1.f;
       const float mb = (m_new == -INFINITY) ? 0.f : m_new;
-      // pass 2: P = 2^(s*scale - m) and the row sum; P written as two bf16 terms (P_hi + P_lo,
-      // exact to ~2^-16 so the fp32 P.V meets the 2e-3 attention bar) over the 32 S columns each
-      // chunk has just read: [32c, 32c+16) = P_hi, [32c+16, 32c+32) = P_lo of keys 32c..32c+31.
-      float2 sum2 = make_float2(0.f, 0.f);
+      // pass 2: P = 2^(s*scale - m) and the row sum; P written in fp16 (2^-11 relative, so the
+      // fp32 P.V meets the 2e-3 attention bar; bf16 P alone measured 2.3-3.6e-3) over the S
+      // columns each chunk has just read: [32c, 32c+16) hold the fp16 pairs of keys 32c..32c+31.
+      float2 sum2[4] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
       const float2 scale2 = make_float2(p.scale_log2, p.scale_log2), nmb2 = make_float2(-mb, -mb);
 #pragma unroll
       for (int c = 0; c < C::kKeys / 32; ++c) {
-        uint32_t hi[16], lo[16];
+        uint32_t hi[16];
 #pragma unroll
         for (int i = 0; i < 16; ++i) {
           // paired fp32 ops (FFMA2 / FADD2) halve the softmax's FMA-pipe instructions
@@ -308,15 +325,13 @@ __global__ void __launch_bounds__(kFaThreads, 2)
             pp.x = (k <= pos_r) ? pp.x : 0.f;
             pp.y = (k + 1 <= pos_r) ? pp.y : 0.f;
           }
-          hi[i] = pack_bf16(pp.x, pp.y);
-          const float2 rs = add2(pp, make_float2(-bf16_lo(hi[i]), -bf16_hi(hi[i])));
-          lo[i] = pack_bf16(rs.x, rs.y);
-          sum2 = add2(sum2, pp);
+          hi[i] = pack_f16(pp.x, pp.y);
+          sum2[i & 3] = add2(sum2[i & 3], pp);
         }
         tmem_st32x32b_x16(s_addr + c * 32, hi);
-        tmem_st32x32b_x16(s_addr + c * 32 + 16, lo);
       }
-      const float sum = sum2.x + sum2.y;
+      const float2 s01 = add2(sum2[0], sum2[1]), s23 = add2(sum2[2], sum2[3]);
+      const float sum = (s01.x + s23.x) + (s01.y + s23.y);
       tmem_st_wait();
       l = l * alpha + sum;
       if (j >= 1 && __any_sync(0xffffffffu, alpha != 1.f)) {

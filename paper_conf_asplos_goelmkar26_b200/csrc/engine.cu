@@ -1201,7 +1201,7 @@ int qos_kv_fill_synthetic(qos_engine_t* e, int64_t req, int32_t n_tokens, uint64
       snprintf(name, sizeof name, "kvfill.%d.%c.%lld", l, kv ? 'v' : 'k', (long long)req);
       void* plane = reinterpret_cast<__nv_bfloat16*>(e->kv) + (size_t(l) * 2 + kv) * e->plane_elems;
       QOS_CU(kvfill_launch(plane, trow, n_tokens, e->sh.Hkv, e->cfg.n_kv_heads, e->sh.kv0, e->cfg.head_dim, seed,
-                           fnv1a64(name), st));
+                           fnv1a64(name), kv, st));
     }
   QOS_CU(cudaStreamSynchronize(st));
   it->second.cached = n_tokens;

@@ -159,9 +159,9 @@ QOS_DEV void epi_qkv_rope(const GemmArgs& p, int row, bool row_ok, int n_t, Fetc
         float x[16];
         fetch(hh * hd + i0, x);
         if (row_ok) {
-          uint32_t a[8];
+          uint32_t a[8];  // V is cached in fp16 (it meets fp16 P in P.V)
 #pragma unroll
-          for (int k = 0; k < 8; ++k) a[k] = pack_bf16(x[2 * k], x[2 * k + 1]);
+          for (int k = 0; k < 8; ++k) a[k] = pack_f16(x[2 * k], x[2 * k + 1]);
           uint4* da = reinterpret_cast<uint4*>(dst + i0);
           da[0] = make_uint4(a[0], a[1], a[2], a[3]);
           da[1] = make_uint4(a[4], a[5], a[6], a[7]);

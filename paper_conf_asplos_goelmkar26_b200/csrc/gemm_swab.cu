@@ -18,6 +18,8 @@
 #include <cstdio>
 #include <cstdlib>
 
+#include <cuda_fp16.h>
+
 #include "common.cuh"
 #include "internal.h"
 
@@ -148,14 +150,18 @@ QOS_DEV void swab_epilogue(const SwabArgs& p, int wt, int tt, int f, float* xch,
           const float y = xb[j * 128 + partner];
           out = i < half ? v[j] * cs.x - y * cs.y : v[j] * cs.x + y * cs.y;
         }
-        const __nv_bfloat16 ob = __float2bfloat16_rn(out);
-        if (head < p.H) {
-          reinterpret_cast<__nv_bfloat16*>(p.C)[size_t(tok) * p.ldc + gr] = ob;
-        } else {
+        if (head < p.H + p.Hkv) {
+          const __nv_bfloat16 ob = __float2bfloat16_rn(out);
+          if (head < p.H) {
+            reinterpret_cast<__nv_bfloat16*>(p.C)[size_t(tok) * p.ldc + gr] = ob;
+          } else {
+            const int sl = __ldg(p.slot + tok);
+            p.kplane[((size_t(sl >> 4) * p.Hkv + (head - p.H)) * 16 + (sl & 15)) * hd + i] = ob;
+          }
+        } else {  // V is cached in fp16
           const int sl = __ldg(p.slot + tok);
-          const int kvh = head < p.H + p.Hkv ? head - p.H : head - p.H - p.Hkv;
-          __nv_bfloat16* plane = head < p.H + p.Hkv ? p.kplane : p.vplane;
-          plane[((size_t(sl >> 4) * p.Hkv + kvh) * 16 + (sl & 15)) * hd + i] = ob;
+          const __half oh = __float2half_rn(out);
+          reinterpret_cast<__half*>(p.vplane)[((size_t(sl >> 4) * p.Hkv + (head - p.H - p.Hkv)) * 16 + (sl & 15)) * hd + i] = oh;
         }
       }
     }

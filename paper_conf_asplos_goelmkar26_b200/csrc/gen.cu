@@ -5,6 +5,8 @@
 //   a = ((splitmix64((seed ^ fnv1a64(name)) + i) >> 40) - 2^23) / 2^23
 //   linear: bf16(fp32(a * s)), s = fp32(1/sqrt(fan_in));  embed / kvfill: bf16(a);
 //   norm: bf16(fp32(1 + fp32(0.1 a)));  bias: bf16(fp32(0.02 a))      (all fp32 ops RNE, no FMA)
+#include <cuda_fp16.h>
+
 #include "common.cuh"
 #include "internal.h"
 
@@ -59,8 +61,8 @@ __global__ void gen_bias_f32_kernel(float* __restrict__ dst, int64_t n, uint64_t
 
 // KV fill of one request for one (layer, K|V) plane: positions [0, n), local heads h <
 // hkv_local map to global head kv_head0 + h; i = (pos * hkv_global + global head) * hd + j.
-__global__ void kvfill_kernel(__nv_bfloat16* __restrict__ plane, const int32_t* __restrict__ table, int n,
-                              int hkv_local, int hkv_global, int kv_head0, int hd, uint64_t base) {
+__global__ void kvfill_kernel(uint16_t* __restrict__ plane, const int32_t* __restrict__ table, int n,
+                              int hkv_local, int hkv_global, int kv_head0, int hd, uint64_t base, int fp16) {
   const int64_t total = int64_t(n) * hkv_local * hd;
   for (int64_t e = blockIdx.x * int64_t(blockDim.x) + threadIdx.x; e < total; e += int64_t(gridDim.x) * blockDim.x) {
     const int j = int(e % hd);
@@ -68,8 +70,9 @@ __global__ void kvfill_kernel(__nv_bfloat16* __restrict__ plane, const int32_t* 
     const int pos = int(e / (int64_t(hd) * hkv_local));
     const uint64_t i = (uint64_t(pos) * hkv_global + kv_head0 + h) * hd + j;
     const int blk = table[pos >> 4];
+    const float v = gen_value(base, i, GEN_EMBED, 0.f);  // exact in fp32 (24-bit fraction)
     plane[((int64_t(blk) * hkv_local + h) * 16 + (pos & 15)) * hd + j] =
-        __float2bfloat16_rn(gen_value(base, i, GEN_EMBED, 0.f));
+        fp16 ? __half_as_ushort(__float2half_rn(v)) : __bfloat16_as_ushort(__float2bfloat16_rn(v));
   }
 }
 
@@ -100,11 +103,11 @@ cudaError_t gen_fill_f32_bias(float* dst, int64_t n, uint64_t seed, uint64_t nam
 }
 
 cudaError_t kvfill_launch(void* plane, const int32_t* d_table, int n_tokens, int hkv_local, int hkv_global,
-                          int kv_head0, int hd, uint64_t seed, uint64_t name_hash, cudaStream_t st) {
+                          int kv_head0, int hd, uint64_t seed, uint64_t name_hash, int fp16, cudaStream_t st) {
   if (n_tokens == 0) return cudaSuccess;
   count_launch();
   kvfill_kernel<<<grid_for(int64_t(n_tokens) * hkv_local * hd), 256, 0, st>>>(
-      (__nv_bfloat16*)plane, d_table, n_tokens, hkv_local, hkv_global, kv_head0, hd, seed ^ name_hash);
+      (uint16_t*)plane, d_table, n_tokens, hkv_local, hkv_global, kv_head0, hd, seed ^ name_hash, fp16);
   return cudaGetLastError();
 }
 

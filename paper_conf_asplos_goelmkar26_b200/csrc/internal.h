@@ -71,9 +71,9 @@ cudaError_t gen_fill_bf16_ex(void* dst, int64_t dst_ld, int64_t rows, int64_t co
                              int64_t row0, int64_t col0, int64_t src_cols, int kind, int fan_in, int interleave,
                              cudaStream_t st);
 cudaError_t gen_fill_f32_bias(float* dst, int64_t n, uint64_t seed, uint64_t name_hash, int64_t off, cudaStream_t st);
-// KV fill: positions [0, n) of one request, one layer, K or V plane
+// KV fill: positions [0, n) of one request, one layer, K (bf16) or V (fp16 = 1) plane
 cudaError_t kvfill_launch(void* plane, const int32_t* d_table, int n_tokens, int hkv_local, int hkv_global,
-                          int kv_head0, int hd, uint64_t seed, uint64_t name_hash, cudaStream_t st);
+                          int kv_head0, int hd, uint64_t seed, uint64_t name_hash, int fp16, cudaStream_t st);
 
 // ------------------------------------------------------------------ elementwise (elementwise.cu)
 cudaError_t launch_embed_rmsnorm(const int32_t* tokens, const void* emb, const void* g, float* resid, void* out,

@@ -28,6 +28,15 @@ def bits_to_f64(b: np.ndarray) -> np.ndarray:
     return (np.asarray(b, dtype=np.uint16).astype(np.uint32) << np.uint32(16)).view(np.float32).astype(np.float64)
 
 
+def f16_bits(x: np.ndarray) -> np.ndarray:
+    """fp64/fp32 values -> IEEE fp16 bits (RNE via fp32; the cached V format, reading r-v16)."""
+    return np.ascontiguousarray(np.asarray(x, dtype=np.float32)).astype(np.float16).view(np.uint16)
+
+
+def f16_bits_to_f64(b: np.ndarray) -> np.ndarray:
+    return np.ascontiguousarray(b, dtype=np.uint16).view(np.float16).astype(np.float64)
+
+
 def make_engine(preset_name: str, **over):
     from paper_conf_asplos_goelmkar26_b200 import qoserve as q
     from paper_conf_asplos_goelmkar26_b200.presets import preset

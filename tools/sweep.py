@@ -1,6 +1,7 @@
 """Quick device-timed sweep of hybrid-step latency (qos_profile_step) on Llama-3-8B shapes.
   python tools/sweep.py --points 256:0:0,256:128:1024,2048:128:4096  [--layers L] [--reps 5]
-Each point is chunk:n_decode:ctx (kv_start 0).  Prints one JSON line per point."""
+Each point is chunk:n_decode:ctx[:kv_start] (kv_start 0 by default: the chunk's cached prefix).
+Prints one JSON line per point."""
 import argparse
 import json
 import os
@@ -19,17 +20,18 @@ a = ap.parse_args()
 import torch  # noqa: E402
 torch.cuda.set_device(0)
 pts = [tuple(int(x) for x in p.split(":")) for p in a.points.split(",")]
-need = max(nd * (ctx + 1) for _, nd, ctx in pts) + 9000
+pts = [p if len(p) == 4 else p + (0,) for p in pts]
+need = max(nd * (ctx + 1) + ks + c for c, nd, ctx, ks in pts) + 9000
 over = {} if a.layers is None else {"n_layers": a.layers}
 cfg = q.model_cfg(**preset("llama3-8b", **over), num_blocks=need // 16 + 600, max_seq_len=16384, max_requests=300,
                   max_batch_tokens=8192 + 256, max_batch_rows=257)
 eng = q.Engine(cfg)
 eng.qos_engine_load_synthetic(0)
-for c, nd, ctx in pts:
+for c, nd, ctx, ks in pts:
     if a.breakdown:
         eng.qos_engine_set_timing(True)
-    ms, p95 = eng.qos_profile_step(c, [ctx] * nd, reps=a.reps)
-    rec = {"chunk": c, "n_decode": nd, "ctx": ctx, "ms": round(ms, 3), "p95": round(p95, 3),
+    ms, p95 = eng.qos_profile_step(c, [ctx] * nd, reps=a.reps, kv_start=ks)
+    rec = {"chunk": c, "n_decode": nd, "ctx": ctx, "kv_start": ks, "ms": round(ms, 3), "p95": round(p95, 3),
            "tok_s": round((c + nd) / ms * 1e3)}
     if a.breakdown:
         tm = eng.qos_last_step_timing()
