@@ -7,15 +7,20 @@ uses it to pick the largest chunk that keeps every decode's next-token deadline
 engine's OWN device-timed steps (`qos_profile_step`) with features that follow the step's
 work and the engine's tiling:
 
-    t(batch) = c0 * Wgemm(T) + c1 * T + c2 * Bdec + c3 * n_dec + c4 * [n_dec > 0] + c5 + c6 * Fpre
+    t(batch) = c0 * Wgemm(T) + c1 * T + c2 * Bdec + c3 * n_dec + c4 * [n_dec > 0] + c5 + c6 * Fdiag
+               + c7 * Wstream(T) + c8 * Fprefix
 
-* Wgemm(T): sum over the four projections of (waves of 128 x BN tiles over the SMs) x (k-blocks
-  per tile) x BN/256 — the tensor-core GEMM time with the engine's tile-quantisation (the
-  same BN / split-K choice as csrc/gemm.cu), T = sum(chunk_len) + n_decode;
+* Wgemm(T): sum over the projections run by the tile kernel (csrc/gemm.cu) of (waves of
+  128 x BN tiles over the SMs) x (k-blocks per tile) x BN/256 — the tensor-core GEMM time with
+  the engine's tile-quantisation (same BN / split-K choice), T = sum(chunk_len) + n_decode;
+* Wstream(T): weight elements N*K of the projections run by the weight-streaming kernel
+  (csrc/gemm_swab.cu, same selection rule as swab_prefer) — HBM-bound;
 * T: per-token elementwise work (norms, RoPE/append, embedding);
 * Bdec = sum_j (ctx_j + 1): decode-attention KV bytes (HBM-bound);
 * n_dec and [n_dec > 0]: per-decode and per-launch latency of the split-K decode attention;
-* Fpre = sum_c [len_c * kv_start_c + len_c (len_c + 1) / 2]: prefill-attention work.
+* Fdiag = sum_c len_c (len_c + 1) / 2 and Fprefix = sum_c len_c * kv_start_c: prefill-attention
+  work on the chunk's own (causal, masked diagonal tiles) and on its cached prefix (unmasked
+  tiles, measured ~1.6x more efficient per FLOP on B200) — kept apart, as their costs differ.
 
 Least squares (numpy, relative weights) over profiled points; `predict` is host arithmetic.
 The north star asks iteration latency to be predictable within 5% across chunks 256-8192.
@@ -28,7 +33,7 @@ from dataclasses import dataclass, field
 
 import numpy as np
 
-N_FEAT = 7
+N_FEAT = 9
 
 
 @dataclass
@@ -59,11 +64,25 @@ def _bn(M: int, N: int, sms: int) -> int:      # mirrors gemm_pick_bn (csrc/gemm
     return 256 if (mt * ((N + 255) // 256) >= sms and N % 256 == 0) else 128
 
 
+def swab_prefer(M: int, N: int, sms: int) -> bool:   # mirrors swab_prefer (csrc/gemm_swab.cu)
+    if N % 128:
+        return False
+    if M <= 16:
+        return True
+    if M <= 32 and N // 128 < sms:
+        return True
+    if M > 256:
+        return False
+    return ((M + 127) // 128) * (N // 128) * 4 < sms
+
+
 def gemm_work(T: int, g: GemmShapes) -> float:
     if T <= 0:
         return 0.0
     tot = 0.0
     for N, K in g.gemms:
+        if swab_prefer(T, N, g.num_sms):
+            continue
         bn = _bn(T, N, g.num_sms)
         tiles = ((T + 127) // 128) * ((N + bn - 1) // bn)
         ks = 1                                 # mirrors gemm_pick_ksplit
@@ -73,10 +92,15 @@ def gemm_work(T: int, g: GemmShapes) -> float:
     return tot
 
 
+def stream_work(T: int, g: GemmShapes) -> float:
+    return float(sum(N * K for N, K in g.gemms if T > 0 and swab_prefer(T, N, g.num_sms)))
+
+
 def features(s: StepShape, g: GemmShapes = GemmShapes()) -> np.ndarray:
     nd = len(s.ctx)
     return np.array([gemm_work(s.T, g) / 100.0, s.T / 1000.0, sum(c + 1 for c in s.ctx) / 1e6, nd / 100.0,
-                     1.0 if nd else 0.0, 1.0, sum(n * ks + n * (n + 1) / 2 for ks, n in s.chunks) / 1e7])
+                     1.0 if nd else 0.0, 1.0, sum(n * (n + 1) / 2 for ks, n in s.chunks) / 1e7,
+                     stream_work(s.T, g) / 1e8, sum(n * ks for ks, n in s.chunks) / 1e7])
 
 
 class LatencyModel:

@@ -6,15 +6,16 @@ import os
 
 import numpy as np
 
-from paper_conf_asplos_goelmkar26_b200.latency_model import GemmShapes, LatencyModel, StepShape, features, gemm_work
+from paper_conf_asplos_goelmkar26_b200.latency_model import (GemmShapes, LatencyModel, StepShape, features, gemm_work,
+                                                             stream_work)
 
 PROF = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles", "latency_table_r1.json")
 
 
 def test_recovers_known_coefficients():
     rng = np.random.default_rng(0)
-    true = np.array([2.0, 3.0, 20.0, 0.5, 1.0, 4.0, 9.0])
-    shapes = []
+    true = np.array([2.0, 3.0, 20.0, 0.5, 1.0, 4.0, 9.0, 6.0, 5.0])
+    shapes = [StepShape([], list(rng.integers(1024, 8193, nd))) for nd in (1, 8, 16, 24, 32, 64, 100, 200, 256)]
     for _ in range(120):
         c = int(rng.integers(0, 8193))
         nd = int(rng.integers(0, 257))
@@ -34,6 +35,14 @@ def test_gemm_work_is_tile_quantised():
     assert all(a <= b for a, b in zip(w, w[1:]))                   # steps, never decreasing
     assert len(set(w)) > 20
     assert gemm_work(8448, g) > 3 * gemm_work(2176, g)
+
+
+def test_small_steps_use_the_weight_streaming_gemm():
+    g = GemmShapes()
+    assert stream_work(1, g) == sum(n * k for n, k in g.gemms)        # every projection streams
+    assert stream_work(2176, g) == 0 and gemm_work(1, g) == 0
+    # T = 64: only the O and down projections (32 output tiles) take the streaming kernel
+    assert stream_work(64, g) == 4096 * 4096 + 4096 * 14336
 
 
 def test_committed_profile_predictability():

@@ -67,6 +67,11 @@ def main():
     for chunk in (256, 1024, 2048, 4096):
         for nd in (0, 128):
             grid.append((chunk, nd, 2048, 4096))
+    # small, decode-dominated steps (the weight-streaming GEMM regime the scheduler also prices)
+    for nd in (1, 8, 16, 32, 64):
+        grid.append((0, nd, 2048, 0))
+    for chunk in (16, 64, 128):
+        grid.append((chunk, 0, 0, 0))
     order = rng.permutation(len(grid))   # random order: no systematic clock drift along the grid
     fit_shapes, fit_ms, table = [], [], []
     for gi in order:

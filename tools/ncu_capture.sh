@@ -1,0 +1,27 @@
+#!/bin/bash
+# ncu evidence for one round (run on the GPU box from the repo root):
+#   bash tools/ncu_capture.sh <tag>
+# 1. launch list of one 32-layer bench step (serialised, cold-cache per-launch times)
+# 2. `--set full` captures of the dominant kernels on a 2-layer model of the same shapes
+set -u
+TAG=${1:-r1c}
+OUT=gpurun_out
+mkdir -p $OUT
+if [ "${SKIP_LAUNCHES:-0}" != 1 ]; then
+ncu --metrics gpu__time_duration.sum --clock-control none --nvtx --nvtx-include "step/" --csv \
+    --log-file $OUT/launches_$TAG.csv python tools/profile_step.py --steps 1 > $OUT/ncu_launch_$TAG.log 2>&1
+fi
+cap() {  # name, kernel regex, skip
+  QOS_OVERLAP_ATTN=0 ncu --set full --clock-control none --import-source on --nvtx --nvtx-include "step/" \
+      --kernel-name-base demangled -k "regex:$2" -s "$3" -c 1 -o $OUT/prof_${1}_$TAG \
+      python tools/profile_step.py --steps 1 --layers 2 > $OUT/ncu_${1}_$TAG.log 2>&1
+}
+# tile-GEMM launches per layer at T = 2176: QKV(+RoPE), O, gate/up, down -> layer 1 = 4..7
+cap gemm_qkv_rope 'gemm_tcgen05_kernel' 4
+cap gemm_gateup 'gemm_tcgen05_kernel' 6
+cap gemm_down 'gemm_tcgen05_kernel' 7
+if [ "${ONLY_GEMM:-0}" != 1 ]; then
+cap decode_attn 'decode_attn_kernel' 1
+cap prefill_attn 'prefill_attn_tc_kernel' 1
+fi
+ls -la $OUT

@@ -58,8 +58,8 @@ def main():
                 ms.append(t)
         model = LatencyModel().fit(shapes, ms)
     else:
-        model = LatencyModel.from_json(json.dumps(
-            json.load(open(os.path.join(ROOT, "profiles", "latency_table_r1.json")))["refit"]["model_json"]))
+        prof = json.load(open(os.path.join(ROOT, "profiles", "latency_table_r1.json")))
+        model = LatencyModel.from_json(json.dumps(prof.get("refit", prof)["model_json"]))
 
     def pred(chunks, ctx):
         return model.predict(StepShape(list(chunks), list(ctx)))
