@@ -87,6 +87,31 @@ class EngineExecutor:
 
 
 def replay(trace, scheduler: QoServeScheduler, executor, max_steps: int = 10**9, log_chunks: bool = True):
+    return summarize(*_run(trace, scheduler, executor, max_steps, log_chunks))
+
+
+def replay_replicas(trace, n_replicas: int, make_scheduler, make_executor, max_steps: int = 10**9):
+    """Round-robin load balancing over independent replicas (one TP1
+    replica per GPU): request i goes to replica i mod n in arrival order; replicas share
+    nothing, so each replays its share of the trace on its own clock.  Metrics are computed
+    over all requests of all replicas."""
+    order = sorted(range(len(trace)), key=lambda i: trace[i]["t_arrival"])
+    reqs, done, t_end, steps, chunk_log, wall = [], [], 0.0, 0, [], 0.0
+    for k in range(n_replicas):
+        part = [trace[i] for i in order[k::n_replicas]]
+        r, d, t, st, cl, w = _run(part, make_scheduler(), make_executor(), max_steps, True)
+        reqs += r
+        done += d
+        t_end = max(t_end, t)
+        steps += st
+        chunk_log += cl
+        wall += w
+    out = summarize(reqs, done, t_end, steps, chunk_log, wall)
+    out["replicas"] = n_replicas
+    return out
+
+
+def _run(trace, scheduler: QoServeScheduler, executor, max_steps: int, log_chunks: bool):
     reqs = [Request(**t) for t in trace]
     pending = sorted(reqs, key=lambda r: r.t_arrival)
     now, k, steps = 0.0, 0, 0
@@ -112,7 +137,7 @@ def replay(trace, scheduler: QoServeScheduler, executor, max_steps: int = 10**9,
         for r in scheduler.complete(chunks, decodes, now):
             executor.release(r)
             done.append(r)
-    return summarize(reqs, done, now, steps, chunk_log, time.time() - wall0)
+    return reqs, done, now, steps, chunk_log, time.time() - wall0
 
 
 def summarize(reqs, done, t_end, steps, chunk_log, wall_s):

@@ -120,6 +120,11 @@ class SchedulerConfig:
     chunk_step: int = 64
     margin: float = 0.05              # under-predict the chunk
     max_decodes: int = 256
+    # "slack": QoServe's dynamic chunking (the chunk fits the minimum decode slack);
+    # "medha": Medha-style adaptive chunking (NEXT-4 variant): every step
+    # targets a fixed latency, so chunks shrink as the prefill's cached prefix grows
+    chunk_policy: str = "slack"
+    medha_target_ms: float = 50.0
 
 
 class QoServeScheduler:
@@ -162,24 +167,32 @@ class QoServeScheduler:
     def min_slack(self, now: float) -> float:
         return min((self.slack(r, now) for r in self.decode_q), default=math.inf)
 
-    def prefill_budget(self, ctx: list, min_slack_s: float) -> int:
+    def prefill_budget(self, ctx: list, min_slack_s: float, kv_start: int = 0) -> int:
         """GET_PREFILL_BUDGET (Alg. 1 line 7): largest chunk with predicted latency within the
-        minimum decode slack (with margin); max_chunk when no decode constrains the step."""
-        if not math.isfinite(min_slack_s):
+        minimum decode slack (with margin); max_chunk when no decode constrains the step.  The
+        prediction prices the chunk at `kv_start` (the cached prefix of the request it will
+        come from: attention over the prefix grows for later chunks).
+        Medha policy: the budget is a fixed per-step latency target instead of the slack."""
+        if self.cfg.chunk_policy == "medha":
+            budget_ms = self.cfg.medha_target_ms * (1 - self.cfg.margin)
+            if math.isfinite(min_slack_s):
+                budget_ms = min(budget_ms, max(0.0, min_slack_s) * 1e3 * (1 - self.cfg.margin))
+        elif not math.isfinite(min_slack_s):
             return self.cfg.max_chunk
-        budget_ms = max(0.0, min_slack_s) * 1e3 * (1 - self.cfg.margin)
+        else:
+            budget_ms = max(0.0, min_slack_s) * 1e3 * (1 - self.cfg.margin)
         best = 0
         c = self.cfg.min_chunk
         while c <= self.cfg.max_chunk:
-            if self.predict_ms([(0, c)], ctx) <= budget_ms:
+            if self.predict_ms([(kv_start, c)], ctx) <= budget_ms:
                 best = c
             else:
                 break
             c += self.cfg.chunk_step
         return best
 
-    def step_estimate_s(self, chunk: int, ctx: list) -> float:
-        return self.predict_ms([(0, chunk)] if chunk else [], ctx) * 1e-3
+    def step_estimate_s(self, chunk: int, ctx: list, kv_start: int = 0) -> float:
+        return self.predict_ms([(kv_start, chunk)] if chunk else [], ctx) * 1e-3
 
     def will_violate(self, r: Request, now: float, chunk: int, ctx: list) -> bool:
         """now + predicted time to finish the current phase > deadline (reading s19)."""
@@ -197,8 +210,9 @@ class QoServeScheduler:
         """Returns (chunks [(Request, n_tokens)], decodes [Request])."""
         decodes = list(self.decode_q)[: self.cfg.max_decodes]          # GET_ALL_DECODES
         ctx = [r.ctx_len for r in decodes]                              # GET_DECODE_CONTEXT
-        C = self.prefill_budget(ctx, self.min_slack(now))               # lines 5-7
         queue = sorted(self.prefill_q, key=self.sort_key)               # line 8
+        kv0 = queue[0].prefill_done if queue else 0                     # prefix of the head chunk
+        C = self.prefill_budget(ctx, self.min_slack(now), kv0)          # lines 5-7
         chunks, count = [], 0
         inflight_skipped = []
         i = 0

@@ -139,3 +139,59 @@ def test_model_replay_conserves_requests():
 def test_decode_history_default():
     h = DecodeHistory(default=77.0)
     assert h.estimate("new") == 77.0
+
+
+def prefix_model(chunks, ctx):
+    """Stand-in model whose chunk cost grows with the cached prefix (attention over it)."""
+    T = sum(n for _, n in chunks) + len(ctx)
+    return 5.0 + 0.01 * T + 1e-3 * sum(c + 1 for c in ctx) / 1000.0 + 2e-6 * sum(n * ks for ks, n in chunks)
+
+
+def test_budget_prices_the_chunk_prefix():
+    """Dynamic chunking prices the chunk at its request's cached prefix: later chunks of a
+    long prompt get smaller budgets (attention grows for later chunks)."""
+    s = QoServeScheduler(SchedulerConfig(max_chunk=4096, margin=0.0), prefix_model)
+    ctx = [2000] * 16
+    b0, b8k = s.prefill_budget(ctx, 0.030, 0), s.prefill_budget(ctx, 0.030, 8192)
+    assert 0 < b8k < b0
+    assert prefix_model([(8192, b8k)], ctx) <= 30.0 < prefix_model([(8192, b8k + 64)], ctx)
+
+
+def test_medha_policy_shrinks_chunks_of_a_long_prefill():
+    """NEXT-4 variant (Medha, PAPER.md:1597-1649): one 10K-token prefill next to 500 decodes;
+    with a fixed per-step target every step fits it and the chunk shrinks as the prefix grows."""
+    cfg = SchedulerConfig(max_chunk=8192, margin=0.0, chunk_policy="medha", medha_target_ms=40.0)
+    s = QoServeScheduler(cfg, prefix_model)
+    decs = []
+    for i in range(500):
+        r = Request(1000 + i, 0.0, 1000, "Q2", decode_len=10 ** 6)
+        r.prefill_done = r.prompt_len
+        decs.append(r)
+    s.decode_q.extend(decs)
+    big = Request(1, 0.0, 10_000, "Q2", decode_len=500)
+    s.submit(big)
+    now, sizes = 0.0, []
+    while big.prefill_rem > 0 and len(sizes) < 100:
+        chunks, decodes = s.create_batch(now)
+        c = sum(n for r, n in chunks if r is big)
+        assert c > 0
+        ms = prefix_model([(big.prefill_done, c)], [r.ctx_len for r in decodes])
+        assert ms <= 40.0 + 1e-9
+        sizes.append(c)
+        now += ms * 1e-3
+        s.complete(chunks, decodes, now)
+    full = sizes[:-1]                      # the last chunk is the remainder
+    assert len(full) >= 2 and all(a >= b for a, b in zip(full, full[1:])) and full[0] > full[-1]
+
+
+def test_round_robin_replicas():
+    """8 TP1 replicas with round-robin routing: every request is served
+    once, and 8 replicas at 8x the load see no more violations than one replica at 1x."""
+    from paper_conf_asplos_goelmkar26_b200.replay import replay_replicas
+    tr8 = synth.trace(16.0, 20.0, "azure_conv")
+    out8 = replay_replicas(tr8, 8, lambda: QoServeScheduler(SchedulerConfig(max_chunk=2048), lin_model),
+                           lambda: ModelExecutor(lin_model))
+    assert out8["requests"] == out8["finished"] == len(tr8) and out8["replicas"] == 8
+    tr1 = synth.trace(2.0, 20.0, "azure_conv")
+    out1 = replay(tr1, QoServeScheduler(SchedulerConfig(max_chunk=2048), lin_model), ModelExecutor(lin_model))
+    assert out8["violations_pct"] <= out1["violations_pct"] + 1.0

@@ -2,6 +2,7 @@
 
   python tools/replay_run.py --mode engine --dataset azure_conv --qps 10,20,30 --duration 60
   python tools/replay_run.py --mode model  --dataset azure_code --qps 5,10,20,30,40 --duration 1800
+  python tools/replay_run.py --mode model  --dataset azure_conv --qps 80,160,240 --replicas 8
 
 engine: every step is a real device-timed qos_hybrid_step (virtual clock += measured ms); the
         scheduler's latency model is fitted to a quick qos_profile_step sweep of this engine.
@@ -19,7 +20,7 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 
 import synth  # noqa: E402
 from paper_conf_asplos_goelmkar26_b200.latency_model import LatencyModel, StepShape  # noqa: E402
-from paper_conf_asplos_goelmkar26_b200.replay import EngineExecutor, ModelExecutor, replay  # noqa: E402
+from paper_conf_asplos_goelmkar26_b200.replay import EngineExecutor, ModelExecutor, replay, replay_replicas  # noqa: E402
 from paper_conf_asplos_goelmkar26_b200.scheduler import QoServeScheduler, SchedulerConfig  # noqa: E402
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
@@ -34,6 +35,7 @@ def main():
     ap.add_argument("--alpha", type=float, default=8.0)
     ap.add_argument("--max-chunk", type=int, default=4096)
     ap.add_argument("--out", default=None)
+    ap.add_argument("--replicas", type=int, default=1, help="model mode: round-robin TP1 replicas (1 per GPU)")
     a = ap.parse_args()
     results = []
     eng = None
@@ -66,20 +68,25 @@ def main():
 
     for qps in [float(x) for x in a.qps.split(",")]:
         tr = synth.trace(qps, a.duration, a.dataset)
-        sched = QoServeScheduler(SchedulerConfig(alpha_ms_per_token=a.alpha, max_chunk=a.max_chunk), pred)
+
+        def mk_sched():
+            return QoServeScheduler(SchedulerConfig(alpha_ms_per_token=a.alpha, max_chunk=a.max_chunk), pred)
         if a.mode == "engine":
             ex = EngineExecutor(eng, 128256, lambda r, s, n: synth.request_tokens(r, n, 128256, start=s))
+            out = replay(tr, mk_sched(), ex)
+        elif a.replicas > 1:
+            out = replay_replicas(tr, a.replicas, mk_sched, lambda: ModelExecutor(pred))
         else:
-            ex = ModelExecutor(pred)
-        out = replay(tr, sched, ex)
-        out.update({"qps": qps, "dataset": a.dataset, "mode": a.mode, "duration_s": a.duration, "alpha": a.alpha})
+            out = replay(tr, mk_sched(), ModelExecutor(pred))
+        out.update({"qps": qps, "dataset": a.dataset, "mode": a.mode, "duration_s": a.duration, "alpha": a.alpha,
+                    "replicas": a.replicas})
         series = out.pop("chunk_series", None)
         print(json.dumps(out), flush=True)
         out["chunk_series"] = series
         results.append(out)
     ok = [r["qps"] for r in results if r["violations_pct"] <= 1.0]
     summary = {"goodput_qps": max(ok) if ok else 0.0, "dataset": a.dataset, "mode": a.mode,
-               "qps_tested": [r["qps"] for r in results]}
+               "replicas": a.replicas, "qps_tested": [r["qps"] for r in results]}
     print(json.dumps(summary), flush=True)
     if a.out:
         json.dump({"summary": summary, "runs": results}, open(a.out, "w"), indent=1)
