@@ -182,6 +182,9 @@ ATTN_CASES = [
     ("tiny-mha", {}, [(5, 77)], [33, 64], 1.0),
     ("llama3-70b", dict(n_layers=1, n_heads=8, n_kv_heads=1, d_model=1024, ffn_dim=1024, num_blocks=1024),
      [(0, 48)], [700, 3000], 1.0),   # group 8 = Llama-3-70B at TP8
+    # configs[3] maximum context: a chunk deep into a 20k prefix and a decode over 32k keys
+    ("llama3-70b", dict(n_layers=1, n_heads=8, n_kv_heads=1, d_model=1024, ffn_dim=1024, num_blocks=4096,
+                        max_seq_len=32784), [(20000, 96)], [32767], 1.0),
 ]
 
 
@@ -189,7 +192,7 @@ ATTN_CASES = [
 def test_attention_parity(case):
     from oracle.model import causal_attention
     preset, over, chunks, ctxs, scale = ATTN_CASES[case]
-    q, cfg, eng = make_engine(preset, max_seq_len=8192, **over)
+    q, cfg, eng = make_engine(preset, **{"max_seq_len": 8192, **over})
     H, Hkv, hd = cfg.n_heads, cfg.n_kv_heads, cfg.head_dim
     g = H // Hkv
     rng = np.random.default_rng(100 + case)

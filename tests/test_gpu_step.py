@@ -226,3 +226,31 @@ def test_execution_options_do_not_change_results(opts):
         eng.qos_engine_set_option("no_such_option", 1)
     eng.qos_engine_set_option("pdl", 1)  # process-wide: restore the default
     eng.close()
+
+
+def test_long_context_step_parity():
+    """Maximum context (configs[3]: up to 32k): a 100-token chunk at kv_start 16000 and decodes
+    at ctx 32767 / 20000 / 17, all prefixes synthetic KV, through qos_hybrid_step vs the oracle
+    (logits rows <= 1e-2, same greedy tokens) — long block tables, many decode splits."""
+    q, cfg, eng = make_engine("tiny", num_blocks=4600, max_seq_len=32784, max_requests=8)
+    eng.qos_engine_load_synthetic(0)
+    orc = _oracle("tiny", num_blocks=4600)
+    rng = np.random.default_rng(5)
+    plan = {1: 16000, 2: 32767, 3: 20000, 4: 17}
+    for r, n in plan.items():
+        total = n + (100 if r == 1 else 1)
+        eng.qos_kv_alloc(r, total)
+        orc.kv_alloc(r, total)
+        eng.qos_kv_fill_synthetic(r, n, synth.SEED_KVFILL)
+        orc.kv_fill_synthetic(r, n, synth.SEED_KVFILL)
+    toks = [int(x) for x in rng.integers(0, cfg.vocab, 100)]
+    decs = [(r, plan[r], int(rng.integers(0, cfg.vocab))) for r in (2, 3, 4)]
+    b = q.make_batch([(1, plan[1], np.array(toks, np.int32))], decs)
+    lg, tk = eng.step_host(b, cfg.vocab)
+    ref = orc.hybrid_step([(1, plan[1], toks)], decs)
+    assert row_rel_err(lg, ref) <= TOL_LOGITS
+    top = np.argsort(ref, axis=1)
+    gap = ref[np.arange(len(ref)), top[:, -1]] - ref[np.arange(len(ref)), top[:, -2]]
+    clear = gap > 2 * TOL_LOGITS * np.abs(ref).max(axis=1)
+    assert np.array_equal(np.asarray(tk)[clear], top[clear, -1])
+    eng.close()

@@ -17,7 +17,7 @@ from test_gpu_ops import ATTN_CASES  # noqa: E402
 from oracle.model import causal_attention  # noqa: E402
 
 for case, (preset, over, chunks, ctxs, scale) in enumerate(ATTN_CASES):
-    q, cfg, eng = make_engine(preset, max_seq_len=8192, **over)
+    q, cfg, eng = make_engine(preset, **{"max_seq_len": 8192, **over})
     H, Hkv, hd = cfg.n_heads, cfg.n_kv_heads, cfg.head_dim
     g = H // Hkv
     rng = np.random.default_rng(100 + case)
