@@ -17,6 +17,7 @@
 // other's MMAs.
 #include <cfloat>
 #include <climits>
+#include <cstdlib>
 
 #include "common.cuh"
 #include "internal.h"
@@ -86,6 +87,26 @@ QOS_DEV float2 add2(float2 a, float2 b) {
   return d;
 }
 
+// 2^x for a pair on the FMA pipe (relieves MUFU, which at 16 ex2/clk/SM is as slow as the
+// tensor core on a 128x64 S tile): x = j + f with j = rint(x) (1.5*2^23 round trick), f in
+// [-0.5, 0.5]; 2^f by a degree-3 minimax polynomial (max relative error 7.5e-5, below the
+// fp16 rounding of P, 2^-11); 2^j is added into the exponent field.  x is clamped at -125 so
+// the biased exponent of the result stays >= 1 (2^-125 rounds to 0 in fp16, like MUFU's
+// flush-to-zero; masked scores arrive here as -inf).
+QOS_DEV float2 ex2_poly2(float2 x) {
+  x.x = fmaxf(x.x, -125.f);
+  x.y = fmaxf(x.y, -125.f);
+  const float2 magic = make_float2(12582912.f, 12582912.f), nmagic = make_float2(-12582912.f, -12582912.f);
+  const float2 t = add2(x, magic);
+  const float2 f = fma2(add2(t, nmagic), make_float2(-1.f, -1.f), x);  // x - rint(x), exact
+  float2 p = fma2(make_float2(0.05517150089144707f, 0.05517150089144707f), f,
+                  make_float2(0.24261096119880676f, 0.24261096119880676f));
+  p = fma2(p, f, make_float2(0.6932609677314758f, 0.6932609677314758f));
+  p = fma2(p, f, make_float2(0.9999280571937561f, 0.9999280571937561f));
+  return make_float2(__uint_as_float(__float_as_uint(p.x) + (__float_as_uint(t.x) << 23)),
+                     __uint_as_float(__float_as_uint(p.y) + (__float_as_uint(t.y) << 23)));
+}
+
 // D[tmem] (+)= A[tmem] · B[smem desc]   (kind::f16, A = 16-bit pairs packed in 32-bit columns)
 QOS_DEV void umma_bf16_ts(uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc, uint32_t idesc, uint32_t accumulate) {
   asm volatile(
@@ -121,7 +142,7 @@ struct FaParams {
   float scale_log2;
 };
 
-template <int HD>
+template <int HD, int POLY>
 __global__ void __launch_bounds__(kFaThreads, 2)
     prefill_attn_tc_kernel(const __grid_constant__ CUtensorMap kvmap, const FaParams p,
                            const PrefillItem* __restrict__ items) {
@@ -273,6 +294,11 @@ __global__ void __launch_bounds__(kFaThreads, 2)
       const int sb = j & 1;
       mbar_wait(&s_full[sb], (j >> 1) & 1);
       tc_fence_after();
+      if (POLY < 0) {  // measurement-only variant: MMA + TMA pipeline without the softmax
+        tc_fence_before();
+        mbar_arrive(&p_full[sb]);
+        continue;
+      }
       const uint32_t s_addr = lane_base + (sb ? C::kColS1 : C::kColS0);
       const int key0 = j * C::kKeys;
       // masking only where a key of this tile can exceed a row's position
@@ -284,21 +310,21 @@ __global__ void __launch_bounds__(kFaThreads, 2)
       for (int c = 0; c < C::kKeys / 16; ++c)
         tmem_ld32x32b_x16(s_addr + c * 16, *reinterpret_cast<uint32_t(*)[16]>(&r[c * 16]));
       tmem_ld_wait();
+      // causal mask (only the tiles that reach past a row's position): masked scores become
+      // -inf, so the max and exp passes below are the same for every tile (2^-inf = 0).  Kept a
+      // real branch so unmasked tiles do not execute predicated selects.
+      if (masked) {
+        const int lim = (pos_r < 0 ? -1 : pos_r) - key0;  // key i is visible iff i <= lim
+#pragma unroll
+        for (int i = 0; i < C::kKeys; ++i)
+          if (i > lim) r[i] = 0xff800000u;  // -inf
+      }
       // row max of the raw scores (scaled afterwards; the scale is positive)
       // (four independent 3-input max chains: a short dependency chain)
       float mq[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
-      if (masked) {
 #pragma unroll
-        for (int i = 0; i < C::kKeys; i += 2) {
-          const float a = key0 + i <= pos_r ? __uint_as_float(r[i]) : -INFINITY;
-          const float b = key0 + i + 1 <= pos_r ? __uint_as_float(r[i + 1]) : -INFINITY;
-          mq[(i >> 1) & 3] = fmax3(mq[(i >> 1) & 3], a, b);
-        }
-      } else {
-#pragma unroll
-        for (int i = 0; i < C::kKeys; i += 2)
-          mq[(i >> 1) & 3] = fmax3(mq[(i >> 1) & 3], __uint_as_float(r[i]), __uint_as_float(r[i + 1]));
-      }
+      for (int i = 0; i < C::kKeys; i += 2)
+        mq[(i >> 1) & 3] = fmax3(mq[(i >> 1) & 3], __uint_as_float(r[i]), __uint_as_float(r[i + 1]));
       float mx = fmax3(mq[0], mq[1], fmaxf(mq[2], mq[3]));
       mx *= p.scale_log2;
       // lazy rescale: keep the previous max unless the new one exceeds it by > 8 (P <= 2^8)
@@ -319,12 +345,8 @@ __global__ void __launch_bounds__(kFaThreads, 2)
           // paired fp32 ops (FFMA2 / FADD2) halve the softmax's FMA-pipe instructions
           const float2 x = fma2(make_float2(__uint_as_float(r[c * 32 + 2 * i]), __uint_as_float(r[c * 32 + 2 * i + 1])),
                                 scale2, nmb2);
-          float2 pp = make_float2(ex2(x.x), ex2(x.y));
-          if (masked) {
-            const int k = key0 + c * 32 + 2 * i;
-            pp.x = (k <= pos_r) ? pp.x : 0.f;
-            pp.y = (k + 1 <= pos_r) ? pp.y : 0.f;
-          }
+          // every POLY-th pair on the FMA pipe (POLY = 0: none), the rest on MUFU
+          float2 pp = (POLY > 0 && i % (POLY > 0 ? POLY : 1) == (POLY > 0 ? POLY : 1) - 1) ? ex2_poly2(x) : make_float2(ex2(x.x), ex2(x.y));
           hi[i] = pack_f16(pp.x, pp.y);
           sum2[i & 3] = add2(sum2[i & 3], pp);
         }
@@ -394,11 +416,13 @@ __global__ void __launch_bounds__(kFaThreads, 2)
   }
 }
 
-template <int HD>
+static int g_fa_poly = getenv("QOS_FA_POLY") ? atoi(getenv("QOS_FA_POLY")) : 4;
+
+template <int HD, int POLY>
 static cudaError_t prefill_tc_t(const AttnLaunch& a, const PrefillItem* items, int n_items, cudaStream_t st) {
   static bool set = false;
   if (!set) {
-    cudaError_t e = cudaFuncSetAttribute(prefill_attn_tc_kernel<HD>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaError_t e = cudaFuncSetAttribute(prefill_attn_tc_kernel<HD, POLY>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          FaCfg<HD>::kSmem);
     if (e != cudaSuccess) return e;
     set = true;
@@ -415,17 +439,30 @@ static cudaError_t prefill_tc_t(const AttnLaunch& a, const PrefillItem* items, i
   p.tables = a.tables;
   p.table_w = a.table_w;
   p.scale_log2 = a.scale_log2;
-  return launch_pdl(prefill_attn_tc_kernel<HD>, dim3(n_items), dim3(kFaThreads), FaCfg<HD>::kSmem, st, *a.kv_tmap, p,
+  return launch_pdl(prefill_attn_tc_kernel<HD, POLY>, dim3(n_items), dim3(kFaThreads), FaCfg<HD>::kSmem, st, *a.kv_tmap, p,
                     items);
 }
+
+void set_fa_poly(int n) { g_fa_poly = n; }
 
 int prefill_tc_positions_per_tile(int group) { return 128 / group; }
 
 cudaError_t launch_prefill_attention_tc(const AttnLaunch& a, const PrefillItem* items, int n_items, cudaStream_t st) {
   if (n_items == 0) return cudaSuccess;
   count_launch(1);
-  if (a.hd == 128) return prefill_tc_t<128>(a, items, n_items, st);
-  if (a.hd == 64) return prefill_tc_t<64>(a, items, n_items, st);
+  const int poly = g_fa_poly;
+  if (a.hd == 128) {
+    if (poly == 0) return prefill_tc_t<128, 0>(a, items, n_items, st);
+    if (poly < 0) return prefill_tc_t<128, -1>(a, items, n_items, st);
+    if (poly == 2) return prefill_tc_t<128, 2>(a, items, n_items, st);
+    if (poly == 3) return prefill_tc_t<128, 3>(a, items, n_items, st);
+    if (poly == 8) return prefill_tc_t<128, 8>(a, items, n_items, st);
+    return prefill_tc_t<128, 4>(a, items, n_items, st);
+  }
+  if (a.hd == 64) {
+    if (poly == 0) return prefill_tc_t<64, 0>(a, items, n_items, st);
+    return prefill_tc_t<64, 4>(a, items, n_items, st);
+  }
   return cudaErrorInvalidValue;
 }
 

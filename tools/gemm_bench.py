@@ -28,11 +28,13 @@ ap.add_argument("--ms", default="1,16,64,128,256,384,512,1024,2176")
 ap.add_argument("--ksplit", type=int, default=0)
 ap.add_argument("--iters", type=int, default=24)
 ap.add_argument("--shapes", default=",".join(SHAPES))
+ap.add_argument("--epi", default=None, help="override the epilogue of every shape")
 a = ap.parse_args()
 torch.cuda.set_device(0)
 L2 = 126 * 1024 * 1024
 for name in a.shapes.split(","):
     N, K, epi = SHAPES[name]
+    epi = a.epi or epi
     wbytes = N * K * 2
     ncopy = max(2, -(-3 * L2 // wbytes))
     Bs = [(torch.randn(N, K, device="cuda") / K ** 0.5).to(torch.bfloat16) for _ in range(ncopy)]
@@ -64,7 +66,7 @@ for name in a.shapes.split(","):
         e1.record()
         torch.cuda.synchronize()
         us = e0.elapsed_time(e1) * 1e3 / a.iters
-        print(json.dumps({"gemm": name, "M": M, "N": N, "K": K, "ksplit": a.ksplit, "us": round(us, 2),
+        print(json.dumps({"gemm": name, "epi": epi, "M": M, "N": N, "K": K, "ksplit": a.ksplit, "us": round(us, 2),
                           "tflops": round(2 * M * N * K / us / 1e6, 1),
                           "weight_gbs": round(wbytes / us / 1e3, 1)}), flush=True)
         del A, Cout
