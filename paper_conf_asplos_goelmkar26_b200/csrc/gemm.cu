@@ -46,7 +46,10 @@ struct GemmCfg {
   static constexpr int kBBytes = BN * kBK * 2;
   static constexpr int kStageBytes = kABytes + kBBytes;
   static constexpr int kTmemCols = 2 * BN;
-  static constexpr int kSmemBytes = kStages * kStageBytes + 1024 /*align*/ + 256 /*barriers*/;
+  // per epilogue warp: a 32-row staging tile (up to 256 B per row) so that the warp's stores
+  // are coalesced row segments instead of one row per thread
+  static constexpr int kStageWarpBytes = 32 * 256;
+  static constexpr int kSmemBytes = kStages * kStageBytes + 1024 /*align*/ + 256 /*barriers*/ + 4 * kStageWarpBytes;
 };
 
 struct GemmArgs {
@@ -171,6 +174,128 @@ QOS_DEV void epi_qkv_rope(const GemmArgs& p, int row, bool row_ok, int n_t, Fetc
   }
 }
 
+// ---- staged epilogue: a warp's 32 rows (thread = row, as tcgen05.ld 32x32b delivers them)
+// are written to a smem tile of RB bytes per row and leave as coalesced 16-byte chunks
+// (RB/16 threads per row segment).  16-byte chunk k of row r sits at chunk k ^ sw(r) so both
+// the row-per-thread writes and the chunk-per-thread reads are bank-conflict free.
+template <int RB>
+QOS_DEV uint32_t stg_off(int r, int k) {
+  return uint32_t(r * RB + 16 * (k ^ (RB >= 128 ? (r & 7) : ((r >> 1) & 3))));
+}
+template <int RB>
+QOS_DEV void stg_put(uint8_t* stg, int r, int k, uint4 v) {
+  *reinterpret_cast<uint4*>(stg + stg_off<RB>(r, k)) = v;
+}
+// dst(rr, k, v): store chunk k (16 B) of row rr
+template <int RB, typename Dst>
+QOS_DEV void stg_flush(const uint8_t* stg, int lane, Dst dst) {
+  constexpr int kPer = RB / 16;  // threads per row segment
+  __syncwarp();
+#pragma unroll
+  for (int pass = 0; pass < RB * 32 / 512; ++pass) {
+    const int idx = pass * 32 + lane;
+    const int rr = idx / kPer, k = idx % kPer;
+    dst(rr, k, *reinterpret_cast<const uint4*>(stg + stg_off<RB>(rr, k)));
+  }
+  __syncwarp();
+}
+QOS_DEV void red_add_v4(float* addr, uint4 v) {  // fire-and-forget fp32 add at L2
+  asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(addr), "f"(__uint_as_float(v.x)),
+               "f"(__uint_as_float(v.y)), "f"(__uint_as_float(v.z)), "f"(__uint_as_float(v.w))
+               : "memory");
+}
+
+// The fused a4+a5+a6 epilogue, staged: per head of the tile, RoPE'd q (or k) and v rows are
+// built in smem, then written as coalesced row segments to the qkv buffer (q) or to the paged
+// cache at each row's slot (k, v).  row0 = first row of this warp; `sl` = this thread's slot.
+template <int BN, typename Fetch>
+QOS_DEV void epi_qkv_rope_staged(const GemmArgs& p, uint8_t* stg, int lane, int row0, int n_t, Fetch fetch) {
+  const int hd = p.hd, half = hd / 2;
+  const int row = row0 + lane;
+  const bool row_ok = row < p.M;
+  const int ps = row_ok ? __ldg(p.pos + row) : 0;
+  const int sl = row_ok ? __ldg(p.slot + row) : 0;
+  for (int hh = 0; hh < BN / hd; ++hh) {
+    const int col0 = n_t * BN + hh * hd;
+    if (col0 >= p.N) break;  // warp-uniform
+    const int head = col0 / hd;
+    const int kind = head < p.H ? 0 : head < p.H + p.Hkv ? 1 : 2;
+    const int kvh = kind == 1 ? head - p.H : head - p.H - p.Hkv;
+    auto put = [&](int k, const uint32_t (&a)[8]) {  // 16 bf16/f16 values = chunks k, k+1
+      if (hd == 128) {
+        stg_put<256>(stg, lane, k, make_uint4(a[0], a[1], a[2], a[3]));
+        stg_put<256>(stg, lane, k + 1, make_uint4(a[4], a[5], a[6], a[7]));
+      } else {
+        stg_put<128>(stg, lane, k, make_uint4(a[0], a[1], a[2], a[3]));
+        stg_put<128>(stg, lane, k + 1, make_uint4(a[4], a[5], a[6], a[7]));
+      }
+    };
+    if (kind < 2) {
+      // RoPE with coalesced cos/sin reads: the 16 (x, y) pairs of chunk i0 are staged in fp32
+      // (x in chunks 0-3, y in 4-7 of a 128-B row), then each lane rotates 2 pairs of one row
+      // (8 lanes per row read its 128 B of the table) and stores 2 x 4 B of q (or k).
+      for (int i0 = 0; i0 < half; i0 += 16) {
+        // this lane's cos/sin for its 8 (row, pair couple) slots, requested before the TMEM
+        // loads so their latency overlaps the staging
+        float4 c[8];
+        int slr[8];
+#pragma unroll
+        for (int pass = 0; pass < 8; ++pass) {
+          const int rr = pass * 4 + (lane >> 3), k = lane & 7;
+          const int prr = __shfl_sync(0xffffffffu, ps, rr);
+          slr[pass] = __shfl_sync(0xffffffffu, sl, rr);
+          c[pass] = __ldg(reinterpret_cast<const float4*>(p.rope + size_t(prr) * half + i0 + 2 * k));
+        }
+        float x[16], y[16];
+        fetch(hh * hd + i0, x);
+        fetch(hh * hd + half + i0, y);
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          stg_put<128>(stg, lane, k, make_uint4(__float_as_uint(x[4 * k]), __float_as_uint(x[4 * k + 1]),
+                                                __float_as_uint(x[4 * k + 2]), __float_as_uint(x[4 * k + 3])));
+          stg_put<128>(stg, lane, 4 + k, make_uint4(__float_as_uint(y[4 * k]), __float_as_uint(y[4 * k + 1]),
+                                                    __float_as_uint(y[4 * k + 2]), __float_as_uint(y[4 * k + 3])));
+        }
+        __syncwarp();
+#pragma unroll
+        for (int pass = 0; pass < 8; ++pass) {
+          const int rr = pass * 4 + (lane >> 3), k = lane & 7;  // row, pair couple (2k, 2k+1)
+          const float2 xv = *reinterpret_cast<const float2*>(stg + stg_off<128>(rr, k >> 1) + (k & 1) * 8);
+          const float2 yv = *reinterpret_cast<const float2*>(stg + stg_off<128>(rr, 4 + (k >> 1)) + (k & 1) * 8);
+          const float4 cc = c[pass];
+          const uint32_t lo = pack_bf16(xv.x * cc.x - yv.x * cc.y, xv.y * cc.z - yv.y * cc.w);
+          const uint32_t hi = pack_bf16(yv.x * cc.x + xv.x * cc.y, yv.y * cc.z + xv.y * cc.w);
+          const int r = row0 + rr;
+          if (r < p.M) {
+            __nv_bfloat16* d = kind == 0 ? reinterpret_cast<__nv_bfloat16*>(p.C) + size_t(r) * p.ldc + col0
+                                         : p.kplane + ((size_t(slr[pass] >> 4) * p.Hkv + kvh) * 16 + (slr[pass] & 15)) * hd;
+            *reinterpret_cast<uint32_t*>(d + i0 + 2 * k) = lo;
+            *reinterpret_cast<uint32_t*>(d + half + i0 + 2 * k) = hi;
+          }
+        }
+        __syncwarp();
+      }
+      continue;
+    }
+    // v head: fp16 rows staged whole, then coalesced row segments into the paged cache
+    for (int i0 = 0; i0 < hd; i0 += 16) {
+      float x[16];
+      fetch(hh * hd + i0, x);
+      uint32_t a[8];  // V is cached in fp16 (it meets fp16 P in P.V)
+#pragma unroll
+      for (int k = 0; k < 8; ++k) a[k] = pack_f16(x[2 * k], x[2 * k + 1]);
+      put(i0 / 8, a);
+    }
+    auto dst = [&](int rr, int k, uint4 v) {
+      const int slr = __shfl_sync(0xffffffffu, sl, rr);
+      if (row0 + rr >= p.M) return;
+      reinterpret_cast<uint4*>(p.vplane + ((size_t(slr >> 4) * p.Hkv + kvh) * 16 + (slr & 15)) * hd)[k] = v;
+    };
+    if (hd == 128) stg_flush<256>(stg, lane, dst);
+    else stg_flush<128>(stg, lane, dst);
+  }
+}
+
 // Epilogue of one row of a tile from summed fp32 partials, in independent column units
 // u0, u0 + ustep, ... (32 columns; SiLU: 32 outputs = 32 gate + 32 up columns; QKV: one head),
 // so several CTAs can share the reduction of one tile.  fetch32(col, v) / fetch16(col, v)
@@ -227,6 +352,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
   uint64_t* tempty = tfull + 2;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
   int* s_last = reinterpret_cast<int*>(tmem_slot + 1);
+  uint8_t* stg_all = smem + S * Cfg::kStageBytes + 256;  // 4 x kStageWarpBytes
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -395,9 +521,14 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     const int rit = q * 32 + lane;  // row inside the tile
     int acc = 0;
     uint32_t acc_phase = 0;
+    uint8_t* stg = stg_all + q * Cfg::kStageWarpBytes;
+    // whole tile straight from TMEM, staged through smem (coalesced stores); row = this thread's
+    // row, row0 = the warp's first row
     auto epi_tmem = [&](int n_t, int row, bool row_ok, uint32_t tbase) {
+        const int row0 = row - lane;
+        (void)row_ok;
         if constexpr (EPI == EPI_QKV_ROPE) {
-          epi_qkv_rope<BN>(p, row, row_ok, n_t, [&](int col, float (&v)[16]) {
+          epi_qkv_rope_staged<BN>(p, stg, lane, row0, n_t, [&](int col, float (&v)[16]) {
             uint32_t r[16];
             tmem_ld32x32b_x16(tbase + col, r);
             tmem_ld_wait();
@@ -413,34 +544,17 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
               tmem_ld32(tbase + g * 128 + h * 32, gv);
               tmem_ld32(tbase + g * 128 + 64 + h * 32, uv);
               const int col = n_t * (BN / 2) + g * 64 + h * 32;
-              if (row_ok && col < p.N / 2) epi_silu32(p, row, col, gv, uv);
+              if (col >= p.N / 2) continue;  // warp-uniform
+              uint32_t pk[16];
+#pragma unroll
+              for (int i = 0; i < 16; ++i) pk[i] = pack_bf16(silu(gv[2 * i]) * uv[2 * i], silu(gv[2 * i + 1]) * uv[2 * i + 1]);
+#pragma unroll
+              for (int k = 0; k < 4; ++k) stg_put<64>(stg, lane, k, make_uint4(pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]));
+              stg_flush<64>(stg, lane, [&](int rr, int k, uint4 v) {
+                if (row0 + rr < p.M)
+                  reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.C) + size_t(row0 + rr) * p.ldc + col)[k] = v;
+              });
             }
-          }
-        } else if constexpr (EPI == EPI_ADD_F32) {
-          // residual read-modify-write, software-pipelined: the residual loads of chunk c+1 are
-          // in flight while chunk c is added and stored (one exposed load latency per tile)
-          float* rrow = reinterpret_cast<float*>(p.C) + size_t(row) * p.ldc + n_t * BN;
-          const bool ok0 = row_ok;
-          float4 cur[8], nxt[8];
-#pragma unroll
-          for (int i = 0; i < 8; ++i) cur[i] = (ok0 && n_t * BN < p.N) ? reinterpret_cast<const float4*>(rrow)[i] : make_float4(0, 0, 0, 0);
-#pragma unroll 1
-          for (int c = 0; c < BN / 32; ++c) {
-            const bool ok_next = ok0 && c + 1 < BN / 32 && n_t * BN + (c + 1) * 32 < p.N;
-#pragma unroll
-            for (int i = 0; i < 8; ++i)
-              nxt[i] = ok_next ? reinterpret_cast<const float4*>(rrow + (c + 1) * 32)[i] : make_float4(0, 0, 0, 0);
-            float v[32];
-            tmem_ld32(tbase + c * 32, v);
-            if (row_ok && n_t * BN + c * 32 < p.N) {
-              float4* dst = reinterpret_cast<float4*>(rrow + c * 32);
-#pragma unroll
-              for (int i = 0; i < 8; ++i)
-                dst[i] = make_float4(cur[i].x + v[4 * i], cur[i].y + v[4 * i + 1], cur[i].z + v[4 * i + 2],
-                                     cur[i].w + v[4 * i + 3]);
-            }
-#pragma unroll
-            for (int i = 0; i < 8; ++i) cur[i] = nxt[i];
           }
         } else {
 #pragma unroll 1
@@ -448,7 +562,36 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
             float v[32];
             tmem_ld32(tbase + c * 32, v);
             const int col = n_t * BN + c * 32;
-            if (row_ok && col < p.N) epi_store32<EPI>(p, row, col, v);
+            if (col >= p.N) continue;  // warp-uniform (N % 32 == 0)
+            if constexpr (EPI == EPI_STORE_BF16 || EPI == EPI_BIAS_BF16) {
+              uint32_t pk[16];
+#pragma unroll
+              for (int i = 0; i < 16; ++i) {
+                float a0 = v[2 * i], a1 = v[2 * i + 1];
+                if constexpr (EPI == EPI_BIAS_BF16) {
+                  a0 += __ldg(p.bias + col + 2 * i);
+                  a1 += __ldg(p.bias + col + 2 * i + 1);
+                }
+                pk[i] = pack_bf16(a0, a1);
+              }
+#pragma unroll
+              for (int k = 0; k < 4; ++k) stg_put<64>(stg, lane, k, make_uint4(pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]));
+              stg_flush<64>(stg, lane, [&](int rr, int k, uint4 x) {
+                if (row0 + rr < p.M)
+                  reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.C) + size_t(row0 + rr) * p.ldc + col)[k] = x;
+              });
+            } else {
+#pragma unroll
+              for (int k = 0; k < 8; ++k)
+                stg_put<128>(stg, lane, k, make_uint4(__float_as_uint(v[4 * k]), __float_as_uint(v[4 * k + 1]),
+                                                      __float_as_uint(v[4 * k + 2]), __float_as_uint(v[4 * k + 3])));
+              stg_flush<128>(stg, lane, [&](int rr, int k, uint4 x) {
+                if (row0 + rr >= p.M) return;
+                float* d = reinterpret_cast<float*>(p.C) + size_t(row0 + rr) * p.ldc + col + 4 * k;
+                if constexpr (EPI == EPI_ADD_F32) red_add_v4(d, x);  // residual += tile (one add per element)
+                else *reinterpret_cast<uint4*>(d) = x;
+              });
+            }
           }
         }
     };

@@ -87,6 +87,7 @@ def run_point(c, nd, ctx, ks, tag):
         per = t / n
         by = 4 * hd * Hkv * nd * (ctx + 1)
         rec.update(decode_us_per_layer=round(per * 1e3, 2), decode_gbs=round(by / (per * 1e-3) / 1e9, 1))
+    rec["us_per_launch"] = {k: round(t / n * 1e3, 1) for k, (t, n) in tm.items() if n}
     print(json.dumps(rec), flush=True)
 
 
