@@ -208,6 +208,13 @@ int qos_profile_step_ex(qos_engine_t* eng, int32_t chunk_len, int32_t kv_start,
  *   "pdl" (1)              programmatic dependent launch of the step's kernel chain (each
  *                          kernel's prologue and weight prefetch overlap the previous kernel's
  *                          tail); process-wide, env QOS_PDL
+ *   "decode_round_split" (1) decode split-K ranges: the key blocks of a decode in a rounded
+ *                          number of near-equal block-aligned ranges (0: fixed 64..512-key
+ *                          ranges with a short last one)
+ *   "fa_poly" (4)          prefill attention: every n-th exp2 pair on the FMA pipe by a
+ *                          polynomial, the rest on MUFU (0 = all MUFU; -1 = measurement-only
+ *                          variant without the softmax, results invalid); process-wide,
+ *                          env QOS_FA_POLY
  * Results do not depend on the options (parity tests run with the defaults and variants). */
 int qos_engine_set_option(qos_engine_t* eng, const char* name, int64_t value);
 

@@ -243,6 +243,7 @@ struct qos_engine {
   bool dual_stream = false;       // QOS_DUAL=1: prefill rows and decode rows on two streams
   int dual_min_prefill = 512, dual_min_decode = 16;
   int dual_sms_pre = 0, dual_sms_dec = 0;  // SM budgets of the two streams' GEMMs (0 = all)
+  bool decode_round_split = true;  // option decode_round_split (A/B of the split-K ranges)
   bool overlap_attn = true;       // QOS_OVERLAP_ATTN=0 serialises a7 and a8 (for measurement)
   bool gemm_splitk = true;        // QOS_GEMM_SPLITK=0 disables split-K for small-M GEMMs
   int gemm_swab = 1;              // weight-streaming GEMM (gemm_swab.cu): 0 never, 1 auto, 2 always
@@ -437,11 +438,20 @@ int build_step(qos_engine* e, const qos_batch* b, bool check_lengths, uint8_t* b
   int64_t total_keys = 0;
   for (int i = 0; i < b->n_decode; ++i) total_keys += int64_t(b->decode[i].ctx_len) + 1;
   int split = 512;
+  // splits per decode: the key blocks in nsplit near-equal block-aligned ranges of about
+  // `split` keys (rounded to the nearest count, so 4097 keys make 8 ranges of 32-33 blocks, not
+  // 8 full ranges and a 1-key straggler that pays a whole CTA prologue and merge)
+  const bool round_split = e->decode_round_split;
+  auto nsplit_of = [&](int keys, int s) {
+    if (!round_split) return (keys + s - 1) / s;
+    const int nb = (keys + 15) / 16, sb = s / 16;
+    return std::max(1, (nb + sb / 2) / sb);
+  };
   {
     const int64_t target = int64_t(e->num_sms) * 4;  // items per kv head per ... heuristic
     auto count_items = [&](int s) {
       int64_t n = 0;
-      for (int i = 0; i < b->n_decode; ++i) n += (int64_t(b->decode[i].ctx_len) + s) / s;
+      for (int i = 0; i < b->n_decode; ++i) n += nsplit_of(b->decode[i].ctx_len + 1, s);
       return n * e->sh.Hkv;
     };
     while (split > 64 && count_items(split) < target) split /= 2;
@@ -460,15 +470,21 @@ int build_step(qos_engine* e, const qos_batch* b, bool check_lengths, uint8_t* b
     slot[t] = rs->blocks[p >> 4] * 16 + (p & 15);
     rows[b->n_prefill + i] = t;
     const int keys = p + 1;
-    const int nsplit = (keys + split - 1) / split;
+    const int nsplit = nsplit_of(keys, split);
+    const int nb = (keys + 15) / 16;
     for (int h = 0; h < e->sh.Hkv; ++h)
       for (int s = 0; s < nsplit; ++s) {
         DecodeItem it;
         it.row = t;
         it.table = rs->row;
         it.kv_head = h;
-        it.key0 = s * split;
-        it.key1 = std::min(keys, (s + 1) * split);
+        if (round_split) {
+          it.key0 = 16 * int(int64_t(s) * nb / nsplit);
+          it.key1 = std::min(keys, 16 * int(int64_t(s + 1) * nb / nsplit));
+        } else {
+          it.key0 = s * split;
+          it.key1 = std::min(keys, (s + 1) * split);
+        }
         it.part_base = part + h * nsplit;
         it.part = it.part_base + s;
         it.nsplit = nsplit;
@@ -1279,6 +1295,7 @@ int qos_engine_set_option(qos_engine_t* e, const char* name, int64_t value) {
   if (!e || !name) return set_error(QOS_ERR_INVALID_ARG, "args");
   const std::string n(name);
   if (n == "overlap_attn") e->overlap_attn = value != 0;
+  else if (n == "decode_round_split") e->decode_round_split = value != 0;
   else if (n == "gemm_splitk") e->gemm_splitk = value != 0;
   else if (n == "pdl") set_pdl(value != 0);  // process-wide
   else if (n == "fa_poly") set_fa_poly(int(value));  // process-wide

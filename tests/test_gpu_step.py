@@ -202,7 +202,7 @@ def test_llama8b_shapes_bench_batch_sampled_parity():
 
 @pytest.mark.parametrize("opts", [{"overlap_attn": 0}, {"gemm_splitk": 0}, {"pdl": 0}, {"gemm_swab": 0},
                                   {"gemm_streamk": 0}, {"gemm_streamk": 2, "gemm_swab": 0},
-                                  {"gemm_swab": 2},
+                                  {"gemm_swab": 2}, {"decode_round_split": 0}, {"fa_poly": 0}, {"fa_poly": 2},
                                   {"dual_stream": 1, "dual_min_prefill": 1, "dual_min_decode": 1}])
 def test_execution_options_do_not_change_results(opts):
     """qos_engine_set_option variants (serial attention, no split-K, two-stream sub-batches)
@@ -224,7 +224,8 @@ def test_execution_options_do_not_change_results(opts):
         assert row_rel_err(lg, ref) <= TOL_LOGITS
     with pytest.raises(q.QosError):
         eng.qos_engine_set_option("no_such_option", 1)
-    eng.qos_engine_set_option("pdl", 1)  # process-wide: restore the default
+    eng.qos_engine_set_option("pdl", 1)  # process-wide: restore the defaults
+    eng.qos_engine_set_option("fa_poly", 4)
     eng.close()
 
 
