@@ -34,8 +34,9 @@ int qos_op_gemm(const void* A, const void* B, void* C, int64_t M, int64_t N, int
 /* Same with an explicit kernel choice:
  *   ksplit = 0   automatic: the weight-streaming kernel when N % 128 == 0 and M <= 16, or
  *                M <= 32 with fewer output tiles of 128 than SMs, or M <= 256 with fewer than
- *                SMs/4 tiles (env QOS_GEMM_SWAB=0 disables it), else the tile kernel with
- *                automatic split-K;
+ *                SMs/4 tiles (env QOS_GEMM_SWAB=0 disables it), else the CTA-pair kernel
+ *                when N % 256 == 0 and 128 x 256 tiles fill the SMs (env QOS_GEMM_2CTA=0
+ *                disables it), else the tile kernel with automatic split-K;
  *   ksplit >= 1  the tile kernel (128-token x 128/256-feature tiles) with that split-K factor:
  *                each of `ksplit` CTAs accumulates a K slice of a tile, parks an fp32 partial,
  *                and the last one to arrive sums the slices in slice order (deterministic);
@@ -48,7 +49,10 @@ int qos_op_gemm(const void* A, const void* B, void* C, int64_t M, int64_t N, int
  *                tile as W_tile(128 rows) · A^T on tcgen05 (token count = UMMA N), the
  *                (tile, k-block) space split in equal contiguous ranges over the SMs
  *                ("stream-K"); tiles cut by a range boundary are summed by their last
- *                arriving CTA in CTA order (deterministic). */
+ *                arriving CTA in CTA order (deterministic).
+ *   ksplit = -3  the CTA-pair kernel (requires N % 256 == 0): clusters of 2 CTAs on 2 SMs,
+ *                256 x 256 tiles, UMMA M = 256 (tcgen05 cta_group::2); each CTA stages its
+ *                128 rows of A and 128 of the tile's 256 rows of B, no split-K. */
 int qos_op_gemm_ex(const void* A, const void* B, void* C, int64_t M, int64_t N, int64_t K, int epi,
                    const float* bias, int ksplit, void* stream);
 

@@ -28,23 +28,32 @@
 
 namespace qos {
 
-template <int HD>
+// NQ = q tiles per CTA.  Both share every K/V tile.
+//   NQ = 1: 2 CTAs per SM: Q + 2-stage K and V rings (96 KB at HD 128) and 256 TMEM columns
+//           each (two 64-column S/P buffers + the O accumulator).
+//   NQ = 2: 1 CTA per SM, 8 softmax warps (one group of 4 per q tile): Q0, Q1 + 4-stage K and
+//           V rings (192 KB), 512 TMEM columns (S/P double buffer and O per q tile).  Each K/V
+//           tile feeds 256 query rows, halving the L2 -> SM traffic per FLOP, and the deeper
+//           ring covers the L2 latency (with NQ = 1 the MMA-only and QK-only variants run as
+//           long as the full kernel: the 2-deep K/V feed, not the tensor core, bounds it).
+// With two S buffers per q tile the MMA warp issues QK of tile j+1 before PV of tile j, so a
+// softmax group never waits on its own PV.
+template <int HD, int NQ>
 struct FaCfg {
   static constexpr int kRows = 128;                  // Q-tile rows (UMMA M)
   static constexpr int kKeys = 64;                   // keys per K/V tile (4 paged blocks)
   static constexpr int kHalves = HD / 64;
   static constexpr int kQBytes = kRows * HD * 2;     // 32 KB at HD 128
   static constexpr int kTileBytes = kKeys * HD * 2;  // one K or V tile
-  // 2 CTAs per SM: Q + 2-stage K and V rings (96 KB at HD 128) and 256 TMEM columns each
-  // (two 64-column S/P buffers + the O accumulator).  With two S buffers the MMA warp issues
-  // QK of tile j+1 before PV of tile j, so the softmax never waits on its own PV.
-  static constexpr int kStages = 2;
-  static constexpr int kSmem = kQBytes + 2 * kStages * kTileBytes + 1024 + 256;
-  static constexpr uint32_t kColS0 = 0, kColS1 = 64, kColO = 128;
-  static constexpr uint32_t kTmemCols = 256;
+  static constexpr int kStages = NQ == 1 ? 2 : 4;
+  static constexpr int kSmem = NQ * kQBytes + 2 * kStages * kTileBytes + 1024 + 512;
+  static constexpr int kThreads = 64 + NQ * 128;
+  static constexpr int kMinBlocks = NQ == 1 ? 2 : 1;
+  // TMEM columns: S/P buffer b of q tile g at g*128 + b*64, O of q tile g at NQ*128 + g*128
+  static constexpr uint32_t kTmemCols = NQ * 256;
+  static constexpr uint32_t col_s(int g, int b) { return uint32_t(g * 128 + b * 64); }
+  static constexpr uint32_t col_o(int g) { return uint32_t(NQ * 128 + g * 128); }
 };
-
-constexpr int kFaThreads = 192;
 
 QOS_DEV void tmem_st32x32b_x16(uint32_t taddr, const uint32_t (&r)[16]) {
   asm volatile(
@@ -142,53 +151,62 @@ struct FaParams {
   float scale_log2;
 };
 
-template <int HD, int POLY>
-__global__ void __launch_bounds__(kFaThreads, 2)
+// Work item = NQ consecutive entries of `items`: q tiles of one (chunk, kv head) that share
+// grp_last (the host pads a short group with a duplicate that stores nothing).
+template <int HD, int POLY, int NQ>
+__global__ void __launch_bounds__(FaCfg<HD, NQ>::kThreads, FaCfg<HD, NQ>::kMinBlocks)
     prefill_attn_tc_kernel(const __grid_constant__ CUtensorMap kvmap, const FaParams p,
                            const PrefillItem* __restrict__ items) {
-  using C = FaCfg<HD>;
+  using C = FaCfg<HD, NQ>;
+  constexpr int S = C::kStages;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  uint8_t* sQ = smem;
-  uint8_t* sK = smem + C::kQBytes;
-  uint8_t* sV = sK + C::kStages * C::kTileBytes;
-  uint64_t* bar = reinterpret_cast<uint64_t*>(sV + C::kStages * C::kTileBytes);
-  uint64_t* k_full = bar + 0;
-  uint64_t* k_empty = bar + 2;
-  uint64_t* v_full = bar + 4;
-  uint64_t* v_empty = bar + 6;
-  uint64_t* s_full = bar + 8;
-  uint64_t* p_full = bar + 10;
-  uint64_t* o_full = bar + 12;
-  uint64_t* o_final = bar + 13;   // completes once, when the last PV has landed
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 14);
+  uint8_t* sQ = smem;                          // NQ x kQBytes
+  uint8_t* sK = smem + NQ * C::kQBytes;
+  uint8_t* sV = sK + S * C::kTileBytes;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(sV + S * C::kTileBytes);
+  uint64_t* k_full = bar;
+  uint64_t* k_empty = k_full + S;
+  uint64_t* v_full = k_empty + S;
+  uint64_t* v_empty = v_full + S;
+  uint64_t* s_full = v_empty + S;        // [NQ][2]
+  uint64_t* p_full = s_full + 2 * NQ;    // [NQ][2]
+  uint64_t* o_full = p_full + 2 * NQ;    // [NQ]
+  uint64_t* o_final = o_full + NQ;       // [NQ] completes once, when the last PV has landed
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(o_final + NQ);
 
-  const PrefillItem it = items[blockIdx.x];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const PrefillItem it0 = items[blockIdx.x * NQ];
   const int group = p.H / p.Hkv;
   const int ppt = C::kRows / group;  // positions per tile
-  const int last_pos = it.pos0 + it.npos - 1;
+  const int last_pos = it0.grp_last;  // over the NQ q tiles
   const int ntiles = last_pos / C::kKeys + 1;
   const int last_blk = last_pos >> 4;
 
   if (threadIdx.x == 0) {
-    for (int i = 0; i < 2; ++i) {
+    for (int i = 0; i < S; ++i) {
       mbar_init(&k_full[i], 1);
       mbar_init(&k_empty[i], 1);
       mbar_init(&v_full[i], 1);
       mbar_init(&v_empty[i], 1);
-      mbar_init(&s_full[i], 1);
-      mbar_init(&p_full[i], 128);
     }
-    mbar_init(o_full, 1);
-    mbar_init(o_final, 1);
+    for (int g = 0; g < NQ; ++g) {
+      for (int b = 0; b < 2; ++b) {
+        mbar_init(&s_full[g * 2 + b], 1);
+        mbar_init(&p_full[g * 2 + b], 128);
+      }
+      mbar_init(&o_full[g], 1);
+      mbar_init(&o_final[g], 1);
+    }
     fence_mbar_init();
   }
   if (warp == 1) tmem_alloc<C::kTmemCols>(tmem_slot);
   griddep_wait();  // q and the appended K/V come from the previous kernel
   griddep_launch_dependents();
 
-  // ---- Q tile -> smem (softmax warps; one row per thread), K-major 128-B swizzle
+  // ---- Q tiles -> smem (softmax group g = (warp - 2) / 4; one row per thread), K-major 128-B swizzle
+  const int qg = warp >= 2 ? (warp - 2) >> 2 : 0;
+  const PrefillItem it = items[blockIdx.x * NQ + qg];
   int row = 0, pos_r = -1;
   size_t tok_off = 0;
   if (warp >= 2) {
@@ -198,13 +216,14 @@ __global__ void __launch_bounds__(kFaThreads, 2)
     pos_r = ok ? it.pos0 + pi : -1;
     tok_off = size_t(it.row0 + pi) * p.out_ld + size_t(it.kv_head * group + hh) * HD;
     const __nv_bfloat16* src = p.q + size_t(it.row0 + pi) * p.q_ld + size_t(it.kv_head * group + hh) * HD;
+    uint8_t* q_dst = sQ + qg * C::kQBytes;
     uint4 v[HD / 8];
 #pragma unroll
     for (int ch = 0; ch < HD / 8; ++ch) v[ch] = ok ? *reinterpret_cast<const uint4*>(src + ch * 8) : make_uint4(0, 0, 0, 0);
 #pragma unroll
     for (int ch = 0; ch < HD / 8; ++ch) {
       const int hf = ch >> 3, c = ch & 7;
-      *reinterpret_cast<uint4*>(sQ + hf * (C::kRows * 128) + row * 128 + ((c ^ (row & 7)) << 4)) = v[ch];
+      *reinterpret_cast<uint4*>(q_dst + hf * (C::kRows * 128) + row * 128 + ((c ^ (row & 7)) << 4)) = v[ch];
     }
     fence_proxy_async_smem();
   }
@@ -217,19 +236,19 @@ __global__ void __launch_bounds__(kFaThreads, 2)
     // ------------------------------------------------------------------ TMA producer
     if (elect_one()) {
       tma_prefetch_desc(&kvmap);
-      const int32_t* trow = p.tables + size_t(it.table) * p.table_w;
+      const int32_t* trow = p.tables + size_t(it0.table) * p.table_w;
       auto load_tile = [&](uint8_t* dst, uint64_t* full, int j, int plane) {
         for (int b = 0; b < C::kKeys / 16; ++b) {
           const int blk = min(j * (C::kKeys / 16) + b, last_blk);  // past the causal end: a valid block (P = 0)
-          const int r = (__ldg(trow + blk) * p.Hkv + it.kv_head) * 16;
+          const int r = (__ldg(trow + blk) * p.Hkv + it0.kv_head) * 16;
 #pragma unroll
           for (int hf = 0; hf < C::kHalves; ++hf)
             tma_load_3d(dst + hf * (C::kKeys * 128) + b * 2048, &kvmap, full, hf * 64, r, p.layer * 2 + plane);
         }
       };
       for (int j = 0; j < ntiles; ++j) {
-        const int s = j & 1;
-        const uint32_t ph = (j >> 1) & 1;
+        const int s = j % S;
+        const uint32_t ph = (j / S) & 1;
         mbar_wait(&k_empty[s], ph ^ 1);
         mbar_arrive_expect_tx(&k_full[s], C::kTileBytes);
         load_tile(sK + s * C::kTileBytes, &k_full[s], j, 0);
@@ -244,62 +263,66 @@ __global__ void __launch_bounds__(kFaThreads, 2)
       constexpr uint32_t idesc_qk = umma_idesc_bf16(128, C::kKeys);
       // P.V in fp16 (A = P in TMEM, B = V cached in fp16, MN-major): formats a/b = f16 (0)
       constexpr uint32_t idesc_pv = (1u << 4) | (1u << 16) | ((uint32_t(HD) >> 3) << 17) | ((128u >> 4) << 24);
-      const uint32_t q_base = smem_u32(sQ);
       auto issue_pv = [&](int t) {
-        const int s = t & 1;
-        const uint32_t ph = (t >> 1) & 1;
-        mbar_wait(&p_full[s], ph);
-        mbar_wait(&v_full[s], ph);
-        tc_fence_after();
+        const int s = t % S;
+        mbar_wait(&v_full[s], (t / S) & 1);
         const uint32_t v_base = smem_u32(sV + s * C::kTileBytes);
-        const uint32_t p_tmem = tmem + (s ? C::kColS1 : C::kColS0);
+        for (int g = 0; g < NQ; ++g) {
+          mbar_wait(&p_full[g * 2 + (t & 1)], (t >> 1) & 1);
+          tc_fence_after();
+          const uint32_t p_tmem = tmem + C::col_s(g, t & 1);
 #pragma unroll
-        for (int kk = 0; kk < C::kKeys / 16; ++kk) {
-          const uint64_t vd = umma_desc_sw128_mn(v_base + kk * 2048, C::kKeys * 128);
-          const uint32_t pc = p_tmem + (kk >> 1) * 32 + (kk & 1) * 8;
-          umma_bf16_ts(tmem + C::kColO, pc, vd, idesc_pv, (t | kk) != 0);
+          for (int kk = 0; kk < C::kKeys / 16; ++kk) {
+            const uint64_t vd = umma_desc_sw128_mn(v_base + kk * 2048, C::kKeys * 128);
+            const uint32_t pc = p_tmem + (kk >> 1) * 32 + (kk & 1) * 8;
+            if (POLY != -2) umma_bf16_ts(tmem + C::col_o(g), pc, vd, idesc_pv, (t | kk) != 0);
+          }
+          umma_commit(&o_full[g]);
         }
-        umma_commit(o_full);
         umma_commit(&v_empty[s]);
       };
       for (int j = 0; j < ntiles; ++j) {
-        // S_j = Q K_j^T into S[j%2]; its previous tenant P_{j-2} was consumed by PV_{j-2},
-        // which is issued before this point (tcgen05 ops execute in issue order)
-        const int s = j & 1;
-        const uint32_t ph = (j >> 1) & 1;
-        mbar_wait(&k_full[s], ph);
+        // S_g(j) = Q_g K_j^T into S buffer j%2 of q tile g; its previous tenant P_g(j-2) was
+        // consumed by PV(j-2), issued before this point (tcgen05 ops execute in issue order)
+        const int s = j % S;
+        mbar_wait(&k_full[s], (j / S) & 1);
         tc_fence_after();
         const uint32_t k_base = smem_u32(sK + s * C::kTileBytes);
-        const uint32_t s_tmem = tmem + (s ? C::kColS1 : C::kColS0);
+        for (int g = 0; g < NQ; ++g) {
+          const uint32_t q_base = smem_u32(sQ + g * C::kQBytes);
+          const uint32_t s_tmem = tmem + C::col_s(g, j & 1);
 #pragma unroll
-        for (int ks = 0; ks < HD / 16; ++ks) {
-          const uint32_t qoff = (ks >> 2) * (C::kRows * 128) + (ks & 3) * 32;
-          const uint32_t koff = (ks >> 2) * (C::kKeys * 128) + (ks & 3) * 32;
-          umma_bf16(s_tmem, umma_desc_sw128(q_base + qoff), umma_desc_sw128(k_base + koff), idesc_qk, ks != 0);
+          for (int ks = 0; ks < HD / 16; ++ks) {
+            const uint32_t qoff = (ks >> 2) * (C::kRows * 128) + (ks & 3) * 32;
+            const uint32_t koff = (ks >> 2) * (C::kKeys * 128) + (ks & 3) * 32;
+            if (POLY != -3) umma_bf16(s_tmem, umma_desc_sw128(q_base + qoff), umma_desc_sw128(k_base + koff), idesc_qk, ks != 0);
+          }
+          umma_commit(&s_full[g * 2 + (j & 1)]);
         }
-        umma_commit(&s_full[s]);
         umma_commit(&k_empty[s]);
-        if (j >= 1) issue_pv(j - 1);   // O += P_{j-1} V_{j-1} while the softmax works on S_j
+        if (j >= 1) issue_pv(j - 1);   // O += P(j-1) V(j-1) while the softmax works on S(j)
       }
       issue_pv(ntiles - 1);
-      umma_commit(o_final);
+      for (int g = 0; g < NQ; ++g) umma_commit(&o_final[g]);
     }
   } else {
-    // ------------------------------------------------------------------ softmax (warps 2..5)
+    // ------------------------------------------------------------------ softmax (group qg)
     const uint32_t lane_base = tmem + (uint32_t((warp & 3) * 32) << 16);
-    const uint32_t o_addr = tmem + (uint32_t((warp & 3) * 32) << 16) + C::kColO;
+    const uint32_t o_addr = lane_base + C::col_o(qg);
+    uint64_t* my_s_full = s_full + qg * 2;
+    uint64_t* my_p_full = p_full + qg * 2;
     const int warp_min_pos = __shfl_sync(0xffffffffu, pos_r < 0 ? INT_MAX : pos_r, 0);  // row 0 of the warp
     float m_used = -INFINITY, l = 0.f;
     for (int j = 0; j < ntiles; ++j) {
       const int sb = j & 1;
-      mbar_wait(&s_full[sb], (j >> 1) & 1);
+      mbar_wait(&my_s_full[sb], (j >> 1) & 1);
       tc_fence_after();
-      if (POLY < 0) {  // measurement-only variant: MMA + TMA pipeline without the softmax
+      if (POLY < 0) {  // measurement-only variants: MMA + TMA pipeline without the softmax
         tc_fence_before();
-        mbar_arrive(&p_full[sb]);
+        mbar_arrive(&my_p_full[sb]);
         continue;
       }
-      const uint32_t s_addr = lane_base + (sb ? C::kColS1 : C::kColS0);
+      const uint32_t s_addr = lane_base + C::col_s(qg, sb);
       const int key0 = j * C::kKeys;
       // masking only where a key of this tile can exceed a row's position
       const bool masked = __any_sync(0xffffffffu, key0 + C::kKeys - 1 > (pos_r < 0 ? -1 : pos_r)) ||
@@ -357,53 +380,53 @@ __global__ void __launch_bounds__(kFaThreads, 2)
       tmem_st_wait();
       l = l * alpha + sum;
       if (j >= 1 && __any_sync(0xffffffffu, alpha != 1.f)) {
-        // rescale O (tiles < j) before PV_j accumulates into it.  Wait for PV_{j-1} only here:
-        // PV_{j-2} was issued before QK_j, whose completion was awaited above, so o_full is at
+        // rescale O (tiles < j) before PV(j) accumulates into it.  Wait for PV(j-1) only here:
+        // PV(j-2) was issued before QK(j), whose completion was awaited above, so o_full is at
         // phase j-1 or j and this parity wait cannot alias.
-        mbar_wait(o_full, (j - 1) & 1);
+        mbar_wait(&o_full[qg], (j - 1) & 1);
         tc_fence_after();
 #pragma unroll 1
         for (int c = 0; c < HD / 16; ++c) {
-          uint32_t r[16];
-          tmem_ld32x32b_x16(o_addr + c * 16, r);
+          uint32_t r2[16];
+          tmem_ld32x32b_x16(o_addr + c * 16, r2);
           tmem_ld_wait();
 #pragma unroll
-          for (int i = 0; i < 16; ++i) r[i] = __float_as_uint(__uint_as_float(r[i]) * alpha);
-          tmem_st32x32b_x16(o_addr + c * 16, r);
+          for (int i = 0; i < 16; ++i) r2[i] = __float_as_uint(__uint_as_float(r2[i]) * alpha);
+          tmem_st32x32b_x16(o_addr + c * 16, r2);
         }
         tmem_st_wait();
       }
       m_used = m_new;
       tc_fence_before();
-      mbar_arrive(&p_full[sb]);
+      mbar_arrive(&my_p_full[sb]);
     }
     // epilogue: O / l
     // o_full may be anywhere in phases n-2..n here (its waits are skipped when no rescale is
     // needed), so a parity wait on it could alias; the dedicated o_final barrier completes once
-    mbar_wait(o_final, 0);
+    mbar_wait(&o_final[qg], 0);
     tc_fence_after();
     const float inv = (l > 0.f) ? 1.f / l : 0.f;
 #pragma unroll 1
     for (int c = 0; c < HD / 32; ++c) {
-      uint32_t r[32];
-      tmem_ld32x32b_x16(o_addr + c * 32, *reinterpret_cast<uint32_t(*)[16]>(&r[0]));
-      tmem_ld32x32b_x16(o_addr + c * 32 + 16, *reinterpret_cast<uint32_t(*)[16]>(&r[16]));
+      uint32_t r2[32];
+      tmem_ld32x32b_x16(o_addr + c * 32, *reinterpret_cast<uint32_t(*)[16]>(&r2[0]));
+      tmem_ld32x32b_x16(o_addr + c * 32 + 16, *reinterpret_cast<uint32_t(*)[16]>(&r2[16]));
       tmem_ld_wait();
-      if (pos_r >= 0) {
+      if (pos_r >= 0 && !it.pad) {
         if (p.out_f32) {
           float4* dst = reinterpret_cast<float4*>(reinterpret_cast<float*>(p.out) + tok_off + c * 32);
 #pragma unroll
           for (int i = 0; i < 8; ++i)
-            dst[i] = make_float4(__uint_as_float(r[4 * i]) * inv, __uint_as_float(r[4 * i + 1]) * inv,
-                                 __uint_as_float(r[4 * i + 2]) * inv, __uint_as_float(r[4 * i + 3]) * inv);
+            dst[i] = make_float4(__uint_as_float(r2[4 * i]) * inv, __uint_as_float(r2[4 * i + 1]) * inv,
+                                 __uint_as_float(r2[4 * i + 2]) * inv, __uint_as_float(r2[4 * i + 3]) * inv);
         } else {
           uint4* dst = reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.out) + tok_off + c * 32);
 #pragma unroll
           for (int i = 0; i < 4; ++i)
-            dst[i] = make_uint4(pack_bf16(__uint_as_float(r[8 * i]) * inv, __uint_as_float(r[8 * i + 1]) * inv),
-                                pack_bf16(__uint_as_float(r[8 * i + 2]) * inv, __uint_as_float(r[8 * i + 3]) * inv),
-                                pack_bf16(__uint_as_float(r[8 * i + 4]) * inv, __uint_as_float(r[8 * i + 5]) * inv),
-                                pack_bf16(__uint_as_float(r[8 * i + 6]) * inv, __uint_as_float(r[8 * i + 7]) * inv));
+            dst[i] = make_uint4(pack_bf16(__uint_as_float(r2[8 * i]) * inv, __uint_as_float(r2[8 * i + 1]) * inv),
+                                pack_bf16(__uint_as_float(r2[8 * i + 2]) * inv, __uint_as_float(r2[8 * i + 3]) * inv),
+                                pack_bf16(__uint_as_float(r2[8 * i + 4]) * inv, __uint_as_float(r2[8 * i + 5]) * inv),
+                                pack_bf16(__uint_as_float(r2[8 * i + 6]) * inv, __uint_as_float(r2[8 * i + 7]) * inv));
         }
       }
     }
@@ -418,12 +441,13 @@ __global__ void __launch_bounds__(kFaThreads, 2)
 
 static int g_fa_poly = getenv("QOS_FA_POLY") ? atoi(getenv("QOS_FA_POLY")) : 4;
 
-template <int HD, int POLY>
+template <int HD, int POLY, int NQ>
 static cudaError_t prefill_tc_t(const AttnLaunch& a, const PrefillItem* items, int n_items, cudaStream_t st) {
+  using C = FaCfg<HD, NQ>;
   static bool set = false;
   if (!set) {
-    cudaError_t e = cudaFuncSetAttribute(prefill_attn_tc_kernel<HD, POLY>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         FaCfg<HD>::kSmem);
+    cudaError_t e = cudaFuncSetAttribute(prefill_attn_tc_kernel<HD, POLY, NQ>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         C::kSmem);
     if (e != cudaSuccess) return e;
     set = true;
   }
@@ -439,8 +463,9 @@ static cudaError_t prefill_tc_t(const AttnLaunch& a, const PrefillItem* items, i
   p.tables = a.tables;
   p.table_w = a.table_w;
   p.scale_log2 = a.scale_log2;
-  return launch_pdl(prefill_attn_tc_kernel<HD, POLY>, dim3(n_items), dim3(kFaThreads), FaCfg<HD>::kSmem, st, *a.kv_tmap, p,
-                    items);
+  if (n_items % NQ) return cudaErrorInvalidValue;  // the item list comes in whole groups
+  return launch_pdl(prefill_attn_tc_kernel<HD, POLY, NQ>, dim3(n_items / NQ), dim3(C::kThreads), C::kSmem, st,
+                    *a.kv_tmap, p, items);
 }
 
 void set_fa_poly(int n) { g_fa_poly = n; }
@@ -451,18 +476,24 @@ cudaError_t launch_prefill_attention_tc(const AttnLaunch& a, const PrefillItem* 
   if (n_items == 0) return cudaSuccess;
   count_launch(1);
   const int poly = g_fa_poly;
+  const int nq = a.q_tiles;
+  if (nq != 1 && nq != 2) return cudaErrorInvalidValue;
+#define QOS_FA_NQ(HDV, PV) \
+  return nq == 1 ? prefill_tc_t<HDV, PV, 1>(a, items, n_items, st) : prefill_tc_t<HDV, PV, 2>(a, items, n_items, st);
   if (a.hd == 128) {
-    if (poly == 0) return prefill_tc_t<128, 0>(a, items, n_items, st);
-    if (poly < 0) return prefill_tc_t<128, -1>(a, items, n_items, st);
-    if (poly == 2) return prefill_tc_t<128, 2>(a, items, n_items, st);
-    if (poly == 3) return prefill_tc_t<128, 3>(a, items, n_items, st);
-    if (poly == 8) return prefill_tc_t<128, 8>(a, items, n_items, st);
-    return prefill_tc_t<128, 4>(a, items, n_items, st);
+    // measurement-only variants: -1 no softmax, -2 also no P.V MMAs, -3 no softmax and no QK MMAs
+    if (poly == -1) { QOS_FA_NQ(128, -1) }
+    if (poly == -2) { QOS_FA_NQ(128, -2) }
+    if (poly == -3) { QOS_FA_NQ(128, -3) }
+    if (poly == 0) { QOS_FA_NQ(128, 0) }
+    if (poly == 2) { QOS_FA_NQ(128, 2) }
+    QOS_FA_NQ(128, 4)
   }
   if (a.hd == 64) {
-    if (poly == 0) return prefill_tc_t<64, 0>(a, items, n_items, st);
-    return prefill_tc_t<64, 4>(a, items, n_items, st);
+    if (poly == 0) { QOS_FA_NQ(64, 0) }
+    QOS_FA_NQ(64, 4)
   }
+#undef QOS_FA_NQ
   return cudaErrorInvalidValue;
 }
 

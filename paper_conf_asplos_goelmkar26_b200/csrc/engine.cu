@@ -175,7 +175,8 @@ static WsLayout ws_layout(const qos_model_cfg& c, const Shard& s, int tp) {
   w.gemm_cnt2 = take(size_t(kGemmMaxTiles) * 4);
   // metadata: tokens, pos, slot [Tm]; logit rows [Rm]; prefill items; decode items/rows; table updates
   const int ppt = prefill_tc_positions_per_tile(int(group));
-  const size_t max_pitems = (Tm / ppt + Rm + 1) * size_t(s.Hkv);
+  // (+ up to 3 group-filling duplicates per (chunk, kv head))
+  const size_t max_pitems = (Tm / ppt + 4 * (Rm + 1)) * size_t(s.Hkv);
   w.meta_bytes = align_up(3 * Tm * 4 + Rm * 4 + 64, 256) + align_up(max_pitems * sizeof(PrefillItem), 256) +
                  align_up(size_t(w.max_items) * sizeof(DecodeItem), 256) +
                  align_up(size_t(3) * 65536 * 4, 256);
@@ -190,6 +191,7 @@ static WsLayout ws_layout(const qos_model_cfg& c, const Shard& s, int tp) {
 struct StepMeta {
   int T = 0, R = 0, n_prefill = 0, n_decode = 0;
   int n_pitems = 0, n_ditems = 0, n_upd = 0;
+  int fa_qtiles = 1;  // prefill items come in groups of this many q tiles (one CTA each group)
   // offsets (bytes) inside the metadata block
   size_t o_tok, o_pos, o_slot, o_rows, o_pitems, o_ditems, o_upd, used;
 };
@@ -243,7 +245,9 @@ struct qos_engine {
   bool dual_stream = false;       // QOS_DUAL=1: prefill rows and decode rows on two streams
   int dual_min_prefill = 512, dual_min_decode = 16;
   int dual_sms_pre = 0, dual_sms_dec = 0;  // SM budgets of the two streams' GEMMs (0 = all)
+  bool gemm_2cta = true;            // option gemm_2cta: CTA-pair GEMM (256 x 256 tiles) at large M
   bool decode_round_split = true;  // option decode_round_split (A/B of the split-K ranges)
+  int fa_qtiles = 2;                // option fa_qtiles: prefill q tiles per CTA sharing K/V tiles
   bool overlap_attn = true;       // QOS_OVERLAP_ATTN=0 serialises a7 and a8 (for measurement)
   bool gemm_splitk = true;        // QOS_GEMM_SPLITK=0 disables split-K for small-M GEMMs
   int gemm_swab = 1;              // weight-streaming GEMM (gemm_swab.cu): 0 never, 1 auto, 2 always
@@ -402,6 +406,7 @@ int build_step(qos_engine* e, const qos_batch* b, bool check_lengths, uint8_t* b
 
   const int group = c.n_heads / c.n_kv_heads;
   const int ppt = prefill_tc_positions_per_tile(group);
+  const int CS = e->fa_qtiles;
   std::vector<PrefillItem> pitems;
   int t = 0;
   for (int i = 0; i < b->n_prefill; ++i) {
@@ -416,24 +421,46 @@ int build_step(qos_engine* e, const qos_batch* b, bool check_lengths, uint8_t* b
       pos[t + j] = p;
       slot[t + j] = rs->blocks[p >> 4] * 16 + (p & 15);
     }
-    for (int p0 = 0; p0 < ch.chunk_len; p0 += ppt) {
-      for (int h = 0; h < e->sh.Hkv; ++h) {
-        PrefillItem it;
-        it.row0 = t + p0;
-        it.npos = std::min(ppt, ch.chunk_len - p0);
-        it.pos0 = ch.kv_start + p0;
-        it.table = rs->row;
-        it.kv_head = h;
-        it.pad = 0;
-        pitems.push_back(it);
-      }
+    // groups of CS consecutive q tiles of one kv head run in one CTA and share every K/V tile;
+    // a short last group is filled with a duplicate of its last tile that stores nothing
+    const int ntile = (ch.chunk_len + ppt - 1) / ppt;
+    for (int c0 = 0; c0 < ntile; c0 += CS) {
+      const int last_tile = std::min(ntile, c0 + CS) - 1;
+      const int grp_last = ch.kv_start + std::min(ch.chunk_len, (last_tile + 1) * ppt) - 1;
+      for (int h = 0; h < e->sh.Hkv; ++h)
+        for (int k = 0; k < CS; ++k) {
+          const int qt = std::min(c0 + k, last_tile);
+          PrefillItem it;
+          it.row0 = t + qt * ppt;
+          it.npos = std::min(ppt, ch.chunk_len - qt * ppt);
+          it.pos0 = ch.kv_start + qt * ppt;
+          it.table = rs->row;
+          it.kv_head = h;
+          it.pad = c0 + k > last_tile ? 1 : 0;
+          it.grp_last = grp_last;
+          pitems.push_back(it);
+        }
     }
     t += ch.chunk_len;
     rows[i] = t - 1;
   }
-  // LPT: longest key ranges first
-  std::stable_sort(pitems.begin(), pitems.end(),
-                   [](const PrefillItem& a, const PrefillItem& b2) { return a.pos0 + a.npos > b2.pos0 + b2.npos; });
+  // LPT: longest key ranges first, whole groups (the items of a group share grp_last, and the
+  // stable sort keeps them adjacent and in order)
+  if (CS == 1)
+    std::stable_sort(pitems.begin(), pitems.end(),
+                     [](const PrefillItem& a, const PrefillItem& b2) { return a.pos0 + a.npos > b2.pos0 + b2.npos; });
+  else {
+    std::vector<int> order(pitems.size() / CS);
+    for (size_t i = 0; i < order.size(); ++i) order[i] = int(i);
+    std::stable_sort(order.begin(), order.end(),
+                     [&](int a, int b2) { return pitems[size_t(a) * CS].grp_last > pitems[size_t(b2) * CS].grp_last; });
+    std::vector<PrefillItem> sorted;
+    sorted.reserve(pitems.size());
+    for (int g2 : order)
+      for (int k = 0; k < CS; ++k) sorted.push_back(pitems[size_t(g2) * CS + k]);
+    pitems.swap(sorted);
+  }
+  m.fa_qtiles = CS;
   // decode split-K work list (balanced on sum of keys)
   int64_t total_keys = 0;
   for (int i = 0; i < b->n_decode; ++i) total_keys += int64_t(b->decode[i].ctx_len) + 1;
@@ -567,6 +594,8 @@ int gemm_any(qos_engine* e, const qos_engine::ActMap& am, const CUtensorMap (&tb
     return gemm_swab_run(tb[0], am.sw[swab_index(bnt)], bnt, M, N, K, epi, C, ldc, bias, sms, st, part, cnt,
                          int64_t(kGemmMaxUnits) * 128 * 256, kGemmMaxTiles, a_row0, rope, !e->dual_stream);
   }
+  if (e->gemm_2cta && gemm2_eligible(M, N, K, sms))
+    return gemm2_run(am.m128, tb[0], M, N, K, epi, C, ldc, bias, sms, st, a_row0, sms, rope);
   const int bn = gemm_pick_bn(M, N, epi, sms);
   const int ks = e->gemm_splitk ? gemm_pick_ksplit(M, N, K, bn, sms, kGemmMaxUnits) : 1;
   return gemm_run(am.m128, tb[bn == 256 ? 1 : 0], bn, M, N, K, epi, C, ldc, bias, sms, st, ks, part, cnt, a_row0, sms,
@@ -642,6 +671,7 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
   al.tables = e->d_tables;
   al.table_w = e->table_w;
   al.scale_log2 = float(1.4426950408889634 / std::sqrt(double(hd)));
+  al.q_tiles = m.fa_qtiles;
   const int n_pre_rows = T - m.n_decode;
   float* gpart0 = reinterpret_cast<float*>(e->ws + s.gemm_part);
   int* gcnt0 = reinterpret_cast<int*>(e->ws + s.gemm_cnt);
@@ -1296,6 +1326,11 @@ int qos_engine_set_option(qos_engine_t* e, const char* name, int64_t value) {
   const std::string n(name);
   if (n == "overlap_attn") e->overlap_attn = value != 0;
   else if (n == "decode_round_split") e->decode_round_split = value != 0;
+  else if (n == "gemm_2cta") e->gemm_2cta = value != 0;
+  else if (n == "fa_qtiles") {
+    if (value != 1 && value != 2) return set_error(QOS_ERR_INVALID_ARG, "fa_qtiles must be 1 or 2");
+    e->fa_qtiles = int(value);
+  }
   else if (n == "gemm_splitk") e->gemm_splitk = value != 0;
   else if (n == "pdl") set_pdl(value != 0);  // process-wide
   else if (n == "fa_poly") set_fa_poly(int(value));  // process-wide
@@ -1378,6 +1413,16 @@ static int op_gemm(const void* A, const void* B, void* C, int64_t M, int64_t N, 
     count_launch();
     return gemm_swab_run(tw, tt, bnt, M, N, K, epi, C, ldc, bias, sms, reinterpret_cast<cudaStream_t>(stream), part,
                          cnt, int64_t(kGemmMaxUnits) * 128 * 256, kGemmMaxTiles, 0, nullptr);
+  }
+  static const bool g2_env = !(getenv("QOS_GEMM_2CTA") && atoi(getenv("QOS_GEMM_2CTA")) == 0);
+  if (ksplit == -3 || (ksplit == 0 && g2_env && gemm2_eligible(M, N, K, sms))) {
+    // CTA-pair kernel (256 x 256 tiles)
+    if (N % 256) return set_error(QOS_ERR_UNSUPPORTED, "gemm: the CTA-pair kernel needs N % 256 == 0");
+    CUtensorMap ta, tb;
+    QOS_TRY(make_tmap_2d_bf16(&ta, A, uint64_t(M), uint64_t(K), uint64_t(K), 128, 64, true));
+    QOS_TRY(make_tmap_2d_bf16(&tb, B, uint64_t(N), uint64_t(K), uint64_t(K), 128, 64, true));
+    count_launch();
+    return gemm2_run(ta, tb, M, N, K, epi, C, ldc, bias, sms, reinterpret_cast<cudaStream_t>(stream), 0, 0, nullptr);
   }
   const int64_t tiles = ((M + 127) / 128) * ((N + bn - 1) / bn);
   const int sk_mode = ksplit <= -2 ? 2 : 0;
@@ -1514,6 +1559,7 @@ int qos_op_attention(qos_engine_t* e, int32_t layer, const qos_batch* b, const u
   al.tables = e->d_tables;
   al.table_w = e->table_w;
   al.scale_log2 = float(1.4426950408889634 / std::sqrt(double(hd)));
+  al.q_tiles = m.fa_qtiles;
   QOS_CU(launch_prefill_attention_tc(al, reinterpret_cast<const PrefillItem*>(dm + m.o_pitems), m.n_pitems, st));
   QOS_CU(launch_decode_attention(al, reinterpret_cast<const DecodeItem*>(dm + m.o_ditems), m.n_ditems,
                                  reinterpret_cast<float*>(e->ws + e->wsl.partials),

@@ -16,6 +16,7 @@
 //     one time share a weight (B) tile and the activation matrix stays L2-resident.
 #include <cudaTypedefs.h>
 
+#include <algorithm>
 #include <cstdio>
 #include <cstdlib>
 
@@ -338,6 +339,81 @@ QOS_DEV void tmem_ld32(uint32_t taddr, float (&v)[32]) {
 
 QOS_DEV void epi_bar_sync() { asm volatile("bar.sync 1, 128;" ::: "memory"); }  // the 4 epilogue warps
 
+// Whole tile straight from TMEM, staged through smem (coalesced stores).  Thread = one
+// accumulator row (`row`, the warp's rows start at row - lane); tbase = this warp's TMEM lane
+// quarter + the accumulator's first column; n_t = the tile's BN-wide column block.
+template <int BN, int EPI>
+QOS_DEV void epi_tile_staged(const GemmArgs& p, uint8_t* stg, int lane, int n_t, int row, uint32_t tbase) {
+        const int row0 = row - lane;
+        if constexpr (EPI == EPI_QKV_ROPE) {
+          epi_qkv_rope_staged<BN>(p, stg, lane, row0, n_t, [&](int col, float (&v)[16]) {
+            uint32_t r[16];
+            tmem_ld32x32b_x16(tbase + col, r);
+            tmem_ld_wait();
+#pragma unroll
+            for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]) + (p.bias ? __ldg(p.bias + n_t * BN + col + i) : 0.f);
+          });
+        } else if constexpr (EPI == EPI_SILU_GATE) {
+#pragma unroll 1
+          for (int g = 0; g < BN / 128; ++g) {
+#pragma unroll 1
+            for (int h = 0; h < 2; ++h) {
+              float gv[32], uv[32];
+              tmem_ld32(tbase + g * 128 + h * 32, gv);
+              tmem_ld32(tbase + g * 128 + 64 + h * 32, uv);
+              const int col = n_t * (BN / 2) + g * 64 + h * 32;
+              if (col >= p.N / 2) continue;  // warp-uniform
+              uint32_t pk[16];
+#pragma unroll
+              for (int i = 0; i < 16; ++i) pk[i] = pack_bf16(silu(gv[2 * i]) * uv[2 * i], silu(gv[2 * i + 1]) * uv[2 * i + 1]);
+#pragma unroll
+              for (int k = 0; k < 4; ++k) stg_put<64>(stg, lane, k, make_uint4(pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]));
+              stg_flush<64>(stg, lane, [&](int rr, int k, uint4 v) {
+                if (row0 + rr < p.M)
+                  reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.C) + size_t(row0 + rr) * p.ldc + col)[k] = v;
+              });
+            }
+          }
+        } else {
+#pragma unroll 1
+          for (int c = 0; c < BN / 32; ++c) {
+            float v[32];
+            tmem_ld32(tbase + c * 32, v);
+            const int col = n_t * BN + c * 32;
+            if (col >= p.N) continue;  // warp-uniform (N % 32 == 0)
+            if constexpr (EPI == EPI_STORE_BF16 || EPI == EPI_BIAS_BF16) {
+              uint32_t pk[16];
+#pragma unroll
+              for (int i = 0; i < 16; ++i) {
+                float a0 = v[2 * i], a1 = v[2 * i + 1];
+                if constexpr (EPI == EPI_BIAS_BF16) {
+                  a0 += __ldg(p.bias + col + 2 * i);
+                  a1 += __ldg(p.bias + col + 2 * i + 1);
+                }
+                pk[i] = pack_bf16(a0, a1);
+              }
+#pragma unroll
+              for (int k = 0; k < 4; ++k) stg_put<64>(stg, lane, k, make_uint4(pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]));
+              stg_flush<64>(stg, lane, [&](int rr, int k, uint4 x) {
+                if (row0 + rr < p.M)
+                  reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.C) + size_t(row0 + rr) * p.ldc + col)[k] = x;
+              });
+            } else {
+#pragma unroll
+              for (int k = 0; k < 8; ++k)
+                stg_put<128>(stg, lane, k, make_uint4(__float_as_uint(v[4 * k]), __float_as_uint(v[4 * k + 1]),
+                                                      __float_as_uint(v[4 * k + 2]), __float_as_uint(v[4 * k + 3])));
+              stg_flush<128>(stg, lane, [&](int rr, int k, uint4 x) {
+                if (row0 + rr >= p.M) return;
+                float* d = reinterpret_cast<float*>(p.C) + size_t(row0 + rr) * p.ldc + col + 4 * k;
+                if constexpr (EPI == EPI_ADD_F32) red_add_v4(d, x);  // residual += tile (one add per element)
+                else *reinterpret_cast<uint4*>(d) = x;
+              });
+            }
+          }
+        }
+}
+
 template <int BN, int EPI>
 __global__ void __launch_bounds__(kGemmThreads, 1)
     gemm_tcgen05_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
@@ -525,75 +601,8 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     // whole tile straight from TMEM, staged through smem (coalesced stores); row = this thread's
     // row, row0 = the warp's first row
     auto epi_tmem = [&](int n_t, int row, bool row_ok, uint32_t tbase) {
-        const int row0 = row - lane;
-        (void)row_ok;
-        if constexpr (EPI == EPI_QKV_ROPE) {
-          epi_qkv_rope_staged<BN>(p, stg, lane, row0, n_t, [&](int col, float (&v)[16]) {
-            uint32_t r[16];
-            tmem_ld32x32b_x16(tbase + col, r);
-            tmem_ld_wait();
-#pragma unroll
-            for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]) + (p.bias ? __ldg(p.bias + n_t * BN + col + i) : 0.f);
-          });
-        } else if constexpr (EPI == EPI_SILU_GATE) {
-#pragma unroll 1
-          for (int g = 0; g < BN / 128; ++g) {
-#pragma unroll 1
-            for (int h = 0; h < 2; ++h) {
-              float gv[32], uv[32];
-              tmem_ld32(tbase + g * 128 + h * 32, gv);
-              tmem_ld32(tbase + g * 128 + 64 + h * 32, uv);
-              const int col = n_t * (BN / 2) + g * 64 + h * 32;
-              if (col >= p.N / 2) continue;  // warp-uniform
-              uint32_t pk[16];
-#pragma unroll
-              for (int i = 0; i < 16; ++i) pk[i] = pack_bf16(silu(gv[2 * i]) * uv[2 * i], silu(gv[2 * i + 1]) * uv[2 * i + 1]);
-#pragma unroll
-              for (int k = 0; k < 4; ++k) stg_put<64>(stg, lane, k, make_uint4(pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]));
-              stg_flush<64>(stg, lane, [&](int rr, int k, uint4 v) {
-                if (row0 + rr < p.M)
-                  reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.C) + size_t(row0 + rr) * p.ldc + col)[k] = v;
-              });
-            }
-          }
-        } else {
-#pragma unroll 1
-          for (int c = 0; c < BN / 32; ++c) {
-            float v[32];
-            tmem_ld32(tbase + c * 32, v);
-            const int col = n_t * BN + c * 32;
-            if (col >= p.N) continue;  // warp-uniform (N % 32 == 0)
-            if constexpr (EPI == EPI_STORE_BF16 || EPI == EPI_BIAS_BF16) {
-              uint32_t pk[16];
-#pragma unroll
-              for (int i = 0; i < 16; ++i) {
-                float a0 = v[2 * i], a1 = v[2 * i + 1];
-                if constexpr (EPI == EPI_BIAS_BF16) {
-                  a0 += __ldg(p.bias + col + 2 * i);
-                  a1 += __ldg(p.bias + col + 2 * i + 1);
-                }
-                pk[i] = pack_bf16(a0, a1);
-              }
-#pragma unroll
-              for (int k = 0; k < 4; ++k) stg_put<64>(stg, lane, k, make_uint4(pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]));
-              stg_flush<64>(stg, lane, [&](int rr, int k, uint4 x) {
-                if (row0 + rr < p.M)
-                  reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.C) + size_t(row0 + rr) * p.ldc + col)[k] = x;
-              });
-            } else {
-#pragma unroll
-              for (int k = 0; k < 8; ++k)
-                stg_put<128>(stg, lane, k, make_uint4(__float_as_uint(v[4 * k]), __float_as_uint(v[4 * k + 1]),
-                                                      __float_as_uint(v[4 * k + 2]), __float_as_uint(v[4 * k + 3])));
-              stg_flush<128>(stg, lane, [&](int rr, int k, uint4 x) {
-                if (row0 + rr >= p.M) return;
-                float* d = reinterpret_cast<float*>(p.C) + size_t(row0 + rr) * p.ldc + col + 4 * k;
-                if constexpr (EPI == EPI_ADD_F32) red_add_v4(d, x);  // residual += tile (one add per element)
-                else *reinterpret_cast<uint4*>(d) = x;
-              });
-            }
-          }
-        }
+      (void)row_ok;
+      epi_tile_staged<BN, EPI>(p, stg, lane, n_t, row, tbase);
     };
     if (p.sk) {
       // stream-K: whole tiles straight from TMEM; a tile cut by a range boundary parks one fp32
@@ -808,6 +817,165 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
   }
 }
 
+
+// ------------------------------------------------------------------------------ CTA-pair GEMM
+// cta_group::2 variant for large token counts (the shapes cuBLAS also runs on CTA pairs):
+// a cluster of 2 CTAs on 2 SMs computes a 256 x 256 tile with UMMA M=256 N=256 K=16 issued by
+// CTA 0.  Each CTA stages its own 128 rows of A and its own 128 rows (output columns) of B per
+// k-block (32 KB instead of 48 KB for a 128 x 256 single-CTA tile) and holds the fp32
+// accumulator of its 128 rows x 256 columns in its own TMEM, so per SM the shared-memory
+// traffic (TMA writes + MMA operand reads) per FLOP drops by a third.  The peer CTA's TMA
+// loads complete on the leader's full barrier; the leader's MMA commits arrive on both CTAs'
+// empty / accumulator-full barriers; both CTAs' epilogue warps release an accumulator on the
+// leader's barrier.  No split-K / stream-K: used where 128 x 256 tiles already fill the SMs.
+constexpr int kG2Stages = 6;
+constexpr int kG2Half = 128 * kBK * 2;          // 16 KB: 128 rows x 64 k of A or of B
+constexpr int kG2Stage = 2 * kG2Half;
+constexpr int kG2StageWarpBytes = 32 * 256;
+constexpr int kG2Smem = kG2Stages * kG2Stage + 1024 + 256 + 4 * kG2StageWarpBytes;
+
+template <int EPI>
+__global__ void __launch_bounds__(kGemmThreads, 1)
+    gemm2_tcgen05_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                         const GemmArgs p) {
+  constexpr int S = kG2Stages, BN = 256;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + S * kG2Stage);
+  uint64_t* empty = full + S;
+  uint64_t* tfull = empty + S;
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+  uint8_t* stg_all = smem + S * kG2Stage + 256;
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t rank = cluster_ctarank();
+  const bool leader = rank == 0;
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], 1);
+    }
+    for (int a = 0; a < 2; ++a) {
+      mbar_init(&tfull[a], 1);
+      mbar_init(&tempty[a], 8);  // leader's: 4 epilogue warps of each CTA
+    }
+    fence_mbar_init();
+  }
+  if (warp == 0 && lane == 0) {
+    tma_prefetch_desc(&tmA);
+    tma_prefetch_desc(&tmB);
+  }
+  if (warp == 1) tmem_alloc2<512>(tmem_slot);
+  tc_fence_before();
+  cluster_sync();  // barrier inits and the TMEM address visible pair-wide
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+  griddep_launch_dependents();
+  if (warp != 0) griddep_wait();
+
+  const int pair = blockIdx.x >> 1, npairs = gridDim.x >> 1;
+  const int mt2 = (p.M + 255) / 256;
+  const int num_units = mt2 * p.nt;
+  const int kblocks = p.K / kBK;
+
+  if (warp == 0) {
+    // ------------------------------------------------------------ TMA producer (both CTAs)
+    if (elect_one()) {
+      const uint64_t pol_a = l2_evict_last();
+      const uint64_t pol_b = l2_evict_first();
+      const uint32_t full_leader = mapa_shared(smem_u32(full), 0);
+      int stage = 0;
+      uint32_t phase = 0;
+      int npre = 0;
+      if (pair < num_units) {  // PDL: weight halves of the first stages before the wait
+        const int n_t = pair / mt2;
+        npre = min(S, kblocks);
+        for (int i = 0; i < npre; ++i) {
+          if (leader) mbar_arrive_expect_tx(&full[i], 2 * kG2Stage);
+          tma_load_2d_2cta(smem + i * kG2Stage + kG2Half, &tmB, full_leader + i * 8, i * kBK, n_t * BN + rank * 128, pol_b);
+        }
+        griddep_wait();
+        const int m_t = pair % mt2;
+        for (int i = 0; i < npre; ++i)
+          tma_load_2d_2cta(smem + i * kG2Stage, &tmA, full_leader + i * 8, i * kBK, p.a_row0 + m_t * 256 + rank * 128, pol_a);
+      } else {
+        griddep_wait();
+      }
+      int it = 0;
+      for (int u = pair; u < num_units; u += npairs) {
+        const int m_t = u % mt2, n_t = u / mt2;
+        for (int kb = 0; kb < kblocks; ++kb, ++it) {
+          if (it < npre) {
+            if (++stage == S) { stage = 0; phase ^= 1; }
+            continue;
+          }
+          mbar_wait(&empty[stage], phase ^ 1);
+          if (leader) mbar_arrive_expect_tx(&full[stage], 2 * kG2Stage);
+          uint8_t* sa = smem + stage * kG2Stage;
+          tma_load_2d_2cta(sa, &tmA, full_leader + stage * 8, kb * kBK, p.a_row0 + m_t * 256 + rank * 128, pol_a);
+          tma_load_2d_2cta(sa + kG2Half, &tmB, full_leader + stage * 8, kb * kBK, n_t * BN + rank * 128, pol_b);
+          if (++stage == S) { stage = 0; phase ^= 1; }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ------------------------------------------------------------ MMA issuer (leader only)
+    if (leader && elect_one()) {
+      constexpr uint32_t idesc = umma_idesc_bf16(256, BN);
+      int stage = 0;
+      uint32_t phase = 0;
+      int acc = 0;
+      uint32_t acc_phase = 0;
+      for (int u = pair; u < num_units; u += npairs) {
+        mbar_wait(&tempty[acc], acc_phase ^ 1);
+        tc_fence_after();
+        const uint32_t d_tmem = tmem_base + acc * BN;
+        for (int kb = 0; kb < kblocks; ++kb) {
+          mbar_wait(&full[stage], phase);
+          tc_fence_after();
+          const uint32_t a_base = smem_u32(smem + stage * kG2Stage);
+          const uint32_t b_base = a_base + kG2Half;
+#pragma unroll
+          for (int k = 0; k < kBK / 16; ++k)
+            umma_bf16_2cta(d_tmem, umma_desc_sw128(a_base + k * 32), umma_desc_sw128(b_base + k * 32), idesc,
+                           (kb > 0 || k > 0) ? 1u : 0u);
+          umma_commit_2cta(&empty[stage]);
+          if (++stage == S) { stage = 0; phase ^= 1; }
+        }
+        umma_commit_2cta(&tfull[acc]);
+        if (++acc == 2) { acc = 0; acc_phase ^= 1; }
+      }
+    }
+  } else {
+    // ------------------------------------------------------------ epilogue (both CTAs)
+    const int q = warp & 3;
+    uint8_t* stg = stg_all + q * kG2StageWarpBytes;
+    const uint32_t tempty_leader = mapa_shared(smem_u32(tempty), 0);
+    int acc = 0;
+    uint32_t acc_phase = 0;
+    for (int u = pair; u < num_units; u += npairs) {
+      const int m_t = u % mt2, n_t = u / mt2;
+      mbar_wait(&tfull[acc], acc_phase);
+      tc_fence_after();
+      const int row = m_t * 256 + int(rank) * 128 + q * 32 + lane;
+      epi_tile_staged<BN, EPI>(p, stg, lane, n_t, row, tmem_base + (uint32_t(q * 32) << 16) + acc * BN);
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive_cluster(tempty_leader + acc * 8);
+      if (++acc == 2) { acc = 0; acc_phase ^= 1; }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  cluster_sync();  // the peer's MMAs, commits and remote arrivals are done before TMEM is freed
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc2<512>(tmem_base);
+  }
+}
+
 // ------------------------------------------------------------------------------ host side
 static PFN_cuTensorMapEncodeTiled_v12000 get_encode_fn() {
   static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
@@ -948,6 +1116,73 @@ int gemm_run(const CUtensorMap& ta, const CUtensorMap& tb, int bn, int64_t M, in
   return set_error(QOS_ERR_INVALID_ARG, "gemm: bad tile/epilogue");
 #undef QOS_GEMM_CASE
   if (e != cudaSuccess) return set_cuda_error(e, "gemm launch");
+  return QOS_OK;
+}
+
+template <int EPI>
+static cudaError_t launch_gemm2_t(const CUtensorMap& ta, const CUtensorMap& tb, const GemmArgs& a, int grid,
+                                  cudaStream_t st) {
+  auto kern = gemm2_tcgen05_kernel<EPI>;
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kG2Smem);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  return launch_pdl_cluster(kern, dim3(grid), dim3(kGemmThreads), kG2Smem, 2, st, ta, tb, a);
+}
+
+bool gemm2_eligible(int64_t M, int64_t N, int64_t K, int num_sms) {
+  // 256 x 256 pair tiles, whole N tiles; taken once the single-CTA 128 x 256 tiles fill the SMs
+  // and the pair tiles need no more waves (each SM does a 128 x 256 x 64 step per k-block
+  // either way; the pair kernel does it with a third less smem traffic, but pads M to 256:
+  // at M = 2176 the gate/up GEMM needs 14 pair waves vs 13 single-CTA waves and is slower)
+  if (N % 256 || K % kBK) return false;
+  const int64_t t1 = ((M + 127) / 128) * (N / 256), t2 = ((M + 255) / 256) * (N / 256);
+  if (t1 < num_sms) return false;
+  const int64_t w1 = (t1 + num_sms - 1) / num_sms, w2 = (t2 + num_sms / 2 - 1) / (num_sms / 2);
+  return w2 <= w1;
+}
+
+// tb: tensor map over B with 128-row boxes; ta: over A with 128-row boxes
+int gemm2_run(const CUtensorMap& ta, const CUtensorMap& tb, int64_t M, int64_t N, int64_t K, int epi, void* C,
+              int64_t ldc, const float* bias, int num_sms, cudaStream_t st, int a_row0, int max_ctas,
+              const QkvRopeArgs* rope) {
+  GemmArgs a{};
+  a.M = int(M);
+  a.N = int(N);
+  a.K = int(K);
+  a.mt = int((M + 255) / 256);
+  a.nt = int(N / 256);
+  a.ksplit = 1;
+  a.C = C;
+  a.ldc = int(ldc);
+  a.bias = bias;
+  a.a_row0 = a_row0;
+  a.pos = rope ? rope->pos : nullptr;
+  a.slot = rope ? rope->slot : nullptr;
+  a.rope = rope ? rope->tab : nullptr;
+  a.kplane = rope ? reinterpret_cast<__nv_bfloat16*>(rope->kplane) : nullptr;
+  a.vplane = rope ? reinterpret_cast<__nv_bfloat16*>(rope->vplane) : nullptr;
+  a.H = rope ? rope->H : 0;
+  a.Hkv = rope ? rope->Hkv : 0;
+  a.hd = rope ? rope->hd : 0;
+  if (epi == EPI_QKV_ROPE && (!rope || a.hd <= 0 || 256 % a.hd))
+    return set_error(QOS_ERR_INVALID_ARG, "gemm2: QKV_ROPE needs rope args and 256 % hd == 0");
+  const int units = a.mt * a.nt;
+  int pairs = std::min(units, (max_ctas > 0 ? std::min(max_ctas, num_sms) : num_sms) / 2);
+  if (pairs < 1) pairs = 1;
+  cudaError_t e;
+  switch (epi) {
+    case EPI_STORE_BF16: e = launch_gemm2_t<EPI_STORE_BF16>(ta, tb, a, 2 * pairs, st); break;
+    case EPI_STORE_F32: e = launch_gemm2_t<EPI_STORE_F32>(ta, tb, a, 2 * pairs, st); break;
+    case EPI_BIAS_BF16: e = launch_gemm2_t<EPI_BIAS_BF16>(ta, tb, a, 2 * pairs, st); break;
+    case EPI_SILU_GATE: e = launch_gemm2_t<EPI_SILU_GATE>(ta, tb, a, 2 * pairs, st); break;
+    case EPI_ADD_F32: e = launch_gemm2_t<EPI_ADD_F32>(ta, tb, a, 2 * pairs, st); break;
+    case EPI_QKV_ROPE: e = launch_gemm2_t<EPI_QKV_ROPE>(ta, tb, a, 2 * pairs, st); break;
+    default: return set_error(QOS_ERR_INVALID_ARG, "gemm2: bad epilogue");
+  }
+  if (e != cudaSuccess) return set_cuda_error(e, "gemm2 launch");
   return QOS_OK;
 }
 

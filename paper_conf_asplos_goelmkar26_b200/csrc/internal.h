@@ -47,6 +47,12 @@ int gemm_run(const CUtensorMap& ta, const CUtensorMap& tb, int bn, int64_t M, in
              int64_t ldc, const float* bias, int num_sms, cudaStream_t st, int ksplit = 1, float* part = nullptr,
              int* counters = nullptr, int a_row0 = 0, int max_ctas = 0, const QkvRopeArgs* rope = nullptr,
              int sk_mode = 1, bool coop = true);
+// CTA-pair (cta_group::2) GEMM with 256 x 256 tiles for large M (gemm.cu); ta / tb: tensor
+// maps with 128-row boxes over A and B.  gemm2_eligible: the shapes it takes.
+bool gemm2_eligible(int64_t M, int64_t N, int64_t K, int num_sms);
+int gemm2_run(const CUtensorMap& ta, const CUtensorMap& tb, int64_t M, int64_t N, int64_t K, int epi, void* C,
+              int64_t ldc, const float* bias, int num_sms, cudaStream_t st, int a_row0 = 0, int max_ctas = 0,
+              const QkvRopeArgs* rope = nullptr);
 // sk_mode: 0 no stream-K, 1 automatic (last-wave quantisation), 2 always (needs part/counters:
 // part >= 512 x 128 x 256 fp32, counters >= 4096); coop as in gemm_swab_run.
 
@@ -116,7 +122,9 @@ struct PrefillItem {     // one (chunk, q-tile, kv head) work item
   int32_t pos0;          // absolute position of row0
   int32_t table;         // block-table row
   int32_t kv_head;
-  int32_t pad;
+  int32_t pad;           // 1: duplicate that fills a CTA's group of q tiles (computes, stores nothing)
+  int32_t grp_last;      // last position over the q tiles one CTA processes together (their
+                         // key-tile count and the block clamp of the shared K/V tiles)
 };
 struct AttnLaunch {
   const void* q;          // [T][H][hd] bf16, row stride q_ld (elements)
@@ -131,6 +139,7 @@ struct AttnLaunch {
   const int32_t* tables;  // [max_requests][table_w]
   int table_w;
   float scale_log2;       // log2(e) / sqrt(hd)
+  int q_tiles = 1;        // prefill: q tiles per CTA sharing every K/V tile (1 or 2)
 };
 cudaError_t launch_decode_attention(const AttnLaunch& a, const DecodeItem* items, int n_items, float* partials,
                                     int* counters, cudaStream_t st);

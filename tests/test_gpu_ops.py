@@ -188,11 +188,15 @@ ATTN_CASES = [
 ]
 
 
+@pytest.mark.parametrize("qtiles", [1, 2])
 @pytest.mark.parametrize("case", range(len(ATTN_CASES)))
-def test_attention_parity(case):
+def test_attention_parity(case, qtiles):
+    """Prefill + decode attention (fp32 output) vs the fp64 oracle; prefill with 1 or 2 q tiles
+    per CTA sharing every K/V tile (odd tile counts padded with a duplicate)."""
     from oracle.model import causal_attention
     preset, over, chunks, ctxs, scale = ATTN_CASES[case]
     q, cfg, eng = make_engine(preset, **{"max_seq_len": 8192, **over})
+    eng.qos_engine_set_option("fa_qtiles", qtiles)
     H, Hkv, hd = cfg.n_heads, cfg.n_kv_heads, cfg.head_dim
     g = H // Hkv
     rng = np.random.default_rng(100 + case)
@@ -265,6 +269,51 @@ def test_gemm_splitk_parity(torch_cuda, M, N, K, ks, epi):
         got = dC.float().cpu().numpy()
         tol = 1e-5 if epi in ("store_f32", "add_f32") else 8e-3
         assert row_rel_err(got, ref) <= tol
+
+
+@pytest.mark.parametrize("M,N,K", [(1, 256, 64), (77, 512, 320), (300, 768, 128), (1000, 4096, 512),
+                                   (2176, 1024, 1024), (4100, 512, 256)])
+@pytest.mark.parametrize("epi", ["store_f32", "store_bf16", "add_f32", "bias_bf16", "silu_gate"])
+def test_gemm_2cta_parity(torch_cuda, M, N, K, epi):
+    """CTA-pair kernel (ksplit = -3; tcgen05 cta_group::2, 256 x 256 tiles over 2 SMs): every
+    epilogue, ragged M (half-empty and fully-empty 128-row halves of a pair tile), more tiles
+    than CTA pairs (persistent loop over both TMEM accumulators)."""
+    torch = torch_cuda
+    from oracle.model import silu
+    from paper_conf_asplos_goelmkar26_b200 import qoserve as q
+    rng = np.random.default_rng(M * 5 + N + K)
+    A = bits_to_f64(bf16_bits(rng.uniform(-1, 1, (M, K))))
+    B = bits_to_f64(bf16_bits(rng.uniform(-1, 1, (N, K)) / np.sqrt(K)))
+    dA, dB = _dev_bf16(torch, A), _dev_bf16(torch, B)
+    ref = A @ B.T
+    bias = None
+    init = None
+    if epi == "silu_gate":
+        g = np.concatenate([ref[:, 128 * j:128 * j + 64] for j in range(N // 128)], axis=1)
+        u = np.concatenate([ref[:, 128 * j + 64:128 * j + 128] for j in range(N // 128)], axis=1)
+        ref = silu(g) * u
+        dC = torch.empty((M, N // 2), dtype=torch.bfloat16, device="cuda")
+    elif epi in ("store_f32", "add_f32"):
+        init = rng.uniform(-1, 1, (M, N)).astype(np.float32) if epi == "add_f32" else np.zeros((M, N), np.float32)
+        dC = torch.from_numpy(init.copy()).cuda()
+        ref = ref + init.astype(np.float64)
+    else:
+        dC = torch.empty((M, N), dtype=torch.bfloat16, device="cuda")
+        if epi == "bias_bf16":
+            bvals = bits_to_f64(bf16_bits(rng.uniform(-0.02, 0.02, N)))
+            bias = torch.from_numpy(bvals.astype(np.float32)).cuda()
+            ref = ref + bvals
+    outs = []
+    for _ in range(2):
+        if init is not None:
+            dC.copy_(torch.from_numpy(init.copy()).cuda())
+        q.qos_op_gemm_ex(dA.data_ptr(), dB.data_ptr(), dC.data_ptr(), M, N, K, epi,
+                         bias.data_ptr() if bias is not None else None, -3)
+        torch.cuda.synchronize()
+        outs.append(dC.float().cpu().numpy())
+    tol = 1e-5 if epi in ("store_f32", "add_f32") else 8e-3
+    assert row_rel_err(outs[0], ref) <= tol
+    assert np.array_equal(outs[0], outs[1])
 
 
 @pytest.mark.parametrize("M,N,K", [(1, 128, 64), (16, 4096, 4096), (17, 1024, 2048), (100, 640, 1536),
