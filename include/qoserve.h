@@ -215,9 +215,12 @@ int qos_profile_step_ex(qos_engine_t* eng, int32_t chunk_len, int32_t kv_start,
  *                          polynomial, the rest on MUFU (0 = all MUFU; -1 = measurement-only
  *                          variant without the softmax, results invalid); process-wide,
  *                          env QOS_FA_POLY
- *   "fa_qtiles" (2)        prefill attention: q tiles (128 rows each) per CTA sharing every
+ *   "fa_qtiles" (1)        prefill attention: q tiles (128 rows each) per CTA sharing every
  *                          K/V tile (1: two CTAs per SM with 2-deep K/V rings; 2: one CTA per
- *                          SM, half the L2 -> SM traffic, 4-deep rings)
+ *                          SM, half the L2 -> SM traffic, 4-deep rings; measured ~6% more
+ *                          cycles than 1, tools/ncu_ab.py)
+ *   "gemm_2cta" (1)        CTA-pair GEMM (tcgen05 cta_group::2, 256 x 256 tiles) where it
+ *                          needs no more waves than 128 x 256 single-CTA tiles; env QOS_GEMM_2CTA
  * Results do not depend on the options (parity tests run with the defaults and variants). */
 int qos_engine_set_option(qos_engine_t* eng, const char* name, int64_t value);
 
