@@ -8,11 +8,14 @@ engine's OWN device-timed steps (`qos_profile_step`) with features that follow t
 work and the engine's tiling:
 
     t(batch) = c0 * Wgemm(T) + c1 * T + c2 * Bdec + c3 * n_dec + c4 * [n_dec > 0] + c5 + c6 * Fdiag
-               + c7 * Wstream(T) + c8 * Fprefix
+               + c7 * Wstream(T) + c8 * Fprefix + c9 * Wpair(T)
 
-* Wgemm(T): sum over the projections run by the tile kernel (csrc/gemm.cu) of (waves of
-  128 x BN tiles over the SMs) x (k-blocks per tile) x BN/256 — the tensor-core GEMM time with
-  the engine's tile-quantisation (same BN / split-K choice), T = sum(chunk_len) + n_decode;
+* Wgemm(T): sum over the projections run by the single-CTA tile kernel (csrc/gemm.cu) of (waves
+  of 128 x BN tiles over the SMs) x (k-blocks per tile) x BN/256 — the tensor-core GEMM time
+  with the engine's tile-quantisation (same BN / split-K choice), T = sum(chunk_len) + n_decode;
+* Wpair(T): the same for the projections run by the CTA-pair kernel (256 x 256 tiles over 2
+  SMs, same selection rule as gemm2_eligible): (waves of pair tiles over SMs/2) x k-blocks —
+  a separate term because its per-k-block cost differs;
 * Wstream(T): weight elements N*K of the projections run by the weight-streaming kernel
   (csrc/gemm_swab.cu, same selection rule as swab_prefer) — HBM-bound;
 * T: per-token elementwise work (norms, RoPE/append, embedding);
@@ -33,7 +36,7 @@ from dataclasses import dataclass, field
 
 import numpy as np
 
-N_FEAT = 9
+N_FEAT = 10
 
 
 @dataclass
@@ -76,12 +79,27 @@ def swab_prefer(M: int, N: int, sms: int) -> bool:   # mirrors swab_prefer (csrc
     return ((M + 127) // 128) * (N // 128) * 4 < sms
 
 
+def pair_eligible(M: int, N: int, K: int, sms: int) -> bool:   # mirrors gemm2_eligible (csrc/gemm.cu)
+    if N % 256 or K % 64:
+        return False
+    t1 = ((M + 127) // 128) * (N // 256)
+    t2 = ((M + 255) // 256) * (N // 256)
+    if t1 < sms:
+        return False
+    return -(-t2 // (sms // 2)) <= -(-t1 // sms)
+
+
+def pair_work(T: int, g: GemmShapes) -> float:
+    return float(sum(-(-(((T + 255) // 256) * (N // 256)) // (g.num_sms // 2)) * (K // 64)
+                     for N, K in g.gemms if T > 0 and pair_eligible(T, N, K, g.num_sms)))
+
+
 def gemm_work(T: int, g: GemmShapes) -> float:
     if T <= 0:
         return 0.0
     tot = 0.0
     for N, K in g.gemms:
-        if swab_prefer(T, N, g.num_sms):
+        if swab_prefer(T, N, g.num_sms) or pair_eligible(T, N, K, g.num_sms):
             continue
         bn = _bn(T, N, g.num_sms)
         tiles = ((T + 127) // 128) * ((N + bn - 1) // bn)
@@ -100,7 +118,7 @@ def features(s: StepShape, g: GemmShapes = GemmShapes()) -> np.ndarray:
     nd = len(s.ctx)
     return np.array([gemm_work(s.T, g) / 100.0, s.T / 1000.0, sum(c + 1 for c in s.ctx) / 1e6, nd / 100.0,
                      1.0 if nd else 0.0, 1.0, sum(n * (n + 1) / 2 for ks, n in s.chunks) / 1e7,
-                     stream_work(s.T, g) / 1e8, sum(n * ks for ks, n in s.chunks) / 1e7])
+                     stream_work(s.T, g) / 1e8, sum(n * ks for ks, n in s.chunks) / 1e7, pair_work(s.T, g) / 100.0])
 
 
 class LatencyModel:

@@ -7,14 +7,14 @@ import os
 import numpy as np
 
 from paper_conf_asplos_goelmkar26_b200.latency_model import (GemmShapes, LatencyModel, StepShape, features, gemm_work,
-                                                             stream_work)
+                                                             pair_eligible, pair_work, stream_work)
 
 PROF = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles", "latency_table_r1.json")
 
 
 def test_recovers_known_coefficients():
     rng = np.random.default_rng(0)
-    true = np.array([2.0, 3.0, 20.0, 0.5, 1.0, 4.0, 9.0, 6.0, 5.0])
+    true = np.array([2.0, 3.0, 20.0, 0.5, 1.0, 4.0, 9.0, 6.0, 5.0, 1.5])
     shapes = [StepShape([], list(rng.integers(1024, 8193, nd))) for nd in (1, 8, 16, 24, 32, 64, 100, 200, 256)]
     for _ in range(120):
         c = int(rng.integers(0, 8193))
@@ -30,11 +30,24 @@ def test_recovers_known_coefficients():
 
 def test_gemm_work_is_tile_quantised():
     g = GemmShapes()
-    assert gemm_work(2048, g) == gemm_work(2048 - 100, g)        # same 16 M-tiles
-    w = [gemm_work(t, g) for t in range(128, 8449, 128)]
+    assert gemm_work(1024, g) == gemm_work(1024 - 100, g)        # same 8 M-tiles
+    go = GemmShapes(((4096, 4096),), 148)                         # the O projection alone
+    assert pair_work(4096, go) == pair_work(4096 - 200, go)      # same 16 pair M-tiles
+    w = [pair_work(t, go) for t in range(2048, 8449, 256)]
     assert all(a <= b for a, b in zip(w, w[1:]))                   # steps, never decreasing
-    assert len(set(w)) > 20
-    assert gemm_work(8448, g) > 3 * gemm_work(2176, g)
+    assert len(set(w)) > 5
+    assert gemm_work(8448, g) + pair_work(8448, g) > 3 * (gemm_work(2176, g) + pair_work(2176, g))
+
+
+def test_pair_gemm_selection_mirrors_the_engine():
+    """gemm2_eligible (csrc/gemm.cu): pair tiles once 128 x 256 tiles fill the 148 SMs and the
+    256-row padding costs no extra wave — at T = 2176 the QKV, O and down projections take the
+    CTA-pair kernel and gate/up (13 single vs 14 pair waves) keeps single-CTA tiles."""
+    (qkv, o, gu, down) = GemmShapes().gemms
+    assert pair_eligible(2176, *qkv, 148) and pair_eligible(2176, *o, 148) and pair_eligible(2176, *down, 148)
+    assert not pair_eligible(2176, *gu, 148)
+    assert not pair_eligible(512, *o, 148)                        # 4 x 16 tiles < 148 SMs
+    assert pair_eligible(8192, *gu, 148)
 
 
 def test_small_steps_use_the_weight_streaming_gemm():
