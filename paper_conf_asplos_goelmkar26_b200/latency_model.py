@@ -8,7 +8,7 @@ engine's OWN device-timed steps (`qos_profile_step`) with features that follow t
 work and the engine's tiling:
 
     t(batch) = c0 * Wgemm(T) + c1 * T + c2 * Bdec + c3 * n_dec + c4 * [n_dec > 0] + c5 + c6 * Fdiag
-               + c7 * Wstream(T) + c8 * Fprefix + c9 * Wpair(T)
+               + c7 * Wstream(T) + c8 * Fprefix + c9 * Wpair(T) + c10 * Npair(T) + c11 * Ntile(T)
 
 * Wgemm(T): sum over the projections run by the single-CTA tile kernel (csrc/gemm.cu) of (waves
   of 128 x BN tiles over the SMs) x (k-blocks per tile) x BN/256 — the tensor-core GEMM time
@@ -16,6 +16,8 @@ work and the engine's tiling:
 * Wpair(T): the same for the projections run by the CTA-pair kernel (256 x 256 tiles over 2
   SMs, same selection rule as gemm2_eligible): (waves of pair tiles over SMs/2) x k-blocks —
   a separate term because its per-k-block cost differs;
+* Npair(T), Ntile(T): how many of the 4 projections run on the pair / single-CTA tile kernel
+  (per-launch prologue, pipeline fill and exposed last-wave epilogue, x L layers);
 * Wstream(T): weight elements N*K of the projections run by the weight-streaming kernel
   (csrc/gemm_swab.cu, same selection rule as swab_prefer) — HBM-bound;
 * T: per-token elementwise work (norms, RoPE/append, embedding);
@@ -36,7 +38,7 @@ from dataclasses import dataclass, field
 
 import numpy as np
 
-N_FEAT = 10
+N_FEAT = 12
 
 
 @dataclass
@@ -116,9 +118,12 @@ def stream_work(T: int, g: GemmShapes) -> float:
 
 def features(s: StepShape, g: GemmShapes = GemmShapes()) -> np.ndarray:
     nd = len(s.ctx)
+    n_pair = sum(1 for N, K in g.gemms if s.T > 0 and pair_eligible(s.T, N, K, g.num_sms))
+    n_stream = sum(1 for N, K in g.gemms if s.T > 0 and swab_prefer(s.T, N, g.num_sms))
     return np.array([gemm_work(s.T, g) / 100.0, s.T / 1000.0, sum(c + 1 for c in s.ctx) / 1e6, nd / 100.0,
                      1.0 if nd else 0.0, 1.0, sum(n * (n + 1) / 2 for ks, n in s.chunks) / 1e7,
-                     stream_work(s.T, g) / 1e8, sum(n * ks for ks, n in s.chunks) / 1e7, pair_work(s.T, g) / 100.0])
+                     stream_work(s.T, g) / 1e8, sum(n * ks for ks, n in s.chunks) / 1e7, pair_work(s.T, g) / 100.0,
+                     float(n_pair), float(len(g.gemms) - n_pair - n_stream)])
 
 
 class LatencyModel:
