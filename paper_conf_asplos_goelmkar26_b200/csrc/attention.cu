@@ -22,22 +22,21 @@
 
 namespace qos {
 
-constexpr int kAttnStages = 8;
 constexpr int kConsumerWarps = 4;
 constexpr int kAttnThreads = (kConsumerWarps + 1) * 32;
-// Block i goes to consumer warp i % kConsumerWarps and ring stage i % kAttnStages.  With a
-// multiple, stage s is always consumed by the same warp, in order, so no waiter can run a full
-// phase ahead of an mbarrier (parity waits would then alias).
-static_assert(kAttnStages % kConsumerWarps == 0, "ring depth must be a multiple of the consumer warps");
+// Block i goes to consumer warp i % kConsumerWarps and ring stage i % NS (NS = ring depth, 8 or
+// 4).  With a multiple, stage s is always consumed by the same warp, in order, so no waiter can
+// run a full phase ahead of an mbarrier (parity waits would then alias).
 
-template <int HD>
+template <int HD, int NS>
 struct AttnCfg {
+  static_assert(NS % kConsumerWarps == 0, "ring depth must be a multiple of the consumer warps");
   static constexpr int kBlockBytes = 16 * HD * 2;     // one (block, head) tile
   static constexpr int kStageBytes = 2 * kBlockBytes; // K + V
   static constexpr int kHalves = HD / 64;
   static constexpr int kNT = HD / 8;                  // n-tiles of the output (8 dims each)
   static constexpr int kKS = HD / 16;                 // k-steps of Q K^T
-  static constexpr int kSmemBytes = kAttnStages * kStageBytes + 1024 + 2 * kAttnStages * 8 + 64;
+  static constexpr int kSmemBytes = NS * kStageBytes + 1024 + 2 * NS * 8 + 64;
 };
 
 struct AttnParams {
@@ -59,7 +58,7 @@ QOS_DEV uint32_t tile_off(int kr, int ch) {
 
 template <int HD>
 QOS_DEV void issue_block_load(const CUtensorMap* map, uint8_t* stage, uint64_t* bar, int layer, int row) {
-  using C = AttnCfg<HD>;
+  using C = AttnCfg<HD, 4>;
 #pragma unroll
   for (int h = 0; h < C::kHalves; ++h) {
     tma_load_3d(stage + h * 2048, map, bar, h * 64, row, layer * 2 + 0);
@@ -103,15 +102,15 @@ QOS_DEV void pv_block_t(uint32_t b0, uint32_t b1, uint32_t vtile, int lane, floa
 }
 
 // ------------------------------------------------------------------------------ decode
-template <int HD>
+template <int HD, int NS>
 __global__ void __launch_bounds__(kAttnThreads, 3)
     decode_attn_kernel(const __grid_constant__ CUtensorMap kvmap, const AttnParams p, const DecodeItem* __restrict__ items,
                        float* __restrict__ partials, int* __restrict__ counters) {
-  using C = AttnCfg<HD>;
+  using C = AttnCfg<HD, NS>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + kAttnStages * C::kStageBytes);
-  uint64_t* empty = full + kAttnStages;
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + NS * C::kStageBytes);
+  uint64_t* empty = full + NS;
 
   griddep_wait();  // q and the appended K/V come from the previous kernel
   griddep_launch_dependents();
@@ -122,7 +121,7 @@ __global__ void __launch_bounds__(kAttnThreads, 3)
   const int nblk = ((it.key1 + 15) >> 4) - blk0;
 
   if (threadIdx.x == 0) {
-    for (int s = 0; s < kAttnStages; ++s) {
+    for (int s = 0; s < NS; ++s) {
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], 1);
     }
@@ -135,8 +134,8 @@ __global__ void __launch_bounds__(kAttnThreads, 3)
       tma_prefetch_desc(&kvmap);
       const int32_t* trow = p.tables + size_t(it.table) * p.table_w;
       for (int i = 0; i < nblk; ++i) {
-        const int s = i % kAttnStages;
-        const uint32_t ph = (i / kAttnStages) & 1;
+        const int s = i % NS;
+        const uint32_t ph = (i / NS) & 1;
         mbar_wait(&empty[s], ph ^ 1);
         mbar_arrive_expect_tx(&full[s], C::kStageBytes);
         const int block = __ldg(trow + blk0 + i);
@@ -162,8 +161,8 @@ __global__ void __launch_bounds__(kAttnThreads, 3)
       qb[ks][1] = g < group ? *reinterpret_cast<const uint32_t*>(qh + ks * 16 + 2 * t + 8) : 0u;
     }
     for (int i = warp; i < nblk; i += kConsumerWarps) {
-      const int s = i % kAttnStages;
-      const uint32_t ph = (i / kAttnStages) & 1;
+      const int s = i % NS;
+      const uint32_t ph = (i / NS) & 1;
       mbar_wait(&full[s], ph);
       const uint32_t kt = smem_u32(smem + s * C::kStageBytes);
       float sc[4];
@@ -314,17 +313,17 @@ static AttnParams to_params(const AttnLaunch& a) {
   return p;
 }
 
-template <int HD>
+template <int HD, int NS>
 static cudaError_t decode_t(const AttnLaunch& a, const DecodeItem* items, int n_items, float* partials, int* counters,
                             cudaStream_t st) {
   static bool set = false;
   if (!set) {
-    cudaError_t e = cudaFuncSetAttribute(decode_attn_kernel<HD>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         AttnCfg<HD>::kSmemBytes);
+    cudaError_t e = cudaFuncSetAttribute(decode_attn_kernel<HD, NS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         AttnCfg<HD, NS>::kSmemBytes);
     if (e != cudaSuccess) return e;
     set = true;
   }
-  return launch_pdl(decode_attn_kernel<HD>, dim3(n_items), dim3(kAttnThreads), AttnCfg<HD>::kSmemBytes, st,
+  return launch_pdl(decode_attn_kernel<HD, NS>, dim3(n_items), dim3(kAttnThreads), AttnCfg<HD, NS>::kSmemBytes, st,
                     *a.kv_tmap, to_params(a), items, partials, counters);
 }
 
@@ -332,8 +331,12 @@ cudaError_t launch_decode_attention(const AttnLaunch& a, const DecodeItem* items
                                     int* counters, cudaStream_t st) {
   if (n_items == 0) return cudaSuccess;
   count_launch(1);
-  if (a.hd == 128) return decode_t<128>(a, items, n_items, partials, counters, st);
-  if (a.hd == 64) return decode_t<64>(a, items, n_items, partials, counters, st);
+  if (a.hd == 128)
+    return a.decode_stages == 4 ? decode_t<128, 4>(a, items, n_items, partials, counters, st)
+                                : decode_t<128, 8>(a, items, n_items, partials, counters, st);
+  if (a.hd == 64)
+    return a.decode_stages == 4 ? decode_t<64, 4>(a, items, n_items, partials, counters, st)
+                                : decode_t<64, 8>(a, items, n_items, partials, counters, st);
   return cudaErrorInvalidValue;
 }
 

@@ -247,6 +247,7 @@ struct qos_engine {
   int dual_sms_pre = 0, dual_sms_dec = 0;  // SM budgets of the two streams' GEMMs (0 = all)
   bool gemm_2cta = true;            // option gemm_2cta: CTA-pair GEMM (256 x 256 tiles) at large M
   bool decode_round_split = true;  // option decode_round_split (A/B of the split-K ranges)
+  int decode_stages = 8;            // option decode_stages: decode K/V ring depth (8 or 4)
   int fa_qtiles = 1;                // option fa_qtiles: prefill q tiles per CTA sharing K/V tiles
   bool overlap_attn = true;       // QOS_OVERLAP_ATTN=0 serialises a7 and a8 (for measurement)
   bool gemm_splitk = true;        // QOS_GEMM_SPLITK=0 disables split-K for small-M GEMMs
@@ -672,6 +673,7 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
   al.table_w = e->table_w;
   al.scale_log2 = float(1.4426950408889634 / std::sqrt(double(hd)));
   al.q_tiles = m.fa_qtiles;
+  al.decode_stages = e->decode_stages;
   const int n_pre_rows = T - m.n_decode;
   float* gpart0 = reinterpret_cast<float*>(e->ws + s.gemm_part);
   int* gcnt0 = reinterpret_cast<int*>(e->ws + s.gemm_cnt);
@@ -1327,6 +1329,10 @@ int qos_engine_set_option(qos_engine_t* e, const char* name, int64_t value) {
   if (n == "overlap_attn") e->overlap_attn = value != 0;
   else if (n == "decode_round_split") e->decode_round_split = value != 0;
   else if (n == "gemm_2cta") e->gemm_2cta = value != 0;
+  else if (n == "decode_stages") {
+    if (value != 4 && value != 8) return set_error(QOS_ERR_INVALID_ARG, "decode_stages must be 4 or 8");
+    e->decode_stages = int(value);
+  }
   else if (n == "fa_qtiles") {
     if (value != 1 && value != 2) return set_error(QOS_ERR_INVALID_ARG, "fa_qtiles must be 1 or 2");
     e->fa_qtiles = int(value);
@@ -1560,6 +1566,7 @@ int qos_op_attention(qos_engine_t* e, int32_t layer, const qos_batch* b, const u
   al.table_w = e->table_w;
   al.scale_log2 = float(1.4426950408889634 / std::sqrt(double(hd)));
   al.q_tiles = m.fa_qtiles;
+  al.decode_stages = e->decode_stages;
   QOS_CU(launch_prefill_attention_tc(al, reinterpret_cast<const PrefillItem*>(dm + m.o_pitems), m.n_pitems, st));
   QOS_CU(launch_decode_attention(al, reinterpret_cast<const DecodeItem*>(dm + m.o_ditems), m.n_ditems,
                                  reinterpret_cast<float*>(e->ws + e->wsl.partials),

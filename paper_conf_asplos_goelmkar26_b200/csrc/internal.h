@@ -140,6 +140,7 @@ struct AttnLaunch {
   int table_w;
   float scale_log2;       // log2(e) / sqrt(hd)
   int q_tiles = 1;        // prefill: q tiles per CTA sharing every K/V tile (1 or 2)
+  int decode_stages = 8;  // decode: K/V ring depth in (block, head) tiles (8 or 4)
 };
 cudaError_t launch_decode_attention(const AttnLaunch& a, const DecodeItem* items, int n_items, float* partials,
                                     int* counters, cudaStream_t st);

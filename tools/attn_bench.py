@@ -19,6 +19,8 @@ ap.add_argument("--layers", type=int, default=4)
 ap.add_argument("--reps", type=int, default=5)
 ap.add_argument("--variants", default="", help="A/B in one process: 'fa_poly=0;fa_poly=4' (engine options)")
 ap.add_argument("--rounds", type=int, default=1, help="interleaved repetitions of all variants")
+ap.add_argument("--step-only", action="store_true",
+                help="whole-step device time only (no per-kernel events, attention overlap left on)")
 a = ap.parse_args()
 import threading  # noqa: E402
 import time  # noqa: E402
@@ -65,11 +67,18 @@ cfg = q.model_cfg(**P, num_blocks=need // 16 + 600, max_seq_len=16384, max_reque
 eng = q.Engine(cfg)
 eng.qos_engine_load_synthetic(0)
 L, H, Hkv, hd = P["n_layers"], P["n_heads"], P["n_kv_heads"], P["head_dim"]
-eng.qos_engine_set_option("overlap_attn", 0)
+if not a.step_only:
+    eng.qos_engine_set_option("overlap_attn", 0)
 variants = [v for v in a.variants.split(";") if v] or [""]
 
 
 def run_point(c, nd, ctx, ks, tag):
+    if a.step_only:
+        with ClockSampler() as clk:
+            ms, _ = eng.qos_profile_step(c, [ctx] * nd, reps=a.reps, kv_start=ks)
+        print(json.dumps({"variant": tag, "chunk": c, "n_decode": nd, "ctx": ctx, "kv_start": ks, "layers": L,
+                          "step_ms": round(ms, 3), "sm_mhz": clk.median()}), flush=True)
+        return
     eng.qos_engine_set_timing(True)
     with ClockSampler() as clk:
         ms, _ = eng.qos_profile_step(c, [ctx] * nd, reps=a.reps, kv_start=ks)
