@@ -439,6 +439,314 @@ __global__ void __launch_bounds__(FaCfg<HD, NQ>::kThreads, FaCfg<HD, NQ>::kMinBl
   }
 }
 
+
+// ---------------------------------------------------------------- ping-pong variant (fa_qtiles=2)
+// Two q tiles per CTA (one CTA per SM), 128-key K/V tiles, one S/P buffer per q tile (TMEM:
+// S0 [0,128) S1 [128,256) O0 [256,384) O1 [384,512)).  QKᵀ runs as UMMA N = 128 (twice the
+// work per instruction of the 64-key kernel) and the tensor core alternates between the two
+// q tiles: while softmax group 1 works on S1(j) it executes PV0(j) and QK0(j+1), while group
+// 0 works on S0(j+1) it executes PV1(j) and QK1(j+1).  QK_g(j+1) is issued after PV_g(j)
+// (same TMEM columns; tcgen05 ops run in issue order), so when a softmax group sees S_g(j+1)
+// its PV_g(j) has landed and it may rescale O_g without a wait.
+template <int HD>
+struct PpCfg {
+  static constexpr int kRows = 128, kKeys = 128, kHalves = HD / 64;
+  static constexpr int kQBytes = kRows * HD * 2;      // 32 KB at HD 128
+  static constexpr int kTileBytes = kKeys * HD * 2;   // 32 KB: one K or V tile
+  static constexpr int kStages = 2;
+  static constexpr int kSmem = 2 * kQBytes + 2 * kStages * kTileBytes + 1024 + 512 + 2 * 2 * 128 * 4;
+  // 2 TMA/MMA warps + per q tile 8 softmax warps: two threads per row, each owning 64 of the
+  // tile's 128 keys (and 64 of the row's HD/... output columns for rescale and epilogue)
+  static constexpr int kThreads = 64 + 2 * 256;
+  static constexpr uint32_t col_s(int g) { return uint32_t(g * 128); }
+  static constexpr uint32_t col_o(int g) { return uint32_t(256 + g * HD); }
+};
+
+template <int HD, int POLY>
+__global__ void __launch_bounds__(PpCfg<HD>::kThreads, 1)
+    prefill_attn_pp_kernel(const __grid_constant__ CUtensorMap kvmap, const FaParams p,
+                           const PrefillItem* __restrict__ items) {
+  using C = PpCfg<HD>;
+  constexpr int S = C::kStages;
+  constexpr int KH = C::kKeys / 2;   // keys per softmax thread
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sQ = smem;                          // 2 x kQBytes
+  uint8_t* sK = smem + 2 * C::kQBytes;
+  uint8_t* sV = sK + S * C::kTileBytes;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(sV + S * C::kTileBytes);
+  uint64_t* k_full = bar;
+  uint64_t* k_empty = k_full + S;
+  uint64_t* v_full = k_empty + S;
+  uint64_t* v_empty = v_full + S;
+  uint64_t* s_full = v_empty + S;   // [2]
+  uint64_t* p_full = s_full + 2;    // [2]
+  uint64_t* o_final = p_full + 2;   // [2]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(o_final + 2);
+  float* xch = reinterpret_cast<float*>(bar + 64);   // [2 groups][2 halves][128 rows]: row max / sum exchange
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const PrefillItem it0 = items[blockIdx.x * 2];
+  const int group = p.H / p.Hkv;
+  const int ppt = C::kRows / group;
+  const int last_pos = it0.grp_last;
+  const int ntiles = last_pos / C::kKeys + 1;
+  const int last_blk = last_pos >> 4;
+
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < S; ++i) {
+      mbar_init(&k_full[i], 1);
+      mbar_init(&k_empty[i], 1);
+      mbar_init(&v_full[i], 1);
+      mbar_init(&v_empty[i], 1);
+    }
+    for (int g = 0; g < 2; ++g) {
+      mbar_init(&s_full[g], 1);
+      mbar_init(&p_full[g], 256);
+      mbar_init(&o_final[g], 1);
+    }
+    fence_mbar_init();
+  }
+  if (warp == 1) tmem_alloc<512>(tmem_slot);
+  griddep_wait();
+  griddep_launch_dependents();
+
+  // softmax warp w >= 2: q tile qg, key half kh, TMEM lane quarter w & 3
+  const int sw = warp - 2;
+  const int qg = warp >= 2 ? sw >> 3 : 0;
+  const int kh = warp >= 2 ? (sw >> 2) & 1 : 0;
+  const PrefillItem it = items[blockIdx.x * 2 + qg];
+  int row = 0, pos_r = -1;
+  size_t tok_off = 0;
+  if (warp >= 2) {
+    row = (warp & 3) * 32 + lane;
+    const int pi = row / group, hh = row % group;
+    const bool ok = row < ppt * group && pi < it.npos;
+    pos_r = ok ? it.pos0 + pi : -1;
+    tok_off = size_t(it.row0 + pi) * p.out_ld + size_t(it.kv_head * group + hh) * HD;
+    if (kh == 0) {  // the first half's threads stage the q row
+      const __nv_bfloat16* src = p.q + size_t(it.row0 + pi) * p.q_ld + size_t(it.kv_head * group + hh) * HD;
+      uint8_t* q_dst = sQ + qg * C::kQBytes;
+      uint4 v[HD / 8];
+#pragma unroll
+      for (int ch = 0; ch < HD / 8; ++ch) v[ch] = ok ? *reinterpret_cast<const uint4*>(src + ch * 8) : make_uint4(0, 0, 0, 0);
+#pragma unroll
+      for (int ch = 0; ch < HD / 8; ++ch) {
+        const int hf = ch >> 3, c = ch & 7;
+        *reinterpret_cast<uint4*>(q_dst + hf * (C::kRows * 128) + row * 128 + ((c ^ (row & 7)) << 4)) = v[ch];
+      }
+      fence_proxy_async_smem();
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == 0) {
+    // ------------------------------------------------------------------ TMA producer
+    if (elect_one()) {
+      tma_prefetch_desc(&kvmap);
+      const int32_t* trow = p.tables + size_t(it0.table) * p.table_w;
+      auto load_tile = [&](uint8_t* dst, uint64_t* full, int j, int plane) {
+        for (int b = 0; b < C::kKeys / 16; ++b) {
+          const int blk = min(j * (C::kKeys / 16) + b, last_blk);
+          const int r = (__ldg(trow + blk) * p.Hkv + it0.kv_head) * 16;
+#pragma unroll
+          for (int hf = 0; hf < C::kHalves; ++hf)
+            tma_load_3d(dst + hf * (C::kKeys * 128) + b * 2048, &kvmap, full, hf * 64, r, p.layer * 2 + plane);
+        }
+      };
+      for (int j = 0; j < ntiles; ++j) {
+        const int s = j % S;
+        const uint32_t ph = (j / S) & 1;
+        mbar_wait(&k_empty[s], ph ^ 1);
+        mbar_arrive_expect_tx(&k_full[s], C::kTileBytes);
+        load_tile(sK + s * C::kTileBytes, &k_full[s], j, 0);
+        mbar_wait(&v_empty[s], ph ^ 1);
+        mbar_arrive_expect_tx(&v_full[s], C::kTileBytes);
+        load_tile(sV + s * C::kTileBytes, &v_full[s], j, 1);
+      }
+    }
+  } else if (warp == 1) {
+    // ------------------------------------------------------------------ MMA issuer
+    if (elect_one()) {
+      constexpr uint32_t idesc_qk = umma_idesc_bf16(128, C::kKeys);
+      constexpr uint32_t idesc_pv = (1u << 4) | (1u << 16) | ((uint32_t(HD) >> 3) << 17) | ((128u >> 4) << 24);
+      auto issue_qk = [&](int g, int j) {
+        const int s = j % S;
+        const uint32_t k_base = smem_u32(sK + s * C::kTileBytes);
+        const uint32_t q_base = smem_u32(sQ + g * C::kQBytes);
+#pragma unroll
+        for (int ks = 0; ks < HD / 16; ++ks) {
+          const uint32_t qoff = (ks >> 2) * (C::kRows * 128) + (ks & 3) * 32;
+          const uint32_t koff = (ks >> 2) * (C::kKeys * 128) + (ks & 3) * 32;
+          if (POLY != -3)
+            umma_bf16(tmem + C::col_s(g), umma_desc_sw128(q_base + qoff), umma_desc_sw128(k_base + koff), idesc_qk, ks != 0);
+        }
+        umma_commit(&s_full[g]);
+      };
+      auto issue_pv = [&](int g, int j) {
+        const int s = j % S;
+        mbar_wait(&p_full[g], j & 1);
+        tc_fence_after();
+        const uint32_t v_base = smem_u32(sV + s * C::kTileBytes);
+#pragma unroll
+        for (int kk = 0; kk < C::kKeys / 16; ++kk) {
+          const uint64_t vd = umma_desc_sw128_mn(v_base + kk * 2048, C::kKeys * 128);
+          const uint32_t pc = tmem + C::col_s(g) + (kk >> 1) * 32 + (kk & 1) * 8;
+          if (POLY != -2) umma_bf16_ts(tmem + C::col_o(g), pc, vd, idesc_pv, (j | kk) != 0);
+        }
+      };
+      mbar_wait(&k_full[0], 0);
+      tc_fence_after();
+      issue_qk(0, 0);
+      issue_qk(1, 0);
+      umma_commit(&k_empty[0]);
+      for (int j = 0; j < ntiles; ++j) {
+        const int s = j % S, s1 = (j + 1) % S;
+        const bool more = j + 1 < ntiles;
+        mbar_wait(&v_full[s], (j / S) & 1);
+        issue_pv(0, j);                       // O0 += P0(j) V(j)
+        if (more) {                           // S0(j+1) = Q0 K(j+1)^T (after PV0(j): same columns)
+          mbar_wait(&k_full[s1], ((j + 1) / S) & 1);
+          tc_fence_after();
+          issue_qk(0, j + 1);
+        }
+        issue_pv(1, j);                       // O1 += P1(j) V(j)
+        umma_commit(&v_empty[s]);
+        if (more) {
+          issue_qk(1, j + 1);
+          umma_commit(&k_empty[s1]);
+        }
+      }
+      umma_commit(&o_final[0]);
+      umma_commit(&o_final[1]);
+    }
+  } else {
+    // ------------------------------------------------------------------ softmax (q tile qg, key half kh)
+    const uint32_t lane_base = tmem + (uint32_t((warp & 3) * 32) << 16);
+    const uint32_t s_addr = lane_base + C::col_s(qg) + kh * (KH / 2);  // this half's 32 fp16-pair columns...
+    const uint32_t s_rd = lane_base + C::col_s(qg) + kh * KH;          // ...and its 64 fp32 S columns
+    const uint32_t o_addr = lane_base + C::col_o(qg) + kh * (HD / 2);
+    const int bar_id = 1 + qg * 4 + (warp & 3);   // the two warps (halves) of one row quarter
+    float* my_x = xch + (qg * 2 + kh) * 128;
+    const float* pe_x = xch + (qg * 2 + (kh ^ 1)) * 128;
+    auto pair_sync = [&]() { asm volatile("bar.sync %0, 64;" ::"r"(bar_id) : "memory"); };
+    const int warp_min_pos = __shfl_sync(0xffffffffu, pos_r < 0 ? INT_MAX : pos_r, 0);
+    float m_used = -INFINITY, l = 0.f;
+    for (int j = 0; j < ntiles; ++j) {
+      mbar_wait(&s_full[qg], j & 1);
+      tc_fence_after();
+      if (POLY < 0) {
+        tc_fence_before();
+        mbar_arrive(&p_full[qg]);
+        continue;
+      }
+      const int key0 = j * C::kKeys + kh * KH;
+      const bool masked = __any_sync(0xffffffffu, key0 + KH - 1 > (pos_r < 0 ? -1 : pos_r)) || warp_min_pos == INT_MAX;
+      uint32_t r[KH];
+#pragma unroll
+      for (int c = 0; c < KH / 16; ++c)
+        tmem_ld32x32b_x16(s_rd + c * 16, *reinterpret_cast<uint32_t(*)[16]>(&r[c * 16]));
+      tmem_ld_wait();
+      if (masked) {
+        const int lim = (pos_r < 0 ? -1 : pos_r) - key0;
+#pragma unroll
+        for (int i = 0; i < KH; ++i)
+          if (i > lim) r[i] = 0xff800000u;
+      }
+      float mq[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
+#pragma unroll
+      for (int i = 0; i < KH; i += 2)
+        mq[(i >> 1) & 3] = fmax3(mq[(i >> 1) & 3], __uint_as_float(r[i]), __uint_as_float(r[i + 1]));
+      float mx = fmax3(mq[0], mq[1], fmaxf(mq[2], mq[3]));
+      // row max over both halves (partner thread: same row, other key half)
+      my_x[row] = mx;
+      pair_sync();
+      mx = fmaxf(mx, pe_x[row]) * p.scale_log2;
+      const bool rescale = mx > m_used + QOS_FA_LAZY;
+      const float m_new = rescale ? mx : m_used;
+      const float alpha = (rescale && m_used != -INFINITY) ? ex2(m_used - m_new) : 1.f;
+      const float mb = (m_new == -INFINITY) ? 0.f : m_new;
+      float2 sum2[4] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+      const float2 scale2 = make_float2(p.scale_log2, p.scale_log2), nmb2 = make_float2(-mb, -mb);
+#pragma unroll
+      for (int c = 0; c < KH / 32; ++c) {
+        uint32_t hi[16];
+#pragma unroll
+        for (int i = 0; i < 16; ++i) {
+          const float2 x = fma2(make_float2(__uint_as_float(r[c * 32 + 2 * i]), __uint_as_float(r[c * 32 + 2 * i + 1])),
+                                scale2, nmb2);
+          float2 pp = (POLY > 0 && i % (POLY > 0 ? POLY : 1) == (POLY > 0 ? POLY : 1) - 1) ? ex2_poly2(x) : make_float2(ex2(x.x), ex2(x.y));
+          hi[i] = pack_f16(pp.x, pp.y);
+          sum2[i & 3] = add2(sum2[i & 3], pp);
+        }
+        // keys [32c', 32c'+32) of the tile (c' = kh*2 + c) -> fp16 pairs at columns [32c', 32c'+16)
+        tmem_st32x32b_x16(lane_base + C::col_s(qg) + (kh * 2 + c) * 32, hi);
+      }
+      (void)s_addr;
+      const float2 s01 = add2(sum2[0], sum2[1]), s23 = add2(sum2[2], sum2[3]);
+      l = l * alpha + ((s01.x + s23.x) + (s01.y + s23.y));   // this half's share of the row sum
+      if (j >= 1 && __any_sync(0xffffffffu, alpha != 1.f)) {
+        // PV_g(j-1) was issued before QK_g(j), whose completion was awaited above
+#pragma unroll 1
+        for (int c = 0; c < HD / 32; ++c) {
+          uint32_t r2[16];
+          tmem_ld32x32b_x16(o_addr + c * 16, r2);
+          tmem_ld_wait();
+#pragma unroll
+          for (int i = 0; i < 16; ++i) r2[i] = __float_as_uint(__uint_as_float(r2[i]) * alpha);
+          tmem_st32x32b_x16(o_addr + c * 16, r2);
+        }
+      }
+      tmem_st_wait();
+      m_used = m_new;
+      tc_fence_before();
+      mbar_arrive(&p_full[qg]);
+    }
+    // row sum over both halves
+    pair_sync();   // the partner has read my_x of the last tile
+    my_x[row] = l;
+    pair_sync();
+    l += pe_x[row];
+    mbar_wait(&o_final[qg], 0);
+    tc_fence_after();
+    const float inv = (l > 0.f) ? 1.f / l : 0.f;
+#pragma unroll 1
+    for (int c = 0; c < HD / 64; ++c) {
+      uint32_t r2[32];
+      tmem_ld32x32b_x16(o_addr + c * 32, *reinterpret_cast<uint32_t(*)[16]>(&r2[0]));
+      tmem_ld32x32b_x16(o_addr + c * 32 + 16, *reinterpret_cast<uint32_t(*)[16]>(&r2[16]));
+      tmem_ld_wait();
+      const size_t off = tok_off + kh * (HD / 2) + c * 32;
+      if (pos_r >= 0 && !it.pad) {
+        if (p.out_f32) {
+          float4* dst = reinterpret_cast<float4*>(reinterpret_cast<float*>(p.out) + off);
+#pragma unroll
+          for (int i = 0; i < 8; ++i)
+            dst[i] = make_float4(__uint_as_float(r2[4 * i]) * inv, __uint_as_float(r2[4 * i + 1]) * inv,
+                                 __uint_as_float(r2[4 * i + 2]) * inv, __uint_as_float(r2[4 * i + 3]) * inv);
+        } else {
+          uint4* dst = reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.out) + off);
+#pragma unroll
+          for (int i = 0; i < 4; ++i)
+            dst[i] = make_uint4(pack_bf16(__uint_as_float(r2[8 * i]) * inv, __uint_as_float(r2[8 * i + 1]) * inv),
+                                pack_bf16(__uint_as_float(r2[8 * i + 2]) * inv, __uint_as_float(r2[8 * i + 3]) * inv),
+                                pack_bf16(__uint_as_float(r2[8 * i + 4]) * inv, __uint_as_float(r2[8 * i + 5]) * inv),
+                                pack_bf16(__uint_as_float(r2[8 * i + 6]) * inv, __uint_as_float(r2[8 * i + 7]) * inv));
+        }
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc<512>(tmem);
+  }
+}
+
 static int g_fa_poly = getenv("QOS_FA_POLY") ? atoi(getenv("QOS_FA_POLY")) : 4;
 
 template <int HD, int POLY, int NQ>
@@ -468,6 +776,33 @@ static cudaError_t prefill_tc_t(const AttnLaunch& a, const PrefillItem* items, i
                     *a.kv_tmap, p, items);
 }
 
+template <int HD, int POLY>
+static cudaError_t prefill_pp_t(const AttnLaunch& a, const PrefillItem* items, int n_items, cudaStream_t st) {
+  using C = PpCfg<HD>;
+  static bool set = false;
+  if (!set) {
+    cudaError_t e = cudaFuncSetAttribute(prefill_attn_pp_kernel<HD, POLY>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         C::kSmem);
+    if (e != cudaSuccess) return e;
+    set = true;
+  }
+  FaParams p;
+  p.q = reinterpret_cast<const __nv_bfloat16*>(a.q);
+  p.q_ld = a.q_ld;
+  p.out = a.out;
+  p.out_ld = a.out_ld;
+  p.out_f32 = a.out_f32;
+  p.layer = a.layer;
+  p.H = a.H;
+  p.Hkv = a.Hkv;
+  p.tables = a.tables;
+  p.table_w = a.table_w;
+  p.scale_log2 = a.scale_log2;
+  if (n_items % 2) return cudaErrorInvalidValue;
+  return launch_pdl(prefill_attn_pp_kernel<HD, POLY>, dim3(n_items / 2), dim3(C::kThreads), C::kSmem, st, *a.kv_tmap,
+                    p, items);
+}
+
 void set_fa_poly(int n) { g_fa_poly = n; }
 
 int prefill_tc_positions_per_tile(int group) { return 128 / group; }
@@ -479,7 +814,7 @@ cudaError_t launch_prefill_attention_tc(const AttnLaunch& a, const PrefillItem* 
   const int nq = a.q_tiles;
   if (nq != 1 && nq != 2) return cudaErrorInvalidValue;
 #define QOS_FA_NQ(HDV, PV) \
-  return nq == 1 ? prefill_tc_t<HDV, PV, 1>(a, items, n_items, st) : prefill_tc_t<HDV, PV, 2>(a, items, n_items, st);
+  return nq == 1 ? prefill_tc_t<HDV, PV, 1>(a, items, n_items, st) : prefill_pp_t<HDV, PV>(a, items, n_items, st);
   if (a.hd == 128) {
     // measurement-only variants: -1 no softmax, -2 also no P.V MMAs, -3 no softmax and no QK MMAs
     if (poly == -1) { QOS_FA_NQ(128, -1) }
