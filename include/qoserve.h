@@ -49,7 +49,7 @@ enum {
   QOS_ERR_BAD_KV_START = -4,  /* kv_start / ctx_len != the request's cached length         */
   QOS_ERR_NOT_ALLOCATED = -5, /* the step would write past the request's allocated blocks  */
   QOS_ERR_CUDA = -6,          /* CUDA runtime / driver error (message in qos_last_error)   */
-  QOS_ERR_COMM = -7,          /* NCCL error; the communicator is aborted                   */
+  QOS_ERR_COMM = -7,          /* NCCL error or peer-group abort; the communicator is aborted */
   QOS_ERR_UNSUPPORTED = -8    /* shape the kernels do not support (e.g. head_dim != 64/128) */
 };
 
@@ -95,6 +95,31 @@ int qos_engine_mem_sizes(const qos_model_cfg* cfg, int tp_size, qos_mem_sizes* o
 int qos_engine_create(const qos_model_cfg* cfg, int device, int tp_rank, int tp_size,
                       const uint8_t* nccl_uid, const qos_mem* mem, qos_engine_t** out);
 int qos_engine_destroy(qos_engine_t* eng);
+
+/* In-process peer group: the alternative to NCCL for tp_size > 1 when all TP ranks of one model
+ * live in ONE process (one engine and one host thread per rank, on one GPU or on GPUs with peer
+ * access over NVLink/NVSwitch).  The all-reduce after the O and down projections
+ * (vLLM TP, §3.6) is then one kernel per rank that reads every
+ * rank's bf16 partial straight from its workspace (peer loads), sums in fp32 in rank order (all
+ * ranks get bit-identical results) and fuses the residual add and the next RMSNorm
+ * (SURVEY.md §8(f) NEXT-2); the vocab-parallel logits are gathered the same way.  Ordering is by
+ * CUDA events: at each collective every rank records "partial ready", the host threads meet at a
+ * barrier (so every record precedes every wait), and each rank's stream waits on its peers'
+ * events — no kernel spins on another rank.
+ * Every rank must issue the same sequence of qos_hybrid_step / qos_profile_step calls, from its
+ * own thread, concurrently.  A rank that does not reach a collective within
+ * QOS_GROUP_TIMEOUT_MS (env, default 120000) aborts the group: the waiting calls return
+ * QOS_ERR_COMM and the group stays unusable.
+ * qos_group_create: tp_size in 2..8.  qos_group_destroy: after all its engines are destroyed
+ * (QOS_ERR_INVALID_ARG otherwise).  qos_engine_create_peer: as qos_engine_create with
+ * tp_size = the group's size; the ranks need identical configs; ranks on different devices
+ * enable peer access both ways (QOS_ERR_UNSUPPORTED without it); QOS_ERR_INVALID_ARG if the rank
+ * is already taken. */
+typedef struct qos_group qos_group_t;
+int qos_group_create(int tp_size, qos_group_t** out);
+int qos_group_destroy(qos_group_t* group);
+int qos_engine_create_peer(const qos_model_cfg* cfg, int device, int tp_rank, qos_group_t* group,
+                           const qos_mem* mem, qos_engine_t** out);
 
 /* This rank's slice under tensor parallelism (pure host function):
  * q heads [head0, head0+n_heads), kv heads [kv_head0, +n_kv_heads), FFN columns

@@ -316,13 +316,8 @@ static AttnParams to_params(const AttnLaunch& a) {
 template <int HD, int NS>
 static cudaError_t decode_t(const AttnLaunch& a, const DecodeItem* items, int n_items, float* partials, int* counters,
                             cudaStream_t st) {
-  static bool set = false;
-  if (!set) {
-    cudaError_t e = cudaFuncSetAttribute(decode_attn_kernel<HD, NS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         AttnCfg<HD, NS>::kSmemBytes);
-    if (e != cudaSuccess) return e;
-    set = true;
-  }
+  static std::atomic<uint64_t> set{0};
+  if (cudaError_t e = smem_attr_once(decode_attn_kernel<HD, NS>, int(AttnCfg<HD, NS>::kSmemBytes), set); e != cudaSuccess) return e;
   return launch_pdl(decode_attn_kernel<HD, NS>, dim3(n_items), dim3(kAttnThreads), AttnCfg<HD, NS>::kSmemBytes, st,
                     *a.kv_tmap, to_params(a), items, partials, counters);
 }

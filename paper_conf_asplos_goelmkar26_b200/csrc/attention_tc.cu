@@ -752,13 +752,8 @@ static int g_fa_poly = getenv("QOS_FA_POLY") ? atoi(getenv("QOS_FA_POLY")) : 4;
 template <int HD, int POLY, int NQ>
 static cudaError_t prefill_tc_t(const AttnLaunch& a, const PrefillItem* items, int n_items, cudaStream_t st) {
   using C = FaCfg<HD, NQ>;
-  static bool set = false;
-  if (!set) {
-    cudaError_t e = cudaFuncSetAttribute(prefill_attn_tc_kernel<HD, POLY, NQ>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         C::kSmem);
-    if (e != cudaSuccess) return e;
-    set = true;
-  }
+  static std::atomic<uint64_t> set{0};
+  if (cudaError_t e = smem_attr_once(prefill_attn_tc_kernel<HD, POLY, NQ>, int(C::kSmem), set); e != cudaSuccess) return e;
   FaParams p;
   p.q = reinterpret_cast<const __nv_bfloat16*>(a.q);
   p.q_ld = a.q_ld;
@@ -779,13 +774,8 @@ static cudaError_t prefill_tc_t(const AttnLaunch& a, const PrefillItem* items, i
 template <int HD, int POLY>
 static cudaError_t prefill_pp_t(const AttnLaunch& a, const PrefillItem* items, int n_items, cudaStream_t st) {
   using C = PpCfg<HD>;
-  static bool set = false;
-  if (!set) {
-    cudaError_t e = cudaFuncSetAttribute(prefill_attn_pp_kernel<HD, POLY>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         C::kSmem);
-    if (e != cudaSuccess) return e;
-    set = true;
-  }
+  static std::atomic<uint64_t> set{0};
+  if (cudaError_t e = smem_attr_once(prefill_attn_pp_kernel<HD, POLY>, int(C::kSmem), set); e != cudaSuccess) return e;
   FaParams p;
   p.q = reinterpret_cast<const __nv_bfloat16*>(a.q);
   p.q_ld = a.q_ld;

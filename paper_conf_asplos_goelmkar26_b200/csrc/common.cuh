@@ -8,6 +8,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <atomic>
 #include <utility>
 
 #define QOS_DEV __device__ __forceinline__
@@ -245,6 +246,19 @@ QOS_DEV void griddep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory");
 QOS_DEV void griddep_launch_dependents() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
 
 bool pdl_enabled();  // engine-wide switch (QOS_PDL=0 disables)
+
+// cudaFuncSetAttribute is per device: raise a kernel's dynamic smem limit once per device (bit per
+// device; engines of one process may sit on several GPUs, and a concurrent duplicate call is harmless)
+template <typename Kern>
+inline cudaError_t smem_attr_once(Kern kern, int bytes, std::atomic<uint64_t>& done) {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  const uint64_t bit = uint64_t(1) << (dev & 63);
+  if (done.load(std::memory_order_acquire) & bit) return cudaSuccess;
+  const cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+  if (e == cudaSuccess) done.fetch_or(bit, std::memory_order_release);
+  return e;
+}
 
 template <typename... KArgs, typename... Args>
 inline cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,

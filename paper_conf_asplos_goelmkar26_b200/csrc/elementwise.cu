@@ -152,6 +152,53 @@ __global__ void __launch_bounds__(kRowThreads) add_rmsnorm_kernel(float* __restr
   norm_row(r, g, out + size_t(t) * d, d, eps, red);
 }
 
+// Peer-memory TP reduction (in-process peer group, qos_engine_create_peer): row t of every
+// rank's bf16 partial (O or down projection output of its head / FFN slice) is
+// read straight from that rank's workspace (same device, or a peer GPU over NVLink), summed in
+// fp32 in rank order — so every rank computes the bit-identical sum — and added to the fp32
+// residual; with g != nullptr the row is then RMS-normalised into `out` (the next GEMM's A
+// operand).  One kernel replaces all-reduce + add + RMSNorm.  Ordering against the producers'
+// GEMMs is by stream events (engine.cu: peer_sync); loads bypass L1 (__ldcg).
+__global__ void __launch_bounds__(kRowThreads) peer_add_rmsnorm_kernel(PeerPtrs parts, int tp, float* __restrict__ resid,
+                                                                       const __nv_bfloat16* __restrict__ g,
+                                                                       __nv_bfloat16* __restrict__ out, int d,
+                                                                       float eps) {
+  griddep_wait();
+  griddep_launch_dependents();
+  __shared__ float red[32];
+  const int t = blockIdx.x;
+  float* r = resid + size_t(t) * d;
+  for (int c = threadIdx.x * 8; c < d; c += blockDim.x * 8) {
+    float s[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+    for (int k = 0; k < tp; ++k) {
+      const uint4 w = __ldcg(reinterpret_cast<const uint4*>(
+          reinterpret_cast<const __nv_bfloat16*>(parts.p[k]) + size_t(t) * d + c));
+      s[0] += bf16_lo(w.x); s[1] += bf16_hi(w.x); s[2] += bf16_lo(w.y); s[3] += bf16_hi(w.y);
+      s[4] += bf16_lo(w.z); s[5] += bf16_hi(w.z); s[6] += bf16_lo(w.w); s[7] += bf16_hi(w.w);
+    }
+    float4 x0 = *reinterpret_cast<float4*>(r + c), x1 = *reinterpret_cast<float4*>(r + c + 4);
+    x0.x += s[0]; x0.y += s[1]; x0.z += s[2]; x0.w += s[3];
+    x1.x += s[4]; x1.y += s[5]; x1.z += s[6]; x1.w += s[7];
+    *reinterpret_cast<float4*>(r + c) = x0;
+    *reinterpret_cast<float4*>(r + c + 4) = x1;
+  }
+  if (g) norm_row(r, g, out + size_t(t) * d, d, eps, red);  // same thread -> element map: no barrier
+}
+
+// Vocab-parallel LM head gather over peer memory: rank k's [R][Vl] f32 logits slice -> columns
+// [k*Vl, (k+1)*Vl) of out [R][tp*Vl].
+__global__ void peer_gather_logits_kernel(PeerPtrs loc, int tp, int R, int Vl, float* __restrict__ out) {
+  griddep_wait();
+  griddep_launch_dependents();
+  const int64_t per = int64_t(R) * Vl, n = per * tp;
+  for (int64_t i = blockIdx.x * int64_t(blockDim.x) + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x) {
+    const int k = int(i / per);
+    const int64_t rem = i - int64_t(k) * per;
+    const int r = int(rem / Vl), j = int(rem - int64_t(r) * Vl);
+    out[int64_t(r) * Vl * tp + int64_t(k) * Vl + j] = __ldcg(reinterpret_cast<const float*>(loc.p[k]) + rem);
+  }
+}
+
 __global__ void add_f32_kernel(float* __restrict__ resid, const __nv_bfloat16* __restrict__ add, int64_t n) {
   griddep_wait();
   griddep_launch_dependents();
@@ -300,6 +347,19 @@ cudaError_t launch_add_f32(float* resid, const void* add_bf16, size_t n, cudaStr
   if (n == 0) return cudaSuccess;
   count_launch();
   return launch_pdl(add_f32_kernel, dim3(grid_of(int64_t(n))), dim3(256), 0, st, resid, (const __nv_bfloat16*)add_bf16, int64_t(n));
+}
+cudaError_t launch_peer_add_rmsnorm(const PeerPtrs& parts, int tp, float* resid, const void* g, void* out, int T, int d,
+                                    float eps, cudaStream_t st) {
+  if (T == 0) return cudaSuccess;
+  count_launch();
+  return launch_pdl(peer_add_rmsnorm_kernel, dim3(T), dim3(kRowThreads), 0, st, parts, tp, resid,
+                    (const __nv_bfloat16*)g, (__nv_bfloat16*)out, d, eps);
+}
+cudaError_t launch_peer_gather_logits(const PeerPtrs& loc, int tp, int R, int Vl, float* out, cudaStream_t st) {
+  if (R == 0) return cudaSuccess;
+  count_launch();
+  return launch_pdl(peer_gather_logits_kernel, dim3(grid_of(int64_t(R) * Vl * tp)), dim3(256), 0, st, loc, tp, R, Vl,
+                    out);
 }
 cudaError_t launch_unshard_logits(const float* in, float* out, int R, int Vl, int tp, cudaStream_t st) {
   count_launch();

@@ -7,11 +7,13 @@
 
 #include <algorithm>
 #include <atomic>
+#include <chrono>
 #include <cmath>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
 #include <mutex>
+#include <condition_variable>
 #include <queue>
 #include <string>
 #include <unordered_map>
@@ -138,7 +140,7 @@ static WeightLayout weight_layout(const qos_model_cfg& c, const Shard& s) {
 }
 
 struct WsLayout {
-  size_t resid, h, qkv, attn, act, hR, logits, logits_loc, argmax, partials, counters, gemm_part, gemm_cnt, gemm_part2,
+  size_t resid, h, qkv, attn, act, hR, logits, logits_loc, part[2], argmax, partials, counters, gemm_part, gemm_cnt, gemm_part2,
       gemm_cnt2, meta[2], dbg, total;
   size_t meta_bytes;
   int max_items;
@@ -165,6 +167,9 @@ static WsLayout ws_layout(const qos_model_cfg& c, const Shard& s, int tp) {
   w.hR = take(Rm * d * 2);
   w.logits = take(Rm * size_t(c.vocab) * 4);
   w.logits_loc = tp > 1 ? take(Rm * size_t(c.vocab) * 4) : 0;
+  // peer-group TP: the O / down partials, double-buffered by collective parity (read by the peers)
+  w.part[0] = tp > 1 ? take(Tm * d * 2) : 0;
+  w.part[1] = tp > 1 ? take(Tm * d * 2) : 0;
   w.argmax = take(Rm * 4);
   w.max_items = kMaxDecodeItems;
   w.partials = take(size_t(w.max_items) * group * (hd + 2) * 4);
@@ -205,6 +210,45 @@ struct ReqState {
 }  // namespace qos
 
 using namespace qos;
+
+// In-process peer group (qos_group_create / qos_engine_create_peer): the TP ranks of one model
+// as engines of ONE process — one host thread per rank, on one GPU or on peer GPUs — whose
+// collectives are stream-event-ordered peer-memory kernels instead of NCCL (SURVEY.md §8(e),
+// §8(f) NEXT-2).  The host barrier only orders the ranks' ENQUEUEING at each collective (every
+// rank has recorded its "partial ready" event before any rank waits on it); the GPUs never spin.
+struct qos_group {
+  int n = 0;
+  std::vector<qos_engine*> eng;
+  std::mutex mu;
+  std::condition_variable cv;
+  int arrived = 0;
+  uint64_t gen = 0;
+  bool aborted = false;
+  int timeout_ms = 120000;
+
+  int barrier() {
+    std::unique_lock<std::mutex> lk(mu);
+    if (aborted) return qos::set_error(QOS_ERR_COMM, "peer group aborted");
+    const uint64_t g = gen;
+    if (++arrived == n) {
+      arrived = 0;
+      ++gen;
+      cv.notify_all();
+      return QOS_OK;
+    }
+    if (!cv.wait_for(lk, std::chrono::milliseconds(timeout_ms), [&] { return gen != g || aborted; })) {
+      aborted = true;
+      cv.notify_all();
+      return qos::set_error(QOS_ERR_COMM, "peer group barrier timed out (a rank did not reach the collective)");
+    }
+    return aborted ? qos::set_error(QOS_ERR_COMM, "peer group aborted") : QOS_OK;
+  }
+  void abort() {
+    std::lock_guard<std::mutex> lk(mu);
+    aborted = true;
+    cv.notify_all();
+  }
+};
 
 struct qos_engine {
   qos_model_cfg cfg{};
@@ -261,6 +305,11 @@ struct qos_engine {
   size_t ev_used = 0;
   // comm
   ncclComm_t comm = nullptr;
+  qos_group* group = nullptr;       // peer group (tp > 1 without NCCL)
+  bool shares_device = false;       // another rank of the group runs on this GPU: no cooperative
+                                    // (co-residency-dependent) GEMM reductions
+  uint64_t coll_seq = 0;            // collectives issued so far (identical on every rank)
+  cudaEvent_t ev_coll[2] = {nullptr, nullptr};  // "my partial is ready", by collective parity
   int64_t last_h2d = 0, last_d2h = 0;  // bytes moved host<->device by the last step
   // debug buffers for ops
   void* dbg = nullptr;
@@ -593,14 +642,14 @@ int gemm_any(qos_engine* e, const qos_engine::ActMap& am, const CUtensorMap (&tb
   if (N % 128 == 0 && (e->gemm_swab == 2 || (e->gemm_swab == 1 && swab_prefer(M, N, sms)))) {
     const int bnt = swab_pick_bnt(M);
     return gemm_swab_run(tb[0], am.sw[swab_index(bnt)], bnt, M, N, K, epi, C, ldc, bias, sms, st, part, cnt,
-                         int64_t(kGemmMaxUnits) * 128 * 256, kGemmMaxTiles, a_row0, rope, !e->dual_stream);
+                         int64_t(kGemmMaxUnits) * 128 * 256, kGemmMaxTiles, a_row0, rope, !e->dual_stream && !e->shares_device);
   }
   if (e->gemm_2cta && gemm2_eligible(M, N, K, sms))
     return gemm2_run(am.m128, tb[0], M, N, K, epi, C, ldc, bias, sms, st, a_row0, sms, rope);
   const int bn = gemm_pick_bn(M, N, epi, sms);
   const int ks = e->gemm_splitk ? gemm_pick_ksplit(M, N, K, bn, sms, kGemmMaxUnits) : 1;
   return gemm_run(am.m128, tb[bn == 256 ? 1 : 0], bn, M, N, K, epi, C, ldc, bias, sms, st, ks, part, cnt, a_row0, sms,
-                  rope, e->gemm_streamk, !e->dual_stream);
+                  rope, e->gemm_streamk, !e->dual_stream && !e->shares_device);
 }
 
 int gemm(qos_engine* e, const qos_engine::ActMap& am, const CUtensorMap (&tb)[2], int64_t M, int64_t N, int64_t K,
@@ -617,6 +666,56 @@ int allreduce_bf16(qos_engine* e, void* buf, size_t count, cudaStream_t st) {
     e->comm = nullptr;
     return set_error(QOS_ERR_COMM, g_nccl.errStr ? g_nccl.errStr(r) : "ncclAllReduce failed");
   }
+  return QOS_OK;
+}
+
+// Where the O / down projection of a TP rank writes its partial: `h` (reduced in place by NCCL)
+// or, in a peer group, this collective's parity buffer (read by every rank's reduction).  A
+// parity buffer is rewritten two collectives later, after this rank's stream has waited on every
+// peer's event of the collective in between, which each peer recorded after its reduction had
+// read the buffer.
+void* tp_partial_dst(qos_engine* e) {
+  return e->group ? e->ws + e->wsl.part[e->coll_seq & 1] : e->ws + e->wsl.h;
+}
+
+// Peer group: record "my input of this collective is ready", meet the other ranks' host threads,
+// then order this rank's stream after every peer's record (cross-device waits are legal).
+int peer_sync(qos_engine* e, cudaStream_t st) {
+  const int par = int(e->coll_seq & 1);
+  QOS_CU(cudaEventRecord(e->ev_coll[par], st));
+  QOS_TRY(e->group->barrier());
+  for (int k = 0; k < e->tp_size; ++k)
+    if (k != e->tp_rank) QOS_CU(cudaStreamWaitEvent(st, e->group->eng[size_t(k)]->ev_coll[par], 0));
+  return QOS_OK;
+}
+
+PeerPtrs peer_ptrs(qos_engine* e, size_t ws_off) {
+  PeerPtrs p{};
+  for (int k = 0; k < e->tp_size; ++k) p.p[k] = e->group->eng[size_t(k)]->ws + ws_off;
+  return p;
+}
+
+// a10 + a3: sum the ranks' partials into the fp32 residual, then RMSNorm with gain g into h
+// (g == nullptr after the last layer: add only).
+int tp_reduce_add_norm(qos_engine* e, const void* g, int T, cudaStream_t st) {
+  const int d = e->cfg.d_model;
+  float* resid = reinterpret_cast<float*>(e->ws + e->wsl.resid);
+  __nv_bfloat16* h = reinterpret_cast<__nv_bfloat16*>(e->ws + e->wsl.h);
+  if (!e->group) {
+    {
+      TimerScope ts(e, QOS_T_ALLREDUCE, st);
+      QOS_TRY(allreduce_bf16(e, h, size_t(T) * d, st));
+    }
+    TimerScope ts(e, QOS_T_NORM, st);
+    if (g) QOS_CU(launch_add_rmsnorm(resid, h, g, h, T, d, e->cfg.rms_eps, st));
+    else QOS_CU(launch_add_f32(resid, h, size_t(T) * d, st));
+    return QOS_OK;
+  }
+  TimerScope ts(e, QOS_T_ALLREDUCE, st);
+  QOS_TRY(peer_sync(e, st));
+  QOS_CU(launch_peer_add_rmsnorm(peer_ptrs(e, e->wsl.part[e->coll_seq & 1]), e->tp_size, resid, g, h, T, d,
+                                 e->cfg.rms_eps, st));
+  ++e->coll_seq;
   return QOS_OK;
 }
 
@@ -746,15 +845,13 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
       } else {
         {
           TimerScope ts(e, QOS_T_GEMM_O, gs);
-          QOS_TRY(gemm_seg(e, g, e->a_attn, M.o, d, e->sh.H * hd, EPI_STORE_BF16, h, d, nullptr));
+          QOS_TRY(gemm_seg(e, g, e->a_attn, M.o, d, e->sh.H * hd, EPI_STORE_BF16, tp_partial_dst(e), d, nullptr));
         }
-        TimerScope ts(e, QOS_T_ALLREDUCE, gs);
-        QOS_TRY(allreduce_bf16(e, h, size_t(T) * d, gs));
+        QOS_TRY(tp_reduce_add_norm(e, W(e, L.ln2), T, gs));
       }
-      {
+      if (!tp) {
         TimerScope ts(e, QOS_T_NORM, gs);
-        if (tp) QOS_CU(launch_add_rmsnorm(resid, h, W(e, L.ln2), h, T, d, c.rms_eps, gs));
-        else QOS_CU(launch_rmsnorm(resid + r0 * d, W(e, L.ln2), h + r0 * d, g.n, d, c.rms_eps, gs));
+        QOS_CU(launch_rmsnorm(resid + r0 * d, W(e, L.ln2), h + r0 * d, g.n, d, c.rms_eps, gs));
       }
       {
         TimerScope ts(e, QOS_T_GEMM_GATEUP, gs);
@@ -766,19 +863,9 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
       } else {
         {
           TimerScope ts(e, QOS_T_GEMM_DOWN, gs);
-          QOS_TRY(gemm_seg(e, g, e->a_act, M.d, d, e->sh.F, EPI_STORE_BF16, h, d, nullptr));
+          QOS_TRY(gemm_seg(e, g, e->a_act, M.d, d, e->sh.F, EPI_STORE_BF16, tp_partial_dst(e), d, nullptr));
         }
-        {
-          TimerScope ts(e, QOS_T_ALLREDUCE, gs);
-          QOS_TRY(allreduce_bf16(e, h, size_t(T) * d, gs));
-        }
-        if (l + 1 < c.n_layers) {
-          TimerScope ts(e, QOS_T_NORM, gs);
-          QOS_CU(launch_add_rmsnorm(resid, h, W(e, e->wl.layers[l + 1].ln1), h, T, d, c.rms_eps, gs));
-        } else {
-          TimerScope ts(e, QOS_T_NORM, gs);
-          QOS_CU(launch_add_f32(resid, h, size_t(T) * d, gs));
-        }
+        QOS_TRY(tp_reduce_add_norm(e, l + 1 < c.n_layers ? W(e, e->wl.layers[l + 1].ln1) : nullptr, T, gs));
       }
     }
   }
@@ -802,12 +889,18 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
     } else {
       float* loc = reinterpret_cast<float*>(e->ws + s.logits_loc);
       QOS_TRY(gemm(e, e->a_hR, e->head_map, R, e->sh.V, d, EPI_STORE_F32, loc, e->sh.V, nullptr, st));
+      if (e->group) {  // peer group: read every rank's vocab slice directly
+        QOS_TRY(peer_sync(e, st));
+        QOS_CU(launch_peer_gather_logits(peer_ptrs(e, s.logits_loc), e->tp_size, R, e->sh.V, lg, st));
+        ++e->coll_seq;
+      } else {
       // all-gather of [R][V/tp] shards -> [tp][R][V/tp], then transpose into [R][V]
       ncclResult_t r = g_nccl.allGather(loc, lg, size_t(R) * e->sh.V, ncclFloat32, e->comm, st);
       if (r != ncclSuccess) return set_error(QOS_ERR_COMM, "ncclAllGather failed");
       // gathered layout [tp][R][V/tp] -> [R][V] (logits_loc holds Rm*V floats when tp > 1)
       QOS_CU(launch_unshard_logits(lg, loc, R, e->sh.V, e->tp_size, st));
       lout = loc;
+      }
     }
   }
   {
@@ -850,7 +943,11 @@ int do_step(qos_engine* e, const qos_batch* b, void* logits, int logits_dtype, i
     TimerScope ts(e, QOS_T_META, st);
     QOS_TRY(upload_meta(e, m, st, &dm));
   }
-  QOS_TRY(run_layers(e, m, dm, logits, logits_dtype, next_tokens, !on_host, st));
+  r = run_layers(e, m, dm, logits, logits_dtype, next_tokens, !on_host, st);
+  if (r != QOS_OK) {
+    if (e->group) e->group->abort();  // the peers would wait for this rank's collectives
+    return r;
+  }
   QOS_TRY(release_staging(e, st));
   e->last_h2d = int64_t(m.used);
   e->last_d2h = on_host ? int64_t(m.R) * ((next_tokens ? 4 : 0) +
@@ -878,7 +975,7 @@ const char* qos_strerror(int code) {
     case QOS_ERR_BAD_KV_START: return "kv_start/ctx_len does not match cached length";
     case QOS_ERR_NOT_ALLOCATED: return "KV blocks not allocated";
     case QOS_ERR_CUDA: return "CUDA error";
-    case QOS_ERR_COMM: return "NCCL error";
+    case QOS_ERR_COMM: return "communication error (NCCL or peer group)";
     case QOS_ERR_UNSUPPORTED: return "unsupported shape";
     default: return "unknown error";
   }
@@ -912,12 +1009,33 @@ int qos_nccl_unique_id(uint8_t out[128]) {
   return QOS_OK;
 }
 
-int qos_engine_create(const qos_model_cfg* cfg, int device, int tp_rank, int tp_size, const uint8_t* nccl_uid,
-                      const qos_mem* mem, qos_engine_t** out) {
+int qos_group_create(int tp_size, qos_group_t** out) {
+  if (!out || tp_size < 2 || tp_size > kMaxPeers) return set_error(QOS_ERR_INVALID_ARG, "group size must be 2..8");
+  auto* g = new qos_group();
+  g->n = tp_size;
+  g->eng.assign(size_t(tp_size), nullptr);
+  if (const char* t = getenv("QOS_GROUP_TIMEOUT_MS")) g->timeout_ms = atoi(t);
+  *out = g;
+  return QOS_OK;
+}
+
+int qos_group_destroy(qos_group_t* g) {
+  if (!g) return QOS_OK;
+  {
+    std::lock_guard<std::mutex> lk(g->mu);
+    for (auto* e : g->eng)
+      if (e) return set_error(QOS_ERR_INVALID_ARG, "destroy the group's engines first");
+  }
+  delete g;
+  return QOS_OK;
+}
+
+static int create_engine(const qos_model_cfg* cfg, int device, int tp_rank, int tp_size, const uint8_t* nccl_uid,
+                         qos_group* group, const qos_mem* mem, qos_engine_t** out) {
   QOS_TRY(check_cfg(cfg, tp_size));
   if (!out) return set_error(QOS_ERR_INVALID_ARG, "out is NULL");
   if (tp_rank < 0 || tp_rank >= tp_size) return set_error(QOS_ERR_INVALID_ARG, "tp_rank");
-  if (tp_size > 1 && !nccl_uid) return set_error(QOS_ERR_INVALID_ARG, "nccl_uid required for tp_size > 1");
+  if (tp_size > 1 && !nccl_uid && !group) return set_error(QOS_ERR_INVALID_ARG, "nccl_uid required for tp_size > 1");
   QOS_CU(cudaSetDevice(device));
   auto* e = new qos_engine();
   e->cfg = *cfg;
@@ -1006,7 +1124,32 @@ int qos_engine_create(const qos_model_cfg* cfg, int device, int tp_rank, int tp_
   e->free_rows.resize(size_t(cfg->max_requests));
   for (int i = 0; i < cfg->max_requests; ++i) e->free_rows[size_t(i)] = i;
   if ((r = build_maps(e)) != QOS_OK) return fail(r);
-  if (tp_size > 1) {
+  if (group) {
+    for (int i = 0; i < 2; ++i) cudaEventCreateWithFlags(&e->ev_coll[i], cudaEventDisableTiming);
+    std::lock_guard<std::mutex> lk(group->mu);
+    if (group->eng[size_t(tp_rank)]) return fail(set_error(QOS_ERR_INVALID_ARG, "tp_rank already in the group"));
+    for (auto* p : group->eng) {
+      if (!p) continue;
+      if (std::memcmp(&p->cfg, cfg, sizeof(*cfg)) != 0)
+        return fail(set_error(QOS_ERR_INVALID_ARG, "group ranks need identical model configs"));
+      if (p->device == device) p->shares_device = e->shares_device = true;
+      if (p->device != device) {  // peer reads in both directions over NVLink
+        int ok1 = 0, ok2 = 0;
+        cudaDeviceCanAccessPeer(&ok1, device, p->device);
+        cudaDeviceCanAccessPeer(&ok2, p->device, device);
+        if (!ok1 || !ok2) return fail(set_error(QOS_ERR_UNSUPPORTED, "group devices lack peer access"));
+        cudaError_t a = cudaDeviceEnablePeerAccess(p->device, 0);
+        if (a != cudaSuccess && a != cudaErrorPeerAccessAlreadyEnabled) return fail(set_cuda_error(a, "peer access"));
+        cudaSetDevice(p->device);
+        a = cudaDeviceEnablePeerAccess(device, 0);
+        cudaSetDevice(device);
+        if (a != cudaSuccess && a != cudaErrorPeerAccessAlreadyEnabled) return fail(set_cuda_error(a, "peer access"));
+        cudaGetLastError();
+      }
+    }
+    group->eng[size_t(tp_rank)] = e;
+    e->group = group;
+  } else if (tp_size > 1) {
     std::lock_guard<std::mutex> g(g_nccl_mu);
     if (!g_nccl.load()) return fail(set_error(QOS_ERR_COMM, "libnccl.so.2 not loadable"));
     ncclUniqueId id;
@@ -1019,10 +1162,27 @@ int qos_engine_create(const qos_model_cfg* cfg, int device, int tp_rank, int tp_
   return QOS_OK;
 }
 
+int qos_engine_create(const qos_model_cfg* cfg, int device, int tp_rank, int tp_size, const uint8_t* nccl_uid,
+                      const qos_mem* mem, qos_engine_t** out) {
+  return create_engine(cfg, device, tp_rank, tp_size, nccl_uid, nullptr, mem, out);
+}
+
+int qos_engine_create_peer(const qos_model_cfg* cfg, int device, int tp_rank, qos_group_t* group, const qos_mem* mem,
+                           qos_engine_t** out) {
+  if (!group) return set_error(QOS_ERR_INVALID_ARG, "group is NULL");
+  return create_engine(cfg, device, tp_rank, group->n, nullptr, group, mem, out);
+}
+
 int qos_engine_destroy(qos_engine_t* e) {
   if (!e) return QOS_OK;
   cudaSetDevice(e->device);
   cudaDeviceSynchronize();
+  if (e->group) {
+    std::lock_guard<std::mutex> lk(e->group->mu);
+    if (e->group->eng[size_t(e->tp_rank)] == e) e->group->eng[size_t(e->tp_rank)] = nullptr;
+  }
+  for (auto ev : e->ev_coll)
+    if (ev) cudaEventDestroy(ev);
   if (e->comm && g_nccl.commDestroy) g_nccl.commDestroy(e->comm);
   if (e->own_w) cudaFree(e->w);
   if (e->own_kv) cudaFree(e->kv);

@@ -1029,12 +1029,8 @@ template <int BN, int EPI>
 static cudaError_t launch_gemm_t(const CUtensorMap& ta, const CUtensorMap& tb, const GemmArgs& a, int grid,
                                  cudaStream_t st) {
   auto kern = gemm_tcgen05_kernel<BN, EPI>;
-  static bool attr_set = false;  // per template instantiation
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, GemmCfg<BN>::kSmemBytes);
-    if (e != cudaSuccess) return e;
-    attr_set = true;
-  }
+  static std::atomic<uint64_t> attr_set{0};
+  if (cudaError_t e = smem_attr_once(kern, int(GemmCfg<BN>::kSmemBytes), attr_set); e != cudaSuccess) return e;
   return launch_pdl(kern, dim3(grid), dim3(kGemmThreads), GemmCfg<BN>::kSmemBytes, st, ta, tb, a);
 }
 
@@ -1123,12 +1119,8 @@ template <int EPI>
 static cudaError_t launch_gemm2_t(const CUtensorMap& ta, const CUtensorMap& tb, const GemmArgs& a, int grid,
                                   cudaStream_t st) {
   auto kern = gemm2_tcgen05_kernel<EPI>;
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kG2Smem);
-    if (e != cudaSuccess) return e;
-    attr_set = true;
-  }
+  static std::atomic<uint64_t> attr_set{0};
+  if (cudaError_t e = smem_attr_once(kern, int(kG2Smem), attr_set); e != cudaSuccess) return e;
   return launch_pdl_cluster(kern, dim3(grid), dim3(kGemmThreads), kG2Smem, 2, st, ta, tb, a);
 }
 

@@ -399,12 +399,8 @@ template <int BNT, int EPI>
 cudaError_t launch_swab_t(const CUtensorMap& tw, const CUtensorMap& tt, const SwabArgs& a, int grid,
                           cudaStream_t st) {
   auto kern = gemm_swab_kernel<BNT, EPI>;
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SwCfg<BNT>::kSmemBytes);
-    if (e != cudaSuccess) return e;
-    attr_set = true;
-  }
+  static std::atomic<uint64_t> attr_set{0};
+  if (cudaError_t e = smem_attr_once(kern, int(SwCfg<BNT>::kSmemBytes), attr_set); e != cudaSuccess) return e;
   return launch_pdl(kern, dim3(grid), dim3(kSwThreads), SwCfg<BNT>::kSmemBytes, st, tw, tt, a);
 }
 

@@ -102,6 +102,16 @@ cudaError_t launch_add_rmsnorm(float* resid, const void* add, const void* g, voi
 cudaError_t launch_add_f32(float* resid, const void* add_bf16, size_t n, cudaStream_t st);
 // [tp][R][Vl] -> [R][tp*Vl]
 cudaError_t launch_unshard_logits(const float* in, float* out, int R, int Vl, int tp, cudaStream_t st);
+// in-process peer group (tp > 1 without NCCL): pointers to every rank's buffer, rank order
+constexpr int kMaxPeers = 8;
+struct PeerPtrs {
+  const void* p[kMaxPeers];
+};
+// resid += sum_k parts[k] (bf16, fp32 sum in rank order); out = RMSNorm(resid) * g if g != NULL
+cudaError_t launch_peer_add_rmsnorm(const PeerPtrs& parts, int tp, float* resid, const void* g, void* out, int T, int d,
+                                    float eps, cudaStream_t st);
+// out[R][tp*Vl] <- rank k's [R][Vl] slice
+cudaError_t launch_peer_gather_logits(const PeerPtrs& loc, int tp, int R, int Vl, float* out, cudaStream_t st);
 cudaError_t launch_argmax(const void* logits, int logits_f32, int R, int V, int32_t* out, cudaStream_t st);
 cudaError_t launch_f32_to_bf16(const float* x, void* y, int64_t n, cudaStream_t st);
 

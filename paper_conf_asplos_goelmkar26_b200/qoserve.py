@@ -80,6 +80,9 @@ _SIGS = {
     "qos_engine_create": [C.POINTER(qos_model_cfg), C.c_int, C.c_int, C.c_int, C.c_char_p,
                           C.POINTER(qos_mem), C.POINTER(_P)],
     "qos_engine_destroy": [_P],
+    "qos_group_create": [C.c_int, C.POINTER(_P)],
+    "qos_group_destroy": [_P],
+    "qos_engine_create_peer": [C.POINTER(qos_model_cfg), C.c_int, C.c_int, _P, C.POINTER(qos_mem), C.POINTER(_P)],
     "qos_nccl_unique_id": [C.c_char_p],
     "qos_shard_plan": [C.POINTER(qos_model_cfg), C.c_int, C.c_int, C.POINTER(qos_shard)],
     "qos_engine_load_synthetic": [_P, C.c_uint64],
@@ -205,11 +208,36 @@ def model_cfg(n_layers, d_model, n_heads, n_kv_heads, head_dim, ffn_dim, vocab, 
                          max_batch_rows)
 
 
+class Group:
+    """In-process peer group of tp_size ranks (qos_group_create); destroy after its engines."""
+
+    def __init__(self, tp_size: int):
+        self.tp_size = tp_size
+        h = _P()
+        _call("qos_group_create", tp_size, C.byref(h))
+        self.h = h
+
+    def close(self):
+        if getattr(self, "h", None):
+            _call("qos_group_destroy", self.h)
+            self.h = None
+
+
+def run_ranks(fn, engines):
+    """Call fn(rank, engine) on one thread per rank (a peer group's ranks must step concurrently;
+    ctypes releases the GIL during the C calls).  Returns the per-rank results; re-raises the
+    first failure."""
+    import concurrent.futures as cf
+    with cf.ThreadPoolExecutor(max_workers=len(engines)) as ex:
+        futs = [ex.submit(fn, r, e) for r, e in enumerate(engines)]
+        return [f.result() for f in futs]
+
+
 class Engine:
     """One libqoserve engine on one GPU (one TP rank).  Device arenas are torch tensors."""
 
     def __init__(self, cfg: qos_model_cfg, device: int = 0, tp_rank: int = 0, tp_size: int = 1,
-                 nccl_uid: bytes | None = None, torch_arenas: bool = True):
+                 nccl_uid: bytes | None = None, torch_arenas: bool = True, group: "Group | None" = None):
         import torch
         self.cfg = cfg
         self.device = device
@@ -224,9 +252,15 @@ class Engine:
             self._arenas = arenas
             mem = qos_mem(arenas[0].data_ptr(), arenas[1].data_ptr(), arenas[2].data_ptr())
         h = _P()
-        _call("qos_engine_create", C.byref(cfg), device, tp_rank, tp_size, nccl_uid,
-              C.byref(mem) if mem is not None else None, C.byref(h))
+        if group is not None:
+            assert tp_size == group.tp_size
+            _call("qos_engine_create_peer", C.byref(cfg), device, tp_rank, group.h,
+                  C.byref(mem) if mem is not None else None, C.byref(h))
+        else:
+            _call("qos_engine_create", C.byref(cfg), device, tp_rank, tp_size, nccl_uid,
+                  C.byref(mem) if mem is not None else None, C.byref(h))
         self.h = h
+        self.group = group
 
     def close(self):
         if getattr(self, "h", None):

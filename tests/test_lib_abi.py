@@ -73,3 +73,15 @@ def test_engine_create_fails_loudly_without_gpu(q):
     with pytest.raises(q.QosError) as ei:
         q.Engine(cfg, torch_arenas=False)
     assert ei.value.name in ("CUDA", "OOM")
+
+
+def test_peer_group_host_calls(q):
+    """qos_group_create / qos_group_destroy are pure host calls (the in-process TP peer group)."""
+    with pytest.raises(q.QosError) as ei:
+        q.Group(1)
+    assert ei.value.name == "INVALID_ARG"
+    with pytest.raises(q.QosError):
+        q.Group(9)
+    g = q.Group(4)
+    g.close()
+    g.close()  # idempotent in the binding
