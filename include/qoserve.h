@@ -244,6 +244,10 @@ int qos_profile_step_ex(qos_engine_t* eng, int32_t chunk_len, int32_t kv_start,
  *                          K/V tile (1: two CTAs per SM with 2-deep K/V rings; 2: one CTA per
  *                          SM, half the L2 -> SM traffic, 4-deep rings; measured ~6% more
  *                          cycles than 1, tools/ncu_ab.py)
+ *   "tp_twoshot" (-1)      peer-group TP reduction: 0 one-shot (every rank reads all partials of
+ *                          all rows), 1 two-shot (each rank reduces + normalises a row slice and
+ *                          stores it into every peer: ~2(tp-1)/tp of one partial per rank instead
+ *                          of tp-1), -1 automatic (two-shot when tp >= 4)
  *   "gemm_2cta" (1)        CTA-pair GEMM (tcgen05 cta_group::2, 256 x 256 tiles) where it
  *                          needs no more waves than 128 x 256 single-CTA tiles; env QOS_GEMM_2CTA
  * Results do not depend on the options (parity tests run with the defaults and variants). */

@@ -185,6 +185,55 @@ __global__ void __launch_bounds__(kRowThreads) peer_add_rmsnorm_kernel(PeerPtrs 
   if (g) norm_row(r, g, out + size_t(t) * d, d, eps, red);  // same thread -> element map: no barrier
 }
 
+// Two-shot form of the same reduction for larger groups (tp >= 4): rank `rank` reduces only the
+// rows [row0, row0 + gridDim.x) it owns (reduce-scatter by row slices: reads (tp-1)/tp of one
+// partial instead of tp-1 partials), adds them to its residual rows, normalises them into its own
+// h and stores the normalised bf16 rows into every peer's h (the all-gather, by peer stores).
+// store_resid (last layer, g == nullptr): the updated fp32 residual rows are stored into every
+// peer's residual instead, so the final gather + norm of the logit rows sees fresh rows.
+__global__ void __launch_bounds__(kRowThreads) peer_rs_norm_ag_kernel(PeerPtrs parts, PeerPtrs hs, PeerPtrs resids,
+                                                                      int tp, int rank, int row0,
+                                                                      const __nv_bfloat16* __restrict__ g, int d,
+                                                                      float eps) {
+  griddep_wait();
+  griddep_launch_dependents();
+  __shared__ float red[32];
+  const int t = row0 + blockIdx.x;
+  float* r = reinterpret_cast<float*>(const_cast<void*>(resids.p[rank])) + size_t(t) * d;
+  for (int c = threadIdx.x * 8; c < d; c += blockDim.x * 8) {
+    float s[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+    for (int k = 0; k < tp; ++k) {
+      const uint4 w = __ldcg(reinterpret_cast<const uint4*>(
+          reinterpret_cast<const __nv_bfloat16*>(parts.p[k]) + size_t(t) * d + c));
+      s[0] += bf16_lo(w.x); s[1] += bf16_hi(w.x); s[2] += bf16_lo(w.y); s[3] += bf16_hi(w.y);
+      s[4] += bf16_lo(w.z); s[5] += bf16_hi(w.z); s[6] += bf16_lo(w.w); s[7] += bf16_hi(w.w);
+    }
+    float4 x0 = *reinterpret_cast<float4*>(r + c), x1 = *reinterpret_cast<float4*>(r + c + 4);
+    x0.x += s[0]; x0.y += s[1]; x0.z += s[2]; x0.w += s[3];
+    x1.x += s[4]; x1.y += s[5]; x1.z += s[6]; x1.w += s[7];
+    *reinterpret_cast<float4*>(r + c) = x0;
+    *reinterpret_cast<float4*>(r + c + 4) = x1;
+    if (!g) {
+      for (int k = 0; k < tp; ++k) {
+        if (k == rank) continue;
+        float* pr = reinterpret_cast<float*>(const_cast<void*>(resids.p[k])) + size_t(t) * d + c;
+        *reinterpret_cast<float4*>(pr) = x0;
+        *reinterpret_cast<float4*>(pr + 4) = x1;
+      }
+    }
+  }
+  if (!g) return;
+  __nv_bfloat16* own = reinterpret_cast<__nv_bfloat16*>(const_cast<void*>(hs.p[rank])) + size_t(t) * d;
+  norm_row(r, g, own, d, eps, red);
+  // the thread re-reads only the h elements it wrote and forwards them to the peers
+  for (int c = threadIdx.x * 8; c < d; c += blockDim.x * 8) {
+    const uint4 v = *reinterpret_cast<const uint4*>(own + c);
+    for (int k = 0; k < tp; ++k)
+      if (k != rank)
+        *reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(const_cast<void*>(hs.p[k])) + size_t(t) * d + c) = v;
+  }
+}
+
 // Vocab-parallel LM head gather over peer memory: rank k's [R][Vl] f32 logits slice -> columns
 // [k*Vl, (k+1)*Vl) of out [R][tp*Vl].
 __global__ void peer_gather_logits_kernel(PeerPtrs loc, int tp, int R, int Vl, float* __restrict__ out) {
@@ -354,6 +403,13 @@ cudaError_t launch_peer_add_rmsnorm(const PeerPtrs& parts, int tp, float* resid,
   count_launch();
   return launch_pdl(peer_add_rmsnorm_kernel, dim3(T), dim3(kRowThreads), 0, st, parts, tp, resid,
                     (const __nv_bfloat16*)g, (__nv_bfloat16*)out, d, eps);
+}
+cudaError_t launch_peer_rs_norm_ag(const PeerPtrs& parts, const PeerPtrs& hs, const PeerPtrs& resids, int tp, int rank,
+                                   int row0, int nrows, const void* g, int d, float eps, cudaStream_t st) {
+  if (nrows <= 0) return cudaSuccess;
+  count_launch();
+  return launch_pdl(peer_rs_norm_ag_kernel, dim3(nrows), dim3(kRowThreads), 0, st, parts, hs, resids, tp, rank, row0,
+                    (const __nv_bfloat16*)g, d, eps);
 }
 cudaError_t launch_peer_gather_logits(const PeerPtrs& loc, int tp, int R, int Vl, float* out, cudaStream_t st) {
   if (R == 0) return cudaSuccess;

@@ -308,8 +308,10 @@ struct qos_engine {
   qos_group* group = nullptr;       // peer group (tp > 1 without NCCL)
   bool shares_device = false;       // another rank of the group runs on this GPU: no cooperative
                                     // (co-residency-dependent) GEMM reductions
-  uint64_t coll_seq = 0;            // collectives issued so far (identical on every rank)
-  cudaEvent_t ev_coll[2] = {nullptr, nullptr};  // "my partial is ready", by collective parity
+  uint64_t sync_seq = 0;            // peer syncs issued so far (identical on every rank)
+  uint64_t red_seq = 0;             // O / down reductions issued so far (partial buffer parity)
+  cudaEvent_t ev_coll[2] = {nullptr, nullptr};  // "my side of this sync is ready", by sync parity
+  int tp_twoshot = -1;              // option tp_twoshot: 0 one-shot, 1 two-shot, -1 auto (tp >= 4)
   int64_t last_h2d = 0, last_d2h = 0;  // bytes moved host<->device by the last step
   // debug buffers for ops
   void* dbg = nullptr;
@@ -675,13 +677,15 @@ int allreduce_bf16(qos_engine* e, void* buf, size_t count, cudaStream_t st) {
 // peer's event of the collective in between, which each peer recorded after its reduction had
 // read the buffer.
 void* tp_partial_dst(qos_engine* e) {
-  return e->group ? e->ws + e->wsl.part[e->coll_seq & 1] : e->ws + e->wsl.h;
+  return e->group ? e->ws + e->wsl.part[e->red_seq & 1] : e->ws + e->wsl.h;
 }
 
 // Peer group: record "my input of this collective is ready", meet the other ranks' host threads,
 // then order this rank's stream after every peer's record (cross-device waits are legal).
+// An event of parity x is re-recorded two syncs later, i.e. after the barrier of the sync in
+// between, which every rank reaches only after it has issued its waits on this one.
 int peer_sync(qos_engine* e, cudaStream_t st) {
-  const int par = int(e->coll_seq & 1);
+  const int par = int(e->sync_seq++ & 1);
   QOS_CU(cudaEventRecord(e->ev_coll[par], st));
   QOS_TRY(e->group->barrier());
   for (int k = 0; k < e->tp_size; ++k)
@@ -712,10 +716,18 @@ int tp_reduce_add_norm(qos_engine* e, const void* g, int T, cudaStream_t st) {
     return QOS_OK;
   }
   TimerScope ts(e, QOS_T_ALLREDUCE, st);
-  QOS_TRY(peer_sync(e, st));
-  QOS_CU(launch_peer_add_rmsnorm(peer_ptrs(e, e->wsl.part[e->coll_seq & 1]), e->tp_size, resid, g, h, T, d,
-                                 e->cfg.rms_eps, st));
-  ++e->coll_seq;
+  const PeerPtrs parts = peer_ptrs(e, e->wsl.part[e->red_seq++ & 1]);
+  QOS_TRY(peer_sync(e, st));  // every rank's partial is complete
+  const bool two = e->tp_twoshot > 0 || (e->tp_twoshot < 0 && e->tp_size >= 4);
+  if (!two) {
+    QOS_CU(launch_peer_add_rmsnorm(parts, e->tp_size, resid, g, h, T, d, e->cfg.rms_eps, st));
+    return QOS_OK;
+  }
+  // two-shot: this rank reduces + normalises its row slice and stores the rows into every peer
+  const int rs = (T + e->tp_size - 1) / e->tp_size, row0 = std::min(T, e->tp_rank * rs);
+  QOS_CU(launch_peer_rs_norm_ag(parts, peer_ptrs(e, e->wsl.h), peer_ptrs(e, e->wsl.resid), e->tp_size, e->tp_rank,
+                                row0, std::min(rs, T - row0), g, d, e->cfg.rms_eps, st));
+  QOS_TRY(peer_sync(e, st));  // every rank's rows have landed in every h (or residual)
   return QOS_OK;
 }
 
@@ -892,7 +904,6 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
       if (e->group) {  // peer group: read every rank's vocab slice directly
         QOS_TRY(peer_sync(e, st));
         QOS_CU(launch_peer_gather_logits(peer_ptrs(e, s.logits_loc), e->tp_size, R, e->sh.V, lg, st));
-        ++e->coll_seq;
       } else {
       // all-gather of [R][V/tp] shards -> [tp][R][V/tp], then transpose into [R][V]
       ncclResult_t r = g_nccl.allGather(loc, lg, size_t(R) * e->sh.V, ncclFloat32, e->comm, st);
@@ -1489,6 +1500,7 @@ int qos_engine_set_option(qos_engine_t* e, const char* name, int64_t value) {
   if (n == "overlap_attn") e->overlap_attn = value != 0;
   else if (n == "decode_round_split") e->decode_round_split = value != 0;
   else if (n == "gemm_2cta") e->gemm_2cta = value != 0;
+  else if (n == "tp_twoshot") e->tp_twoshot = value < 0 ? -1 : value > 0 ? 1 : 0;
   else if (n == "decode_stages") {
     if (value != 4 && value != 8) return set_error(QOS_ERR_INVALID_ARG, "decode_stages must be 4 or 8");
     e->decode_stages = int(value);

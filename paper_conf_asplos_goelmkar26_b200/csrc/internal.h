@@ -110,6 +110,11 @@ struct PeerPtrs {
 // resid += sum_k parts[k] (bf16, fp32 sum in rank order); out = RMSNorm(resid) * g if g != NULL
 cudaError_t launch_peer_add_rmsnorm(const PeerPtrs& parts, int tp, float* resid, const void* g, void* out, int T, int d,
                                     float eps, cudaStream_t st);
+// two-shot: rank `rank` reduces rows [row0, row0+nrows) into its residual, normalises them and
+// stores the bf16 rows into every rank's h (hs); g == NULL: stores the fp32 residual rows into
+// every rank's residual (resids) instead
+cudaError_t launch_peer_rs_norm_ag(const PeerPtrs& parts, const PeerPtrs& hs, const PeerPtrs& resids, int tp, int rank,
+                                   int row0, int nrows, const void* g, int d, float eps, cudaStream_t st);
 // out[R][tp*Vl] <- rank k's [R][Vl] slice
 cudaError_t launch_peer_gather_logits(const PeerPtrs& loc, int tp, int R, int Vl, float* out, cudaStream_t st);
 cudaError_t launch_argmax(const void* logits, int logits_f32, int R, int V, int32_t* out, cudaStream_t st);
