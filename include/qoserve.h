@@ -118,6 +118,17 @@ int qos_engine_destroy(qos_engine_t* eng);
 typedef struct qos_group qos_group_t;
 int qos_group_create(int tp_size, qos_group_t** out);
 int qos_group_destroy(qos_group_t* group);
+/* Cross-process form of the peer group: one process (and one engine) per rank on one node, e.g.
+ * one process per GPU under torchrun.  Rank 0 calls qos_group_unique_id (a NUL-terminated POSIX
+ * shared-memory name in 64 bytes) and broadcasts it (e.g. over torch.distributed); every rank
+ * then calls qos_group_open with it (rank 0 creates the segment, the others wait for it up to
+ * QOS_GROUP_TIMEOUT_MS) and qos_engine_create_peer with tp_rank = its group rank.  Engine
+ * creation and destruction are collective: each rank exports its workspace (CUDA IPC memory
+ * handle) and its two sync events (interprocess events) and maps its peers'; the barrier is a
+ * spin barrier in the segment.  Collectives, ordering, abort and results are as above.  The
+ * segment is unlinked when the last rank destroys its group. */
+int qos_group_unique_id(uint8_t out[64]);
+int qos_group_open(const uint8_t id[64], int tp_size, int tp_rank, qos_group_t** out);
 int qos_engine_create_peer(const qos_model_cfg* cfg, int device, int tp_rank, qos_group_t* group,
                            const qos_mem* mem, qos_engine_t** out);
 

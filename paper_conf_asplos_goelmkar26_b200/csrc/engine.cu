@@ -4,6 +4,11 @@
 // builder that turns a QoServe batch descriptor (all decodes + the
 // deadline-selected prefill chunks, Alg. 1) into the kernels' work lists.
 #include <dlfcn.h>
+#include <fcntl.h>
+#include <sched.h>
+#include <sys/mman.h>
+#include <sys/stat.h>
+#include <unistd.h>
 
 #include <algorithm>
 #include <atomic>
@@ -18,7 +23,10 @@
 #include <string>
 #include <unordered_map>
 #include <unordered_set>
+#include <array>
+#include <random>
 #include <vector>
+#include <memory>
 
 #include "internal.h"
 #include <cuda_bf16.h>
@@ -216,6 +224,26 @@ using namespace qos;
 // collectives are stream-event-ordered peer-memory kernels instead of NCCL (SURVEY.md §8(e),
 // §8(f) NEXT-2).  The host barrier only orders the ranks' ENQUEUEING at each collective (every
 // rank has recorded its "partial ready" event before any rank waits on it); the GPUs never spin.
+// Cross-process form (qos_group_open; one process per GPU on one node): the same collectives
+// over CUDA IPC — every rank exports its workspace and its two sync events (interprocess
+// events) through a POSIX shared-memory segment, opens its peers' at engine creation, and the
+// host barrier is a spin barrier in that segment.
+struct IpcSlot {
+  cudaIpcMemHandle_t ws;
+  uint64_t ws_off;                 // workspace offset inside the exported allocation
+  cudaIpcEventHandle_t ev[2];
+  uint8_t uuid[16];                // device UUID (ranks sharing a GPU disable cooperative GEMMs)
+  qos_model_cfg cfg;
+};
+struct IpcShm {
+  static constexpr uint64_t kMagic = 0x716f7367726f7570ull;  // "qosgroup"
+  std::atomic<uint64_t> magic;
+  std::atomic<uint64_t> gen;
+  std::atomic<int32_t> arrived, aborted, attached;
+  int32_t n;
+  IpcSlot slot[8];
+};
+
 struct qos_group {
   int n = 0;
   std::vector<qos_engine*> eng;
@@ -225,8 +253,14 @@ struct qos_group {
   uint64_t gen = 0;
   bool aborted = false;
   int timeout_ms = 120000;
+  // cross-process group
+  bool ipc = false;
+  int rank = -1;
+  IpcShm* shm = nullptr;
+  std::string shm_name;
 
   int barrier() {
+    if (ipc) return ipc_barrier();
     std::unique_lock<std::mutex> lk(mu);
     if (aborted) return qos::set_error(QOS_ERR_COMM, "peer group aborted");
     const uint64_t g = gen;
@@ -243,7 +277,32 @@ struct qos_group {
     }
     return aborted ? qos::set_error(QOS_ERR_COMM, "peer group aborted") : QOS_OK;
   }
+  int ipc_barrier() {
+    if (shm->aborted.load(std::memory_order_acquire)) return qos::set_error(QOS_ERR_COMM, "peer group aborted");
+    const uint64_t g = shm->gen.load(std::memory_order_acquire);
+    if (shm->arrived.fetch_add(1, std::memory_order_acq_rel) + 1 == n) {
+      shm->arrived.store(0, std::memory_order_relaxed);
+      shm->gen.fetch_add(1, std::memory_order_release);
+      return QOS_OK;
+    }
+    const auto t0 = std::chrono::steady_clock::now();
+    for (uint64_t spin = 0; shm->gen.load(std::memory_order_acquire) == g; ++spin) {
+      if (shm->aborted.load(std::memory_order_acquire)) return qos::set_error(QOS_ERR_COMM, "peer group aborted");
+      if (spin > 2048) {
+        sched_yield();
+        if ((spin & 1023) == 0 && std::chrono::steady_clock::now() - t0 > std::chrono::milliseconds(timeout_ms)) {
+          shm->aborted.store(1, std::memory_order_release);
+          return qos::set_error(QOS_ERR_COMM, "peer group barrier timed out (a rank did not reach the collective)");
+        }
+      }
+    }
+    return QOS_OK;
+  }
   void abort() {
+    if (ipc) {
+      shm->aborted.store(1, std::memory_order_release);
+      return;
+    }
     std::lock_guard<std::mutex> lk(mu);
     aborted = true;
     cv.notify_all();
@@ -311,6 +370,9 @@ struct qos_engine {
   uint64_t sync_seq = 0;            // peer syncs issued so far (identical on every rank)
   uint64_t red_seq = 0;             // O / down reductions issued so far (partial buffer parity)
   cudaEvent_t ev_coll[2] = {nullptr, nullptr};  // "my side of this sync is ready", by sync parity
+  std::vector<uint8_t*> ipc_ws;                 // cross-process group: peers' mapped workspaces
+  std::vector<uint8_t*> ipc_base;               //   (their IPC mapping bases, for closing)
+  std::vector<std::array<cudaEvent_t, 2>> ipc_ev;  //   and their opened sync events
   int tp_twoshot = -1;              // option tp_twoshot: 0 one-shot, 1 two-shot, -1 auto (tp >= 4)
   int64_t last_h2d = 0, last_d2h = 0;  // bytes moved host<->device by the last step
   // debug buffers for ops
@@ -684,18 +746,26 @@ void* tp_partial_dst(qos_engine* e) {
 // then order this rank's stream after every peer's record (cross-device waits are legal).
 // An event of parity x is re-recorded two syncs later, i.e. after the barrier of the sync in
 // between, which every rank reaches only after it has issued its waits on this one.
+uint8_t* peer_ws(qos_engine* e, int k) {
+  if (k == e->tp_rank) return e->ws;
+  return e->group->ipc ? e->ipc_ws[size_t(k)] : e->group->eng[size_t(k)]->ws;
+}
+cudaEvent_t peer_event(qos_engine* e, int k, int par) {
+  return e->group->ipc ? e->ipc_ev[size_t(k)][size_t(par)] : e->group->eng[size_t(k)]->ev_coll[par];
+}
+
 int peer_sync(qos_engine* e, cudaStream_t st) {
   const int par = int(e->sync_seq++ & 1);
   QOS_CU(cudaEventRecord(e->ev_coll[par], st));
   QOS_TRY(e->group->barrier());
   for (int k = 0; k < e->tp_size; ++k)
-    if (k != e->tp_rank) QOS_CU(cudaStreamWaitEvent(st, e->group->eng[size_t(k)]->ev_coll[par], 0));
+    if (k != e->tp_rank) QOS_CU(cudaStreamWaitEvent(st, peer_event(e, k, par), 0));
   return QOS_OK;
 }
 
 PeerPtrs peer_ptrs(qos_engine* e, size_t ws_off) {
   PeerPtrs p{};
-  for (int k = 0; k < e->tp_size; ++k) p.p[k] = e->group->eng[size_t(k)]->ws + ws_off;
+  for (int k = 0; k < e->tp_size; ++k) p.p[k] = peer_ws(e, k) + ws_off;
   return p;
 }
 
@@ -1037,7 +1107,144 @@ int qos_group_destroy(qos_group_t* g) {
     for (auto* e : g->eng)
       if (e) return set_error(QOS_ERR_INVALID_ARG, "destroy the group's engines first");
   }
+  if (g->ipc && g->shm) {
+    if (g->shm->attached.fetch_sub(1, std::memory_order_acq_rel) == 1) shm_unlink(g->shm_name.c_str());
+    munmap(g->shm, sizeof(IpcShm));
+  }
   delete g;
+  return QOS_OK;
+}
+
+int qos_group_unique_id(uint8_t out[64]) {
+  if (!out) return set_error(QOS_ERR_INVALID_ARG, "out is NULL");
+  std::random_device rd;
+  const unsigned long long r = (uint64_t(rd()) << 32) ^ rd();
+  char name[64];
+  snprintf(name, sizeof name, "/qoserve_grp_%d_%016llx", int(getpid()), r);
+  memset(out, 0, 64);
+  memcpy(out, name, strlen(name));
+  return QOS_OK;
+}
+
+int qos_group_open(const uint8_t id[64], int tp_size, int tp_rank, qos_group_t** out) {
+  if (!id || !out || tp_size < 2 || tp_size > kMaxPeers || tp_rank < 0 || tp_rank >= tp_size)
+    return set_error(QOS_ERR_INVALID_ARG, "group id / size 2..8 / rank");
+  const std::string name(reinterpret_cast<const char*>(id), strnlen(reinterpret_cast<const char*>(id), 64));
+  if (name.size() < 2 || name[0] != '/' || name.size() >= 64) return set_error(QOS_ERR_INVALID_ARG, "group id");
+  auto g = std::make_unique<qos_group>();
+  g->n = tp_size;
+  g->ipc = true;
+  g->rank = tp_rank;
+  g->shm_name = name;
+  g->eng.assign(size_t(tp_size), nullptr);
+  if (const char* t = getenv("QOS_GROUP_TIMEOUT_MS")) g->timeout_ms = atoi(t);
+  const auto t0 = std::chrono::steady_clock::now();
+  auto timed_out = [&] { return std::chrono::steady_clock::now() - t0 > std::chrono::milliseconds(g->timeout_ms); };
+  int fd = -1;
+  if (tp_rank == 0) {
+    fd = shm_open(name.c_str(), O_CREAT | O_EXCL | O_RDWR, 0600);
+    if (fd < 0) return set_error(QOS_ERR_COMM, "shm_open (create) of the group segment failed");
+    if (ftruncate(fd, sizeof(IpcShm)) != 0) {
+      close(fd);
+      shm_unlink(name.c_str());
+      return set_error(QOS_ERR_COMM, "ftruncate of the group segment failed");
+    }
+  } else {  // wait for rank 0's segment to exist at full size
+    for (;;) {
+      fd = shm_open(name.c_str(), O_RDWR, 0600);
+      if (fd >= 0) {
+        struct stat st {};
+        if (fstat(fd, &st) == 0 && size_t(st.st_size) >= sizeof(IpcShm)) break;
+        close(fd);
+        fd = -1;
+      }
+      if (timed_out()) return set_error(QOS_ERR_COMM, "group segment never appeared (rank 0 did not open the group)");
+      usleep(1000);
+    }
+  }
+  void* m = mmap(nullptr, sizeof(IpcShm), PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
+  close(fd);
+  if (m == MAP_FAILED) return set_error(QOS_ERR_COMM, "mmap of the group segment failed");
+  g->shm = static_cast<IpcShm*>(m);
+  if (tp_rank == 0) {
+    memset(m, 0, sizeof(IpcShm));
+    g->shm->n = tp_size;
+    g->shm->magic.store(IpcShm::kMagic, std::memory_order_release);
+  } else {
+    while (g->shm->magic.load(std::memory_order_acquire) != IpcShm::kMagic) {
+      if (timed_out()) {
+        munmap(m, sizeof(IpcShm));
+        return set_error(QOS_ERR_COMM, "group segment never initialised");
+      }
+      usleep(1000);
+    }
+    if (g->shm->n != tp_size) {
+      munmap(m, sizeof(IpcShm));
+      return set_error(QOS_ERR_INVALID_ARG, "tp_size differs from rank 0's");
+    }
+  }
+  g->shm->attached.fetch_add(1, std::memory_order_acq_rel);
+  *out = g.release();
+  return QOS_OK;
+}
+
+// Cross-process group: export this rank's workspace + sync events, meet the peers, open theirs.
+using PFN_memGetAddressRange = CUresult (*)(CUdeviceptr*, size_t*, CUdeviceptr);
+static int ipc_attach(qos_engine* e, qos_group* g) {
+  if (e->tp_rank != g->rank) return set_error(QOS_ERR_INVALID_ARG, "tp_rank differs from the group rank");
+  for (int i = 0; i < 2; ++i)
+    QOS_CU(cudaEventCreateWithFlags(&e->ev_coll[i], cudaEventDisableTiming | cudaEventInterprocess));
+  static PFN_memGetAddressRange range = nullptr;
+  if (!range) {
+    void* fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &fn, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      return set_error(QOS_ERR_CUDA, "cuMemGetAddressRange unavailable");
+    range = reinterpret_cast<PFN_memGetAddressRange>(fn);
+  }
+  CUdeviceptr base = 0;
+  size_t bytes = 0;
+  if (range(&base, &bytes, CUdeviceptr(e->ws)) != CUDA_SUCCESS) return set_error(QOS_ERR_CUDA, "workspace range");
+  IpcSlot& me = g->shm->slot[e->tp_rank];
+  QOS_CU(cudaIpcGetMemHandle(&me.ws, reinterpret_cast<void*>(base)));
+  me.ws_off = uint64_t(CUdeviceptr(e->ws) - base);
+  for (int i = 0; i < 2; ++i) QOS_CU(cudaIpcGetEventHandle(&me.ev[i], e->ev_coll[i]));
+  cudaDeviceProp prop{};
+  QOS_CU(cudaGetDeviceProperties(&prop, e->device));
+  memcpy(me.uuid, &prop.uuid, 16);
+  me.cfg = e->cfg;
+  QOS_TRY(g->barrier());  // every rank has published its slot
+  e->ipc_ws.assign(size_t(g->n), nullptr);
+  e->ipc_base.assign(size_t(g->n), nullptr);
+  e->ipc_ev.assign(size_t(g->n), {nullptr, nullptr});
+  for (int k = 0; k < g->n; ++k) {
+    if (k == e->tp_rank) continue;
+    const IpcSlot& p = g->shm->slot[k];
+    if (std::memcmp(&p.cfg, &e->cfg, sizeof(e->cfg)) != 0) {
+      g->abort();
+      return set_error(QOS_ERR_INVALID_ARG, "group ranks need identical model configs");
+    }
+    if (std::memcmp(p.uuid, me.uuid, 16) == 0) e->shares_device = true;
+    void* ptr = nullptr;
+    cudaError_t er = cudaIpcOpenMemHandle(&ptr, p.ws, cudaIpcMemLazyEnablePeerAccess);
+    if (er != cudaSuccess) {
+      g->abort();
+      return set_cuda_error(er, "cudaIpcOpenMemHandle (peer workspace)");
+    }
+    e->ipc_base[size_t(k)] = static_cast<uint8_t*>(ptr);
+    e->ipc_ws[size_t(k)] = static_cast<uint8_t*>(ptr) + p.ws_off;
+    for (int i = 0; i < 2; ++i) {
+      er = cudaIpcOpenEventHandle(&e->ipc_ev[size_t(k)][size_t(i)], p.ev[i]);
+      if (er != cudaSuccess) {
+        g->abort();
+        return set_cuda_error(er, "cudaIpcOpenEventHandle (peer sync event)");
+      }
+    }
+  }
+  QOS_TRY(g->barrier());  // every rank has mapped its peers
+  g->eng[size_t(e->tp_rank)] = e;
+  e->group = g;
   return QOS_OK;
 }
 
@@ -1135,7 +1342,9 @@ static int create_engine(const qos_model_cfg* cfg, int device, int tp_rank, int 
   e->free_rows.resize(size_t(cfg->max_requests));
   for (int i = 0; i < cfg->max_requests; ++i) e->free_rows[size_t(i)] = i;
   if ((r = build_maps(e)) != QOS_OK) return fail(r);
-  if (group) {
+  if (group && group->ipc) {
+    if ((r = ipc_attach(e, group)) != QOS_OK) return fail(r);
+  } else if (group) {
     for (int i = 0; i < 2; ++i) cudaEventCreateWithFlags(&e->ev_coll[i], cudaEventDisableTiming);
     std::lock_guard<std::mutex> lk(group->mu);
     if (group->eng[size_t(tp_rank)]) return fail(set_error(QOS_ERR_INVALID_ARG, "tp_rank already in the group"));
@@ -1188,6 +1397,14 @@ int qos_engine_destroy(qos_engine_t* e) {
   if (!e) return QOS_OK;
   cudaSetDevice(e->device);
   cudaDeviceSynchronize();
+  if (e->group && e->group->ipc) {
+    e->group->barrier();  // no peer still reads this workspace (errors ignored: a dead peer)
+    for (auto* b : e->ipc_base)
+      if (b) cudaIpcCloseMemHandle(b);
+    for (auto& evs : e->ipc_ev)
+      for (auto ev : evs)
+        if (ev) cudaEventDestroy(ev);
+  }
   if (e->group) {
     std::lock_guard<std::mutex> lk(e->group->mu);
     if (e->group->eng[size_t(e->tp_rank)] == e) e->group->eng[size_t(e->tp_rank)] = nullptr;

@@ -82,6 +82,8 @@ _SIGS = {
     "qos_engine_destroy": [_P],
     "qos_group_create": [C.c_int, C.POINTER(_P)],
     "qos_group_destroy": [_P],
+    "qos_group_unique_id": [C.c_char_p],
+    "qos_group_open": [C.c_char_p, C.c_int, C.c_int, C.POINTER(_P)],
     "qos_engine_create_peer": [C.POINTER(qos_model_cfg), C.c_int, C.c_int, _P, C.POINTER(qos_mem), C.POINTER(_P)],
     "qos_nccl_unique_id": [C.c_char_p],
     "qos_shard_plan": [C.POINTER(qos_model_cfg), C.c_int, C.c_int, C.POINTER(qos_shard)],
@@ -208,13 +210,24 @@ def model_cfg(n_layers, d_model, n_heads, n_kv_heads, head_dim, ffn_dim, vocab, 
                          max_batch_rows)
 
 
-class Group:
-    """In-process peer group of tp_size ranks (qos_group_create); destroy after its engines."""
+def qos_group_unique_id() -> bytes:
+    buf = C.create_string_buffer(64)
+    _call("qos_group_unique_id", buf)
+    return buf.raw
 
-    def __init__(self, tp_size: int):
+
+class Group:
+    """Peer group of tp_size ranks: in-process (qos_group_create) or, with `group_id`, this
+    process's membership (rank `rank`) of a cross-process group (qos_group_open).  Destroy after
+    its engines."""
+
+    def __init__(self, tp_size: int, group_id: bytes | None = None, rank: int = 0):
         self.tp_size = tp_size
         h = _P()
-        _call("qos_group_create", tp_size, C.byref(h))
+        if group_id is None:
+            _call("qos_group_create", tp_size, C.byref(h))
+        else:
+            _call("qos_group_open", bytes(group_id).ljust(64, b"\0")[:64], tp_size, rank, C.byref(h))
         self.h = h
 
     def close(self):

@@ -216,3 +216,78 @@ def test_llama70b_shapes_tp8_hybrid_step_sampled_parity():
     got = np.concatenate([lg[:1], lg[[1 + j for j in sample]]])
     assert row_rel_err(got, ref) <= TOL_LOGITS
     _close(g, engs)
+
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _ipc_worker(rank, tp, gid, preset_name, ffn, twoshot, out_q):
+    import sys
+    sys.path.insert(0, ROOT)
+    sys.path.insert(0, os.path.join(ROOT, "tests"))
+    try:
+        import torch
+        torch.cuda.set_device(0)
+        import synth as sy
+        from paper_conf_asplos_goelmkar26_b200 import qoserve as q
+        from paper_conf_asplos_goelmkar26_b200.presets import preset
+        over = {"ffn_dim": ffn} if ffn else {}
+        cfg = q.model_cfg(**preset(preset_name, **over), num_blocks=256, max_seq_len=4096, max_requests=64,
+                          max_batch_tokens=1024, max_batch_rows=32)
+        g = q.Group(tp, gid, rank)
+        e = q.Engine(cfg, 0, rank, tp, group=g)
+        e.qos_engine_set_option("tp_twoshot", twoshot)
+        e.qos_engine_load_synthetic(0)
+        ctxs, warm, main, second = sy.tiny_scenario(cfg.vocab)
+        for r, n in ctxs.items():
+            e.qos_kv_alloc(r, n + 2)
+        e.qos_kv_alloc(0, 256)
+        outs = [e.step_host(q.batch_from_synth(b), cfg.vocab) for b in warm + [main, second]]
+        tables = {r: e.qos_kv_table(r) for r in list(ctxs) + [0]}
+        e.close()
+        g.close()
+        out_q.put((rank, outs, tables, None))
+    except Exception as ex:  # surfaced by the parent
+        out_q.put((rank, None, None, repr(ex)))
+
+
+@pytest.mark.parametrize("preset,tp,ffn,twoshot", [("tiny", 2, None, 0), ("tiny-mha", 4, 1024, 1)])
+def test_tp_cross_process_group_tiny_scenario(preset, tp, ffn, twoshot):
+    """One process per rank (the torchrun layout), all on cuda:0: the group is opened from a
+    shared-memory id, workspaces and sync events are exchanged as CUDA IPC handles, and the
+    collectives read / store peer memory of other processes.  Results vs the unsharded oracle;
+    all ranks bit-identical."""
+    import multiprocessing as mp
+
+    from paper_conf_asplos_goelmkar26_b200 import qoserve as q
+    ctx = mp.get_context("spawn")
+    out_q = ctx.Queue()
+    gid = q.qos_group_unique_id()
+    procs = [ctx.Process(target=_ipc_worker, args=(r, tp, gid, preset, ffn, twoshot, out_q)) for r in range(tp)]
+    for p in procs:
+        p.start()
+    res = {}
+    try:
+        for _ in range(tp):
+            rank, outs, tables, err = out_q.get(timeout=600)
+            assert err is None, (rank, err)
+            res[rank] = (outs, tables)
+    finally:
+        for p in procs:
+            p.join(timeout=60)
+            if p.is_alive():
+                p.kill()
+    orc = _oracle(preset, ffn_dim=ffn, num_blocks=256)
+    ctxs, warm, main, second = synth.tiny_scenario(1024)
+    for r, n in ctxs.items():
+        orc.kv_alloc(r, n + 2)
+    orc.kv_alloc(0, 256)
+    for k, b in enumerate(warm + [main, second]):
+        ref = orc.hybrid_step(*b.as_oracle())
+        lg0, tk0 = res[0][0][k]
+        for rank in range(1, tp):
+            assert np.array_equal(res[rank][0][k][0], lg0) and np.array_equal(res[rank][0][k][1], tk0)
+        assert row_rel_err(lg0, ref) <= TOL_LOGITS
+    for r in list(ctxs) + [0]:
+        for rank in range(tp):
+            assert res[rank][1][r] == orc.kv_table(r)

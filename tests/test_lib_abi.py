@@ -85,3 +85,32 @@ def test_peer_group_host_calls(q):
     g = q.Group(4)
     g.close()
     g.close()  # idempotent in the binding
+
+
+def test_cross_process_group_host_calls(q):
+    """qos_group_unique_id / qos_group_open / qos_group_destroy are host calls (POSIX shm):
+    rank 0 creates the segment; a second open of the same id as rank 0 fails (O_EXCL); a
+    non-zero rank of a missing segment times out."""
+    import os
+    gid = q.qos_group_unique_id()
+    assert gid.startswith(b"/qoserve_grp_") and len(gid) == 64
+    g0 = q.Group(2, gid, 0)
+    with pytest.raises(q.QosError) as ei:
+        q.Group(2, gid, 0)
+    assert ei.value.name == "COMM"
+    with pytest.raises(q.QosError) as ei:   # size mismatch with rank 0's segment
+        q.Group(4, gid, 1)
+    assert ei.value.name == "INVALID_ARG"
+    g1 = q.Group(2, gid, 1)
+    name = gid.rstrip(b"\0").decode()
+    assert os.path.exists("/dev/shm" + name)
+    g1.close()
+    g0.close()
+    assert not os.path.exists("/dev/shm" + name)     # unlinked by the last rank
+    os.environ["QOS_GROUP_TIMEOUT_MS"] = "200"
+    try:
+        with pytest.raises(q.QosError) as ei:
+            q.Group(2, q.qos_group_unique_id(), 1)
+        assert ei.value.name == "COMM"
+    finally:
+        del os.environ["QOS_GROUP_TIMEOUT_MS"]
