@@ -8,6 +8,8 @@ with 128 ongoing decodes at context ~4096 whose KV prefixes are resident in the 
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
     torchrun --nproc-per-node N bench.py --gpus N ...   (N replicas, one per GPU; weak scaling)
+    torchrun --nproc-per-node N bench.py --gpus N --tp N --model qwen2.5-14b   (configs[2]/[3]:
+        one tensor-parallel model over the N ranks, cross-process peer group; strong scaling)
 
 Rank 0 prints ONE JSON line.  `--impl reference` times the fp64 CPU oracle (the only other
 place this file runs oracle/ code besides the cpu_baseline leg).
@@ -101,7 +103,8 @@ class Workload:
     synthetic ctx-4096 prefixes, and a fresh 2048-token chunk request per step.  Decodes advance
     one token per step (steady-state serving); each step's chunk request is freed after it."""
 
-    def __init__(self, device: int, n_steps: int, chunk=CHUNK, n_dec=N_DEC, ctx=CTX, n_layers=None):
+    def __init__(self, device: int, n_steps: int, chunk=CHUNK, n_dec=N_DEC, ctx=CTX, n_layers=None,
+                 model="llama3-8b", tp=1, rank=0, group=None):
         import synth
         from paper_conf_asplos_goelmkar26_b200 import qoserve as q
         from paper_conf_asplos_goelmkar26_b200.presets import preset
@@ -110,9 +113,10 @@ class Workload:
         ctx_cap = ctx + n_steps + 2
         over = {} if n_layers is None else {"n_layers": n_layers}
         num_blocks = n_dec * ((ctx_cap + 15) // 16) + (n_steps + 4) * ((chunk + 15) // 16) + 64
-        self.cfg = q.model_cfg(**preset("llama3-8b", **over), num_blocks=num_blocks, max_seq_len=8192,
+        self.preset = preset(model, **over)
+        self.cfg = q.model_cfg(**self.preset, num_blocks=num_blocks, max_seq_len=8192,
                                max_requests=n_dec + 64, max_batch_tokens=chunk + n_dec, max_batch_rows=n_dec + 1)
-        self.eng = q.Engine(self.cfg, device=device)
+        self.eng = q.Engine(self.cfg, device=device, tp_rank=rank, tp_size=tp, group=group)
         self.eng.qos_engine_load_synthetic(synth.SEED_WEIGHTS)
         self.dec_reqs = list(range(1, n_dec + 1))
         for r in self.dec_reqs:
@@ -149,12 +153,26 @@ def run_ours(args):
     import torch.distributed as dist
 
     ws, rank, local = _dist()
+    local = local % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
+    tp = args.tp
+    shared_gpu = ws > torch.cuda.device_count()   # smoke runs of --tp on one GPU: NCCL refuses that
     if ws > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if shared_gpu:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     K, W = args.steps, args.warmup
-    wl = Workload(local, W + 3 * K + 2)
+    group = None
+    if tp > 1:  # one model over the ranks: cross-process peer group (id from rank 0)
+        from paper_conf_asplos_goelmkar26_b200 import qoserve as qq
+        assert ws == tp, "--tp needs WORLD_SIZE == tp (one rank per GPU)"
+        box = [qq.qos_group_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(box, src=0)
+        group = qq.Group(tp, box[0], rank)
+    wl = Workload(local, W + 3 * K + 2, model=args.model, n_layers=args.layers, tp=tp, rank=rank, group=group)
     q, eng, T = wl.q, wl.eng, wl.tokens_per_step
+    replicas = ws // tp
     stream = torch.cuda.current_stream()
     sptr = stream.cuda_stream
     out_tok = torch.empty(N_DEC + 1, dtype=torch.int32, device="cuda")
@@ -207,11 +225,13 @@ def run_ours(args):
     h2d, d2h = eng.qos_last_step_io()
     # -------- max over ranks
     if ws > 1:
-        t = torch.tensor([ms_step, e2e_ms, ms_instr], device="cuda")
+        t = torch.tensor([ms_step, e2e_ms, ms_instr], device="cpu" if shared_gpu else "cuda")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms_step, e2e_ms, ms_instr = float(t[0]), float(t[1]), float(t[2])
     peaks = _peaks()
-    d, F, hd, Hkv = 4096, 14336, 128, 8
+    pr = wl.preset
+    d, F, hd, Hkv = pr["d_model"], pr["ffn_dim"] // tp, pr["head_dim"], pr["n_kv_heads"] // tp
+    L = pr["n_layers"]
     gu_ms, gu_n = per_class["gemm_gateup"]
     gu_flops = 2.0 * T * d * (2 * F)                    # algorithmic FLOPs per launch (one layer)
     gu_tfs = gu_flops / (gu_ms / gu_n * 1e-3) / 1e12
@@ -225,24 +245,30 @@ def run_ours(args):
     peak_hbm = peaks.get("hbm_gbs") or 6650.0
     traffic = None
     try:
+        assert args.model == "llama3-8b" and tp == 1 and args.layers is None   # the committed capture
         prof = json.load(open(os.path.join(ROOT, "profiles", "roofline_traffic.json")))
         traffic = prof.get("gemm_gateup", {}).get("dram_bytes_per_launch")
     except Exception:
         pass
+    tag = args.model + (f" TP{tp}" if tp > 1 else "")
     rec = {
-        "metric": "hybrid-step tokens/s (llama3-8b, chunk 2048 + 128 decodes @4k)",
-        "value": round(ws * T / (ms_step * 1e-3), 1),
+        "metric": f"hybrid-step tokens/s ({tag}, chunk 2048 + 128 decodes @4k)",
+        "value": round(replicas * T / (ms_step * 1e-3), 1),
         "unit": "tokens/s",
         "n_gpus": ws, "steps": K, "warmup": W,
         "ms_per_step": round(ms_step, 4),
         "higher_is_better": True,
-        "scaling": "weak",
+        "scaling": "weak" if tp == 1 else "strong",
         "vs_baseline": None,
         "dtype": "bf16",
         "data": "synthetic (seeded weights + synthetic KV prefixes; DESIGN.md §3)",
-        "config": {"workload": WORKLOAD, "model": "llama3-8b (32 layers, random-init)", "chunk_len": CHUNK,
-                   "n_decode": N_DEC, "ctx": CTX, "tokens_per_step": T, "parallelism": f"replicas{ws}",
-                   "l2": "inputs larger than L2 (16 GB weights + 69 GB KV streamed per step)"},
+        "config": {"workload": WORKLOAD.replace("llama3-8b", tag),
+                   "model": f"{args.model} ({L} layers, random-init)", "chunk_len": CHUNK,
+                   "n_decode": N_DEC, "ctx": CTX, "tokens_per_step": T,
+                   "parallelism": f"replicas{ws}" if tp == 1 else f"tp{tp} (peer-memory collectives)",
+                   "l2": ("inputs larger than L2 (16 GB weights + 69 GB KV streamed per step)" if tp == 1 and
+                          args.model == "llama3-8b" and args.layers is None else
+                          "inputs larger than L2 (weight shard + KV of 128 x 4k contexts streamed per step)")},
         "latency_ms": {"median": round(statistics.median(steps_ms), 4), "min": round(min(steps_ms), 4),
                        "max": round(max(steps_ms), 4), "instrumented_pass_serial_attention": round(ms_instr, 4)},
         "breakdown_ms_per_step": {k: round(v[0] / K, 4) for k, v in per_class.items() if v[1]},
@@ -255,14 +281,16 @@ def run_ours(args):
                                  "peak_source": "MEASURED_PEAKS.json hbm_gbs (of measured)"},
         "gpu_launches": int(launches),
         "clocks": clk,
-        "e2e": {"value": round(ws * T / (e2e_ms * 1e-3), 1), "unit": "tokens/s",
+        "e2e": {"value": round(replicas * T / (e2e_ms * 1e-3), 1), "unit": "tokens/s",
                 "ms_per_step": round(e2e_ms, 4),
                 "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
                 "how": "qos_hybrid_step with host descriptor and host next_tokens (outputs_on_host=1), wall clock"},
     }
-    if rank == 0 and not args.no_cpu_baseline:
+    if rank == 0 and not args.no_cpu_baseline and tp == 1 and args.model == "llama3-8b" and args.layers is None:
         rec["cpu_baseline"] = cpu_baseline(args.cpu_seconds)
     eng.close()
+    if group is not None:
+        group.close()
     if ws > 1:
         dist.destroy_process_group()
     if rank == 0:
@@ -357,6 +385,9 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=20.0)
+    ap.add_argument("--tp", type=int, default=1, help="tensor-parallel degree (= WORLD_SIZE under torchrun)")
+    ap.add_argument("--model", default="llama3-8b", help="llama3-8b | qwen2.5-14b | llama3-70b")
+    ap.add_argument("--layers", type=int, default=None, help="fewer layers (smoke runs only)")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "ours":
         args.warmup = 3
