@@ -230,7 +230,10 @@ int qos_profile_step_ex(qos_engine_t* eng, int32_t chunk_len, int32_t kv_start,
  * meaning set the defaults at engine creation):
  *   "overlap_attn" (1)     run prefill attention on a high-priority side stream concurrently
  *                          with the decode attention of the same layer
- *   "gemm_splitk" (1)      split-K for weight-bound small-M projections
+ *   "gemm_splitk" (0)      split-K of the tile GEMM for weight-bound small-M projections (off:
+ *                          slower at every shape the engine gives the tile kernel — the QKV
+ *                          GEMM at T 33..128 takes 26 us split vs 17 us unsplit; the weight-
+ *                          streaming kernel covers the small-T O and down projections)
  *   "dual_stream" (0)      prefill rows and decode rows as two sub-batches on two streams
  *                          (measured slower on B200; kept for experiments), with
  *                          "dual_min_prefill" (512), "dual_min_decode" (16),

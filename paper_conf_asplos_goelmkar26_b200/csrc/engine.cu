@@ -353,7 +353,8 @@ struct qos_engine {
   int decode_stages = 8;            // option decode_stages: decode K/V ring depth (8 or 4)
   int fa_qtiles = 1;                // option fa_qtiles: prefill q tiles per CTA sharing K/V tiles
   bool overlap_attn = true;       // QOS_OVERLAP_ATTN=0 serialises a7 and a8 (for measurement)
-  bool gemm_splitk = true;        // QOS_GEMM_SPLITK=0 disables split-K for small-M GEMMs
+  bool gemm_splitk = false;       // QOS_GEMM_SPLITK=1: split-K for small-M tile GEMMs (measured slower on
+                                  // B200 at every shape where the engine picks the tile kernel, r1e)
   int gemm_swab = 1;              // weight-streaming GEMM (gemm_swab.cu): 0 never, 1 auto, 2 always
   int gemm_streamk = 0;           // stream-K tile GEMM: 0 never (default: measured slower on B200,
                                   // unaligned ranges lose the L2 reuse of lock-step waves), 1 auto, 2 always
@@ -703,7 +704,7 @@ int gemm_any(qos_engine* e, const qos_engine::ActMap& am, const CUtensorMap (&tb
              int epi, void* C, int64_t ldc, const float* bias, cudaStream_t st, int sms, float* part, int* cnt,
              int a_row0, const QkvRopeArgs* rope) {
   count_launch();
-  if (N % 128 == 0 && (e->gemm_swab == 2 || (e->gemm_swab == 1 && swab_prefer(M, N, sms)))) {
+  if (N % 128 == 0 && (e->gemm_swab == 2 || (e->gemm_swab == 1 && swab_prefer_k(M, N, K, sms)))) {
     const int bnt = swab_pick_bnt(M);
     return gemm_swab_run(tb[0], am.sw[swab_index(bnt)], bnt, M, N, K, epi, C, ldc, bias, sms, st, part, cnt,
                          int64_t(kGemmMaxUnits) * 128 * 256, kGemmMaxTiles, a_row0, rope, !e->dual_stream && !e->shares_device);
@@ -1799,7 +1800,7 @@ static int op_gemm(const void* A, const void* B, void* C, int64_t M, int64_t N, 
   }
   static const bool swab_env = !(getenv("QOS_GEMM_SWAB") && atoi(getenv("QOS_GEMM_SWAB")) == 0);
   const int64_t ldc = epi == QOS_EPI_SILU_GATE ? N / 2 : N;
-  if (ksplit == -1 || (ksplit == 0 && swab_env && swab_prefer(M, N, sms))) {
+  if (ksplit == -1 || (ksplit == 0 && swab_env && swab_prefer_k(M, N, K, sms))) {
     // weight-streaming swap-AB kernel (gemm_swab.cu)
     const int bnt = swab_pick_bnt(M);
     CUtensorMap tw, tt;

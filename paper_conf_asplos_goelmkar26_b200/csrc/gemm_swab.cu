@@ -423,6 +423,14 @@ bool swab_prefer(int64_t M, int64_t N, int num_sms) {
   const int64_t tiles = ((M + 127) / 128) * (N / 128);
   return tiles * 4 < num_sms;
 }
+// with K: long-K projections (the down projection, K = F) stream more weight bytes per output
+// tile, so the weight-streaming kernel keeps winning up to twice as many tiles (T <= 256 at
+// N = d: 39 vs 51 us at T = 256, tools/gemm_bench.py r1e)
+bool swab_prefer_k(int64_t M, int64_t N, int64_t K, int num_sms) {
+  if (swab_prefer(M, N, num_sms)) return true;
+  if (N % 128 || M > 256 || K < 8192) return false;
+  return ((M + 127) / 128) * (N / 128) * 2 < num_sms;
+}
 
 int swab_grid(int64_t M, int64_t N, int64_t K, int bnt, int num_sms) {
   const int64_t work = (N / 128) * ((M + bnt - 1) / bnt) * (K / kSwBK);

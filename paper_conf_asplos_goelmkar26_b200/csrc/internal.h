@@ -64,6 +64,7 @@ int gemm2_run(const CUtensorMap& ta, const CUtensorMap& tb, int64_t M, int64_t N
 // false in the two-stream mode, where the last arriving CTA reduces alone).
 int swab_pick_bnt(int64_t M);
 bool swab_prefer(int64_t M, int64_t N, int num_sms);  // automatic kernel choice
+bool swab_prefer_k(int64_t M, int64_t N, int64_t K, int num_sms);  // + long-K rule (the engine's choice)
 int swab_grid(int64_t M, int64_t N, int64_t K, int bnt, int num_sms);
 int gemm_swab_run(const CUtensorMap& tw, const CUtensorMap& tt, int bnt, int64_t M, int64_t N, int64_t K, int epi,
                   void* C, int64_t ldc, const float* bias, int num_sms, cudaStream_t st, float* part, int* counters,

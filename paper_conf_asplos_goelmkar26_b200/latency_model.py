@@ -81,6 +81,14 @@ def swab_prefer(M: int, N: int, sms: int) -> bool:   # mirrors swab_prefer (csrc
     return ((M + 127) // 128) * (N // 128) * 4 < sms
 
 
+def swab_prefer_k(M: int, N: int, K: int, sms: int) -> bool:   # mirrors swab_prefer_k (csrc/gemm_swab.cu)
+    if swab_prefer(M, N, sms):
+        return True
+    if N % 128 or M > 256 or K < 8192:
+        return False
+    return ((M + 127) // 128) * (N // 128) * 2 < sms
+
+
 def pair_eligible(M: int, N: int, K: int, sms: int) -> bool:   # mirrors gemm2_eligible (csrc/gemm.cu)
     if N % 256 or K % 64:
         return False
@@ -101,25 +109,22 @@ def gemm_work(T: int, g: GemmShapes) -> float:
         return 0.0
     tot = 0.0
     for N, K in g.gemms:
-        if swab_prefer(T, N, g.num_sms) or pair_eligible(T, N, K, g.num_sms):
+        if swab_prefer_k(T, N, K, g.num_sms) or pair_eligible(T, N, K, g.num_sms):
             continue
         bn = _bn(T, N, g.num_sms)
-        tiles = ((T + 127) // 128) * ((N + bn - 1) // bn)
-        ks = 1                                 # mirrors gemm_pick_ksplit
-        while tiles * ks * 2 <= g.num_sms + g.num_sms // 4 and (K // 64) // (ks * 2) >= 4:
-            ks *= 2
-        tot += math.ceil(tiles * ks / g.num_sms) * (K // 64 // ks) * (bn / 256)
+        tiles = ((T + 127) // 128) * ((N + bn - 1) // bn)   # no split-K (engine default gemm_splitk = 0)
+        tot += math.ceil(tiles / g.num_sms) * (K // 64) * (bn / 256)
     return tot
 
 
 def stream_work(T: int, g: GemmShapes) -> float:
-    return float(sum(N * K for N, K in g.gemms if T > 0 and swab_prefer(T, N, g.num_sms)))
+    return float(sum(N * K for N, K in g.gemms if T > 0 and swab_prefer_k(T, N, K, g.num_sms)))
 
 
 def features(s: StepShape, g: GemmShapes = GemmShapes()) -> np.ndarray:
     nd = len(s.ctx)
     n_pair = sum(1 for N, K in g.gemms if s.T > 0 and pair_eligible(s.T, N, K, g.num_sms))
-    n_stream = sum(1 for N, K in g.gemms if s.T > 0 and swab_prefer(s.T, N, g.num_sms))
+    n_stream = sum(1 for N, K in g.gemms if s.T > 0 and swab_prefer_k(s.T, N, K, g.num_sms))
     return np.array([gemm_work(s.T, g) / 100.0, s.T / 1000.0, sum(c + 1 for c in s.ctx) / 1e6, nd / 100.0,
                      1.0 if nd else 0.0, 1.0, sum(n * (n + 1) / 2 for ks, n in s.chunks) / 1e7,
                      stream_work(s.T, g) / 1e8, sum(n * ks for ks, n in s.chunks) / 1e7, pair_work(s.T, g) / 100.0,

@@ -200,7 +200,7 @@ def test_llama8b_shapes_bench_batch_sampled_parity():
     eng.close()
 
 
-@pytest.mark.parametrize("opts", [{"overlap_attn": 0}, {"gemm_splitk": 0}, {"pdl": 0}, {"gemm_swab": 0},
+@pytest.mark.parametrize("opts", [{"overlap_attn": 0}, {"gemm_splitk": 1}, {"pdl": 0}, {"gemm_swab": 0},
                                   {"gemm_streamk": 0}, {"gemm_streamk": 2, "gemm_swab": 0},
                                   {"gemm_swab": 2}, {"decode_round_split": 0}, {"fa_poly": 0}, {"fa_poly": 2},
                                   {"fa_qtiles": 2}, {"gemm_2cta": 0}, {"decode_stages": 4},

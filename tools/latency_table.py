@@ -25,6 +25,22 @@ from paper_conf_asplos_goelmkar26_b200.latency_model import LatencyModel, StepSh
 from paper_conf_asplos_goelmkar26_b200.presets import preset  # noqa: E402
 
 
+def random_batches(rng, n, cap_tokens):
+    """The heterogeneous test batches: chunk U[256, 8192], kv_start
+    U[0, 4096], n_dec U[0, 256], ctx_j U[1k, 8k], cut to the KV capacity.  Deterministic in the
+    rng state, so tools/latency_refit.py can replay the exact batches of a recorded table."""
+    out = []
+    for _ in range(n):
+        chunk = int(rng.integers(256, 8193))
+        nd = int(rng.integers(0, 257))
+        ks = int(rng.integers(0, 4097))
+        ctx = rng.integers(1024, 8193, size=nd)
+        while ctx.sum() + nd > cap_tokens:
+            ctx = ctx[: max(0, len(ctx) - 8)]
+        out.append((chunk, ks, [int(c) for c in ctx]))
+    return out
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--out", default="gpurun_out/latency_table.json")
@@ -67,6 +83,13 @@ def main():
     for chunk in (256, 1024, 2048, 4096):
         for nd in (0, 128):
             grid.append((chunk, nd, 2048, 4096))
+    # chunks on a cached prefix mixed with decodes (the scheduler's common case: later chunks of a
+    # prompt while decodes run)
+    for chunk in (512, 2048, 6144):
+        for nd in (64, 192):
+            for ctx in (2048, 6144):
+                if nd * (ctx + 1) <= cap_tokens:
+                    grid.append((chunk, nd, ctx, 2048))
     # small, decode-dominated steps (the weight-streaming GEMM regime the scheduler also prices)
     for nd in (1, 8, 16, 32, 64):
         grid.append((0, nd, 2048, 0))
@@ -85,19 +108,12 @@ def main():
     model = LatencyModel().fit(fit_shapes, fit_ms)
     fit_err = [abs(model.predict(s) - m) / m for s, m in zip(fit_shapes, fit_ms)]
     tests = []
-    for _ in range(a.test):
-        chunk = int(rng.integers(256, 8193))
-        nd = int(rng.integers(0, 257))
-        ks = int(rng.integers(0, 4097))
-        ctx = rng.integers(1024, 8193, size=nd)
-        while ctx.sum() + nd > cap_tokens:
-            ctx = ctx[: max(0, len(ctx) - 8)]
-        ctx = [int(c) for c in ctx]
+    for chunk, ks, ctx in random_batches(rng, a.test, cap_tokens):
         ms, p95 = prof(chunk, ctx, kv_start=ks)
         s = StepShape([(ks, chunk)], ctx)
         pred = model.predict(s)
         tests.append({"chunk": chunk, "kv_start": ks, "n_decode": len(ctx), "sum_ctx": int(sum(ctx)), "ms": ms,
-                      "pred_ms": pred, "rel_err": abs(pred - ms) / ms})
+                      "pred_ms": pred, "rel_err": abs(pred - ms) / ms, "ctx": ctx})
     errs = np.array([t["rel_err"] for t in tests]) if tests else np.zeros(1)
     out = {"model": "llama3-8b" + (f" (L={a.layers})" if a.layers else ""), "reps": a.reps,
            "kv_capacity_tokens": cap_tokens, "fit_points": len(fit_ms),
