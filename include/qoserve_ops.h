@@ -32,11 +32,13 @@ enum {
 int qos_op_gemm(const void* A, const void* B, void* C, int64_t M, int64_t N, int64_t K, int epi,
                 const float* bias, void* stream);
 /* Same with an explicit kernel choice:
- *   ksplit = 0   automatic: the weight-streaming kernel when N % 128 == 0 and M <= 16, or
- *                M <= 32 with fewer output tiles of 128 than SMs, or M <= 256 with fewer than
- *                SMs/4 tiles (env QOS_GEMM_SWAB=0 disables it), else the CTA-pair kernel
- *                when N % 256 == 0 and 128 x 256 tiles fill the SMs (env QOS_GEMM_2CTA=0
- *                disables it), else the tile kernel with automatic split-K;
+ *   ksplit = 0   automatic (the engine's choice): the weight-streaming kernel when
+ *                N % 128 == 0 and M <= 16, or M <= 32 with fewer output tiles of 128 than SMs,
+ *                or M <= 256 with fewer than SMs/4 tiles (SMs/2 when K >= 8192) (env
+ *                QOS_GEMM_SWAB=0 disables it), else the CTA-pair kernel when N % 256 == 0 and
+ *                128 x 256 tiles fill the SMs (env QOS_GEMM_2CTA=0 disables it), else the tile
+ *                kernel with the tile width of fewer cost-weighted waves and no split-K (env
+ *                QOS_GEMM_SPLITK=1: automatic split-K);
  *   ksplit >= 1  the tile kernel (128-token x 128/256-feature tiles) with that split-K factor:
  *                each of `ksplit` CTAs accumulates a K slice of a tile, parks an fp32 partial,
  *                and the last one to arrive sums the slices in slice order (deterministic);

@@ -1822,7 +1822,9 @@ static int op_gemm(const void* A, const void* B, void* C, int64_t M, int64_t N, 
   }
   const int64_t tiles = ((M + 127) / 128) * ((N + bn - 1) / bn);
   const int sk_mode = ksplit <= -2 ? 2 : 0;
-  int ks = ksplit <= -2 ? 1 : ksplit <= 0 ? gemm_pick_ksplit(M, N, K, bn, sms, kGemmMaxUnits) : ksplit;
+  // automatic = the engine's default: no split-K (QOS_GEMM_SPLITK=1 restores the split heuristic)
+  static const bool sk_env = getenv("QOS_GEMM_SPLITK") && atoi(getenv("QOS_GEMM_SPLITK")) != 0;
+  int ks = ksplit <= -2 ? 1 : ksplit <= 0 ? (sk_env ? gemm_pick_ksplit(M, N, K, bn, sms, kGemmMaxUnits) : 1) : ksplit;
   if (ks > 1 && (tiles > kGemmMaxTiles || tiles * ks > kGemmMaxUnits || (K / 64) < ks))
     return set_error(QOS_ERR_INVALID_ARG, "gemm: ksplit too large for the shape / workspace");
   CUtensorMap ta, tb;

@@ -1035,10 +1035,17 @@ static cudaError_t launch_gemm_t(const CUtensorMap& ta, const CUtensorMap& tb, c
 }
 
 int gemm_pick_bn(int64_t M, int64_t N, int epi, int num_sms) {
+  // Tile width by cost: waves x cycles per 64-deep k-block of one tile on one SM, measured on
+  // B200 (tools/gemm_bench.py, ncu cycles): ~445 for 128 x 128 tiles (L2 -> smem feed bound:
+  // 32 KB per 256 MMA cycles) and ~630 for 128 x 256 tiles (48 KB per 512 MMA cycles).  One
+  // wave of wide tiles beats two waves of narrow ones (e.g. T = 768: QKV 33 -> ~21 us, down
+  // 99 -> ~74 us); at large M this reduces to the old rule (wide once they fill the SMs).
+  (void)epi;
+  if (N % 256 != 0) return 128;
   const int64_t mt = (M + kBM - 1) / kBM;
-  if (N % 256 != 0 && epi == EPI_SILU_GATE) return 128;
-  const int64_t t256 = mt * ((N + 255) / 256);
-  return (t256 >= num_sms && N % 256 == 0) ? 256 : 128;
+  const int64_t w128 = (mt * (N / 128) + num_sms - 1) / num_sms;
+  const int64_t w256 = (mt * (N / 256) + num_sms - 1) / num_sms;
+  return w256 * 630 < w128 * 445 ? 256 : 128;
 }
 
 int gemm_pick_ksplit(int64_t M, int64_t N, int64_t K, int bn, int num_sms, int64_t max_units) {

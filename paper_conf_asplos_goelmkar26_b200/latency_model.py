@@ -65,8 +65,12 @@ class GemmShapes:
 
 
 def _bn(M: int, N: int, sms: int) -> int:      # mirrors gemm_pick_bn (csrc/gemm.cu)
+    if N % 256:
+        return 128
     mt = (M + 127) // 128
-    return 256 if (mt * ((N + 255) // 256) >= sms and N % 256 == 0) else 128
+    w128 = -(-(mt * (N // 128)) // sms)
+    w256 = -(-(mt * (N // 256)) // sms)
+    return 256 if w256 * 630 < w128 * 445 else 128
 
 
 def swab_prefer(M: int, N: int, sms: int) -> bool:   # mirrors swab_prefer (csrc/gemm_swab.cu)
