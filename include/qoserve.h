@@ -262,6 +262,10 @@ int qos_profile_step_ex(qos_engine_t* eng, int32_t chunk_len, int32_t kv_start,
  *                          all rows), 1 two-shot (each rank reduces + normalises a row slice and
  *                          stores it into every peer: ~2(tp-1)/tp of one partial per rank instead
  *                          of tp-1), -1 automatic (two-shot when tp >= 4)
+ *   "fa_persist" (1)       prefill attention (fa_qtiles 1) as persistent CTAs, 2 per SM, each
+ *                          running a host-dealt list of work items back to back (LPT greedy by
+ *                          key tiles); the next item's Q is staged under the current epilogue
+ *                          (0: one CTA per work item)
  *   "gemm_2cta" (1)        CTA-pair GEMM (tcgen05 cta_group::2, 256 x 256 tiles) where it
  *                          needs no more waves than 128 x 256 single-CTA tiles; env QOS_GEMM_2CTA
  * Results do not depend on the options (parity tests run with the defaults and variants). */

@@ -440,6 +440,287 @@ __global__ void __launch_bounds__(FaCfg<HD, NQ>::kThreads, FaCfg<HD, NQ>::kMinBl
 }
 
 
+// ---------------------------------------------------------------- persistent variant (fa_persist=1)
+// The single-q-tile kernel above as a persistent CTA (2 per SM): CTA c runs the work items
+// items[cta_off[c] .. cta_off[c+1]) back to back (the host assigns the LPT-sorted items to CTAs
+// greedily by key tiles, like the hardware block scheduler would).  Barrier phases and the
+// K/V ring run on per-CTA cumulative tile counts, TMEM and barriers are set up once, and the
+// next item's Q is staged while the current item's epilogue drains O, so the MMA warp starts
+// the next item's QK(0) under that epilogue and the producer streams its K/V tiles under the
+// current item's tail.  With short causal chunks (2048 tokens from position 0: 16 key tiles
+// per item on average) the per-CTA prologue/epilogue was a third of the launch.
+template <int HD, int POLY>
+__global__ void __launch_bounds__(FaCfg<HD, 1>::kThreads, 2)
+    prefill_attn_persist_kernel(const __grid_constant__ CUtensorMap kvmap, const FaParams p,
+                                const PrefillItem* __restrict__ items, const int32_t* __restrict__ cta_off) {
+  using C = FaCfg<HD, 1>;
+  constexpr int S = C::kStages;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sQ = smem;
+  uint8_t* sK = smem + C::kQBytes;
+  uint8_t* sV = sK + S * C::kTileBytes;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(sV + S * C::kTileBytes);
+  uint64_t* k_full = bar;
+  uint64_t* k_empty = k_full + S;
+  uint64_t* v_full = k_empty + S;
+  uint64_t* v_empty = v_full + S;
+  uint64_t* s_full = v_empty + S;   // [2]
+  uint64_t* p_full = s_full + 2;    // [2]
+  uint64_t* o_full = p_full + 2;    // completes once per P.V
+  uint64_t* o_final = o_full + 1;   // completes once per item
+  uint64_t* q_full = o_final + 1;   // completes once per item (Q staged by the softmax warps)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(q_full + 1);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int i_begin = cta_off[blockIdx.x], i_end = cta_off[blockIdx.x + 1];
+  const int group = p.H / p.Hkv;
+  const int ppt = C::kRows / group;
+
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < S; ++i) {
+      mbar_init(&k_full[i], 1);
+      mbar_init(&k_empty[i], 1);
+      mbar_init(&v_full[i], 1);
+      mbar_init(&v_empty[i], 1);
+    }
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&s_full[b], 1);
+      mbar_init(&p_full[b], 128);
+    }
+    mbar_init(o_full, 1);
+    mbar_init(o_final, 1);
+    mbar_init(q_full, 128);
+    fence_mbar_init();
+  }
+  if (warp == 1) tmem_alloc<C::kTmemCols>(tmem_slot);
+  griddep_wait();  // q and the appended K/V come from the previous kernel
+  griddep_launch_dependents();
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == 0) {
+    // ------------------------------------------------------------------ TMA producer
+    if (elect_one()) {
+      tma_prefetch_desc(&kvmap);
+      uint32_t jg = 0;
+      for (int ii = i_begin; ii < i_end; ++ii) {
+        const PrefillItem it = items[ii];
+        const int nt = it.grp_last / C::kKeys + 1, last_blk = it.grp_last >> 4;
+        const int32_t* trow = p.tables + size_t(it.table) * p.table_w;
+        auto load_tile = [&](uint8_t* dst, uint64_t* full, int j, int plane) {
+          for (int b = 0; b < C::kKeys / 16; ++b) {
+            const int blk = min(j * (C::kKeys / 16) + b, last_blk);  // past the causal end: a valid block (P = 0)
+            const int r = (__ldg(trow + blk) * p.Hkv + it.kv_head) * 16;
+#pragma unroll
+            for (int hf = 0; hf < C::kHalves; ++hf)
+              tma_load_3d(dst + hf * (C::kKeys * 128) + b * 2048, &kvmap, full, hf * 64, r, p.layer * 2 + plane);
+          }
+        };
+        for (int j = 0; j < nt; ++j, ++jg) {
+          const int s = int(jg % S);
+          const uint32_t ph = (jg / S) & 1;
+          mbar_wait(&k_empty[s], ph ^ 1);
+          mbar_arrive_expect_tx(&k_full[s], C::kTileBytes);
+          load_tile(sK + s * C::kTileBytes, &k_full[s], j, 0);
+          mbar_wait(&v_empty[s], ph ^ 1);
+          mbar_arrive_expect_tx(&v_full[s], C::kTileBytes);
+          load_tile(sV + s * C::kTileBytes, &v_full[s], j, 1);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ------------------------------------------------------------------ MMA issuer
+    if (elect_one()) {
+      constexpr uint32_t idesc_qk = umma_idesc_bf16(128, C::kKeys);
+      constexpr uint32_t idesc_pv = (1u << 4) | (1u << 16) | ((uint32_t(HD) >> 3) << 17) | ((128u >> 4) << 24);
+      // O += P(tg) V(tg); `first`: the item's first tile (overwrites O)
+      auto issue_pv = [&](uint32_t tg, bool first) {
+        const int s = int(tg % S);
+        mbar_wait(&v_full[s], (tg / S) & 1);
+        const uint32_t v_base = smem_u32(sV + s * C::kTileBytes);
+        mbar_wait(&p_full[tg & 1], (tg >> 1) & 1);
+        tc_fence_after();
+        const uint32_t p_tmem = tmem + C::col_s(0, int(tg & 1));
+#pragma unroll
+        for (int kk = 0; kk < C::kKeys / 16; ++kk) {
+          const uint64_t vd = umma_desc_sw128_mn(v_base + kk * 2048, C::kKeys * 128);
+          const uint32_t pc = p_tmem + (kk >> 1) * 32 + (kk & 1) * 8;
+          umma_bf16_ts(tmem + C::col_o(0), pc, vd, idesc_pv, (!first || kk != 0) ? 1u : 0u);
+        }
+        umma_commit(o_full);
+        umma_commit(&v_empty[s]);
+      };
+      uint32_t jg = 0;
+      for (int ii = i_begin, n = 0; ii < i_end; ++ii, ++n) {
+        const int nt = items[ii].grp_last / C::kKeys + 1;
+        mbar_wait(q_full, uint32_t(n) & 1);  // this item's Q is in smem
+        tc_fence_after();
+        const uint32_t q_base = smem_u32(sQ);
+        for (int j = 0; j < nt; ++j) {
+          const uint32_t tg = jg + uint32_t(j);
+          const int s = int(tg % S);
+          mbar_wait(&k_full[s], (tg / S) & 1);
+          tc_fence_after();
+          const uint32_t k_base = smem_u32(sK + s * C::kTileBytes);
+          const uint32_t s_tmem = tmem + C::col_s(0, int(tg & 1));
+#pragma unroll
+          for (int ks = 0; ks < HD / 16; ++ks) {
+            const uint32_t qoff = (ks >> 2) * (C::kRows * 128) + (ks & 3) * 32;
+            const uint32_t koff = (ks >> 2) * (C::kKeys * 128) + (ks & 3) * 32;
+            umma_bf16(s_tmem, umma_desc_sw128(q_base + qoff), umma_desc_sw128(k_base + koff), idesc_qk, ks != 0);
+          }
+          umma_commit(&s_full[tg & 1]);
+          umma_commit(&k_empty[s]);
+          if (j >= 1) issue_pv(tg - 1, j == 1);   // O += P(j-1) V(j-1) while the softmax works on S(j)
+        }
+        issue_pv(jg + uint32_t(nt) - 1, nt == 1);
+        umma_commit(o_final);
+        jg += uint32_t(nt);
+      }
+    }
+  } else {
+    // ------------------------------------------------------------------ softmax + Q staging + epilogue
+    const int row = (warp & 3) * 32 + lane;  // the TMEM lane quarter this warp may access
+    const uint32_t lane_base = tmem + (uint32_t((warp & 3) * 32) << 16);
+    const uint32_t o_addr = lane_base + C::col_o(0);
+    const int pi = row / group, hh = row % group;
+    auto stage_q = [&](const PrefillItem& it) {
+      const bool ok = row < ppt * group && pi < it.npos;
+      const __nv_bfloat16* src = p.q + size_t(it.row0 + pi) * p.q_ld + size_t(it.kv_head * group + hh) * HD;
+      uint4 v[HD / 8];
+#pragma unroll
+      for (int ch = 0; ch < HD / 8; ++ch) v[ch] = ok ? *reinterpret_cast<const uint4*>(src + ch * 8) : make_uint4(0, 0, 0, 0);
+#pragma unroll
+      for (int ch = 0; ch < HD / 8; ++ch) {
+        const int hf = ch >> 3, c = ch & 7;
+        *reinterpret_cast<uint4*>(sQ + hf * (C::kRows * 128) + row * 128 + ((c ^ (row & 7)) << 4)) = v[ch];
+      }
+      fence_proxy_async_smem();
+      mbar_arrive(q_full);
+    };
+    if (i_begin < i_end) stage_q(items[i_begin]);
+    uint32_t jg = 0;
+    for (int ii = i_begin, n = 0; ii < i_end; ++ii, ++n) {
+      const PrefillItem it = items[ii];
+      const int nt = it.grp_last / C::kKeys + 1;
+      const bool ok = row < ppt * group && pi < it.npos;
+      const int pos_r = ok ? it.pos0 + pi : -1;
+      const size_t tok_off = size_t(it.row0 + pi) * p.out_ld + size_t(it.kv_head * group + hh) * HD;
+      const int warp_min_pos = __shfl_sync(0xffffffffu, pos_r < 0 ? INT_MAX : pos_r, 0);  // row 0 of the warp
+      float m_used = -INFINITY, l = 0.f;
+      for (int j = 0; j < nt; ++j) {
+        const uint32_t tg = jg + uint32_t(j);
+        const int sb = int(tg & 1);
+        mbar_wait(&s_full[sb], (tg >> 1) & 1);
+        tc_fence_after();
+        const uint32_t s_addr = lane_base + C::col_s(0, sb);
+        const int key0 = j * C::kKeys;
+        const bool masked = __any_sync(0xffffffffu, key0 + C::kKeys - 1 > (pos_r < 0 ? -1 : pos_r)) ||
+                            warp_min_pos == INT_MAX;
+        uint32_t r[C::kKeys];
+#pragma unroll
+        for (int c = 0; c < C::kKeys / 16; ++c)
+          tmem_ld32x32b_x16(s_addr + c * 16, *reinterpret_cast<uint32_t(*)[16]>(&r[c * 16]));
+        tmem_ld_wait();
+        if (masked) {
+          const int lim = (pos_r < 0 ? -1 : pos_r) - key0;
+#pragma unroll
+          for (int i = 0; i < C::kKeys; ++i)
+            if (i > lim) r[i] = 0xff800000u;  // -inf
+        }
+        float mq[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
+#pragma unroll
+        for (int i = 0; i < C::kKeys; i += 2)
+          mq[(i >> 1) & 3] = fmax3(mq[(i >> 1) & 3], __uint_as_float(r[i]), __uint_as_float(r[i + 1]));
+        float mx = fmax3(mq[0], mq[1], fmaxf(mq[2], mq[3]));
+        mx *= p.scale_log2;
+        const bool rescale = mx > m_used + QOS_FA_LAZY;
+        const float m_new = rescale ? mx : m_used;
+        const float alpha = (rescale && m_used != -INFINITY) ? ex2(m_used - m_new) : 1.f;
+        const float mb = (m_new == -INFINITY) ? 0.f : m_new;
+        float2 sum2[4] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+        const float2 scale2 = make_float2(p.scale_log2, p.scale_log2), nmb2 = make_float2(-mb, -mb);
+#pragma unroll
+        for (int c = 0; c < C::kKeys / 32; ++c) {
+          uint32_t hi[16];
+#pragma unroll
+          for (int i = 0; i < 16; ++i) {
+            const float2 x = fma2(make_float2(__uint_as_float(r[c * 32 + 2 * i]), __uint_as_float(r[c * 32 + 2 * i + 1])),
+                                  scale2, nmb2);
+            float2 pp = (POLY > 0 && i % (POLY > 0 ? POLY : 1) == (POLY > 0 ? POLY : 1) - 1) ? ex2_poly2(x) : make_float2(ex2(x.x), ex2(x.y));
+            hi[i] = pack_f16(pp.x, pp.y);
+            sum2[i & 3] = add2(sum2[i & 3], pp);
+          }
+          tmem_st32x32b_x16(s_addr + c * 32, hi);
+        }
+        const float2 s01 = add2(sum2[0], sum2[1]), s23 = add2(sum2[2], sum2[3]);
+        const float sum = (s01.x + s23.x) + (s01.y + s23.y);
+        tmem_st_wait();
+        l = l * alpha + sum;
+        if (j >= 1 && __any_sync(0xffffffffu, alpha != 1.f)) {
+          // rescale O before PV(j) accumulates into it; PV(tg-2) completed before QK(tg) (awaited
+          // above), so o_full has completed tg-1 or tg times and this parity wait cannot alias
+          mbar_wait(o_full, (tg - 1) & 1);
+          tc_fence_after();
+#pragma unroll 1
+          for (int c = 0; c < HD / 16; ++c) {
+            uint32_t r2[16];
+            tmem_ld32x32b_x16(o_addr + c * 16, r2);
+            tmem_ld_wait();
+#pragma unroll
+            for (int i = 0; i < 16; ++i) r2[i] = __float_as_uint(__uint_as_float(r2[i]) * alpha);
+            tmem_st32x32b_x16(o_addr + c * 16, r2);
+          }
+          tmem_st_wait();
+        }
+        m_used = m_new;
+        tc_fence_before();
+        mbar_arrive(&p_full[sb]);
+      }
+      // every QK of this item has completed (its S was awaited): stage the next item's Q now so
+      // the MMA warp starts it under this epilogue
+      if (ii + 1 < i_end) stage_q(items[ii + 1]);
+      mbar_wait(o_final, uint32_t(n) & 1);
+      tc_fence_after();
+      const float inv = (l > 0.f) ? 1.f / l : 0.f;
+#pragma unroll 1
+      for (int c = 0; c < HD / 32; ++c) {
+        uint32_t r2[32];
+        tmem_ld32x32b_x16(o_addr + c * 32, *reinterpret_cast<uint32_t(*)[16]>(&r2[0]));
+        tmem_ld32x32b_x16(o_addr + c * 32 + 16, *reinterpret_cast<uint32_t(*)[16]>(&r2[16]));
+        tmem_ld_wait();
+        if (pos_r >= 0 && !it.pad) {
+          if (p.out_f32) {
+            float4* dst = reinterpret_cast<float4*>(reinterpret_cast<float*>(p.out) + tok_off + c * 32);
+#pragma unroll
+            for (int i = 0; i < 8; ++i)
+              dst[i] = make_float4(__uint_as_float(r2[4 * i]) * inv, __uint_as_float(r2[4 * i + 1]) * inv,
+                                   __uint_as_float(r2[4 * i + 2]) * inv, __uint_as_float(r2[4 * i + 3]) * inv);
+          } else {
+            uint4* dst = reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.out) + tok_off + c * 32);
+#pragma unroll
+            for (int i = 0; i < 4; ++i)
+              dst[i] = make_uint4(pack_bf16(__uint_as_float(r2[8 * i]) * inv, __uint_as_float(r2[8 * i + 1]) * inv),
+                                  pack_bf16(__uint_as_float(r2[8 * i + 2]) * inv, __uint_as_float(r2[8 * i + 3]) * inv),
+                                  pack_bf16(__uint_as_float(r2[8 * i + 4]) * inv, __uint_as_float(r2[8 * i + 5]) * inv),
+                                  pack_bf16(__uint_as_float(r2[8 * i + 6]) * inv, __uint_as_float(r2[8 * i + 7]) * inv));
+          }
+        }
+      }
+      jg += uint32_t(nt);
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc<C::kTmemCols>(tmem);
+  }
+}
+
 // ---------------------------------------------------------------- ping-pong variant (fa_qtiles=2)
 // Two q tiles per CTA (one CTA per SM), 128-key K/V tiles, one S/P buffer per q tile (TMEM:
 // S0 [0,128) S1 [128,256) O0 [256,384) O1 [384,512)).  QKᵀ runs as UMMA N = 128 (twice the
@@ -793,6 +1074,29 @@ static cudaError_t prefill_pp_t(const AttnLaunch& a, const PrefillItem* items, i
                     p, items);
 }
 
+template <int HD, int POLY>
+static cudaError_t prefill_persist_t(const AttnLaunch& a, const PrefillItem* items, const int32_t* cta_off, int n_cta,
+                                     cudaStream_t st) {
+  using C = FaCfg<HD, 1>;
+  static std::atomic<uint64_t> set{0};
+  if (cudaError_t e = smem_attr_once(prefill_attn_persist_kernel<HD, POLY>, int(C::kSmem), set); e != cudaSuccess)
+    return e;
+  FaParams p;
+  p.q = reinterpret_cast<const __nv_bfloat16*>(a.q);
+  p.q_ld = a.q_ld;
+  p.out = a.out;
+  p.out_ld = a.out_ld;
+  p.out_f32 = a.out_f32;
+  p.layer = a.layer;
+  p.H = a.H;
+  p.Hkv = a.Hkv;
+  p.tables = a.tables;
+  p.table_w = a.table_w;
+  p.scale_log2 = a.scale_log2;
+  return launch_pdl(prefill_attn_persist_kernel<HD, POLY>, dim3(n_cta), dim3(C::kThreads), C::kSmem, st, *a.kv_tmap,
+                    p, items, cta_off);
+}
+
 void set_fa_poly(int n) { g_fa_poly = n; }
 
 int prefill_tc_positions_per_tile(int group) { return 128 / group; }
@@ -801,6 +1105,13 @@ cudaError_t launch_prefill_attention_tc(const AttnLaunch& a, const PrefillItem* 
   if (n_items == 0) return cudaSuccess;
   count_launch(1);
   const int poly = g_fa_poly;
+  if (a.cta_off && a.q_tiles == 1 && poly >= 0) {  // persistent CTAs over per-CTA item lists
+    if (a.hd == 128) return poly == 0 ? prefill_persist_t<128, 0>(a, items, a.cta_off, a.n_cta, st)
+                                      : prefill_persist_t<128, 4>(a, items, a.cta_off, a.n_cta, st);
+    if (a.hd == 64) return poly == 0 ? prefill_persist_t<64, 0>(a, items, a.cta_off, a.n_cta, st)
+                                     : prefill_persist_t<64, 4>(a, items, a.cta_off, a.n_cta, st);
+    return cudaErrorInvalidValue;
+  }
   const int nq = a.q_tiles;
   if (nq != 1 && nq != 2) return cudaErrorInvalidValue;
 #define QOS_FA_NQ(HDV, PV) \

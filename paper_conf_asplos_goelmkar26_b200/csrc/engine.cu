@@ -192,7 +192,7 @@ static WsLayout ws_layout(const qos_model_cfg& c, const Shard& s, int tp) {
   const size_t max_pitems = (Tm / ppt + 4 * (Rm + 1)) * size_t(s.Hkv);
   w.meta_bytes = align_up(3 * Tm * 4 + Rm * 4 + 64, 256) + align_up(max_pitems * sizeof(PrefillItem), 256) +
                  align_up(size_t(w.max_items) * sizeof(DecodeItem), 256) +
-                 align_up(size_t(3) * 65536 * 4, 256);
+                 align_up(size_t(3) * 65536 * 4, 256) + align_up(1025 * 4, 256);  // + persistent CTA offsets
   w.meta[0] = take(w.meta_bytes);
   w.meta[1] = take(w.meta_bytes);
   w.dbg = 0;
@@ -205,6 +205,8 @@ struct StepMeta {
   int T = 0, R = 0, n_prefill = 0, n_decode = 0;
   int n_pitems = 0, n_ditems = 0, n_upd = 0;
   int fa_qtiles = 1;  // prefill items come in groups of this many q tiles (one CTA each group)
+  int n_pcta = 0;     // persistent prefill attention: CTAs (0: one CTA per item group)
+  size_t o_pcta = 0;  // offsets [n_pcta + 1] into the prefill items
   // offsets (bytes) inside the metadata block
   size_t o_tok, o_pos, o_slot, o_rows, o_pitems, o_ditems, o_upd, used;
 };
@@ -352,6 +354,7 @@ struct qos_engine {
   bool decode_round_split = true;  // option decode_round_split (A/B of the split-K ranges)
   int decode_stages = 8;            // option decode_stages: decode K/V ring depth (8 or 4)
   int fa_qtiles = 1;                // option fa_qtiles: prefill q tiles per CTA sharing K/V tiles
+  bool fa_persist = true;           // option fa_persist: persistent prefill-attention CTAs (fa_qtiles 1)
   bool overlap_attn = true;       // QOS_OVERLAP_ATTN=0 serialises a7 and a8 (for measurement)
   bool gemm_splitk = false;       // QOS_GEMM_SPLITK=1: split-K for small-M tile GEMMs (measured slower on
                                   // B200 at every shape where the engine picks the tile kernel, r1e)
@@ -576,6 +579,30 @@ int build_step(qos_engine* e, const qos_batch* b, bool check_lengths, uint8_t* b
     pitems.swap(sorted);
   }
   m.fa_qtiles = CS;
+  // persistent prefill attention: the LPT-sorted items dealt greedily to 2 CTAs per SM by key
+  // tiles (+2 tiles for an item's Q staging and epilogue), each CTA's items kept longest first
+  std::vector<int32_t> pcta;
+  if (CS == 1 && e->fa_persist && !pitems.empty()) {
+    const int G = int(std::min<size_t>({pitems.size(), size_t(2 * e->num_sms), size_t(1024)}));
+    std::priority_queue<std::pair<int64_t, int>, std::vector<std::pair<int64_t, int>>, std::greater<>> heap;
+    for (int g = 0; g < G; ++g) heap.push({0, g});
+    std::vector<std::vector<int>> lists(static_cast<size_t>(G));
+    for (size_t i = 0; i < pitems.size(); ++i) {
+      auto [load, g] = heap.top();
+      heap.pop();
+      lists[size_t(g)].push_back(int(i));
+      heap.push({load + pitems[i].grp_last / 64 + 1 + 2, g});
+    }
+    std::vector<PrefillItem> dealt;
+    dealt.reserve(pitems.size());
+    pcta.push_back(0);
+    for (const auto& li : lists) {
+      for (int i : li) dealt.push_back(pitems[size_t(i)]);
+      pcta.push_back(int32_t(dealt.size()));
+    }
+    pitems.swap(dealt);
+    m.n_pcta = G;
+  }
   // decode split-K work list (balanced on sum of keys)
   int64_t total_keys = 0;
   for (int i = 0; i < b->n_decode; ++i) total_keys += int64_t(b->decode[i].ctx_len) + 1;
@@ -643,6 +670,7 @@ int build_step(qos_engine* e, const qos_batch* b, bool check_lengths, uint8_t* b
   m.n_ditems = int(ditems.size());
   m.o_pitems = take(pitems.size() * sizeof(PrefillItem));
   m.o_ditems = take(ditems.size() * sizeof(DecodeItem));
+  m.o_pcta = take(pcta.size() * 4);
   const size_t max_upd = 65536;
   m.n_upd = int(std::min(e->pending_upd.size() / 3, max_upd));
   m.o_upd = take(size_t(m.n_upd) * 12);
@@ -650,6 +678,7 @@ int build_step(qos_engine* e, const qos_batch* b, bool check_lengths, uint8_t* b
   if (m.used > e->wsl.meta_bytes) return set_error(QOS_ERR_INVALID_ARG, "metadata exceeds workspace");
   if (!pitems.empty()) memcpy(buf + m.o_pitems, pitems.data(), pitems.size() * sizeof(PrefillItem));
   if (!ditems.empty()) memcpy(buf + m.o_ditems, ditems.data(), ditems.size() * sizeof(DecodeItem));
+  if (!pcta.empty()) memcpy(buf + m.o_pcta, pcta.data(), pcta.size() * 4);
   if (m.n_upd) memcpy(buf + m.o_upd, e->pending_upd.data(), size_t(m.n_upd) * 12);
   (void)out_rows_tables;
   return QOS_OK;
@@ -855,6 +884,8 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
   al.table_w = e->table_w;
   al.scale_log2 = float(1.4426950408889634 / std::sqrt(double(hd)));
   al.q_tiles = m.fa_qtiles;
+  al.cta_off = m.n_pcta ? reinterpret_cast<const int32_t*>(dm + m.o_pcta) : nullptr;
+  al.n_cta = m.n_pcta;
   al.decode_stages = e->decode_stages;
   const int n_pre_rows = T - m.n_decode;
   float* gpart0 = reinterpret_cast<float*>(e->ws + s.gemm_part);
@@ -1718,6 +1749,7 @@ int qos_engine_set_option(qos_engine_t* e, const char* name, int64_t value) {
   if (n == "overlap_attn") e->overlap_attn = value != 0;
   else if (n == "decode_round_split") e->decode_round_split = value != 0;
   else if (n == "gemm_2cta") e->gemm_2cta = value != 0;
+  else if (n == "fa_persist") e->fa_persist = value != 0;
   else if (n == "tp_twoshot") e->tp_twoshot = value < 0 ? -1 : value > 0 ? 1 : 0;
   else if (n == "decode_stages") {
     if (value != 4 && value != 8) return set_error(QOS_ERR_INVALID_ARG, "decode_stages must be 4 or 8");
@@ -1958,6 +1990,8 @@ int qos_op_attention(qos_engine_t* e, int32_t layer, const qos_batch* b, const u
   al.table_w = e->table_w;
   al.scale_log2 = float(1.4426950408889634 / std::sqrt(double(hd)));
   al.q_tiles = m.fa_qtiles;
+  al.cta_off = m.n_pcta ? reinterpret_cast<const int32_t*>(dm + m.o_pcta) : nullptr;
+  al.n_cta = m.n_pcta;
   al.decode_stages = e->decode_stages;
   QOS_CU(launch_prefill_attention_tc(al, reinterpret_cast<const PrefillItem*>(dm + m.o_pitems), m.n_pitems, st));
   QOS_CU(launch_decode_attention(al, reinterpret_cast<const DecodeItem*>(dm + m.o_ditems), m.n_ditems,

@@ -157,6 +157,8 @@ struct AttnLaunch {
   float scale_log2;       // log2(e) / sqrt(hd)
   int q_tiles = 1;        // prefill: q tiles per CTA sharing every K/V tile (1 or 2)
   int decode_stages = 8;  // decode: K/V ring depth in (block, head) tiles (8 or 4)
+  const int32_t* cta_off = nullptr;  // prefill, persistent mode: CTA c runs items [cta_off[c], cta_off[c+1])
+  int n_cta = 0;
 };
 cudaError_t launch_decode_attention(const AttnLaunch& a, const DecodeItem* items, int n_items, float* partials,
                                     int* counters, cudaStream_t st);

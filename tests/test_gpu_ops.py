@@ -185,18 +185,22 @@ ATTN_CASES = [
     # configs[3] maximum context: a chunk deep into a 20k prefix and a decode over 32k keys
     ("llama3-70b", dict(n_layers=1, n_heads=8, n_kv_heads=1, d_model=1024, ffn_dim=1024, num_blocks=4096,
                         max_seq_len=32784), [(20000, 96)], [32767], 1.0),
+    # the bench chunk: 512 work items (more than 2 per SM), so persistent CTAs run several each
+    ("llama3-8b", dict(n_layers=1, num_blocks=2048), [(0, 2048), (512, 700)], [100], 1.0),
 ]
 
 
-@pytest.mark.parametrize("qtiles", [1, 2])
+@pytest.mark.parametrize("qtiles,persist", [(1, 1), (1, 0), (2, 0)])
 @pytest.mark.parametrize("case", range(len(ATTN_CASES)))
-def test_attention_parity(case, qtiles):
+def test_attention_parity(case, qtiles, persist):
     """Prefill + decode attention (fp32 output) vs the fp64 oracle; prefill with 1 or 2 q tiles
-    per CTA sharing every K/V tile (odd tile counts padded with a duplicate)."""
+    per CTA sharing every K/V tile (odd tile counts padded with a duplicate), and the persistent
+    single-tile kernel (several work items per CTA)."""
     from oracle.model import causal_attention
     preset, over, chunks, ctxs, scale = ATTN_CASES[case]
-    q, cfg, eng = make_engine(preset, **{"max_seq_len": 8192, **over})
+    q, cfg, eng = make_engine(preset, **{"max_seq_len": 8192, "max_batch_tokens": 4096, **over})
     eng.qos_engine_set_option("fa_qtiles", qtiles)
+    eng.qos_engine_set_option("fa_persist", persist)
     H, Hkv, hd = cfg.n_heads, cfg.n_kv_heads, cfg.head_dim
     g = H // Hkv
     rng = np.random.default_rng(100 + case)
