@@ -36,6 +36,9 @@ namespace qos {
 
 static thread_local std::string g_last_error;
 static std::atomic<int64_t> g_launches{0};
+// QOS_SKIP_NORM=1: measurement only (results invalid): skips the per-layer RMSNorm launches to
+// price them inside the step
+static const bool g_skip_norm = getenv("QOS_SKIP_NORM") && atoi(getenv("QOS_SKIP_NORM")) != 0;
 
 int set_error(int code, const char* msg) {
   g_last_error = msg ? msg : "";
@@ -148,7 +151,7 @@ static WeightLayout weight_layout(const qos_model_cfg& c, const Shard& s) {
 }
 
 struct WsLayout {
-  size_t resid, h, qkv, attn, act, hR, logits, logits_loc, part[2], argmax, partials, counters, gemm_part, gemm_cnt, gemm_part2,
+  size_t resid, h, qkv, attn, act, hR, logits, logits_loc, part[2], ss[2], rs[2], fcnt, argmax, partials, counters, gemm_part, gemm_cnt, gemm_part2,
       gemm_cnt2, meta[2], dbg, total;
   size_t meta_bytes;
   int max_items;
@@ -176,6 +179,11 @@ static WsLayout ws_layout(const qos_model_cfg& c, const Shard& s, int tp) {
   w.logits = take(Rm * size_t(c.vocab) * 4);
   w.logits_loc = tp > 1 ? take(Rm * size_t(c.vocab) * 4) : 0;
   // peer-group TP: the O / down partials, double-buffered by collective parity (read by the peers)
+  w.ss[0] = take(Tm * kFoldSlots * 4);  // folded RMSNorm: per-row sums of squares per 128 columns
+  w.ss[1] = take(Tm * kFoldSlots * 4);
+  w.rs[0] = take(Tm * 4);
+  w.rs[1] = take(Tm * 4);
+  w.fcnt = take((Tm / 128 + 2) * 4);
   w.part[0] = tp > 1 ? take(Tm * d * 2) : 0;
   w.part[1] = tp > 1 ? take(Tm * d * 2) : 0;
   w.argmax = take(Rm * 4);
@@ -355,6 +363,7 @@ struct qos_engine {
   int decode_stages = 8;            // option decode_stages: decode K/V ring depth (8 or 4)
   int fa_qtiles = 1;                // option fa_qtiles: prefill q tiles per CTA sharing K/V tiles
   bool fa_persist = true;           // option fa_persist: persistent prefill-attention CTAs (fa_qtiles 1)
+  bool norm_fold = true;            // option norm_fold: RMSNorm folded into the O / down and QKV / gate-up GEMMs
   bool overlap_attn = true;       // QOS_OVERLAP_ATTN=0 serialises a7 and a8 (for measurement)
   bool gemm_splitk = false;       // QOS_GEMM_SPLITK=1: split-K for small-M tile GEMMs (measured slower on
                                   // B200 at every shape where the engine picks the tile kernel, r1e)
@@ -729,21 +738,29 @@ static int swab_index(int bnt) { return bnt == 16 ? 0 : bnt == 32 ? 1 : bnt == 6
 
 // One projection GEMM of M rows: gemm_swab.cu (weight-streaming, swap-AB, stream-K) at small M,
 // else gemm.cu (activation-stationary tiles, optional split-K).
+// the kernel gemm_any takes for this shape runs whole tiles in one pass (the folded RMSNorm's
+// producer and consumer epilogues live there): not the weight-streaming kernel, no split-K
+bool gemm_one_pass(const qos_engine* e, int64_t M, int64_t N, int64_t K, int sms) {
+  if (N % 128 == 0 && (e->gemm_swab == 2 || (e->gemm_swab == 1 && swab_prefer_k(M, N, K, sms)))) return false;
+  return !e->gemm_splitk;
+}
+
 int gemm_any(qos_engine* e, const qos_engine::ActMap& am, const CUtensorMap (&tb)[2], int64_t M, int64_t N, int64_t K,
              int epi, void* C, int64_t ldc, const float* bias, cudaStream_t st, int sms, float* part, int* cnt,
-             int a_row0, const QkvRopeArgs* rope) {
+             int a_row0, const QkvRopeArgs* rope, const NormFold* fold = nullptr) {
   count_launch();
+  if (fold && !gemm_one_pass(e, M, N, K, sms)) return set_error(QOS_ERR_INVALID_ARG, "folded norm on a split GEMM");
   if (N % 128 == 0 && (e->gemm_swab == 2 || (e->gemm_swab == 1 && swab_prefer_k(M, N, K, sms)))) {
     const int bnt = swab_pick_bnt(M);
     return gemm_swab_run(tb[0], am.sw[swab_index(bnt)], bnt, M, N, K, epi, C, ldc, bias, sms, st, part, cnt,
                          int64_t(kGemmMaxUnits) * 128 * 256, kGemmMaxTiles, a_row0, rope, !e->dual_stream && !e->shares_device);
   }
   if (e->gemm_2cta && gemm2_eligible(M, N, K, sms))
-    return gemm2_run(am.m128, tb[0], M, N, K, epi, C, ldc, bias, sms, st, a_row0, sms, rope);
+    return gemm2_run(am.m128, tb[0], M, N, K, epi, C, ldc, bias, sms, st, a_row0, sms, rope, fold);
   const int bn = gemm_pick_bn(M, N, epi, sms);
   const int ks = e->gemm_splitk ? gemm_pick_ksplit(M, N, K, bn, sms, kGemmMaxUnits) : 1;
   return gemm_run(am.m128, tb[bn == 256 ? 1 : 0], bn, M, N, K, epi, C, ldc, bias, sms, st, ks, part, cnt, a_row0, sms,
-                  rope, e->gemm_streamk, !e->dual_stream && !e->shares_device);
+                  rope, e->gemm_streamk, !e->dual_stream && !e->shares_device, fold);
 }
 
 int gemm(qos_engine* e, const qos_engine::ActMap& am, const CUtensorMap (&tb)[2], int64_t M, int64_t N, int64_t K,
@@ -844,11 +861,12 @@ struct Seg {
 };
 
 int gemm_seg(qos_engine* e, const Seg& g, const qos_engine::ActMap& am, const CUtensorMap (&tb)[2], int64_t N,
-             int64_t K, int epi, void* C, int64_t ldc, const float* bias, const QkvRopeArgs* rope = nullptr) {
+             int64_t K, int epi, void* C, int64_t ldc, const float* bias, const QkvRopeArgs* rope = nullptr,
+             const NormFold* fold = nullptr) {
   const int sms = g.sms > 0 ? g.sms : e->num_sms;
   const size_t esz = (epi == EPI_STORE_F32 || epi == EPI_ADD_F32) ? 4 : 2;
   return gemm_any(e, am, tb, g.n, N, K, epi, reinterpret_cast<uint8_t*>(C) + size_t(g.row0) * ldc * esz, ldc, bias,
-                  g.st, sms, g.gpart, g.gcnt, g.row0, rope);
+                  g.st, sms, g.gpart, g.gcnt, g.row0, rope, fold);
 }
 
 // The layer loop.  `dm` = device metadata block of this step.
@@ -906,9 +924,40 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
   } else {
     segs[nseg++] = Seg{0, T, st, m.n_pitems > 0, m.n_ditems > 0, gpart0, gcnt0, 0};
   }
+  // RMSNorm folded into the projections (NormFold, internal.h) when all four GEMMs of the step
+  // run whole tiles in one pass: the O / down epilogues produce r, h = bf16(r * g) and per-row
+  // sums of squares, the QKV / gate-up epilogues scale their rows by 1/rms — no norm launches
+  const int sms_all = e->num_sms;
+  // (from T = 1536: below, the read-add-write epilogue of the last wave costs what the norm
+  //  launches cost — 512 tokens +1.5%, 1024 neutral, 2176 -1.5%, 4096 -4.6%, tools/attn_bench.py r1f)
+  const bool fold = e->norm_fold && !tp && nseg == 1 && !g_skip_norm && T >= kFoldMinTokens && d % 128 == 0 &&
+                    d / 128 <= kFoldSlots &&
+                    gemm_one_pass(e, T, e->nqkv, d, sms_all) && gemm_one_pass(e, T, d, e->sh.H * hd, sms_all) &&
+                    gemm_one_pass(e, T, 2 * e->sh.F, d, sms_all) && gemm_one_pass(e, T, d, e->sh.F, sms_all);
+  float* ssb[2] = {reinterpret_cast<float*>(e->ws + s.ss[0]), reinterpret_cast<float*>(e->ws + s.ss[1])};
+  float* rsb[2] = {reinterpret_cast<float*>(e->ws + s.rs[0]), reinterpret_cast<float*>(e->ws + s.rs[1])};
+  auto fold_args = [&](int in, int out, uint64_t g_off) {  // in / out: ss/rs buffer index or -1
+    NormFold f;
+    f.rs_in = in >= 0 ? rsb[in] : nullptr;
+    f.ss_out = out >= 0 ? ssb[out] : nullptr;
+    f.rs_out = out >= 0 ? rsb[out] : nullptr;
+    f.cnt = out >= 0 ? reinterpret_cast<int*>(e->ws + s.fcnt) : nullptr;
+    f.g_out = out >= 0 ? W(e, g_off) : nullptr;
+    f.h_out = out >= 0 ? h : nullptr;
+    f.ss_n = d / 128;
+    f.d = d;
+    f.eps = c.rms_eps;
+    return f;
+  };
   for (int l = 0; l < c.n_layers; ++l) {
     const auto& L = e->wl.layers[l];
     const auto& M = e->lmaps[l];
+    // fold: ss[1] carries ln1's statistics (down -> next QKV), ss[0] ln2's (O -> gate/up)
+    const NormFold f_qkv = fold_args(l > 0 ? 1 : -1, -1, 0);
+    const NormFold f_o = fold_args(-1, 0, L.ln2);
+    const NormFold f_gu = fold_args(0, -1, 0);
+    const NormFold f_down = fold_args(-1, 1, l + 1 < c.n_layers ? e->wl.layers[l + 1].ln1 : 0);
+    const bool fold_down = fold && l + 1 < c.n_layers;
     __nv_bfloat16* kpl = reinterpret_cast<__nv_bfloat16*>(e->kv) + (size_t(l) * 2 + 0) * plane;
     __nv_bfloat16* vpl = reinterpret_cast<__nv_bfloat16*>(e->kv) + (size_t(l) * 2 + 1) * plane;
     al.layer = l;
@@ -920,16 +969,17 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
         TimerScope ts(e, QOS_T_EMBED, gs);
         QOS_CU(launch_embed_rmsnorm(tok + r0, W(e, e->wl.emb), W(e, L.ln1), resid + r0 * d, h + r0 * d, g.n, d,
                                     c.rms_eps, gs));
-      } else if (!tp) {  // (tp: ln1 was applied by the add+norm after the previous all-reduce)
+      } else if (!tp && !fold) {  // (tp: ln1 was applied by the add+norm after the previous all-reduce)
         TimerScope ts(e, QOS_T_NORM, gs);
-        QOS_CU(launch_rmsnorm(resid + r0 * d, W(e, L.ln1), h + r0 * d, g.n, d, c.rms_eps, gs));
+        if (!g_skip_norm) QOS_CU(launch_rmsnorm(resid + r0 * d, W(e, L.ln1), h + r0 * d, g.n, d, c.rms_eps, gs));
       }
       {
         // a4 + a5 + a6: QKV projection (+bias) with RoPE and the paged KV append in its epilogue
         TimerScope ts(e, QOS_T_GEMM_QKV, gs);
         const QkvRopeArgs ra{pos + r0, slot + r0, e->rope_tab, kpl, vpl, e->sh.H, e->sh.Hkv, hd};
         QOS_TRY(gemm_seg(e, g, e->a_h, M.qkv, e->nqkv, d, EPI_QKV_ROPE, qkv, e->nqkv,
-                         c.qkv_bias ? reinterpret_cast<const float*>(e->w + L.bqkv) : nullptr, &ra));
+                         c.qkv_bias ? reinterpret_cast<const float*>(e->w + L.bqkv) : nullptr, &ra,
+                         fold && l > 0 ? &f_qkv : nullptr));
       }
       // a7 || a8: within one segment, the prefill tiles go to the high-priority side stream and
       // the decode split-K items stay on the segment's stream (disjoint rows of `attn`)
@@ -955,7 +1005,8 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
       }
       if (!tp) {
         TimerScope ts(e, QOS_T_GEMM_O, gs);
-        QOS_TRY(gemm_seg(e, g, e->a_attn, M.o, d, e->sh.H * hd, EPI_ADD_F32, resid, d, nullptr));
+        QOS_TRY(gemm_seg(e, g, e->a_attn, M.o, d, e->sh.H * hd, EPI_ADD_F32, resid, d, nullptr, nullptr,
+                         fold ? &f_o : nullptr));
       } else {
         {
           TimerScope ts(e, QOS_T_GEMM_O, gs);
@@ -963,17 +1014,19 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
         }
         QOS_TRY(tp_reduce_add_norm(e, W(e, L.ln2), T, gs));
       }
-      if (!tp) {
+      if (!tp && !fold) {
         TimerScope ts(e, QOS_T_NORM, gs);
-        QOS_CU(launch_rmsnorm(resid + r0 * d, W(e, L.ln2), h + r0 * d, g.n, d, c.rms_eps, gs));
+        if (!g_skip_norm) QOS_CU(launch_rmsnorm(resid + r0 * d, W(e, L.ln2), h + r0 * d, g.n, d, c.rms_eps, gs));
       }
       {
         TimerScope ts(e, QOS_T_GEMM_GATEUP, gs);
-        QOS_TRY(gemm_seg(e, g, e->a_h, M.gu, 2 * e->sh.F, d, EPI_SILU_GATE, act, e->sh.F, nullptr));
+        QOS_TRY(gemm_seg(e, g, e->a_h, M.gu, 2 * e->sh.F, d, EPI_SILU_GATE, act, e->sh.F, nullptr, nullptr,
+                         fold ? &f_gu : nullptr));
       }
       if (!tp) {
         TimerScope ts(e, QOS_T_GEMM_DOWN, gs);
-        QOS_TRY(gemm_seg(e, g, e->a_act, M.d, d, e->sh.F, EPI_ADD_F32, resid, d, nullptr));
+        QOS_TRY(gemm_seg(e, g, e->a_act, M.d, d, e->sh.F, EPI_ADD_F32, resid, d, nullptr, nullptr,
+                         fold_down ? &f_down : nullptr));
       } else {
         {
           TimerScope ts(e, QOS_T_GEMM_DOWN, gs);
@@ -1327,7 +1380,10 @@ static int create_engine(const qos_model_cfg* cfg, int device, int tp_rank, int 
   // split-K arrival counters start at zero; the combining item / reducing CTA resets its counter
   if (cudaMemset(e->ws + e->wsl.counters, 0, size_t(cfg->max_batch_rows) * e->sh.Hkv * 4) != cudaSuccess ||
       cudaMemset(e->ws + e->wsl.gemm_cnt, 0, size_t(kGemmMaxTiles) * 4) != cudaSuccess ||
-      cudaMemset(e->ws + e->wsl.gemm_cnt2, 0, size_t(kGemmMaxTiles) * 4) != cudaSuccess)
+      cudaMemset(e->ws + e->wsl.gemm_cnt2, 0, size_t(kGemmMaxTiles) * 4) != cudaSuccess ||
+      cudaMemset(e->ws + e->wsl.ss[0], 0, size_t(cfg->max_batch_tokens) * kFoldSlots * 4) != cudaSuccess ||
+      cudaMemset(e->ws + e->wsl.ss[1], 0, size_t(cfg->max_batch_tokens) * kFoldSlots * 4) != cudaSuccess ||
+      cudaMemset(e->ws + e->wsl.fcnt, 0, size_t(cfg->max_batch_tokens / 128 + 2) * 4) != cudaSuccess)
     return fail(set_error(QOS_ERR_CUDA, "counter memset"));
   if (cudaMalloc(&e->d_tables, size_t(cfg->max_requests) * e->table_w * 4) != cudaSuccess)
     return fail(set_error(QOS_ERR_OOM, "block tables"));
@@ -1750,6 +1806,7 @@ int qos_engine_set_option(qos_engine_t* e, const char* name, int64_t value) {
   else if (n == "decode_round_split") e->decode_round_split = value != 0;
   else if (n == "gemm_2cta") e->gemm_2cta = value != 0;
   else if (n == "fa_persist") e->fa_persist = value != 0;
+  else if (n == "norm_fold") e->norm_fold = value != 0;
   else if (n == "tp_twoshot") e->tp_twoshot = value < 0 ? -1 : value > 0 ? 1 : 0;
   else if (n == "decode_stages") {
     if (value != 4 && value != 8) return set_error(QOS_ERR_INVALID_ARG, "decode_stages must be 4 or 8");

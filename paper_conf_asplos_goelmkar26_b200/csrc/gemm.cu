@@ -73,7 +73,28 @@ struct GemmArgs {
   __nv_bfloat16* kplane;  // [blocks][Hkv][16][hd] of this layer
   __nv_bfloat16* vplane;
   int H, Hkv, hd;
+  // folded RMSNorm (NormFold, internal.h)
+  const float* rs_in;
+  float* ss_out;
+  float* rs_out;
+  int* fcnt;
+  const __nv_bfloat16* g_out;
+  __nv_bfloat16* h_out;
+  int ss_n;
+  float inv_d, rms_eps;
 };
+
+static void set_fold(GemmArgs& a, const NormFold* f) {
+  a.rs_in = f ? f->rs_in : nullptr;
+  a.ss_out = f ? f->ss_out : nullptr;
+  a.rs_out = f ? f->rs_out : nullptr;
+  a.fcnt = f ? f->cnt : nullptr;
+  a.g_out = f ? reinterpret_cast<const __nv_bfloat16*>(f->g_out) : nullptr;
+  a.h_out = f ? reinterpret_cast<__nv_bfloat16*>(f->h_out) : nullptr;
+  a.ss_n = f ? f->ss_n : 0;
+  a.inv_d = f && f->d ? 1.f / float(f->d) : 0.f;
+  a.rms_eps = f ? f->eps : 0.f;
+}
 
 // ---- epilogue stores of one thread's 32 consecutive accumulator columns of one row
 template <int EPI>
@@ -345,13 +366,19 @@ QOS_DEV void epi_bar_sync() { asm volatile("bar.sync 1, 128;" ::: "memory"); }  
 template <int BN, int EPI>
 QOS_DEV void epi_tile_staged(const GemmArgs& p, uint8_t* stg, int lane, int n_t, int row, uint32_t tbase) {
         const int row0 = row - lane;
+        // folded RMSNorm, consumer side: this row's 1/rms from the producer's per-block sums
+        float rs = 1.f;
+        if constexpr (EPI == EPI_QKV_ROPE || EPI == EPI_SILU_GATE) {
+          if (p.rs_in != nullptr && row < p.M) rs = __ldcg(p.rs_in + row);
+        }
         if constexpr (EPI == EPI_QKV_ROPE) {
           epi_qkv_rope_staged<BN>(p, stg, lane, row0, n_t, [&](int col, float (&v)[16]) {
             uint32_t r[16];
             tmem_ld32x32b_x16(tbase + col, r);
             tmem_ld_wait();
 #pragma unroll
-            for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]) + (p.bias ? __ldg(p.bias + n_t * BN + col + i) : 0.f);
+            for (int i = 0; i < 16; ++i)
+              v[i] = __uint_as_float(r[i]) * rs + (p.bias ? __ldg(p.bias + n_t * BN + col + i) : 0.f);
           });
         } else if constexpr (EPI == EPI_SILU_GATE) {
 #pragma unroll 1
@@ -363,6 +390,11 @@ QOS_DEV void epi_tile_staged(const GemmArgs& p, uint8_t* stg, int lane, int n_t,
               tmem_ld32(tbase + g * 128 + 64 + h * 32, uv);
               const int col = n_t * (BN / 2) + g * 64 + h * 32;
               if (col >= p.N / 2) continue;  // warp-uniform
+#pragma unroll
+              for (int i = 0; i < 32; ++i) {
+                gv[i] *= rs;
+                uv[i] *= rs;
+              }
               uint32_t pk[16];
 #pragma unroll
               for (int i = 0; i < 16; ++i) pk[i] = pack_bf16(silu(gv[2 * i]) * uv[2 * i], silu(gv[2 * i + 1]) * uv[2 * i + 1]);
@@ -373,6 +405,93 @@ QOS_DEV void epi_tile_staged(const GemmArgs& p, uint8_t* stg, int lane, int n_t,
                   reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.C) + size_t(row0 + rr) * p.ldc + col)[k] = v;
               });
             }
+          }
+        } else if (EPI == EPI_ADD_F32 && p.ss_out != nullptr) {
+          // folded RMSNorm, producer side: r += tile (read-add-write), h = bf16(r * g_out), and
+          // per 128-column block the row's sum of r^2.  Lane = (row rr = pass*4 + lane/8, 16-B
+          // chunk k = lane%8) of the staged 32 x 32 fp32 block; the 8 lanes of a row reduce by
+          // shuffles, per-block sums accumulate over the block's four 32-column chunks.
+          float acc8[8];
+#pragma unroll
+          for (int i = 0; i < 8; ++i) acc8[i] = 0.f;
+#pragma unroll 1
+          for (int c = 0; c < BN / 32; ++c) {
+            float v[32];
+            tmem_ld32(tbase + c * 32, v);
+            const int col = n_t * BN + c * 32;
+            if (col >= p.N) continue;  // warp-uniform (whole 128-column blocks: N % 128 == 0)
+#pragma unroll
+            for (int k = 0; k < 8; ++k)
+              stg_put<128>(stg, lane, k, make_uint4(__float_as_uint(v[4 * k]), __float_as_uint(v[4 * k + 1]),
+                                                    __float_as_uint(v[4 * k + 2]), __float_as_uint(v[4 * k + 3])));
+            __syncwarp();
+            // the residual chunks of all 8 passes requested at once (one L2 latency per chunk)
+            float4 old[8];
+#pragma unroll
+            for (int pass = 0; pass < 8; ++pass) {
+              const int r = row0 + pass * 4 + (lane >> 3);
+              old[pass] = r < p.M ? *reinterpret_cast<const float4*>(reinterpret_cast<const float*>(p.C) +
+                                                                    size_t(r) * p.ldc + col + 4 * (lane & 7))
+                                  : make_float4(0.f, 0.f, 0.f, 0.f);
+            }
+            const uint2 gg = __ldg(reinterpret_cast<const uint2*>(p.g_out + col + 4 * (lane & 7)));
+#pragma unroll
+            for (int pass = 0; pass < 8; ++pass) {
+              const int rr = pass * 4 + (lane >> 3), k = lane & 7;
+              const int r = row0 + rr;
+              float sq = 0.f;
+              if (r < p.M) {
+                const uint4 x = *reinterpret_cast<const uint4*>(stg + stg_off<128>(rr, k));
+                float* dr = reinterpret_cast<float*>(p.C) + size_t(r) * p.ldc + col + 4 * k;
+                float4 o = old[pass];
+                o.x += __uint_as_float(x.x);
+                o.y += __uint_as_float(x.y);
+                o.z += __uint_as_float(x.z);
+                o.w += __uint_as_float(x.w);
+                *reinterpret_cast<float4*>(dr) = o;
+                *reinterpret_cast<uint2*>(p.h_out + size_t(r) * p.N + col + 4 * k) =
+                    make_uint2(pack_bf16(o.x * bf16_lo(gg.x), o.y * bf16_hi(gg.x)),
+                               pack_bf16(o.z * bf16_lo(gg.y), o.w * bf16_hi(gg.y)));
+                sq = (o.x * o.x + o.y * o.y) + (o.z * o.z + o.w * o.w);
+              }
+              sq += __shfl_xor_sync(0xffffffffu, sq, 1);
+              sq += __shfl_xor_sync(0xffffffffu, sq, 2);
+              sq += __shfl_xor_sync(0xffffffffu, sq, 4);
+              acc8[pass] += sq;
+            }
+            __syncwarp();
+            if ((c & 3) == 3) {  // end of a 128-column block: one partial per row
+              if ((lane & 7) == 0) {
+#pragma unroll
+                for (int pass = 0; pass < 8; ++pass) {
+                  const int r = row0 + pass * 4 + (lane >> 3);
+                  if (r < p.M) p.ss_out[size_t(r) * kFoldSlots + col / 128] = acc8[pass];
+                }
+              }
+#pragma unroll
+              for (int i = 0; i < 8; ++i) acc8[i] = 0.f;
+            }
+          }
+          // the last tile of this 128-row block to finish turns the per-block sums into 1/rms
+          __shared__ int s_fold_last;
+          __threadfence();
+          epi_bar_sync();
+          const int rb = row >> 7;
+          if ((row & 127) == 0) s_fold_last = atomicAdd(p.fcnt + rb, 1) == p.nt - 1;
+          epi_bar_sync();
+          if (s_fold_last) {
+            __threadfence();
+            if (row < p.M) {
+              const float4* sp = reinterpret_cast<const float4*>(p.ss_out + size_t(row) * kFoldSlots);
+              float4 x[kFoldSlots / 4];
+#pragma unroll
+              for (int j = 0; j < kFoldSlots / 4; ++j) x[j] = __ldcg(sp + j);
+              float t = 0.f;
+#pragma unroll
+              for (int j = 0; j < kFoldSlots / 4; ++j) t += (x[j].x + x[j].y) + (x[j].z + x[j].w);
+              p.rs_out[row] = rsqrtf(t * p.inv_d + p.rms_eps);
+            }
+            if ((row & 127) == 0) p.fcnt[rb] = 0;  // ready for the next launch
           }
         } else {
 #pragma unroll 1
@@ -1058,8 +1177,11 @@ int gemm_pick_ksplit(int64_t M, int64_t N, int64_t K, int bn, int num_sms, int64
 
 int gemm_run(const CUtensorMap& ta, const CUtensorMap& tb, int bn, int64_t M, int64_t N, int64_t K, int epi, void* C,
              int64_t ldc, const float* bias, int num_sms, cudaStream_t st, int ksplit, float* part, int* counters,
-             int a_row0, int max_ctas, const QkvRopeArgs* rope, int sk_mode, bool coop) {
+             int a_row0, int max_ctas, const QkvRopeArgs* rope, int sk_mode, bool coop, const NormFold* fold) {
   GemmArgs a;
+  set_fold(a, fold);
+  if (fold && ksplit > 1) return set_error(QOS_ERR_INVALID_ARG, "gemm: folded norm needs one pass");
+  if (fold) sk_mode = 0;  // whole tiles only
   a.M = int(M);
   a.N = int(N);
   a.K = int(K);
@@ -1146,8 +1268,9 @@ bool gemm2_eligible(int64_t M, int64_t N, int64_t K, int num_sms) {
 // tb: tensor map over B with 128-row boxes; ta: over A with 128-row boxes
 int gemm2_run(const CUtensorMap& ta, const CUtensorMap& tb, int64_t M, int64_t N, int64_t K, int epi, void* C,
               int64_t ldc, const float* bias, int num_sms, cudaStream_t st, int a_row0, int max_ctas,
-              const QkvRopeArgs* rope) {
+              const QkvRopeArgs* rope, const NormFold* fold) {
   GemmArgs a{};
+  set_fold(a, fold);
   a.M = int(M);
   a.N = int(N);
   a.K = int(K);

@@ -43,16 +43,35 @@ int gemm_check_shape(int64_t M, int64_t N, int64_t K, int epi);
 int gemm_pick_ksplit(int64_t M, int64_t N, int64_t K, int bn, int num_sms, int64_t max_units);
 // ksplit > 1: split-K with fp32 partials in `part` ([units][128][bn]) and per-tile arrival
 // counters (zero-initialised; each reducing CTA resets its own) — deterministic reduction order
+// RMSNorm folded into the projections (single-pass tile kernels, no split-K / stream-K):
+//   consumer (QKV, gate/up): A = bf16(r * g) rows; the accumulator of row t is scaled by
+//     rs_in[t] = 1/rms(r_t) (before the bias) — diag(s)(A W) = (diag(s) A) W;
+//   producer (O, down with EPI_ADD_F32): r += tile as a read-add-write, h_out = bf16(r * g_out),
+//     ss_out[t][col / 128] = the sum of r^2 over that 128-column block; the last tile to finish
+//     a 128-row block (arrival counter) sums each row's blocks in slot order into rs_out[t]
+//     (fixed order: deterministic).
+constexpr int kFoldSlots = 64;
+constexpr int kFoldMinTokens = 1536;  // the engine folds the norms from this many tokens per step  // ss row stride: 128-column blocks of d <= 8192 (unused slots stay 0)
+struct NormFold {
+  const float* rs_in = nullptr;  // consumer: [M] 1/rms per row
+  float* ss_out = nullptr;       // producer: [M][kFoldSlots] per-block sums of squares
+  float* rs_out = nullptr;       // producer: [M] 1/rms, written by the last tile of each 128-row block
+  int* cnt = nullptr;            // producer: [M/128 + 1] tile arrival counters (zero between launches)
+  const void* g_out = nullptr;  // bf16 [d]
+  void* h_out = nullptr;        // bf16 [M][d]
+  int ss_n = 0, d = 0;
+  float eps = 0.f;
+};
 int gemm_run(const CUtensorMap& ta, const CUtensorMap& tb, int bn, int64_t M, int64_t N, int64_t K, int epi, void* C,
              int64_t ldc, const float* bias, int num_sms, cudaStream_t st, int ksplit = 1, float* part = nullptr,
              int* counters = nullptr, int a_row0 = 0, int max_ctas = 0, const QkvRopeArgs* rope = nullptr,
-             int sk_mode = 1, bool coop = true);
+             int sk_mode = 1, bool coop = true, const NormFold* fold = nullptr);
 // CTA-pair (cta_group::2) GEMM with 256 x 256 tiles for large M (gemm.cu); ta / tb: tensor
 // maps with 128-row boxes over A and B.  gemm2_eligible: the shapes it takes.
 bool gemm2_eligible(int64_t M, int64_t N, int64_t K, int num_sms);
 int gemm2_run(const CUtensorMap& ta, const CUtensorMap& tb, int64_t M, int64_t N, int64_t K, int epi, void* C,
               int64_t ldc, const float* bias, int num_sms, cudaStream_t st, int a_row0 = 0, int max_ctas = 0,
-              const QkvRopeArgs* rope = nullptr);
+              const QkvRopeArgs* rope = nullptr, const NormFold* fold = nullptr);
 // sk_mode: 0 no stream-K, 1 automatic (last-wave quantisation), 2 always (needs part/counters:
 // part >= 512 x 128 x 256 fp32, counters >= 4096); coop as in gemm_swab_run.
 

@@ -38,7 +38,8 @@ from dataclasses import dataclass, field
 
 import numpy as np
 
-N_FEAT = 12
+N_FEAT = 14
+FOLD_MIN_TOKENS = 1536   # kFoldMinTokens (csrc/internal.h)
 
 
 @dataclass
@@ -129,10 +130,11 @@ def features(s: StepShape, g: GemmShapes = GemmShapes()) -> np.ndarray:
     nd = len(s.ctx)
     n_pair = sum(1 for N, K in g.gemms if s.T > 0 and pair_eligible(s.T, N, K, g.num_sms))
     n_stream = sum(1 for N, K in g.gemms if s.T > 0 and swab_prefer_k(s.T, N, K, g.num_sms))
+    fold = 1.0 if (s.T >= FOLD_MIN_TOKENS and n_stream == 0) else 0.0   # mirrors run_layers' norm fold
     return np.array([gemm_work(s.T, g) / 100.0, s.T / 1000.0, sum(c + 1 for c in s.ctx) / 1e6, nd / 100.0,
                      1.0 if nd else 0.0, 1.0, sum(n * (n + 1) / 2 for ks, n in s.chunks) / 1e7,
                      stream_work(s.T, g) / 1e8, sum(n * ks for ks, n in s.chunks) / 1e7, pair_work(s.T, g) / 100.0,
-                     float(n_pair), float(len(g.gemms) - n_pair - n_stream)])
+                     float(n_pair), float(len(g.gemms) - n_pair - n_stream), fold, fold * s.T / 1000.0])
 
 
 class LatencyModel:

@@ -203,7 +203,8 @@ def test_llama8b_shapes_bench_batch_sampled_parity():
 @pytest.mark.parametrize("opts", [{"overlap_attn": 0}, {"gemm_splitk": 1}, {"pdl": 0}, {"gemm_swab": 0},
                                   {"gemm_streamk": 0}, {"gemm_streamk": 2, "gemm_swab": 0},
                                   {"gemm_swab": 2}, {"decode_round_split": 0}, {"fa_poly": 0}, {"fa_poly": 2},
-                                  {"fa_qtiles": 2}, {"fa_persist": 0}, {"gemm_2cta": 0}, {"decode_stages": 4},
+                                  {"fa_qtiles": 2}, {"fa_persist": 0}, {"gemm_2cta": 0},
+                                  {"norm_fold": 0}, {"gemm_swab": 0, "norm_fold": 1}, {"gemm_swab": 0, "gemm_2cta": 0}, {"decode_stages": 4},
                                   {"dual_stream": 1, "dual_min_prefill": 1, "dual_min_decode": 1}])
 def test_execution_options_do_not_change_results(opts):
     """qos_engine_set_option variants (serial attention, no split-K, two-stream sub-batches)
@@ -255,4 +256,30 @@ def test_long_context_step_parity():
     gap = ref[np.arange(len(ref)), top[:, -1]] - ref[np.arange(len(ref)), top[:, -2]]
     clear = gap > 2 * TOL_LOGITS * np.abs(ref).max(axis=1)
     assert np.array_equal(np.asarray(tk)[clear], top[clear, -1])
+    eng.close()
+
+
+@pytest.mark.parametrize("fold", [1, 0])
+def test_norm_fold_large_step_parity(fold):
+    """The RMSNorm folded into the projections (taken from 1536 tokens per step: the O / down
+    epilogues write r, bf16(r * g) and per-block sums of squares, the QKV / gate-up epilogues
+    scale rows by 1/rms) against the oracle on a 1700-token chunk + decodes, tiny shapes."""
+    q, cfg, eng = make_engine("tiny", num_blocks=512, max_batch_tokens=2048, max_seq_len=4096)
+    eng.qos_engine_load_synthetic(0)
+    eng.qos_engine_set_option("norm_fold", fold)
+    orc = _oracle("tiny", num_blocks=512)
+    rng = np.random.default_rng(11)
+    toks = [int(x) for x in rng.integers(0, cfg.vocab, 1700)]
+    eng.qos_kv_alloc(1, 1700)
+    orc.kv_alloc(1, 1700)
+    decs = []
+    for r, n in ((2, 40), (3, 300)):
+        eng.qos_kv_alloc(r, n + 1)
+        orc.kv_alloc(r, n + 1)
+        eng.qos_kv_fill_synthetic(r, n, synth.SEED_KVFILL)
+        orc.kv_fill_synthetic(r, n, synth.SEED_KVFILL)
+        decs.append((r, n, int(rng.integers(0, cfg.vocab))))
+    lg, tk = eng.step_host(q.make_batch([(1, 0, np.array(toks, np.int32))], decs), cfg.vocab)
+    ref = orc.hybrid_step([(1, 0, toks)], decs)
+    assert row_rel_err(lg, ref) <= TOL_LOGITS
     eng.close()

@@ -6,7 +6,7 @@ import os
 
 import numpy as np
 
-from paper_conf_asplos_goelmkar26_b200.latency_model import (GemmShapes, LatencyModel, StepShape, features, gemm_work,
+from paper_conf_asplos_goelmkar26_b200.latency_model import (N_FEAT, GemmShapes, LatencyModel, StepShape, features, gemm_work,
                                                              pair_eligible, pair_work, stream_work)
 
 PROF = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles", "latency_table_r1.json")
@@ -14,7 +14,8 @@ PROF = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))),
 
 def test_recovers_known_coefficients():
     rng = np.random.default_rng(0)
-    true = np.array([2.0, 3.0, 20.0, 0.5, 1.0, 4.0, 9.0, 6.0, 5.0, 1.5, 0.3, 0.2])
+    true = np.array([2.0, 3.0, 20.0, 0.5, 1.0, 4.0, 9.0, 6.0, 5.0, 1.5, 0.3, 0.2, -0.4, -0.3])
+    assert len(true) == N_FEAT
     shapes = [StepShape([], list(rng.integers(1024, 8193, nd))) for nd in (1, 8, 16, 24, 32, 64, 100, 200, 256)]
     for _ in range(120):
         c = int(rng.integers(0, 8193))

@@ -17,16 +17,17 @@ cap() {  # name, kernel regex, skip
       python tools/profile_step.py --steps 1 --layers 2 > $OUT/ncu_${1}_$TAG.log 2>&1
 }
 # GEMM launches per layer at T = 2176: QKV(+RoPE), O and down on the CTA-pair kernel
-# (gemm2_tcgen05_kernel: layer 1 = launches 3, 4, 5), gate/up on the single-CTA tile kernel
+# (gemm2_tcgen05_kernel: layer 1 QKV = 3, O = 4; layer 0 down = 2, whose epilogue carries the folded
+# norm), gate/up on the single-CTA tile kernel
 # (gemm_tcgen05_kernel: layer 1 = launch 1)
 if [ "${ONLY_ATTN:-0}" != 1 ]; then
 cap gemm_qkv_rope 'gemm2_tcgen05_kernel' 3
 cap gemm_o 'gemm2_tcgen05_kernel' 4
-cap gemm_down 'gemm2_tcgen05_kernel' 5
+cap gemm_down 'gemm2_tcgen05_kernel' 2
 cap gemm_gateup 'gemm_tcgen05_kernel' 1
 fi
 if [ "${ONLY_GEMM:-0}" != 1 ]; then
 cap decode_attn 'decode_attn_kernel' 1
-cap prefill_attn 'prefill_attn_tc_kernel' 1
+cap prefill_attn 'prefill_attn_(tc|persist)_kernel' 1
 fi
 ls -la $OUT
