@@ -410,46 +410,49 @@ QOS_DEV void epi_tile_staged(const GemmArgs& p, uint8_t* stg, int lane, int n_t,
           // folded RMSNorm, producer side: r += tile (read-add-write), h = bf16(r * g_out), and
           // per 128-column block the row's sum of r^2.  Lane = (row rr = pass*4 + lane/8, 16-B
           // chunk k = lane%8) of the staged 32 x 32 fp32 block; the 8 lanes of a row reduce by
-          // shuffles, per-block sums accumulate over the block's four 32-column chunks.
+          // shuffles, per-block sums accumulate over the block's four 32-column chunks.  The
+          // residual chunks of 32-column block c+1 are requested before block c is processed
+          // (two register sets), so the read-add-write costs about one L2 latency per tile.
+          const int k8 = lane & 7;
+          auto load_old = [&](int c, float4 (&o)[8]) {
+            const int col = n_t * BN + c * 32;
+#pragma unroll
+            for (int pass = 0; pass < 8; ++pass) {
+              const int r = row0 + pass * 4 + (lane >> 3);
+              o[pass] = (r < p.M && col < p.N)
+                            ? *reinterpret_cast<const float4*>(reinterpret_cast<const float*>(p.C) + size_t(r) * p.ldc +
+                                                               col + 4 * k8)
+                            : make_float4(0.f, 0.f, 0.f, 0.f);
+            }
+          };
           float acc8[8];
 #pragma unroll
           for (int i = 0; i < 8; ++i) acc8[i] = 0.f;
-#pragma unroll 1
-          for (int c = 0; c < BN / 32; ++c) {
+          auto process = [&](int c, const float4 (&old)[8]) {
             float v[32];
             tmem_ld32(tbase + c * 32, v);
             const int col = n_t * BN + c * 32;
-            if (col >= p.N) continue;  // warp-uniform (whole 128-column blocks: N % 128 == 0)
+            if (col >= p.N) return;  // warp-uniform (whole 128-column blocks: N % 128 == 0)
 #pragma unroll
             for (int k = 0; k < 8; ++k)
               stg_put<128>(stg, lane, k, make_uint4(__float_as_uint(v[4 * k]), __float_as_uint(v[4 * k + 1]),
                                                     __float_as_uint(v[4 * k + 2]), __float_as_uint(v[4 * k + 3])));
             __syncwarp();
-            // the residual chunks of all 8 passes requested at once (one L2 latency per chunk)
-            float4 old[8];
+            const uint2 gg = __ldg(reinterpret_cast<const uint2*>(p.g_out + col + 4 * k8));
 #pragma unroll
             for (int pass = 0; pass < 8; ++pass) {
-              const int r = row0 + pass * 4 + (lane >> 3);
-              old[pass] = r < p.M ? *reinterpret_cast<const float4*>(reinterpret_cast<const float*>(p.C) +
-                                                                    size_t(r) * p.ldc + col + 4 * (lane & 7))
-                                  : make_float4(0.f, 0.f, 0.f, 0.f);
-            }
-            const uint2 gg = __ldg(reinterpret_cast<const uint2*>(p.g_out + col + 4 * (lane & 7)));
-#pragma unroll
-            for (int pass = 0; pass < 8; ++pass) {
-              const int rr = pass * 4 + (lane >> 3), k = lane & 7;
+              const int rr = pass * 4 + (lane >> 3);
               const int r = row0 + rr;
               float sq = 0.f;
               if (r < p.M) {
-                const uint4 x = *reinterpret_cast<const uint4*>(stg + stg_off<128>(rr, k));
-                float* dr = reinterpret_cast<float*>(p.C) + size_t(r) * p.ldc + col + 4 * k;
+                const uint4 x = *reinterpret_cast<const uint4*>(stg + stg_off<128>(rr, k8));
                 float4 o = old[pass];
                 o.x += __uint_as_float(x.x);
                 o.y += __uint_as_float(x.y);
                 o.z += __uint_as_float(x.z);
                 o.w += __uint_as_float(x.w);
-                *reinterpret_cast<float4*>(dr) = o;
-                *reinterpret_cast<uint2*>(p.h_out + size_t(r) * p.N + col + 4 * k) =
+                *reinterpret_cast<float4*>(reinterpret_cast<float*>(p.C) + size_t(r) * p.ldc + col + 4 * k8) = o;
+                *reinterpret_cast<uint2*>(p.h_out + size_t(r) * p.N + col + 4 * k8) =
                     make_uint2(pack_bf16(o.x * bf16_lo(gg.x), o.y * bf16_hi(gg.x)),
                                pack_bf16(o.z * bf16_lo(gg.y), o.w * bf16_hi(gg.y)));
                 sq = (o.x * o.x + o.y * o.y) + (o.z * o.z + o.w * o.w);
@@ -461,7 +464,7 @@ QOS_DEV void epi_tile_staged(const GemmArgs& p, uint8_t* stg, int lane, int n_t,
             }
             __syncwarp();
             if ((c & 3) == 3) {  // end of a 128-column block: one partial per row
-              if ((lane & 7) == 0) {
+              if (k8 == 0) {
 #pragma unroll
                 for (int pass = 0; pass < 8; ++pass) {
                   const int r = row0 + pass * 4 + (lane >> 3);
@@ -471,6 +474,15 @@ QOS_DEV void epi_tile_staged(const GemmArgs& p, uint8_t* stg, int lane, int n_t,
 #pragma unroll
               for (int i = 0; i < 8; ++i) acc8[i] = 0.f;
             }
+          };
+          float4 oa[8], ob[8];
+          load_old(0, oa);
+#pragma unroll 1
+          for (int c = 0; c < BN / 32; c += 2) {  // BN / 32 is even
+            load_old(c + 1, ob);
+            process(c, oa);
+            if (c + 2 < BN / 32) load_old(c + 2, oa);
+            process(c + 1, ob);
           }
           // the last tile of this 128-row block to finish turns the per-block sums into 1/rms
           __shared__ int s_fold_last;
