@@ -61,7 +61,7 @@ def main():
         model = LatencyModel().fit(shapes, ms)
     else:
         prof = json.load(open(os.path.join(ROOT, "profiles", "latency_table_r1.json")))
-        model = LatencyModel.from_json(json.dumps(prof.get("refit", prof)["model_json"]))
+        model = LatencyModel.from_json(json.dumps(prof["model_json"]))
 
     def pred(chunks, ctx):
         return model.predict(StepShape(list(chunks), list(ctx)))
