@@ -420,8 +420,8 @@ QOS_DEV void epi_tile_staged(const GemmArgs& p, uint8_t* stg, int lane, int n_t,
             for (int pass = 0; pass < 8; ++pass) {
               const int r = row0 + pass * 4 + (lane >> 3);
               o[pass] = (r < p.M && col < p.N)
-                            ? *reinterpret_cast<const float4*>(reinterpret_cast<const float*>(p.C) + size_t(r) * p.ldc +
-                                                               col + 4 * k8)
+                            ? __ldcg(reinterpret_cast<const float4*>(reinterpret_cast<const float*>(p.C) + size_t(r) * p.ldc +
+                                                                     col + 4 * k8))
                             : make_float4(0.f, 0.f, 0.f, 0.f);
             }
           };
@@ -485,11 +485,15 @@ QOS_DEV void epi_tile_staged(const GemmArgs& p, uint8_t* stg, int lane, int n_t,
             process(c + 1, ob);
           }
           // the last tile of this 128-row block to finish turns the per-block sums into 1/rms
+          // (the barrier orders the 4 warps' stores before thread 0's fence + arrival — one fence
+          //  per tile, as in a grid barrier, instead of a full fence in every thread)
           __shared__ int s_fold_last;
-          __threadfence();
           epi_bar_sync();
           const int rb = row >> 7;
-          if ((row & 127) == 0) s_fold_last = atomicAdd(p.fcnt + rb, 1) == p.nt - 1;
+          if ((row & 127) == 0) {
+            __threadfence();
+            s_fold_last = atomicAdd(p.fcnt + rb, 1) == p.nt - 1;
+          }
           epi_bar_sync();
           if (s_fold_last) {
             __threadfence();

@@ -120,6 +120,7 @@ class SchedulerConfig:
     chunk_step: int = 64
     margin: float = 0.05              # under-predict the chunk
     max_decodes: int = 256
+    max_rows: int = 264               # engine capacity: chunks + decodes per step (max_batch_rows)
     # "slack": QoServe's dynamic chunking (the chunk fits the minimum decode slack);
     # "medha": Medha-style adaptive chunking (NEXT-4 variant): every step
     # targets a fixed latency, so chunks shrink as the prefill's cached prefix grows
@@ -216,8 +217,12 @@ class QoServeScheduler:
         chunks, count = [], 0
         inflight_skipped = []
         i = 0
-        while count < C and i < len(queue):                           # line 10
+        while count < C and i < len(queue) and len(chunks) + len(decodes) < self.cfg.max_rows:   # line 10
             top = queue[i]
+            if top.prefill_done == 0 and len(self.decode_q) >= self.cfg.max_decodes:
+                # admission: a new prompt would finish into a full decode set (engine capacity)
+                i += 1
+                continue
             if not top.relegated and self.will_violate(top, now, C, ctx):   # line 12
                 # eager relegation with hints: free-tier first; important requests only once
                 # they have actually missed their deadline
@@ -239,6 +244,8 @@ class QoServeScheduler:
                 if self.will_violate(r, now + self.step_estimate_s(C, ctx), max(C, 1), ctx):
                     inflight_skipped.append(r)
         for r in inflight_skipped:
+            if len(chunks) + len(decodes) >= self.cfg.max_rows:
+                break
             take = min(max(self.cfg.min_chunk, C - count), r.prefill_rem)
             chunks.append((r, take))
             count += take

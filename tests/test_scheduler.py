@@ -160,7 +160,8 @@ def test_budget_prices_the_chunk_prefix():
 def test_medha_policy_shrinks_chunks_of_a_long_prefill():
     """NEXT-4 variant (Medha, PAPER.md:1597-1649): one 10K-token prefill next to 500 decodes;
     with a fixed per-step target every step fits it and the chunk shrinks as the prefix grows."""
-    cfg = SchedulerConfig(max_chunk=8192, margin=0.0, chunk_policy="medha", medha_target_ms=40.0)
+    cfg = SchedulerConfig(max_chunk=8192, margin=0.0, chunk_policy="medha", medha_target_ms=40.0, max_decodes=512,
+                          max_rows=520)
     s = QoServeScheduler(cfg, prefix_model)
     decs = []
     for i in range(500):
@@ -195,3 +196,23 @@ def test_round_robin_replicas():
     tr1 = synth.trace(2.0, 20.0, "azure_conv")
     out1 = replay(tr1, QoServeScheduler(SchedulerConfig(max_chunk=2048), lin_model), ModelExecutor(lin_model))
     assert out8["violations_pct"] <= out1["violations_pct"] + 1.0
+
+
+def test_batches_respect_engine_capacity():
+    """Every batch fits the engine (chunks + decodes <= max_rows), and no new prompt is started
+    while the decode set is full (it would finish into a decode the engine cannot take)."""
+    cfg = SchedulerConfig(max_chunk=4096, max_decodes=8, max_rows=10)
+    s = QoServeScheduler(cfg, lambda chunks, ctx: 5.0 + 0.002 * sum(n for _, n in chunks) + 0.01 * len(ctx))
+    for i in range(8):
+        r = Request(100 + i, 0.0, 64, "Q2", decode_len=10 ** 6)
+        r.prefill_done = r.prompt_len
+        s.decode_q.append(r)
+    fresh = [Request(i, 0.0, 32, "Q1", decode_len=4) for i in range(6)]
+    for r in fresh:
+        s.submit(r)
+    chunks, decodes = s.create_batch(0.0)
+    assert len(chunks) + len(decodes) <= cfg.max_rows
+    assert not chunks                       # decode set full: no prompt is admitted
+    s.decode_q = s.decode_q[:4]             # four decodes leave
+    chunks, decodes = s.create_batch(0.0)
+    assert chunks and len(chunks) + len(decodes) <= cfg.max_rows

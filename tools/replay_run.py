@@ -70,7 +70,8 @@ def main():
         tr = synth.trace(qps, a.duration, a.dataset)
 
         def mk_sched():
-            return QoServeScheduler(SchedulerConfig(alpha_ms_per_token=a.alpha, max_chunk=a.max_chunk), pred)
+            return QoServeScheduler(SchedulerConfig(alpha_ms_per_token=a.alpha, max_chunk=a.max_chunk,
+                                                    max_decodes=256, max_rows=257), pred)
         if a.mode == "engine":
             ex = EngineExecutor(eng, 128256, lambda r, s, n: synth.request_tokens(r, n, 128256, start=s))
             out = replay(tr, mk_sched(), ex)
