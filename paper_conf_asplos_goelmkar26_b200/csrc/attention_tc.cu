@@ -1106,8 +1106,10 @@ cudaError_t launch_prefill_attention_tc(const AttnLaunch& a, const PrefillItem* 
   count_launch(1);
   const int poly = g_fa_poly;
   if (a.cta_off && a.q_tiles == 1 && poly >= 0) {  // persistent CTAs over per-CTA item lists
-    if (a.hd == 128) return poly == 0 ? prefill_persist_t<128, 0>(a, items, a.cta_off, a.n_cta, st)
-                                      : prefill_persist_t<128, 4>(a, items, a.cta_off, a.n_cta, st);
+    if (a.hd == 128) return poly == 0   ? prefill_persist_t<128, 0>(a, items, a.cta_off, a.n_cta, st)
+                            : poly == 2 ? prefill_persist_t<128, 2>(a, items, a.cta_off, a.n_cta, st)
+                            : poly == 3 ? prefill_persist_t<128, 3>(a, items, a.cta_off, a.n_cta, st)
+                                        : prefill_persist_t<128, 4>(a, items, a.cta_off, a.n_cta, st);
     if (a.hd == 64) return poly == 0 ? prefill_persist_t<64, 0>(a, items, a.cta_off, a.n_cta, st)
                                      : prefill_persist_t<64, 4>(a, items, a.cta_off, a.n_cta, st);
     return cudaErrorInvalidValue;
