@@ -262,6 +262,10 @@ int qos_profile_step_ex(qos_engine_t* eng, int32_t chunk_len, int32_t kv_start,
  *                          all rows), 1 two-shot (each rank reduces + normalises a row slice and
  *                          stores it into every peer: ~2(tp-1)/tp of one partial per rank instead
  *                          of tp-1), -1 automatic (two-shot when tp >= 4)
+ *   "tp_scatter" (1)       peer-group two-shot reduction with the reduce-scatter fused into the O /
+ *                          down GEMM epilogue: each partial row is stored straight into its owner
+ *                          rank's receive slot (peer memory) while the remaining tiles compute
+ *                          (one-pass tile kernels only; else the reducer reads the peers' partials)
  *   "fa_persist" (1)       prefill attention (fa_qtiles 1) as persistent CTAs, 2 per SM, each
  *                          running a host-dealt list of work items back to back (LPT greedy by
  *                          key tiles); the next item's Q is staged under the current epilogue

@@ -151,7 +151,7 @@ static WeightLayout weight_layout(const qos_model_cfg& c, const Shard& s) {
 }
 
 struct WsLayout {
-  size_t resid, h, qkv, attn, act, hR, logits, logits_loc, part[2], ss[2], rs[2], fcnt, argmax, partials, counters, gemm_part, gemm_cnt, gemm_part2,
+  size_t resid, h, qkv, attn, act, hR, logits, logits_loc, part[2], recv[2], ss[2], rs[2], fcnt, argmax, partials, counters, gemm_part, gemm_cnt, gemm_part2,
       gemm_cnt2, meta[2], dbg, total;
   size_t meta_bytes;
   int max_items;
@@ -184,6 +184,10 @@ static WsLayout ws_layout(const qos_model_cfg& c, const Shard& s, int tp) {
   w.rs[0] = take(Tm * 4);
   w.rs[1] = take(Tm * 4);
   w.fcnt = take((Tm / 128 + 2) * 4);
+  // peer-group reduce-scatter: receive slots [tp][ceil(Tm/tp)][d] bf16, by collective parity
+  const size_t rs_max = (Tm + size_t(tp) - 1) / size_t(tp);
+  w.recv[0] = tp > 1 ? take(size_t(tp) * rs_max * d * 2) : 0;
+  w.recv[1] = tp > 1 ? take(size_t(tp) * rs_max * d * 2) : 0;
   w.part[0] = tp > 1 ? take(Tm * d * 2) : 0;
   w.part[1] = tp > 1 ? take(Tm * d * 2) : 0;
   w.argmax = take(Rm * 4);
@@ -387,6 +391,7 @@ struct qos_engine {
   std::vector<uint8_t*> ipc_base;               //   (their IPC mapping bases, for closing)
   std::vector<std::array<cudaEvent_t, 2>> ipc_ev;  //   and their opened sync events
   int tp_twoshot = -1;              // option tp_twoshot: 0 one-shot, 1 two-shot, -1 auto (tp >= 4)
+  bool tp_scatter = true;           // option tp_scatter: two-shot with the reduce-scatter in the GEMM epilogue
   int64_t last_h2d = 0, last_d2h = 0;  // bytes moved host<->device by the last step
   // debug buffers for ops
   void* dbg = nullptr;
@@ -818,7 +823,26 @@ PeerPtrs peer_ptrs(qos_engine* e, size_t ws_off) {
 
 // a10 + a3: sum the ranks' partials into the fp32 residual, then RMSNorm with gain g into h
 // (g == nullptr after the last layer: add only).
-int tp_reduce_add_norm(qos_engine* e, const void* g, int T, cudaStream_t st) {
+bool tp_two_shot(const qos_engine* e) { return e->tp_twoshot > 0 || (e->tp_twoshot < 0 && e->tp_size >= 4); }
+
+// Peer-group two-shot with the reduce-scatter fused into the producing GEMM's epilogue: each
+// partial row is stored straight into its owner rank's receive slot for this rank (peer
+// memory), tile by tile while the remaining tiles compute.  Needs the one-pass tile kernels.
+bool tp_scatter_on(const qos_engine* e, int64_t T, int64_t N, int64_t K) {
+  return e->group && e->tp_scatter && tp_two_shot(e) && gemm_one_pass(e, T, N, K, e->num_sms);
+}
+NormFold tp_scatter_args(qos_engine* e, int T) {
+  NormFold f;
+  const int rs = (T + e->tp_size - 1) / e->tp_size;
+  const size_t rs_max = (size_t(e->cfg.max_batch_tokens) + e->tp_size - 1) / e->tp_size;
+  const size_t d = size_t(e->cfg.d_model);
+  for (int k = 0; k < e->tp_size; ++k)  // owner k's slot for this rank
+    f.scat[k] = peer_ws(e, k) + e->wsl.recv[e->red_seq & 1] + size_t(e->tp_rank) * rs_max * d * 2;
+  f.scat_rs = rs;
+  return f;
+}
+
+int tp_reduce_add_norm(qos_engine* e, const void* g, int T, cudaStream_t st, bool scattered = false) {
   const int d = e->cfg.d_model;
   float* resid = reinterpret_cast<float*>(e->ws + e->wsl.resid);
   __nv_bfloat16* h = reinterpret_cast<__nv_bfloat16*>(e->ws + e->wsl.h);
@@ -833,15 +857,21 @@ int tp_reduce_add_norm(qos_engine* e, const void* g, int T, cudaStream_t st) {
     return QOS_OK;
   }
   TimerScope ts(e, QOS_T_ALLREDUCE, st);
-  const PeerPtrs parts = peer_ptrs(e, e->wsl.part[e->red_seq++ & 1]);
-  QOS_TRY(peer_sync(e, st));  // every rank's partial is complete
-  const bool two = e->tp_twoshot > 0 || (e->tp_twoshot < 0 && e->tp_size >= 4);
+  const int par = int(e->red_seq++ & 1);
+  PeerPtrs parts = peer_ptrs(e, e->wsl.part[par]);
+  const int rs = (T + e->tp_size - 1) / e->tp_size, row0 = std::min(T, e->tp_rank * rs);
+  if (scattered) {  // the peers' partial rows of this rank's slice are already in its receive slots
+    const size_t rs_max = (size_t(e->cfg.max_batch_tokens) + e->tp_size - 1) / e->tp_size;
+    for (int k = 0; k < e->tp_size; ++k)  // slot k, shifted so that row t indexes its local row t - row0
+      parts.p[k] = e->ws + e->wsl.recv[par] + (size_t(k) * rs_max * d - size_t(row0) * d) * 2;
+  }
+  QOS_TRY(peer_sync(e, st));  // every rank's partial is complete (scattered: landed in the owners' slots)
+  const bool two = tp_two_shot(e);
   if (!two) {
     QOS_CU(launch_peer_add_rmsnorm(parts, e->tp_size, resid, g, h, T, d, e->cfg.rms_eps, st));
     return QOS_OK;
   }
   // two-shot: this rank reduces + normalises its row slice and stores the rows into every peer
-  const int rs = (T + e->tp_size - 1) / e->tp_size, row0 = std::min(T, e->tp_rank * rs);
   QOS_CU(launch_peer_rs_norm_ag(parts, peer_ptrs(e, e->wsl.h), peer_ptrs(e, e->wsl.resid), e->tp_size, e->tp_rank,
                                 row0, std::min(rs, T - row0), g, d, e->cfg.rms_eps, st));
   QOS_TRY(peer_sync(e, st));  // every rank's rows have landed in every h (or residual)
@@ -1008,11 +1038,14 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
         QOS_TRY(gemm_seg(e, g, e->a_attn, M.o, d, e->sh.H * hd, EPI_ADD_F32, resid, d, nullptr, nullptr,
                          fold ? &f_o : nullptr));
       } else {
+        const bool sc = tp_scatter_on(e, T, d, e->sh.H * hd);
+        const NormFold fs = sc ? tp_scatter_args(e, T) : NormFold{};
         {
           TimerScope ts(e, QOS_T_GEMM_O, gs);
-          QOS_TRY(gemm_seg(e, g, e->a_attn, M.o, d, e->sh.H * hd, EPI_STORE_BF16, tp_partial_dst(e), d, nullptr));
+          QOS_TRY(gemm_seg(e, g, e->a_attn, M.o, d, e->sh.H * hd, EPI_STORE_BF16, tp_partial_dst(e), d, nullptr,
+                           nullptr, sc ? &fs : nullptr));
         }
-        QOS_TRY(tp_reduce_add_norm(e, W(e, L.ln2), T, gs));
+        QOS_TRY(tp_reduce_add_norm(e, W(e, L.ln2), T, gs, sc));
       }
       if (!tp && !fold) {
         TimerScope ts(e, QOS_T_NORM, gs);
@@ -1028,11 +1061,14 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
         QOS_TRY(gemm_seg(e, g, e->a_act, M.d, d, e->sh.F, EPI_ADD_F32, resid, d, nullptr, nullptr,
                          fold_down ? &f_down : nullptr));
       } else {
+        const bool sc = tp_scatter_on(e, T, d, e->sh.F);
+        const NormFold fs = sc ? tp_scatter_args(e, T) : NormFold{};
         {
           TimerScope ts(e, QOS_T_GEMM_DOWN, gs);
-          QOS_TRY(gemm_seg(e, g, e->a_act, M.d, d, e->sh.F, EPI_STORE_BF16, tp_partial_dst(e), d, nullptr));
+          QOS_TRY(gemm_seg(e, g, e->a_act, M.d, d, e->sh.F, EPI_STORE_BF16, tp_partial_dst(e), d, nullptr, nullptr,
+                           sc ? &fs : nullptr));
         }
-        QOS_TRY(tp_reduce_add_norm(e, l + 1 < c.n_layers ? W(e, e->wl.layers[l + 1].ln1) : nullptr, T, gs));
+        QOS_TRY(tp_reduce_add_norm(e, l + 1 < c.n_layers ? W(e, e->wl.layers[l + 1].ln1) : nullptr, T, gs, sc));
       }
     }
   }
@@ -1807,6 +1843,7 @@ int qos_engine_set_option(qos_engine_t* e, const char* name, int64_t value) {
   else if (n == "gemm_2cta") e->gemm_2cta = value != 0;
   else if (n == "fa_persist") e->fa_persist = value != 0;
   else if (n == "norm_fold") e->norm_fold = value != 0;
+  else if (n == "tp_scatter") e->tp_scatter = value != 0;
   else if (n == "tp_twoshot") e->tp_twoshot = value < 0 ? -1 : value > 0 ? 1 : 0;
   else if (n == "decode_stages") {
     if (value != 4 && value != 8) return set_error(QOS_ERR_INVALID_ARG, "decode_stages must be 4 or 8");

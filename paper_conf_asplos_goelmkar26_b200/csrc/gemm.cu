@@ -82,6 +82,8 @@ struct GemmArgs {
   __nv_bfloat16* h_out;
   int ss_n;
   float inv_d, rms_eps;
+  void* scat[8];  // reduce-scatter destinations (NormFold::scat), scat_rs = 0: plain store to C
+  int scat_rs;
 };
 
 static void set_fold(GemmArgs& a, const NormFold* f) {
@@ -94,6 +96,8 @@ static void set_fold(GemmArgs& a, const NormFold* f) {
   a.ss_n = f ? f->ss_n : 0;
   a.inv_d = f && f->d ? 1.f / float(f->d) : 0.f;
   a.rms_eps = f ? f->eps : 0.f;
+  for (int k = 0; k < 8; ++k) a.scat[k] = f ? f->scat[k] : nullptr;
+  a.scat_rs = f ? f->scat_rs : 0;
 }
 
 // ---- epilogue stores of one thread's 32 consecutive accumulator columns of one row
@@ -530,8 +534,15 @@ QOS_DEV void epi_tile_staged(const GemmArgs& p, uint8_t* stg, int lane, int n_t,
 #pragma unroll
               for (int k = 0; k < 4; ++k) stg_put<64>(stg, lane, k, make_uint4(pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]));
               stg_flush<64>(stg, lane, [&](int rr, int k, uint4 x) {
-                if (row0 + rr < p.M)
-                  reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.C) + size_t(row0 + rr) * p.ldc + col)[k] = x;
+                const int r = row0 + rr;
+                if (r >= p.M) return;
+                if (p.scat_rs) {  // TP reduce-scatter: the row's owner rank, over peer memory
+                  const int own = r / p.scat_rs;
+                  reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.scat[own]) +
+                                           size_t(r - own * p.scat_rs) * p.ldc + col)[k] = x;
+                } else {
+                  reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.C) + size_t(r) * p.ldc + col)[k] = x;
+                }
               });
             } else {
 #pragma unroll

@@ -61,6 +61,11 @@ struct NormFold {
   void* h_out = nullptr;        // bf16 [M][d]
   int ss_n = 0, d = 0;
   float eps = 0.f;
+  // TP peer group, reduce-scatter in the epilogue (EPI_STORE_BF16): row r of the partial goes to
+  // its owner rank o = r / scat_rs, at scat[o] + (r - o * scat_rs) * ldc (this rank's slot of the
+  // owner's receive buffer; peer memory) — the transfer overlaps the remaining tiles' MMAs
+  void* scat[8] = {};
+  int scat_rs = 0;
 };
 int gemm_run(const CUtensorMap& ta, const CUtensorMap& tb, int bn, int64_t M, int64_t N, int64_t K, int epi, void* C,
              int64_t ldc, const float* bias, int num_sms, cudaStream_t st, int ksplit = 1, float* part = nullptr,

@@ -55,14 +55,18 @@ def _all(q, engs, fn):
     return q.run_ranks(fn, engs)
 
 
-@pytest.mark.parametrize("preset,tp,ffn,twoshot", [("tiny", 2, None, -1), ("tiny", 2, None, 1),
-                                                   ("tiny-qwen", 2, None, -1), ("tiny-mha", 2, None, -1),
-                                                   ("tiny-mha", 4, 1024, -1), ("tiny-mha", 4, 1024, 0)])
-def test_tp_peer_group_tiny_scenario(preset, tp, ffn, twoshot):
-    # (tp 4 needs F/tp % 128 == 0: F = 1024 instead of 768); twoshot: one-shot / two-shot reduction
+@pytest.mark.parametrize("preset,tp,ffn,twoshot,swab", [("tiny", 2, None, -1, 1), ("tiny", 2, None, 1, 1),
+                                                         ("tiny", 2, None, 1, 0), ("tiny-qwen", 2, None, -1, 1),
+                                                         ("tiny-mha", 2, None, -1, 1), ("tiny-mha", 4, 1024, -1, 1),
+                                                         ("tiny-mha", 4, 1024, 0, 1), ("tiny-mha", 4, 1024, -1, 0)])
+def test_tp_peer_group_tiny_scenario(preset, tp, ffn, twoshot, swab):
+    # (tp 4 needs F/tp % 128 == 0: F = 1024 instead of 768); twoshot: one-shot / two-shot
+    # reduction; swab = 0 puts the O / down projections on the one-pass tile kernels, whose
+    # epilogue then stores each partial row straight into its owner's receive slot (tp_scatter)
     q, cfg, g, engs = _group_engines(preset, tp, **({"ffn_dim": ffn} if ffn else {}))
     for e in engs:
         e.qos_engine_set_option("tp_twoshot", twoshot)
+        e.qos_engine_set_option("gemm_swab", swab)
     _all(q, engs, lambda r, e: e.qos_engine_load_synthetic(0))
     orc = _oracle(preset, ffn_dim=ffn, num_blocks=256)
     ctxs, warm, main, second = synth.tiny_scenario(cfg.vocab)
