@@ -225,7 +225,7 @@ def test_llama70b_shapes_tp8_hybrid_step_sampled_parity():
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-def _ipc_worker(rank, tp, gid, preset_name, ffn, twoshot, out_q):
+def _ipc_worker(rank, tp, gid, preset_name, ffn, twoshot, out_q, swab=1):
     import sys
     sys.path.insert(0, ROOT)
     sys.path.insert(0, os.path.join(ROOT, "tests"))
@@ -241,6 +241,7 @@ def _ipc_worker(rank, tp, gid, preset_name, ffn, twoshot, out_q):
         g = q.Group(tp, gid, rank)
         e = q.Engine(cfg, 0, rank, tp, group=g)
         e.qos_engine_set_option("tp_twoshot", twoshot)
+        e.qos_engine_set_option("gemm_swab", swab)
         e.qos_engine_load_synthetic(0)
         ctxs, warm, main, second = sy.tiny_scenario(cfg.vocab)
         for r, n in ctxs.items():
@@ -255,8 +256,9 @@ def _ipc_worker(rank, tp, gid, preset_name, ffn, twoshot, out_q):
         out_q.put((rank, None, None, repr(ex)))
 
 
-@pytest.mark.parametrize("preset,tp,ffn,twoshot", [("tiny", 2, None, 0), ("tiny-mha", 4, 1024, 1)])
-def test_tp_cross_process_group_tiny_scenario(preset, tp, ffn, twoshot):
+@pytest.mark.parametrize("preset,tp,ffn,twoshot,swab", [("tiny", 2, None, 0, 1), ("tiny-mha", 4, 1024, 1, 1),
+                                                         ("tiny-mha", 4, 1024, 1, 0)])
+def test_tp_cross_process_group_tiny_scenario(preset, tp, ffn, twoshot, swab):
     """One process per rank (the torchrun layout), all on cuda:0: the group is opened from a
     shared-memory id, workspaces and sync events are exchanged as CUDA IPC handles, and the
     collectives read / store peer memory of other processes.  Results vs the unsharded oracle;
@@ -267,7 +269,7 @@ def test_tp_cross_process_group_tiny_scenario(preset, tp, ffn, twoshot):
     ctx = mp.get_context("spawn")
     out_q = ctx.Queue()
     gid = q.qos_group_unique_id()
-    procs = [ctx.Process(target=_ipc_worker, args=(r, tp, gid, preset, ffn, twoshot, out_q)) for r in range(tp)]
+    procs = [ctx.Process(target=_ipc_worker, args=(r, tp, gid, preset, ffn, twoshot, out_q, swab)) for r in range(tp)]
     for p in procs:
         p.start()
     res = {}
