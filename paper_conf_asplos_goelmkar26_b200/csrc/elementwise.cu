@@ -268,45 +268,73 @@ __global__ void unshard_logits_kernel(const float* __restrict__ in, float* __res
 }
 
 // argmax per row; ties -> lowest index.  logits f32 or bf16 [R][V].
-__global__ void argmax_kernel(const void* __restrict__ logits, int is_f32, int V, int32_t* __restrict__ out) {
+// argmax per row; ties -> lowest index.  logits f32 or bf16 [R][V].  Grid (R, S): CTA (r, s)
+// scans the s-th of S contiguous slices of row r (16-byte loads on the f32 path), parks its
+// (value, index) in part[r][s]; the last of the row's S CTAs to arrive merges the slices in
+// slice order (arrival counter, reset for the next launch).  S = 1 writes out directly.
+QOS_DEV void amax_merge(float& best, int& bi, float v, int i) {
+  if (v > best || (v == best && i < bi)) {
+    best = v;
+    bi = i;
+  }
+}
+__global__ void argmax_kernel(const void* __restrict__ logits, int is_f32, int V, int32_t* __restrict__ out,
+                              float2* __restrict__ part, int* __restrict__ cnt) {
   griddep_wait();
   griddep_launch_dependents();
-  const int r = blockIdx.x;
+  const int r = blockIdx.x, S = gridDim.y, sl = blockIdx.y;
+  const int per = ((V + S - 1) / S + 3) & ~3;  // slice length, a multiple of 4
+  const int i0 = sl * per, i1 = min(V, i0 + per);
   float best = -INFINITY;
   int bi = 0x7fffffff;
-  for (int i = threadIdx.x; i < V; i += blockDim.x) {
-    const float v = is_f32 ? reinterpret_cast<const float*>(logits)[size_t(r) * V + i]
-                           : __bfloat162float(reinterpret_cast<const __nv_bfloat16*>(logits)[size_t(r) * V + i]);
-    if (v > best || (v == best && i < bi)) {
-      best = v;
-      bi = i;
+  if (is_f32 && (V & 3) == 0) {
+    const float4* row = reinterpret_cast<const float4*>(reinterpret_cast<const float*>(logits) + size_t(r) * V);
+    for (int q = (i0 >> 2) + threadIdx.x; q < (i1 >> 2); q += blockDim.x) {  // this thread's indices increase
+      const float4 x = __ldcs(row + q);
+      const int i = q << 2;
+      if (x.x > best) { best = x.x; bi = i; }
+      if (x.y > best) { best = x.y; bi = i + 1; }
+      if (x.z > best) { best = x.z; bi = i + 2; }
+      if (x.w > best) { best = x.w; bi = i + 3; }
+    }
+  } else {
+    for (int i = i0 + threadIdx.x; i < i1; i += blockDim.x) {
+      const float v = is_f32 ? reinterpret_cast<const float*>(logits)[size_t(r) * V + i]
+                             : __bfloat162float(reinterpret_cast<const __nv_bfloat16*>(logits)[size_t(r) * V + i]);
+      if (v > best) { best = v; bi = i; }
     }
   }
 #pragma unroll
-  for (int o = 16; o > 0; o >>= 1) {
-    const float ov = __shfl_xor_sync(0xffffffffu, best, o);
-    const int oi = __shfl_xor_sync(0xffffffffu, bi, o);
-    if (ov > best || (ov == best && oi < bi)) {
-      best = ov;
-      bi = oi;
-    }
-  }
+  for (int o = 16; o > 0; o >>= 1)
+    amax_merge(best, bi, __shfl_xor_sync(0xffffffffu, best, o), __shfl_xor_sync(0xffffffffu, bi, o));
   __shared__ float sv[32];
   __shared__ int si[32];
+  __shared__ int s_last;
   const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
   if (l == 0) {
     sv[w] = best;
     si[w] = bi;
   }
   __syncthreads();
-  if (threadIdx.x == 0) {
-    for (int k = 1; k < (int)(blockDim.x >> 5); ++k)
-      if (sv[k] > best || (sv[k] == best && si[k] < bi)) {
-        best = sv[k];
-        bi = si[k];
-      }
+  if (threadIdx.x != 0) return;
+  for (int k = 1; k < (int)(blockDim.x >> 5); ++k) amax_merge(best, bi, sv[k], si[k]);
+  if (S == 1) {
     out[r] = bi;
+    return;
   }
+  part[size_t(r) * S + sl] = make_float2(best, __int_as_float(bi));
+  __threadfence();
+  s_last = atomicAdd(cnt + r, 1) == S - 1;
+  if (!s_last) return;
+  __threadfence();
+  float b2 = -INFINITY;
+  int i2 = 0x7fffffff;
+  for (int k = 0; k < S; ++k) {
+    const float2 pk = __ldcg(part + size_t(r) * S + k);
+    amax_merge(b2, i2, pk.x, __float_as_int(pk.y));
+  }
+  out[r] = i2;
+  cnt[r] = 0;
 }
 
 __global__ void f32_to_bf16_kernel(const float* __restrict__ x, __nv_bfloat16* __restrict__ y, int64_t n) {
@@ -421,10 +449,13 @@ cudaError_t launch_unshard_logits(const float* in, float* out, int R, int Vl, in
   count_launch();
   return launch_pdl(unshard_logits_kernel, dim3(grid_of(int64_t(R) * Vl * tp)), dim3(256), 0, st, in, out, R, Vl, tp);
 }
-cudaError_t launch_argmax(const void* logits, int logits_f32, int R, int V, int32_t* out, cudaStream_t st) {
+cudaError_t launch_argmax(const void* logits, int logits_f32, int R, int V, int32_t* out, cudaStream_t st,
+                          float2* part, int* cnt) {
   if (R == 0) return cudaSuccess;
   count_launch();
-  return launch_pdl(argmax_kernel, dim3(R), dim3(1024), 0, st, logits, logits_f32, V, out);
+  // slices per row: fill about two CTAs per SM (R = 129 logit rows -> 3 slices of ~43k entries)
+  int S = part && cnt ? std::max(1, std::min(kArgmaxMaxSlices, (2 * 148 + R - 1) / R)) : 1;
+  return launch_pdl(argmax_kernel, dim3(R, S), dim3(512), 0, st, logits, logits_f32, V, out, part, cnt);
 }
 cudaError_t launch_f32_to_bf16(const float* x, void* y, int64_t n, cudaStream_t st) {
   if (n == 0) return cudaSuccess;

@@ -151,7 +151,7 @@ static WeightLayout weight_layout(const qos_model_cfg& c, const Shard& s) {
 }
 
 struct WsLayout {
-  size_t resid, h, qkv, attn, act, hR, logits, logits_loc, part[2], recv[2], ss[2], rs[2], fcnt, argmax, partials, counters, gemm_part, gemm_cnt, gemm_part2,
+  size_t resid, h, qkv, attn, act, hR, logits, logits_loc, part[2], recv[2], ss[2], rs[2], fcnt, am_part, am_cnt, argmax, partials, counters, gemm_part, gemm_cnt, gemm_part2,
       gemm_cnt2, meta[2], dbg, total;
   size_t meta_bytes;
   int max_items;
@@ -191,6 +191,8 @@ static WsLayout ws_layout(const qos_model_cfg& c, const Shard& s, int tp) {
   w.part[0] = tp > 1 ? take(Tm * d * 2) : 0;
   w.part[1] = tp > 1 ? take(Tm * d * 2) : 0;
   w.argmax = take(Rm * 4);
+  w.am_part = take(Rm * kArgmaxMaxSlices * 8);
+  w.am_cnt = take(Rm * 4);
   w.max_items = kMaxDecodeItems;
   w.partials = take(size_t(w.max_items) * group * (hd + 2) * 4);
   w.counters = take(Rm * size_t(s.Hkv) * 4);
@@ -1108,7 +1110,8 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
   {
     TimerScope ts(e, QOS_T_ARGMAX, st);
     int32_t* am = reinterpret_cast<int32_t*>(e->ws + s.argmax);
-    QOS_CU(launch_argmax(lout, 1, R, c.vocab, am, st));
+    QOS_CU(launch_argmax(lout, 1, R, c.vocab, am, st, reinterpret_cast<float2*>(e->ws + s.am_part),
+                         reinterpret_cast<int*>(e->ws + s.am_cnt)));
     if (next_tokens) {
       QOS_CU(cudaMemcpyAsync(next_tokens, am, size_t(R) * 4, out_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost,
                              st));
@@ -1419,7 +1422,8 @@ static int create_engine(const qos_model_cfg* cfg, int device, int tp_rank, int 
       cudaMemset(e->ws + e->wsl.gemm_cnt2, 0, size_t(kGemmMaxTiles) * 4) != cudaSuccess ||
       cudaMemset(e->ws + e->wsl.ss[0], 0, size_t(cfg->max_batch_tokens) * kFoldSlots * 4) != cudaSuccess ||
       cudaMemset(e->ws + e->wsl.ss[1], 0, size_t(cfg->max_batch_tokens) * kFoldSlots * 4) != cudaSuccess ||
-      cudaMemset(e->ws + e->wsl.fcnt, 0, size_t(cfg->max_batch_tokens / 128 + 2) * 4) != cudaSuccess)
+      cudaMemset(e->ws + e->wsl.fcnt, 0, size_t(cfg->max_batch_tokens / 128 + 2) * 4) != cudaSuccess ||
+      cudaMemset(e->ws + e->wsl.am_cnt, 0, size_t(cfg->max_batch_rows) * 4) != cudaSuccess)
     return fail(set_error(QOS_ERR_CUDA, "counter memset"));
   if (cudaMalloc(&e->d_tables, size_t(cfg->max_requests) * e->table_w * 4) != cudaSuccess)
     return fail(set_error(QOS_ERR_OOM, "block tables"));

@@ -142,7 +142,10 @@ cudaError_t launch_peer_rs_norm_ag(const PeerPtrs& parts, const PeerPtrs& hs, co
                                    int row0, int nrows, const void* g, int d, float eps, cudaStream_t st);
 // out[R][tp*Vl] <- rank k's [R][Vl] slice
 cudaError_t launch_peer_gather_logits(const PeerPtrs& loc, int tp, int R, int Vl, float* out, cudaStream_t st);
-cudaError_t launch_argmax(const void* logits, int logits_f32, int R, int V, int32_t* out, cudaStream_t st);
+constexpr int kArgmaxMaxSlices = 8;
+// part: [R][kArgmaxMaxSlices] scratch, cnt: [R] zero-initialised counters (NULL: one CTA per row)
+cudaError_t launch_argmax(const void* logits, int logits_f32, int R, int V, int32_t* out, cudaStream_t st,
+                          float2* part = nullptr, int* cnt = nullptr);
 cudaError_t launch_f32_to_bf16(const float* x, void* y, int64_t n, cudaStream_t st);
 
 // ------------------------------------------------------------------ attention (attention.cu)
