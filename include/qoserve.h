@@ -262,6 +262,9 @@ int qos_profile_step_ex(qos_engine_t* eng, int32_t chunk_len, int32_t kv_start,
  *                          all rows), 1 two-shot (each rank reduces + normalises a row slice and
  *                          stores it into every peer: ~2(tp-1)/tp of one partial per rank instead
  *                          of tp-1), -1 automatic (two-shot when tp >= 4)
+ *   "attn_order" (0)       with overlap_attn: 0 prefill attention first on a high-priority side
+ *                          stream; 1 decode first, prefill on a normal-priority side stream; 2
+ *                          decode first, prefill high priority (measured equal within noise)
  *   "tp_scatter" (1)       peer-group two-shot reduction with the reduce-scatter fused into the O /
  *                          down GEMM epilogue: each partial row is stored straight into its owner
  *                          rank's receive slot (peer memory) while the remaining tiles compute

@@ -360,6 +360,9 @@ struct qos_engine {
   int meta_cur = 0;
   cudaStream_t stream = nullptr;  // internal stream for synchronous calls
   cudaStream_t side = nullptr;    // high-priority stream: prefill attention overlapped with decode
+  cudaStream_t side_lo = nullptr; // normal-priority side stream (option attn_order = 1)
+  int attn_order = 0;             // option attn_order: 0 prefill first on `side`; 1 decode first, prefill
+                                  // on `side_lo`; 2 decode first, prefill on `side`
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr, ev_fork2 = nullptr, ev_join2 = nullptr;
   bool dual_stream = false;       // QOS_DUAL=1: prefill rows and decode rows on two streams
   int dual_min_prefill = 512, dual_min_decode = 16;
@@ -1016,23 +1019,38 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
       // a7 || a8: within one segment, the prefill tiles go to the high-priority side stream and
       // the decode split-K items stay on the segment's stream (disjoint rows of `attn`)
       const bool overlap = !dual && e->overlap_attn && g.pre && g.dec;
-      cudaStream_t pst = overlap ? e->side : gs;
+      cudaStream_t side = e->attn_order == 1 ? e->side_lo : e->side;
+      cudaStream_t pst = overlap ? side : gs;
       if (overlap) {
         QOS_CU(cudaEventRecord(e->ev_fork2, gs));
-        QOS_CU(cudaStreamWaitEvent(e->side, e->ev_fork2, 0));
+        QOS_CU(cudaStreamWaitEvent(side, e->ev_fork2, 0));
       }
-      if (g.pre && m.n_pitems) {
-        TimerScope ts(e, QOS_T_PREFILL_ATTN, pst);
-        QOS_CU(launch_prefill_attention_tc(al, reinterpret_cast<const PrefillItem*>(dm + m.o_pitems), m.n_pitems, pst));
-      }
-      if (g.dec && m.n_ditems) {
-        TimerScope ts(e, QOS_T_DECODE_ATTN, gs);
-        QOS_CU(launch_decode_attention(al, reinterpret_cast<const DecodeItem*>(dm + m.o_ditems), m.n_ditems,
-                                       reinterpret_cast<float*>(e->ws + s.partials),
-                                       reinterpret_cast<int*>(e->ws + s.counters), gs));
+      auto prefill = [&]() -> int {
+        if (g.pre && m.n_pitems) {
+          TimerScope ts(e, QOS_T_PREFILL_ATTN, pst);
+          QOS_CU(launch_prefill_attention_tc(al, reinterpret_cast<const PrefillItem*>(dm + m.o_pitems), m.n_pitems,
+                                             pst));
+        }
+        return QOS_OK;
+      };
+      auto decode = [&]() -> int {
+        if (g.dec && m.n_ditems) {
+          TimerScope ts(e, QOS_T_DECODE_ATTN, gs);
+          QOS_CU(launch_decode_attention(al, reinterpret_cast<const DecodeItem*>(dm + m.o_ditems), m.n_ditems,
+                                         reinterpret_cast<float*>(e->ws + s.partials),
+                                         reinterpret_cast<int*>(e->ws + s.counters), gs));
+        }
+        return QOS_OK;
+      };
+      if (e->attn_order == 0) {
+        QOS_TRY(prefill());
+        QOS_TRY(decode());
+      } else {
+        QOS_TRY(decode());
+        QOS_TRY(prefill());
       }
       if (overlap) {
-        QOS_CU(cudaEventRecord(e->ev_join2, e->side));
+        QOS_CU(cudaEventRecord(e->ev_join2, side));
         QOS_CU(cudaStreamWaitEvent(gs, e->ev_join2, 0));
       }
       if (!tp) {
@@ -1460,6 +1478,7 @@ static int create_engine(const qos_model_cfg* cfg, int device, int tp_rank, int 
     int lo = 0, hi = 0;
     cudaDeviceGetStreamPriorityRange(&lo, &hi);
     cudaStreamCreateWithPriority(&e->side, cudaStreamNonBlocking, hi);
+    cudaStreamCreateWithPriority(&e->side_lo, cudaStreamNonBlocking, lo);
     cudaEventCreateWithFlags(&e->ev_fork, cudaEventDisableTiming);
     cudaEventCreateWithFlags(&e->ev_join, cudaEventDisableTiming);
     cudaEventCreateWithFlags(&e->ev_fork2, cudaEventDisableTiming);
@@ -1553,6 +1572,7 @@ int qos_engine_destroy(qos_engine_t* e) {
   for (auto ev : e->ev_pool) cudaEventDestroy(ev);
   if (e->stream) cudaStreamDestroy(e->stream);
   if (e->side) cudaStreamDestroy(e->side);
+  if (e->side_lo) cudaStreamDestroy(e->side_lo);
   if (e->ev_fork) cudaEventDestroy(e->ev_fork);
   if (e->ev_join) cudaEventDestroy(e->ev_join);
   if (e->ev_fork2) cudaEventDestroy(e->ev_fork2);
@@ -1848,6 +1868,10 @@ int qos_engine_set_option(qos_engine_t* e, const char* name, int64_t value) {
   else if (n == "fa_persist") e->fa_persist = value != 0;
   else if (n == "norm_fold") e->norm_fold = value != 0;
   else if (n == "tp_scatter") e->tp_scatter = value != 0;
+  else if (n == "attn_order") {
+    if (value < 0 || value > 2) return set_error(QOS_ERR_INVALID_ARG, "attn_order must be 0, 1 or 2");
+    e->attn_order = int(value);
+  }
   else if (n == "tp_twoshot") e->tp_twoshot = value < 0 ? -1 : value > 0 ? 1 : 0;
   else if (n == "decode_stages") {
     if (value != 4 && value != 8) return set_error(QOS_ERR_INVALID_ARG, "decode_stages must be 4 or 8");
