@@ -451,8 +451,9 @@ __global__ void __launch_bounds__(FaCfg<HD, NQ>::kThreads, FaCfg<HD, NQ>::kMinBl
 // per item on average) the per-CTA prologue/epilogue was a third of the launch.
 template <int HD, int POLY>
 __global__ void __launch_bounds__(FaCfg<HD, 1>::kThreads, 2)
-    prefill_attn_persist_kernel(const __grid_constant__ CUtensorMap kvmap, const FaParams p,
-                                const PrefillItem* __restrict__ items, const int32_t* __restrict__ cta_off) {
+    prefill_attn_persist_kernel(const __grid_constant__ CUtensorMap kvmap, const __grid_constant__ CUtensorMap qmap,
+                                const FaParams p, const PrefillItem* __restrict__ items,
+                                const int32_t* __restrict__ cta_off) {
   using C = FaCfg<HD, 1>;
   constexpr int S = C::kStages;
   extern __shared__ uint8_t smem_raw[];
@@ -469,8 +470,9 @@ __global__ void __launch_bounds__(FaCfg<HD, 1>::kThreads, 2)
   uint64_t* p_full = s_full + 2;    // [2]
   uint64_t* o_full = p_full + 2;    // completes once per P.V
   uint64_t* o_final = o_full + 1;   // completes once per item
-  uint64_t* q_full = o_final + 1;   // completes once per item (Q staged by the softmax warps)
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(q_full + 1);
+  uint64_t* q_full = o_final + 1;   // completes once per item (Q tile landed, TMA)
+  uint64_t* q_empty = q_full + 1;   // completes once per item (its last QK done: sQ free)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(q_empty + 1);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int i_begin = cta_off[blockIdx.x], i_end = cta_off[blockIdx.x + 1];
@@ -490,7 +492,8 @@ __global__ void __launch_bounds__(FaCfg<HD, 1>::kThreads, 2)
     }
     mbar_init(o_full, 1);
     mbar_init(o_final, 1);
-    mbar_init(q_full, 128);
+    mbar_init(q_full, 1);
+    mbar_init(q_empty, 1);
     fence_mbar_init();
   }
   if (warp == 1) tmem_alloc<C::kTmemCols>(tmem_slot);
@@ -505,10 +508,18 @@ __global__ void __launch_bounds__(FaCfg<HD, 1>::kThreads, 2)
     // ------------------------------------------------------------------ TMA producer
     if (elect_one()) {
       tma_prefetch_desc(&kvmap);
+      tma_prefetch_desc(&qmap);
       uint32_t jg = 0;
-      for (int ii = i_begin; ii < i_end; ++ii) {
+      for (int ii = i_begin, n = 0; ii < i_end; ++ii, ++n) {
         const PrefillItem it = items[ii];
         const int nt = it.grp_last / C::kKeys + 1, last_blk = it.grp_last >> 4;
+        // Q tile of the item: rows (position, head-in-group) = a {64 dims, group heads, ppt rows}
+        // box per 64-dim half; issued as soon as the previous item's last QK has read sQ
+        if (n > 0) mbar_wait(q_empty, uint32_t(n - 1) & 1);
+        mbar_arrive_expect_tx(q_full, C::kQBytes);
+#pragma unroll
+        for (int hf = 0; hf < C::kHalves; ++hf)
+          tma_load_3d(sQ + hf * (C::kRows * 128), &qmap, q_full, hf * 64, it.kv_head * group, it.row0);
         const int32_t* trow = p.tables + size_t(it.table) * p.table_w;
         auto load_tile = [&](uint8_t* dst, uint64_t* full, int j, int plane) {
           for (int b = 0; b < C::kKeys / 16; ++b) {
@@ -576,6 +587,7 @@ __global__ void __launch_bounds__(FaCfg<HD, 1>::kThreads, 2)
           umma_commit(&k_empty[s]);
           if (j >= 1) issue_pv(tg - 1, j == 1);   // O += P(j-1) V(j-1) while the softmax works on S(j)
         }
+        umma_commit(q_empty);  // every QK of this item has been issued: sQ is free once they complete
         issue_pv(jg + uint32_t(nt) - 1, nt == 1);
         umma_commit(o_final);
         jg += uint32_t(nt);
@@ -587,21 +599,6 @@ __global__ void __launch_bounds__(FaCfg<HD, 1>::kThreads, 2)
     const uint32_t lane_base = tmem + (uint32_t((warp & 3) * 32) << 16);
     const uint32_t o_addr = lane_base + C::col_o(0);
     const int pi = row / group, hh = row % group;
-    auto stage_q = [&](const PrefillItem& it) {
-      const bool ok = row < ppt * group && pi < it.npos;
-      const __nv_bfloat16* src = p.q + size_t(it.row0 + pi) * p.q_ld + size_t(it.kv_head * group + hh) * HD;
-      uint4 v[HD / 8];
-#pragma unroll
-      for (int ch = 0; ch < HD / 8; ++ch) v[ch] = ok ? *reinterpret_cast<const uint4*>(src + ch * 8) : make_uint4(0, 0, 0, 0);
-#pragma unroll
-      for (int ch = 0; ch < HD / 8; ++ch) {
-        const int hf = ch >> 3, c = ch & 7;
-        *reinterpret_cast<uint4*>(sQ + hf * (C::kRows * 128) + row * 128 + ((c ^ (row & 7)) << 4)) = v[ch];
-      }
-      fence_proxy_async_smem();
-      mbar_arrive(q_full);
-    };
-    if (i_begin < i_end) stage_q(items[i_begin]);
     uint32_t jg = 0;
     for (int ii = i_begin, n = 0; ii < i_end; ++ii, ++n) {
       const PrefillItem it = items[ii];
@@ -680,9 +677,6 @@ __global__ void __launch_bounds__(FaCfg<HD, 1>::kThreads, 2)
         tc_fence_before();
         mbar_arrive(&p_full[sb]);
       }
-      // every QK of this item has completed (its S was awaited): stage the next item's Q now so
-      // the MMA warp starts it under this epilogue
-      if (ii + 1 < i_end) stage_q(items[ii + 1]);
       mbar_wait(o_final, uint32_t(n) & 1);
       tc_fence_after();
       const float inv = (l > 0.f) ? 1.f / l : 0.f;
@@ -1078,6 +1072,15 @@ template <int HD, int POLY>
 static cudaError_t prefill_persist_t(const AttnLaunch& a, const PrefillItem* items, const int32_t* cta_off, int n_cta,
                                      cudaStream_t st) {
   using C = FaCfg<HD, 1>;
+  const int group = a.H / a.Hkv;
+  CUtensorMap qm;
+  const CUtensorMap* qmp = a.q_tmap;
+  if (!qmp) {  // op entry points: a map over this launch's q buffer
+    if (make_tmap_3d_bf16_strided(&qm, a.q, uint64_t(HD), uint64_t(a.H), uint64_t(a.q_rows), uint64_t(HD) * 2,
+                                  uint64_t(a.q_ld) * 2, 64, uint32_t(group), uint32_t(C::kRows / group)) != QOS_OK)
+      return cudaErrorInvalidValue;
+    qmp = &qm;
+  }
   static std::atomic<uint64_t> set{0};
   if (cudaError_t e = smem_attr_once(prefill_attn_persist_kernel<HD, POLY>, int(C::kSmem), set); e != cudaSuccess)
     return e;
@@ -1094,7 +1097,7 @@ static cudaError_t prefill_persist_t(const AttnLaunch& a, const PrefillItem* ite
   p.table_w = a.table_w;
   p.scale_log2 = a.scale_log2;
   return launch_pdl(prefill_attn_persist_kernel<HD, POLY>, dim3(n_cta), dim3(C::kThreads), C::kSmem, st, *a.kv_tmap,
-                    p, items, cta_off);
+                    *qmp, p, items, cta_off);
 }
 
 void set_fa_poly(int n) { g_fa_poly = n; }

@@ -347,6 +347,7 @@ struct qos_engine {
   };
   ActMap a_h, a_attn, a_act, a_hR;
   CUtensorMap kv_map;
+  CUtensorMap q_map;  // {hd, H, max_batch_tokens} over the q columns of `qkv` (prefill attention's Q tiles)
   float2* rope_tab = nullptr;
   int32_t* d_tables = nullptr;
   // host state
@@ -472,6 +473,12 @@ int build_maps(qos_engine* e) {
   QOS_TRY(act(e->a_hR, e->ws + s.hR, c.max_batch_rows, d));
   QOS_TRY(make_tmap_3d_bf16(&e->kv_map, e->kv, hd, uint64_t(c.num_blocks) * e->sh.Hkv * 16, uint64_t(c.n_layers) * 2,
                             64, 16, 1));
+  {
+    const int group = c.n_heads / c.n_kv_heads;
+    QOS_TRY(make_tmap_3d_bf16_strided(&e->q_map, e->ws + s.qkv, uint64_t(hd), uint64_t(e->sh.H),
+                                      uint64_t(c.max_batch_tokens), uint64_t(hd) * 2, uint64_t(e->nqkv) * 2, 64,
+                                      uint32_t(group), uint32_t(128 / group)));
+  }
   return QOS_OK;
 }
 
@@ -939,6 +946,8 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
   al.q_tiles = m.fa_qtiles;
   al.cta_off = m.n_pcta ? reinterpret_cast<const int32_t*>(dm + m.o_pcta) : nullptr;
   al.n_cta = m.n_pcta;
+  al.q_tmap = &e->q_map;
+  al.q_rows = c.max_batch_tokens;
   al.decode_stages = e->decode_stages;
   const int n_pre_rows = T - m.n_decode;
   float* gpart0 = reinterpret_cast<float*>(e->ws + s.gemm_part);
@@ -2114,6 +2123,8 @@ int qos_op_attention(qos_engine_t* e, int32_t layer, const qos_batch* b, const u
   al.q_tiles = m.fa_qtiles;
   al.cta_off = m.n_pcta ? reinterpret_cast<const int32_t*>(dm + m.o_pcta) : nullptr;
   al.n_cta = m.n_pcta;
+  al.q_tmap = nullptr;  // per-launch map over the op's q buffer
+  al.q_rows = m.T;
   al.decode_stages = e->decode_stages;
   QOS_CU(launch_prefill_attention_tc(al, reinterpret_cast<const PrefillItem*>(dm + m.o_pitems), m.n_pitems, st));
   QOS_CU(launch_decode_attention(al, reinterpret_cast<const DecodeItem*>(dm + m.o_ditems), m.n_ditems,

@@ -1171,6 +1171,22 @@ int make_tmap_3d_bf16(CUtensorMap* out, const void* base, uint64_t d0, uint64_t 
   return QOS_OK;
 }
 
+// 3-D map with explicit byte strides of dims 1 and 2 (dim 0 contiguous), 128-B swizzle
+int make_tmap_3d_bf16_strided(CUtensorMap* out, const void* base, uint64_t d0, uint64_t d1, uint64_t d2, uint64_t s1,
+                              uint64_t s2, uint32_t b0, uint32_t b1, uint32_t b2) {
+  auto fn = get_encode_fn();
+  if (!fn) return set_error(QOS_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+  cuuint64_t dims[3] = {d0, d1, d2};
+  cuuint64_t strides[2] = {s1, s2};
+  cuuint32_t box[3] = {b0, b1, b2};
+  cuuint32_t estr[3] = {1, 1, 1};
+  CUresult r = fn(out, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, const_cast<void*>(base), dims, strides, box, estr,
+                  CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return set_error(QOS_ERR_CUDA, "cuTensorMapEncodeTiled (3d strided) failed");
+  return QOS_OK;
+}
+
 template <int BN, int EPI>
 static cudaError_t launch_gemm_t(const CUtensorMap& ta, const CUtensorMap& tb, const GemmArgs& a, int grid,
                                  cudaStream_t st) {

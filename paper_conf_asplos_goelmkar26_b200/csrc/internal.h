@@ -38,6 +38,8 @@ int make_tmap_2d_bf16(CUtensorMap* out, const void* base, uint64_t rows, uint64_
                       uint32_t box_rows, uint32_t box_cols, bool swizzle128);
 int make_tmap_3d_bf16(CUtensorMap* out, const void* base, uint64_t d0, uint64_t d1, uint64_t d2, uint32_t b0,
                       uint32_t b1, uint32_t b2);
+int make_tmap_3d_bf16_strided(CUtensorMap* out, const void* base, uint64_t d0, uint64_t d1, uint64_t d2, uint64_t s1,
+                              uint64_t s2, uint32_t b0, uint32_t b1, uint32_t b2);
 int gemm_pick_bn(int64_t M, int64_t N, int epi, int num_sms);
 int gemm_check_shape(int64_t M, int64_t N, int64_t K, int epi);
 int gemm_pick_ksplit(int64_t M, int64_t N, int64_t K, int bn, int num_sms, int64_t max_units);
@@ -185,6 +187,9 @@ struct AttnLaunch {
   int q_tiles = 1;        // prefill: q tiles per CTA sharing every K/V tile (1 or 2)
   int decode_stages = 8;  // decode: K/V ring depth in (block, head) tiles (8 or 4)
   const int32_t* cta_off = nullptr;  // prefill, persistent mode: CTA c runs items [cta_off[c], cta_off[c+1])
+  const CUtensorMap* q_tmap = nullptr;  // prefill, persistent mode: 3-D map {hd, H, rows} over q with a
+                                        // {64, H/Hkv, 128/(H/Hkv)} box (NULL: built per launch)
+  int q_rows = 0;                       // rows the q map covers (its dim 2)
   int n_cta = 0;
 };
 cudaError_t launch_decode_attention(const AttnLaunch& a, const DecodeItem* items, int n_items, float* partials,
