@@ -515,8 +515,10 @@ __global__ void __launch_bounds__(FaCfg<HD, 1>::kThreads, 2)
         const int nt = it.grp_last / C::kKeys + 1, last_blk = it.grp_last >> 4;
         // Q tile of the item: rows (position, head-in-group) = a {64 dims, group heads, ppt rows}
         // box per 64-dim half; issued as soon as the previous item's last QK has read sQ
+        // (group * ppt rows: 125 when the GQA group is 5 — the remaining rows of sQ are never
+        //  valid rows (pos_r < 0: fully masked, nothing stored) and the box fills only the others)
         if (n > 0) mbar_wait(q_empty, uint32_t(n - 1) & 1);
-        mbar_arrive_expect_tx(q_full, C::kQBytes);
+        mbar_arrive_expect_tx(q_full, uint32_t(C::kHalves) * 128u * uint32_t(group * ppt));
 #pragma unroll
         for (int hf = 0; hf < C::kHalves; ++hf)
           tma_load_3d(sQ + hf * (C::kRows * 128), &qmap, q_full, hf * 64, it.kv_head * group, it.row0);

@@ -185,6 +185,9 @@ ATTN_CASES = [
     # configs[3] maximum context: a chunk deep into a 20k prefix and a decode over 32k keys
     ("llama3-70b", dict(n_layers=1, n_heads=8, n_kv_heads=1, d_model=1024, ffn_dim=1024, num_blocks=4096,
                         max_seq_len=32784), [(20000, 96)], [32767], 1.0),
+    # GQA group 5 (Qwen-2.5-14B per rank at TP2): 125 valid rows per q tile, not 128
+    ("qwen2.5-14b", dict(n_layers=1, n_heads=10, n_kv_heads=2, d_model=1280, ffn_dim=1024, num_blocks=1024),
+     [(0, 300), (100, 77)], [500, 31], 1.0),
     # the bench chunk: 512 work items (more than 2 per SM), so persistent CTAs run several each
     ("llama3-8b", dict(n_layers=1, num_blocks=2048), [(0, 2048), (512, 700)], [100], 1.0),
 ]
