@@ -370,6 +370,7 @@ struct qos_engine {
   int dual_sms_pre = 0, dual_sms_dec = 0;  // SM budgets of the two streams' GEMMs (0 = all)
   bool gemm_2cta = true;            // option gemm_2cta: CTA-pair GEMM (256 x 256 tiles) at large M
   bool decode_round_split = true;  // option decode_round_split (A/B of the split-K ranges)
+  int decode_split = 512;          // option decode_split: longest split-K key range tried first
   int decode_stages = 8;            // option decode_stages: decode K/V ring depth (8 or 4)
   int fa_qtiles = 1;                // option fa_qtiles: prefill q tiles per CTA sharing K/V tiles
   bool fa_persist = true;           // option fa_persist: persistent prefill-attention CTAs (fa_qtiles 1)
@@ -632,7 +633,7 @@ int build_step(qos_engine* e, const qos_batch* b, bool check_lengths, uint8_t* b
   // decode split-K work list (balanced on sum of keys)
   int64_t total_keys = 0;
   for (int i = 0; i < b->n_decode; ++i) total_keys += int64_t(b->decode[i].ctx_len) + 1;
-  int split = 512;
+  int split = e->decode_split;
   // splits per decode: the key blocks in nsplit near-equal block-aligned ranges of about
   // `split` keys (rounded to the nearest count, so 4097 keys make 8 ranges of 32-33 blocks, not
   // 8 full ranges and a 1-key straggler that pays a whole CTA prologue and merge)
@@ -1873,6 +1874,10 @@ int qos_engine_set_option(qos_engine_t* e, const char* name, int64_t value) {
   const std::string n(name);
   if (n == "overlap_attn") e->overlap_attn = value != 0;
   else if (n == "decode_round_split") e->decode_round_split = value != 0;
+  else if (n == "decode_split") {
+    if (value < 64 || value > 65536 || (value & (value - 1))) return set_error(QOS_ERR_INVALID_ARG, "decode_split must be a power of two in [64, 65536]");
+    e->decode_split = int(value);
+  }
   else if (n == "gemm_2cta") e->gemm_2cta = value != 0;
   else if (n == "fa_persist") e->fa_persist = value != 0;
   else if (n == "norm_fold") e->norm_fold = value != 0;

@@ -205,6 +205,7 @@ def test_llama8b_shapes_bench_batch_sampled_parity():
                                   {"gemm_swab": 2}, {"decode_round_split": 0}, {"fa_poly": 0}, {"fa_poly": 2},
                                   {"fa_qtiles": 2}, {"fa_persist": 0}, {"gemm_2cta": 0},
                                   {"norm_fold": 0}, {"gemm_swab": 0, "norm_fold": 1}, {"attn_order": 1}, {"gemm_swab": 0, "gemm_2cta": 0}, {"decode_stages": 4},
+                                  {"decode_split": 64}, {"decode_split": 4096},
                                   {"dual_stream": 1, "dual_min_prefill": 1, "dual_min_decode": 1}])
 def test_execution_options_do_not_change_results(opts):
     """qos_engine_set_option variants (serial attention, no split-K, two-stream sub-batches)
@@ -226,6 +227,8 @@ def test_execution_options_do_not_change_results(opts):
         assert row_rel_err(lg, ref) <= TOL_LOGITS
     with pytest.raises(q.QosError):
         eng.qos_engine_set_option("no_such_option", 1)
+    with pytest.raises(q.QosError):
+        eng.qos_engine_set_option("decode_split", 100)  # not a power of two
     eng.qos_engine_set_option("pdl", 1)  # process-wide: restore the defaults
     eng.qos_engine_set_option("fa_poly", 4)
     eng.close()
