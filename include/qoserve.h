@@ -250,7 +250,7 @@ int qos_profile_step_ex(qos_engine_t* eng, int32_t chunk_len, int32_t kv_start,
  *   "decode_round_split" (1) decode split-K ranges: the key blocks of a decode in a rounded
  *                          number of near-equal block-aligned ranges (0: fixed 64..512-key
  *                          ranges with a short last one)
- *   "decode_split" (512)   decode split-K: the longest key range tried first (power of two,
+ *   "decode_split" (4096)  decode split-K: the longest key range tried first (power of two,
  *                          64..65536); halved while the step has fewer than 4 items per SM
  *   "fa_poly" (4)          prefill attention: every n-th exp2 pair on the FMA pipe by a
  *                          polynomial, the rest on MUFU (0 = all MUFU; -1 = measurement-only

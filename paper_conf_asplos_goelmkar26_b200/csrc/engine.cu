@@ -370,7 +370,9 @@ struct qos_engine {
   int dual_sms_pre = 0, dual_sms_dec = 0;  // SM budgets of the two streams' GEMMs (0 = all)
   bool gemm_2cta = true;            // option gemm_2cta: CTA-pair GEMM (256 x 256 tiles) at large M
   bool decode_round_split = true;  // option decode_round_split (A/B of the split-K ranges)
-  int decode_split = 512;          // option decode_split: longest split-K key range tried first
+  int decode_split = 4096;         // option decode_split: longest split-K key range tried first
+                                   // (4096: 5-10% faster decode attention than 512 on B200,
+                                   // profiles/decode_split_ab_r1k.jsonl)
   int decode_stages = 8;            // option decode_stages: decode K/V ring depth (8 or 4)
   int fa_qtiles = 1;                // option fa_qtiles: prefill q tiles per CTA sharing K/V tiles
   bool fa_persist = true;           // option fa_persist: persistent prefill-attention CTAs (fa_qtiles 1)
