@@ -17,7 +17,9 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--points", default="512:0:0:0,2048:0:0:0,2048:0:0:6144,8192:0:0:0,0:128:4096:0")
 ap.add_argument("--layers", type=int, default=4)
 ap.add_argument("--reps", type=int, default=5)
-ap.add_argument("--variants", default="", help="A/B in one process: 'fa_poly=0;fa_poly=4' (engine options)")
+ap.add_argument("--variants", default="",
+                help="A/B in one process: 'fa_poly=0;fa_poly=4' (engine options; they persist from one "
+                     "variant to the next, so name every option a variant touches in every variant)")
 ap.add_argument("--rounds", type=int, default=1, help="interleaved repetitions of all variants")
 ap.add_argument("--step-only", action="store_true",
                 help="whole-step device time only (no per-kernel events, attention overlap left on)")
