@@ -169,14 +169,19 @@ def test_kv_tables_match_oracle_under_churn():
 
 
 @pytest.mark.slow
-def test_llama8b_shapes_bench_batch_sampled_parity():
+@pytest.mark.parametrize("split", [None, 512])
+def test_llama8b_shapes_bench_batch_sampled_parity(split):
     """2-layer Llama-3-8B (full width) at the bench launch shape: a 2048-token chunk at
-    kv_start 0 + 128 decodes @ ctx 4096 whose prefixes hold synthetic KV."""
+    kv_start 0 + 128 decodes @ ctx 4096 whose prefixes hold synthetic KV.
+    Default decode_split: one 4097-key item per (decode, kv head); 512: 8 splits merged by the
+    last arriving item."""
     C, ND, CTX = 2048, 128, 4096
     q, cfg, eng = make_engine("llama3-8b", n_layers=2, num_blocks=(C + ND * (CTX + 1)) // 16 + 200,
                               max_seq_len=8192, max_batch_tokens=C + ND, max_batch_rows=ND + 1,
                               max_requests=ND + 8)
     eng.qos_engine_load_synthetic(0)
+    if split:
+        eng.qos_engine_set_option("decode_split", split)
     b = synth.hybrid_batch(cfg.vocab, C, ND, CTX)
     eng.qos_kv_alloc(0, C)
     for d in b.decode:
