@@ -67,7 +67,8 @@ typedef struct {
   int32_t max_seq_len;      /* max tokens per request; block-table width = ceil(/16)         */
   int32_t max_requests;     /* max live requests (block-table rows)                          */
   int32_t max_batch_tokens; /* max T = sum(chunk_len) + n_decode per step                    */
-  int32_t max_batch_rows;   /* max R = n_prefill + n_decode per step                         */
+  int32_t max_batch_rows;   /* max R = n_prefill + n_decode per step; max_batch_rows x       */
+                            /* n_kv_heads/tp <= 65536 (decode work items; QOS_ERR_UNSUPPORTED) */
 } qos_model_cfg;
 
 typedef struct {
@@ -163,7 +164,11 @@ int qos_engine_read_weight(qos_engine_t* eng, const char* name, int64_t row0, in
  * the engine's internal stream before the next step.  KV is held only while needed
  * (§3.4). */
 int qos_kv_alloc(qos_engine_t* eng, int64_t req, int32_t n_tokens_total);
-/* Release all of req's blocks (QOS_ERR_UNKNOWN_REQ if it has none). */
+/* Release all of req's blocks (QOS_ERR_UNKNOWN_REQ if it has none).  The blocks and the table
+ * row are reusable at once on the host side.  Ordering: the engine's own device work (KV fills,
+ * table flushes, op entry points) waits for the last step enqueued through qos_hybrid_step; a
+ * later qos_hybrid_step on ANOTHER caller stream is not ordered after an in-flight step that
+ * read the freed blocks -- use one stream for steps, or synchronise before reusing them. */
 int qos_kv_free(qos_engine_t* eng, int64_t req);
 /* Inspect req's table: writes min(cap, n) block ids to out, n to *n_out. */
 int qos_kv_table(qos_engine_t* eng, int64_t req, int32_t* out, int32_t cap, int32_t* n_out);

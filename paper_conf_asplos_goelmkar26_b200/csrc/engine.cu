@@ -365,6 +365,7 @@ struct qos_engine {
   int attn_order = 0;             // option attn_order: 0 prefill first on `side`; 1 decode first, prefill
                                   // on `side_lo`; 2 decode first, prefill on `side`
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr, ev_fork2 = nullptr, ev_join2 = nullptr;
+  cudaEvent_t ev_step_done = nullptr;  // end of the last step, on the caller's stream
   bool dual_stream = false;       // QOS_DUAL=1: prefill rows and decode rows on two streams
   int dual_min_prefill = 512, dual_min_decode = 16;
   int dual_sms_pre = 0, dual_sms_dec = 0;  // SM budgets of the two streams' GEMMs (0 = all)
@@ -501,6 +502,8 @@ int check_cfg(const qos_model_cfg* c, int tp) {
       c->max_batch_rows < 1)
     return set_error(QOS_ERR_INVALID_ARG, "capacities must be >= 1");
   if (c->max_batch_rows > c->max_batch_tokens) return set_error(QOS_ERR_INVALID_ARG, "max_batch_rows > max_batch_tokens");
+  if (int64_t(c->max_batch_rows) * (c->n_kv_heads / tp) > kMaxDecodeItems)
+    return set_error(QOS_ERR_UNSUPPORTED, "max_batch_rows * kv heads per rank exceeds the decode item workspace");
   return QOS_OK;
 }
 
@@ -653,7 +656,12 @@ int build_step(qos_engine* e, const qos_batch* b, bool check_lengths, uint8_t* b
       return n * e->sh.Hkv;
     };
     while (split > 64 && count_items(split) < target) split /= 2;
-    while (count_items(split) > e->wsl.max_items) split *= 2;
+    // every decode contributes >= 1 item per kv head however long the ranges get, so the
+    // doubling stops at the longest possible context; a step that still exceeds the item
+    // workspace (n_decode * Hkv > max_items) is refused
+    while (split < (1 << 24) && count_items(split) > e->wsl.max_items) split *= 2;
+    if (count_items(split) > e->wsl.max_items)
+      return set_error(QOS_ERR_UNSUPPORTED, "decode work list exceeds the item workspace (n_decode * kv heads)");
   }
   std::vector<DecodeItem> ditems;
   int part = 0;
@@ -737,6 +745,14 @@ int acquire_staging(qos_engine* e) {
 int release_staging(qos_engine* e, cudaStream_t st) {
   QOS_CU(cudaEventRecord(e->meta_free[e->meta_cur], st));
   return QOS_OK;
+}
+
+// The internal stream, ordered after the last step enqueued on the caller's stream: KV fills,
+// table flushes and the op entry points may touch blocks / table rows that an in-flight step
+// (freed and re-allocated meanwhile) still reads (qos_kv_free returns them at once).
+cudaStream_t internal_stream(qos_engine* e) {
+  if (e->ev_step_done) cudaStreamWaitEvent(e->stream, e->ev_step_done, 0);
+  return e->stream;
 }
 
 int flush_table_updates(qos_engine* e, cudaStream_t st) {
@@ -1184,6 +1200,7 @@ int do_step(qos_engine* e, const qos_batch* b, void* logits, int logits_dtype, i
     return r;
   }
   QOS_TRY(release_staging(e, st));
+  QOS_CU(cudaEventRecord(e->ev_step_done, st));
   e->last_h2d = int64_t(m.used);
   e->last_d2h = on_host ? int64_t(m.R) * ((next_tokens ? 4 : 0) +
                                           (logits ? int64_t(e->cfg.vocab) * (logits_dtype == QOS_F32 ? 4 : 2) : 0))
@@ -1495,6 +1512,7 @@ static int create_engine(const qos_model_cfg* cfg, int device, int tp_rank, int 
     cudaEventCreateWithFlags(&e->ev_join, cudaEventDisableTiming);
     cudaEventCreateWithFlags(&e->ev_fork2, cudaEventDisableTiming);
     cudaEventCreateWithFlags(&e->ev_join2, cudaEventDisableTiming);
+    cudaEventCreateWithFlags(&e->ev_step_done, cudaEventDisableTiming);
   }
   e->free_heap.resize(size_t(cfg->num_blocks));
   for (int64_t i = 0; i < cfg->num_blocks; ++i) e->free_heap[size_t(i)] = int32_t(i);  // sorted = valid min-heap
@@ -1589,6 +1607,7 @@ int qos_engine_destroy(qos_engine_t* e) {
   if (e->ev_join) cudaEventDestroy(e->ev_join);
   if (e->ev_fork2) cudaEventDestroy(e->ev_fork2);
   if (e->ev_join2) cudaEventDestroy(e->ev_join2);
+  if (e->ev_step_done) cudaEventDestroy(e->ev_step_done);
   delete e;
   return QOS_OK;
 }
@@ -1599,7 +1618,7 @@ int qos_engine_load_synthetic(qos_engine_t* e, uint64_t seed) {
   const auto& c = e->cfg;
   const auto& sh = e->sh;
   const int d = c.d_model, hd = c.head_dim;
-  cudaStream_t st = e->stream;
+  cudaStream_t st = internal_stream(e);
   char name[256];
   auto H = [&](const char* s) { return fnv1a64(s); };
   for (int l = 0; l < c.n_layers; ++l) {
@@ -1759,7 +1778,7 @@ int qos_kv_table_device(qos_engine_t* e, int64_t req, int32_t* out, int32_t cap,
   auto it = e->reqs.find(req);
   if (it == e->reqs.end()) return set_error(QOS_ERR_UNKNOWN_REQ, "unknown request");
   QOS_CU(cudaSetDevice(e->device));
-  QOS_TRY(flush_table_updates(e, e->stream));
+  QOS_TRY(flush_table_updates(e, internal_stream(e)));
   QOS_CU(cudaStreamSynchronize(e->stream));
   const int n = int(it->second.blocks.size());
   *n_out = n;
@@ -1788,7 +1807,7 @@ int qos_kv_fill_synthetic(qos_engine_t* e, int64_t req, int32_t n_tokens, uint64
   if (it == e->reqs.end()) return set_error(QOS_ERR_UNKNOWN_REQ, "unknown request");
   if (int64_t(it->second.blocks.size()) * 16 < n_tokens) return set_error(QOS_ERR_NOT_ALLOCATED, "not allocated");
   QOS_CU(cudaSetDevice(e->device));
-  cudaStream_t st = e->stream;
+  cudaStream_t st = internal_stream(e);
   QOS_TRY(flush_table_updates(e, st));
   const int32_t* trow = e->d_tables + size_t(it->second.row) * e->table_w;
   char name[128];
@@ -1842,7 +1861,7 @@ int qos_profile_step_ex(qos_engine_t* e, int32_t chunk_len, int32_t kv_start, in
     dec[size_t(j)] = qos_decode{id, ctx_lens[j], int32_t((j * 31 + 7) % e->cfg.vocab)};
   }
   qos_batch b{chunk_len > 0 ? 1 : 0, &ch, n_decode, dec.data()};
-  cudaStream_t st = e->stream;
+  cudaStream_t st = internal_stream(e);
   cudaEvent_t a, z;
   cudaEventCreate(&a);
   cudaEventCreate(&z);
@@ -2038,7 +2057,7 @@ static int kv_rw(qos_engine* e, int32_t layer, int64_t req, int32_t pos0, int32_
   if (it == e->reqs.end()) return set_error(QOS_ERR_UNKNOWN_REQ, "unknown request");
   if (int64_t(pos0) + n > int64_t(it->second.blocks.size()) * 16) return set_error(QOS_ERR_NOT_ALLOCATED, "range");
   QOS_CU(cudaSetDevice(e->device));
-  cudaStream_t st = e->stream;
+  cudaStream_t st = internal_stream(e);
   QOS_TRY(flush_table_updates(e, st));
   const size_t bytes = size_t(n) * e->sh.Hkv * e->cfg.head_dim * 2;
   QOS_TRY(ensure_dbg(e, bytes));
@@ -2070,7 +2089,7 @@ int qos_kv_read(qos_engine_t* e, int32_t layer, int64_t req, int32_t pos0, int32
 int qos_op_qkv_rope_append(qos_engine_t* e, int32_t layer, const qos_batch* b, const uint16_t* h_in, uint16_t* q_out) {
   if (!e || !h_in || !q_out || layer < 0 || layer >= e->cfg.n_layers) return set_error(QOS_ERR_INVALID_ARG, "args");
   QOS_CU(cudaSetDevice(e->device));
-  cudaStream_t st = e->stream;
+  cudaStream_t st = internal_stream(e);
   QOS_TRY(acquire_staging(e));
   StepMeta m;
   int r = build_step(e, b, false, e->h_meta[e->meta_cur], m);
@@ -2099,7 +2118,7 @@ int qos_op_qkv_rope_append(qos_engine_t* e, int32_t layer, const qos_batch* b, c
 int qos_op_attention(qos_engine_t* e, int32_t layer, const qos_batch* b, const uint16_t* q_in, float* out) {
   if (!e || !q_in || !out || layer < 0 || layer >= e->cfg.n_layers) return set_error(QOS_ERR_INVALID_ARG, "args");
   QOS_CU(cudaSetDevice(e->device));
-  cudaStream_t st = e->stream;
+  cudaStream_t st = internal_stream(e);
   QOS_TRY(acquire_staging(e));
   StepMeta m;
   int r = build_step(e, b, false, e->h_meta[e->meta_cur], m);

@@ -121,6 +121,8 @@ class SchedulerConfig:
     margin: float = 0.05              # under-predict the chunk
     max_decodes: int = 256
     max_rows: int = 264               # engine capacity: chunks + decodes per step (max_batch_rows)
+    max_tokens: int | None = None     # engine capacity: prefill tokens + decodes per step
+                                      # (max_batch_tokens); None = unbounded
     # "slack": QoServe's dynamic chunking (the chunk fits the minimum decode slack);
     # "medha": Medha-style adaptive chunking (NEXT-4 variant): every step
     # targets a fixed latency, so chunks shrink as the prefill's cached prefix grows
@@ -208,19 +210,35 @@ class QoServeScheduler:
 
     # ---------------------------------------------------------------- Algorithm 1
     def create_batch(self, now: float):
-        """Returns (chunks [(Request, n_tokens)], decodes [Request])."""
+        """Returns (chunks [(Request, n_tokens)], decodes [Request]).
+
+        Capacity (the engine's, not the paper's): a chunk that completes its request's prefill
+        turns it into a decode at the end of the step, so such chunks are only taken while
+        decodes + finishing prefills stay within max_decodes; a chunk that would overflow the
+        decode set is cut one token short of the prompt's end (it keeps progressing and finishes
+        once a decode slot frees).  The decode set therefore never exceeds max_decodes and every
+        decode is scheduled every step (decodes are never preempted)."""
         decodes = list(self.decode_q)[: self.cfg.max_decodes]          # GET_ALL_DECODES
         ctx = [r.ctx_len for r in decodes]                              # GET_DECODE_CONTEXT
         queue = sorted(self.prefill_q, key=self.sort_key)               # line 8
         kv0 = queue[0].prefill_done if queue else 0                     # prefix of the head chunk
         C = self.prefill_budget(ctx, self.min_slack(now), kv0)          # lines 5-7
+        if self.cfg.max_tokens is not None:
+            C = max(0, min(C, self.cfg.max_tokens - len(decodes)))
         chunks, count = [], 0
-        inflight_skipped = []
+        finishing = 0                     # chunks of this batch that complete their prefill
+
+        def fit(r: Request, want: int) -> int:
+            """Tokens of r to take: want, unless that finishes r into a full decode set."""
+            if want >= r.prefill_rem and len(self.decode_q) + finishing >= self.cfg.max_decodes:
+                return r.prefill_rem - 1
+            return want
+
         i = 0
         while count < C and i < len(queue) and len(chunks) + len(decodes) < self.cfg.max_rows:   # line 10
             top = queue[i]
-            if top.prefill_done == 0 and len(self.decode_q) >= self.cfg.max_decodes:
-                # admission: a new prompt would finish into a full decode set (engine capacity)
+            if top.prefill_done == 0 and len(self.decode_q) + finishing >= self.cfg.max_decodes:
+                # admission: a new prompt is not started while the decode set is full
                 i += 1
                 continue
             if not top.relegated and self.will_violate(top, now, C, ctx):   # line 12
@@ -231,24 +249,26 @@ class QoServeScheduler:
                     top.relegated = True                                # lines 13-14
                     queue.append(queue.pop(i))                          # re-pushed, sorts last
                     continue
-            take = min(C - count, top.prefill_rem)                      # line 17
+            take = fit(top, min(C - count, top.prefill_rem))            # line 17
             if take > 0:
                 chunks.append((top, take))                              # lines 18-20
                 count += take
+                finishing += take == top.prefill_rem
             i += 1                                                      # line 21 (POP)
         # selective preemption: an already started prefill that was displaced keeps its slot
-        # when waiting one more iteration would make it violate
+        # when waiting one more iteration would make it violate -- but only
+        # within what is left of the budget C (the decode slack bounds the whole step)
         chosen = {r.req_id for r, _ in chunks}
         for r in queue[i:]:
+            if count >= C or len(chunks) + len(decodes) >= self.cfg.max_rows:
+                break
             if r.prefill_done > 0 and r.req_id not in chosen and not r.relegated:
                 if self.will_violate(r, now + self.step_estimate_s(C, ctx), max(C, 1), ctx):
-                    inflight_skipped.append(r)
-        for r in inflight_skipped:
-            if len(chunks) + len(decodes) >= self.cfg.max_rows:
-                break
-            take = min(max(self.cfg.min_chunk, C - count), r.prefill_rem)
-            chunks.append((r, take))
-            count += take
+                    take = fit(r, min(C - count, r.prefill_rem))
+                    if take > 0:
+                        chunks.append((r, take))
+                        count += take
+                        finishing += take == r.prefill_rem
         return chunks, decodes
 
     def complete(self, chunks, decodes, t_end: float) -> list[Request]:

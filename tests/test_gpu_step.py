@@ -135,6 +135,49 @@ def test_step_errors_leave_state_unchanged():
     eng.close()
 
 
+def test_engine_refuses_a_decode_work_list_beyond_its_workspace():
+    """max_batch_rows x kv heads must fit the decode item workspace (65536 items): a config
+    that could exceed it is refused at creation instead of looping in the split search."""
+    from paper_conf_asplos_goelmkar26_b200 import qoserve as q
+    with pytest.raises(q.QosError) as ei:
+        make_engine("tiny", max_batch_tokens=40000, max_batch_rows=40000)   # 40000 x 2 kv heads
+    assert ei.value.name == "UNSUPPORTED"
+    q_, cfg, eng = make_engine("tiny", max_batch_tokens=32768, max_batch_rows=32768)   # exactly 65536
+    eng.close()
+
+
+def test_free_realloc_fill_is_ordered_after_an_inflight_step():
+    """qos_kv_free returns blocks at once; a fill of a new request that reuses them runs on the
+    engine's internal stream, which must wait for the step still reading them (step enqueued
+    asynchronously with device outputs on the caller's stream)."""
+    import torch
+    q, cfg, eng = make_engine("tiny", num_blocks=64)
+    eng.qos_engine_load_synthetic(0)
+    ctx = 600
+    eng.qos_kv_alloc(1, ctx + 1)
+    eng.qos_kv_fill_synthetic(1, ctx, 2)
+    b = q.make_batch([], [(1, ctx, 7)])
+    ref_lg, _ = eng.step_host(b, cfg.vocab)
+    eng.qos_kv_free(1)
+    eng.qos_kv_alloc(1, ctx + 1)                 # the same blocks again (lowest free first)
+    eng.qos_kv_fill_synthetic(1, ctx, 2)
+    lg = torch.empty((1, cfg.vocab), dtype=torch.float32, device="cuda")
+    s = torch.cuda.Stream()
+    for _ in range(3):
+        with torch.cuda.stream(s):
+            eng.qos_hybrid_step(b, lg.data_ptr(), q.QOS_F32, 0, 0, s.cuda_stream)
+        # while the step may still run: free, take the blocks for another request, overwrite them
+        eng.qos_kv_free(1)
+        eng.qos_kv_alloc(2, ctx + 1)
+        eng.qos_kv_fill_synthetic(2, ctx, 99)
+        s.synchronize()
+        assert row_rel_err(lg.cpu().numpy(), ref_lg) == 0.0
+        eng.qos_kv_free(2)
+        eng.qos_kv_alloc(1, ctx + 1)
+        eng.qos_kv_fill_synthetic(1, ctx, 2)
+    eng.close()
+
+
 def test_kv_tables_match_oracle_under_churn():
     from oracle.kv import BlockAllocator, OracleOOM
     q, cfg, eng = make_engine("tiny", num_blocks=300)

@@ -216,3 +216,86 @@ def test_batches_respect_engine_capacity():
     s.decode_q = s.decode_q[:4]             # four decodes leave
     chunks, decodes = s.create_batch(0.0)
     assert chunks and len(chunks) + len(decodes) <= cfg.max_rows
+
+
+def test_decode_set_never_exceeds_max_decodes():
+    """Prompts that finish in the same batch count toward the decode limit: with 3 decodes
+    running and max_decodes = 4, three short prompts must not all finish into the decode set
+    (which would leave some decodes unscheduled while their TBT deadlines pass)."""
+    cfg = SchedulerConfig(max_chunk=4096, max_decodes=4, max_rows=16, margin=0.0)
+    s = QoServeScheduler(cfg, lambda chunks, ctx: 5.0 + 0.002 * sum(n for _, n in chunks) + 0.01 * len(ctx))
+    for i in range(3):
+        r = Request(100 + i, 0.0, 64, "Q1", decode_len=6)
+        r.prefill_done = r.prompt_len
+        r.decoded = 1
+        s.decode_q.append(r)
+    for i in range(3):
+        s.submit(Request(i, 0.0, 32, "Q1", decode_len=3))
+    now = 0.0
+    for _ in range(60):
+        chunks, decodes = s.create_batch(now)
+        if not chunks and not decodes:
+            break
+        assert len(decodes) == len(s.decode_q) <= cfg.max_decodes       # every decode runs every step
+        fin = sum(1 for r, n in chunks if n == r.prefill_rem)
+        assert len(s.decode_q) + fin <= cfg.max_decodes
+        now += 0.01
+        s.complete(chunks, decodes, now)
+        assert len(s.decode_q) <= cfg.max_decodes
+    assert not s.decode_q and not s.prefill_q                            # everything finished
+
+
+def test_partial_prefill_waits_one_token_short_of_a_full_decode_set():
+    """A started prefill whose last chunk would finish into a full decode set is cut one token
+    short; it completes once a decode slot frees."""
+    cfg = SchedulerConfig(max_chunk=4096, max_decodes=2, max_rows=16, margin=0.0)
+    s = QoServeScheduler(cfg, lambda chunks, ctx: 5.0)
+    for i in range(2):
+        r = Request(100 + i, 0.0, 64, "Q2", decode_len=3)
+        r.prefill_done, r.decoded = r.prompt_len, 1
+        s.decode_q.append(r)
+    p = Request(1, 0.0, 100, "Q2", decode_len=2)
+    p.prefill_done = 40
+    s.submit(p)
+    chunks, decodes = s.create_batch(0.0)
+    assert chunks == [(p, 59)] and len(decodes) == 2
+    s.complete(chunks, decodes, 0.01)
+    chunks, decodes = s.create_batch(0.01)
+    assert chunks == [] and len(decodes) == 2                           # still full: no finishing chunk
+    s.complete(chunks, decodes, 0.02)                                   # both decodes finish (3 tokens)
+    chunks, decodes = s.create_batch(0.02)
+    assert chunks == [(p, 1)] and decodes == []
+
+
+def test_preemption_stays_within_the_budget_and_token_capacity():
+    """Selective preemption takes displaced in-flight prefills only from what is left of the
+    budget C, and no batch exceeds the engine's token capacity (max_tokens)."""
+    C = 256
+    cfg = SchedulerConfig(max_chunk=C, min_chunk=64, chunk_step=64, max_decodes=64, max_rows=64, margin=0.0,
+                          max_tokens=C + 8)
+    # every step takes 1 s, so any started prompt with a 6 s TTFT is about to violate
+    s = QoServeScheduler(cfg, lambda chunks, ctx: 1000.0)
+    started = []
+    for i in range(6):
+        r = Request(i, 0.0, 4000, "Q1", decode_len=2)
+        r.prefill_done = 100
+        s.submit(r)
+        started.append(r)
+    for i in range(16):
+        r = Request(100 + i, 0.0, 64, "Q2", decode_len=10 ** 6)
+        r.prefill_done, r.decoded = r.prompt_len, 1
+        s.decode_q.append(r)
+    for t in (0.0, 1.0, 2.0, 3.0):
+        chunks, decodes = s.create_batch(t)
+        tok = sum(n for _, n in chunks)
+        assert tok <= C and tok + len(decodes) <= cfg.max_tokens
+    # the token capacity also caps an unconstrained budget
+    s2 = QoServeScheduler(SchedulerConfig(max_chunk=4096, max_tokens=1000, max_decodes=64, max_rows=64),
+                          lambda chunks, ctx: 1.0)
+    for i in range(8):
+        r = Request(100 + i, 0.0, 64, "Q2", decode_len=10 ** 6)
+        r.prefill_done, r.decoded = r.prompt_len, 1
+        s2.decode_q.append(r)
+    s2.submit(Request(1, 0.0, 5000, "Q2"))
+    chunks, decodes = s2.create_batch(0.0)
+    assert sum(n for _, n in chunks) + len(decodes) == 1000

@@ -51,13 +51,17 @@ def main():
         eng.qos_engine_load_synthetic(0)
         shapes, ms = [], []
         eng.qos_profile_step(2048, [2048] * 64, reps=5, warmup=5)
+        # the grid varies every feature the model separates: chunk length, the chunk's cached
+        # prefix (kv_start), decode count and decode context (KV bytes), so neither the prefix
+        # coefficient nor the per-KV-byte coefficient is left unidentified
         for c in (0, 256, 512, 1024, 2048, 3072, 4096):
             for nd in (0, 16, 64, 128, 256):
-                if (c == 0 and nd == 0) or c > a.max_chunk:
-                    continue
-                t, _ = eng.qos_profile_step(c, [1536] * nd, reps=3, warmup=3)
-                shapes.append(StepShape([(0, c)] if c else [], [1536] * nd))
-                ms.append(t)
+                for ctx, ks in ((512, 0), (2048, 2048), (6144, 0), (1536, 4096)):
+                    if (c == 0 and nd == 0) or c > a.max_chunk or (c == 0 and ks) or nd * (ctx + 1) > 1_000_000:
+                        continue
+                    t, _ = eng.qos_profile_step(c, [ctx] * nd, reps=3, warmup=2, kv_start=ks)
+                    shapes.append(StepShape([(ks, c)] if c else [], [ctx] * nd))
+                    ms.append(t)
         model = LatencyModel().fit(shapes, ms)
     else:
         prof = json.load(open(os.path.join(ROOT, "profiles", "latency_table_r1.json")))
@@ -71,7 +75,8 @@ def main():
 
         def mk_sched():
             return QoServeScheduler(SchedulerConfig(alpha_ms_per_token=a.alpha, max_chunk=a.max_chunk,
-                                                    max_decodes=256, max_rows=257), pred)
+                                                    max_decodes=256, max_rows=257,
+                                                    max_tokens=a.max_chunk + 512), pred)
         if a.mode == "engine":
             ex = EngineExecutor(eng, 128256, lambda r, s, n: synth.request_tokens(r, n, 128256, start=s))
             out = replay(tr, mk_sched(), ex)
