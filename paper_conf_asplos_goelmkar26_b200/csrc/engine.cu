@@ -369,6 +369,8 @@ struct qos_engine {
   bool dual_stream = false;       // QOS_DUAL=1: prefill rows and decode rows on two streams
   int dual_min_prefill = 512, dual_min_decode = 16;
   int dual_sms_pre = 0, dual_sms_dec = 0;  // SM budgets of the two streams' GEMMs (0 = all)
+  int gemm_sms = 0;                // option gemm_sms: SM budget of the fused step's GEMMs (0 = all)
+  bool add_split = true;           // option add_split: ordered split-K of the O / down projections
   bool gemm_2cta = true;            // option gemm_2cta: CTA-pair GEMM (256 x 256 tiles) at large M
   bool decode_round_split = true;  // option decode_round_split (A/B of the split-K ranges)
   int decode_split = 4096;         // option decode_split: longest split-K key range tried first
@@ -793,10 +795,14 @@ int gemm_any(qos_engine* e, const qos_engine::ActMap& am, const CUtensorMap (&tb
   }
   if (e->gemm_2cta && gemm2_eligible(M, N, K, sms))
     return gemm2_run(am.m128, tb[0], M, N, K, epi, C, ldc, bias, sms, st, a_row0, sms, rope, fold);
-  const int bn = gemm_pick_bn(M, N, epi, sms);
-  const int ks = e->gemm_splitk ? gemm_pick_ksplit(M, N, K, bn, sms, kGemmMaxUnits) : 1;
+  int bn = gemm_pick_bn(M, N, epi, sms);
+  int ks = e->gemm_splitk ? gemm_pick_ksplit(M, N, K, bn, sms, kGemmMaxUnits) : 1;
+  const bool coop = !e->dual_stream && !e->shares_device;
+  // O / down below the fold threshold: tile width + ordered in-place split-K by wave cost
+  if (epi == EPI_ADD_F32 && !fold && coop && e->add_split && !e->gemm_splitk && !e->gemm_streamk)
+    gemm_pick_add_split(M, N, K, sms, kGemmMaxTiles, &bn, &ks);
   return gemm_run(am.m128, tb[bn == 256 ? 1 : 0], bn, M, N, K, epi, C, ldc, bias, sms, st, ks, part, cnt, a_row0, sms,
-                  rope, e->gemm_streamk, !e->dual_stream && !e->shares_device, fold);
+                  rope, e->gemm_streamk, coop, fold);
 }
 
 int gemm(qos_engine* e, const qos_engine::ActMap& am, const CUtensorMap (&tb)[2], int64_t M, int64_t N, int64_t K,
@@ -985,12 +991,12 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
     QOS_CU(cudaEventRecord(e->ev_fork, st));
     QOS_CU(cudaStreamWaitEvent(e->side, e->ev_fork, 0));
   } else {
-    segs[nseg++] = Seg{0, T, st, m.n_pitems > 0, m.n_ditems > 0, gpart0, gcnt0, 0};
+    segs[nseg++] = Seg{0, T, st, m.n_pitems > 0, m.n_ditems > 0, gpart0, gcnt0, e->gemm_sms};
   }
   // RMSNorm folded into the projections (NormFold, internal.h) when all four GEMMs of the step
   // run whole tiles in one pass: the O / down epilogues produce r, h = bf16(r * g) and per-row
   // sums of squares, the QKV / gate-up epilogues scale their rows by 1/rms — no norm launches
-  const int sms_all = e->num_sms;
+  const int sms_all = e->gemm_sms > 0 ? e->gemm_sms : e->num_sms;
   // (from T = 1536: below, the read-add-write epilogue of the last wave costs what the norm
   //  launches cost — 512 tokens +1.5%, 1024 neutral, 2176 -1.5%, 4096 -4.6%, tools/attn_bench.py r1f)
   const bool fold = e->norm_fold && !tp && nseg == 1 && !g_skip_norm && T >= kFoldMinTokens && d % 128 == 0 &&
@@ -1499,6 +1505,7 @@ static int create_engine(const qos_model_cfg* cfg, int device, int tp_rank, int 
   if (const char* sw = getenv("QOS_GEMM_SWAB")) e->gemm_swab = atoi(sw);
   if (const char* sk = getenv("QOS_GEMM_STREAMK")) e->gemm_streamk = atoi(sk);
   if (const char* du = getenv("QOS_DUAL")) e->dual_stream = atoi(du) != 0;
+  if (const char* as = getenv("QOS_ADD_SPLIT")) e->add_split = atoi(as) != 0;
   if (const char* a = getenv("QOS_DUAL_MIN_PREFILL")) e->dual_min_prefill = atoi(a);
   if (const char* a = getenv("QOS_DUAL_MIN_DECODE")) e->dual_min_decode = atoi(a);
   if (const char* a = getenv("QOS_DUAL_SMS_PRE")) e->dual_sms_pre = atoi(a);
@@ -1926,6 +1933,8 @@ int qos_engine_set_option(qos_engine_t* e, const char* name, int64_t value) {
   else if (n == "dual_min_decode") e->dual_min_decode = int(value);
   else if (n == "dual_sms_prefill") e->dual_sms_pre = int(value);
   else if (n == "dual_sms_decode") e->dual_sms_dec = int(value);
+  else if (n == "add_split") e->add_split = value != 0;
+  else if (n == "gemm_sms") e->gemm_sms = int(value < 0 ? 0 : value > e->num_sms ? e->num_sms : value);
   else return set_error(QOS_ERR_INVALID_ARG, "unknown option");
   return QOS_OK;
 }
@@ -1979,7 +1988,7 @@ static int op_gemm(const void* A, const void* B, void* C, int64_t M, int64_t N, 
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  const int bn = gemm_pick_bn(M, N, epi, sms);
+  int bn = gemm_pick_bn(M, N, epi, sms);
   static float* part = nullptr;  // process-wide split-K workspace of the op entry point
   static int* cnt = nullptr;
   if (!part) {
@@ -2009,12 +2018,19 @@ static int op_gemm(const void* A, const void* B, void* C, int64_t M, int64_t N, 
     count_launch();
     return gemm2_run(ta, tb, M, N, K, epi, C, ldc, bias, sms, reinterpret_cast<cudaStream_t>(stream), 0, 0, nullptr);
   }
-  const int64_t tiles = ((M + 127) / 128) * ((N + bn - 1) / bn);
   const int sk_mode = ksplit <= -2 ? 2 : 0;
   // automatic = the engine's default: no split-K (QOS_GEMM_SPLITK=1 restores the split heuristic)
   static const bool sk_env = getenv("QOS_GEMM_SPLITK") && atoi(getenv("QOS_GEMM_SPLITK")) != 0;
   int ks = ksplit <= -2 ? 1 : ksplit <= 0 ? (sk_env ? gemm_pick_ksplit(M, N, K, bn, sms, kGemmMaxUnits) : 1) : ksplit;
-  if (ks > 1 && (tiles > kGemmMaxTiles || tiles * ks > kGemmMaxUnits || (K / 64) < ks))
+  static const bool as_env = !(getenv("QOS_ADD_SPLIT") && atoi(getenv("QOS_ADD_SPLIT")) == 0);
+  if (ksplit == 0 && !sk_env && as_env && epi == QOS_EPI_ADD_F32) gemm_pick_add_split(M, N, K, sms, kGemmMaxTiles, &bn, &ks);
+  if (const char* fb = getenv("QOS_GEMM_BN")) {  // measurement only: force the tile width
+    const int v = atoi(fb);
+    if (v == 128 || (v == 256 && N % 256 == 0)) bn = v;
+  }
+  const int64_t tiles = ((M + 127) / 128) * ((N + bn - 1) / bn);
+  const bool ordered = epi == QOS_EPI_ADD_F32;  // in-place ordered slices: no partial slots
+  if (ks > 1 && (tiles > kGemmMaxTiles || (!ordered && tiles * ks > kGemmMaxUnits) || (K / 64) < ks))
     return set_error(QOS_ERR_INVALID_ARG, "gemm: ksplit too large for the shape / workspace");
   CUtensorMap ta, tb;
   QOS_TRY(make_tmap_2d_bf16(&ta, A, uint64_t(M), uint64_t(K), uint64_t(K), 128, 64, true));

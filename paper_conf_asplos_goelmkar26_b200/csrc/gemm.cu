@@ -20,6 +20,9 @@
 #include <cstdio>
 #include <cstdlib>
 
+#include <climits>
+#include <cstdlib>
+
 #include "common.cuh"
 #include "internal.h"
 
@@ -59,6 +62,9 @@ struct GemmArgs {
   int ksplit;       // K slices per tile (split-K for weight-bound small-M GEMMs); 1 = off
   int sk;           // stream-K: the (tile, k-block) space in equal contiguous ranges per CTA
   int coop;         // stream-K: cut tiles reduced by all their CTAs after their ranges
+  int ordered;      // split-K of EPI_ADD_F32 (ksplit > 1): every slice red.adds its partial into
+                    // C in slice order (slice s waits for counters[tile] == s): no partials,
+                    // deterministic; units split-major so a slice never waits on a later unit
   int64_t work;     // stream-K: mt * nt * kblocks
   void* C;
   int ldc;          // elements
@@ -607,10 +613,18 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
   const int num_units = p.mt * p.nt * ks;
   const int kblocks = p.K / kBK;
   auto decode_unit = [&](int u, int& m_t, int& n_t, int& sp, int& kb0, int& kb1) {
-    m_t = u % p.mt;
-    const int r = u / p.mt;
-    sp = r % ks;
-    n_t = r / ks;
+    if (p.ordered) {  // u = sp * tiles + n_t * mt + m_t
+      const int tiles = p.mt * p.nt;
+      sp = u / tiles;
+      const int t = u - sp * tiles;
+      m_t = t % p.mt;
+      n_t = t / p.mt;
+    } else {
+      m_t = u % p.mt;
+      const int r = u / p.mt;
+      sp = r % ks;
+      n_t = r / ks;
+    }
     kb0 = sp * kblocks / ks;
     kb1 = (sp + 1) * kblocks / ks;
   };
@@ -876,6 +890,30 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
         tc_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(&tempty[acc]);
+      } else if (p.ordered) {
+        // ordered split-K (EPI_ADD_F32): slice sp adds its partial after slices 0..sp-1 (their
+        // red.adds are visible once counters[tile] == sp), so C sees a fixed summation order
+        const int tile = n_t * p.mt + m_t;
+        if (sp > 0) {
+          if (threadIdx.x == 64) {
+            int v;
+            do {
+              asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p.counters + tile) : "memory");
+            } while (v != sp);
+          }
+          epi_bar_sync();
+        }
+        epi_tmem(n_t, row, row_ok, tbase);
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&tempty[acc]);
+        if (sp + 1 < ks) {
+          __threadfence();
+          epi_bar_sync();
+          if (threadIdx.x == 64) asm volatile("st.release.gpu.global.b32 [%0], %1;" ::"l"(p.counters + tile), "r"(sp + 1) : "memory");
+        } else if (threadIdx.x == 64) {
+          p.counters[tile] = 0;  // ready for the next launch (no slice waits after the last)
+        }
       } else {
         // split-K: park the fp32 partial, release TMEM, the last slice of the tile reduces
         float* mine = p.part + (size_t(u) * kBM + rit) * BN;
@@ -1210,6 +1248,47 @@ int gemm_pick_bn(int64_t M, int64_t N, int epi, int num_sms) {
   return w256 * 630 < w128 * 445 ? 256 : 128;
 }
 
+// Tile width and ordered split-K of an EPI_ADD_F32 projection (the O and down projections of
+// a step below the fold threshold).  The mid-T steps (T 256-1024) leave most SMs idle with
+// whole tiles (T = 512: 64 tiles of 128 x 256 on 148 SMs); slicing K fills them, but every
+// extra slice serialises one more red.add epilogue of the tile.  Cost of a launch =
+// waves x k-blocks per unit x c(BN) + (slices - 1) x E(BN), with c and E fitted (relative
+// least squares, max error 19%, mean 4%) to the O and down projections of Llama-3-8B at
+// T = 256..1536 over BN {128, 256} x slices {1..4} (tools/gemm_bench.py with QOS_GEMM_BN,
+// profiles/gemm_addsplit_grid_r2.jsonl): c = 403 / 687 cycles per k-block, E = 5600 / 8500
+// cycles (at BN 128 / 256; at these sizes the 128 x 256 tile is L2-fed, not MMA-bound).
+// Inside the step (PDL neighbours, the residual's L2 state) a split only paid off where the model
+// predicts a large gain on a long-K projection: slices are taken for K >= 8192 (down) when they
+// beat the best whole-tile choice by >= 15% (in-process A/B on the 32-layer step,
+// profiles/step_addsplit_r2c.jsonl: the O projection split and down at T = 512 were slower).
+void gemm_pick_add_split(int64_t M, int64_t N, int64_t K, int num_sms, int64_t max_tiles, int* bn_out, int* ks_out) {
+  const int64_t mt = (M + kBM - 1) / kBM, kblocks = K / kBK;
+  int64_t best = INT64_MAX, best1 = INT64_MAX;
+  int bn1 = 128, bns = 128, kss = 1;
+  for (int bn = 128; bn <= 256; bn += 128) {
+    if (bn == 256 && N % 256) continue;
+    const int64_t tiles = mt * ((N + bn - 1) / bn);
+    const int64_t ckb = bn == 256 ? 687 : 403, epi = bn == 256 ? 8500 : 5600;
+    for (int ks = 1; ks <= 4; ++ks) {
+      if (ks > 1 && (kblocks < 128 || kblocks / ks < 8 || tiles > max_tiles)) break;
+      const int64_t waves = (tiles * ks + num_sms - 1) / num_sms;
+      const int64_t cost = waves * ((kblocks + ks - 1) / ks) * ckb + int64_t(ks - 1) * epi;
+      if (ks == 1 && cost < best1) {
+        best1 = cost;
+        bn1 = bn;
+      }
+      if (cost < best) {
+        best = cost;
+        bns = bn;
+        kss = ks;
+      }
+    }
+  }
+  const bool split = kss > 1 && best * 100 <= best1 * 85;
+  *bn_out = split ? bns : bn1;
+  *ks_out = split ? kss : 1;
+}
+
 int gemm_pick_ksplit(int64_t M, int64_t N, int64_t K, int bn, int num_sms, int64_t max_units) {
   // weight-bound small-M GEMMs: split K until the units cover the SMs (>= 4 k-blocks each)
   const int64_t tiles = ((M + kBM - 1) / kBM) * ((N + bn - 1) / bn);
@@ -1221,7 +1300,7 @@ int gemm_pick_ksplit(int64_t M, int64_t N, int64_t K, int bn, int num_sms, int64
 int gemm_run(const CUtensorMap& ta, const CUtensorMap& tb, int bn, int64_t M, int64_t N, int64_t K, int epi, void* C,
              int64_t ldc, const float* bias, int num_sms, cudaStream_t st, int ksplit, float* part, int* counters,
              int a_row0, int max_ctas, const QkvRopeArgs* rope, int sk_mode, bool coop, const NormFold* fold) {
-  GemmArgs a;
+  GemmArgs a{};
   set_fold(a, fold);
   if (fold && ksplit > 1) return set_error(QOS_ERR_INVALID_ARG, "gemm: folded norm needs one pass");
   if (fold) sk_mode = 0;  // whole tiles only
@@ -1247,7 +1326,12 @@ int gemm_run(const CUtensorMap& ta, const CUtensorMap& tb, int bn, int64_t M, in
   a.hd = rope ? rope->hd : 0;
   if (epi == EPI_QKV_ROPE && (!rope || a.hd <= 0 || bn % a.hd))
     return set_error(QOS_ERR_INVALID_ARG, "gemm: QKV_ROPE needs rope args and BN % hd == 0");
-  if (a.ksplit > 1 && (!part || !counters)) return set_error(QOS_ERR_INVALID_ARG, "gemm: split-K needs workspace");
+  // EPI_ADD_F32 split-K accumulates in place in slice order (needs only the tile counters, and
+  // every CTA resident so a waiting slice cannot block the one it waits for)
+  a.ordered = (a.ksplit > 1 && epi == EPI_ADD_F32) ? 1 : 0;
+  if (a.ordered && !coop) return set_error(QOS_ERR_INVALID_ARG, "gemm: ordered split-K needs co-resident CTAs");
+  if (a.ksplit > 1 && (!counters || (!a.ordered && !part)))
+    return set_error(QOS_ERR_INVALID_ARG, "gemm: split-K needs workspace");
   const int tiles = a.mt * a.nt * a.ksplit;
   int grid = tiles < num_sms ? tiles : num_sms;
   if (max_ctas > 0 && grid > max_ctas) grid = max_ctas;   // SM budget (co-scheduled streams)

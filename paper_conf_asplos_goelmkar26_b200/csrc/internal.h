@@ -43,6 +43,8 @@ int make_tmap_3d_bf16_strided(CUtensorMap* out, const void* base, uint64_t d0, u
 int gemm_pick_bn(int64_t M, int64_t N, int epi, int num_sms);
 int gemm_check_shape(int64_t M, int64_t N, int64_t K, int epi);
 int gemm_pick_ksplit(int64_t M, int64_t N, int64_t K, int bn, int num_sms, int64_t max_units);
+// EPI_ADD_F32: tile width and ordered split-K slices (1 = whole tiles) by a wave cost model
+void gemm_pick_add_split(int64_t M, int64_t N, int64_t K, int num_sms, int64_t max_tiles, int* bn_out, int* ks_out);
 // ksplit > 1: split-K with fp32 partials in `part` ([units][128][bn]) and per-tile arrival
 // counters (zero-initialised; each reducing CTA resets its own) — deterministic reduction order
 // RMSNorm folded into the projections (single-pass tile kernels, no split-K / stream-K):

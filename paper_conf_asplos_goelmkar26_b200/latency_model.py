@@ -12,7 +12,9 @@ work and the engine's tiling:
 
 * Wgemm(T): sum over the projections run by the single-CTA tile kernel (csrc/gemm.cu) of (waves
   of 128 x BN tiles over the SMs) x (k-blocks per tile) x BN/256 — the tensor-core GEMM time
-  with the engine's tile-quantisation (same BN / split-K choice), T = sum(chunk_len) + n_decode;
+  with the engine's tile-quantisation (same BN choice), T = sum(chunk_len) + n_decode; the O
+  and down projections below the fold threshold enter with the cost of the engine's ordered
+  split-K choice (`add_split`, mirroring gemm_pick_add_split) in the same units;
 * Wpair(T): the same for the projections run by the CTA-pair kernel (256 x 256 tiles over 2
   SMs, same selection rule as gemm2_eligible): (waves of pair tiles over SMs/2) x k-blocks —
   a separate term because its per-k-block cost differs;
@@ -109,15 +111,43 @@ def pair_work(T: int, g: GemmShapes) -> float:
                      for N, K in g.gemms if T > 0 and pair_eligible(T, N, K, g.num_sms)))
 
 
-def gemm_work(T: int, g: GemmShapes) -> float:
+def add_split(M: int, N: int, K: int, sms: int, max_tiles: int = 4096):
+    """(BN, slices, cost in cycles) of an EPI_ADD_F32 projection; mirrors gemm_pick_add_split
+    (csrc/gemm.cu): waves x k-blocks per unit x c(BN) + (slices - 1) x E(BN)."""
+    mt, kb = (M + 127) // 128, K // 64
+    best = best1 = None
+    for bn in (128, 256):
+        if bn == 256 and N % 256:
+            continue
+        tiles = mt * ((N + bn - 1) // bn)
+        ckb, epi = (687, 8500) if bn == 256 else (403, 5600)
+        for ks in (1, 2, 3, 4):
+            if ks > 1 and (kb < 128 or kb // ks < 8 or tiles > max_tiles):
+                break
+            cost = -(-tiles * ks // sms) * (-(-kb // ks)) * ckb + (ks - 1) * epi
+            if ks == 1 and (best1 is None or cost < best1[2]):
+                best1 = (bn, 1, cost)
+            if best is None or cost < best[2]:
+                best = (bn, ks, cost)
+    return best if best[1] > 1 and best[2] * 100 <= best1[2] * 85 else best1
+
+
+# the projections with the residual-add epilogue (O and down): ordered split-K below the fold
+ADD_GEMMS = (1, 3)
+
+
+def gemm_work(T: int, g: GemmShapes, fold: bool = False) -> float:
     if T <= 0:
         return 0.0
     tot = 0.0
-    for N, K in g.gemms:
+    for i, (N, K) in enumerate(g.gemms):
         if swab_prefer_k(T, N, K, g.num_sms) or pair_eligible(T, N, K, g.num_sms):
             continue
+        if i in ADD_GEMMS and not fold:
+            tot += add_split(T, N, K, g.num_sms)[2] / 630.0
+            continue
         bn = _bn(T, N, g.num_sms)
-        tiles = ((T + 127) // 128) * ((N + bn - 1) // bn)   # no split-K (engine default gemm_splitk = 0)
+        tiles = ((T + 127) // 128) * ((N + bn - 1) // bn)   # whole tiles
         tot += math.ceil(tiles / g.num_sms) * (K // 64) * (bn / 256)
     return tot
 
@@ -131,7 +161,7 @@ def features(s: StepShape, g: GemmShapes = GemmShapes()) -> np.ndarray:
     n_pair = sum(1 for N, K in g.gemms if s.T > 0 and pair_eligible(s.T, N, K, g.num_sms))
     n_stream = sum(1 for N, K in g.gemms if s.T > 0 and swab_prefer_k(s.T, N, K, g.num_sms))
     fold = 1.0 if (s.T >= FOLD_MIN_TOKENS and n_stream == 0) else 0.0   # mirrors run_layers' norm fold
-    return np.array([gemm_work(s.T, g) / 100.0, s.T / 1000.0, sum(c + 1 for c in s.ctx) / 1e6, nd / 100.0,
+    return np.array([gemm_work(s.T, g, fold > 0) / 100.0, s.T / 1000.0, sum(c + 1 for c in s.ctx) / 1e6, nd / 100.0,
                      1.0 if nd else 0.0, 1.0, sum(n * (n + 1) / 2 for ks, n in s.chunks) / 1e7,
                      stream_work(s.T, g) / 1e8, sum(n * ks for ks, n in s.chunks) / 1e7, pair_work(s.T, g) / 100.0,
                      float(n_pair), float(len(g.gemms) - n_pair - n_stream), fold, fold * s.T / 1000.0])

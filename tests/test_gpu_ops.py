@@ -278,6 +278,33 @@ def test_gemm_splitk_parity(torch_cuda, M, N, K, ks, epi):
         assert row_rel_err(got, ref) <= tol
 
 
+@pytest.mark.parametrize("M,N,K,ks", [(512, 4096, 4096, 2), (288, 4096, 14336, 3), (1000, 4096, 2048, 3),
+                                      (777, 1280, 2048, 4), (512, 4096, 14336, 0), (640, 4096, 4096, 0)])
+def test_gemm_ordered_split_add_parity(torch_cuda, M, N, K, ks):
+    """Ordered in-place split-K of EPI_ADD_F32 (the O / down projections of mid-size steps):
+    every K slice red.adds its fp32 partial into C after the previous slice of its tile, so the
+    result is deterministic (bit-identical run to run) and within fp32 rounding of the fp64
+    product; 768 units at (1000, 4096, 2048, 3) exercise several units per CTA and slices
+    waiting on other CTAs; ks = 0 is the engine's automatic (tile width, slices) choice."""
+    torch = torch_cuda
+    from paper_conf_asplos_goelmkar26_b200 import qoserve as q
+    rng = np.random.default_rng(M + N + K + ks)
+    A = bits_to_f64(bf16_bits(rng.uniform(-1, 1, (M, K))))
+    B = bits_to_f64(bf16_bits(rng.uniform(-1, 1, (N, K)) / np.sqrt(K)))
+    dA, dB = _dev_bf16(torch, A), _dev_bf16(torch, B)
+    init = rng.uniform(-1, 1, (M, N)).astype(np.float32)
+    ref = A @ B.T + init.astype(np.float64)
+    dC = torch.from_numpy(init.copy()).cuda()
+    outs = []
+    for _ in range(3):   # the tile counters must be back at 0 after every launch
+        dC.copy_(torch.from_numpy(init.copy()).cuda())
+        q.qos_op_gemm_ex(dA.data_ptr(), dB.data_ptr(), dC.data_ptr(), M, N, K, "add_f32", None, ks)
+        torch.cuda.synchronize()
+        outs.append(dC.cpu().numpy().copy())
+    assert row_rel_err(outs[0], ref) <= 1e-5
+    assert np.array_equal(outs[0], outs[1]) and np.array_equal(outs[0], outs[2])
+
+
 @pytest.mark.parametrize("M,N,K", [(1, 256, 64), (77, 512, 320), (300, 768, 128), (1000, 4096, 512),
                                    (2176, 1024, 1024), (4100, 512, 256)])
 @pytest.mark.parametrize("epi", ["store_f32", "store_bf16", "add_f32", "bias_bf16", "silu_gate"])
