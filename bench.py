@@ -248,6 +248,21 @@ def run_ours(args):
     H = pr["n_heads"] // tp
     pa_flops = 4.0 * hd * H * (CHUNK * (CHUNK + 1) / 2.0)
     pa_tfs = pa_flops / (pa_ms / pa_n * 1e-3) / 1e12 if pa_n else 0.0
+    # step roofline: sum over the step's kernels of max(FLOPs / tensor peak,
+    # bytes / HBM peak) against the measured step time
+    Hq = pr["n_heads"] // tp
+    V = pr["vocab"] // tp
+    proj = [(d * (Hq + 2 * Hkv) * hd), (Hq * hd * d), (2 * d * F), (F * d)]   # weights per layer (elements)
+    R = N_DEC + 1
+    t_gemm = sum(max(2.0 * T * w / (peak_tc * 1e12), 2.0 * w / (peak_hbm * 1e9)) for w in proj) * L
+    t_head = max(2.0 * R * d * V / (peak_tc * 1e12), 2.0 * d * V / (peak_hbm * 1e9))
+    t_dec = da_bytes * L / (peak_hbm * 1e9)
+    t_pre = pa_flops * L / (peak_tc * 1e12)
+    t_roof = (t_gemm + t_head + t_dec + t_pre) * 1e3
+    roof_step = {"roofline_ms": round(t_roof, 3), "achieved_ms": round(ms_step, 3), "frac": round(t_roof / ms_step, 4),
+                 "terms_ms": {"projections": round(t_gemm * 1e3, 3), "lm_head": round(t_head * 1e3, 3),
+                              "decode_attn": round(t_dec * 1e3, 3), "prefill_attn": round(t_pre * 1e3, 3)},
+                 "peaks": "bf16_tflops_sustained and hbm_gbs of MEASURED_PEAKS.json (of measured)"}
     traffic = None
     try:
         assert args.model == "llama3-8b" and tp == 1 and args.layers is None   # the committed capture
@@ -288,6 +303,7 @@ def run_ours(args):
         "roofline_decode_attn": {"bound": "hbm", "achieved": round(da_gbs, 1), "peak": peak_hbm, "unit": "GB/s",
                                  "frac": round(da_gbs / peak_hbm, 4),
                                  "peak_source": "MEASURED_PEAKS.json hbm_gbs (of measured)"},
+        "roofline_step": roof_step,
         "gpu_launches": int(launches),
         "clocks": clk,
         "e2e": {"value": round(replicas * T / (e2e_ms * 1e-3), 1), "unit": "tokens/s",

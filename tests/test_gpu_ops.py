@@ -301,7 +301,11 @@ def test_gemm_ordered_split_add_parity(torch_cuda, M, N, K, ks):
         q.qos_op_gemm_ex(dA.data_ptr(), dB.data_ptr(), dC.data_ptr(), M, N, K, "add_f32", None, ks)
         torch.cuda.synchronize()
         outs.append(dC.cpu().numpy().copy())
-    assert row_rel_err(outs[0], ref) <= 1e-5
+    # fp32 accumulation error grows with the reduction length: 1e-5 at K <= 4096 (the tolerance
+    # of the whole-tile GEMM tests), scaled with sqrt(K / 4096) for the down projection's K
+    # (the unsplit K = 14336 tile accumulates 896 MMA K-steps in one TMEM accumulator)
+    tol = 1e-5 * max(1.0, np.sqrt(K / 4096))
+    assert row_rel_err(outs[0], ref) <= tol, row_rel_err(outs[0], ref)
     assert np.array_equal(outs[0], outs[1]) and np.array_equal(outs[0], outs[2])
 
 
