@@ -32,6 +32,10 @@ sys.path.insert(0, ROOT)
 
 CHUNK, N_DEC, CTX = 2048, 128, 4096
 WORKLOAD = f"llama3-8b hybrid step: chunk {CHUNK} @kv_start 0 + {N_DEC} decodes @ctx {CTX}"
+# --workload: the headline hybrid step (configs[1]'s point above), or the prefill-node step of a
+# PD-disaggregated deployment (one 8192-token chunk, no decodes: §4.1.3,
+# SURVEY.md §8(f) NEXT-4)
+WORKLOADS = {"hybrid": (CHUNK, N_DEC, CTX), "pd-prefill": (8192, 0, 0)}
 
 
 def _peaks():
@@ -170,12 +174,14 @@ def run_ours(args):
         box = [qq.qos_group_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(box, src=0)
         group = qq.Group(tp, box[0], rank)
-    wl = Workload(local, W + 3 * K + 2, model=args.model, n_layers=args.layers, tp=tp, rank=rank, group=group)
+    chunk, n_dec, ctx = WORKLOADS[args.workload]
+    wl = Workload(local, W + 3 * K + 2, chunk=chunk, n_dec=n_dec, ctx=ctx, model=args.model, n_layers=args.layers,
+                  tp=tp, rank=rank, group=group)
     q, eng, T = wl.q, wl.eng, wl.tokens_per_step
     replicas = ws // tp
     stream = torch.cuda.current_stream()
     sptr = stream.cuda_stream
-    out_tok = torch.empty(N_DEC + 1, dtype=torch.int32, device="cuda")
+    out_tok = torch.empty(n_dec + 1, dtype=torch.int32, device="cuda")
     # -------- warm-up
     for _ in range(W):
         wl.step(wl.next_batch(), out_tok.data_ptr(), False, sptr)
@@ -216,7 +222,7 @@ def run_ours(args):
     eng.qos_engine_set_option("overlap_attn", 1)
     # -------- e2e: through the public API with host buffers (descriptor in, tokens out)
     batches = [wl.next_batch() for _ in range(K)]
-    host_tok = np.empty(N_DEC + 1, dtype=np.int32)
+    host_tok = np.empty(n_dec + 1, dtype=np.int32)
     torch.cuda.synchronize()
     t0 = time.perf_counter()
     for b in batches:
@@ -236,24 +242,24 @@ def run_ours(args):
     gu_flops = 2.0 * T * d * (2 * F)                    # algorithmic FLOPs per launch (one layer)
     gu_tfs = gu_flops / (gu_ms / gu_n * 1e-3) / 1e12
     peak_tc = peaks.get("bf16_tflops_sustained") or 1400.0
-    da_ms, da_n = per_class["decode_attn"]
+    da_ms, da_n = per_class.get("decode_attn", (0.0, 0))
     # decode attention: K+V bytes of every decode's (ctx+1) keys per layer;
     # the instrumented pass ran after warm-up + one timed pass, contexts grew 1 token per step
-    mean_ctx = CTX + W + K + (K - 1) / 2.0
-    da_bytes = 4.0 * hd * Hkv * N_DEC * (mean_ctx + 1)
-    da_gbs = da_bytes / (da_ms / da_n * 1e-3) / 1e9
+    mean_ctx = ctx + W + K + (K - 1) / 2.0
+    da_bytes = 4.0 * hd * Hkv * n_dec * (mean_ctx + 1)
+    da_gbs = da_bytes / (da_ms / da_n * 1e-3) / 1e9 if da_n else 0.0
     peak_hbm = peaks.get("hbm_gbs") or 6650.0
     # prefill attention (a7): causal FLOPs of the chunk per layer, chunk at kv_start 0
     pa_ms, pa_n = per_class.get("prefill_attn", (0.0, 0))
     H = pr["n_heads"] // tp
-    pa_flops = 4.0 * hd * H * (CHUNK * (CHUNK + 1) / 2.0)
+    pa_flops = 4.0 * hd * H * (chunk * (chunk + 1) / 2.0)
     pa_tfs = pa_flops / (pa_ms / pa_n * 1e-3) / 1e12 if pa_n else 0.0
     # step roofline: sum over the step's kernels of max(FLOPs / tensor peak,
     # bytes / HBM peak) against the measured step time
     Hq = pr["n_heads"] // tp
     V = pr["vocab"] // tp
     proj = [(d * (Hq + 2 * Hkv) * hd), (Hq * hd * d), (2 * d * F), (F * d)]   # weights per layer (elements)
-    R = N_DEC + 1
+    R = n_dec + 1
     t_gemm = sum(max(2.0 * T * w / (peak_tc * 1e12), 2.0 * w / (peak_hbm * 1e9)) for w in proj) * L
     t_head = max(2.0 * R * d * V / (peak_tc * 1e12), 2.0 * d * V / (peak_hbm * 1e9))
     t_dec = da_bytes * L / (peak_hbm * 1e9)
@@ -265,14 +271,15 @@ def run_ours(args):
                  "peaks": "bf16_tflops_sustained and hbm_gbs of MEASURED_PEAKS.json (of measured)"}
     traffic = None
     try:
-        assert args.model == "llama3-8b" and tp == 1 and args.layers is None   # the committed capture
+        assert args.model == "llama3-8b" and tp == 1 and args.layers is None and args.workload == "hybrid"
         prof = json.load(open(os.path.join(ROOT, "profiles", "roofline_traffic.json")))
         traffic = prof.get("gemm_gateup", {}).get("dram_bytes_per_launch")
     except Exception:
         pass
     tag = args.model + (f" TP{tp}" if tp > 1 else "")
     rec = {
-        "metric": f"hybrid-step tokens/s ({tag}, chunk 2048 + 128 decodes @4k)",
+        "metric": (f"hybrid-step tokens/s ({tag}, chunk 2048 + 128 decodes @4k)" if args.workload == "hybrid" else
+                   f"prefill-node step tokens/s ({tag}, chunk 8192, no decodes)"),
         "value": round(replicas * T / (ms_step * 1e-3), 1),
         "unit": "tokens/s",
         "n_gpus": ws, "steps": K, "warmup": W,
@@ -282,12 +289,14 @@ def run_ours(args):
         "vs_baseline": None,
         "dtype": "bf16",
         "data": "synthetic (seeded weights + synthetic KV prefixes; DESIGN.md §3)",
-        "config": {"workload": WORKLOAD.replace("llama3-8b", tag),
-                   "model": f"{args.model} ({L} layers, random-init)", "chunk_len": CHUNK,
-                   "n_decode": N_DEC, "ctx": CTX, "tokens_per_step": T,
+        "config": {"workload": (WORKLOAD.replace("llama3-8b", tag) if args.workload == "hybrid" else
+                                f"{tag} PD-disaggregated prefill-node step: chunk {chunk} @kv_start 0, no decodes"),
+                   "model": f"{args.model} ({L} layers, random-init)", "chunk_len": chunk,
+                   "n_decode": n_dec, "ctx": ctx, "tokens_per_step": T,
                    "parallelism": f"replicas{ws}" if tp == 1 else f"tp{tp} (peer-memory collectives)",
                    "l2": ("inputs larger than L2 (16 GB weights + 69 GB KV streamed per step)" if tp == 1 and
-                          args.model == "llama3-8b" and args.layers is None else
+                          args.model == "llama3-8b" and args.layers is None and n_dec else
+                          "inputs larger than L2 (16 GB of weights streamed per step)" if not n_dec else
                           "inputs larger than L2 (weight shard + KV of 128 x 4k contexts streamed per step)")},
         "latency_ms": {"median": round(statistics.median(steps_ms), 4), "min": round(min(steps_ms), 4),
                        "max": round(max(steps_ms), 4), "instrumented_pass_serial_attention": round(ms_instr, 4)},
@@ -298,11 +307,10 @@ def run_ours(args):
                      "peak_source": "MEASURED_PEAKS.json bf16_tflops_sustained (of measured)"},
         "roofline_prefill_attn": {"bound": "tensor", "achieved": round(pa_tfs, 1), "peak": peak_tc, "unit": "TFLOP/s",
                                   "frac": round(pa_tfs / peak_tc, 4) if peak_tc else None,
-                                  "note": "2048-token causal chunk from position 0 (short key ranges); "
-                                          "longer contexts reach higher fractions (DESIGN.md §6)"},
-        "roofline_decode_attn": {"bound": "hbm", "achieved": round(da_gbs, 1), "peak": peak_hbm, "unit": "GB/s",
-                                 "frac": round(da_gbs / peak_hbm, 4),
-                                 "peak_source": "MEASURED_PEAKS.json hbm_gbs (of measured)"},
+                                  "note": f"{chunk}-token causal chunk from position 0"},
+        "roofline_decode_attn": ({"bound": "hbm", "achieved": round(da_gbs, 1), "peak": peak_hbm, "unit": "GB/s",
+                                  "frac": round(da_gbs / peak_hbm, 4),
+                                  "peak_source": "MEASURED_PEAKS.json hbm_gbs (of measured)"} if n_dec else None),
         "roofline_step": roof_step,
         "gpu_launches": int(launches),
         "clocks": clk,
@@ -311,7 +319,8 @@ def run_ours(args):
                 "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
                 "how": "qos_hybrid_step with host descriptor and host next_tokens (outputs_on_host=1), wall clock"},
     }
-    if rank == 0 and not args.no_cpu_baseline and tp == 1 and args.model == "llama3-8b" and args.layers is None:
+    if (rank == 0 and not args.no_cpu_baseline and tp == 1 and args.model == "llama3-8b" and args.layers is None
+            and args.workload == "hybrid"):
         rec["cpu_baseline"] = cpu_baseline()
     eng.close()
     if group is not None:
@@ -425,6 +434,8 @@ def main():
     ap.add_argument("--tp", type=int, default=1, help="tensor-parallel degree (= WORLD_SIZE under torchrun)")
     ap.add_argument("--model", default="llama3-8b", help="llama3-8b | qwen2.5-14b | llama3-70b")
     ap.add_argument("--layers", type=int, default=None, help="fewer layers (smoke runs only)")
+    ap.add_argument("--workload", default="hybrid", choices=sorted(WORKLOADS),
+                    help="hybrid: the headline step; pd-prefill: the 8192-token prefill-node step (NEXT-4)")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "ours":
         args.warmup = 3

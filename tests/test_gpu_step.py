@@ -283,6 +283,51 @@ def test_execution_options_do_not_change_results(opts):
     eng.close()
 
 
+@pytest.mark.slow
+@pytest.mark.parametrize("add_split", [1, 0])
+def test_llama8b_mid_t_step_parity(add_split):
+    """Mid-size step at full Llama-3-8B width (2 layers): a 512-token chunk at kv_start 0 + 128
+    decodes @ ctx 1024 (T = 640).  The down projection (K = 14336) runs the ordered in-place
+    split-K of the tile kernel here (3 K slices of 128 x 256 tiles, round 2); add_split = 0 is
+    the whole-tile path.  Sampled rows vs the oracle within 1e-2, and the split step is
+    bit-identical when repeated (slice order fixed)."""
+    C, ND, CTX = 512, 128, 1024
+    q, cfg, eng = make_engine("llama3-8b", n_layers=2, num_blocks=(2 * C + ND * (CTX + 2)) // 16 + 400,
+                              max_seq_len=4096, max_batch_tokens=C + ND, max_batch_rows=ND + 1,
+                              max_requests=ND + 8)
+    eng.qos_engine_load_synthetic(0)
+    eng.qos_engine_set_option("add_split", add_split)
+    b = synth.hybrid_batch(cfg.vocab, C, ND, CTX)
+    for d in b.decode:
+        eng.qos_kv_alloc(d.req, CTX + 1)
+        eng.qos_kv_fill_synthetic(d.req, CTX, synth.SEED_KVFILL)
+    outs = []
+    for rep in range(2):   # the same step twice on fresh chunk requests (decode KV rewritten in place)
+        b.prefill[0].req = 1000 + rep
+        eng.qos_kv_alloc(1000 + rep, C)
+        lg, _ = eng.step_host(q.batch_from_synth(b), cfg.vocab)
+        outs.append(lg)
+        for d in b.decode:   # rewind the decodes: their position-CTX entries are rewritten next time
+            eng.qos_kv_free(d.req)
+            eng.qos_kv_alloc(d.req, CTX + 1)
+            eng.qos_kv_fill_synthetic(d.req, CTX, synth.SEED_KVFILL)
+    assert np.array_equal(outs[0][1:], outs[1][1:])
+    orc = _oracle("llama3-8b", n_layers=2, num_blocks=C // 16 + 4 + 4 * (CTX // 16 + 2))
+    sample = [0, 77, 127]
+    orc.kv_alloc(0, C)
+    pre = [(0, 0, [int(t) for t in b.prefill[0].tokens])]
+    decs = []
+    for j in sample:
+        d = b.decode[j]
+        orc.kv_alloc(d.req, CTX + 1)
+        orc.kv_fill_synthetic(d.req, CTX, synth.SEED_KVFILL)
+        decs.append((d.req, d.ctx_len, d.token))
+    ref = orc.hybrid_step(pre, decs)
+    got = np.concatenate([outs[0][:1], outs[0][[1 + j for j in sample]]])
+    assert row_rel_err(got, ref) <= TOL_LOGITS, row_rel_err(got, ref)
+    eng.close()
+
+
 def test_long_context_step_parity():
     """Maximum context (configs[3]: up to 32k): a 100-token chunk at kv_start 16000 and decodes
     at ctx 32767 / 20000 / 17, all prefixes synthetic KV, through qos_hybrid_step vs the oracle
