@@ -771,10 +771,11 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
       int pend[2], npend = 0;
       auto slot_of = [&](int t, int cc) { return rstart(cc) >= int64_t(t) * kblocks ? 2 * cc : 2 * cc + 1; };
       auto red32 = [&](int t, int cf, int cl) {
+        const bool ok = (t % p.mt) * kBM + rit < p.M;  // partials of rows past M were never written
         return [=](int col, float (&v)[32]) {
 #pragma unroll
           for (int i = 0; i < 32; ++i) v[i] = 0.f;
-          for (int cc = cf; cc <= cl; ++cc) {  // CTA order: deterministic
+          for (int cc = cf; ok && cc <= cl; ++cc) {  // CTA order: deterministic
             const float4* pr = reinterpret_cast<const float4*>(p.part + (size_t(slot_of(t, cc)) * kBM + rit) * BN + col);
             float4 x[8];
 #pragma unroll
@@ -790,10 +791,11 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
         };
       };
       auto red16 = [&](int t, int cf, int cl, int n_t) {
+        const bool ok = (t % p.mt) * kBM + rit < p.M;
         return [=](int col, float (&v)[16]) {
 #pragma unroll
           for (int i = 0; i < 16; ++i) v[i] = p.bias ? __ldg(p.bias + n_t * BN + col + i) : 0.f;
-          for (int cc = cf; cc <= cl; ++cc) {
+          for (int cc = cf; ok && cc <= cl; ++cc) {
             const float4* pr = reinterpret_cast<const float4*>(p.part + (size_t(slot_of(t, cc)) * kBM + rit) * BN + col);
             float4 x[4];
 #pragma unroll
