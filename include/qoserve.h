@@ -282,6 +282,16 @@ int qos_profile_step_ex(qos_engine_t* eng, int32_t chunk_len, int32_t kv_start,
  *                          (0: one CTA per work item)
  *   "gemm_2cta" (1)        CTA-pair GEMM (tcgen05 cta_group::2, 256 x 256 tiles) where it
  *                          needs no more waves than 128 x 256 single-CTA tiles; env QOS_GEMM_2CTA
+ *   "add_split" (1)        ordered in-place split-K of the residual-add projections below the
+ *                          norm-fold threshold (down projection at mid T; slices add in a fixed
+ *                          order, so results stay deterministic); env QOS_ADD_SPLIT
+ *   "gemm_sms" (0)         SM budget of the step's GEMM grids (0 = all; experiments)
+ *   "shares_device" (0)    1: another engine may run kernels concurrently on this GPU (e.g. two
+ *                          engines on two streams of one process).  Switches off the GEMM paths
+ *                          that need every CTA of a grid resident at once (the weight-streaming
+ *                          kernel's cooperative reduction, the ordered split-K): two such grids
+ *                          sharing the SMs could each wait on CTAs the other keeps out.  Set
+ *                          automatically for peer-group ranks on one device.
  * Results do not depend on the options (parity tests run with the defaults and variants). */
 int qos_engine_set_option(qos_engine_t* eng, const char* name, int64_t value);
 

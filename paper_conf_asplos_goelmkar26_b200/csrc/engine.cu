@@ -1934,6 +1934,7 @@ int qos_engine_set_option(qos_engine_t* e, const char* name, int64_t value) {
   else if (n == "dual_sms_prefill") e->dual_sms_pre = int(value);
   else if (n == "dual_sms_decode") e->dual_sms_dec = int(value);
   else if (n == "add_split") e->add_split = value != 0;
+  else if (n == "shares_device") e->shares_device = value != 0 || (e->group && e->shares_device);
   else if (n == "gemm_sms") e->gemm_sms = int(value < 0 ? 0 : value > e->num_sms ? e->num_sms : value);
   else return set_error(QOS_ERR_INVALID_ARG, "unknown option");
   return QOS_OK;

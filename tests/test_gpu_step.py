@@ -255,7 +255,7 @@ def test_llama8b_shapes_bench_batch_sampled_parity(split):
                                   {"norm_fold": 0}, {"gemm_swab": 0, "norm_fold": 1}, {"attn_order": 1}, {"gemm_swab": 0, "gemm_2cta": 0}, {"decode_stages": 4},
                                   {"decode_split": 64}, {"decode_split": 4096},
                                   {"dual_stream": 1, "dual_min_prefill": 1, "dual_min_decode": 1},
-                                  {"add_split": 0}])
+                                  {"add_split": 0}, {"shares_device": 1}])
 def test_execution_options_do_not_change_results(opts):
     """qos_engine_set_option variants (serial attention, no split-K, two-stream sub-batches)
     stay within tolerance of the oracle and give the same greedy tokens."""

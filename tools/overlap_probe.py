@@ -70,7 +70,7 @@ def mk(n_dec, chunk):
                       max_batch_tokens=chunk + n_dec + 2, max_batch_rows=n_dec + 2)
     e = q.Engine(cfg)
     e.qos_engine_load_synthetic(synth.SEED_WEIGHTS)
-    e.qos_engine_set_option("dual_stream", 1)   # cooperative GEMM reductions off (two engines share the GPU)
+    e.qos_engine_set_option("shares_device", 1)   # no co-residency-dependent GEMM paths (two engines, one GPU)
     return cfg, e
 
 

@@ -35,7 +35,8 @@ def main():
     ap.add_argument("--alpha", type=float, default=8.0)
     ap.add_argument("--max-chunk", type=int, default=4096)
     ap.add_argument("--out", default=None)
-    ap.add_argument("--replicas", type=int, default=1, help="model mode: round-robin TP1 replicas (1 per GPU)")
+    ap.add_argument("--replicas", type=int, default=1,
+                    help="round-robin TP1 replicas (1 per GPU); engine mode replays them one after another")
     a = ap.parse_args()
     results = []
     eng = None
@@ -77,7 +78,13 @@ def main():
             return QoServeScheduler(SchedulerConfig(alpha_ms_per_token=a.alpha, max_chunk=a.max_chunk,
                                                     max_decodes=256, max_rows=257,
                                                     max_tokens=a.max_chunk + 512), pred)
-        if a.mode == "engine":
+        if a.mode == "engine" and a.replicas > 1:
+            # round-robin replicas replayed one after another on the one GPU (replicas share
+            # nothing; each runs its share of the trace on its own virtual clock)
+            out = replay_replicas(tr, a.replicas, mk_sched,
+                                  lambda: EngineExecutor(eng, 128256,
+                                                         lambda r, s, n: synth.request_tokens(r, n, 128256, start=s)))
+        elif a.mode == "engine":
             ex = EngineExecutor(eng, 128256, lambda r, s, n: synth.request_tokens(r, n, 128256, start=s))
             out = replay(tr, mk_sched(), ex)
         elif a.replicas > 1:
