@@ -122,6 +122,16 @@ def test_step_errors_leave_state_unchanged():
     with pytest.raises(q.QosError) as ei:
         eng.step_host(q.make_batch([(1, 0, np.array([cfg.vocab], np.int32))], []), cfg.vocab)
     assert ei.value.name == "INVALID_ARG"
+    with pytest.raises(q.QosError) as ei:
+        eng.step_host(q.make_batch([], []), cfg.vocab)                       # empty batch
+    assert ei.value.name == "INVALID_ARG"
+    with pytest.raises(q.QosError) as ei:                                    # a request twice in one step
+        eng.step_host(q.make_batch([(1, 0, np.zeros(3, np.int32))], [(1, 0, 1)]), cfg.vocab)
+    assert ei.value.name == "INVALID_ARG"
+    with pytest.raises(q.QosError) as ei:                                    # rows > max_batch_rows (32)
+        eng.step_host(q.make_batch([(1, 0, np.zeros(1, np.int32))], [(1000 + i, 0, 1) for i in range(32)]),
+                      cfg.vocab)
+    assert ei.value.name == "INVALID_ARG"
     assert eng.qos_kv_cached_len(1) == 0
     free = eng.qos_kv_free_blocks()
     with pytest.raises(q.QosError) as ei:
