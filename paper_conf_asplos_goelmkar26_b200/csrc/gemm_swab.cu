@@ -416,9 +416,13 @@ bool swab_prefer(int64_t M, int64_t N, int num_sms) {
   // B200 measurements (tools/gemm_bench.py, profiles/gemm_small_m_r1.md): the weight-streaming
   // kernel wins at very small T, and up to T = 256 when the tile kernel would leave most SMs
   // idle (few 128-wide output tiles: the O and down projections, N = d)
+  // Round 2, measured inside the 32-layer step (profiles/step_swab_r2a.jsonl): taking it for
+  // every projection up to T = 64 (the QKV and gate/up projections went to the tile kernel from
+  // T = 17 / 33) makes decode-heavy steps 5-13% faster; at T = 96-112 it is 2% slower.
+  // (Isolated op timings mislead here: an op's A tensor has exactly M rows, so the tile kernel's
+  // 128-row boxes read out of bounds, which the engine's workspace-wide maps never do.)
   if (N % 128) return false;
-  if (M <= 16) return true;
-  if (M <= 32 && N / 128 < num_sms) return true;
+  if (M <= 64) return true;
   if (M > 256) return false;
   const int64_t tiles = ((M + 127) / 128) * (N / 128);
   return tiles * 4 < num_sms;

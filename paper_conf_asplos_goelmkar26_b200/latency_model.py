@@ -79,9 +79,7 @@ def _bn(M: int, N: int, sms: int) -> int:      # mirrors gemm_pick_bn (csrc/gemm
 def swab_prefer(M: int, N: int, sms: int) -> bool:   # mirrors swab_prefer (csrc/gemm_swab.cu)
     if N % 128:
         return False
-    if M <= 16:
-        return True
-    if M <= 32 and N // 128 < sms:
+    if M <= 64:
         return True
     if M > 256:
         return False

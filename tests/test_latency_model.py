@@ -55,8 +55,10 @@ def test_small_steps_use_the_weight_streaming_gemm():
     g = GemmShapes()
     assert stream_work(1, g) == sum(n * k for n, k in g.gemms)        # every projection streams
     assert stream_work(2176, g) == 0 and gemm_work(1, g) == 0
-    # T = 64: only the O and down projections (32 output tiles) take the streaming kernel
-    assert stream_work(64, g) == 4096 * 4096 + 4096 * 14336
+    # up to T = 64 every projection streams (round-2 rule, csrc/gemm_swab.cu: swab_prefer)
+    assert stream_work(64, g) == sum(n * k for n, k in g.gemms)
+    # T = 128: only the O and down projections (32 output tiles) take the streaming kernel
+    assert stream_work(128, g) == 4096 * 4096 + 4096 * 14336
 
 
 def test_committed_profile_predictability():
