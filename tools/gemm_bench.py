@@ -8,6 +8,12 @@ to the next kernel and hides the small-M behaviour).
 
   python tools/gemm_bench.py [--ms 1,16,64,128,256,512,2176] [--ksplit 0] [--shapes qkv,o]
   ksplit: 0 auto, >= 1 tile kernel with that split-K, -1 weight-streaming (swap-AB) kernel
+
+Caveat (round 2): the op entry point maps A with exactly M rows, so at M not a multiple of 128
+the tile kernels' 128-row A boxes read out of bounds (TMA zero fill), which is measurably slower
+(gate/up: 62 us at M = 112 vs 48 us at M = 128).  Inside the engine the activation maps span the
+whole workspace and never go out of bounds — confirm kernel choices with an in-step A/B
+(tools/attn_bench.py --step-only --variants ...), as profiles/step_swab_r2a.jsonl did.
 """
 import argparse
 import json
