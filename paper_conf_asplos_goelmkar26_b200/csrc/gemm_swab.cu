@@ -428,11 +428,13 @@ bool swab_prefer(int64_t M, int64_t N, int num_sms) {
   return tiles * 4 < num_sms;
 }
 // with K: long-K projections (the down projection, K = F) stream more weight bytes per output
-// tile, so the weight-streaming kernel keeps winning up to twice as many tiles (T <= 256 at
-// N = d: 39 vs 51 us at T = 256, tools/gemm_bench.py r1e)
+// tile, so the weight-streaming kernel keeps winning up to twice as many tiles — up to T = 128
+// (round 2, in-step A/B, profiles/step_swab_r2c.jsonl: at T = 96-128 it is 2% faster, at
+// T = 160-256 the tile kernel is 0.4-4% faster; the round-1 bound of 256 came from isolated
+// timings with out-of-bounds A boxes)
 bool swab_prefer_k(int64_t M, int64_t N, int64_t K, int num_sms) {
   if (swab_prefer(M, N, num_sms)) return true;
-  if (N % 128 || M > 256 || K < 8192) return false;
+  if (N % 128 || M > 128 || K < 8192) return false;
   return ((M + 127) / 128) * (N / 128) * 2 < num_sms;
 }
 

@@ -89,7 +89,7 @@ def swab_prefer(M: int, N: int, sms: int) -> bool:   # mirrors swab_prefer (csrc
 def swab_prefer_k(M: int, N: int, K: int, sms: int) -> bool:   # mirrors swab_prefer_k (csrc/gemm_swab.cu)
     if swab_prefer(M, N, sms):
         return True
-    if N % 128 or M > 256 or K < 8192:
+    if N % 128 or M > 128 or K < 8192:
         return False
     return ((M + 127) // 128) * (N // 128) * 2 < sms
 
