@@ -286,6 +286,9 @@ int qos_profile_step_ex(qos_engine_t* eng, int32_t chunk_len, int32_t kv_start,
  *                          norm-fold threshold (down projection at mid T; slices add in a fixed
  *                          order, so results stay deterministic); env QOS_ADD_SPLIT
  *   "gemm_sms" (0)         SM budget of the step's GEMM grids (0 = all; experiments)
+ *   "gemm_bn" (0)          force the tile width (128 / 256) of the QKV and gate/up tile GEMMs
+ *                          (0 = the wave-cost choice; experiments: in-step A/B in
+ *                          profiles/step_bn_r2a.jsonl found the automatic choice best)
  *   "shares_device" (0)    1: another engine may run kernels concurrently on this GPU (e.g. two
  *                          engines on two streams of one process).  Switches off the GEMM paths
  *                          that need every CTA of a grid resident at once (the weight-streaming

@@ -371,6 +371,8 @@ struct qos_engine {
   int dual_sms_pre = 0, dual_sms_dec = 0;  // SM budgets of the two streams' GEMMs (0 = all)
   int gemm_sms = 0;                // option gemm_sms: SM budget of the fused step's GEMMs (0 = all)
   bool add_split = true;           // option add_split: ordered split-K of the O / down projections
+  int gemm_bn = 0;                 // option gemm_bn (experiments): force the tile width of the
+                                   // non-residual tile GEMMs (QKV, gate/up): 0 auto, 128, 256
   bool gemm_2cta = true;            // option gemm_2cta: CTA-pair GEMM (256 x 256 tiles) at large M
   bool decode_round_split = true;  // option decode_round_split (A/B of the split-K ranges)
   int decode_split = 4096;         // option decode_split: longest split-K key range tried first
@@ -796,6 +798,7 @@ int gemm_any(qos_engine* e, const qos_engine::ActMap& am, const CUtensorMap (&tb
   if (e->gemm_2cta && gemm2_eligible(M, N, K, sms))
     return gemm2_run(am.m128, tb[0], M, N, K, epi, C, ldc, bias, sms, st, a_row0, sms, rope, fold);
   int bn = gemm_pick_bn(M, N, epi, sms);
+  if (e->gemm_bn && epi != EPI_ADD_F32 && (e->gemm_bn == 128 || N % 256 == 0)) bn = e->gemm_bn;  // experiments
   int ks = e->gemm_splitk ? gemm_pick_ksplit(M, N, K, bn, sms, kGemmMaxUnits) : 1;
   const bool coop = !e->dual_stream && !e->shares_device;
   // O / down below the fold threshold: tile width + ordered in-place split-K by wave cost
@@ -1934,6 +1937,7 @@ int qos_engine_set_option(qos_engine_t* e, const char* name, int64_t value) {
   else if (n == "dual_sms_prefill") e->dual_sms_pre = int(value);
   else if (n == "dual_sms_decode") e->dual_sms_dec = int(value);
   else if (n == "add_split") e->add_split = value != 0;
+  else if (n == "gemm_bn") e->gemm_bn = (value == 128 || value == 256) ? int(value) : 0;
   else if (n == "shares_device") e->shares_device = value != 0 || (e->group && e->shares_device);
   else if (n == "gemm_sms") e->gemm_sms = int(value < 0 ? 0 : value > e->num_sms ? e->num_sms : value);
   else return set_error(QOS_ERR_INVALID_ARG, "unknown option");
