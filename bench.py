@@ -176,7 +176,7 @@ def run_ours(args):
         group = qq.Group(tp, box[0], rank)
     chunk, n_dec, ctx = WORKLOADS[args.workload]
     wl = Workload(local, W + 3 * K + 2, chunk=chunk, n_dec=n_dec, ctx=ctx, model=args.model, n_layers=args.layers,
-                  tp=tp, rank=rank, group=group)
+                  tp=tp, rank=rank % tp, group=group)
     q, eng, T = wl.q, wl.eng, wl.tokens_per_step
     replicas = ws // tp
     stream = torch.cuda.current_stream()
@@ -398,6 +398,14 @@ def run_reference(args):
     ws, rank, local = _dist()
     if rank != 0:
         return
+    if ws > 1:
+        # torchrun sets OMP_NUM_THREADS=1 for multi-process jobs; the oracle's rank runs alone, so
+        # give its BLAS the host's cores as in the single-process run
+        try:
+            from threadpoolctl import threadpool_limits
+            threadpool_limits(limits=os.cpu_count(), user_api="blas")
+        except Exception:
+            pass
     for _ in range(args.warmup if args.warmup < 1 else 1):
         pass   # the oracle has no warm-up state; one untimed generation pass happens inside
     t_start = time.perf_counter()
