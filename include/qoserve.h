@@ -286,6 +286,9 @@ int qos_profile_step_ex(qos_engine_t* eng, int32_t chunk_len, int32_t kv_start,
  *                          norm-fold threshold (down projection at mid T; slices add in a fixed
  *                          order, so results stay deterministic); env QOS_ADD_SPLIT
  *   "gemm_sms" (0)         SM budget of the step's GEMM grids (0 = all; experiments)
+ *   "swab_gran" (-1)       weight-streaming GEMM range granule in k-blocks (-1 automatic, 0 whole
+ *                          tiles); process-wide, experiments (profiles/step_swabgran_r2a.jsonl:
+ *                          the automatic granule is best in-step)
  *   "gemm_bn" (0)          force the tile width (128 / 256) of the QKV and gate/up tile GEMMs
  *                          (0 = the wave-cost choice; experiments: in-step A/B in
  *                          profiles/step_bn_r2a.jsonl found the automatic choice best)

@@ -1929,6 +1929,7 @@ int qos_engine_set_option(qos_engine_t* e, const char* name, int64_t value) {
   else if (n == "gemm_splitk") e->gemm_splitk = value != 0;
   else if (n == "pdl") set_pdl(value != 0);  // process-wide
   else if (n == "fa_poly") set_fa_poly(int(value));  // process-wide
+  else if (n == "swab_gran") set_swab_gran(int(value));  // process-wide (experiments)
   else if (n == "gemm_swab") e->gemm_swab = int(value < 0 ? 0 : value > 2 ? 2 : value);
   else if (n == "gemm_streamk") e->gemm_streamk = int(value < 0 ? 0 : value > 2 ? 2 : value);
   else if (n == "dual_stream") e->dual_stream = value != 0;

@@ -438,6 +438,9 @@ bool swab_prefer_k(int64_t M, int64_t N, int64_t K, int num_sms) {
   return ((M + 127) / 128) * (N / 128) * 2 < num_sms;
 }
 
+static int g_swab_gran = -1;  // option swab_gran (process-wide): -1 automatic
+void set_swab_gran(int v) { g_swab_gran = v; }
+
 int swab_grid(int64_t M, int64_t N, int64_t K, int bnt, int num_sms) {
   const int64_t work = (N / 128) * ((M + bnt - 1) / bnt) * (K / kSwBK);
   const int64_t g = work / 4;  // >= 4 k-blocks (64 KB of weights) per CTA
@@ -489,8 +492,9 @@ int gemm_swab_run(const CUtensorMap& tw, const CUtensorMap& tt, int bnt, int64_t
       }
     }
   }
-  if (const char* g = getenv("QOS_SWAB_GRAN")) {  // experiment knob: force a granule (0 = whole tiles)
-    int v = atoi(g);
+  const char* genv = getenv("QOS_SWAB_GRAN");
+  if (g_swab_gran >= 0 || genv) {  // experiment knob: force a granule (0 = whole tiles)
+    int v = g_swab_gran >= 0 ? g_swab_gran : atoi(genv);
     if (v == 0) v = a.kblocks;
     while (v > 1 && a.kblocks % v) --v;
     a.gran = v < 1 ? 1 : v;

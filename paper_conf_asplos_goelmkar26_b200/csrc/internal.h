@@ -14,6 +14,7 @@ bool pdl_enabled();
 void set_pdl(bool on);
 // prefill attention: every n-th exp2 pair on the FMA pipe (0 = all on MUFU); process-wide
 void set_fa_poly(int n);
+void set_swab_gran(int v);  // weight-streaming GEMM range granule (k-blocks; -1 automatic, 0 whole tiles)
 
 enum { EPI_STORE_BF16 = QOS_EPI_STORE_BF16, EPI_STORE_F32 = QOS_EPI_STORE_F32, EPI_BIAS_BF16 = QOS_EPI_BIAS_BF16,
        EPI_SILU_GATE = QOS_EPI_SILU_GATE, EPI_ADD_F32 = QOS_EPI_ADD_F32,
