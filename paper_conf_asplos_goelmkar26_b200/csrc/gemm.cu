@@ -1053,6 +1053,7 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
     tma_prefetch_desc(&tmA);
     tma_prefetch_desc(&tmB);
   }
+  cluster_sync();  // both CTAs of the pair resident before the pair-wide TMEM allocation
   if (warp == 1) tmem_alloc2<512>(tmem_slot);
   tc_fence_before();
   cluster_sync();  // barrier inits and the TMEM address visible pair-wide
