@@ -5,6 +5,7 @@ on the tiny config): every kernel family of the step, each launched at least onc
   compute-sanitizer --tool racecheck  python tools/sanitize_step.py
   compute-sanitizer --tool synccheck  python tools/sanitize_step.py --sync
   bash tools/sanitize.sh            (all four tools, summaries in gpurun_out/sanitize_*.log)
+  compute-sanitizer --tool racecheck  python tools/sanitize_step.py --wide   (Llama-3-8B width)
 
 --sync skips the prefill chunks (decode-only steps on synthetic KV): synccheck flags the
 prefill attention's o_full barrier, whose phases are completed once per P.V but observed by the
@@ -60,7 +61,28 @@ def decode_only(engs, vocab):
         run(lambda e: e.step_host(kb, vocab))
 
 
+def wide():
+    """Llama-3-8B width, 2 layers: a 2048-token chunk + 16 decodes @1k (CTA-pair GEMMs with the
+    folded norm, persistent prefill attention over 512 items, split decode attention)."""
+    cfg = q.model_cfg(**preset("llama3-8b", n_layers=2), num_blocks=(2048 + 16 * 1100) // 16 + 64,
+                      max_seq_len=4096, max_requests=32, max_batch_tokens=2048 + 16, max_batch_rows=17)
+    eng = q.Engine(cfg)
+    eng.qos_engine_load_synthetic(0)
+    b = synth.hybrid_batch(cfg.vocab, 2048, 16, 1024)
+    eng.qos_kv_alloc(0, 2048)
+    for d in b.decode:
+        eng.qos_kv_alloc(d.req, 1025)
+        eng.qos_kv_fill_synthetic(d.req, 1024, 2)
+    eng.step_host(q.batch_from_synth(b), cfg.vocab)
+    eng.close()
+    print("sanitize workload done")
+
+
 def main():
+    if "--wide" in sys.argv:
+        torch.cuda.set_device(0)
+        wide()
+        return
     sync = "--sync" in sys.argv
     torch.cuda.set_device(0)
     cfg = tiny_engine()
