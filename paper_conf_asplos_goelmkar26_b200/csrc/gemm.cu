@@ -21,7 +21,6 @@
 #include <cstdlib>
 
 #include <climits>
-#include <cstdlib>
 
 #include "common.cuh"
 #include "internal.h"
