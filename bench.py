@@ -108,7 +108,7 @@ class Workload:
     one token per step (steady-state serving); each step's chunk request is freed after it."""
 
     def __init__(self, device: int, n_steps: int, chunk=CHUNK, n_dec=N_DEC, ctx=CTX, n_layers=None,
-                 model="llama3-8b", tp=1, rank=0, group=None):
+                 model="llama3-8b", tp=1, rank=0, group=None, max_tokens=None):
         import synth
         from paper_conf_asplos_goelmkar26_b200 import qoserve as q
         from paper_conf_asplos_goelmkar26_b200.presets import preset
@@ -119,7 +119,8 @@ class Workload:
         num_blocks = n_dec * ((ctx_cap + 15) // 16) + (n_steps + 4) * ((chunk + 15) // 16) + 64
         self.preset = preset(model, **over)
         self.cfg = q.model_cfg(**self.preset, num_blocks=num_blocks, max_seq_len=8192,
-                               max_requests=n_dec + 64, max_batch_tokens=chunk + n_dec, max_batch_rows=n_dec + 1)
+                               max_requests=n_dec + 64, max_batch_tokens=max(chunk + n_dec, max_tokens or 0),
+                               max_batch_rows=n_dec + 1)
         self.eng = q.Engine(self.cfg, device=device, tp_rank=rank, tp_size=tp, group=group)
         self.eng.qos_engine_load_synthetic(synth.SEED_WEIGHTS)
         self.dec_reqs = list(range(1, n_dec + 1))
@@ -175,6 +176,10 @@ def run_ours(args):
         dist.broadcast_object_list(box, src=0)
         group = qq.Group(tp, box[0], rank)
     chunk, n_dec, ctx = WORKLOADS[args.workload]
+    # the chunk-size sweep after the timed passes (the metric is tokens/s and latency vs chunk
+    # size): the engine needs room for the largest chunk
+    sweep_chunks = (256, 512, 1024, 2048, 4096, 8192) if (args.workload == "hybrid" and tp == 1 and
+                                                          not args.no_sweep) else ()
     wl = Workload(local, W + 3 * K + 2, chunk=chunk, n_dec=n_dec, ctx=ctx, model=args.model, n_layers=args.layers,
                   tp=tp, rank=rank % tp, group=group)
     q, eng, T = wl.q, wl.eng, wl.tokens_per_step
@@ -229,6 +234,23 @@ def run_ours(args):
         wl.step(b, host_tok.ctypes.data, True, sptr)
     e2e_ms = (time.perf_counter() - t0) * 1e3 / K
     h2d, d2h = eng.qos_last_step_io()
+    # -------- chunk-size sweep (configs[1] row: chunk 256..8192 with the bench's 128 decodes @ctx
+    # 4096): device-timed median of qos_profile_step on scratch requests (the bench's decode
+    # requests are released first; their KV pool is reused)
+    sweep = []
+    if sweep_chunks:
+        # a second engine with room for the largest chunk (the headline engine keeps exactly the
+        # bench shape's workspace); the first one is released first
+        eng.close()
+        wl2 = Workload(local, 4, chunk=chunk, n_dec=n_dec, ctx=ctx, model=args.model, n_layers=args.layers,
+                       max_tokens=max(sweep_chunks) + n_dec)
+        for r in wl2.dec_reqs:
+            wl2.eng.qos_kv_free(r)
+        for c in sweep_chunks:
+            ms_c, p95_c = wl2.eng.qos_profile_step(c, [ctx] * n_dec, reps=3, warmup=2)
+            sweep.append({"chunk": c, "n_decode": n_dec, "ctx": ctx, "ms": round(ms_c, 3),
+                          "tokens_per_s": round(replicas * (c + n_dec) / (ms_c * 1e-3), 1)})
+        eng = wl2.eng
     # -------- max over ranks
     if ws > 1:
         t = torch.tensor([ms_step, e2e_ms, ms_instr], device="cpu" if shared_gpu else "cuda")
@@ -312,6 +334,7 @@ def run_ours(args):
                                   "frac": round(da_gbs / peak_hbm, 4),
                                   "peak_source": "MEASURED_PEAKS.json hbm_gbs (of measured)"} if n_dec else None),
         "roofline_step": roof_step,
+        "chunk_sweep": sweep or None,
         "gpu_launches": int(launches),
         "clocks": clk,
         "e2e": {"value": round(replicas * T / (e2e_ms * 1e-3), 1), "unit": "tokens/s",
@@ -438,6 +461,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-sweep", action="store_true", help="skip the chunk-size sweep after the timed passes")
     ap.add_argument("--cpu-seconds", type=float, default=20.0)
     ap.add_argument("--tp", type=int, default=1, help="tensor-parallel degree (= WORLD_SIZE under torchrun)")
     ap.add_argument("--model", default="llama3-8b", help="llama3-8b | qwen2.5-14b | llama3-70b")
