@@ -234,23 +234,6 @@ def run_ours(args):
         wl.step(b, host_tok.ctypes.data, True, sptr)
     e2e_ms = (time.perf_counter() - t0) * 1e3 / K
     h2d, d2h = eng.qos_last_step_io()
-    # -------- chunk-size sweep (configs[1] row: chunk 256..8192 with the bench's 128 decodes @ctx
-    # 4096): device-timed median of qos_profile_step on scratch requests (the bench's decode
-    # requests are released first; their KV pool is reused)
-    sweep = []
-    if sweep_chunks:
-        # a second engine with room for the largest chunk (the headline engine keeps exactly the
-        # bench shape's workspace); the first one is released first
-        eng.close()
-        wl2 = Workload(local, 4, chunk=chunk, n_dec=n_dec, ctx=ctx, model=args.model, n_layers=args.layers,
-                       max_tokens=max(sweep_chunks) + n_dec)
-        for r in wl2.dec_reqs:
-            wl2.eng.qos_kv_free(r)
-        for c in sweep_chunks:
-            ms_c, p95_c = wl2.eng.qos_profile_step(c, [ctx] * n_dec, reps=3, warmup=2)
-            sweep.append({"chunk": c, "n_decode": n_dec, "ctx": ctx, "ms": round(ms_c, 3),
-                          "tokens_per_s": round(replicas * (c + n_dec) / (ms_c * 1e-3), 1)})
-        eng = wl2.eng
     # -------- max over ranks
     if ws > 1:
         t = torch.tensor([ms_step, e2e_ms, ms_instr], device="cpu" if shared_gpu else "cuda")
@@ -281,12 +264,39 @@ def run_ours(args):
     Hq = pr["n_heads"] // tp
     V = pr["vocab"] // tp
     proj = [(d * (Hq + 2 * Hkv) * hd), (Hq * hd * d), (2 * d * F), (F * d)]   # weights per layer (elements)
-    R = n_dec + 1
-    t_gemm = sum(max(2.0 * T * w / (peak_tc * 1e12), 2.0 * w / (peak_hbm * 1e9)) for w in proj) * L
-    t_head = max(2.0 * R * d * V / (peak_tc * 1e12), 2.0 * d * V / (peak_hbm * 1e9))
-    t_dec = da_bytes * L / (peak_hbm * 1e9)
-    t_pre = pa_flops * L / (peak_tc * 1e12)
+
+    def step_terms(c, nd, cx, kv_bytes=None):
+        Tt, R = c + nd, (1 if c else 0) + nd
+        tg = sum(max(2.0 * Tt * w / (peak_tc * 1e12), 2.0 * w / (peak_hbm * 1e9)) for w in proj) * L
+        th = max(2.0 * R * d * V / (peak_tc * 1e12), 2.0 * d * V / (peak_hbm * 1e9))
+        kvb = kv_bytes if kv_bytes is not None else 4.0 * hd * Hkv * nd * (cx + 1)
+        td = kvb * L / (peak_hbm * 1e9)
+        tp_ = 4.0 * hd * Hq * (c * (c + 1) / 2.0) * L / (peak_tc * 1e12)
+        return tg, th, td, tp_
+
+    def step_roofline_ms(c, nd, cx):
+        return sum(step_terms(c, nd, cx)) * 1e3
+
+    t_gemm, t_head, t_dec, t_pre = step_terms(chunk, n_dec, ctx, kv_bytes=da_bytes)
     t_roof = (t_gemm + t_head + t_dec + t_pre) * 1e3
+    # -------- chunk-size sweep (configs[1] row: chunk 256..8192 with the bench's 128 decodes @ctx
+    # 4096): device-timed median of qos_profile_step on scratch requests (the bench's decode
+    # requests are released first; their KV pool is reused)
+    sweep = []
+    if sweep_chunks:
+        # a second engine with room for the largest chunk (the headline engine keeps exactly the
+        # bench shape's workspace); the first one is released first
+        eng.close()
+        wl2 = Workload(local, 4, chunk=chunk, n_dec=n_dec, ctx=ctx, model=args.model, n_layers=args.layers,
+                       max_tokens=max(sweep_chunks) + n_dec)
+        for r in wl2.dec_reqs:
+            wl2.eng.qos_kv_free(r)
+        for c in sweep_chunks:
+            ms_c, p95_c = wl2.eng.qos_profile_step(c, [ctx] * n_dec, reps=3, warmup=2)
+            sweep.append({"chunk": c, "n_decode": n_dec, "ctx": ctx, "ms": round(ms_c, 3),
+                          "tokens_per_s": round(replicas * (c + n_dec) / (ms_c * 1e-3), 1),
+                          "roofline_frac": round(step_roofline_ms(c, n_dec, ctx) / ms_c, 4)})
+        eng = wl2.eng
     roof_step = {"roofline_ms": round(t_roof, 3), "achieved_ms": round(ms_step, 3), "frac": round(t_roof / ms_step, 4),
                  "terms_ms": {"projections": round(t_gemm * 1e3, 3), "lm_head": round(t_head * 1e3, 3),
                               "decode_attn": round(t_dec * 1e3, 3), "prefill_attn": round(t_pre * 1e3, 3)},
