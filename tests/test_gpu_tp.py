@@ -140,12 +140,13 @@ def test_tp_peer_group_profile_step_and_missing_rank_aborts():
 
 
 @pytest.mark.slow
-def test_qwen14b_shapes_tp2_hybrid_step_sampled_parity():
+@pytest.mark.parametrize("tp", [2, 4])
+def test_qwen14b_shapes_tp2_hybrid_step_sampled_parity(tp):
     """configs[2] launch shape: Qwen-2.5-14B (2 layers, full width: d 5120, 40 q / 8 kv heads,
-    QKV bias, F 13824, V 152064) at TP2 — a 2048-token chunk + 128 decodes @ ctx 4096 with
-    synthetic KV prefixes — sampled logits rows vs the unsharded oracle."""
+    QKV bias, F 13824, V 152064) at TP2 and TP4 — a 2048-token chunk + 128 decodes @ ctx 4096
+    with synthetic KV prefixes — sampled logits rows vs the unsharded oracle, ranks identical."""
     C, ND, CTX = 2048, 128, 4096
-    q, cfg, g, engs = _group_engines("qwen2.5-14b", 2, n_layers=2,
+    q, cfg, g, engs = _group_engines("qwen2.5-14b", tp, n_layers=2,
                                      num_blocks=(C + ND * (CTX + 1)) // 16 + 200, max_seq_len=8192,
                                      max_batch_tokens=C + ND, max_batch_rows=ND + 1, max_requests=ND + 8)
     _all(q, engs, lambda r, e: e.qos_engine_load_synthetic(0))
@@ -159,7 +160,7 @@ def test_qwen14b_shapes_tp2_hybrid_step_sampled_parity():
     _all(q, engs, prep)
     kb = q.batch_from_synth(b)
     outs = _all(q, engs, lambda r, e: e.step_host(kb, cfg.vocab))
-    assert np.array_equal(outs[0][0], outs[1][0])
+    assert all(np.array_equal(outs[0][0], o[0]) for o in outs[1:])
     lg = outs[0][0]
     orc = _oracle("qwen2.5-14b", n_layers=2, num_blocks=2 * (C // 16 + 1) + 8 * (CTX // 16 + 2))
     sample = [0, 77, 127]
