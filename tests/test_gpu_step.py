@@ -338,6 +338,32 @@ def test_llama8b_mid_t_step_parity(add_split):
     eng.close()
 
 
+def test_capacity_boundaries_step_parity():
+    """Edge of every capacity at once: a chunk of exactly max_batch_tokens - 1 tokens whose last
+    position is max_seq_len - 1 (the last block-table column), a decode at position
+    max_seq_len - 1, and R = max_batch_rows; logits vs the oracle, then one position further is
+    refused without changing state."""
+    q, cfg, eng = make_engine("tiny", num_blocks=256, max_seq_len=1024, max_batch_tokens=512, max_batch_rows=2)
+    eng.qos_engine_load_synthetic(0)
+    orc = _oracle("tiny", num_blocks=256)
+    for alloc, fill in ((eng.qos_kv_alloc, eng.qos_kv_fill_synthetic), (orc.kv_alloc, orc.kv_fill_synthetic)):
+        alloc(1, 1024)
+        fill(1, 1024 - 511, synth.SEED_KVFILL)
+        alloc(2, 1024)
+        fill(2, 1023, synth.SEED_KVFILL)
+    rng = np.random.default_rng(3)
+    toks = [int(x) for x in rng.integers(0, cfg.vocab, 511)]
+    b = q.make_batch([(1, 1024 - 511, np.array(toks, np.int32))], [(2, 1023, 5)])
+    lg, _ = eng.step_host(b, cfg.vocab)
+    ref = orc.hybrid_step([(1, 1024 - 511, toks)], [(2, 1023, 5)])
+    assert row_rel_err(lg, ref) <= TOL_LOGITS
+    assert eng.qos_kv_cached_len(1) == 1024 and eng.qos_kv_cached_len(2) == 1024
+    with pytest.raises(q.QosError):                       # position 1024 >= max_seq_len / past the table
+        eng.step_host(q.make_batch([], [(2, 1024, 5)]), cfg.vocab)
+    assert eng.qos_kv_cached_len(2) == 1024
+    eng.close()
+
+
 def test_long_context_step_parity():
     """Maximum context (configs[3]: up to 32k): a 100-token chunk at kv_start 16000 and decodes
     at ctx 32767 / 20000 / 17, all prefixes synthetic KV, through qos_hybrid_step vs the oracle
