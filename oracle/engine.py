@@ -120,6 +120,47 @@ class OracleEngine:
             return np.zeros((0, self.cfg.vocab))
         return logits_of(self.cfg, self.W, np.stack(last))
 
+    def hybrid_step_layer_major(self, prefill, decode) -> np.ndarray:
+        """hybrid_step with the loops exchanged: layer by layer, every request of the step
+        through that layer (each layer's weights are needed once, not once per request — the
+        form that makes full-depth bench-size checks affordable).  Per request the operations
+        and their order are exactly forward_run's, so the result is identical (pinned in
+        tests/test_oracle_model.py)."""
+        c = self.cfg
+        runs = [(req, list(tokens), kv_start) for req, kv_start, tokens in prefill] + \
+               [(req, [token], ctx_len) for req, ctx_len, token in decode]
+        reqs = [r[0] for r in runs]
+        if len(set(reqs)) != len(reqs):
+            raise ValueError("a request appears twice in one step")
+        if not runs:
+            return np.zeros((0, c.vocab))
+        xs, poss = [], []
+        for req, tokens, start in runs:
+            if self.cached_len(req) != start:
+                raise OracleBadKVStart(f"req {req}: cached {self.cached_len(req)} != start {start}")
+            self._check_alloc(req, start + len(tokens))
+            if req not in self.kv:
+                z = np.zeros((0, c.n_kv_heads, c.head_dim))
+                self.kv[req] = [(z, z) for _ in range(c.n_layers)]
+            xs.append(self.W.embed(tokens))
+            poss.append(start + np.arange(len(tokens)))
+        group = c.n_heads // c.n_kv_heads
+        for l in range(c.n_layers):
+            w = self.W.layer(l)
+            for i, (req, tokens, start) in enumerate(runs):
+                x, n = xs[i], len(tokens)
+                h = rms_norm(x, w["ln1"], c.rms_eps)
+                q, k, v = layer_qkv(c, w, h, poss[i])
+                K, V = self.kv[req][l]
+                K = np.concatenate([K, k], axis=0)
+                V = np.concatenate([V, v], axis=0)
+                self.kv[req][l] = (K, V)
+                o = causal_attention(q, K, V, start, group)
+                x = x + o.reshape(n, c.n_heads * c.head_dim) @ w["wo"].T
+                h2 = rms_norm(x, w["ln2"], c.rms_eps)
+                xs[i] = x + swiglu_mlp(h2, w["wg"], w["wu"], w["wd"])
+        return logits_of(c, self.W, np.stack([x[-1] for x in xs]))
+
 
 def greedy(logits: np.ndarray) -> np.ndarray:
     """Greedy argmax per row, lowest index on ties (reading s11; np.argmax returns the first

@@ -149,6 +149,7 @@ struct FaParams {
   const int32_t* tables;
   int table_w;
   float scale_log2;
+  int kv_first = 0;  // persistent kernel: issue an item's first K/V tile before its Q (option fa_kvfirst)
 };
 
 // Work item = NQ consecutive entries of `items`: q tiles of one (chunk, kv head) that share
@@ -513,6 +514,37 @@ __global__ void __launch_bounds__(FaCfg<HD, 1>::kThreads, 2)
       for (int ii = i_begin, n = 0; ii < i_end; ++ii, ++n) {
         const PrefillItem it = items[ii];
         const int nt = it.grp_last / C::kKeys + 1, last_blk = it.grp_last >> 4;
+        const int32_t* trow = p.tables + size_t(it.table) * p.table_w;
+        // tile j of the item into ring slot jg % S; the tile's 4 block-table entries are read
+        // once (independent loads) for its K and V halves; past the causal end a valid block (P = 0)
+        auto load_kv = [&](int j) {
+          const int s = int(jg % S);
+          const uint32_t ph = (jg / S) & 1;
+          int r[C::kKeys / 16];
+#pragma unroll
+          for (int b = 0; b < C::kKeys / 16; ++b)
+            r[b] = (__ldg(trow + min(j * (C::kKeys / 16) + b, last_blk)) * p.Hkv + it.kv_head) * 16;
+          mbar_wait(&k_empty[s], ph ^ 1);
+          mbar_arrive_expect_tx(&k_full[s], C::kTileBytes);
+#pragma unroll
+          for (int b = 0; b < C::kKeys / 16; ++b)
+#pragma unroll
+            for (int hf = 0; hf < C::kHalves; ++hf)
+              tma_load_3d(sK + s * C::kTileBytes + hf * (C::kKeys * 128) + b * 2048, &kvmap, &k_full[s], hf * 64, r[b],
+                          p.layer * 2);
+          mbar_wait(&v_empty[s], ph ^ 1);
+          mbar_arrive_expect_tx(&v_full[s], C::kTileBytes);
+#pragma unroll
+          for (int b = 0; b < C::kKeys / 16; ++b)
+#pragma unroll
+            for (int hf = 0; hf < C::kHalves; ++hf)
+              tma_load_3d(sV + s * C::kTileBytes + hf * (C::kKeys * 128) + b * 2048, &kvmap, &v_full[s], hf * 64, r[b],
+                          p.layer * 2 + 1);
+          ++jg;
+        };
+        // with kv_first the item's first K/V tile goes out before its Q, which has to wait for
+        // the previous item's last QK to release sQ
+        if (p.kv_first) load_kv(0);
         // Q tile of the item: rows (position, head-in-group) = a {64 dims, group heads, ppt rows}
         // box per 64-dim half; issued as soon as the previous item's last QK has read sQ
         // (group * ppt rows: 125 when the GQA group is 5 — the remaining rows of sQ are never
@@ -522,26 +554,7 @@ __global__ void __launch_bounds__(FaCfg<HD, 1>::kThreads, 2)
 #pragma unroll
         for (int hf = 0; hf < C::kHalves; ++hf)
           tma_load_3d(sQ + hf * (C::kRows * 128), &qmap, q_full, hf * 64, it.kv_head * group, it.row0);
-        const int32_t* trow = p.tables + size_t(it.table) * p.table_w;
-        auto load_tile = [&](uint8_t* dst, uint64_t* full, int j, int plane) {
-          for (int b = 0; b < C::kKeys / 16; ++b) {
-            const int blk = min(j * (C::kKeys / 16) + b, last_blk);  // past the causal end: a valid block (P = 0)
-            const int r = (__ldg(trow + blk) * p.Hkv + it.kv_head) * 16;
-#pragma unroll
-            for (int hf = 0; hf < C::kHalves; ++hf)
-              tma_load_3d(dst + hf * (C::kKeys * 128) + b * 2048, &kvmap, full, hf * 64, r, p.layer * 2 + plane);
-          }
-        };
-        for (int j = 0; j < nt; ++j, ++jg) {
-          const int s = int(jg % S);
-          const uint32_t ph = (jg / S) & 1;
-          mbar_wait(&k_empty[s], ph ^ 1);
-          mbar_arrive_expect_tx(&k_full[s], C::kTileBytes);
-          load_tile(sK + s * C::kTileBytes, &k_full[s], j, 0);
-          mbar_wait(&v_empty[s], ph ^ 1);
-          mbar_arrive_expect_tx(&v_full[s], C::kTileBytes);
-          load_tile(sV + s * C::kTileBytes, &v_full[s], j, 1);
-        }
+        for (int j = p.kv_first ? 1 : 0; j < nt; ++j) load_kv(j);
       }
     }
   } else if (warp == 1) {
@@ -714,6 +727,315 @@ __global__ void __launch_bounds__(FaCfg<HD, 1>::kThreads, 2)
   if (warp == 1) {
     tc_fence_after();
     tmem_dealloc<C::kTmemCols>(tmem);
+  }
+}
+
+// ---------------------------------------------------------------- CTA-pair variant (fa_pair=1)
+// The persistent kernel above on a thread-block cluster of 2 CTAs (2 SMs of one TPC) issuing
+// tcgen05.mma.cta_group::2: one work item = two consecutive 128-row q tiles of one (chunk, kv
+// head), CTA r holding q tile r in its smem and its 128 rows of S / P / O in its own TMEM.
+//   S = Q K^T  (UMMA M = 256, N = 64 keys): B is split by N, so CTA r stages only keys
+//              [32r, 32r + 32) of each 64-key tile;
+//   O += P V   (UMMA M = 256, N = HD = 128, A = P from each CTA's TMEM): B = V is split by N,
+//              so CTA r stages only dims [64r, 64r + 64) of the tile's 64 keys.
+// Each K/V tile therefore costs every SM 16 KB of L2 -> SM traffic for 128 rows instead of
+// 32 KB: the single-CTA kernel moves 128 FLOP per L2 byte (4.2 MFLOP of QK + PV per 32 KB),
+// which at ~42 B/cycle/SM of L2 throughput caps it near 66% of the tensor peak — the measured
+// ceiling of its MMA + TMA pipeline (profiles/prefill_attn_caps_ncu_r2a.jsonl).  (TMA
+// multicast does not help at cluster size 2: the L2 de-duplicates only within ~4 requests.)
+// Both CTAs' TMA loads complete on the leader's full barriers; the leader's commits arrive
+// on both CTAs' barriers (multicast); the softmax warps of both CTAs release a P buffer on the
+// leader's barrier (one remote arrive per warp).  2 pairs share an SM pair (96 KB smem and 256
+// TMEM columns per CTA), so one pair's softmax overlaps the other's MMAs, as in the
+// single-CTA kernel.  HD = 128 only (a 64-dim half of V is exactly one 128-B swizzle atom).
+struct PairCfg {
+  static constexpr int HD = 128;
+  static constexpr int kRows = 128;                  // rows per CTA (UMMA M = 256 over the pair)
+  static constexpr int kKeys = 64;                   // keys per K/V tile of the pair
+  static constexpr int kQBytes = kRows * HD * 2;     // 32 KB
+  static constexpr int kKBytes = (kKeys / 2) * HD * 2;  // this CTA's 32 keys x 128 dims: 8 KB
+  static constexpr int kVBytes = kKeys * (HD / 2) * 2;  // 64 keys x this CTA's 64 dims: 8 KB
+  static constexpr int kStages = 4;
+  static constexpr int kSmem = kQBytes + kStages * (kKBytes + kVBytes) + 1024 + 512;
+  static constexpr int kThreads = 192;
+  static constexpr uint32_t kTmemCols = 256;         // S/P buffers at 0 and 64, O at 128
+};
+
+template <int POLY>
+__global__ void __launch_bounds__(PairCfg::kThreads, 2)
+    prefill_attn_pair_kernel(const __grid_constant__ CUtensorMap kvmap, const __grid_constant__ CUtensorMap qmap,
+                             const FaParams p, const PrefillItem* __restrict__ items,
+                             const int32_t* __restrict__ cta_off) {
+  using C = PairCfg;
+  constexpr int S = C::kStages;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sQ = smem;
+  uint8_t* sK = smem + C::kQBytes;
+  uint8_t* sV = sK + S * C::kKBytes;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(sV + S * C::kVBytes);
+  uint64_t* k_full = bar;            // leader's: both CTAs' K halves landed
+  uint64_t* k_empty = k_full + S;    // each CTA's: QK of the slot's tile done
+  uint64_t* v_full = k_empty + S;    // leader's
+  uint64_t* v_empty = v_full + S;    // each CTA's
+  uint64_t* s_full = v_empty + S;    // [2] each CTA's
+  uint64_t* p_full = s_full + 2;     // [2] leader's: 4 softmax warps of each CTA
+  uint64_t* o_full = p_full + 2;     // each CTA's: completes once per P.V
+  uint64_t* o_final = o_full + 1;    // each CTA's: completes once per item
+  uint64_t* q_full = o_final + 1;    // leader's: both Q tiles landed
+  uint64_t* q_empty = q_full + 1;    // each CTA's: the item's last QK done
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(q_empty + 1);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t rank = cluster_ctarank();
+  const bool leader = rank == 0;
+  const int pair = int(blockIdx.x >> 1);
+  const int g_begin = cta_off[pair], g_end = cta_off[pair + 1];
+  const int group = p.H / p.Hkv;
+  const int ppt = C::kRows / group;
+
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < S; ++i) {
+      mbar_init(&k_full[i], 1);
+      mbar_init(&k_empty[i], 1);
+      mbar_init(&v_full[i], 1);
+      mbar_init(&v_empty[i], 1);
+    }
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&s_full[b], 1);
+      mbar_init(&p_full[b], 8);
+    }
+    mbar_init(o_full, 1);
+    mbar_init(o_final, 1);
+    mbar_init(q_full, 1);
+    mbar_init(q_empty, 1);
+    fence_mbar_init();
+  }
+  cluster_sync();  // both CTAs resident before the pair-wide TMEM allocation
+  if (warp == 1) tmem_alloc2<C::kTmemCols>(tmem_slot);
+  tc_fence_before();
+  cluster_sync();  // barrier inits and the TMEM address visible pair-wide
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+  griddep_wait();  // q and the appended K/V come from the previous kernel
+  griddep_launch_dependents();
+
+  if (warp == 0) {
+    // ------------------------------------------------------------------ TMA producer (both CTAs)
+    if (elect_one()) {
+      tma_prefetch_desc(&kvmap);
+      tma_prefetch_desc(&qmap);
+      const uint32_t kf0 = mapa_shared(smem_u32(k_full), 0), vf0 = mapa_shared(smem_u32(v_full), 0);
+      const uint32_t qf0 = mapa_shared(smem_u32(q_full), 0);
+      uint32_t jg = 0;
+      for (int gi = g_begin, n = 0; gi < g_end; ++gi, ++n) {
+        const PrefillItem it = items[2 * gi + int(rank)];
+        const int nt = it.grp_last / C::kKeys + 1, last_blk = it.grp_last >> 4;
+        const int32_t* trow = p.tables + size_t(it.table) * p.table_w;
+        // tile j of this item into ring slot jg % S: K blocks 2r, 2r+1 (both 64-dim halves),
+        // V dims [64r, 64r+64) of all 4 blocks; past the causal end a valid block (P = 0)
+        auto load_kv = [&](int j) {
+          const int s = int(jg % S);
+          const uint32_t ph = (jg / S) & 1;
+          mbar_wait(&k_empty[s], ph ^ 1);
+          if (leader) mbar_arrive_expect_tx(&k_full[s], 2 * C::kKBytes);
+#pragma unroll
+          for (int bb = 0; bb < 2; ++bb) {
+            const int blk = min(j * 4 + int(rank) * 2 + bb, last_blk);
+            const int r = (__ldg(trow + blk) * p.Hkv + it.kv_head) * 16;
+#pragma unroll
+            for (int hf = 0; hf < 2; ++hf)
+              tma_load_3d_2cta(sK + s * C::kKBytes + hf * 4096 + bb * 2048, &kvmap, kf0 + uint32_t(s) * 8, hf * 64, r,
+                               p.layer * 2);
+          }
+          mbar_wait(&v_empty[s], ph ^ 1);
+          if (leader) mbar_arrive_expect_tx(&v_full[s], 2 * C::kVBytes);
+#pragma unroll
+          for (int b = 0; b < 4; ++b) {
+            const int blk = min(j * 4 + b, last_blk);
+            const int r = (__ldg(trow + blk) * p.Hkv + it.kv_head) * 16;
+            tma_load_3d_2cta(sV + s * C::kVBytes + b * 2048, &kvmap, vf0 + uint32_t(s) * 8, int(rank) * 64, r,
+                             p.layer * 2 + 1);
+          }
+          ++jg;
+        };
+        // the item's first K/V tile goes out before its Q, which waits for the previous item's
+        // last QK to release sQ
+        load_kv(0);
+        if (n > 0) mbar_wait(q_empty, uint32_t(n - 1) & 1);
+        if (leader) mbar_arrive_expect_tx(q_full, 2u * 2u * 128u * uint32_t(group * ppt));
+#pragma unroll
+        for (int hf = 0; hf < 2; ++hf)
+          tma_load_3d_2cta(sQ + hf * (C::kRows * 128), &qmap, qf0, hf * 64, it.kv_head * group, it.row0);
+        for (int j = 1; j < nt; ++j) load_kv(j);
+      }
+    }
+  } else if (warp == 1) {
+    // ------------------------------------------------------------------ MMA issuer (leader)
+    if (leader && elect_one()) {
+      constexpr uint32_t idesc_qk = umma_idesc_bf16(256, C::kKeys);
+      constexpr uint32_t idesc_pv = (1u << 4) | (1u << 16) | ((uint32_t(C::HD) >> 3) << 17) | ((256u >> 4) << 24);
+      auto issue_pv = [&](uint32_t tg, bool first) {
+        const int s = int(tg % S);
+        mbar_wait(&v_full[s], (tg / S) & 1);
+        mbar_wait(&p_full[tg & 1], (tg >> 1) & 1);
+        tc_fence_after();
+        const uint32_t v_base = smem_u32(sV + s * C::kVBytes);
+        const uint32_t p_tmem = tmem + (tg & 1) * 64;
+#pragma unroll
+        for (int kk = 0; kk < C::kKeys / 16; ++kk)
+          umma_ts_2cta(tmem + 128, p_tmem + (kk >> 1) * 32 + (kk & 1) * 8, umma_desc_sw128_mn(v_base + kk * 2048, 8192),
+                       idesc_pv, (!first || kk != 0) ? 1u : 0u);
+        umma_commit_2cta(o_full);
+        umma_commit_2cta(&v_empty[s]);
+      };
+      const uint32_t q_base = smem_u32(sQ);
+      uint32_t jg = 0;
+      for (int gi = g_begin, n = 0; gi < g_end; ++gi, ++n) {
+        const int nt = items[2 * gi].grp_last / C::kKeys + 1;
+        mbar_wait(q_full, uint32_t(n) & 1);
+        tc_fence_after();
+        for (int j = 0; j < nt; ++j) {
+          const uint32_t tg = jg + uint32_t(j);
+          const int s = int(tg % S);
+          mbar_wait(&k_full[s], (tg / S) & 1);
+          tc_fence_after();
+          const uint32_t k_base = smem_u32(sK + s * C::kKBytes);
+#pragma unroll
+          for (int ks = 0; ks < C::HD / 16; ++ks)
+            umma_bf16_2cta(tmem + (tg & 1) * 64, umma_desc_sw128(q_base + (ks >> 2) * (C::kRows * 128) + (ks & 3) * 32),
+                           umma_desc_sw128(k_base + (ks >> 2) * 4096 + (ks & 3) * 32), idesc_qk, ks != 0);
+          umma_commit_2cta(&s_full[tg & 1]);
+          umma_commit_2cta(&k_empty[s]);
+          if (j >= 1) issue_pv(tg - 1, j == 1);  // O += P(j-1) V(j-1) while the softmax works on S(j)
+        }
+        umma_commit_2cta(q_empty);  // every QK of this item issued: both sQ free once they complete
+        issue_pv(jg + uint32_t(nt) - 1, nt == 1);
+        umma_commit_2cta(o_final);
+        jg += uint32_t(nt);
+      }
+    }
+  } else {
+    // ------------------------------------------------------------------ softmax + epilogue (both CTAs)
+    const int row = (warp & 3) * 32 + lane;
+    const uint32_t lane_base = tmem + (uint32_t((warp & 3) * 32) << 16);
+    const uint32_t o_addr = lane_base + 128;
+    const uint32_t pf0 = mapa_shared(smem_u32(p_full), 0);
+    const int pi = row / group, hh = row % group;
+    uint32_t jg = 0;
+    for (int gi = g_begin, n = 0; gi < g_end; ++gi, ++n) {
+      const PrefillItem it = items[2 * gi + int(rank)];
+      const int nt = it.grp_last / C::kKeys + 1;
+      const bool ok = row < ppt * group && pi < it.npos;
+      const int pos_r = ok ? it.pos0 + pi : -1;
+      const size_t tok_off = size_t(it.row0 + pi) * p.out_ld + size_t(it.kv_head * group + hh) * C::HD;
+      const int warp_min_pos = __shfl_sync(0xffffffffu, pos_r < 0 ? INT_MAX : pos_r, 0);
+      float m_used = -INFINITY, l = 0.f;
+      for (int j = 0; j < nt; ++j) {
+        const uint32_t tg = jg + uint32_t(j);
+        const int sb = int(tg & 1);
+        mbar_wait(&s_full[sb], (tg >> 1) & 1);
+        tc_fence_after();
+        const uint32_t s_addr = lane_base + uint32_t(sb) * 64;
+        const int key0 = j * C::kKeys;
+        const bool masked = __any_sync(0xffffffffu, key0 + C::kKeys - 1 > (pos_r < 0 ? -1 : pos_r)) ||
+                            warp_min_pos == INT_MAX;
+        uint32_t r[C::kKeys];
+#pragma unroll
+        for (int c = 0; c < C::kKeys / 16; ++c)
+          tmem_ld32x32b_x16(s_addr + c * 16, *reinterpret_cast<uint32_t(*)[16]>(&r[c * 16]));
+        tmem_ld_wait();
+        if (masked) {
+          const int lim = (pos_r < 0 ? -1 : pos_r) - key0;
+#pragma unroll
+          for (int i = 0; i < C::kKeys; ++i)
+            if (i > lim) r[i] = 0xff800000u;  // -inf
+        }
+        float mq[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
+#pragma unroll
+        for (int i = 0; i < C::kKeys; i += 2)
+          mq[(i >> 1) & 3] = fmax3(mq[(i >> 1) & 3], __uint_as_float(r[i]), __uint_as_float(r[i + 1]));
+        float mx = fmax3(mq[0], mq[1], fmaxf(mq[2], mq[3]));
+        mx *= p.scale_log2;
+        const bool rescale = mx > m_used + QOS_FA_LAZY;
+        const float m_new = rescale ? mx : m_used;
+        const float alpha = (rescale && m_used != -INFINITY) ? ex2(m_used - m_new) : 1.f;
+        const float mb = (m_new == -INFINITY) ? 0.f : m_new;
+        float2 sum2[4] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
+        const float2 scale2 = make_float2(p.scale_log2, p.scale_log2), nmb2 = make_float2(-mb, -mb);
+#pragma unroll
+        for (int c = 0; c < C::kKeys / 32; ++c) {
+          uint32_t hi[16];
+#pragma unroll
+          for (int i = 0; i < 16; ++i) {
+            const float2 x = fma2(make_float2(__uint_as_float(r[c * 32 + 2 * i]), __uint_as_float(r[c * 32 + 2 * i + 1])),
+                                  scale2, nmb2);
+            float2 pp = (POLY > 0 && i % (POLY > 0 ? POLY : 1) == (POLY > 0 ? POLY : 1) - 1) ? ex2_poly2(x) : make_float2(ex2(x.x), ex2(x.y));
+            hi[i] = pack_f16(pp.x, pp.y);
+            sum2[i & 3] = add2(sum2[i & 3], pp);
+          }
+          tmem_st32x32b_x16(s_addr + c * 32, hi);
+        }
+        const float2 s01 = add2(sum2[0], sum2[1]), s23 = add2(sum2[2], sum2[3]);
+        const float sum = (s01.x + s23.x) + (s01.y + s23.y);
+        tmem_st_wait();
+        l = l * alpha + sum;
+        if (j >= 1 && __any_sync(0xffffffffu, alpha != 1.f)) {
+          // PV(tg-2) completed before QK(tg) (awaited above): o_full has completed tg-1 or tg times
+          mbar_wait(o_full, (tg - 1) & 1);
+          tc_fence_after();
+#pragma unroll 1
+          for (int c = 0; c < C::HD / 16; ++c) {
+            uint32_t r2[16];
+            tmem_ld32x32b_x16(o_addr + c * 16, r2);
+            tmem_ld_wait();
+#pragma unroll
+            for (int i = 0; i < 16; ++i) r2[i] = __float_as_uint(__uint_as_float(r2[i]) * alpha);
+            tmem_st32x32b_x16(o_addr + c * 16, r2);
+          }
+          tmem_st_wait();
+        }
+        m_used = m_new;
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive_remote(pf0 + uint32_t(sb) * 8);
+      }
+      mbar_wait(o_final, uint32_t(n) & 1);
+      tc_fence_after();
+      const float inv = (l > 0.f) ? 1.f / l : 0.f;
+#pragma unroll 1
+      for (int c = 0; c < C::HD / 32; ++c) {
+        uint32_t r2[32];
+        tmem_ld32x32b_x16(o_addr + c * 32, *reinterpret_cast<uint32_t(*)[16]>(&r2[0]));
+        tmem_ld32x32b_x16(o_addr + c * 32 + 16, *reinterpret_cast<uint32_t(*)[16]>(&r2[16]));
+        tmem_ld_wait();
+        if (pos_r >= 0 && !it.pad) {
+          if (p.out_f32) {
+            float4* dst = reinterpret_cast<float4*>(reinterpret_cast<float*>(p.out) + tok_off + c * 32);
+#pragma unroll
+            for (int i = 0; i < 8; ++i)
+              dst[i] = make_float4(__uint_as_float(r2[4 * i]) * inv, __uint_as_float(r2[4 * i + 1]) * inv,
+                                   __uint_as_float(r2[4 * i + 2]) * inv, __uint_as_float(r2[4 * i + 3]) * inv);
+          } else {
+            uint4* dst = reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(p.out) + tok_off + c * 32);
+#pragma unroll
+            for (int i = 0; i < 4; ++i)
+              dst[i] = make_uint4(pack_bf16(__uint_as_float(r2[8 * i]) * inv, __uint_as_float(r2[8 * i + 1]) * inv),
+                                  pack_bf16(__uint_as_float(r2[8 * i + 2]) * inv, __uint_as_float(r2[8 * i + 3]) * inv),
+                                  pack_bf16(__uint_as_float(r2[8 * i + 4]) * inv, __uint_as_float(r2[8 * i + 5]) * inv),
+                                  pack_bf16(__uint_as_float(r2[8 * i + 6]) * inv, __uint_as_float(r2[8 * i + 7]) * inv));
+          }
+        }
+      }
+      jg += uint32_t(nt);
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  cluster_sync();  // the leader's MMAs / commits into this CTA and the peer's remote arrivals are done
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc2<C::kTmemCols>(tmem);
   }
 }
 
@@ -1025,6 +1347,7 @@ __global__ void __launch_bounds__(PpCfg<HD>::kThreads, 1)
 }
 
 static int g_fa_poly = getenv("QOS_FA_POLY") ? atoi(getenv("QOS_FA_POLY")) : 4;
+static int g_fa_kvfirst = 0;  // neutral in ncu cycles (profiles/ncu_ab_fa_r2c.jsonl)
 
 template <int HD, int POLY, int NQ>
 static cudaError_t prefill_tc_t(const AttnLaunch& a, const PrefillItem* items, int n_items, cudaStream_t st) {
@@ -1098,11 +1421,66 @@ static cudaError_t prefill_persist_t(const AttnLaunch& a, const PrefillItem* ite
   p.tables = a.tables;
   p.table_w = a.table_w;
   p.scale_log2 = a.scale_log2;
+  p.kv_first = g_fa_kvfirst;
   return launch_pdl(prefill_attn_persist_kernel<HD, POLY>, dim3(n_cta), dim3(C::kThreads), C::kSmem, st, *a.kv_tmap,
                     *qmp, p, items, cta_off);
 }
 
+template <int POLY>
+static cudaError_t prefill_pair_t(const AttnLaunch& a, const PrefillItem* items, const int32_t* cta_off, int n_pairs,
+                                  cudaStream_t st) {
+  using C = PairCfg;
+  const int group = a.H / a.Hkv;
+  CUtensorMap qm;
+  const CUtensorMap* qmp = a.q_tmap;
+  if (!qmp) {
+    if (make_tmap_3d_bf16_strided(&qm, a.q, uint64_t(C::HD), uint64_t(a.H), uint64_t(a.q_rows), uint64_t(C::HD) * 2,
+                                  uint64_t(a.q_ld) * 2, 64, uint32_t(group), uint32_t(C::kRows / group)) != QOS_OK)
+      return cudaErrorInvalidValue;
+    qmp = &qm;
+  }
+  static std::atomic<uint64_t> set{0};
+  if (cudaError_t e = smem_attr_once(prefill_attn_pair_kernel<POLY>, int(C::kSmem), set); e != cudaSuccess) return e;
+  FaParams p;
+  p.q = reinterpret_cast<const __nv_bfloat16*>(a.q);
+  p.q_ld = a.q_ld;
+  p.out = a.out;
+  p.out_ld = a.out_ld;
+  p.out_f32 = a.out_f32;
+  p.layer = a.layer;
+  p.H = a.H;
+  p.Hkv = a.Hkv;
+  p.tables = a.tables;
+  p.table_w = a.table_w;
+  p.scale_log2 = a.scale_log2;
+  return launch_pdl_cluster(prefill_attn_pair_kernel<POLY>, dim3(2 * n_pairs), dim3(C::kThreads), C::kSmem, 2, st,
+                            *a.kv_tmap, *qmp, p, items, cta_off);
+}
+
+int prefill_pair_max_clusters() {
+  static std::atomic<uint64_t> set{0};
+  if (smem_attr_once(prefill_attn_pair_kernel<4>, int(PairCfg::kSmem), set) != cudaSuccess) return 0;
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(2);
+  cfg.blockDim = dim3(PairCfg::kThreads);
+  cfg.dynamicSmemBytes = PairCfg::kSmem;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = 2;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  int n = 0;
+  if (cudaOccupancyMaxActiveClusters(&n, prefill_attn_pair_kernel<4>, &cfg) != cudaSuccess) {
+    cudaGetLastError();
+    return 0;
+  }
+  return n;
+}
+
 void set_fa_poly(int n) { g_fa_poly = n; }
+void set_fa_kvfirst(int v) { g_fa_kvfirst = v; }
 
 int prefill_tc_positions_per_tile(int group) { return 128 / group; }
 
@@ -1110,6 +1488,10 @@ cudaError_t launch_prefill_attention_tc(const AttnLaunch& a, const PrefillItem* 
   if (n_items == 0) return cudaSuccess;
   count_launch(1);
   const int poly = g_fa_poly;
+  if (a.pair) {  // CTA pairs over per-pair lists of q-tile pairs (cta_off in pairs of items)
+    if (a.hd != 128 || !a.cta_off || a.q_tiles != 2) return cudaErrorInvalidValue;
+    return poly == 0 ? prefill_pair_t<0>(a, items, a.cta_off, a.n_cta, st) : prefill_pair_t<4>(a, items, a.cta_off, a.n_cta, st);
+  }
   if (a.cta_off && a.q_tiles == 1 && poly >= 0) {  // persistent CTAs over per-CTA item lists
     if (a.hd == 128) return poly == 0   ? prefill_persist_t<128, 0>(a, items, a.cta_off, a.n_cta, st)
                             : poly == 2 ? prefill_persist_t<128, 2>(a, items, a.cta_off, a.n_cta, st)

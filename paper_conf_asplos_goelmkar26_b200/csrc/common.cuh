@@ -148,6 +148,13 @@ QOS_DEV uint32_t mapa_shared(uint32_t addr, uint32_t rank) {
 QOS_DEV void mbar_arrive_cluster(uint32_t cluster_addr) {
   asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
 }
+// the same with the default (.release.cta) semantics, as CUTLASS's ClusterBarrier::arrive(cta_id):
+// for arrivals that order only tcgen05 (TMEM) accesses, which the tcgen05 fences around the
+// barrier already order.  The .cluster release costs a MEMBAR.ALL.GPU per arrival (SASS), i.e.
+// waits for every outstanding global store of the thread.
+QOS_DEV void mbar_arrive_remote(uint32_t cluster_addr) {
+  asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
+}
 template <uint32_t kCols>
 QOS_DEV void tmem_alloc2(uint32_t* dst_smem) {  // one warp in each CTA of the pair
   asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(dst_smem)),
@@ -183,6 +190,23 @@ QOS_DEV void tma_load_2d_2cta(void* dst, const void* tmap, uint32_t bar_cluster,
       "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
       " [%0], [%1, {%3, %4}], [%2], %5;" ::"r"(smem_u32(dst)),
       "l"(reinterpret_cast<uint64_t>(tmap)), "r"(bar_cluster), "r"(c0), "r"(c1), "l"(policy)
+      : "memory");
+}
+
+QOS_DEV void tma_load_3d_2cta(void* dst, const void* tmap, uint32_t bar_cluster, int32_t c0, int32_t c1, int32_t c2) {
+  asm volatile(
+      "cp.async.bulk.tensor.3d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(tmap)), "r"(bar_cluster), "r"(c0), "r"(c1), "r"(c2)
+      : "memory");
+}
+// D[tmem of both CTAs] (+)= A[tmem: 128 rows per CTA] · B[N: N/2 per CTA], kind::f16; issued by CTA 0
+QOS_DEV void umma_ts_2cta(uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc, uint32_t idesc, uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], [%1], %2, %3, p;\n\t}" ::"r"(d_tmem),
+      "r"(a_tmem), "l"(b_desc), "r"(idesc), "r"(accumulate)
       : "memory");
 }
 

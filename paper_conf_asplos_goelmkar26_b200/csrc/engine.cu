@@ -219,6 +219,7 @@ struct StepMeta {
   int T = 0, R = 0, n_prefill = 0, n_decode = 0;
   int n_pitems = 0, n_ditems = 0, n_upd = 0;
   int fa_qtiles = 1;  // prefill items come in groups of this many q tiles (one CTA each group)
+  int fa_pair = 0;    // prefill attention on CTA pairs (groups of 2 q tiles; n_pcta = pairs)
   int n_pcta = 0;     // persistent prefill attention: CTAs (0: one CTA per item group)
   size_t o_pcta = 0;  // offsets [n_pcta + 1] into the prefill items
   // offsets (bytes) inside the metadata block
@@ -381,6 +382,8 @@ struct qos_engine {
   int decode_stages = 8;            // option decode_stages: decode K/V ring depth (8 or 4)
   int fa_qtiles = 1;                // option fa_qtiles: prefill q tiles per CTA sharing K/V tiles
   bool fa_persist = true;           // option fa_persist: persistent prefill-attention CTAs (fa_qtiles 1)
+  bool fa_pair = false;             // option fa_pair: prefill attention on CTA pairs (cta_group::2, hd 128)
+  int pair_clusters = -1;           // co-resident pairs of that kernel (queried once)
   bool norm_fold = true;            // option norm_fold: RMSNorm folded into the O / down and QKV / gate-up GEMMs
   bool overlap_attn = true;       // QOS_OVERLAP_ATTN=0 serialises a7 and a8 (for measurement)
   bool gemm_splitk = false;       // QOS_GEMM_SPLITK=1: split-K for small-M tile GEMMs (measured slower on
@@ -560,7 +563,8 @@ int build_step(qos_engine* e, const qos_batch* b, bool check_lengths, uint8_t* b
 
   const int group = c.n_heads / c.n_kv_heads;
   const int ppt = prefill_tc_positions_per_tile(group);
-  const int CS = e->fa_qtiles;
+  const bool pair = e->fa_pair && c.head_dim == 128 && e->fa_qtiles == 1 && e->fa_persist;
+  const int CS = pair ? 2 : e->fa_qtiles;
   std::vector<PrefillItem> pitems;
   int t = 0;
   for (int i = 0; i < b->n_prefill; ++i) {
@@ -638,6 +642,35 @@ int build_step(qos_engine* e, const qos_batch* b, bool check_lengths, uint8_t* b
     }
     pitems.swap(dealt);
     m.n_pcta = G;
+  } else if (pair && !pitems.empty()) {
+    // CTA pairs: the LPT-sorted groups of 2 q tiles dealt greedily to the co-resident pairs
+    // (2 per SM pair); offsets count groups
+    if (e->pair_clusters < 0) e->pair_clusters = prefill_pair_max_clusters();
+    if (e->pair_clusters <= 0) return set_error(QOS_ERR_CUDA, "prefill pair kernel: no co-resident CTA pair");
+    const size_t ngrp = pitems.size() / 2;
+    const int G = int(std::min<size_t>({ngrp, size_t(e->pair_clusters), size_t(1024)}));
+    std::priority_queue<std::pair<int64_t, int>, std::vector<std::pair<int64_t, int>>, std::greater<>> heap;
+    for (int g = 0; g < G; ++g) heap.push({0, g});
+    std::vector<std::vector<int>> lists(static_cast<size_t>(G));
+    for (size_t i = 0; i < ngrp; ++i) {
+      auto [load, g] = heap.top();
+      heap.pop();
+      lists[size_t(g)].push_back(int(i));
+      heap.push({load + pitems[2 * i].grp_last / 64 + 1 + 2, g});
+    }
+    std::vector<PrefillItem> dealt;
+    dealt.reserve(pitems.size());
+    pcta.push_back(0);
+    for (const auto& li : lists) {
+      for (int i : li) {
+        dealt.push_back(pitems[2 * size_t(i)]);
+        dealt.push_back(pitems[2 * size_t(i) + 1]);
+      }
+      pcta.push_back(int32_t(dealt.size() / 2));
+    }
+    pitems.swap(dealt);
+    m.n_pcta = G;
+    m.fa_pair = 1;
   }
   // decode split-K work list (balanced on sum of keys)
   int64_t total_keys = 0;
@@ -974,6 +1007,7 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
   al.q_tiles = m.fa_qtiles;
   al.cta_off = m.n_pcta ? reinterpret_cast<const int32_t*>(dm + m.o_pcta) : nullptr;
   al.n_cta = m.n_pcta;
+  al.pair = m.fa_pair;
   al.q_tmap = &e->q_map;
   al.q_rows = c.max_batch_tokens;
   al.decode_stages = e->decode_stages;
@@ -1911,6 +1945,7 @@ int qos_engine_set_option(qos_engine_t* e, const char* name, int64_t value) {
   }
   else if (n == "gemm_2cta") e->gemm_2cta = value != 0;
   else if (n == "fa_persist") e->fa_persist = value != 0;
+  else if (n == "fa_pair") e->fa_pair = value != 0;
   else if (n == "norm_fold") e->norm_fold = value != 0;
   else if (n == "tp_scatter") e->tp_scatter = value != 0;
   else if (n == "attn_order") {
@@ -1929,6 +1964,8 @@ int qos_engine_set_option(qos_engine_t* e, const char* name, int64_t value) {
   else if (n == "gemm_splitk") e->gemm_splitk = value != 0;
   else if (n == "pdl") set_pdl(value != 0);  // process-wide
   else if (n == "fa_poly") set_fa_poly(int(value));  // process-wide
+  else if (n == "fa_kvfirst") set_fa_kvfirst(int(value != 0));  // process-wide
+  else if (n == "gemm2_rel_cluster") set_gemm2_rel_cluster(int(value != 0));  // process-wide (experiment)
   else if (n == "swab_gran") set_swab_gran(int(value));  // process-wide (experiments)
   else if (n == "gemm_swab") e->gemm_swab = int(value < 0 ? 0 : value > 2 ? 2 : value);
   else if (n == "gemm_streamk") e->gemm_streamk = int(value < 0 ? 0 : value > 2 ? 2 : value);
@@ -2171,6 +2208,7 @@ int qos_op_attention(qos_engine_t* e, int32_t layer, const qos_batch* b, const u
   al.q_tiles = m.fa_qtiles;
   al.cta_off = m.n_pcta ? reinterpret_cast<const int32_t*>(dm + m.o_pcta) : nullptr;
   al.n_cta = m.n_pcta;
+  al.pair = m.fa_pair;
   al.q_tmap = nullptr;  // per-launch map over the op's q buffer
   al.q_rows = m.T;
   al.decode_stages = e->decode_stages;

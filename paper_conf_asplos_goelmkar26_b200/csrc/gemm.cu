@@ -89,6 +89,7 @@ struct GemmArgs {
   float inv_d, rms_eps;
   void* scat[8];  // reduce-scatter destinations (NormFold::scat), scat_rs = 0: plain store to C
   int scat_rs;
+  int rel_cluster;  // CTA-pair kernel: accumulator release with .release.cluster (experiment; 0 = .cta)
 };
 
 static void set_fold(GemmArgs& a, const NormFold* f) {
@@ -1149,7 +1150,10 @@ __global__ void __launch_bounds__(kGemmThreads, 1)
       epi_tile_staged<BN, EPI>(p, stg, lane, n_t, row, tmem_base + (uint32_t(q * 32) << 16) + acc * BN);
       tc_fence_before();
       __syncwarp();
-      if (lane == 0) mbar_arrive_cluster(tempty_leader + acc * 8);
+      if (lane == 0) {
+        if (p.rel_cluster) mbar_arrive_cluster(tempty_leader + acc * 8);
+        else mbar_arrive_remote(tempty_leader + acc * 8);
+      }
       if (++acc == 2) { acc = 0; acc_phase ^= 1; }
     }
   }
@@ -1395,6 +1399,11 @@ bool gemm2_eligible(int64_t M, int64_t N, int64_t K, int num_sms) {
 }
 
 // tb: tensor map over B with 128-row boxes; ta: over A with 128-row boxes
+// accumulator release of the CTA-pair epilogue: 0 = .release.cta remote arrive (default; the
+// .cluster form costs a MEMBAR.ALL.GPU per arrival, waiting for the epilogue's global stores)
+static int g_gemm2_rel_cluster = 0;
+void set_gemm2_rel_cluster(int v) { g_gemm2_rel_cluster = v; }
+
 int gemm2_run(const CUtensorMap& ta, const CUtensorMap& tb, int64_t M, int64_t N, int64_t K, int epi, void* C,
               int64_t ldc, const float* bias, int num_sms, cudaStream_t st, int a_row0, int max_ctas,
               const QkvRopeArgs* rope, const NormFold* fold) {
@@ -1420,6 +1429,7 @@ int gemm2_run(const CUtensorMap& ta, const CUtensorMap& tb, int64_t M, int64_t N
   a.hd = rope ? rope->hd : 0;
   if (epi == EPI_QKV_ROPE && (!rope || a.hd <= 0 || 256 % a.hd))
     return set_error(QOS_ERR_INVALID_ARG, "gemm2: QKV_ROPE needs rope args and 256 % hd == 0");
+  a.rel_cluster = g_gemm2_rel_cluster;
   const int units = a.mt * a.nt;
   int pairs = std::min(units, (max_ctas > 0 ? std::min(max_ctas, num_sms) : num_sms) / 2);
   if (pairs < 1) pairs = 1;

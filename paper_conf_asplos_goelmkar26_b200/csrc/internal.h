@@ -14,6 +14,8 @@ bool pdl_enabled();
 void set_pdl(bool on);
 // prefill attention: every n-th exp2 pair on the FMA pipe (0 = all on MUFU); process-wide
 void set_fa_poly(int n);
+void set_fa_kvfirst(int v);
+void set_gemm2_rel_cluster(int v);  // process-wide experiment (gemm.cu)  // process-wide: persistent prefill attention loads K/V before Q
 void set_swab_gran(int v);  // weight-streaming GEMM range granule (k-blocks; -1 automatic, 0 whole tiles)
 
 enum { EPI_STORE_BF16 = QOS_EPI_STORE_BF16, EPI_STORE_F32 = QOS_EPI_STORE_F32, EPI_BIAS_BF16 = QOS_EPI_BIAS_BF16,
@@ -193,8 +195,10 @@ struct AttnLaunch {
   const CUtensorMap* q_tmap = nullptr;  // prefill, persistent mode: 3-D map {hd, H, rows} over q with a
                                         // {64, H/Hkv, 128/(H/Hkv)} box (NULL: built per launch)
   int q_rows = 0;                       // rows the q map covers (its dim 2)
-  int n_cta = 0;
+  int n_cta = 0;                        // persistent modes: CTAs (pair mode: CTA pairs)
+  int pair = 0;                         // prefill: CTA-pair kernel (cta_group::2; q_tiles 2, hd 128)
 };
+int prefill_pair_max_clusters();        // co-resident CTA pairs of the pair kernel (0: unavailable)
 cudaError_t launch_decode_attention(const AttnLaunch& a, const DecodeItem* items, int n_items, float* partials,
                                     int* counters, cudaStream_t st);
 cudaError_t launch_prefill_attention_tc(const AttnLaunch& a, const PrefillItem* items, int n_items, cudaStream_t st);

@@ -193,17 +193,19 @@ ATTN_CASES = [
 ]
 
 
-@pytest.mark.parametrize("qtiles,persist", [(1, 1), (1, 0), (2, 0)])
+@pytest.mark.parametrize("qtiles,persist,pair", [(1, 1, 0), (1, 0, 0), (2, 0, 0), (1, 1, 1)])
 @pytest.mark.parametrize("case", range(len(ATTN_CASES)))
-def test_attention_parity(case, qtiles, persist):
+def test_attention_parity(case, qtiles, persist, pair):
     """Prefill + decode attention (fp32 output) vs the fp64 oracle; prefill with 1 or 2 q tiles
-    per CTA sharing every K/V tile (odd tile counts padded with a duplicate), and the persistent
-    single-tile kernel (several work items per CTA)."""
+    per CTA sharing every K/V tile (odd tile counts padded with a duplicate), the persistent
+    single-tile kernel (several work items per CTA), and the persistent CTA-pair kernel
+    (cta_group::2, hd 128; hd 64 presets fall back to the single-CTA kernel)."""
     from oracle.model import causal_attention
     preset, over, chunks, ctxs, scale = ATTN_CASES[case]
     q, cfg, eng = make_engine(preset, **{"max_seq_len": 8192, "max_batch_tokens": 4096, **over})
     eng.qos_engine_set_option("fa_qtiles", qtiles)
     eng.qos_engine_set_option("fa_persist", persist)
+    eng.qos_engine_set_option("fa_pair", pair)
     H, Hkv, hd = cfg.n_heads, cfg.n_kv_heads, cfg.head_dim
     g = H // Hkv
     rng = np.random.default_rng(100 + case)

@@ -132,6 +132,31 @@ def test_batch_composition_invariance():
         assert np.abs(mixed[1 + i] - alone[0]).max() / np.abs(alone).max() < 1e-12
 
 
+@pytest.mark.parametrize("preset", ["tiny", "tiny-qwen"])
+def test_layer_major_step_equals_request_major_step(preset):
+    """hybrid_step_layer_major (layer loop outside, used for the full-depth bench-size check)
+    gives bit-identical logits and KV to hybrid_step (request loop outside) over the whole tiny
+    scenario: the same operations in the same order per request."""
+    cfg = PRESETS[preset]
+    ctxs, warm, main, second = synth.tiny_scenario(cfg.vocab)
+    a, b = _fresh(cfg), _fresh(cfg)
+    for e in (a, b):
+        for r, n in ctxs.items():
+            e.kv_alloc(r, n + 2)
+        e.kv_alloc(0, 256)
+    for st in warm + [main, second]:
+        la = a.hybrid_step(*st.as_oracle())
+        lb = b.hybrid_step_layer_major(*st.as_oracle())
+        assert np.array_equal(la, lb)
+    for r in list(ctxs) + [0]:
+        for l in range(cfg.n_layers):
+            assert np.array_equal(a.kv[r][l][0], b.kv[r][l][0]) and np.array_equal(a.kv[r][l][1], b.kv[r][l][1])
+    with pytest.raises(ValueError):
+        b.hybrid_step_layer_major([(0, 0, [1])], [(0, 0, 1)])
+    with pytest.raises(OracleBadKVStart):
+        b.hybrid_step_layer_major([(0, 3, [1])], [])
+
+
 def test_step_semantics_errors():
     cfg = PRESETS["tiny"]
     e = _fresh(cfg, nb=4)

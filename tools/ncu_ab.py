@@ -46,7 +46,8 @@ for v in [x for x in a.variants.split(";")] or [""]:
                 cyc.append(val)
         c, nd, ctx, ks = (int(x) for x in pt.split(":"))
         rec = {"variant": v, "point": pt, "launches": len(cyc), "kcycles_median": round(statistics.median(cyc) / 1e3, 1),
-               "us_median": round(statistics.median(us), 2)}
+               "us_median": round(statistics.median(us), 2),
+               "kcycles_sum": round(sum(cyc) / 1e3, 1)}
         if c and a.kernel.startswith("prefill"):
             fl = 4 * 128 * 32 * (c * ks + c * (c + 1) // 2)  # Llama-3-8B: hd 128, 32 heads
             rec["flop_per_cycle_per_sm"] = round(fl / (statistics.median(cyc) * 148), 1)
