@@ -150,6 +150,7 @@ struct FaParams {
   int table_w;
   float scale_log2;
   int kv_first = 0;  // persistent kernel: issue an item's first K/V tile before its Q (option fa_kvfirst)
+  int tma5 = 0;      // persistent kernel: a tile's 4 blocks in one 5-D box when their ids are consecutive
 };
 
 // Work item = NQ consecutive entries of `items`: q tiles of one (chunk, kv head) that share
@@ -453,8 +454,8 @@ __global__ void __launch_bounds__(FaCfg<HD, NQ>::kThreads, FaCfg<HD, NQ>::kMinBl
 template <int HD, int POLY>
 __global__ void __launch_bounds__(FaCfg<HD, 1>::kThreads, 2)
     prefill_attn_persist_kernel(const __grid_constant__ CUtensorMap kvmap, const __grid_constant__ CUtensorMap qmap,
-                                const FaParams p, const PrefillItem* __restrict__ items,
-                                const int32_t* __restrict__ cta_off) {
+                                const __grid_constant__ CUtensorMap kvmap5, const FaParams p,
+                                const PrefillItem* __restrict__ items, const int32_t* __restrict__ cta_off) {
   using C = FaCfg<HD, 1>;
   constexpr int S = C::kStages;
   extern __shared__ uint8_t smem_raw[];
@@ -520,26 +521,35 @@ __global__ void __launch_bounds__(FaCfg<HD, 1>::kThreads, 2)
         auto load_kv = [&](int j) {
           const int s = int(jg % S);
           const uint32_t ph = (jg / S) & 1;
-          int r[C::kKeys / 16];
+          constexpr int NB = C::kKeys / 16;
+          int id[NB];
 #pragma unroll
-          for (int b = 0; b < C::kKeys / 16; ++b)
-            r[b] = (__ldg(trow + min(j * (C::kKeys / 16) + b, last_blk)) * p.Hkv + it.kv_head) * 16;
+          for (int b = 0; b < NB; ++b) id[b] = __ldg(trow + min(j * NB + b, last_blk));
+          // the tile's blocks are one run of consecutive ids (the allocator hands out the lowest
+          // free ids, so a fresh request's blocks usually are): one 5-D box per 64-dim half
+          bool run = p.tma5 != 0 && j * NB + NB - 1 <= last_blk;
+#pragma unroll
+          for (int b = 1; b < NB; ++b) run = run && id[b] == id[0] + b;
+          auto load = [&](uint8_t* dst, uint64_t* full, int plane) {
+            if (run) {
+#pragma unroll
+              for (int hf = 0; hf < C::kHalves; ++hf)
+                tma_load_5d(dst + hf * (C::kKeys * 128), &kvmap5, full, hf * 64, 0, it.kv_head, id[0], p.layer * 2 + plane);
+            } else {
+#pragma unroll
+              for (int b = 0; b < NB; ++b)
+#pragma unroll
+                for (int hf = 0; hf < C::kHalves; ++hf)
+                  tma_load_3d(dst + hf * (C::kKeys * 128) + b * 2048, &kvmap, full, hf * 64,
+                              (id[b] * p.Hkv + it.kv_head) * 16, p.layer * 2 + plane);
+            }
+          };
           mbar_wait(&k_empty[s], ph ^ 1);
           mbar_arrive_expect_tx(&k_full[s], C::kTileBytes);
-#pragma unroll
-          for (int b = 0; b < C::kKeys / 16; ++b)
-#pragma unroll
-            for (int hf = 0; hf < C::kHalves; ++hf)
-              tma_load_3d(sK + s * C::kTileBytes + hf * (C::kKeys * 128) + b * 2048, &kvmap, &k_full[s], hf * 64, r[b],
-                          p.layer * 2);
+          load(sK + s * C::kTileBytes, &k_full[s], 0);
           mbar_wait(&v_empty[s], ph ^ 1);
           mbar_arrive_expect_tx(&v_full[s], C::kTileBytes);
-#pragma unroll
-          for (int b = 0; b < C::kKeys / 16; ++b)
-#pragma unroll
-            for (int hf = 0; hf < C::kHalves; ++hf)
-              tma_load_3d(sV + s * C::kTileBytes + hf * (C::kKeys * 128) + b * 2048, &kvmap, &v_full[s], hf * 64, r[b],
-                          p.layer * 2 + 1);
+          load(sV + s * C::kTileBytes, &v_full[s], 1);
           ++jg;
         };
         // with kv_first the item's first K/V tile goes out before its Q, which has to wait for
@@ -1347,6 +1357,7 @@ __global__ void __launch_bounds__(PpCfg<HD>::kThreads, 1)
 }
 
 static int g_fa_poly = getenv("QOS_FA_POLY") ? atoi(getenv("QOS_FA_POLY")) : 4;
+static int g_fa_tma5 = 1;
 static int g_fa_kvfirst = 0;  // neutral in ncu cycles (profiles/ncu_ab_fa_r2c.jsonl)
 
 template <int HD, int POLY, int NQ>
@@ -1422,8 +1433,9 @@ static cudaError_t prefill_persist_t(const AttnLaunch& a, const PrefillItem* ite
   p.table_w = a.table_w;
   p.scale_log2 = a.scale_log2;
   p.kv_first = g_fa_kvfirst;
+  p.tma5 = (g_fa_tma5 && a.kv_tmap5) ? 1 : 0;
   return launch_pdl(prefill_attn_persist_kernel<HD, POLY>, dim3(n_cta), dim3(C::kThreads), C::kSmem, st, *a.kv_tmap,
-                    *qmp, p, items, cta_off);
+                    *qmp, a.kv_tmap5 ? *a.kv_tmap5 : *a.kv_tmap, p, items, cta_off);
 }
 
 template <int POLY>
@@ -1481,6 +1493,7 @@ int prefill_pair_max_clusters() {
 
 void set_fa_poly(int n) { g_fa_poly = n; }
 void set_fa_kvfirst(int v) { g_fa_kvfirst = v; }
+void set_fa_tma5(int v) { g_fa_tma5 = v; }
 
 int prefill_tc_positions_per_tile(int group) { return 128 / group; }
 

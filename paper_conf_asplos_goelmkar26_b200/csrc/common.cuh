@@ -97,6 +97,14 @@ QOS_DEV void tma_load_3d(void* dst, const void* tmap, uint64_t* bar, int32_t c0,
       "l"(reinterpret_cast<uint64_t>(tmap)), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "r"(c2)
       : "memory");
 }
+QOS_DEV void tma_load_5d(void* dst, const void* tmap, uint64_t* bar, int32_t c0, int32_t c1, int32_t c2, int32_t c3,
+                         int32_t c4) {
+  asm volatile(
+      "cp.async.bulk.tensor.5d.shared::cluster.global.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%3, %4, %5, %6, %7}], [%2];" ::"r"(smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(tmap)), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(c4)
+      : "memory");
+}
 // L2 eviction-priority policies (createpolicy) for streamed vs re-used operands.
 QOS_DEV uint64_t l2_evict_first() {
   uint64_t p;

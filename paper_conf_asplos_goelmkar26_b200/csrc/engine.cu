@@ -348,6 +348,7 @@ struct qos_engine {
   };
   ActMap a_h, a_attn, a_act, a_hR;
   CUtensorMap kv_map;
+  CUtensorMap kv_map5;  // the same pool, 4 consecutive blocks of one head per box (prefill attention)
   CUtensorMap q_map;  // {hd, H, max_batch_tokens} over the q columns of `qkv` (prefill attention's Q tiles)
   float2* rope_tab = nullptr;
   int32_t* d_tables = nullptr;
@@ -484,6 +485,7 @@ int build_maps(qos_engine* e) {
   QOS_TRY(act(e->a_hR, e->ws + s.hR, c.max_batch_rows, d));
   QOS_TRY(make_tmap_3d_bf16(&e->kv_map, e->kv, hd, uint64_t(c.num_blocks) * e->sh.Hkv * 16, uint64_t(c.n_layers) * 2,
                             64, 16, 1));
+  QOS_TRY(make_tmap_kv5(&e->kv_map5, e->kv, hd, uint64_t(e->sh.Hkv), uint64_t(c.num_blocks), uint64_t(c.n_layers) * 2, 4));
   {
     const int group = c.n_heads / c.n_kv_heads;
     QOS_TRY(make_tmap_3d_bf16_strided(&e->q_map, e->ws + s.qkv, uint64_t(hd), uint64_t(e->sh.H),
@@ -997,6 +999,7 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
   al.out_ld = e->sh.H * hd;
   al.out_f32 = 0;
   al.kv_tmap = &e->kv_map;
+  al.kv_tmap5 = &e->kv_map5;
   al.H = e->sh.H;
   al.Hkv = e->sh.Hkv;
   al.hd = hd;
@@ -1965,6 +1968,7 @@ int qos_engine_set_option(qos_engine_t* e, const char* name, int64_t value) {
   else if (n == "pdl") set_pdl(value != 0);  // process-wide
   else if (n == "fa_poly") set_fa_poly(int(value));  // process-wide
   else if (n == "fa_kvfirst") set_fa_kvfirst(int(value != 0));  // process-wide
+  else if (n == "fa_tma5") set_fa_tma5(int(value != 0));  // process-wide
   else if (n == "gemm2_rel_cluster") set_gemm2_rel_cluster(int(value != 0));  // process-wide (experiment)
   else if (n == "swab_gran") set_swab_gran(int(value));  // process-wide (experiments)
   else if (n == "gemm_swab") e->gemm_swab = int(value < 0 ? 0 : value > 2 ? 2 : value);
@@ -2197,6 +2201,7 @@ int qos_op_attention(qos_engine_t* e, int32_t layer, const qos_batch* b, const u
   al.out_ld = int(qrow);
   al.out_f32 = 1;
   al.kv_tmap = &e->kv_map;
+  al.kv_tmap5 = &e->kv_map5;
   al.layer = layer;
   al.H = e->sh.H;
   al.Hkv = e->sh.Hkv;

@@ -1231,6 +1231,21 @@ int make_tmap_3d_bf16_strided(CUtensorMap* out, const void* base, uint64_t d0, u
   return QOS_OK;
 }
 
+int make_tmap_kv5(CUtensorMap* out, const void* base, uint64_t hd, uint64_t hkv, uint64_t num_blocks, uint64_t planes,
+                  uint32_t blocks_per_box) {
+  auto fn = get_encode_fn();
+  if (!fn) return set_error(QOS_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+  cuuint64_t dims[5] = {hd, 16, hkv, num_blocks, planes};
+  cuuint64_t strides[4] = {hd * 2, 16 * hd * 2, hkv * 16 * hd * 2, num_blocks * hkv * 16 * hd * 2};
+  cuuint32_t box[5] = {64, 16, 1, blocks_per_box, 1};
+  cuuint32_t estr[5] = {1, 1, 1, 1, 1};
+  CUresult r = fn(out, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 5, const_cast<void*>(base), dims, strides, box, estr,
+                  CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return set_error(QOS_ERR_CUDA, "cuTensorMapEncodeTiled (kv 5d) failed");
+  return QOS_OK;
+}
+
 template <int BN, int EPI>
 static cudaError_t launch_gemm_t(const CUtensorMap& ta, const CUtensorMap& tb, const GemmArgs& a, int grid,
                                  cudaStream_t st) {

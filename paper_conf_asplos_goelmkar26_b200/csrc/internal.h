@@ -15,6 +15,7 @@ void set_pdl(bool on);
 // prefill attention: every n-th exp2 pair on the FMA pipe (0 = all on MUFU); process-wide
 void set_fa_poly(int n);
 void set_fa_kvfirst(int v);
+void set_fa_tma5(int v);  // process-wide: persistent prefill attention loads 4-block runs in one TMA op
 void set_gemm2_rel_cluster(int v);  // process-wide experiment (gemm.cu)  // process-wide: persistent prefill attention loads K/V before Q
 void set_swab_gran(int v);  // weight-streaming GEMM range granule (k-blocks; -1 automatic, 0 whole tiles)
 
@@ -43,6 +44,10 @@ int make_tmap_3d_bf16(CUtensorMap* out, const void* base, uint64_t d0, uint64_t 
                       uint32_t b1, uint32_t b2);
 int make_tmap_3d_bf16_strided(CUtensorMap* out, const void* base, uint64_t d0, uint64_t d1, uint64_t d2, uint64_t s1,
                               uint64_t s2, uint32_t b0, uint32_t b1, uint32_t b2);
+// KV pool [2L][num_blocks][Hkv][16][hd] as a 5-D map {hd, 16, Hkv, num_blocks, 2L} with a
+// {64, 16, 1, blocks_per_box, 1} box: runs of consecutive blocks of one head in one TMA op
+int make_tmap_kv5(CUtensorMap* out, const void* base, uint64_t hd, uint64_t hkv, uint64_t num_blocks, uint64_t planes,
+                  uint32_t blocks_per_box);
 int gemm_pick_bn(int64_t M, int64_t N, int epi, int num_sms);
 int gemm_check_shape(int64_t M, int64_t N, int64_t K, int epi);
 int gemm_pick_ksplit(int64_t M, int64_t N, int64_t K, int bn, int num_sms, int64_t max_units);
@@ -197,6 +202,7 @@ struct AttnLaunch {
   int q_rows = 0;                       // rows the q map covers (its dim 2)
   int n_cta = 0;                        // persistent modes: CTAs (pair mode: CTA pairs)
   int pair = 0;                         // prefill: CTA-pair kernel (cta_group::2; q_tiles 2, hd 128)
+  const CUtensorMap* kv_tmap5 = nullptr;  // prefill, persistent: 5-D map, 4-block boxes (make_tmap_kv5)
 };
 int prefill_pair_max_clusters();        // co-resident CTA pairs of the pair kernel (0: unavailable)
 cudaError_t launch_decode_attention(const AttnLaunch& a, const DecodeItem* items, int n_items, float* partials,
