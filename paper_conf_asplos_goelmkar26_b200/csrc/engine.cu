@@ -381,6 +381,7 @@ struct qos_engine {
                                    // (4096: 5-10% faster decode attention than 512 on B200,
                                    // profiles/decode_split_ab_r1k.jsonl)
   int decode_stages = 8;            // option decode_stages: decode K/V ring depth (8 or 4)
+  bool decode_persist = false;      // option decode_persist: persistent decode-attention CTAs
   int fa_qtiles = 1;                // option fa_qtiles: prefill q tiles per CTA sharing K/V tiles
   bool fa_persist = true;           // option fa_persist: persistent prefill-attention CTAs (fa_qtiles 1)
   bool fa_pair = false;             // option fa_pair: prefill attention on CTA pairs (cta_group::2, hd 128)
@@ -1014,6 +1015,7 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
   al.q_tmap = &e->q_map;
   al.q_rows = c.max_batch_tokens;
   al.decode_stages = e->decode_stages;
+  al.decode_persist = e->decode_persist ? 1 : 0;
   const int n_pre_rows = T - m.n_decode;
   float* gpart0 = reinterpret_cast<float*>(e->ws + s.gemm_part);
   int* gcnt0 = reinterpret_cast<int*>(e->ws + s.gemm_cnt);
@@ -1949,6 +1951,7 @@ int qos_engine_set_option(qos_engine_t* e, const char* name, int64_t value) {
   else if (n == "gemm_2cta") e->gemm_2cta = value != 0;
   else if (n == "fa_persist") e->fa_persist = value != 0;
   else if (n == "fa_pair") e->fa_pair = value != 0;
+  else if (n == "decode_persist") e->decode_persist = value != 0;
   else if (n == "norm_fold") e->norm_fold = value != 0;
   else if (n == "tp_scatter") e->tp_scatter = value != 0;
   else if (n == "attn_order") {
@@ -2217,6 +2220,7 @@ int qos_op_attention(qos_engine_t* e, int32_t layer, const qos_batch* b, const u
   al.q_tmap = nullptr;  // per-launch map over the op's q buffer
   al.q_rows = m.T;
   al.decode_stages = e->decode_stages;
+  al.decode_persist = e->decode_persist ? 1 : 0;
   QOS_CU(launch_prefill_attention_tc(al, reinterpret_cast<const PrefillItem*>(dm + m.o_pitems), m.n_pitems, st));
   QOS_CU(launch_decode_attention(al, reinterpret_cast<const DecodeItem*>(dm + m.o_ditems), m.n_ditems,
                                  reinterpret_cast<float*>(e->ws + e->wsl.partials),

@@ -196,6 +196,7 @@ struct AttnLaunch {
   float scale_log2;       // log2(e) / sqrt(hd)
   int q_tiles = 1;        // prefill: q tiles per CTA sharing every K/V tile (1 or 2)
   int decode_stages = 8;  // decode: K/V ring depth in (block, head) tiles (8 or 4)
+  int decode_persist = 0; // decode: persistent CTAs looping over the item list (ring depth 8)
   const int32_t* cta_off = nullptr;  // prefill, persistent mode: CTA c runs items [cta_off[c], cta_off[c+1])
   const CUtensorMap* q_tmap = nullptr;  // prefill, persistent mode: 3-D map {hd, H, rows} over q with a
                                         // {64, H/Hkv, 128/(H/Hkv)} box (NULL: built per launch)

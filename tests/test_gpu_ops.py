@@ -193,19 +193,22 @@ ATTN_CASES = [
 ]
 
 
-@pytest.mark.parametrize("qtiles,persist,pair", [(1, 1, 0), (1, 0, 0), (2, 0, 0), (1, 1, 1)])
+@pytest.mark.parametrize("qtiles,persist,pair,dpersist", [(1, 1, 0, 0), (1, 0, 0, 0), (2, 0, 0, 0), (1, 1, 1, 0),
+                                                     (1, 1, 0, 1)])
 @pytest.mark.parametrize("case", range(len(ATTN_CASES)))
-def test_attention_parity(case, qtiles, persist, pair):
+def test_attention_parity(case, qtiles, persist, pair, dpersist):
     """Prefill + decode attention (fp32 output) vs the fp64 oracle; prefill with 1 or 2 q tiles
     per CTA sharing every K/V tile (odd tile counts padded with a duplicate), the persistent
     single-tile kernel (several work items per CTA), and the persistent CTA-pair kernel
-    (cta_group::2, hd 128; hd 64 presets fall back to the single-CTA kernel)."""
+    (cta_group::2, hd 128; hd 64 presets fall back to the single-CTA kernel); decode attention
+    one CTA per item or persistent CTAs over the item list (dpersist)."""
     from oracle.model import causal_attention
     preset, over, chunks, ctxs, scale = ATTN_CASES[case]
     q, cfg, eng = make_engine(preset, **{"max_seq_len": 8192, "max_batch_tokens": 4096, **over})
     eng.qos_engine_set_option("fa_qtiles", qtiles)
     eng.qos_engine_set_option("fa_persist", persist)
     eng.qos_engine_set_option("fa_pair", pair)
+    eng.qos_engine_set_option("decode_persist", dpersist)
     H, Hkv, hd = cfg.n_heads, cfg.n_kv_heads, cfg.head_dim
     g = H // Hkv
     rng = np.random.default_rng(100 + case)

@@ -263,7 +263,7 @@ def test_llama8b_shapes_bench_batch_sampled_parity(split):
                                   {"gemm_swab": 2}, {"decode_round_split": 0}, {"fa_poly": 0}, {"fa_poly": 2},
                                   {"fa_qtiles": 2}, {"fa_persist": 0}, {"gemm_2cta": 0},
                                   {"norm_fold": 0}, {"gemm_swab": 0, "norm_fold": 1}, {"attn_order": 1}, {"gemm_swab": 0, "gemm_2cta": 0}, {"decode_stages": 4},
-                                  {"decode_split": 64}, {"decode_split": 4096},
+                                  {"decode_split": 64}, {"decode_split": 4096}, {"decode_persist": 1},
                                   {"dual_stream": 1, "dual_min_prefill": 1, "dual_min_decode": 1},
                                   {"add_split": 0}, {"shares_device": 1}])
 def test_execution_options_do_not_change_results(opts):
