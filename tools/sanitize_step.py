@@ -63,7 +63,8 @@ def decode_only(engs, vocab):
 
 def wide():
     """Llama-3-8B width, 2 layers: a 2048-token chunk + 16 decodes @1k (CTA-pair GEMMs with the
-    folded norm, persistent prefill attention over 512 items, split decode attention)."""
+    folded norm, persistent prefill attention over 512 items with 5-D K/V boxes, split decode
+    attention), then a second step with the CTA-pair prefill and persistent decode kernels."""
     cfg = q.model_cfg(**preset("llama3-8b", n_layers=2), num_blocks=(2048 + 16 * 1100) // 16 + 64,
                       max_seq_len=4096, max_requests=32, max_batch_tokens=2048 + 16, max_batch_rows=17)
     eng = q.Engine(cfg)
@@ -74,6 +75,16 @@ def wide():
         eng.qos_kv_alloc(d.req, 1025)
         eng.qos_kv_fill_synthetic(d.req, 1024, 2)
     eng.step_host(q.batch_from_synth(b), cfg.vocab)
+    # the round-2 options: CTA-pair prefill attention (cta_group::2) and persistent decode
+    # attention, on a second chunk and the decodes' next positions
+    eng.qos_engine_set_option("fa_pair", 1)
+    eng.qos_engine_set_option("decode_persist", 1)
+    eng.qos_kv_alloc(1, 2048)
+    for d in b.decode:
+        eng.qos_kv_alloc(d.req, 1026)
+    b2 = q.make_batch([(1, 0, np.asarray(b.prefill[0].tokens, dtype=np.int32))],
+                      [(d.req, 1025, d.token) for d in b.decode])
+    eng.step_host(b2, cfg.vocab)
     eng.close()
     print("sanitize workload done")
 
