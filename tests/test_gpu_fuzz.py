@@ -24,14 +24,79 @@ pytestmark = pytest.mark.gpu
 NARROW = dict(n_layers=2, d_model=512, n_heads=4, n_kv_heads=1, ffn_dim=1024, vocab=2048)
 
 
-def _run_trace(preset, over, seed, steps=60, opts=None):
+class _Ranks:
+    """The engines of one TP peer group driven as one (every call on every rank, one host thread
+    per rank); step_host checks that every rank returns bit-identical logits and tokens."""
+
+    def __init__(self, q, cfg, tp):
+        self.q, self.g = q, q.Group(tp)
+        self.engs = [q.Engine(cfg, 0, r, tp, group=self.g) for r in range(tp)]
+
+    def _all(self, fn):
+        return self.q.run_ranks(lambda k, e: fn(e), self.engs)
+
+    def qos_engine_load_synthetic(self, seed):
+        self._all(lambda e: e.qos_engine_load_synthetic(seed))
+
+    def qos_engine_set_option(self, k, v):
+        for e in self.engs:
+            e.qos_engine_set_option(k, v)
+
+    def qos_kv_alloc(self, r, n):
+        errs = []
+        for e in self.engs:
+            try:
+                e.qos_kv_alloc(r, n)
+            except self.q.QosError as x:
+                errs.append(x)
+        assert len(errs) in (0, len(self.engs))  # identical allocators on every rank
+        if errs:
+            raise errs[0]
+
+    def qos_kv_free(self, r):
+        for e in self.engs:
+            e.qos_kv_free(r)
+
+    def step_host(self, kb, vocab):
+        outs = self._all(lambda e: e.step_host(kb, vocab))
+        for lg, tk in outs[1:]:
+            assert np.array_equal(lg, outs[0][0]) and np.array_equal(tk, outs[0][1])
+        return outs[0]
+
+    def qos_kv_table(self, r):
+        t = [e.qos_kv_table(r) for e in self.engs]
+        assert all(x == t[0] for x in t)
+        return t[0]
+
+    def qos_kv_table_device(self, r):
+        t = [e.qos_kv_table_device(r) for e in self.engs]
+        assert all(x == t[0] for x in t)
+        return t[0]
+
+    def qos_kv_free_blocks(self):
+        n = [e.qos_kv_free_blocks() for e in self.engs]
+        assert all(x == n[0] for x in n)
+        return n[0]
+
+    def close(self):
+        for e in self.engs:
+            e.close()
+        self.g.close()
+
+
+def _run_trace(preset, over, seed, steps=60, opts=None, tp=1):
     from oracle.engine import OracleEngine
     from oracle.kv import OracleOOM
     from oracle.model import PRESETS
     rng = np.random.default_rng(seed)
     NB = 320 if seed != 3 else 120  # seed 3: a pool small enough that reservations are refused
-    q, cfg, eng = make_engine(preset, num_blocks=NB, max_seq_len=1024, max_requests=64, max_batch_tokens=512,
-                              max_batch_rows=16, **over)
+    caps = dict(num_blocks=NB, max_seq_len=1024, max_requests=64, max_batch_tokens=512, max_batch_rows=16)
+    q, cfg, eng = make_engine(preset, **caps, **over) if tp == 1 else (None, None, None)
+    if tp > 1:
+        from paper_conf_asplos_goelmkar26_b200 import qoserve as q
+        from paper_conf_asplos_goelmkar26_b200.presets import preset as mk_preset
+        cfg = q.model_cfg(**mk_preset(preset, **over), **caps)
+        eng = _Ranks(q, cfg, tp)
     eng.qos_engine_load_synthetic(0)
     for k, v in (opts or {}).items():
         eng.qos_engine_set_option(k, v)
@@ -136,3 +201,17 @@ def test_random_serving_trace_under_execution_options(opts):
     per-block K/V boxes)."""
     worst, stats = _run_trace("llama3-8b", NARROW, 7, steps=40, opts=opts)
     print(f"{opts}: worst row error {worst:.3e} {stats}")
+
+
+@pytest.mark.parametrize("preset,over,tp,opts", [("tiny", {}, 2, {}), ("tiny-qwen", {}, 2, {"tp_twoshot": 1}),
+                                                 ("tiny-mha", {"ffn_dim": 1024}, 4, {}),
+                                                 ("tiny-mha", {"ffn_dim": 1024}, 4, {"gemm_swab": 0}),
+                                                 ("llama3-8b", dict(NARROW, n_kv_heads=2), 2, {})])
+def test_random_serving_trace_tensor_parallel(preset, over, tp, opts):
+    """The same traces on a TP peer group (ranks as engines of one process on cuda:0: q/kv heads,
+    FFN columns and vocab rows sharded, the library's fused peer reduce + residual + RMSNorm and
+    logits gather) against the UNSHARDED oracle; every rank bit-identical every step.
+    gemm_swab 0 puts the O / down projections on the tile kernels with the reduce-scatter in
+    their epilogue (tp_scatter)."""
+    worst, stats = _run_trace(preset, over, 5, steps=40, opts=opts, tp=tp)
+    print(f"{preset} tp{tp} {opts}: worst row error {worst:.3e} {stats}")
