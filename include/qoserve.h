@@ -217,6 +217,17 @@ typedef struct {
  * (INVALID_ARG, UNKNOWN_REQ, BAD_KV_START, NOT_ALLOCATED); state is then unchanged. */
 int qos_hybrid_step(qos_engine_t* eng, const qos_batch* batch, void* logits, int logits_dtype,
                     int32_t* next_tokens, int outputs_on_host, void* stream);
+/* The same, with the decodes' input tokens read from DEVICE memory when the step runs:
+ * decode_tokens_dev[i] (int32, device, >= n_decode entries) replaces batch->decode[i].token, so
+ * a serving loop can feed one step's next_tokens (device, e.g. next_tokens + n_prefill of the
+ * previous step when the decode set keeps its order) into the next step and build / enqueue
+ * that step on the host while the previous one still runs (chunk sizes change
+ * every iteration "at no additional cost").  Stream-ordered: the read happens on `stream` after
+ * the work already enqueued there.  Values are clamped to [0, vocab) (the engine's argmax output
+ * always is in range); the descriptor's decode tokens are still range-checked on the host.
+ * decode_tokens_dev = NULL: exactly qos_hybrid_step. */
+int qos_hybrid_step_ex(qos_engine_t* eng, const qos_batch* batch, void* logits, int logits_dtype,
+                       int32_t* next_tokens, int outputs_on_host, void* stream, const int32_t* decode_tokens_dev);
 
 /* Device-timed latency of one synthetic step for the scheduler's iteration-time model
  * (replaces the paper's Vidur-profiled random forest, §3.6.1): a chunk of

@@ -395,6 +395,19 @@ cudaError_t launch_table_update(int32_t* tables, int table_w, const int32_t* tri
   count_launch();
   return launch_pdl(table_update_kernel, dim3((n + 255) / 256), dim3(256), 0, st, tables, table_w, triples, n);
 }
+// decode tokens taken from device memory (qos_hybrid_step_ex): the step's token array gets
+// src[0..n) at the decode rows, clamped to [0, vocab) (the engine's own argmax outputs always are)
+__global__ void token_patch_kernel(int32_t* __restrict__ dst, const int32_t* __restrict__ src, int n, int vocab) {
+  griddep_wait();
+  griddep_launch_dependents();
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
+    dst[i] = min(max(src[i], 0), vocab - 1);
+}
+cudaError_t launch_token_patch(int32_t* dst, const int32_t* src, int n, int vocab, cudaStream_t st) {
+  if (n == 0) return cudaSuccess;
+  count_launch();
+  return launch_pdl(token_patch_kernel, dim3((n + 255) / 256), dim3(256), 0, st, dst, src, n, vocab);
+}
 cudaError_t launch_embed_rmsnorm(const int32_t* tokens, const void* emb, const void* g, float* resid, void* out,
                                  int T, int d, float eps, cudaStream_t st) {
   if (T == 0) return cudaSuccess;

@@ -1225,7 +1225,7 @@ int run_layers(qos_engine* e, const StepMeta& m, uint8_t* dm, void* logits, int 
 }
 
 int do_step(qos_engine* e, const qos_batch* b, void* logits, int logits_dtype, int32_t* next_tokens, int on_host,
-            cudaStream_t st, bool check_and_advance) {
+            cudaStream_t st, bool check_and_advance, const int32_t* dec_tokens_dev = nullptr) {
   if (logits && logits_dtype != QOS_F32 && logits_dtype != QOS_BF16)
     return set_error(QOS_ERR_INVALID_ARG, "logits_dtype");
   if (cudaSetDevice(e->device) != cudaSuccess) return set_error(QOS_ERR_CUDA, "cudaSetDevice");
@@ -1241,6 +1241,9 @@ int do_step(qos_engine* e, const qos_batch* b, void* logits, int logits_dtype, i
   {
     TimerScope ts(e, QOS_T_META, st);
     QOS_TRY(upload_meta(e, m, st, &dm));
+    if (dec_tokens_dev && m.n_decode)  // decode rows are the last n_decode token rows
+      QOS_CU(launch_token_patch(reinterpret_cast<int32_t*>(dm + m.o_tok) + (m.T - m.n_decode), dec_tokens_dev, m.n_decode,
+                                e->cfg.vocab, st));
   }
   r = run_layers(e, m, dm, logits, logits_dtype, next_tokens, !on_host, st);
   if (r != QOS_OK) {
@@ -1878,6 +1881,13 @@ int qos_hybrid_step(qos_engine_t* e, const qos_batch* batch, void* logits, int l
   if (!e) return set_error(QOS_ERR_INVALID_ARG, "engine is NULL");
   return do_step(e, batch, logits, logits_dtype, next_tokens, outputs_on_host, reinterpret_cast<cudaStream_t>(stream),
                  true);
+}
+
+int qos_hybrid_step_ex(qos_engine_t* e, const qos_batch* batch, void* logits, int logits_dtype, int32_t* next_tokens,
+                       int outputs_on_host, void* stream, const int32_t* decode_tokens_dev) {
+  if (!e) return set_error(QOS_ERR_INVALID_ARG, "engine is NULL");
+  return do_step(e, batch, logits, logits_dtype, next_tokens, outputs_on_host, reinterpret_cast<cudaStream_t>(stream),
+                 true, decode_tokens_dev);
 }
 
 int qos_profile_step_ex(qos_engine_t* e, int32_t chunk_len, int32_t kv_start, int32_t n_decode,

@@ -121,6 +121,7 @@ cudaError_t kvfill_launch(void* plane, const int32_t* d_table, int n_tokens, int
                           int kv_head0, int hd, uint64_t seed, uint64_t name_hash, int fp16, cudaStream_t st);
 
 // ------------------------------------------------------------------ elementwise (elementwise.cu)
+cudaError_t launch_token_patch(int32_t* dst, const int32_t* src, int n, int vocab, cudaStream_t st);
 cudaError_t launch_embed_rmsnorm(const int32_t* tokens, const void* emb, const void* g, float* resid, void* out,
                                  int T, int d, float eps, cudaStream_t st);
 cudaError_t launch_rmsnorm(const float* x, const void* g, void* out, int T, int d, float eps, cudaStream_t st);

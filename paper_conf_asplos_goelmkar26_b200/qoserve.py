@@ -97,6 +97,7 @@ _SIGS = {
     "qos_kv_free_blocks": [_P, C.POINTER(C.c_int64)],
     "qos_kv_fill_synthetic": [_P, C.c_int64, C.c_int32, C.c_uint64],
     "qos_hybrid_step": [_P, C.POINTER(qos_batch), _P, C.c_int, _P, C.c_int, _P],
+    "qos_hybrid_step_ex": [_P, C.POINTER(qos_batch), _P, C.c_int, _P, C.c_int, _P, _P],
     "qos_profile_step": [_P, C.c_int32, C.c_int32, C.POINTER(C.c_int32), C.c_int32, C.POINTER(C.c_float)],
     "qos_profile_step_ex": [_P, C.c_int32, C.c_int32, C.c_int32, C.POINTER(C.c_int32), C.c_int32, C.c_int32,
                             C.POINTER(C.c_float), C.POINTER(C.c_float)],
@@ -346,6 +347,12 @@ class Engine:
                         outputs_on_host: bool = False, stream=None):
         _call("qos_hybrid_step", self.h, C.byref(batch.b), logits, logits_dtype, next_tokens,
               int(bool(outputs_on_host)), stream)
+
+    def qos_hybrid_step_ex(self, batch: _BatchKeep, logits=None, logits_dtype: int = QOS_F32, next_tokens=None,
+                           outputs_on_host: bool = False, stream=None, decode_tokens_dev=None):
+        """qos_hybrid_step with the decodes' tokens read from device memory (int32 pointer)."""
+        _call("qos_hybrid_step_ex", self.h, C.byref(batch.b), logits, logits_dtype, next_tokens,
+              int(bool(outputs_on_host)), stream, decode_tokens_dev)
 
     def step_host(self, batch: _BatchKeep, vocab: int):
         """Convenience: run a step with host outputs; returns (logits f32 [R, V], tokens [R])."""

@@ -87,6 +87,69 @@ def test_tiny_greedy_decode_loop_tokens_identical():
     eng.close()
 
 
+def test_device_token_feedback_loop_matches_host_loop():
+    """qos_hybrid_step_ex: a greedy loop whose decode tokens are the previous step's DEVICE
+    next_tokens (steps enqueued back to back, no host round trip between them) gives exactly the
+    logits and tokens of the same loop fed back through the host, which the oracle checks.  The
+    steps also carry a prefill chunk each (chunk row first, so the decode tokens are
+    next_tokens + 1 of the previous step) and the descriptor's decode tokens are wrong on purpose."""
+    import torch
+    from oracle.engine import OracleEngine
+    from oracle.model import PRESETS
+    V = 1024
+    runs = []
+    for mode in ("host", "device"):
+        q, cfg, eng = make_engine("tiny", num_blocks=256)
+        eng.qos_engine_load_synthetic(0)
+        prompts = {r: synth.request_tokens(r, 20 + 7 * r, V) for r in (1, 2, 3)}
+        for r, p in prompts.items():
+            eng.qos_kv_alloc(r, len(p) + 12)
+        lg, tk = eng.step_host(q.make_batch([(r, 0, p) for r, p in prompts.items()], []), V)
+        toks = {r: int(tk[i]) for i, r in enumerate(prompts)}
+        if mode == "host":
+            init_toks = dict(toks)
+        ctx = {r: len(p) for r, p in prompts.items()}
+        outs = []
+        if mode == "device":
+            st = torch.cuda.current_stream()
+            dev = [torch.empty(4, dtype=torch.int32, device="cuda") for _ in range(10)]
+            dlg = [torch.empty((4, V), dtype=torch.float32, device="cuda") for _ in range(10)]
+            first = torch.tensor([toks[r] for r in sorted(prompts)], dtype=torch.int32, device="cuda")
+        for k in range(10):
+            chunk_req = 100 + k
+            eng.qos_kv_alloc(chunk_req, 16)
+            pre = [(chunk_req, 0, synth.request_tokens(chunk_req, 16, V))]
+            if mode == "host":
+                dec = [(r, ctx[r], toks[r]) for r in sorted(prompts)]
+                lg, tk = eng.step_host(q.make_batch(pre, dec), V)
+                outs.append((lg, tk))
+                toks = {r: int(tk[1 + i]) for i, r in enumerate(sorted(prompts))}
+            else:
+                dec = [(r, ctx[r], 0) for r in sorted(prompts)]  # ignored: tokens come from the device
+                src = first.data_ptr() if k == 0 else dev[k - 1].data_ptr() + 4
+                eng.qos_hybrid_step_ex(q.make_batch(pre, dec), dlg[k].data_ptr(), q.QOS_F32, dev[k].data_ptr(), False,
+                                       st.cuda_stream, src)
+            for r in prompts:
+                ctx[r] += 1
+        if mode == "device":
+            torch.cuda.synchronize()
+            outs = [(dlg[k].cpu().numpy(), dev[k].cpu().numpy()) for k in range(10)]
+        runs.append(outs)
+        eng.close()
+    for (la, ta), (lb, tb) in zip(*runs):
+        assert np.array_equal(la, lb) and np.array_equal(ta, tb)
+    # and the host loop against the oracle for the first decode step (same descriptor)
+    orc = OracleEngine(PRESETS["tiny"], seed=0, num_blocks=256)
+    prompts = {r: synth.request_tokens(r, 20 + 7 * r, V) for r in (1, 2, 3)}
+    for r, p in prompts.items():
+        orc.kv_alloc(r, len(p) + 12)
+    ref0 = orc.hybrid_step([(r, 0, list(p)) for r, p in prompts.items()], [])
+    orc.kv_alloc(100, 16)
+    dec = [(r, len(prompts[r]), init_toks[r]) for r in sorted(prompts)]
+    ref = orc.hybrid_step([(100, 0, list(synth.request_tokens(100, 16, V)))], dec)
+    assert row_rel_err(runs[0][0][0], ref) <= TOL_LOGITS
+
+
 def test_batch_composition_and_split_invariance_on_gpu():
     q, cfg, eng = make_engine("tiny", num_blocks=256)
     eng.qos_engine_load_synthetic(0)
