@@ -151,6 +151,7 @@ struct FaParams {
   float scale_log2;
   int kv_first = 0;  // persistent kernel: issue an item's first K/V tile before its Q (option fa_kvfirst)
   int tma5 = 0;      // persistent kernel: a tile's 4 blocks in one 5-D box when their ids are consecutive
+  int psplit = 0;    // persistent kernel: release P to the P.V MMAs in two halves of 32 keys
 };
 
 // Work item = NQ consecutive entries of `items`: q tiles of one (chunk, kv head) that share
@@ -469,8 +470,8 @@ __global__ void __launch_bounds__(FaCfg<HD, 1>::kThreads, 2)
   uint64_t* v_full = k_empty + S;
   uint64_t* v_empty = v_full + S;
   uint64_t* s_full = v_empty + S;   // [2]
-  uint64_t* p_full = s_full + 2;    // [2]
-  uint64_t* o_full = p_full + 2;    // completes once per P.V
+  uint64_t* p_full = s_full + 2;    // [2 buffers][2 key halves]
+  uint64_t* o_full = p_full + 4;    // completes once per P.V
   uint64_t* o_final = o_full + 1;   // completes once per item
   uint64_t* q_full = o_final + 1;   // completes once per item (Q tile landed, TMA)
   uint64_t* q_empty = q_full + 1;   // completes once per item (its last QK done: sQ free)
@@ -490,7 +491,8 @@ __global__ void __launch_bounds__(FaCfg<HD, 1>::kThreads, 2)
     }
     for (int b = 0; b < 2; ++b) {
       mbar_init(&s_full[b], 1);
-      mbar_init(&p_full[b], 128);
+      mbar_init(&p_full[2 * b], 128);
+      mbar_init(&p_full[2 * b + 1], 128);
     }
     mbar_init(o_full, 1);
     mbar_init(o_final, 1);
@@ -577,14 +579,28 @@ __global__ void __launch_bounds__(FaCfg<HD, 1>::kThreads, 2)
         const int s = int(tg % S);
         mbar_wait(&v_full[s], (tg / S) & 1);
         const uint32_t v_base = smem_u32(sV + s * C::kTileBytes);
-        mbar_wait(&p_full[tg & 1], (tg >> 1) & 1);
-        tc_fence_after();
         const uint32_t p_tmem = tmem + C::col_s(0, int(tg & 1));
-#pragma unroll
-        for (int kk = 0; kk < C::kKeys / 16; ++kk) {
-          const uint64_t vd = umma_desc_sw128_mn(v_base + kk * 2048, C::kKeys * 128);
-          const uint32_t pc = p_tmem + (kk >> 1) * 32 + (kk & 1) * 8;
-          umma_bf16_ts(tmem + C::col_o(0), pc, vd, idesc_pv, (!first || kk != 0) ? 1u : 0u);
+        // P arrives in two halves of 32 keys (fa_psplit: the first half's MMAs run while the
+        // softmax computes the second half; without it only the second barrier is used)
+        auto pv_mmas = [&](int kk0, int kk1) {
+          for (int kk = kk0; kk < kk1; ++kk) {
+            const uint64_t vd = umma_desc_sw128_mn(v_base + kk * 2048, C::kKeys * 128);
+            const uint32_t pc = p_tmem + (kk >> 1) * 32 + (kk & 1) * 8;
+            umma_bf16_ts(tmem + C::col_o(0), pc, vd, idesc_pv, (!first || kk != 0) ? 1u : 0u);
+          }
+        };
+        constexpr int KK = C::kKeys / 16;
+        if (p.psplit) {
+          mbar_wait(&p_full[(tg & 1) * 2], (tg >> 1) & 1);
+          tc_fence_after();
+          pv_mmas(0, KK / 2);
+          mbar_wait(&p_full[(tg & 1) * 2 + 1], (tg >> 1) & 1);
+          tc_fence_after();
+          pv_mmas(KK / 2, KK);
+        } else {
+          mbar_wait(&p_full[(tg & 1) * 2 + 1], (tg >> 1) & 1);
+          tc_fence_after();
+          pv_mmas(0, KK);
         }
         umma_commit(o_full);
         umma_commit(&v_empty[s]);
@@ -663,6 +679,26 @@ __global__ void __launch_bounds__(FaCfg<HD, 1>::kThreads, 2)
         const float m_new = rescale ? mx : m_used;
         const float alpha = (rescale && m_used != -INFINITY) ? ex2(m_used - m_new) : 1.f;
         const float mb = (m_new == -INFINITY) ? 0.f : m_new;
+        // rescale O (tiles < j) before PV(j) accumulates into it; PV(tg-2) completed before
+        // QK(tg) (awaited above), so o_full has completed tg-1 or tg times and this parity wait
+        // cannot alias.  With fa_psplit it happens before the first half of P is released.
+        auto rescale_o = [&]() {
+          if (j >= 1 && __any_sync(0xffffffffu, alpha != 1.f)) {
+            mbar_wait(o_full, (tg - 1) & 1);
+            tc_fence_after();
+#pragma unroll 1
+            for (int c = 0; c < HD / 16; ++c) {
+              uint32_t r2[16];
+              tmem_ld32x32b_x16(o_addr + c * 16, r2);
+              tmem_ld_wait();
+#pragma unroll
+              for (int i = 0; i < 16; ++i) r2[i] = __float_as_uint(__uint_as_float(r2[i]) * alpha);
+              tmem_st32x32b_x16(o_addr + c * 16, r2);
+            }
+            tmem_st_wait();
+          }
+        };
+        if (p.psplit) rescale_o();
         float2 sum2[4] = {make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f), make_float2(0.f, 0.f)};
         const float2 scale2 = make_float2(p.scale_log2, p.scale_log2), nmb2 = make_float2(-mb, -mb);
 #pragma unroll
@@ -677,30 +713,22 @@ __global__ void __launch_bounds__(FaCfg<HD, 1>::kThreads, 2)
             sum2[i & 3] = add2(sum2[i & 3], pp);
           }
           tmem_st32x32b_x16(s_addr + c * 32, hi);
+          if (p.psplit) {
+            tmem_st_wait();
+            tc_fence_before();
+            mbar_arrive(&p_full[sb * 2 + c]);
+          }
         }
         const float2 s01 = add2(sum2[0], sum2[1]), s23 = add2(sum2[2], sum2[3]);
         const float sum = (s01.x + s23.x) + (s01.y + s23.y);
-        tmem_st_wait();
         l = l * alpha + sum;
-        if (j >= 1 && __any_sync(0xffffffffu, alpha != 1.f)) {
-          // rescale O before PV(j) accumulates into it; PV(tg-2) completed before QK(tg) (awaited
-          // above), so o_full has completed tg-1 or tg times and this parity wait cannot alias
-          mbar_wait(o_full, (tg - 1) & 1);
-          tc_fence_after();
-#pragma unroll 1
-          for (int c = 0; c < HD / 16; ++c) {
-            uint32_t r2[16];
-            tmem_ld32x32b_x16(o_addr + c * 16, r2);
-            tmem_ld_wait();
-#pragma unroll
-            for (int i = 0; i < 16; ++i) r2[i] = __float_as_uint(__uint_as_float(r2[i]) * alpha);
-            tmem_st32x32b_x16(o_addr + c * 16, r2);
-          }
+        if (!p.psplit) {
           tmem_st_wait();
+          rescale_o();
+          tc_fence_before();
+          mbar_arrive(&p_full[sb * 2 + 1]);
         }
         m_used = m_new;
-        tc_fence_before();
-        mbar_arrive(&p_full[sb]);
       }
       mbar_wait(o_final, uint32_t(n) & 1);
       tc_fence_after();
@@ -1358,6 +1386,7 @@ __global__ void __launch_bounds__(PpCfg<HD>::kThreads, 1)
 
 static int g_fa_poly = getenv("QOS_FA_POLY") ? atoi(getenv("QOS_FA_POLY")) : 4;
 static int g_fa_tma5 = 1;
+static int g_fa_psplit = 1;
 static int g_fa_kvfirst = 0;  // neutral in ncu cycles (profiles/ncu_ab_fa_r2c.jsonl)
 
 template <int HD, int POLY, int NQ>
@@ -1434,6 +1463,7 @@ static cudaError_t prefill_persist_t(const AttnLaunch& a, const PrefillItem* ite
   p.scale_log2 = a.scale_log2;
   p.kv_first = g_fa_kvfirst;
   p.tma5 = (g_fa_tma5 && a.kv_tmap5) ? 1 : 0;
+  p.psplit = g_fa_psplit;
   return launch_pdl(prefill_attn_persist_kernel<HD, POLY>, dim3(n_cta), dim3(C::kThreads), C::kSmem, st, *a.kv_tmap,
                     *qmp, a.kv_tmap5 ? *a.kv_tmap5 : *a.kv_tmap, p, items, cta_off);
 }
@@ -1494,6 +1524,7 @@ int prefill_pair_max_clusters() {
 void set_fa_poly(int n) { g_fa_poly = n; }
 void set_fa_kvfirst(int v) { g_fa_kvfirst = v; }
 void set_fa_tma5(int v) { g_fa_tma5 = v; }
+void set_fa_psplit(int v) { g_fa_psplit = v; }
 
 int prefill_tc_positions_per_tile(int group) { return 128 / group; }
 

@@ -1982,6 +1982,7 @@ int qos_engine_set_option(qos_engine_t* e, const char* name, int64_t value) {
   else if (n == "fa_poly") set_fa_poly(int(value));  // process-wide
   else if (n == "fa_kvfirst") set_fa_kvfirst(int(value != 0));  // process-wide
   else if (n == "fa_tma5") set_fa_tma5(int(value != 0));  // process-wide
+  else if (n == "fa_psplit") set_fa_psplit(int(value != 0));  // process-wide
   else if (n == "gemm2_rel_cluster") set_gemm2_rel_cluster(int(value != 0));  // process-wide (experiment)
   else if (n == "swab_gran") set_swab_gran(int(value));  // process-wide (experiments)
   else if (n == "gemm_swab") e->gemm_swab = int(value < 0 ? 0 : value > 2 ? 2 : value);

@@ -15,7 +15,8 @@ void set_pdl(bool on);
 // prefill attention: every n-th exp2 pair on the FMA pipe (0 = all on MUFU); process-wide
 void set_fa_poly(int n);
 void set_fa_kvfirst(int v);
-void set_fa_tma5(int v);  // process-wide: persistent prefill attention loads 4-block runs in one TMA op
+void set_fa_tma5(int v);
+void set_fa_psplit(int v);  // process-wide: persistent prefill attention releases P in two halves  // process-wide: persistent prefill attention loads 4-block runs in one TMA op
 void set_gemm2_rel_cluster(int v);  // process-wide experiment (gemm.cu)  // process-wide: persistent prefill attention loads K/V before Q
 void set_swab_gran(int v);  // weight-streaming GEMM range granule (k-blocks; -1 automatic, 0 whole tiles)
 
