@@ -128,6 +128,13 @@ class SchedulerConfig:
     # targets a fixed latency, so chunks shrink as the prefill's cached prefix grows
     chunk_policy: str = "slack"
     medha_target_ms: float = 50.0
+    # ablation switches (the paper's Medha comparison runs "only dynamic chunking under FCFS
+    # scheduling, disabling all other techniques"): fcfs orders the prefill
+    # queue by arrival instead of the hybrid priority; relegation / preemption toggle eager
+    # relegation (Alg. 1 lines 12-15) and selective preemption
+    fcfs: bool = False
+    relegation: bool = True
+    preemption: bool = True
 
 
 class QoServeScheduler:
@@ -152,7 +159,9 @@ class QoServeScheduler:
         return r.t_arrival + r.qos["ttlt"] + a * (r.prefill_rem + decode_rem)
 
     def sort_key(self, r: Request):
-        """COMPARATOR (Alg. 1 lines 26-33): non-relegated first, then priority."""
+        """COMPARATOR (Alg. 1 lines 26-33): non-relegated first, then priority (fcfs: arrival)."""
+        if self.cfg.fcfs:
+            return (r.relegated, r.t_arrival, r.req_id)
         return (r.relegated, self.priority(r), r.t_arrival, r.req_id)
 
     # ---------------------------------------------------------------- slack / budget
@@ -241,7 +250,7 @@ class QoServeScheduler:
                 # admission: a new prompt is not started while the decode set is full
                 i += 1
                 continue
-            if not top.relegated and self.will_violate(top, now, C, ctx):   # line 12
+            if self.cfg.relegation and not top.relegated and self.will_violate(top, now, C, ctx):   # line 12
                 # eager relegation with hints: free-tier first; important requests only once
                 # they have actually missed their deadline
                 deadline = top.d_first() if top.interactive else top.d_total()
@@ -259,7 +268,7 @@ class QoServeScheduler:
         # when waiting one more iteration would make it violate -- but only
         # within what is left of the budget C (the decode slack bounds the whole step)
         chosen = {r.req_id for r, _ in chunks}
-        for r in queue[i:]:
+        for r in (queue[i:] if self.cfg.preemption else []):
             if count >= C or len(chunks) + len(decodes) >= self.cfg.max_rows:
                 break
             if r.prefill_done > 0 and r.req_id not in chosen and not r.relegated:

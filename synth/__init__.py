@@ -147,6 +147,10 @@ LOGNORMAL = {
 }
 
 
+# fixed-length synthetic workloads: (prompt tokens, decode tokens) of every request
+FIXED = {"long_10k": (10_000, 500)}   # the paper's Medha comparison trace
+
+
 def trace(qps: float, duration_s: float, dataset: str = "azure_conv", seed: int = SEED_ARRIVALS,
           low_priority_frac: float = 0.2, max_total: int = 8192):
     """Synthetic request stream shaped like the paper's workloads: Poisson arrivals at `qps`
@@ -155,15 +159,20 @@ def trace(qps: float, duration_s: float, dataset: str = "azure_conv", seed: int 
     free-tier requests, prompt + decode <= max_total (Llama-3-8B window).
     Returns a list of dicts (pure data; the scheduler builds its Request objects from them)."""
     rng = np.random.default_rng(seed)
-    mu_p, sg_p = LOGNORMAL[dataset]["prompt"]
-    mu_d, sg_d = LOGNORMAL[dataset]["decode"]
+    fixed = FIXED.get(dataset)
+    if fixed is None:
+        mu_p, sg_p = LOGNORMAL[dataset]["prompt"]
+        mu_d, sg_d = LOGNORMAL[dataset]["decode"]
     t, out, i = 0.0, [], 0
     while True:
         t += rng.exponential(1.0 / qps)
         if t > duration_s:
             break
-        p = int(np.clip(np.exp(rng.normal(mu_p, sg_p)), 16, max_total - 16))
-        d = int(np.clip(np.exp(rng.normal(mu_d, sg_d)), 1, max_total - p))
+        if fixed is not None:   # fixed lengths; the window check does not apply (max_total unused)
+            p, d = fixed
+        else:
+            p = int(np.clip(np.exp(rng.normal(mu_p, sg_p)), 16, max_total - 16))
+            d = int(np.clip(np.exp(rng.normal(mu_d, sg_d)), 1, max_total - p))
         tier = ("Q1", "Q2", "Q3")[int(rng.integers(0, 3))]
         out.append({"req_id": i, "t_arrival": t, "prompt_len": p, "decode_len": d, "tier": tier,
                     "app_id": f"{dataset}-{tier}", "important": bool(rng.random() >= low_priority_frac)})

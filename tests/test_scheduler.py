@@ -299,3 +299,32 @@ def test_preemption_stays_within_the_budget_and_token_capacity():
     s2.submit(Request(1, 0.0, 5000, "Q2"))
     chunks, decodes = s2.create_batch(0.0)
     assert sum(n for _, n in chunks) + len(decodes) == 1000
+
+
+def test_fcfs_and_ablation_switches():
+    """The ablation of the paper's Medha comparison ("only dynamic chunking under FCFS
+    scheduling, disabling all other techniques"): fcfs serves prefills in
+    arrival order where the hybrid priority (Eq. 4-5) would not; relegation off never relegates."""
+    # a non-interactive request that arrived first vs an interactive one with an earlier
+    # Eq. 4 priority: hybrid priority picks the interactive one, fcfs the earlier arrival
+    early = Request(1, 0.0, 4000, "Q3", decode_len=10)
+    late = Request(2, 1.0, 100, "Q1", decode_len=10)
+    for fcfs, first in ((False, 2), (True, 1)):
+        s = QoServeScheduler(SchedulerConfig(max_chunk=64, fcfs=fcfs), lin_model)
+        s.submit(early)
+        s.submit(late)
+        chunks, _ = s.create_batch(2.0)
+        assert chunks[0][0].req_id == first
+    # an interactive prompt that cannot meet its TTFT: relegated with relegation on, not off
+    for relegation in (True, False):
+        s = QoServeScheduler(SchedulerConfig(max_chunk=64, relegation=relegation), lin_model)
+        r = Request(3, 0.0, 100_000, "Q1", decode_len=10, important=False)
+        s.submit(r)
+        s.create_batch(5.9)
+        assert r.relegated == relegation
+
+
+def test_fixed_length_trace():
+    tr = synth.trace(2.0, 30.0, "long_10k")
+    assert len(tr) > 20 and all(t["prompt_len"] == 10_000 and t["decode_len"] == 500 for t in tr)
+    assert {t["tier"] for t in tr} == {"Q1", "Q2", "Q3"}

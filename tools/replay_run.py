@@ -37,6 +37,15 @@ def main():
     ap.add_argument("--out", default=None)
     ap.add_argument("--replicas", type=int, default=1,
                     help="round-robin TP1 replicas (1 per GPU); engine mode replays them one after another")
+    ap.add_argument("--policy", default="slack", choices=["slack", "medha"],
+                    help="chunk sizing: QoServe's slack-based dynamic chunking or Medha-style fixed-target")
+    ap.add_argument("--medha-target-ms", type=float, default=50.0)
+    ap.add_argument("--only-dc", action="store_true",
+                    help="the paper's Medha-comparison ablation: FCFS order, no relegation, no selective "
+                         "preemption (PAPER.md:1645-1649)")
+    ap.add_argument("--max-seq", type=int, default=8192, help="engine max_seq_len (long_10k needs 10500)")
+    ap.add_argument("--max-decodes", type=int, default=256,
+                    help="decode-set bound (long_10k: 90, so the running requests' KV fits the pool)")
     a = ap.parse_args()
     results = []
     eng = None
@@ -46,7 +55,7 @@ def main():
         from paper_conf_asplos_goelmkar26_b200.presets import preset
         torch.cuda.set_device(0)
         cfg = q.model_cfg(**preset("llama3-8b"), num_blocks=int(140e9 / (32 * 2 * 8 * 128 * 2 * 16)),
-                          max_seq_len=8192, max_requests=4096, max_batch_tokens=a.max_chunk + 512,
+                          max_seq_len=a.max_seq, max_requests=4096, max_batch_tokens=a.max_chunk + 512,
                           max_batch_rows=257)
         eng = q.Engine(cfg)
         eng.qos_engine_load_synthetic(0)
@@ -57,7 +66,8 @@ def main():
         # coefficient nor the per-KV-byte coefficient is left unidentified
         for c in (0, 256, 512, 1024, 2048, 3072, 4096):
             for nd in (0, 16, 64, 128, 256):
-                for ctx, ks in ((512, 0), (2048, 2048), (6144, 0), (1536, 4096)):
+                long = ((10000, 0), (4096, 8192)) if a.max_seq > 10500 else ()
+                for ctx, ks in ((512, 0), (2048, 2048), (6144, 0), (1536, 4096)) + long:
                     if (c == 0 and nd == 0) or c > a.max_chunk or (c == 0 and ks) or nd * (ctx + 1) > 1_000_000:
                         continue
                     t, _ = eng.qos_profile_step(c, [ctx] * nd, reps=3, warmup=2, kv_start=ks)
@@ -76,8 +86,10 @@ def main():
 
         def mk_sched():
             return QoServeScheduler(SchedulerConfig(alpha_ms_per_token=a.alpha, max_chunk=a.max_chunk,
-                                                    max_decodes=256, max_rows=257,
-                                                    max_tokens=a.max_chunk + 512), pred)
+                                                    max_decodes=a.max_decodes, max_rows=257,
+                                                    max_tokens=a.max_chunk + 512, chunk_policy=a.policy,
+                                                    medha_target_ms=a.medha_target_ms, fcfs=a.only_dc,
+                                                    relegation=not a.only_dc, preemption=not a.only_dc), pred)
         if a.mode == "engine" and a.replicas > 1:
             # round-robin replicas replayed one after another on the one GPU (replicas share
             # nothing; each runs its share of the trace on its own virtual clock)
@@ -92,14 +104,15 @@ def main():
         else:
             out = replay(tr, mk_sched(), ModelExecutor(pred))
         out.update({"qps": qps, "dataset": a.dataset, "mode": a.mode, "duration_s": a.duration, "alpha": a.alpha,
-                    "replicas": a.replicas})
+                    "replicas": a.replicas, "policy": a.policy, "only_dc": a.only_dc})
         series = out.pop("chunk_series", None)
         print(json.dumps(out), flush=True)
         out["chunk_series"] = series
         results.append(out)
     ok = [r["qps"] for r in results if r["violations_pct"] <= 1.0]
     summary = {"goodput_qps": max(ok) if ok else 0.0, "dataset": a.dataset, "mode": a.mode,
-               "replicas": a.replicas, "qps_tested": [r["qps"] for r in results]}
+               "replicas": a.replicas, "qps_tested": [r["qps"] for r in results], "policy": a.policy,
+               "only_dc": a.only_dc}
     print(json.dumps(summary), flush=True)
     if a.out:
         json.dump({"summary": summary, "runs": results}, open(a.out, "w"), indent=1)
