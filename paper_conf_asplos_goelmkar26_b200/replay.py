@@ -163,6 +163,6 @@ def summarize(reqs, done, t_end, steps, chunk_log, wall_s):
         out["chunk_mean"] = float(cl[:, 1].mean())
         out["step_ms_mean"] = float(cl[:, 3].mean())
         out["tokens_per_s"] = float((cl[:, 1].sum() + cl[:, 2].sum()) / max(1e-9, cl[:, 3].sum() * 1e-3))
-        out["chunk_series"] = [int(x) for x in cl[:200, 1]]   # Fig. 9 analogue
+        out["chunk_series"] = [int(x) for x in cl[:1000, 1]]   # Fig. 9 / Fig. 15a analogue (1000 batches)
     del fin
     return out

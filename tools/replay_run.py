@@ -66,9 +66,10 @@ def main():
         # coefficient nor the per-KV-byte coefficient is left unidentified
         for c in (0, 256, 512, 1024, 2048, 3072, 4096):
             for nd in (0, 16, 64, 128, 256):
-                long = ((10000, 0), (4096, 8192)) if a.max_seq > 10500 else ()
+                long = ((10000, 0), (4096, 6144)) if a.max_seq > 10500 else ()
                 for ctx, ks in ((512, 0), (2048, 2048), (6144, 0), (1536, 4096)) + long:
-                    if (c == 0 and nd == 0) or c > a.max_chunk or (c == 0 and ks) or nd * (ctx + 1) > 1_000_000:
+                    if ((c == 0 and nd == 0) or c > a.max_chunk or (c == 0 and ks) or nd * (ctx + 1) > 1_000_000
+                            or ks + c > a.max_seq or ctx + 1 > a.max_seq):
                         continue
                     t, _ = eng.qos_profile_step(c, [ctx] * nd, reps=3, warmup=2, kv_start=ks)
                     shapes.append(StepShape([(ks, c)] if c else [], [ctx] * nd))
