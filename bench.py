@@ -238,7 +238,7 @@ def run_ours(args):
     torch.cuda.synchronize()
     read = 0
     t0 = time.perf_counter()
-    src = first.data_ptr()
+    src = first.data_ptr() if n_dec else None
     for k in range(K):
         i = k & 1
         b = wl.next_batch()
@@ -251,10 +251,11 @@ def run_ours(args):
         done[i].record(stream)
         if k >= 1:
             done[i ^ 1].synchronize()
-            read += int(pin_tok[i ^ 1][1])  # the previous step's result, on the host
-        src = dev_tok[i].data_ptr() + 4  # next step's decode tokens: rows 1.. (row 0 is the chunk)
+            read += int(pin_tok[i ^ 1][-1])  # the previous step's result, on the host
+        # next step's decode tokens: rows 1.. (row 0 is the chunk); no decodes: nothing to feed
+        src = dev_tok[i].data_ptr() + 4 if n_dec else None
     done[(K - 1) & 1].synchronize()
-    read += int(pin_tok[(K - 1) & 1][1])
+    read += int(pin_tok[(K - 1) & 1][-1])
     e2e_ms = (time.perf_counter() - t0) * 1e3 / K
     d2h = dec_rows * 4
     # the synchronous form (host outputs, the call returns after the step): host descriptor
