@@ -4,17 +4,20 @@
 //
 // Work item = (chunk, 128-row Q tile, kv head).  The 128 rows pack (position, head-in-group)
 // pairs, so one K/V tile serves the whole GQA group: 128/g positions x g heads.
-//   warp 0      TMA producer: K and V tiles of 128 keys (8 paged blocks x 2 halves of 64 dims,
-//               128-B swizzle)
-//   warp 1      MMA issuer (one lane): S_j = Q K_j^T  (UMMA 128x128x16, A,B from smem) into
+//   warp 0      TMA producer: K and V tiles of 64 keys (4 paged blocks x 2 halves of 64 dims,
+//               128-B swizzle; one 5-D box per half when the 4 block ids are consecutive)
+//   warp 1      MMA issuer (one lane): S_j = Q K_j^T  (UMMA 128x64x16, A,B from smem) into
 //               TMEM;  O += P_j V_j  (UMMA 128xHDx16, A = P from TMEM, B = V MN-major)
 //   warps 2..5  softmax, one TMEM lane (= one row) per thread: masked fp32 online softmax with
 //               exp2, P written back over S in TMEM in fp16 (V is cached in fp16, so P.V is
-//               one kind::f16 MMA with f16 operands); O is rescaled in TMEM
-//               only when the running max grows by more than 2^8 (P <= 2^8 otherwise);
-//               epilogue O / l -> global.
+//               one kind::f16 MMA with f16 operands) and released in two 32-key halves; O is
+//               rescaled in TMEM only when the running max grows by more than 2^8 (P <= 2^8
+//               otherwise); epilogue O / l -> global.
 // Two CTAs share an SM (96 KB smem, 256 TMEM columns each) so one CTA's softmax overlaps the
-// other's MMAs.
+// other's MMAs.  Kernels: prefill_attn_persist_kernel (default: persistent CTAs over host-dealt
+// LPT item lists), prefill_attn_tc_kernel (one item per CTA, option fa_persist=0),
+// prefill_attn_pair_kernel (cta_group::2 CTA pairs, option fa_pair; measured slower) and
+// prefill_attn_pp_kernel (two q tiles ping-ponged in one CTA, option fa_qtiles=2; slower).
 #include <cfloat>
 #include <climits>
 #include <cstdlib>

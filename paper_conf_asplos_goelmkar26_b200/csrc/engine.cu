@@ -385,6 +385,8 @@ struct qos_engine {
   int fa_qtiles = 1;                // option fa_qtiles: prefill q tiles per CTA sharing K/V tiles
   bool fa_persist = true;           // option fa_persist: persistent prefill-attention CTAs (fa_qtiles 1)
   bool fa_pair = false;             // option fa_pair: prefill attention on CTA pairs (cta_group::2, hd 128)
+  int fa_item_cost = 2;             // option fa_item_cost: per-item overhead (key tiles) when dealing
+                                    // persistent prefill-attention items to CTAs
   int pair_clusters = -1;           // co-resident pairs of that kernel (queried once)
   bool norm_fold = true;            // option norm_fold: RMSNorm folded into the O / down and QKV / gate-up GEMMs
   bool overlap_attn = true;       // QOS_OVERLAP_ATTN=0 serialises a7 and a8 (for measurement)
@@ -634,7 +636,7 @@ int build_step(qos_engine* e, const qos_batch* b, bool check_lengths, uint8_t* b
       auto [load, g] = heap.top();
       heap.pop();
       lists[size_t(g)].push_back(int(i));
-      heap.push({load + pitems[i].grp_last / 64 + 1 + 2, g});
+      heap.push({load + pitems[i].grp_last / 64 + 1 + e->fa_item_cost, g});
     }
     std::vector<PrefillItem> dealt;
     dealt.reserve(pitems.size());
@@ -1962,6 +1964,7 @@ int qos_engine_set_option(qos_engine_t* e, const char* name, int64_t value) {
   else if (n == "fa_persist") e->fa_persist = value != 0;
   else if (n == "fa_pair") e->fa_pair = value != 0;
   else if (n == "decode_persist") e->decode_persist = value != 0;
+  else if (n == "fa_item_cost") e->fa_item_cost = int(value < 0 ? 0 : value > 64 ? 64 : value);
   else if (n == "norm_fold") e->norm_fold = value != 0;
   else if (n == "tp_scatter") e->tp_scatter = value != 0;
   else if (n == "attn_order") {
