@@ -13,6 +13,8 @@
 //    heads) is the N = 8 columns: S^T = K Q^T, O^T += V^T P^T (P^T moved into B-fragment
 //    layout with movmatrix).  The 4 consumer warps take interleaved blocks of the item and are
 //    merged in smem; the last split of a (row, kv head) merges the splits (LSE merge).
+//    decode_attn_persist_kernel (option decode_persist, measured slower at small steps) runs the
+//    same item body in persistent CTAs.
 //  (prefill attention (a7) lives in attention_tc.cu on tcgen05/TMEM.)
 // HBM bytes per decode key = 2 * hd * 2 (K + V) per kv head: the kernel is bandwidth-bound.
 #include <algorithm>
