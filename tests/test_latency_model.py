@@ -9,7 +9,7 @@ import numpy as np
 from paper_conf_asplos_goelmkar26_b200.latency_model import (N_FEAT, GemmShapes, LatencyModel, StepShape, features, gemm_work,
                                                              pair_eligible, pair_work, stream_work)
 
-PROF = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles", "latency_table_r2c.json")
+PROF = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles", "latency_table_r2d.json")
 
 
 def test_recovers_known_coefficients():

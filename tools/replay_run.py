@@ -6,7 +6,7 @@
 
 engine: every step is a real device-timed qos_hybrid_step (virtual clock += measured ms); the
         scheduler's latency model is fitted to a quick qos_profile_step sweep of this engine.
-model:  steps are priced by the latency model committed in profiles/latency_table_r2c.json
+model:  steps are priced by the latency model committed in profiles/latency_table_r2d.json
         (fitted to the B200 profile) — fast what-if replays over long horizons.
 Prints one JSON line per QPS and a summary with goodput = max QPS with <= 1% violations
 (PAPER.md:1152-1155).
@@ -76,7 +76,7 @@ def main():
                     ms.append(t)
         model = LatencyModel().fit(shapes, ms)
     else:
-        prof = json.load(open(os.path.join(ROOT, "profiles", "latency_table_r2c.json")))
+        prof = json.load(open(os.path.join(ROOT, "profiles", "latency_table_r2d.json")))
         model = LatencyModel.from_json(json.dumps(prof["model_json"]))
 
     def pred(chunks, ctx):
