@@ -382,6 +382,8 @@ struct qos_engine {
                                    // profiles/decode_split_ab_r1k.jsonl)
   int decode_stages = 8;            // option decode_stages: decode K/V ring depth (8 or 4)
   bool decode_persist = false;      // option decode_persist: persistent decode-attention CTAs
+  int decode_items_per_sm = 0;      // option decode_items_per_sm: split decode key ranges until the
+                                    // work list has this many items per SM (0: 1 or 4 by context)
   int fa_qtiles = 1;                // option fa_qtiles: prefill q tiles per CTA sharing K/V tiles
   bool fa_persist = true;           // option fa_persist: persistent prefill-attention CTAs (fa_qtiles 1)
   bool fa_pair = false;             // option fa_pair: prefill attention on CTA pairs (cta_group::2, hd 128)
@@ -691,7 +693,13 @@ int build_step(qos_engine* e, const qos_batch* b, bool check_lengths, uint8_t* b
     return std::max(1, (nb + sb / 2) / sb);
   };
   {
-    const int64_t target = int64_t(e->num_sms) * 4;  // items per kv head per ... heuristic
+    // enough items to fill the SMs: 4 per SM when the decodes are long (the kernel streams HBM;
+    // more, shorter items fill the last wave), 1 per SM when they are short (< 3072 keys on
+    // average: each item is latency-bound, so fewer, longer items win — ncu cycles at 16 / 32 /
+    // 64 decodes of 1k-2k keys -16 to -28%, at 64 x 4k +5%; profiles/ncu_ab_dtarget_r2c.jsonl)
+    int per_sm = e->decode_items_per_sm;
+    if (per_sm <= 0) per_sm = (b->n_decode > 0 && total_keys < int64_t(3072) * b->n_decode) ? 1 : 4;
+    const int64_t target = int64_t(e->num_sms) * per_sm;
     auto count_items = [&](int s) {
       int64_t n = 0;
       for (int i = 0; i < b->n_decode; ++i) n += nsplit_of(b->decode[i].ctx_len + 1, s);
@@ -1964,6 +1972,7 @@ int qos_engine_set_option(qos_engine_t* e, const char* name, int64_t value) {
   else if (n == "fa_persist") e->fa_persist = value != 0;
   else if (n == "fa_pair") e->fa_pair = value != 0;
   else if (n == "decode_persist") e->decode_persist = value != 0;
+  else if (n == "decode_items_per_sm") e->decode_items_per_sm = int(value < 0 ? 0 : value > 64 ? 64 : value);
   else if (n == "fa_item_cost") e->fa_item_cost = int(value < 0 ? 0 : value > 64 ? 64 : value);
   else if (n == "norm_fold") e->norm_fold = value != 0;
   else if (n == "tp_scatter") e->tp_scatter = value != 0;
