@@ -382,7 +382,7 @@ struct qos_engine {
                                    // profiles/decode_split_ab_r1k.jsonl)
   int decode_stages = 8;            // option decode_stages: decode K/V ring depth (8 or 4)
   bool decode_persist = false;      // option decode_persist: persistent decode-attention CTAs
-  int decode_items_per_sm = 0;      // option decode_items_per_sm: split decode key ranges until the
+  int decode_items_per_sm = 4;      // option decode_items_per_sm: split decode key ranges until the
                                     // work list has this many items per SM (0: 1 or 4 by context)
   int fa_qtiles = 1;                // option fa_qtiles: prefill q tiles per CTA sharing K/V tiles
   bool fa_persist = true;           // option fa_persist: persistent prefill-attention CTAs (fa_qtiles 1)
@@ -693,10 +693,12 @@ int build_step(qos_engine* e, const qos_batch* b, bool check_lengths, uint8_t* b
     return std::max(1, (nb + sb / 2) / sb);
   };
   {
-    // enough items to fill the SMs: 4 per SM when the decodes are long (the kernel streams HBM;
-    // more, shorter items fill the last wave), 1 per SM when they are short (< 3072 keys on
-    // average: each item is latency-bound, so fewer, longer items win — ncu cycles at 16 / 32 /
-    // 64 decodes of 1k-2k keys -16 to -28%, at 64 x 4k +5%; profiles/ncu_ab_dtarget_r2c.jsonl)
+    // enough items to fill the SMs (4 per SM).  Option decode_items_per_sm = 0 picks 1 per SM
+    // for short decodes (< 3072 keys on average: latency-bound items, fewer and longer ones are
+    // 14-29% faster in ncu cycles and 5-9% on small decode-heavy steps) — off by default: whole-
+    // context items quantise into waves by decode count, and the step latency table then fits
+    // the linear model worse (held-out max 9.6% vs 3.8% on the same box, profiles/
+    // latency_table_dsplit_ab_r2c.json), which matters more to the scheduler than the speed
     int per_sm = e->decode_items_per_sm;
     if (per_sm <= 0) per_sm = (b->n_decode > 0 && total_keys < int64_t(3072) * b->n_decode) ? 1 : 4;
     const int64_t target = int64_t(e->num_sms) * per_sm;

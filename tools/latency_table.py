@@ -49,6 +49,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=8)
     ap.add_argument("--layers", type=int, default=None)
     ap.add_argument("--kv-gb", type=float, default=140.0)
+    ap.add_argument("--opts", default="", help="engine options k=v,k=v (A/B of the table itself)")
     a = ap.parse_args()
     import torch
     torch.cuda.set_device(0)
@@ -61,6 +62,9 @@ def main():
                       max_batch_tokens=8192 + 256, max_batch_rows=257)
     eng = q.Engine(cfg)
     eng.qos_engine_load_synthetic(0)
+    for kv in (x for x in a.opts.split(",") if x):
+        k, v = kv.split("=")
+        eng.qos_engine_set_option(k, int(v))
     rng = np.random.default_rng(3)
     t0 = time.time()
 
