@@ -309,6 +309,24 @@ int qos_profile_step_ex(qos_engine_t* eng, int32_t chunk_len, int32_t kv_start,
  *                          kernel's cooperative reduction, the ordered split-K): two such grids
  *                          sharing the SMs could each wait on CTAs the other keeps out.  Set
  *                          automatically for peer-group ranks on one device.
+ *   "fa_tma5" (1)          prefill attention (persistent): a K/V tile whose 4 paged blocks have
+ *                          consecutive ids is loaded as one 5-D TMA box per 64-dim half;
+ *                          process-wide
+ *   "fa_psplit" (1)        prefill attention (persistent): P released to the P.V MMAs in two
+ *                          halves of 32 keys; process-wide
+ *   "fa_kvfirst" (0)       prefill attention (persistent): an item's first K/V tile issued before
+ *                          its Q (measured neutral); process-wide
+ *   "fa_item_cost" (2)     per-item overhead, in key tiles, of the host's LPT dealing of prefill
+ *                          items to persistent CTAs (measured insensitive)
+ *   "fa_pair" (0)          prefill attention on CTA pairs (tcgen05 cta_group::2, each CTA staging
+ *                          half of every K and V tile; hd 128; measured 30-40% slower)
+ *   "decode_persist" (0)   decode attention as persistent CTAs looping over the item list
+ *                          (measured slower at small steps, equal at the bench step)
+ *   "decode_items_per_sm" (4)  split decode key ranges until the work list has this many items
+ *                          per SM; 0: 1 per SM when decodes average < 3072 keys (faster small
+ *                          steps, but a less linear step latency), else 4
+ *   "gemm2_rel_cluster" (0) CTA-pair GEMM accumulator release with .release.cluster instead of
+ *                          the default CTA-scope remote arrive (experiment); process-wide
  * Results do not depend on the options (parity tests run with the defaults and variants). */
 int qos_engine_set_option(qos_engine_t* eng, const char* name, int64_t value);
 

@@ -663,7 +663,7 @@ int build_step(qos_engine* e, const qos_batch* b, bool check_lengths, uint8_t* b
       auto [load, g] = heap.top();
       heap.pop();
       lists[size_t(g)].push_back(int(i));
-      heap.push({load + pitems[2 * i].grp_last / 64 + 1 + 2, g});
+      heap.push({load + pitems[2 * i].grp_last / 64 + 1 + e->fa_item_cost, g});
     }
     std::vector<PrefillItem> dealt;
     dealt.reserve(pitems.size());
