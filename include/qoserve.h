@@ -324,7 +324,7 @@ int qos_profile_step_ex(qos_engine_t* eng, int32_t chunk_len, int32_t kv_start,
  *                          (measured slower at small steps, equal at the bench step)
  *   "decode_items_per_sm" (4)  split decode key ranges until the work list has this many items
  *                          per SM; 0: 1 per SM when decodes average < 3072 keys (faster small
- *                          steps, but a less linear step latency), else 4
+ *                          steps; its latency-model fit is not validated), else 4
  *   "gemm2_rel_cluster" (0) CTA-pair GEMM accumulator release with .release.cluster instead of
  *                          the default CTA-scope remote arrive (experiment); process-wide
  * Results do not depend on the options (parity tests run with the defaults and variants). */
