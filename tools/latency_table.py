@@ -41,6 +41,22 @@ def random_batches(rng, n, cap_tokens):
     return out
 
 
+def short_batches(rng, n, cap_tokens):
+    """Decode-heavy steps with SHORT contexts (ctx_j U[128, 3071]) — the regime the main test set
+    (ctx U[1k, 8k]) barely reaches: chunk 0 (decode-only) or U[256, 2048], kv_start U[0, 2048],
+    n_dec U[1, 256]."""
+    out = []
+    for _ in range(n):
+        chunk = 0 if rng.random() < 0.3 else int(rng.integers(256, 2049))
+        nd = int(rng.integers(1, 257))
+        ks = int(rng.integers(0, 2049)) if chunk else 0
+        ctx = rng.integers(128, 3072, size=nd)
+        while ctx.sum() + nd > cap_tokens:
+            ctx = ctx[: max(1, len(ctx) - 8)]
+        out.append((chunk, ks, [int(c) for c in ctx]))
+    return out
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--out", default="gpurun_out/latency_table.json")
@@ -50,6 +66,8 @@ def main():
     ap.add_argument("--layers", type=int, default=None)
     ap.add_argument("--kv-gb", type=float, default=140.0)
     ap.add_argument("--opts", default="", help="engine options k=v,k=v (A/B of the table itself)")
+    ap.add_argument("--short-test", type=int, default=0,
+                    help="extra short-context decode-heavy test batches (stored as tests_short)")
     a = ap.parse_args()
     import torch
     torch.cuda.set_device(0)
@@ -118,6 +136,13 @@ def main():
         pred = model.predict(s)
         tests.append({"chunk": chunk, "kv_start": ks, "n_decode": len(ctx), "sum_ctx": int(sum(ctx)), "ms": ms,
                       "pred_ms": pred, "rel_err": abs(pred - ms) / ms, "ctx": ctx})
+    tests_short = []
+    for chunk, ks, ctx in short_batches(np.random.default_rng(5), a.short_test, cap_tokens):
+        ms, p95 = prof(chunk, ctx, kv_start=ks)
+        s = StepShape([(ks, chunk)] if chunk else [], ctx)
+        pred = model.predict(s)
+        tests_short.append({"chunk": chunk, "kv_start": ks, "n_decode": len(ctx), "sum_ctx": int(sum(ctx)), "ms": ms,
+                            "pred_ms": pred, "rel_err": abs(pred - ms) / ms, "ctx": ctx})
     errs = np.array([t["rel_err"] for t in tests]) if tests else np.zeros(1)
     out = {"model": "llama3-8b" + (f" (L={a.layers})" if a.layers else ""), "reps": a.reps,
            "kv_capacity_tokens": cap_tokens, "fit_points": len(fit_ms),
@@ -125,9 +150,12 @@ def main():
            "test_rel_err_max": float(errs.max()), "test_rel_err_p95": float(np.percentile(errs, 95)),
            "test_rel_err_mean": float(errs.mean()), "within_5pct": float((errs <= 0.05).mean()),
            "seconds": time.time() - t0, "model_json": json.loads(model.to_json()), "table": table, "tests": tests}
+    if tests_short:
+        es = np.array([t["rel_err"] for t in tests_short])
+        out.update(tests_short=tests_short, short_rel_err_max=float(es.max()), short_within_5pct=float((es <= 0.05).mean()))
     os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
     json.dump(out, open(a.out, "w"), indent=1)
-    print(json.dumps({k: v for k, v in out.items() if k not in ("table", "tests", "model_json")}))
+    print(json.dumps({k: v for k, v in out.items() if k not in ("table", "tests", "tests_short", "model_json")}))
     eng.close()
 
 
