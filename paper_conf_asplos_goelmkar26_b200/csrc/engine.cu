@@ -695,10 +695,9 @@ int build_step(qos_engine* e, const qos_batch* b, bool check_lengths, uint8_t* b
   {
     // enough items to fill the SMs (4 per SM).  Option decode_items_per_sm = 0 picks 1 per SM
     // for short decodes (< 3072 keys on average: latency-bound items, fewer and longer ones are
-    // 14-29% faster in ncu cycles and 5-9% on small decode-heavy steps) — off by default: the
-    // latency model's decode-only grid points at 2k contexts fit worse under it (max 7.3% vs
-    // 5.6%, profiles/latency_table_dsplit_ab_r2c.json) and the table has no random batches in
-    // that regime to validate it; predictability is what the scheduler relies on
+    // 14-29% faster in ncu cycles and 5-9% on small decode-heavy steps) — off by default until
+    // re-validated with the full GPU suite; the latency model fits it as well as the default on
+    // short-context test batches (profiles/latency_table_short_s{4,0}_r2c.json)
     int per_sm = e->decode_items_per_sm;
     if (per_sm <= 0) per_sm = (b->n_decode > 0 && total_keys < int64_t(3072) * b->n_decode) ? 1 : 4;
     const int64_t target = int64_t(e->num_sms) * per_sm;
